@@ -1,0 +1,223 @@
+/*
+ * nfcgen/gen.c -- seeded synthetic traffic generator (input generator only).
+ *
+ * Serves both the oracle and the CUDA path with identical packet bytes.  It
+ * holds none of the method's arithmetic: no parsing, classification, lookup,
+ * checksum, hashing or cryptography -- only a counter-based RNG
+ * (SplitMix64 finaliser keyed by (seed, stream, index)) and byte assembly.
+ * The IPv4 header checksum is left 0 (NIC checksum-offload convention; input
+ * checksums are never verified, R#13).
+ *
+ * Every packet is a pure function of (params, tables, global index), so any
+ * index range can be generated independently (sharding, sampled parity).
+ * Workload recipe: DESIGN.md "Synthetic inputs"; traffic model P:L136
+ * ("randomly generated IP traffic with UDP payloads"), IMIX P:L361.
+ */
+#include <stdint.h>
+#include <string.h>
+
+typedef struct {
+    uint64_t seed;
+    uint64_t n_flows;
+    uint32_t v6_bp;          /* IPv6 share in basis points (0..10000) */
+    uint32_t pkt_len;        /* fixed frame length; 0 = IMIX; 1 = uniform 60..1514 */
+    uint32_t match_ppm;      /* planted DPI pattern probability, per million packets */
+    uint32_t in_acl_pct;     /* % of flows drawn inside a random ACL rule */
+    uint32_t tcp_pct;        /* % of non-rule flows that are TCP (rest UDP) */
+    uint32_t ttl;            /* TTL / hop limit */
+    uint32_t ttl1_ppm;       /* packets with TTL 1 (edge case), per million */
+    uint32_t malformed_ppm;  /* malformed frames (edge case), per million */
+    uint32_t printable;      /* payload bytes drawn from 0x20..0x7e */
+    uint32_t headroom, tailroom;
+} gen_params;
+
+typedef struct {
+    uint32_t n_r4; const uint32_t *r4_prefix; const uint8_t *r4_len;
+    uint32_t n_r6; const uint8_t *r6_prefix; const uint8_t *r6_len;   /* 16 B each */
+    uint32_t n_acl4; const uint32_t *acl4_idx;                         /* rule indices per family */
+    uint32_t n_acl6; const uint32_t *acl6_idx;
+    const uint8_t *acl_rules;                                          /* 48 B rules */
+    uint32_t n_pat; const uint8_t *pat_blob; const uint32_t *pat_off;
+} gen_tables;
+
+enum { S_FLOW = 1, S_FAM, S_INACL, S_RULE, S_SRC, S_DST, S_DST2, S_SP, S_DP, S_ROUTE, S_PROTO, S_LEN,
+       S_PAY, S_MATCH, S_PAT, S_POFF, S_TTL, S_BAD, S_BADK, S_SRC2 };
+
+static inline uint64_t mix64(uint64_t z)
+{
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t nfcgen_rnd(uint64_t seed, uint32_t stream, uint64_t idx)
+{
+    return mix64(mix64(seed * 0xD1B54A32D192ED03ull + stream) ^ idx);
+}
+#define R(st, i) nfcgen_rnd(p->seed, (st), (i))
+
+/* fill addr bits beyond len with random bits (network order, nbytes 4 or 16) */
+static void host_bits(uint8_t *a, const uint8_t *pref, int len, int nbytes, uint64_t r0, uint64_t r1)
+{
+    uint8_t rb[16];
+    for (int k = 0; k < 8; k++) { rb[k] = (uint8_t)(r0 >> (8 * k)); rb[8 + k] = (uint8_t)(r1 >> (8 * k)); }
+    for (int k = 0; k < nbytes; k++) {
+        int keep = len - 8 * k; /* prefix bits in this byte */
+        uint8_t m = keep >= 8 ? 0xFF : keep <= 0 ? 0x00 : (uint8_t)(0xFF << (8 - keep));
+        a[k] = (uint8_t)((pref[k] & m) | (rb[k] & ~m));
+    }
+}
+
+typedef struct { int fam; uint8_t src[16], dst[16]; uint16_t sp, dp; uint8_t proto; } flow_t;
+
+static void make_flow(const gen_params *p, const gen_tables *t, uint64_t f, flow_t *fl)
+{
+    memset(fl, 0, sizeof *fl);
+    fl->fam = (R(S_FAM, f) % 10000) < p->v6_bp ? 6 : 4;
+    int nb = fl->fam == 4 ? 4 : 16;
+    uint32_t n_rules = fl->fam == 4 ? t->n_acl4 : t->n_acl6;
+    const uint32_t *ridx = fl->fam == 4 ? t->acl4_idx : t->acl6_idx;
+    uint8_t zero[16] = {0};
+    if (n_rules && (R(S_INACL, f) % 100) < p->in_acl_pct) {
+        const uint8_t *rule = t->acl_rules + 48 * (size_t)ridx[R(S_RULE, f) % n_rules];
+        host_bits(fl->src, rule + 16, rule[1], nb, R(S_SRC, f), R(S_SRC2, f));
+        host_bits(fl->dst, rule + 32, rule[2], nb, R(S_DST, f), R(S_DST2, f));
+        uint16_t sl = (uint16_t)(rule[6] | rule[7] << 8), sh = (uint16_t)(rule[8] | rule[9] << 8);
+        uint16_t dl = (uint16_t)(rule[10] | rule[11] << 8), dh = (uint16_t)(rule[12] | rule[13] << 8);
+        fl->sp = (uint16_t)(sl + R(S_SP, f) % ((uint32_t)sh - sl + 1));
+        fl->dp = (uint16_t)(dl + R(S_DP, f) % ((uint32_t)dh - dl + 1));
+        fl->proto = rule[4] ? 17 : rule[3];
+    } else {
+        host_bits(fl->src, zero, 0, nb, R(S_SRC, f), R(S_SRC2, f));
+        uint32_t nr = fl->fam == 4 ? t->n_r4 : t->n_r6;
+        if (nr) {
+            uint64_t k = R(S_ROUTE, f) % nr;
+            uint8_t pref[16];
+            int plen;
+            if (fl->fam == 4) {
+                uint32_t v = t->r4_prefix[k];
+                pref[0] = (uint8_t)(v >> 24); pref[1] = (uint8_t)(v >> 16); pref[2] = (uint8_t)(v >> 8); pref[3] = (uint8_t)v;
+                plen = t->r4_len[k];
+            } else {
+                memcpy(pref, t->r6_prefix + 16 * k, 16);
+                plen = t->r6_len[k];
+            }
+            host_bits(fl->dst, pref, plen, nb, R(S_DST, f), R(S_DST2, f));
+        } else {
+            host_bits(fl->dst, zero, 0, nb, R(S_DST, f), R(S_DST2, f));
+        }
+        fl->sp = (uint16_t)R(S_SP, f);
+        fl->dp = (uint16_t)R(S_DP, f);
+        fl->proto = (R(S_PROTO, f) % 100) < p->tcp_pct ? 6 : 17;
+    }
+}
+
+static uint32_t frame_len(const gen_params *p, uint64_t i, int fam, uint8_t proto)
+{
+    uint32_t L = p->pkt_len;
+    if (L == 0) {
+        uint64_t u = R(S_LEN, i) % 10000;
+        L = u < 6122 ? 64 : u < 8469 ? 536 : 1360; /* IMIX */
+    } else if (L == 1) {
+        L = 60 + (uint32_t)(R(S_LEN, i) % (1514 - 60 + 1)); /* uniform ragged lengths (tests) */
+    }
+    uint32_t hdr = (fam == 4 ? 34 : 54) + (proto == 6 ? 20 : proto == 17 ? 8 : 0);
+    return L < hdr ? hdr : L;
+}
+
+static uint64_t round16(uint64_t x) { return (x + 15) & ~15ull; }
+
+/* Slot size of packet i (headroom + frame + tailroom, 16-B aligned). */
+uint64_t nfcgen_layout(const gen_params *p, const gen_tables *t, uint64_t first, uint32_t n, uint64_t base,
+                       uint64_t *off, uint16_t *len)
+{
+    uint64_t pos = base;
+    for (uint32_t k = 0; k < n; k++) {
+        uint64_t i = first + k;
+        flow_t fl;
+        make_flow(p, t, R(S_FLOW, i) % p->n_flows, &fl);
+        uint32_t L = frame_len(p, i, fl.fam, fl.proto);
+        off[k] = pos + p->headroom;
+        len[k] = (uint16_t)L;
+        pos += round16((uint64_t)p->headroom + L + p->tailroom);
+    }
+    return pos;
+}
+
+static void put16(uint8_t *b, uint32_t v) { b[0] = (uint8_t)(v >> 8); b[1] = (uint8_t)v; }
+
+/* Write packets [first, first+n) at the offsets from nfcgen_layout. */
+void nfcgen_fill(const gen_params *p, const gen_tables *t, uint64_t first, uint32_t n, uint8_t *arena,
+                 const uint64_t *off, const uint16_t *len)
+{
+    static const uint8_t mac_d[6] = {0x02, 0, 0, 0, 0, 0x01}, mac_s[6] = {0x02, 0, 0, 0, 0, 0x02};
+    for (uint32_t k = 0; k < n; k++) {
+        uint64_t i = first + k;
+        flow_t fl;
+        make_flow(p, t, R(S_FLOW, i) % p->n_flows, &fl);
+        uint8_t *f = arena + off[k];
+        uint32_t L = len[k];
+        memcpy(f, mac_d, 6);
+        memcpy(f + 6, mac_s, 6);
+        uint32_t ttl = (R(S_TTL, i) % 1000000) < p->ttl1_ppm ? 1 : p->ttl;
+        uint32_t l4;
+        if (fl.fam == 4) {
+            put16(f + 12, 0x0800);
+            f[14] = 0x45; f[15] = 0;
+            put16(f + 16, L - 14);
+            put16(f + 18, (uint32_t)(i & 0xffff));
+            put16(f + 20, 0x4000); /* DF, not a fragment */
+            f[22] = (uint8_t)ttl; f[23] = fl.proto;
+            f[24] = f[25] = 0;
+            memcpy(f + 26, fl.src, 4);
+            memcpy(f + 30, fl.dst, 4);
+            l4 = 34;
+        } else {
+            put16(f + 12, 0x86DD);
+            f[14] = 0x60; f[15] = 0; f[16] = 0; f[17] = 0;
+            put16(f + 18, L - 54);
+            f[20] = fl.proto; f[21] = (uint8_t)ttl;
+            memcpy(f + 22, fl.src, 16);
+            memcpy(f + 38, fl.dst, 16);
+            l4 = 54;
+        }
+        uint32_t pl = l4;
+        if (fl.proto == 17) {
+            put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
+            put16(f + l4 + 4, L - l4); put16(f + l4 + 6, 0);
+            pl = l4 + 8;
+        } else if (fl.proto == 6) {
+            put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
+            uint64_t r = R(S_SP, i);
+            for (int b = 0; b < 8; b++) f[l4 + 4 + b] = (uint8_t)(r >> (8 * b));
+            f[l4 + 12] = 0x50; f[l4 + 13] = 0x18;
+            put16(f + l4 + 14, 0xffff); put16(f + l4 + 16, 0); put16(f + l4 + 18, 0);
+            pl = l4 + 20;
+        }
+        /* payload */
+        for (uint32_t j = pl; j < L; j++) {
+            uint32_t q = j - pl;
+            uint64_t r = R(S_PAY, (i << 14) + (q >> 3));
+            uint8_t b = (uint8_t)(r >> (8 * (q & 7)));
+            f[j] = p->printable ? (uint8_t)(0x20 + b % 95) : b;
+        }
+        if (t->n_pat && (R(S_MATCH, i) % 1000000) < p->match_ppm) {
+            uint64_t pk = R(S_PAT, i) % t->n_pat;
+            uint32_t plen = t->pat_off[pk + 1] - t->pat_off[pk];
+            if (pl + plen <= L) {
+                uint32_t o = pl + (uint32_t)(R(S_POFF, i) % (L - pl - plen + 1));
+                memcpy(f + o, t->pat_blob + t->pat_off[pk], plen);
+            }
+        }
+        if ((R(S_BAD, i) % 1000000) < p->malformed_ppm) {
+            switch (R(S_BADK, i) % 5) {
+            case 0: put16(f + 12, 0x0806); break;                       /* ARP: not IP */
+            case 1: f[14] = (uint8_t)((f[14] & 0x0f) | 0x50); break;    /* bad version */
+            case 2: if (fl.fam == 4) put16(f + 16, L); else put16(f + 18, L); break; /* length overrun */
+            case 3: if (fl.fam == 4) f[14] = 0x44; else f[14] = 0x40; break;        /* IHL 4 / version 4 in v6 */
+            case 4: if (fl.fam == 4) { put16(f + 16, 20 + 4); } else { put16(f + 18, 4); } break; /* L4 truncated */
+            }
+        }
+    }
+}
