@@ -1,0 +1,231 @@
+/*
+ * nfc.h -- C ABI of the B200-native NFCompass SFC hot path.
+ *
+ * One fused, persistent sm_100a kernel applies a Service Function Chain (SFC)
+ * to batches of packets resident in HBM.  The calls follow the paper's problem
+ * statement: traffic traverses a sequence of network functions (NFs) in order
+ * (PAPER.md P:L27, P:L42, P:L79 [SI]); packets arrive and are processed in
+ * batches (P:L87 [SII.B.1]); each NF reads, writes or drops a packet as in
+ * Table II (P:L213-223 [SIV]); a forwarder sets the egress port, the
+ * load balancer picks a destination, IPsec encrypts and authenticates
+ * (P:L130).  NFCompass re-organizes the chain (parallelize, de-duplicate,
+ * early drop, P:L243-271 [SIV.B]) without changing the result of applying the
+ * NFs sequentially in the original order; that sequential result is
+ * what every call below produces.
+ *
+ * Conventions
+ *  - Every call returns an int status: NFC_OK (0) or a negative NFC_E* code.
+ *    Nothing throws across the ABI.  nfc_last_error() returns a thread-local
+ *    message for the last failing call on this thread.
+ *  - "device pointer" = CUDA global memory on the chain's device (e.g. a torch
+ *    CUDA tensor's data_ptr()); "host pointer" = ordinary process memory.
+ *  - A chain is bound to one device and is not thread-safe; use one chain per
+ *    GPU (multi-GPU = one process or thread per GPU, flows sharded by RSS
+ *    hash).
+ *  - All integer fields are little-endian host order unless stated; packet
+ *    bytes and the address fields of specs are network (big-endian) order.
+ */
+#ifndef NFC_H
+#define NFC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define NFC_API __attribute__((visibility("default")))
+#else
+#define NFC_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- status */
+#define NFC_OK 0
+#define NFC_EINVAL (-1)  /* bad argument or malformed spec                        */
+#define NFC_ENOMEM (-2)  /* host or device allocation failed                      */
+#define NFC_ECUDA (-3)   /* CUDA runtime error (message in nfc_last_error)        */
+#define NFC_ESTATE (-4)  /* tables missing for an NF of the chain, or bad state   */
+#define NFC_ECAP (-5)    /* match pairs overflowed match_cap since last collect  */
+#define NFC_EUNSUP (-6)  /* unsupported chain (length > 6, repeated NF kind)      */
+
+/* NF kinds (Table II P:L213-223 rows Firewall, IDS/DPI, LB; P:L128 IPv4/IPv6
+ * forwarders; P:L130 IPsec gateway). */
+#define NFC_ACL 1   /* firewall: 5-tuple first-match classification, DENY drops */
+#define NFC_DPI 2   /* Aho-Corasick multi-pattern DPI (IDS: DROP patterns drop)  */
+#define NFC_LPM4 3  /* IPv4 forwarder, longest-prefix match (DIR-24-8)            */
+#define NFC_LPM6 4  /* IPv6 forwarder, longest-prefix match (Waldvogel levels)    */
+#define NFC_IPSEC 5 /* IPsec ESP gateway: AES-128-CTR + HMAC-SHA1-96              */
+#define NFC_LB 6    /* load balancer: flow hash -> backend -> egress port         */
+
+#define NFC_MAX_CHAIN 6
+
+typedef struct nfc_chain nfc_chain; /* opaque; owned by the library */
+
+typedef struct {
+    int device;              /* CUDA device ordinal                                   */
+    uint32_t flags;          /* reserved, must be 0                                   */
+    uint32_t max_batch_pkts; /* hint: largest packet count per nfc_process_batch call */
+} nfc_chain_opts;
+
+/* Create a chain. kinds[0..n) = NF kinds in ORIGINAL SFC order; 1 <= n <= 6,
+ * each kind at most once (else NFC_EUNSUP).  Allocates device state (stats,
+ * ESP sequence counters, scheduling scratch) on opts->device.  *out is owned by
+ * the caller and released with nfc_destroy_chain. */
+NFC_API int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opts, nfc_chain **out);
+NFC_API void nfc_destroy_chain(nfc_chain *c);
+
+/* Bytes the caller must leave before / after every frame in the arena.
+ * Chains with IPSEC: headroom 16 (the Ethernet+IP header moves 16 B left to
+ * make room for the ESP header and IV, RFC 4303 transport mode), tailroom 32
+ * (ESP trailer + ICV grow the frame by 14..17 B).  Otherwise 0 / 0. */
+NFC_API int nfc_chain_room(const nfc_chain *c, uint32_t *headroom, uint32_t *tailroom);
+
+/* ---------------------------------------------------------------- logical specs
+ * Host structures, copied by nfc_load_tables; the same binary layouts are what
+ * the test oracle reads. */
+typedef struct {                 /* 48 B */
+    uint8_t family;              /* 4 or 6                                        */
+    uint8_t slen, dlen;          /* source / destination prefix lengths           */
+    uint8_t proto;               /* IP protocol (ignored if proto_any)            */
+    uint8_t proto_any;           /* 1 = any protocol                              */
+    uint8_t action;              /* 0 PERMIT, 1 DENY                              */
+    uint16_t sp_lo, sp_hi;       /* source port range, inclusive                  */
+    uint16_t dp_lo, dp_hi;       /* destination port range, inclusive             */
+    uint8_t pad[2];
+    uint8_t src[16], dst[16];    /* prefixes, network order (IPv4: bytes 0..3)    */
+} nfc_acl_rule;
+
+typedef struct {
+    uint32_t n_rules;            /* <= 65534                                      */
+    uint32_t default_action;     /* action when no rule matches: 0/1              */
+    const nfc_acl_rule *rules;   /* host; rule i has priority i (first match)     */
+} nfc_acl_spec;
+
+typedef struct {
+    uint32_t n_patterns;         /* 1..65535                                      */
+    const uint8_t *blob;         /* host; pattern j = blob[off[j] .. off[j+1])    */
+    const uint32_t *off;         /* host; n_patterns+1 offsets                    */
+    const uint8_t *action;       /* host; 0 ALERT, 1 DROP                         */
+} nfc_dpi_spec;
+
+typedef struct { uint32_t prefix; uint8_t len; uint8_t pad; uint16_t nh; } nfc_route4;     /* 8 B  */
+typedef struct { uint8_t prefix[16]; uint16_t nh; uint8_t len; uint8_t pad; } nfc_route6;  /* 20 B */
+typedef struct { uint16_t port; uint8_t mac[6]; } nfc_nexthop;                            /* 8 B  */
+
+typedef struct {
+    uint32_t n_routes;  const nfc_route4 *routes;    /* prefix: host-order u32 value, len 0..32 */
+    uint32_t n_nexthops; const nfc_nexthop *nexthops; /* nh < n_nexthops <= 32767              */
+    uint32_t n_ports;   const uint8_t *port_macs;    /* n_ports x 6 B source MAC per port       */
+} nfc_lpm4_spec;
+
+typedef struct {
+    uint32_t n_routes;  const nfc_route6 *routes;    /* len 0..128                              */
+    uint32_t n_nexthops; const nfc_nexthop *nexthops;
+    uint32_t n_ports;   const uint8_t *port_macs;
+} nfc_lpm6_spec;
+
+typedef struct {                 /* 48 B */
+    uint32_t spi;                /* ESP SPI                                        */
+    uint32_t seq0;               /* initial sequence counter (first packet: seq0+1)*/
+    uint8_t aes_key[16];         /* AES-128 key                                    */
+    uint8_t nonce[4];            /* RFC 3686 nonce                                 */
+    uint8_t auth_key[20];        /* HMAC-SHA1 key                                  */
+} nfc_sa;
+
+typedef struct { uint32_t n_sa; const nfc_sa *sas; } nfc_ipsec_spec; /* 1..255 SAs */
+
+typedef struct {
+    uint32_t n_backends;         /* 1..65535                                       */
+    const uint16_t *backend_port;/* host; egress port per backend                  */
+    const uint8_t *key;          /* host; 40 B Toeplitz key                        */
+} nfc_lb_spec;
+
+/* Build the device image of one NF's tables on the host and copy it to the
+ * device (synchronous).  spec points to the nfc_*_spec matching kind;
+ * spec_bytes = sizeof that struct.  Replaces earlier tables of that kind.
+ * Every NF of the chain needs its tables before nfc_process_batch
+ * (NFC_ESTATE).  Malformed specs -> NFC_EINVAL: duplicate (prefix,len),
+ * len > 32/128, host bits set in a prefix, nh >= n_nexthops, empty pattern,
+ * lo > hi port range, n_sa == 0 or > 255, n_backends == 0. */
+NFC_API int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_bytes);
+
+/* ---------------------------------------------------------------- batches */
+typedef struct {
+    uint8_t *arena;              /* device; packet bytes, rewritten in place              */
+    const uint64_t *off;         /* device; n frame start offsets into arena, each % 16 == 0 */
+    const uint16_t *len;         /* device; n frame lengths (14..16383)                   */
+    uint32_t n;                  /* packets in this batch                                 */
+    uint32_t reserved;
+    uint64_t first_global_index; /* global index of packet 0 (match-pair packet ids)      */
+} nfc_batch;
+
+typedef struct {                 /* 16 B per packet */
+    uint8_t drop_nf;             /* 0xFF forwarded; 0xFE parse failure; else chain position */
+    uint8_t esp_sa;              /* SA index if ESP was applied, else 0xFF                */
+    uint16_t port;               /* egress port; 0 if none set; 0xFFFF if dropped         */
+    uint16_t acl_rule;           /* first matching ACL rule; 0xFFFF none / not reached    */
+    uint16_t lb_backend;         /* LB backend; 0xFFFF if not reached                     */
+    uint16_t dpi_nmatch;         /* number of distinct matched patterns                  */
+    uint16_t out_len;            /* frame length after the chain                          */
+    uint32_t esp_seq;            /* ESP sequence number, 0 if ESP not applied             */
+} nfc_pkt_result;
+
+typedef struct {
+    nfc_pkt_result *rec;         /* device; one record per packet, batches concatenated   */
+    uint32_t *match_pkt;         /* device; match pair packet global index                */
+    uint16_t *match_pat;         /* device; match pair pattern id                         */
+    uint32_t match_cap;          /* capacity of match_pkt / match_pat                     */
+    uint32_t reserved;
+    uint32_t *match_count;       /* device u32, incremented atomically; caller zeroes it   */
+} nfc_result;
+
+/* Apply the chain to n_batches batches (descriptor array in HOST memory),
+ * asynchronously on `stream` (a cudaStream_t; NULL = legacy default stream),
+ * in one persistent kernel launch.  Packets are processed as one stream in
+ * batch order; every per-packet output equals applying the chain's NFs in
+ * original order to each packet, with ESP sequence numbers assigned per SA in
+ * that global order (so outputs never depend on how packets are split into
+ * batches or calls).  Frames are rewritten in place: forwarders rewrite the
+ * Ethernet/IP header; ESP moves the frame start to off-16 and grows the frame
+ * to rec.out_len.  Match pairs are appended in unspecified order; pairs beyond
+ * match_cap are counted in the stats but not written.  Output bytes of
+ * dropped packets are unspecified.  Results are valid after the stream syncs. */
+NFC_API int nfc_process_batch(nfc_chain *c, const nfc_batch *batches, uint32_t n_batches,
+                      const nfc_result *r, void *stream);
+
+/* End-to-end variant with HOST buffers: copies arena[0, arena_bytes) and
+ * off/len to chain-owned device staging buffers on `stream`, runs the chain,
+ * copies the rewritten arena, the records and the match pairs back, and
+ * synchronizes the stream.  Host buffers should be pinned for full PCIe rate.
+ * *n_pairs receives the number of pairs found (may exceed match_cap). */
+NFC_API int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const uint64_t *off,
+                     const uint16_t *len, uint32_t n, uint64_t first_global_index,
+                     nfc_pkt_result *rec, uint32_t *match_pkt, uint16_t *match_pat,
+                     uint32_t match_cap, uint32_t *n_pairs, void *stream);
+
+/* ---------------------------------------------------------------- stats
+ * u64 counter vector (layout in DESIGN.md "Stats vector"): totals, per chain
+ * position in/drop/pass-through/applied, then ACL per-rule hits (+default),
+ * LB per-backend hits and per-SA ESP packets.  Same sequential semantics as
+ * the per-packet records. */
+#define NFC_STATS_RESET 1u
+
+NFC_API int nfc_stats_len(const nfc_chain *c, size_t *len);
+/* Synchronizes the device, copies min(cap, len) counters to out (host) and
+ * optionally resets them.  Returns NFC_ECAP if match pairs were dropped for
+ * capacity since the last reset.  Multi-GPU sums are taken by the caller
+ * (one all-reduce of this vector over NCCL). */
+NFC_API int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags);
+
+/* Number of kernel launches the library issued on this chain so far. */
+NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
+
+NFC_API const char *nfc_last_error(void);
+NFC_API const char *nfc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NFC_H */

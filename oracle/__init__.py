@@ -140,20 +140,22 @@ class OracleChain:
             self._keep.append(a)
             return a.ctypes.data if a.size else None
 
-        if t.acl_rules is not None:
+        ks = {nfcgen.KIND_NAMES[s.kind[i]] for i in range(len(kinds))}
+        # only the chain's own tables are loaded (the stats layout depends on them)
+        if "ACL" in ks and t.acl_rules is not None:
             s.acl, s.n_acl, s.acl_default = P(t.acl_rules), len(t.acl_rules), t.acl_default
-        if t.n_pat:
+        if "DPI" in ks and t.n_pat:
             s.pat_blob, s.pat_off, s.pat_action = P(t.pat_blob), P(t.pat_off), P(t.pat_action)
             s.n_pat = t.n_pat
-        if t.routes4 is not None:
+        if "LPM4" in ks and t.routes4 is not None:
             s.r4, s.n_r4, s.nh4, s.n_nh4 = P(t.routes4), len(t.routes4), P(t.nh4), len(t.nh4)
             s.pmac4, s.n_port4 = P(t.pmac4), len(t.pmac4)
-        if t.routes6 is not None:
+        if "LPM6" in ks and t.routes6 is not None:
             s.r6, s.n_r6, s.nh6, s.n_nh6 = P(t.routes6), len(t.routes6), P(t.nh6), len(t.nh6)
             s.pmac6, s.n_port6 = P(t.pmac6), len(t.pmac6)
-        if t.sas is not None:
+        if "IPSEC" in ks and t.sas is not None:
             s.sa, s.n_sa = P(t.sas), len(t.sas)
-        if t.lb_ports is not None:
+        if "LB" in ks and t.lb_ports is not None:
             s.lb_port, s.n_lb, s.lb_key = P(t.lb_ports), len(t.lb_ports), P(t.lb_key)
         self.spec = s
         self.kinds = list(kinds)

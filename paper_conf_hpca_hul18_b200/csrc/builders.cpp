@@ -1,0 +1,447 @@
+// builders.cpp -- host-side table builders: logical specs -> device images.
+//
+// ACL, Aho-Corasick DFA, IPv4 DIR-24-8
+// ("two memory accesses"), IPv6 binary search on prefix lengths over
+// per-length hash tables ("hashing ... binary search ... up to 7 memory
+// lookups"), AES-128 key schedule + T-tables and HMAC-SHA1 ipad/opad
+// precompute, Toeplitz nibble tables for the RSS / LB flow hash
+// (P:L87).  Product code: independent of oracle/.
+#include <algorithm>
+#include <array>
+#include <cstring>
+#include <map>
+#include <unordered_map>
+
+#include "nfc_internal.h"
+
+namespace nfc {
+
+const uint8_t MS_RSS_KEY[40] = {0x6d, 0x5a, 0x56, 0xda, 0x25, 0x5b, 0x0e, 0xc2, 0x41, 0x67,
+                                0x25, 0x3d, 0x43, 0xa3, 0x8f, 0xb0, 0xd0, 0xca, 0x2b, 0xcb,
+                                0xae, 0x7b, 0x30, 0xb4, 0x77, 0xcb, 0x2d, 0xa3, 0x80, 0x30,
+                                0xf2, 0x0c, 0x6a, 0x42, 0xb7, 0x3b, 0xbe, 0xac, 0x01, 0xfa};
+
+static inline uint32_t be32(const uint8_t *p) { return (uint32_t)p[0] << 24 | (uint32_t)p[1] << 16 | (uint32_t)p[2] << 8 | p[3]; }
+static inline uint32_t mask32(int len) { return len <= 0 ? 0u : len >= 32 ? 0xFFFFFFFFu : 0xFFFFFFFFu << (32 - len); }
+static void mask128(const uint8_t *a, int len, uint32_t w[4])
+{
+    for (int k = 0; k < 4; k++) w[k] = be32(a + 4 * k) & mask32(len - 32 * k);
+}
+
+// ---------------------------------------------------------------- ACL
+std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector<uint4> &r6)
+{
+    if (s.n_rules > 65534) return "acl: too many rules (max 65534)";
+    if (s.n_rules && !s.rules) return "acl: rules == NULL";
+    if (s.default_action > 1) return "acl: default_action must be 0 or 1";
+    r4.clear(); r6.clear();
+    for (uint32_t i = 0; i < s.n_rules; i++) {
+        const nfc_acl_rule &r = s.rules[i];
+        int maxl = r.family == 4 ? 32 : 128;
+        if (r.family != 4 && r.family != 6) return "acl: family must be 4 or 6";
+        if (r.slen > maxl || r.dlen > maxl) return "acl: prefix length out of range";
+        if (r.sp_lo > r.sp_hi || r.dp_lo > r.dp_hi) return "acl: port range lo > hi";
+        if (r.action > 1 || r.proto_any > 1) return "acl: bad action/proto_any";
+        uint4 tail = make_uint4((uint32_t)r.sp_lo | (uint32_t)r.sp_hi << 16, (uint32_t)r.dp_lo | (uint32_t)r.dp_hi << 16,
+                                (uint32_t)r.proto | (uint32_t)r.proto_any << 8 | (uint32_t)r.action << 16, i);
+        if (r.family == 4) {
+            uint32_t sm = mask32(r.slen), dm = mask32(r.dlen);
+            r4.push_back(make_uint4(be32(r.src) & sm, sm, be32(r.dst) & dm, dm));
+            r4.push_back(tail);
+        } else {
+            uint32_t sw[4], dw[4];
+            mask128(r.src, r.slen, sw);
+            mask128(r.dst, r.dlen, dw);
+            r6.push_back(make_uint4(sw[0], sw[1], sw[2], sw[3]));
+            r6.push_back(make_uint4(mask32(r.slen), mask32(r.slen - 32), mask32(r.slen - 64), mask32(r.slen - 96)));
+            r6.push_back(make_uint4(dw[0], dw[1], dw[2], dw[3]));
+            r6.push_back(make_uint4(mask32(r.dlen), mask32(r.dlen - 32), mask32(r.dlen - 64), mask32(r.dlen - 96)));
+            r6.push_back(tail);
+        }
+    }
+    return "";
+}
+
+// ---------------------------------------------------------------- DPI
+// Aho-Corasick (1975) goto/failure construction, converted to a full DFA over
+// byte classes (bytes that occur in no pattern form class 0: from every state
+// they lead to the root).
+std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
+{
+    if (s.n_patterns == 0 || s.n_patterns > 65535) return "dpi: n_patterns must be 1..65535";
+    if (!s.blob || !s.off || !s.action) return "dpi: NULL pointer";
+    // byte classes
+    std::array<int, 256> cls{};
+    cls.fill(0);
+    for (uint32_t j = 0; j < s.n_patterns; j++) {
+        if (s.off[j + 1] <= s.off[j]) return "dpi: empty pattern";
+        if (s.action[j] > 1) return "dpi: action must be 0 or 1";
+        for (uint32_t k = s.off[j]; k < s.off[j + 1]; k++) cls[s.blob[k]] = 1;
+    }
+    int ncls = 1;
+    for (int b = 0; b < 256; b++) cls[b] = cls[b] ? ncls++ : 0;
+    // trie with sparse children
+    std::vector<std::vector<std::pair<int, int>>> kids(1);   // (class, child)
+    std::vector<std::vector<uint16_t>> own(1);
+    for (uint32_t j = 0; j < s.n_patterns; j++) {
+        int st = 0;
+        for (uint32_t k = s.off[j]; k < s.off[j + 1]; k++) {
+            int c = cls[s.blob[k]], nx = -1;
+            for (auto &kc : kids[st]) if (kc.first == c) { nx = kc.second; break; }
+            if (nx < 0) {
+                nx = (int)kids.size();
+                kids.emplace_back();
+                own.emplace_back();
+                kids[st].push_back({c, nx});
+            }
+            st = nx;
+        }
+        own[st].push_back((uint16_t)j);
+    }
+    size_t n = kids.size();
+    // BFS renumbering
+    std::vector<int> order, newid(n, -1), fail(n, 0);
+    order.reserve(n);
+    order.push_back(0);
+    newid[0] = 0;
+    for (size_t h = 0; h < order.size(); h++) {
+        int u = order[h];
+        std::sort(kids[u].begin(), kids[u].end());
+        for (auto &kc : kids[u]) { newid[kc.second] = (int)order.size(); order.push_back(kc.second); }
+    }
+    // full DFA (old ids) in BFS order
+    std::vector<int> delta(n * ncls, 0);
+    std::vector<std::vector<uint16_t>> outc(n);
+    for (int u : order) {
+        int f = fail[u];
+        for (int c = 0; c < ncls; c++) delta[(size_t)u * ncls + c] = (u == 0) ? 0 : delta[(size_t)f * ncls + c];
+        for (auto &kc : kids[u]) {
+            int v = kc.second;
+            fail[v] = (u == 0) ? 0 : delta[(size_t)f * ncls + kc.first];
+            delta[(size_t)u * ncls + kc.first] = v;
+        }
+        // output closure: own(u) U out(fail(u)); fail(u) precedes u in BFS order
+        std::vector<uint16_t> oc = own[u];
+        if (u != 0) oc.insert(oc.end(), outc[fail[u]].begin(), outc[fail[u]].end());
+        std::sort(oc.begin(), oc.end());
+        oc.erase(std::unique(oc.begin(), oc.end()), oc.end());
+        outc[u] = std::move(oc);
+    }
+    o.ncls = (uint32_t)ncls;
+    o.n_states = (uint32_t)n;
+    o.wide = n > 32768 ? 1 : 0;
+    o.cls.resize(256);
+    for (int b = 0; b < 256; b++) o.cls[b] = (uint8_t)cls[b];
+    size_t es = o.wide ? 4 : 2;
+    o.trans.assign(n * ncls * es, 0);
+    for (size_t u = 0; u < n; u++) {
+        for (int c = 0; c < ncls; c++) {
+            int v = delta[u * ncls + c];
+            uint32_t e = (uint32_t)newid[v];
+            if (!outc[v].empty()) e |= o.wide ? 0x80000000u : 0x8000u;
+            size_t at = ((size_t)newid[u] * ncls + c) * es;
+            if (o.wide) memcpy(&o.trans[at], &e, 4);
+            else { uint16_t e16 = (uint16_t)e; memcpy(&o.trans[at], &e16, 2); }
+        }
+    }
+    o.out_off.assign(n + 1, 0);
+    o.out_ids.clear();
+    for (size_t k = 0; k < n; k++) {
+        int u = order[k];
+        o.out_off[k] = (uint32_t)o.out_ids.size();
+        o.out_ids.insert(o.out_ids.end(), outc[u].begin(), outc[u].end());
+    }
+    o.out_off[n] = (uint32_t)o.out_ids.size();
+    if (o.out_ids.empty()) o.out_ids.push_back(0);
+    o.action.assign(s.action, s.action + s.n_patterns);
+    return "";
+}
+
+// ---------------------------------------------------------------- next hops
+static std::string build_nh(uint32_t n_nh, const nfc_nexthop *nh, uint32_t n_ports, const uint8_t *pm,
+                            std::vector<uint2> &dn, std::vector<uint2> &dp)
+{
+    if (n_nh == 0 || n_nh > 32767 || !nh) return "lpm: n_nexthops must be 1..32767";
+    if (n_ports == 0 || !pm) return "lpm: need port MACs";
+    dn.resize(n_nh);
+    for (uint32_t i = 0; i < n_nh; i++) {
+        if (nh[i].port >= n_ports) return "lpm: next hop port >= n_ports";
+        const uint8_t *m = nh[i].mac;
+        dn[i] = make_uint2((uint32_t)m[0] | (uint32_t)m[1] << 8 | (uint32_t)m[2] << 16 | (uint32_t)m[3] << 24,
+                           (uint32_t)m[4] | (uint32_t)m[5] << 8 | (uint32_t)nh[i].port << 16);
+    }
+    dp.resize(n_ports);
+    for (uint32_t p = 0; p < n_ports; p++) {
+        const uint8_t *m = pm + 6 * p;
+        dp[p] = make_uint2((uint32_t)m[0] | (uint32_t)m[1] << 8 | (uint32_t)m[2] << 16 | (uint32_t)m[3] << 24,
+                           (uint32_t)m[4] | (uint32_t)m[5] << 8);
+    }
+    return "";
+}
+
+// ---------------------------------------------------------------- LPM4: DIR-24-8
+std::string build_lpm4(const nfc_lpm4_spec &s, std::vector<uint16_t> &tbl24, std::vector<uint16_t> &tbllong,
+                       std::vector<uint2> &nh, std::vector<uint2> &pmac)
+{
+    std::string e = build_nh(s.n_nexthops, s.nexthops, s.n_ports, s.port_macs, nh, pmac);
+    if (!e.empty()) return e;
+    if (s.n_routes && !s.routes) return "lpm4: routes == NULL";
+    std::vector<uint32_t> idx(s.n_routes);
+    std::unordered_map<uint64_t, int> seen;
+    for (uint32_t i = 0; i < s.n_routes; i++) {
+        const nfc_route4 &r = s.routes[i];
+        if (r.len > 32) return "lpm4: len > 32";
+        if (r.prefix & ~mask32(r.len)) return "lpm4: host bits set in prefix";
+        if (r.nh >= s.n_nexthops) return "lpm4: nh out of range";
+        if (!seen.emplace((uint64_t)r.prefix << 8 | r.len, 1).second) return "lpm4: duplicate prefix";
+        idx[i] = i;
+    }
+    std::stable_sort(idx.begin(), idx.end(), [&](uint32_t a, uint32_t b) { return s.routes[a].len < s.routes[b].len; });
+    tbl24.assign(1u << 24, 0x7FFF);
+    tbllong.clear();
+    for (uint32_t i : idx) {
+        const nfc_route4 &r = s.routes[i];
+        if (r.len <= 24) {
+            uint32_t first = r.prefix >> 8, cnt = 1u << (24 - r.len);
+            for (uint32_t k = 0; k < cnt; k++) tbl24[first + k] = r.nh;
+        } else {
+            uint32_t t = r.prefix >> 8;
+            if (!(tbl24[t] & 0x8000)) {
+                uint32_t g = (uint32_t)(tbllong.size() / 256);
+                if (g >= 0x8000) return "lpm4: too many /25+ groups";
+                tbllong.insert(tbllong.end(), 256, tbl24[t]);
+                tbl24[t] = (uint16_t)(0x8000 | g);
+            }
+            uint32_t g = tbl24[t] & 0x7FFF, first = r.prefix & 0xFF, cnt = 1u << (32 - r.len);
+            for (uint32_t k = 0; k < cnt; k++) tbllong[g * 256 + first + k] = r.nh;
+        }
+    }
+    if (tbllong.empty()) tbllong.assign(256, 0x7FFF);
+    return "";
+}
+
+// ---------------------------------------------------------------- LPM6: Waldvogel
+namespace {
+struct BitTrie {
+    struct N { int c[2]; int nh; };
+    std::vector<N> n{N{{-1, -1}, -1}};
+    void insert(const uint32_t w[4], int len, int nh)
+    {
+        int u = 0;
+        for (int i = 0; i < len; i++) {
+            int b = (w[i >> 5] >> (31 - (i & 31))) & 1;
+            if (n[u].c[b] < 0) { n[u].c[b] = (int)n.size(); n.push_back(N{{-1, -1}, -1}); }
+            u = n[u].c[b];
+        }
+        n[u].nh = nh;
+    }
+    int best(const uint32_t w[4], int len) const  // longest real prefix of length <= len matching w
+    {
+        int u = 0, b = n[0].nh;
+        for (int i = 0; i < len && u >= 0; i++) {
+            u = n[u].c[(w[i >> 5] >> (31 - (i & 31))) & 1];
+            if (u >= 0 && n[u].nh >= 0) b = n[u].nh;
+        }
+        return b;
+    }
+};
+struct K4 {
+    uint32_t w[4];
+    bool operator==(const K4 &o) const { return memcmp(w, o.w, 16) == 0; }
+};
+struct K4H { size_t operator()(const K4 &k) const { return l6_hash(k.w[0], k.w[1], k.w[2], k.w[3]); } };
+} // namespace
+
+std::string build_lpm6(const nfc_lpm6_spec &s, Lpm6Host &o)
+{
+    std::string e = build_nh(s.n_nexthops, s.nexthops, s.n_ports, s.port_macs, o.nh, o.pmac);
+    if (!e.empty()) return e;
+    if (s.n_routes && !s.routes) return "lpm6: routes == NULL";
+    BitTrie trie;
+    std::vector<int> present(129, 0);
+    o.def_nh = 0x7FFF;
+    std::unordered_map<K4, int, K4H> dup[129];
+    for (uint32_t i = 0; i < s.n_routes; i++) {
+        const nfc_route6 &r = s.routes[i];
+        if (r.len > 128) return "lpm6: len > 128";
+        if (r.nh >= s.n_nexthops) return "lpm6: nh out of range";
+        K4 k;
+        mask128(r.prefix, r.len, k.w);
+        for (int q = 0; q < 4; q++)
+            if (be32(r.prefix + 4 * q) != k.w[q]) return "lpm6: host bits set in prefix";
+        if (!dup[r.len].emplace(k, 1).second) return "lpm6: duplicate prefix";
+        trie.insert(k.w, r.len, r.nh);
+        present[r.len] = 1;
+        if (r.len == 0) o.def_nh = r.nh;
+    }
+    o.lens.clear();
+    std::vector<int> lvl(129, -1);
+    for (int L = 1; L <= 128; L++)
+        if (present[L]) { lvl[L] = (int)o.lens.size(); o.lens.push_back((uint8_t)L); }
+    int m = (int)o.lens.size();
+    std::vector<std::unordered_map<K4, uint32_t, K4H>> tab(m);
+    for (uint32_t i = 0; i < s.n_routes; i++) {
+        const nfc_route6 &r = s.routes[i];
+        if (r.len == 0) continue;
+        K4 k;
+        mask128(r.prefix, r.len, k.w);
+        int t = lvl[r.len];
+        tab[t][k] = 0;
+        // markers on the binary-search path towards level t
+        int lo = 0, hi = m - 1;
+        while (lo <= hi) {
+            int mid = (lo + hi) >> 1;
+            if (mid == t) break;
+            if (mid < t) {
+                K4 mk;
+                for (int q = 0; q < 4; q++) mk.w[q] = k.w[q] & mask32(o.lens[mid] - 32 * q);
+                tab[mid].emplace(mk, 0);
+                lo = mid + 1;
+            } else {
+                hi = mid - 1;
+            }
+        }
+    }
+    o.base.assign(m, 0);
+    o.mask.assign(m, 0);
+    o.ent.clear();
+    for (int j = 0; j < m; j++) {
+        size_t cnt = tab[j].size(), sz = 2;
+        while (sz < 2 * cnt) sz <<= 1;
+        o.base[j] = (uint32_t)o.ent.size();
+        o.mask[j] = (uint32_t)(sz - 1);
+        o.ent.resize(o.ent.size() + sz);
+        Lpm6Entry *T = &o.ent[o.base[j]];
+        memset(T, 0, sz * sizeof(Lpm6Entry));
+        for (auto &kv : tab[j]) {
+            int b = trie.best(kv.first.w, o.lens[j]);
+            uint32_t info = (b < 0 ? 0x7FFFu : (uint32_t)b) | L6_VALID;
+            uint32_t h = l6_hash(kv.first.w[0], kv.first.w[1], kv.first.w[2], kv.first.w[3]) & o.mask[j];
+            while (T[h].info & L6_VALID) h = (h + 1) & o.mask[j];
+            memcpy(T[h].key, kv.first.w, 16);
+            T[h].info = info;
+        }
+    }
+    if (o.ent.empty()) o.ent.resize(2);
+    if (o.lens.empty()) { o.base.push_back(0); o.mask.push_back(1); }
+    return "";
+}
+
+// ---------------------------------------------------------------- AES-128 / HMAC-SHA1
+// S-box through exp/log tables of generator 3 in GF(2^8) and the FIPS-197
+// affine map; Te tables as in the classic 32-bit T-table formulation.
+static uint8_t xt(uint8_t x) { return (uint8_t)((x << 1) ^ ((x & 0x80) ? 0x1b : 0)); }
+static void sbox_tables(uint8_t sb[256])
+{
+    uint8_t ex[256], lg[256] = {0};
+    uint8_t x = 1;
+    for (int i = 0; i < 255; i++) { ex[i] = x; lg[x] = (uint8_t)i; x = (uint8_t)(x ^ xt(x)); }
+    for (int v = 0; v < 256; v++) {
+        uint8_t inv = v ? ex[(255 - lg[v]) % 255] : 0;
+        uint8_t r = inv;
+        for (int k = 1; k <= 4; k++) r ^= (uint8_t)((inv << k) | (inv >> (8 - k)));
+        sb[v] = (uint8_t)(r ^ 0x63);
+    }
+}
+
+void build_aes_tables(std::vector<uint32_t> &te)
+{
+    uint8_t sb[256];
+    sbox_tables(sb);
+    te.assign(5 * 256, 0);
+    for (int v = 0; v < 256; v++) {
+        uint8_t s = sb[v], s2 = xt(s), s3 = (uint8_t)(s2 ^ s);
+        uint32_t t0 = (uint32_t)s2 << 24 | (uint32_t)s << 16 | (uint32_t)s << 8 | s3;
+        te[v] = t0;
+        te[256 + v] = (t0 >> 8) | (t0 << 24);
+        te[512 + v] = (t0 >> 16) | (t0 << 16);
+        te[768 + v] = (t0 >> 24) | (t0 << 8);
+        te[1024 + v] = s;
+    }
+}
+
+static void aes_expand(const uint8_t key[16], uint32_t rk[44])
+{
+    uint8_t sb[256];
+    sbox_tables(sb);
+    for (int i = 0; i < 4; i++) rk[i] = be32(key + 4 * i);
+    uint8_t rc = 1;
+    for (int i = 4; i < 44; i++) {
+        uint32_t t = rk[i - 1];
+        if ((i & 3) == 0) {
+            t = (t << 8) | (t >> 24);
+            t = (uint32_t)sb[t >> 24] << 24 | (uint32_t)sb[(t >> 16) & 255] << 16 | (uint32_t)sb[(t >> 8) & 255] << 8 | sb[t & 255];
+            t ^= (uint32_t)rc << 24;
+            rc = xt(rc);
+        }
+        rk[i] = rk[i - 4] ^ t;
+    }
+}
+
+static inline uint32_t rol(uint32_t x, int n) { return (x << n) | (x >> (32 - n)); }
+static void sha1_compress(uint32_t h[5], const uint8_t blk[64])
+{
+    uint32_t w[80];
+    for (int t = 0; t < 16; t++) w[t] = be32(blk + 4 * t);
+    for (int t = 16; t < 80; t++) w[t] = rol(w[t - 3] ^ w[t - 8] ^ w[t - 14] ^ w[t - 16], 1);
+    uint32_t a = h[0], b = h[1], c = h[2], d = h[3], e = h[4];
+    for (int t = 0; t < 80; t++) {
+        uint32_t f, k;
+        if (t < 20) { f = d ^ (b & (c ^ d)); k = 0x5a827999u; }
+        else if (t < 40) { f = b ^ c ^ d; k = 0x6ed9eba1u; }
+        else if (t < 60) { f = (b & c) | (d & (b | c)); k = 0x8f1bbcdcu; }
+        else { f = b ^ c ^ d; k = 0xca62c1d6u; }
+        uint32_t tmp = rol(a, 5) + f + e + k + w[t];
+        e = d; d = c; c = rol(b, 30); b = a; a = tmp;
+    }
+    h[0] += a; h[1] += b; h[2] += c; h[3] += d; h[4] += e;
+}
+
+std::string build_ipsec(const nfc_ipsec_spec &s, std::vector<EspSa> &out)
+{
+    if (s.n_sa == 0 || s.n_sa > 255 || !s.sas) return "ipsec: n_sa must be 1..255";
+    out.assign(s.n_sa, EspSa{});
+    for (uint32_t i = 0; i < s.n_sa; i++) {
+        const nfc_sa &a = s.sas[i];
+        EspSa &d = out[i];
+        aes_expand(a.aes_key, d.rk);
+        d.spi = a.spi;
+        d.nonce = be32(a.nonce);
+        uint8_t blk[64];
+        static const uint32_t IV[5] = {0x67452301u, 0xefcdab89u, 0x98badcfeu, 0x10325476u, 0xc3d2e1f0u};
+        for (int pass = 0; pass < 2; pass++) {
+            uint8_t pad = pass ? 0x5c : 0x36;
+            for (int k = 0; k < 64; k++) blk[k] = (uint8_t)((k < 20 ? a.auth_key[k] : 0) ^ pad);
+            uint32_t *st = pass ? d.opad : d.ipad;
+            memcpy(st, IV, sizeof IV);
+            sha1_compress(st, blk);
+        }
+    }
+    return "";
+}
+
+// ---------------------------------------------------------------- Toeplitz
+// nib[k*16 + v] = XOR of the 32-bit key windows at input bit positions
+// 4k..4k+3 selected by the bits of nibble v (MSB first).
+void build_toeplitz_nibbles(const uint8_t key[40], std::vector<uint32_t> &nib)
+{
+    auto window = [&](int bit) {
+        uint32_t w = 0;
+        for (int j = 0; j < 32; j++) {
+            int kb = bit + j;
+            int v = kb < 320 ? (key[kb >> 3] >> (7 - (kb & 7))) & 1 : 0;
+            w = (w << 1) | (uint32_t)v;
+        }
+        return w;
+    };
+    nib.assign(72 * 16, 0);
+    for (int k = 0; k < 72; k++)
+        for (int v = 0; v < 16; v++) {
+            uint32_t h = 0;
+            for (int j = 0; j < 4; j++)
+                if ((v >> (3 - j)) & 1) h ^= window(4 * k + j);
+            nib[k * 16 + v] = h;
+        }
+}
+
+} // namespace nfc

@@ -1,0 +1,445 @@
+// capi.cu -- the C ABI (include/nfc.h): chain object, table upload, launch,
+// stats.  Host runtime around the fused kernel; no compute happens here
+// beyond building table images (builders.cpp).
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "nfc_internal.h"
+
+using namespace nfc;
+
+static thread_local std::string g_err;
+
+static int fail(int code, const std::string &msg)
+{
+    g_err = msg;
+    return code;
+}
+
+#define CK(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) return fail(NFC_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+    } while (0)
+
+namespace {
+struct DBuf {
+    void *p = nullptr;
+    size_t n = 0;
+    void release()
+    {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+    cudaError_t reserve(size_t bytes)
+    {
+        if (bytes <= n && p) return cudaSuccess;
+        release();
+        cudaError_t e = cudaMalloc(&p, bytes ? bytes : 16);
+        if (e == cudaSuccess) n = bytes;
+        return e;
+    }
+    template <typename T> cudaError_t upload(const std::vector<T> &v)
+    {
+        cudaError_t e = reserve(v.size() * sizeof(T));
+        if (e != cudaSuccess) return e;
+        return v.empty() ? cudaSuccess : cudaMemcpy(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+    }
+    template <typename T> T *as() const { return reinterpret_cast<T *>(p); }
+};
+} // namespace
+
+struct nfc_chain {
+    int device = 0;
+    uint32_t n_nf = 0;
+    uint32_t kind[NFC_MAX_CHAIN] = {0};
+    uint32_t mask = 0;
+    uint32_t esp_pos = 0xFF;
+    bool loaded[8] = {false};
+    // tables
+    DBuf acl_r4, acl_r6;
+    AclImg acl{};
+    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap;
+    DpiImg dpi{};
+    DBuf l4_tbl24, l4_long, l4_nh, l4_pmac;
+    Lpm4Img l4{};
+    DBuf l6_lens, l6_base, l6_mask, l6_ent, l6_nh, l6_pmac;
+    Lpm6Img l6{};
+    DBuf esp_sa, esp_te, esp_nib, esp_seq[2];
+    EspImg esp{};
+    uint32_t seq_parity = 0;
+    DBuf lb_port, lb_nib;
+    LbImg lb{};
+    // stats
+    DBuf stats;
+    uint32_t stats_len = ST_VAR_BASE;
+    uint32_t n_acl_rules = 0, n_lb = 0, n_sa = 0;
+    // scheduling
+    DBuf counter, tile_flag, tile_vec, batches;
+    uint32_t tile_cap = 0;
+    uint32_t epoch = 0;
+    // host e2e staging
+    DBuf h_arena, h_off, h_len, h_rec, h_mp, h_mq, h_mc;
+    uint64_t launches = 0;
+    cudaStream_t last_stream = nullptr;
+};
+
+static int set_device(const nfc_chain *c)
+{
+    CK(cudaSetDevice(c->device));
+    return NFC_OK;
+}
+
+static int realloc_stats(nfc_chain *c)
+{
+    c->stats_len = ST_VAR_BASE + (c->n_acl_rules + 1) + c->n_lb + c->n_sa;
+    CK(c->stats.reserve((size_t)c->stats_len * 8));
+    CK(cudaMemset(c->stats.p, 0, (size_t)c->stats_len * 8));
+    return NFC_OK;
+}
+
+extern "C" {
+
+const char *nfc_last_error(void) { return g_err.c_str(); }
+const char *nfc_version(void) { return "nfc-b200 0.1 (sm_100a)"; }
+
+int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opts, nfc_chain **out)
+{
+    if (!kinds || !out) return fail(NFC_EINVAL, "kinds/out is NULL");
+    if (n < 1 || n > NFC_MAX_CHAIN) return fail(NFC_EUNSUP, "chain length must be 1..6");
+    uint32_t mask = 0;
+    for (uint32_t i = 0; i < n; i++) {
+        if (kinds[i] < NFC_ACL || kinds[i] > NFC_LB) return fail(NFC_EINVAL, "unknown NF kind");
+        if (mask & (1u << kinds[i])) return fail(NFC_EUNSUP, "repeated NF kind in chain");
+        mask |= 1u << kinds[i];
+    }
+    if (opts && opts->flags) return fail(NFC_EINVAL, "opts->flags must be 0");
+    nfc_chain *c = new (std::nothrow) nfc_chain();
+    if (!c) return fail(NFC_ENOMEM, "out of host memory");
+    c->device = opts ? opts->device : 0;
+    c->n_nf = n;
+    c->mask = mask;
+    for (uint32_t i = 0; i < n; i++) {
+        c->kind[i] = kinds[i];
+        if (kinds[i] == NFC_IPSEC) c->esp_pos = i;
+    }
+    int rc = set_device(c);
+    if (rc == NFC_OK) {
+        cudaError_t e = c->counter.reserve(16);
+        if (e == cudaSuccess) e = cudaMemset(c->counter.p, 0, 16);
+        if (e != cudaSuccess) rc = fail(NFC_ECUDA, cudaGetErrorString(e));
+    }
+    if (rc == NFC_OK) rc = realloc_stats(c);
+    if (rc != NFC_OK) {
+        nfc_destroy_chain(c);
+        return rc;
+    }
+    *out = c;
+    return NFC_OK;
+}
+
+void nfc_destroy_chain(nfc_chain *c)
+{
+    if (!c) return;
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
+                   &c->dpi_bitmap, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
+                   &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
+                   &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
+                   &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
+                   &c->h_mp, &c->h_mq, &c->h_mc};
+    for (DBuf *b : all) b->release();
+    delete c;
+}
+
+int nfc_chain_room(const nfc_chain *c, uint32_t *headroom, uint32_t *tailroom)
+{
+    if (!c || !headroom || !tailroom) return fail(NFC_EINVAL, "NULL argument");
+    bool esp = (c->mask & MASK_IPSEC) != 0;
+    *headroom = esp ? 16 : 0;
+    *tailroom = esp ? 32 : 0;
+    return NFC_OK;
+}
+
+int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_bytes)
+{
+    if (!c || !spec) return fail(NFC_EINVAL, "NULL argument");
+    if (kind < NFC_ACL || kind > NFC_LB) return fail(NFC_EINVAL, "unknown NF kind");
+    int rc = set_device(c);
+    if (rc) return rc;
+    cudaDeviceSynchronize();   // tables are replaced atomically w.r.t. later launches
+    std::string err;
+    switch (kind) {
+    case NFC_ACL: {
+        if (spec_bytes != sizeof(nfc_acl_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_acl_spec)");
+        const nfc_acl_spec &s = *static_cast<const nfc_acl_spec *>(spec);
+        std::vector<uint4> r4, r6;
+        err = build_acl(s, r4, r6);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        CK(c->acl_r4.upload(r4));
+        CK(c->acl_r6.upload(r6));
+        c->acl = AclImg{c->acl_r4.as<uint4>(), (uint32_t)(r4.size() / 2), c->acl_r6.as<uint4>(),
+                        (uint32_t)(r6.size() / 5), s.n_rules, s.default_action};
+        c->n_acl_rules = s.n_rules;
+        break;
+    }
+    case NFC_DPI: {
+        if (spec_bytes != sizeof(nfc_dpi_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_dpi_spec)");
+        DpiHost d;
+        err = build_dpi(*static_cast<const nfc_dpi_spec *>(spec), d);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        CK(c->dpi_cls.upload(d.cls));
+        CK(c->dpi_trans.upload(d.trans));
+        CK(c->dpi_off.upload(d.out_off));
+        CK(c->dpi_ids.upload(d.out_ids));
+        CK(c->dpi_act.upload(d.action));
+        c->dpi = DpiImg{};
+        c->dpi.cls = c->dpi_cls.as<uint8_t>();
+        c->dpi.trans = c->dpi_trans.p;
+        c->dpi.ncls = d.ncls;
+        c->dpi.n_states = d.n_states;
+        c->dpi.wide = d.wide;
+        c->dpi.out_off = c->dpi_off.as<uint32_t>();
+        c->dpi.out_ids = c->dpi_ids.as<uint16_t>();
+        c->dpi.pat_action = c->dpi_act.as<uint8_t>();
+        c->dpi.n_pat = (uint32_t)d.action.size();
+        c->dpi.bitmap_words = (c->dpi.n_pat + 31) / 32;
+        break;
+    }
+    case NFC_LPM4: {
+        if (spec_bytes != sizeof(nfc_lpm4_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_lpm4_spec)");
+        std::vector<uint16_t> t24, tl;
+        std::vector<uint2> nh, pm;
+        err = build_lpm4(*static_cast<const nfc_lpm4_spec *>(spec), t24, tl, nh, pm);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        CK(c->l4_tbl24.upload(t24));
+        CK(c->l4_long.upload(tl));
+        CK(c->l4_nh.upload(nh));
+        CK(c->l4_pmac.upload(pm));
+        c->l4 = Lpm4Img{c->l4_tbl24.as<uint16_t>(), c->l4_long.as<uint16_t>(), c->l4_nh.as<uint2>(),
+                        c->l4_pmac.as<uint2>(), (uint32_t)nh.size(), (uint32_t)pm.size()};
+        break;
+    }
+    case NFC_LPM6: {
+        if (spec_bytes != sizeof(nfc_lpm6_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_lpm6_spec)");
+        Lpm6Host h;
+        err = build_lpm6(*static_cast<const nfc_lpm6_spec *>(spec), h);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        CK(c->l6_lens.upload(h.lens));
+        CK(c->l6_base.upload(h.base));
+        CK(c->l6_mask.upload(h.mask));
+        CK(c->l6_ent.upload(h.ent));
+        CK(c->l6_nh.upload(h.nh));
+        CK(c->l6_pmac.upload(h.pmac));
+        c->l6 = Lpm6Img{(uint32_t)h.lens.size(), h.def_nh, c->l6_lens.as<uint8_t>(), c->l6_base.as<uint32_t>(),
+                        c->l6_mask.as<uint32_t>(), c->l6_ent.as<uint4>(), c->l6_nh.as<uint2>(),
+                        c->l6_pmac.as<uint2>(), (uint32_t)h.nh.size(), (uint32_t)h.pmac.size()};
+        break;
+    }
+    case NFC_IPSEC: {
+        if (spec_bytes != sizeof(nfc_ipsec_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_ipsec_spec)");
+        const nfc_ipsec_spec &s = *static_cast<const nfc_ipsec_spec *>(spec);
+        std::vector<EspSa> sa;
+        err = build_ipsec(s, sa);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        std::vector<uint32_t> te, nib, seq(s.n_sa);
+        build_aes_tables(te);
+        build_toeplitz_nibbles(MS_RSS_KEY, nib);
+        for (uint32_t i = 0; i < s.n_sa; i++) seq[i] = s.sas[i].seq0;
+        CK(c->esp_sa.upload(sa));
+        CK(c->esp_te.upload(te));
+        CK(c->esp_nib.upload(nib));
+        CK(c->esp_seq[0].upload(seq));
+        CK(c->esp_seq[1].upload(seq));
+        c->seq_parity = 0;
+        c->esp = EspImg{c->esp_sa.as<EspSa>(), s.n_sa, c->esp_te.as<uint32_t>(), c->esp_nib.as<uint32_t>()};
+        c->n_sa = s.n_sa;
+        break;
+    }
+    case NFC_LB: {
+        if (spec_bytes != sizeof(nfc_lb_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_lb_spec)");
+        const nfc_lb_spec &s = *static_cast<const nfc_lb_spec *>(spec);
+        if (s.n_backends == 0 || s.n_backends > 65535 || !s.backend_port || !s.key)
+            return fail(NFC_EINVAL, "lb: n_backends must be 1..65535 with ports and key");
+        std::vector<uint16_t> ports(s.backend_port, s.backend_port + s.n_backends);
+        std::vector<uint32_t> nib;
+        build_toeplitz_nibbles(s.key, nib);
+        CK(c->lb_port.upload(ports));
+        CK(c->lb_nib.upload(nib));
+        c->lb = LbImg{c->lb_port.as<uint16_t>(), s.n_backends, c->lb_nib.as<uint32_t>()};
+        c->n_lb = s.n_backends;
+        break;
+    }
+    }
+    c->loaded[kind] = true;
+    return realloc_stats(c);
+}
+
+static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nfc_result *r, cudaStream_t st)
+{
+    for (uint32_t i = 0; i < c->n_nf; i++)
+        if (!c->loaded[c->kind[i]]) return fail(NFC_ESTATE, "tables not loaded for an NF of the chain");
+    if (!r || !r->rec) return fail(NFC_EINVAL, "result buffers missing");
+    if ((c->mask & MASK_DPI) && !r->match_count) return fail(NFC_EINVAL, "match_count is required for DPI chains");
+    if (nb && !bs) return fail(NFC_EINVAL, "batches is NULL");
+    std::vector<BatchDev> hb(nb);
+    uint64_t total = 0;
+    for (uint32_t i = 0; i < nb; i++) {
+        if (bs[i].n && (!bs[i].arena || !bs[i].off || !bs[i].len)) return fail(NFC_EINVAL, "batch pointers NULL");
+        hb[i] = BatchDev{bs[i].arena, bs[i].off, bs[i].len, bs[i].n, (uint32_t)total, bs[i].first_global_index};
+        total += bs[i].n;
+    }
+    if (total > 0xFFFFFFFFull - 1024) return fail(NFC_EINVAL, "too many packets in one call");
+    c->last_stream = st;
+    if (total == 0) return NFC_OK;
+    int rc = set_device(c);
+    if (rc) return rc;
+    const uint32_t TILE_N = 256;
+    uint32_t n_tiles = (uint32_t)((total + TILE_N - 1) / TILE_N);
+    CK(c->batches.reserve(hb.size() * sizeof(BatchDev)));
+    CK(cudaMemcpyAsync(c->batches.p, hb.data(), hb.size() * sizeof(BatchDev), cudaMemcpyHostToDevice, st));
+    CK(cudaMemsetAsync(c->counter.p, 0, 4, st));
+
+    KParams p{};
+    p.n_nf = c->n_nf;
+    for (uint32_t i = 0; i < c->n_nf; i++) p.kind[i] = c->kind[i];
+    p.esp_pos = c->esp_pos;
+    p.batches = c->batches.as<BatchDev>();
+    p.n_batches = nb;
+    p.n_pkts = (uint32_t)total;
+    p.n_tiles = n_tiles;
+    p.tile_counter = c->counter.as<uint32_t>();
+    p.rec = r->rec;
+    p.match_pkt = r->match_pkt;
+    p.match_pat = r->match_pat;
+    p.match_cap = r->match_pkt && r->match_pat ? r->match_cap : 0;
+    p.match_count = r->match_count;
+    p.stats = c->stats.as<unsigned long long>();
+    p.stats_len = c->stats_len;
+    p.st_acl = ST_VAR_BASE;
+    p.st_lb = ST_VAR_BASE + c->n_acl_rules + 1;
+    p.st_sa = p.st_lb + c->n_lb;
+    p.smem_stats = c->stats_len <= 4096 ? 1 : 0;
+    p.acl = c->acl;
+    p.dpi = c->dpi;
+    p.l4 = c->l4;
+    p.l6 = c->l6;
+    p.esp = c->esp;
+    p.lb = c->lb;
+    if (c->mask & MASK_IPSEC) {
+        if (n_tiles > c->tile_cap) {
+            uint32_t cap = n_tiles + n_tiles / 4 + 64;
+            CK(c->tile_flag.reserve((size_t)cap * 4));
+            CK(cudaMemset(c->tile_flag.p, 0, (size_t)cap * 4));
+            CK(c->tile_vec.reserve((size_t)cap * 2 * c->n_sa * 4));
+            c->tile_cap = cap;
+            c->epoch = 0;
+        }
+        c->epoch = (c->epoch + 1) & 0x3FFFFFFF;
+        if (c->epoch == 0) {
+            CK(cudaMemsetAsync(c->tile_flag.p, 0, (size_t)c->tile_cap * 4, st));
+            c->epoch = 1;
+        }
+        p.tile_flag = c->tile_flag.as<uint32_t>();
+        p.tile_vec = c->tile_vec.as<uint32_t>();
+        p.epoch = c->epoch;
+        p.seq_in = c->esp_seq[c->seq_parity].as<uint32_t>();
+        p.seq_out = c->esp_seq[c->seq_parity ^ 1].as<uint32_t>();
+    }
+    if (c->mask & MASK_DPI) {
+        LaunchCfg q{};
+        if (sfc_query(c->mask, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");
+        size_t need = (size_t)q.grid * q.block * c->dpi.bitmap_words * 4;
+        CK(c->dpi_bitmap.reserve(need));
+        c->dpi.ovf_bitmap = c->dpi_bitmap.as<uint32_t>();
+        p.dpi.ovf_bitmap = c->dpi.ovf_bitmap;
+    }
+    std::string err;
+    rc = sfc_launch(c->mask, p, c->device, st, err, nullptr);
+    if (rc) return fail(rc, err);
+    c->launches++;
+    if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;
+    return NFC_OK;
+}
+
+int nfc_process_batch(nfc_chain *c, const nfc_batch *batches, uint32_t n_batches, const nfc_result *r, void *stream)
+{
+    if (!c) return fail(NFC_EINVAL, "chain is NULL");
+    return process_impl(c, batches, n_batches, r, static_cast<cudaStream_t>(stream));
+}
+
+int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const uint64_t *off, const uint16_t *len,
+                     uint32_t n, uint64_t first_global_index, nfc_pkt_result *rec, uint32_t *match_pkt,
+                     uint16_t *match_pat, uint32_t match_cap, uint32_t *n_pairs, void *stream)
+{
+    if (!c || (n && (!arena || !off || !len || !rec))) return fail(NFC_EINVAL, "NULL argument");
+    int rc = set_device(c);
+    if (rc) return rc;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    CK(c->h_arena.reserve(arena_bytes + 64));
+    CK(c->h_off.reserve((size_t)n * 8));
+    CK(c->h_len.reserve((size_t)n * 2));
+    CK(c->h_rec.reserve((size_t)n * sizeof(nfc_pkt_result)));
+    CK(c->h_mp.reserve((size_t)match_cap * 4));
+    CK(c->h_mq.reserve((size_t)match_cap * 2));
+    CK(c->h_mc.reserve(4));
+    CK(cudaMemcpyAsync(c->h_arena.p, arena, arena_bytes, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(c->h_off.p, off, (size_t)n * 8, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(c->h_len.p, len, (size_t)n * 2, cudaMemcpyHostToDevice, st));
+    CK(cudaMemsetAsync(c->h_mc.p, 0, 4, st));
+    nfc_batch b{c->h_arena.as<uint8_t>(), c->h_off.as<uint64_t>(), c->h_len.as<uint16_t>(), n, 0, first_global_index};
+    nfc_result r{c->h_rec.as<nfc_pkt_result>(), c->h_mp.as<uint32_t>(), c->h_mq.as<uint16_t>(), match_cap, 0,
+                 c->h_mc.as<uint32_t>()};
+    rc = process_impl(c, &b, 1, &r, st);
+    if (rc) return rc;
+    uint32_t cnt = 0;
+    CK(cudaMemcpyAsync(arena, c->h_arena.p, arena_bytes, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(rec, c->h_rec.p, (size_t)n * sizeof(nfc_pkt_result), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&cnt, c->h_mc.p, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    uint32_t k = cnt < match_cap ? cnt : match_cap;
+    if (k && match_pkt && match_pat) {
+        CK(cudaMemcpyAsync(match_pkt, c->h_mp.p, (size_t)k * 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(match_pat, c->h_mq.p, (size_t)k * 2, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+    }
+    if (n_pairs) *n_pairs = cnt;
+    return NFC_OK;
+}
+
+int nfc_stats_len(const nfc_chain *c, size_t *len)
+{
+    if (!c || !len) return fail(NFC_EINVAL, "NULL argument");
+    *len = c->stats_len;
+    return NFC_OK;
+}
+
+int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags)
+{
+    if (!c || (!out && cap)) return fail(NFC_EINVAL, "NULL argument");
+    int rc = set_device(c);
+    if (rc) return rc;
+    CK(cudaDeviceSynchronize());
+    std::vector<uint64_t> h(c->stats_len);
+    CK(cudaMemcpy(h.data(), c->stats.p, (size_t)c->stats_len * 8, cudaMemcpyDeviceToHost));
+    size_t k = cap < h.size() ? cap : h.size();
+    if (k) memcpy(out, h.data(), k * 8);
+    if (flags & NFC_STATS_RESET) CK(cudaMemset(c->stats.p, 0, (size_t)c->stats_len * 8));
+    if (h[ST_MATCH_OVF]) return fail(NFC_ECAP, "match pairs exceeded match_cap");
+    return NFC_OK;
+}
+
+int nfc_launch_count(const nfc_chain *c, uint64_t *count)
+{
+    if (!c || !count) return fail(NFC_EINVAL, "NULL argument");
+    *count = c->launches;
+    return NFC_OK;
+}
+
+} // extern "C"

@@ -1,0 +1,187 @@
+// nfc_internal.h -- device image formats and kernel parameters shared by the
+// host table builders (builders.cpp), the C ABI (capi.cu) and the fused
+// kernel (sfc_kernel.cu).  Product code only; nothing here is seen by oracle/.
+#pragma once
+#include <stdint.h>
+#include <vector_functions.h>
+#include <vector_types.h>
+#include <string>
+#include <vector>
+
+#include "../../include/nfc.h"
+
+namespace nfc {
+
+// ---------------------------------------------------------------- ACL
+// Linear first-match image, rules of one family in priority order.
+// IPv4 rule = 2 x uint4:  {src, smask, dst, dmask}, {sp_lo|sp_hi<<16, dp_lo|dp_hi<<16,
+//                          proto | proto_any<<8 | action<<16, global rule index}
+// IPv6 rule = 5 x uint4:  src[4], smask[4], dst[4], dmask[4] (BE-value words), then the
+//                          same tail word group.
+struct AclImg {
+    const uint4 *r4; uint32_t n4;
+    const uint4 *r6; uint32_t n6;
+    uint32_t n_rules;
+    uint32_t default_action;
+};
+
+// ---------------------------------------------------------------- DPI
+// Full Aho-Corasick DFA over byte classes, states numbered in BFS order.
+// trans[s * ncls + cls[b]] = next | ACCEPT (bit 15 for u16, bit 31 for u32
+// entries) where ACCEPT means the next state has a non-empty output set.
+// out_off/out_ids: CSR of the output closure (sorted distinct pattern ids).
+struct DpiImg {
+    const uint8_t *cls;          // 256 byte -> class
+    const void *trans;           // u16 or u32 entries
+    uint32_t ncls, n_states, wide;
+    const uint32_t *out_off;     // n_states + 1
+    const uint16_t *out_ids;
+    const uint8_t *pat_action;   // n_pat
+    uint32_t n_pat;
+    uint32_t *ovf_bitmap;        // per resident thread scratch for > DPI_LIST distinct matches
+    uint32_t bitmap_words;       // words per thread
+    uint32_t smem_states;        // rows of trans staged in shared memory (0 = none)
+};
+
+// ---------------------------------------------------------------- LPM4 (DIR-24-8)
+// tbl24[dst>>8]: bit 15 set -> long group g = v & 0x7FFF, nh = tbllong[g*256 + (dst&255)];
+// else nh = v.  nh == 0x7FFF means no route.
+struct Lpm4Img {
+    const uint16_t *tbl24;
+    const uint16_t *tbllong;
+    const uint2 *nh;             // {port | mac0<<16 | mac1<<24, mac2..mac5}
+    const uint2 *pmac;           // per port: {mac0..3, mac4|mac5<<8}
+    uint32_t n_nh, n_ports;
+};
+
+// ---------------------------------------------------------------- LPM6 (Waldvogel)
+// Binary search on the sorted distinct prefix lengths; one hash table per
+// length holding real prefixes and markers, each entry carrying the best
+// matching real prefix (bmp) of length <= its level.
+struct Lpm6Entry { uint32_t key[4]; uint32_t info; uint32_t pad[3]; }; // info: bmp | VALID
+static const uint32_t L6_VALID = 0x80000000u;
+struct Lpm6Img {
+    uint32_t n_levels;
+    uint32_t def_nh;             // ::/0 next hop or 0x7FFF
+    const uint8_t *lens;         // n_levels
+    const uint32_t *base;        // entry offset per level
+    const uint32_t *mask;        // table size - 1 per level
+    const uint4 *ent;            // 2 x uint4 per entry
+    const uint2 *nh;
+    const uint2 *pmac;
+    uint32_t n_nh, n_ports;
+};
+
+// ---------------------------------------------------------------- IPsec
+struct EspSa {                   // 256 B
+    uint32_t rk[44];             // AES-128 round keys, big-endian words (FIPS-197 w[i])
+    uint32_t spi, nonce;         // nonce as big-endian word
+    uint32_t ipad[5], opad[5];   // SHA-1 states after the HMAC ipad / opad blocks
+    uint32_t pad[2];
+};
+struct EspImg {
+    const EspSa *sa;
+    uint32_t n_sa;
+    const uint32_t *te;          // Te0..Te3 (4 x 256 words) + sbox (256 words)
+    const uint32_t *rss_nib;     // Toeplitz nibble table for the MS RSS key (72 x 16)
+};
+
+struct LbImg {
+    const uint16_t *port;
+    uint32_t n_backends;
+    const uint32_t *nib;         // Toeplitz nibble table of the LB key (72 x 16)
+};
+
+// ---------------------------------------------------------------- launch
+struct BatchDev { uint8_t *arena; const uint64_t *off; const uint16_t *len; uint32_t n; uint32_t start; uint64_t first; };
+
+enum { MASK_ACL = 1u << NFC_ACL, MASK_DPI = 1u << NFC_DPI, MASK_LPM4 = 1u << NFC_LPM4,
+       MASK_LPM6 = 1u << NFC_LPM6, MASK_IPSEC = 1u << NFC_IPSEC, MASK_LB = 1u << NFC_LB };
+
+// stats vector layout
+enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, ST_DPI_PAIRS,
+       ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS,
+       ST_POS_BASE = 16, ST_VAR_BASE = 64 };
+
+struct KParams {
+    uint32_t n_nf;
+    uint32_t kind[NFC_MAX_CHAIN];
+    uint32_t esp_pos;            // chain position of IPSEC or 0xFF
+    // work
+    const BatchDev *batches;
+    uint32_t n_batches;
+    uint32_t n_pkts;
+    uint32_t n_tiles;
+    uint32_t *tile_counter;
+    // outputs
+    nfc_pkt_result *rec;
+    uint32_t *match_pkt;
+    uint16_t *match_pat;
+    uint32_t match_cap;
+    uint32_t *match_count;
+    unsigned long long *stats;
+    uint32_t stats_len;
+    uint32_t st_acl, st_lb, st_sa;  // bases of the variable stats sections
+    uint32_t smem_stats;            // 1 = accumulate stats in shared memory
+    // ESP sequence look-back
+    uint32_t *tile_flag;            // n_tiles flags (epoch << 2 | status)
+    uint32_t *tile_vec;             // n_tiles x 2 x n_sa (aggregate, inclusive prefix)
+    uint32_t epoch;
+    const uint32_t *seq_in;
+    uint32_t *seq_out;
+    // tables
+    AclImg acl;
+    DpiImg dpi;
+    Lpm4Img l4;
+    Lpm6Img l6;
+    EspImg esp;
+    LbImg lb;
+};
+
+// host-side builders (builders.cpp); return "" on success or an error message
+struct HostImage { std::vector<uint8_t> bytes; };
+std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector<uint4> &r6);
+struct DpiHost {
+    std::vector<uint8_t> cls;
+    std::vector<uint8_t> trans;   // raw bytes (u16 or u32 entries)
+    uint32_t ncls = 0, n_states = 0, wide = 0;
+    std::vector<uint32_t> out_off;
+    std::vector<uint16_t> out_ids;
+    std::vector<uint8_t> action;
+};
+std::string build_dpi(const nfc_dpi_spec &s, DpiHost &out);
+std::string build_lpm4(const nfc_lpm4_spec &s, std::vector<uint16_t> &tbl24, std::vector<uint16_t> &tbllong,
+                       std::vector<uint2> &nh, std::vector<uint2> &pmac);
+struct Lpm6Host {
+    std::vector<uint8_t> lens;
+    std::vector<uint32_t> base, mask;
+    std::vector<Lpm6Entry> ent;
+    uint32_t def_nh = 0x7FFF;
+    std::vector<uint2> nh, pmac;
+};
+std::string build_lpm6(const nfc_lpm6_spec &s, Lpm6Host &out);
+std::string build_ipsec(const nfc_ipsec_spec &s, std::vector<EspSa> &sa);
+void build_aes_tables(std::vector<uint32_t> &te);           // Te0..3 + sbox
+void build_toeplitz_nibbles(const uint8_t key[40], std::vector<uint32_t> &nib);
+extern const uint8_t MS_RSS_KEY[40];
+
+// Waldvogel level hash (host and device use the same function)
+#ifdef __CUDACC__
+__host__ __device__
+#endif
+inline uint32_t l6_hash(uint32_t k0, uint32_t k1, uint32_t k2, uint32_t k3)
+{
+    uint32_t h = k0 * 0x9E3779B1u;
+    h = (h ^ (h >> 15) ^ k1) * 0x85EBCA77u;
+    h = (h ^ (h >> 13) ^ k2) * 0xC2B2AE3Du;
+    h = (h ^ (h >> 16) ^ k3) * 0x27D4EB2Fu;
+    return h ^ (h >> 15);
+}
+
+// kernel launch (sfc_kernel.cu)
+struct LaunchCfg { int grid, block; size_t smem; };
+int sfc_launch(uint32_t mask, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
+size_t sfc_smem_bytes(uint32_t mask, const KParams &p);
+int sfc_query(uint32_t mask, const KParams &p, int device, LaunchCfg *cfg_out);  // grid for full occupancy
+
+} // namespace nfc

@@ -1,0 +1,253 @@
+"""Thin ctypes binding of libnfc.so (include/nfc.h).
+
+Argument marshalling only: every step of the SFC hot path runs in the CUDA
+kernels behind the C ABI.  There is no CPU fallback: if libnfc.so is missing
+or fails to load, importing this module raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libnfc.so")
+
+NFC_OK, NFC_EINVAL, NFC_ENOMEM, NFC_ECUDA, NFC_ESTATE, NFC_ECAP, NFC_EUNSUP = 0, -1, -2, -3, -4, -5, -6
+ACL, DPI, LPM4, LPM6, IPSEC, LB = 1, 2, 3, 4, 5, 6
+KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB}
+STATS_RESET = 1
+
+# stats vector layout
+ST_PKTS, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP = 0, 1, 2, 3, 4, 5
+ST_DPI_PAIRS, ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS = 6, 7, 8, 9, 10, 11
+ST_POS_BASE, ST_VAR_BASE = 16, 64
+
+RESULT_DTYPE = np.dtype([("drop_nf", "u1"), ("esp_sa", "u1"), ("port", "<u2"), ("acl_rule", "<u2"),
+                         ("lb_backend", "<u2"), ("dpi_nmatch", "<u2"), ("out_len", "<u2"),
+                         ("esp_seq", "<u4")])
+
+_P = ctypes.c_void_p
+_u32 = ctypes.c_uint32
+
+
+class NfcError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"nfc error {code}: {msg}")
+        self.code = code
+
+
+class ChainOpts(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("flags", _u32), ("max_batch_pkts", _u32)]
+
+
+class AclSpec(ctypes.Structure):
+    _fields_ = [("n_rules", _u32), ("default_action", _u32), ("rules", _P)]
+
+
+class DpiSpec(ctypes.Structure):
+    _fields_ = [("n_patterns", _u32), ("blob", _P), ("off", _P), ("action", _P)]
+
+
+class LpmSpec(ctypes.Structure):
+    _fields_ = [("n_routes", _u32), ("routes", _P), ("n_nexthops", _u32), ("nexthops", _P),
+                ("n_ports", _u32), ("port_macs", _P)]
+
+
+class IpsecSpec(ctypes.Structure):
+    _fields_ = [("n_sa", _u32), ("sas", _P)]
+
+
+class LbSpec(ctypes.Structure):
+    _fields_ = [("n_backends", _u32), ("backend_port", _P), ("key", _P)]
+
+
+class Batch(ctypes.Structure):
+    _fields_ = [("arena", _P), ("off", _P), ("len", _P), ("n", _u32), ("reserved", _u32),
+                ("first_global_index", ctypes.c_uint64)]
+
+
+class Result(ctypes.Structure):
+    _fields_ = [("rec", _P), ("match_pkt", _P), ("match_pat", _P), ("match_cap", _u32),
+                ("reserved", _u32), ("match_count", _P)]
+
+
+EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
+           "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
+           "nfc_launch_count", "nfc_last_error", "nfc_version"]
+
+
+def _load_lib():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} not built: run __graft_entry__.build() "
+                          "(no CPU fallback exists for the SFC hot path)")
+    L = ctypes.CDLL(LIB_PATH)
+    L.nfc_build_chain.argtypes = [_P, _u32, ctypes.POINTER(ChainOpts), ctypes.POINTER(_P)]
+    L.nfc_destroy_chain.argtypes = [_P]
+    L.nfc_destroy_chain.restype = None
+    L.nfc_chain_room.argtypes = [_P, ctypes.POINTER(_u32), ctypes.POINTER(_u32)]
+    L.nfc_load_tables.argtypes = [_P, _u32, _P, ctypes.c_size_t]
+    L.nfc_process_batch.argtypes = [_P, _P, _u32, ctypes.POINTER(Result), _P]
+    L.nfc_process_host.argtypes = [_P, _P, ctypes.c_uint64, _P, _P, _u32, ctypes.c_uint64, _P, _P, _P, _u32,
+                                   ctypes.POINTER(_u32), _P]
+    L.nfc_stats_len.argtypes = [_P, ctypes.POINTER(ctypes.c_size_t)]
+    L.nfc_collect_stats.argtypes = [_P, _P, ctypes.c_size_t, _u32]
+    L.nfc_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64)]
+    L.nfc_last_error.restype = ctypes.c_char_p
+    L.nfc_version.restype = ctypes.c_char_p
+    return L
+
+
+lib = _load_lib()
+
+
+def _check(rc: int, allow=()):
+    if rc != NFC_OK and rc not in allow:
+        raise NfcError(rc, lib.nfc_last_error().decode())
+    return rc
+
+
+def _np(a, dtype=None):
+    a = np.ascontiguousarray(a if dtype is None else np.asarray(a, dtype=dtype))
+    return a
+
+
+class Chain:
+    """A service function chain bound to one CUDA device (original SFC order)."""
+
+    def __init__(self, kinds: Sequence, device: int = 0, max_batch_pkts: int = 0):
+        ks = [KINDS[k] if isinstance(k, str) else int(k) for k in kinds]
+        arr = (_u32 * len(ks))(*ks)
+        h = _P()
+        opts = ChainOpts(device, 0, max_batch_pkts)
+        _check(lib.nfc_build_chain(arr, len(ks), ctypes.byref(opts), ctypes.byref(h)))
+        self.h = h
+        self.kinds = ks
+        self.device = device
+        self._keep = []
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.nfc_destroy_chain(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def room(self):
+        hr, tr = _u32(), _u32()
+        _check(lib.nfc_chain_room(self.h, ctypes.byref(hr), ctypes.byref(tr)))
+        return hr.value, tr.value
+
+    # ------------------------------------------------------------ tables
+    def _load(self, kind: int, spec):
+        return _check(lib.nfc_load_tables(self.h, kind, ctypes.byref(spec), ctypes.sizeof(spec)))
+
+    def load_acl(self, rules: np.ndarray, default_action: int = 0):
+        r = _np(rules)
+        return self._load(ACL, AclSpec(len(r), default_action, r.ctypes.data if len(r) else None))
+
+    def load_dpi(self, blob: np.ndarray, off: np.ndarray, action: np.ndarray):
+        b, o, a = _np(blob, np.uint8), _np(off, np.uint32), _np(action, np.uint8)
+        return self._load(DPI, DpiSpec(len(a), b.ctypes.data, o.ctypes.data, a.ctypes.data))
+
+    def load_lpm(self, kind: int, routes: np.ndarray, nexthops: np.ndarray, port_macs: np.ndarray):
+        r, n, p = _np(routes), _np(nexthops), _np(port_macs, np.uint8)
+        return self._load(kind, LpmSpec(len(r), r.ctypes.data if len(r) else None, len(n), n.ctypes.data,
+                                        len(p), p.ctypes.data))
+
+    def load_ipsec(self, sas: np.ndarray):
+        s = _np(sas)
+        return self._load(IPSEC, IpsecSpec(len(s), s.ctypes.data))
+
+    def load_lb(self, ports: np.ndarray, key: np.ndarray):
+        p, k = _np(ports, np.uint16), _np(key, np.uint8)
+        return self._load(LB, LbSpec(len(p), p.ctypes.data, k.ctypes.data))
+
+    def load_tables(self, t):
+        """Load every NF of the chain from an object with the nfcgen.Tables fields."""
+        for k in self.kinds:
+            if k == ACL:
+                self.load_acl(t.acl_rules, t.acl_default)
+            elif k == DPI:
+                self.load_dpi(t.pat_blob, t.pat_off, t.pat_action)
+            elif k == LPM4:
+                self.load_lpm(LPM4, t.routes4, t.nh4, t.pmac4)
+            elif k == LPM6:
+                self.load_lpm(LPM6, t.routes6, t.nh6, t.pmac6)
+            elif k == IPSEC:
+                self.load_ipsec(t.sas)
+            elif k == LB:
+                self.load_lb(t.lb_ports, t.lb_key)
+
+    # ------------------------------------------------------------ processing
+    def process(self, batches, rec_ptr: int, match_pkt_ptr: int = 0, match_pat_ptr: int = 0,
+                match_cap: int = 0, match_count_ptr: int = 0, stream: int = 0):
+        """batches: list of (arena_ptr, off_ptr, len_ptr, n, first_global_index) device pointers."""
+        arr = (Batch * max(1, len(batches)))()
+        for i, (a, o, l, n, fgi) in enumerate(batches):
+            arr[i] = Batch(a, o, l, n, 0, fgi)
+        res = Result(rec_ptr, match_pkt_ptr or None, match_pat_ptr or None, match_cap, 0,
+                     match_count_ptr or None)
+        return _check(lib.nfc_process_batch(self.h, arr, len(batches), ctypes.byref(res), stream or None))
+
+    def process_tensors(self, arena, off, ln, rec, match_pkt=None, match_pat=None, match_count=None,
+                        first_global_index: int = 0, n: Optional[int] = None, stream=None):
+        """torch CUDA tensors (arena u8, off int64/uint64, len int16/uint16, rec u8[n,16])."""
+        import torch
+        n = int(off.numel()) if n is None else n
+        s = stream if stream is not None else torch.cuda.current_stream(arena.device)
+        return self.process([(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), n, first_global_index)],
+                            rec.data_ptr(),
+                            match_pkt.data_ptr() if match_pkt is not None else 0,
+                            match_pat.data_ptr() if match_pat is not None else 0,
+                            int(match_pkt.numel()) if match_pkt is not None else 0,
+                            match_count.data_ptr() if match_count is not None else 0,
+                            s.cuda_stream)
+
+    def process_host(self, arena: np.ndarray, off: np.ndarray, ln: np.ndarray, first_global_index: int = 0,
+                     match_cap: int = 1 << 20, stream: int = 0):
+        """End-to-end call with host buffers (arena rewritten in place). Returns (rec, (pkt, pat), n_pairs)."""
+        off = _np(off, np.uint64)
+        ln = _np(ln, np.uint16)
+        n = len(off)
+        rec = np.zeros(n, dtype=RESULT_DTYPE)
+        mp = np.zeros(max(1, match_cap), dtype=np.uint32)
+        mq = np.zeros(max(1, match_cap), dtype=np.uint16)
+        npairs = _u32()
+        assert arena.flags["C_CONTIGUOUS"] and arena.dtype == np.uint8
+        _check(lib.nfc_process_host(self.h, arena.ctypes.data, arena.nbytes, off.ctypes.data, ln.ctypes.data, n,
+                                    first_global_index, rec.ctypes.data, mp.ctypes.data, mq.ctypes.data,
+                                    match_cap, ctypes.byref(npairs), stream or None))
+        k = min(npairs.value, match_cap)
+        return rec, (mp[:k], mq[:k]), npairs.value
+
+    def process_host_ptr(self, arena_ptr: int, arena_bytes: int, off_ptr: int, len_ptr: int, n: int,
+                         rec_ptr: int, mp_ptr: int, mq_ptr: int, match_cap: int, first_global_index: int = 0,
+                         stream: int = 0) -> int:
+        npairs = _u32()
+        _check(lib.nfc_process_host(self.h, arena_ptr, arena_bytes, off_ptr, len_ptr, n, first_global_index,
+                                    rec_ptr, mp_ptr, mq_ptr, match_cap, ctypes.byref(npairs), stream or None))
+        return npairs.value
+
+    def stats(self, reset: bool = False, allow_cap: bool = True) -> np.ndarray:
+        n = ctypes.c_size_t()
+        _check(lib.nfc_stats_len(self.h, ctypes.byref(n)))
+        out = np.zeros(n.value, dtype=np.uint64)
+        _check(lib.nfc_collect_stats(self.h, out.ctypes.data, n.value, STATS_RESET if reset else 0),
+               allow=(NFC_ECAP,) if allow_cap else ())
+        return out
+
+    def launches(self) -> int:
+        c = ctypes.c_uint64()
+        _check(lib.nfc_launch_count(self.h, ctypes.byref(c)))
+        return c.value
+
+
+def version() -> str:
+    return lib.nfc_version().decode()

@@ -1,0 +1,78 @@
+"""CPU tests of the C-ABI boundary: the library loads, exports every symbol
+include/nfc.h declares, the ctypes layouts match the header's sizes, and the
+argument-validation paths that run before any CUDA call return the documented
+status codes."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def nfc():
+    import __graft_entry__
+    from paper_conf_hpca_hul18_b200 import build
+    build.build()
+    from paper_conf_hpca_hul18_b200 import nfc as m
+    return m
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "nfc.h")).read()
+    return sorted(set(re.findall(r"NFC_API\s+[\w\s\*]*?\b(nfc_\w+)\s*\(", src)))
+
+
+def test_header_declares_the_boundary():
+    names = _declared()
+    for must in ("nfc_build_chain", "nfc_load_tables", "nfc_process_batch", "nfc_collect_stats"):
+        assert must in names
+
+
+def test_library_exports_every_declared_symbol(nfc):
+    lib = ctypes.CDLL(nfc.LIB_PATH)
+    for name in _declared():
+        assert hasattr(lib, name), name
+    assert set(_declared()) == set(nfc.EXPORTS)
+
+
+def test_ctypes_layouts_match_header(nfc):
+    import nfcgen
+    assert ctypes.sizeof(nfc.Batch) == 40
+    assert ctypes.sizeof(nfc.Result) == 40
+    assert nfc.RESULT_DTYPE.itemsize == 16
+    assert nfcgen.ACL_RULE.itemsize == 48 and nfcgen.SA.itemsize == 48
+    assert nfcgen.ROUTE4.itemsize == 8 and nfcgen.ROUTE6.itemsize == 20 and nfcgen.NEXTHOP.itemsize == 8
+
+
+def test_validation_before_cuda(nfc):
+    lib = nfc.lib
+    h = ctypes.c_void_p()
+    opts = nfc.ChainOpts(0, 0, 0)
+    empty = (ctypes.c_uint32 * 1)(1)
+    assert lib.nfc_build_chain(empty, 0, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
+    seven = (ctypes.c_uint32 * 7)(1, 2, 3, 4, 5, 6, 1)
+    assert lib.nfc_build_chain(seven, 7, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
+    rep = (ctypes.c_uint32 * 2)(1, 1)
+    assert lib.nfc_build_chain(rep, 2, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
+    bad = (ctypes.c_uint32 * 1)(9)
+    assert lib.nfc_build_chain(bad, 1, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EINVAL
+    assert lib.nfc_build_chain(None, 1, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EINVAL
+    assert b"repeated" in lib.nfc_last_error() or len(lib.nfc_last_error()) > 0
+    assert lib.nfc_load_tables(None, 1, None, 0) == nfc.NFC_EINVAL
+    assert lib.nfc_collect_stats(None, None, 0, 0) == nfc.NFC_EINVAL
+    assert nfc.version().startswith("nfc-b200")
+
+
+def test_no_oracle_in_product():
+    # the product path never imports, includes or links the oracle
+    pkg = os.path.join(ROOT, "paper_conf_hpca_hul18_b200")
+    bad = re.compile(r"(import\s+oracle|from\s+oracle|#include\s+\S*oracle|liboracle|oracle\.h)")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
+                txt = open(os.path.join(dp, f)).read()
+                assert not bad.search(txt), f
