@@ -1,0 +1,46 @@
+/*
+ * nfc_debug.h -- host-side emulation of the device table images (diagnostics).
+ *
+ * Each handle holds the device image that nfc_load_tables would upload, built
+ * by the same host builders, and walks it on the CPU with the same algorithm
+ * the fused kernel uses.  This lets the table builders (Aho-Corasick DFA,
+ * DIR-24-8, IPv6 binary search on prefix lengths, ACL image, AES T-tables,
+ * Toeplitz nibble tables) be checked on a machine without a GPU.  Not part of
+ * the packet path.  Status codes as in nfc.h.
+ */
+#ifndef NFC_DEBUG_H
+#define NFC_DEBUG_H
+#include "nfc.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct nfc_dbg nfc_dbg;
+
+/* Build the image of `kind` from its logical spec (same validation as nfc_load_tables). */
+NFC_API int nfc_dbg_build(uint32_t kind, const void *spec, size_t spec_bytes, nfc_dbg **out);
+NFC_API void nfc_dbg_destroy(nfc_dbg *d);
+
+/* DPI: distinct matched pattern ids of buf (ascending, up to cap), count, any-DROP flag. */
+NFC_API int nfc_dbg_dpi(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids, uint32_t cap,
+                        uint32_t *count, uint32_t *drop);
+/* DPI image shape: states, byte classes, 1 if 32-bit entries. */
+NFC_API int nfc_dbg_dpi_shape(nfc_dbg *d, uint32_t *n_states, uint32_t *n_classes, uint32_t *wide);
+/* LPM4: next-hop index (0x7FFF = miss) and number of table reads (1 or 2). */
+NFC_API int nfc_dbg_lpm4(nfc_dbg *d, uint32_t dst, uint32_t *nh, uint32_t *reads);
+/* LPM6: next-hop index (0x7FFF = miss), hash-level probes and hash-slot reads. */
+NFC_API int nfc_dbg_lpm6(nfc_dbg *d, const uint8_t dst[16], uint32_t *nh, uint32_t *probes, uint32_t *slot_reads);
+NFC_API int nfc_dbg_lpm6_levels(nfc_dbg *d, uint32_t *n_levels);
+/* ACL: first matching rule (0xFFFF none) and the resulting action (0 permit / 1 deny). */
+NFC_API int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *dst, uint16_t sport,
+                        uint16_t dport, uint8_t proto, uint32_t *rule, uint32_t *action);
+/* Crypto / hash primitives as the kernel computes them (T-tables, nibble tables, ipad/opad states). */
+NFC_API int nfc_dbg_aes128_block(const uint8_t key[16], const uint8_t in[16], uint8_t out[16]);
+NFC_API int nfc_dbg_toeplitz(const uint8_t key[40], const uint8_t *in, size_t n, uint32_t *h);
+NFC_API int nfc_dbg_hmac_sha1(const uint8_t key[20], const uint8_t *msg, size_t n, uint8_t out[20]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libnfc.so")
 ROOT = os.path.dirname(HERE)
-SOURCES = ["capi.cu", "sfc_kernel.cu", "builders.cpp"]
+SOURCES = ["capi.cu", "sfc_kernel.cu", "builders.cpp", "debug_host.cpp"]
 HEADERS = ["nfc_internal.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -19,7 +19,7 @@ def _stale() -> bool:
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)
-    deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS] + [os.path.join(ROOT, "include", "nfc.h")]
+    deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS] + [os.path.join(ROOT, "include", f) for f in ("nfc.h", "nfc_debug.h")]
     return any(os.path.getmtime(d) > t for d in deps)
 
 

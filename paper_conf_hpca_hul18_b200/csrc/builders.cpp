@@ -64,8 +64,8 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector
 
 // ---------------------------------------------------------------- DPI
 // Aho-Corasick (1975) goto/failure construction, converted to a full DFA over
-// byte classes (bytes that occur in no pattern form class 0: from every state
-// they lead to the root).
+// byte classes (bytes that occur in no pattern share one class: from every
+// state they lead to the root).
 std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
 {
     if (s.n_patterns == 0 || s.n_patterns > 65535) return "dpi: n_patterns must be 1..65535";
@@ -78,8 +78,16 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
         if (s.action[j] > 1) return "dpi: action must be 0 or 1";
         for (uint32_t k = s.off[j]; k < s.off[j + 1]; k++) cls[s.blob[k]] = 1;
     }
-    int ncls = 1;
-    for (int b = 0; b < 256; b++) cls[b] = cls[b] ? ncls++ : 0;
+    // used bytes get classes 0..u-1; all unused bytes share class u (if any) -> ncls <= 256
+    int ncls = 0;
+    for (int b = 0; b < 256; b++) if (cls[b]) cls[b] = ++ncls;   // 1-based for now
+    const int other = ncls;
+    bool any_unused = false;
+    for (int b = 0; b < 256; b++) {
+        if (cls[b]) cls[b] -= 1;
+        else { cls[b] = other; any_unused = true; }
+    }
+    if (any_unused) ncls++;
     // trie with sparse children
     std::vector<std::vector<std::pair<int, int>>> kids(1);   // (class, child)
     std::vector<std::vector<uint16_t>> own(1);
@@ -360,7 +368,7 @@ void build_aes_tables(std::vector<uint32_t> &te)
     }
 }
 
-static void aes_expand(const uint8_t key[16], uint32_t rk[44])
+void aes_expand(const uint8_t key[16], uint32_t rk[44])
 {
     uint8_t sb[256];
     sbox_tables(sb);
@@ -379,7 +387,7 @@ static void aes_expand(const uint8_t key[16], uint32_t rk[44])
 }
 
 static inline uint32_t rol(uint32_t x, int n) { return (x << n) | (x >> (32 - n)); }
-static void sha1_compress(uint32_t h[5], const uint8_t blk[64])
+void sha1_compress(uint32_t h[5], const uint8_t blk[64])
 {
     uint32_t w[80];
     for (int t = 0; t < 16; t++) w[t] = be32(blk + 4 * t);

@@ -310,6 +310,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     p.n_nf = c->n_nf;
     for (uint32_t i = 0; i < c->n_nf; i++) p.kind[i] = c->kind[i];
     p.esp_pos = c->esp_pos;
+    p.present = c->mask;
     p.batches = c->batches.as<BatchDev>();
     p.n_batches = nb;
     p.n_pkts = (uint32_t)total;

@@ -1,0 +1,260 @@
+// debug_host.cpp -- include/nfc_debug.h: the device table images walked on the
+// host with the kernel's algorithms, so the builders can be checked without a
+// GPU.  Diagnostics only; not on the packet path.
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/nfc_debug.h"
+#include "nfc_internal.h"
+
+using namespace nfc;
+
+struct nfc_dbg {
+    uint32_t kind = 0;
+    std::vector<uint4> r4, r6;
+    uint32_t n_rules = 0, default_action = 0;
+    DpiHost dpi;
+    std::vector<uint16_t> tbl24, tbllong;
+    std::vector<uint2> nh, pmac;
+    Lpm6Host l6;
+};
+
+static inline uint32_t be32(const uint8_t *p) { return (uint32_t)p[0] << 24 | (uint32_t)p[1] << 16 | (uint32_t)p[2] << 8 | p[3]; }
+static inline uint32_t m32(int len) { return len <= 0 ? 0u : len >= 32 ? 0xFFFFFFFFu : 0xFFFFFFFFu << (32 - len); }
+
+extern "C" {
+
+int nfc_dbg_build(uint32_t kind, const void *spec, size_t spec_bytes, nfc_dbg **out)
+{
+    if (!spec || !out) return NFC_EINVAL;
+    nfc_dbg *d = new (std::nothrow) nfc_dbg();
+    if (!d) return NFC_ENOMEM;
+    d->kind = kind;
+    std::string err = "bad kind";
+    switch (kind) {
+    case NFC_ACL:
+        if (spec_bytes != sizeof(nfc_acl_spec)) break;
+        err = build_acl(*static_cast<const nfc_acl_spec *>(spec), d->r4, d->r6);
+        d->n_rules = static_cast<const nfc_acl_spec *>(spec)->n_rules;
+        d->default_action = static_cast<const nfc_acl_spec *>(spec)->default_action;
+        break;
+    case NFC_DPI:
+        if (spec_bytes != sizeof(nfc_dpi_spec)) break;
+        err = build_dpi(*static_cast<const nfc_dpi_spec *>(spec), d->dpi);
+        break;
+    case NFC_LPM4:
+        if (spec_bytes != sizeof(nfc_lpm4_spec)) break;
+        err = build_lpm4(*static_cast<const nfc_lpm4_spec *>(spec), d->tbl24, d->tbllong, d->nh, d->pmac);
+        break;
+    case NFC_LPM6:
+        if (spec_bytes != sizeof(nfc_lpm6_spec)) break;
+        err = build_lpm6(*static_cast<const nfc_lpm6_spec *>(spec), d->l6);
+        break;
+    }
+    if (!err.empty()) {
+        delete d;
+        return NFC_EINVAL;
+    }
+    *out = d;
+    return NFC_OK;
+}
+
+void nfc_dbg_destroy(nfc_dbg *d) { delete d; }
+
+int nfc_dbg_dpi_shape(nfc_dbg *d, uint32_t *n_states, uint32_t *n_classes, uint32_t *wide)
+{
+    if (!d || d->kind != NFC_DPI) return NFC_EINVAL;
+    *n_states = d->dpi.n_states;
+    *n_classes = d->dpi.ncls;
+    *wide = d->dpi.wide;
+    return NFC_OK;
+}
+
+int nfc_dbg_dpi(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids, uint32_t cap, uint32_t *count,
+                uint32_t *drop)
+{
+    if (!d || d->kind != NFC_DPI) return NFC_EINVAL;
+    const DpiHost &D = d->dpi;
+    std::vector<uint8_t> seen(D.action.size(), 0);
+    std::vector<uint16_t> got;
+    uint32_t s = 0, dr = 0;
+    for (size_t i = 0; i < n; i++) {
+        uint32_t c = D.cls[buf[i]], e;
+        bool acc;
+        if (D.wide) { uint32_t x; memcpy(&x, &D.trans[((size_t)s * D.ncls + c) * 4], 4); acc = x >> 31; e = x & 0x7FFFFFFFu; }
+        else { uint16_t x; memcpy(&x, &D.trans[((size_t)s * D.ncls + c) * 2], 2); acc = x >> 15; e = x & 0x7FFFu; }
+        s = e;
+        if (acc)
+            for (uint32_t k = D.out_off[s]; k < D.out_off[s + 1]; k++) {
+                uint16_t id = D.out_ids[k];
+                dr |= D.action[id];
+                if (!seen[id]) { seen[id] = 1; got.push_back(id); }
+            }
+    }
+    std::sort(got.begin(), got.end());
+    for (uint32_t k = 0; k < got.size() && k < cap; k++) ids[k] = got[k];
+    *count = (uint32_t)got.size();
+    *drop = dr;
+    return NFC_OK;
+}
+
+int nfc_dbg_lpm4(nfc_dbg *d, uint32_t dst, uint32_t *nh, uint32_t *reads)
+{
+    if (!d || d->kind != NFC_LPM4) return NFC_EINVAL;
+    uint32_t e = d->tbl24[dst >> 8], r = 1;
+    if (e & 0x8000) { e = d->tbllong[((e & 0x7FFF) << 8) + (dst & 0xFF)]; r = 2; }
+    *nh = e;
+    *reads = r;
+    return NFC_OK;
+}
+
+int nfc_dbg_lpm6_levels(nfc_dbg *d, uint32_t *n_levels)
+{
+    if (!d || d->kind != NFC_LPM6) return NFC_EINVAL;
+    *n_levels = (uint32_t)d->l6.lens.size();
+    return NFC_OK;
+}
+
+int nfc_dbg_lpm6(nfc_dbg *d, const uint8_t dst[16], uint32_t *nh, uint32_t *probes, uint32_t *slot_reads)
+{
+    if (!d || d->kind != NFC_LPM6) return NFC_EINVAL;
+    const Lpm6Host &T = d->l6;
+    uint32_t w[4] = {be32(dst), be32(dst + 4), be32(dst + 8), be32(dst + 12)};
+    uint32_t best = T.def_nh, pr = 0, sr = 0;
+    int lo = 0, hi = (int)T.lens.size() - 1;
+    while (lo <= hi) {
+        int mid = (lo + hi) >> 1, L = T.lens[mid];
+        uint32_t k[4] = {w[0] & m32(L), w[1] & m32(L - 32), w[2] & m32(L - 64), w[3] & m32(L - 96)};
+        uint32_t m = T.mask[mid], h = l6_hash(k[0], k[1], k[2], k[3]) & m;
+        pr++;
+        bool found = false;
+        uint32_t info = 0;
+        for (;;) {
+            const Lpm6Entry &e = T.ent[T.base[mid] + h];
+            sr++;
+            if (!(e.info & L6_VALID)) break;
+            if (!memcmp(e.key, k, 16)) { found = true; info = e.info; break; }
+            h = (h + 1) & m;
+        }
+        if (found) {
+            if ((info & 0xFFFF) != 0x7FFF) best = info & 0xFFFF;
+            lo = mid + 1;
+        } else {
+            hi = mid - 1;
+        }
+    }
+    *nh = best;
+    *probes = pr;
+    *slot_reads = sr;
+    return NFC_OK;
+}
+
+int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *dst, uint16_t sport,
+                uint16_t dport, uint8_t proto, uint32_t *rule, uint32_t *action)
+{
+    if (!d || d->kind != NFC_ACL) return NFC_EINVAL;
+    auto tail_ok = [&](const uint4 &t) {
+        if (sport < (t.x & 0xFFFF) || sport > (t.x >> 16)) return false;
+        if (dport < (t.y & 0xFFFF) || dport > (t.y >> 16)) return false;
+        if (!((t.z >> 8) & 1) && (t.z & 0xFF) != proto) return false;
+        return true;
+    };
+    *rule = 0xFFFF;
+    *action = d->default_action;
+    if (family == 4) {
+        uint32_t s = be32(src), t = be32(dst);
+        for (size_t i = 0; i + 1 < d->r4.size(); i += 2) {
+            const uint4 &r = d->r4[i];
+            if ((s & r.y) != r.x || (t & r.w) != r.z || !tail_ok(d->r4[i + 1])) continue;
+            *rule = d->r4[i + 1].w;
+            *action = (d->r4[i + 1].z >> 16) & 1;
+            return NFC_OK;
+        }
+    } else {
+        uint32_t s[4], t[4];
+        for (int k = 0; k < 4; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
+        for (size_t i = 0; i + 4 < d->r6.size(); i += 5) {
+            const uint4 *r = &d->r6[i];
+            const uint32_t sv[4] = {r[0].x, r[0].y, r[0].z, r[0].w}, sm[4] = {r[1].x, r[1].y, r[1].z, r[1].w};
+            const uint32_t dv[4] = {r[2].x, r[2].y, r[2].z, r[2].w}, dm[4] = {r[3].x, r[3].y, r[3].z, r[3].w};
+            bool ok = true;
+            for (int k = 0; k < 4; k++) ok &= (s[k] & sm[k]) == sv[k] && (t[k] & dm[k]) == dv[k];
+            if (!ok || !tail_ok(r[4])) continue;
+            *rule = r[4].w;
+            *action = (r[4].z >> 16) & 1;
+            return NFC_OK;
+        }
+    }
+    return NFC_OK;
+}
+
+int nfc_dbg_aes128_block(const uint8_t key[16], const uint8_t in[16], uint8_t out[16])
+{
+    std::vector<uint32_t> te;
+    build_aes_tables(te);
+    uint32_t rk[44];
+    aes_expand(key, rk);
+    const uint32_t *T0 = &te[0], *T1 = &te[256], *T2 = &te[512], *T3 = &te[768], *S = &te[1024];
+    uint32_t s0 = be32(in) ^ rk[0], s1 = be32(in + 4) ^ rk[1], s2 = be32(in + 8) ^ rk[2], s3 = be32(in + 12) ^ rk[3];
+    for (int r = 1; r < 10; r++) {
+        uint32_t t0 = T0[s0 >> 24] ^ T1[(s1 >> 16) & 255] ^ T2[(s2 >> 8) & 255] ^ T3[s3 & 255] ^ rk[4 * r];
+        uint32_t t1 = T0[s1 >> 24] ^ T1[(s2 >> 16) & 255] ^ T2[(s3 >> 8) & 255] ^ T3[s0 & 255] ^ rk[4 * r + 1];
+        uint32_t t2 = T0[s2 >> 24] ^ T1[(s3 >> 16) & 255] ^ T2[(s0 >> 8) & 255] ^ T3[s1 & 255] ^ rk[4 * r + 2];
+        uint32_t t3 = T0[s3 >> 24] ^ T1[(s0 >> 16) & 255] ^ T2[(s1 >> 8) & 255] ^ T3[s2 & 255] ^ rk[4 * r + 3];
+        s0 = t0; s1 = t1; s2 = t2; s3 = t3;
+    }
+    uint32_t o[4];
+    o[0] = (S[s0 >> 24] << 24 | S[(s1 >> 16) & 255] << 16 | S[(s2 >> 8) & 255] << 8 | S[s3 & 255]) ^ rk[40];
+    o[1] = (S[s1 >> 24] << 24 | S[(s2 >> 16) & 255] << 16 | S[(s3 >> 8) & 255] << 8 | S[s0 & 255]) ^ rk[41];
+    o[2] = (S[s2 >> 24] << 24 | S[(s3 >> 16) & 255] << 16 | S[(s0 >> 8) & 255] << 8 | S[s1 & 255]) ^ rk[42];
+    o[3] = (S[s3 >> 24] << 24 | S[(s0 >> 16) & 255] << 16 | S[(s1 >> 8) & 255] << 8 | S[s2 & 255]) ^ rk[43];
+    for (int i = 0; i < 4; i++) {
+        out[4 * i] = (uint8_t)(o[i] >> 24); out[4 * i + 1] = (uint8_t)(o[i] >> 16);
+        out[4 * i + 2] = (uint8_t)(o[i] >> 8); out[4 * i + 3] = (uint8_t)o[i];
+    }
+    return NFC_OK;
+}
+
+int nfc_dbg_toeplitz(const uint8_t key[40], const uint8_t *in, size_t n, uint32_t *h)
+{
+    if (n > 36) return NFC_EINVAL;
+    std::vector<uint32_t> nib;
+    build_toeplitz_nibbles(key, nib);
+    uint32_t x = 0;
+    for (size_t i = 0; i < n; i++) x ^= nib[(2 * i) * 16 + (in[i] >> 4)] ^ nib[(2 * i + 1) * 16 + (in[i] & 15)];
+    *h = x;
+    return NFC_OK;
+}
+
+int nfc_dbg_hmac_sha1(const uint8_t key[20], const uint8_t *msg, size_t n, uint8_t out[20])
+{
+    nfc_sa sa{};
+    memcpy(sa.auth_key, key, 20);
+    nfc_ipsec_spec spec{1, &sa};
+    std::vector<EspSa> v;
+    if (!build_ipsec(spec, v).empty()) return NFC_EINVAL;
+    // inner: ipad state, then msg with padding counting the 64-B ipad block
+    uint32_t h[5];
+    memcpy(h, v[0].ipad, 20);
+    std::vector<uint8_t> m(msg, msg + n);
+    m.push_back(0x80);
+    while ((m.size() % 64) != 56) m.push_back(0);
+    uint64_t bits = (uint64_t)(64 + n) * 8;
+    for (int i = 7; i >= 0; i--) m.push_back((uint8_t)(bits >> (8 * i)));
+    for (size_t b = 0; b < m.size(); b += 64) sha1_compress(h, &m[b]);
+    uint8_t blk[64] = {0};
+    for (int i = 0; i < 5; i++) { blk[4 * i] = (uint8_t)(h[i] >> 24); blk[4 * i + 1] = (uint8_t)(h[i] >> 16); blk[4 * i + 2] = (uint8_t)(h[i] >> 8); blk[4 * i + 3] = (uint8_t)h[i]; }
+    blk[20] = 0x80;
+    uint64_t ob = (64 + 20) * 8;
+    for (int i = 0; i < 8; i++) blk[63 - i] = (uint8_t)(ob >> (8 * i));
+    uint32_t g[5];
+    memcpy(g, v[0].opad, 20);
+    sha1_compress(g, blk);
+    for (int i = 0; i < 5; i++) { out[4 * i] = (uint8_t)(g[i] >> 24); out[4 * i + 1] = (uint8_t)(g[i] >> 16); out[4 * i + 2] = (uint8_t)(g[i] >> 8); out[4 * i + 3] = (uint8_t)g[i]; }
+    return NFC_OK;
+}
+
+} // extern "C"

@@ -77,8 +77,9 @@ struct EspSa {                   // 256 B
     uint32_t rk[44];             // AES-128 round keys, big-endian words (FIPS-197 w[i])
     uint32_t spi, nonce;         // nonce as big-endian word
     uint32_t ipad[5], opad[5];   // SHA-1 states after the HMAC ipad / opad blocks
-    uint32_t pad[2];
+    uint32_t pad[8];
 };
+static_assert(sizeof(EspSa) == 256, "EspSa must stay 16-B aligned in arrays");
 struct EspImg {
     const EspSa *sa;
     uint32_t n_sa;
@@ -107,6 +108,7 @@ struct KParams {
     uint32_t n_nf;
     uint32_t kind[NFC_MAX_CHAIN];
     uint32_t esp_pos;            // chain position of IPSEC or 0xFF
+    uint32_t present;            // MASK_* bits of the NFs in the chain
     // work
     const BatchDev *batches;
     uint32_t n_batches;
@@ -164,6 +166,8 @@ std::string build_ipsec(const nfc_ipsec_spec &s, std::vector<EspSa> &sa);
 void build_aes_tables(std::vector<uint32_t> &te);           // Te0..3 + sbox
 void build_toeplitz_nibbles(const uint8_t key[40], std::vector<uint32_t> &nib);
 extern const uint8_t MS_RSS_KEY[40];
+void aes_expand(const uint8_t key[16], uint32_t rk[44]);
+void sha1_compress(uint32_t h[5], const uint8_t blk[64]);
 
 // Waldvogel level hash (host and device use the same function)
 #ifdef __CUDACC__

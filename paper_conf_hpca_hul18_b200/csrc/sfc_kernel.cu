@@ -557,13 +557,15 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 1 : 2) sfc_kernel(
     uint32_t *ms_nib = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
     uint32_t *lb_nib = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
     uint8_t *cls = smem + L.cls;
-    if constexpr ((MASK & MASK_IPSEC) != 0) {
+    // NFs compiled into this variant but absent from the chain are skipped at run time
+    const bool has_esp = (MASK & MASK_IPSEC) && P.esp_pos < P.n_nf;
+    if ((MASK & MASK_IPSEC) && has_esp) {
         for (uint32_t i = tid; i < 5 * 256; i += TILE) te[i] = __ldg(P.esp.te + i);
         for (uint32_t i = tid; i < 72 * 16; i += TILE) ms_nib[i] = __ldg(P.esp.rss_nib + i);
     }
-    if constexpr ((MASK & MASK_LB) != 0)
+    if ((MASK & MASK_LB) && (P.present & MASK_LB))
         for (uint32_t i = tid; i < 72 * 16; i += TILE) lb_nib[i] = __ldg(P.lb.nib + i);
-    if constexpr ((MASK & MASK_DPI) != 0)
+    if ((MASK & MASK_DPI) && (P.present & MASK_DPI))
         for (uint32_t i = tid; i < 256; i += TILE) cls[i] = __ldg(P.dpi.cls + i);
     // variable stats live in smem or go straight to global memory
     auto stat_add = [&](uint32_t idx, unsigned long long v) {
@@ -681,10 +683,10 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 1 : 2) sfc_kernel(
             if (dropped) { drop = pos; alive = false; }
         };
 
-        const uint32_t n_pre = (MASK & MASK_IPSEC) ? P.esp_pos : P.n_nf;
+        const uint32_t n_pre = has_esp ? P.esp_pos : P.n_nf;
         for (uint32_t pos = 0; pos < n_pre && alive; pos++) run_nf(pos);
 
-        if constexpr ((MASK & MASK_IPSEC) != 0) {
+        if ((MASK & MASK_IPSEC) && has_esp) {   // uniform across the CTA
             // ---- ESP sequence numbers: per SA, global packet order (decoupled look-back)
             const uint32_t nsa = P.esp.n_sa;
             uint16_t *wcnt = reinterpret_cast<uint16_t *>(smem + L.wcnt);

@@ -77,6 +77,9 @@ class Result(ctypes.Structure):
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
            "nfc_launch_count", "nfc_last_error", "nfc_version"]
+DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_lpm4",
+                 "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
+                 "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
 
 
 def _load_lib():
@@ -97,6 +100,19 @@ def _load_lib():
     L.nfc_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64)]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
+    P32 = ctypes.POINTER(_u32)
+    L.nfc_dbg_build.argtypes = [_u32, _P, ctypes.c_size_t, ctypes.POINTER(_P)]
+    L.nfc_dbg_destroy.argtypes = [_P]
+    L.nfc_dbg_destroy.restype = None
+    L.nfc_dbg_dpi.argtypes = [_P, _P, ctypes.c_size_t, _P, _u32, P32, P32]
+    L.nfc_dbg_dpi_shape.argtypes = [_P, P32, P32, P32]
+    L.nfc_dbg_lpm4.argtypes = [_P, _u32, P32, P32]
+    L.nfc_dbg_lpm6.argtypes = [_P, _P, P32, P32, P32]
+    L.nfc_dbg_lpm6_levels.argtypes = [_P, P32]
+    L.nfc_dbg_acl.argtypes = [_P, _u32, _P, _P, ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint8, P32, P32]
+    L.nfc_dbg_aes128_block.argtypes = [_P, _P, _P]
+    L.nfc_dbg_toeplitz.argtypes = [_P, _P, ctypes.c_size_t, P32]
+    L.nfc_dbg_hmac_sha1.argtypes = [_P, _P, ctypes.c_size_t, _P]
     return L
 
 
@@ -247,6 +263,92 @@ class Chain:
         c = ctypes.c_uint64()
         _check(lib.nfc_launch_count(self.h, ctypes.byref(c)))
         return c.value
+
+
+def _cbuf(b: bytes):
+    return ctypes.create_string_buffer(bytes(b), max(1, len(b)))
+
+
+class HostImage:
+    """include/nfc_debug.h: a device table image built by the product's builders and
+    walked on the host with the kernel's algorithm (diagnostics, no GPU needed)."""
+
+    def __init__(self, kind, **tables):
+        self._keep = []
+        kind = KINDS[kind] if isinstance(kind, str) else kind
+        if kind == ACL:
+            r = _np(tables["rules"])
+            self._keep.append(r)
+            spec = AclSpec(len(r), tables.get("default_action", 0), r.ctypes.data)
+        elif kind == DPI:
+            b, o, a = _np(tables["blob"], np.uint8), _np(tables["off"], np.uint32), _np(tables["action"], np.uint8)
+            self._keep += [b, o, a]
+            spec = DpiSpec(len(a), b.ctypes.data, o.ctypes.data, a.ctypes.data)
+        elif kind in (LPM4, LPM6):
+            r, n, p = _np(tables["routes"]), _np(tables["nexthops"]), _np(tables["port_macs"], np.uint8)
+            self._keep += [r, n, p]
+            spec = LpmSpec(len(r), r.ctypes.data, len(n), n.ctypes.data, len(p), p.ctypes.data)
+        else:
+            raise ValueError(kind)
+        h = _P()
+        _check(lib.nfc_dbg_build(kind, ctypes.byref(spec), ctypes.sizeof(spec), ctypes.byref(h)))
+        self.h = h
+        self.kind = kind
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib.nfc_dbg_destroy(self.h)
+            self.h = None
+
+    def dpi(self, data: bytes, cap: int = 65536):
+        ids = np.zeros(cap, dtype=np.uint16)
+        c, d = _u32(), _u32()
+        _check(lib.nfc_dbg_dpi(self.h, _cbuf(data), len(data), ids.ctypes.data, cap, ctypes.byref(c), ctypes.byref(d)))
+        return [int(x) for x in ids[:min(c.value, cap)]], bool(d.value)
+
+    def dpi_shape(self):
+        a, b, c = _u32(), _u32(), _u32()
+        _check(lib.nfc_dbg_dpi_shape(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+        return a.value, b.value, c.value
+
+    def lpm4(self, dst: int):
+        nh, r = _u32(), _u32()
+        _check(lib.nfc_dbg_lpm4(self.h, dst, ctypes.byref(nh), ctypes.byref(r)))
+        return nh.value, r.value
+
+    def lpm6(self, dst: bytes):
+        nh, p, s = _u32(), _u32(), _u32()
+        _check(lib.nfc_dbg_lpm6(self.h, _cbuf(dst), ctypes.byref(nh), ctypes.byref(p), ctypes.byref(s)))
+        return nh.value, p.value, s.value
+
+    def lpm6_levels(self):
+        n = _u32()
+        _check(lib.nfc_dbg_lpm6_levels(self.h, ctypes.byref(n)))
+        return n.value
+
+    def acl(self, family, src: bytes, dst: bytes, sport, dport, proto):
+        r, a = _u32(), _u32()
+        _check(lib.nfc_dbg_acl(self.h, family, _cbuf(src), _cbuf(dst), sport, dport, proto,
+                               ctypes.byref(r), ctypes.byref(a)))
+        return r.value, a.value
+
+
+def dbg_aes128_block(key: bytes, block: bytes) -> bytes:
+    out = ctypes.create_string_buffer(16)
+    _check(lib.nfc_dbg_aes128_block(_cbuf(key), _cbuf(block), out))
+    return out.raw
+
+
+def dbg_toeplitz(key: bytes, data: bytes) -> int:
+    h = _u32()
+    _check(lib.nfc_dbg_toeplitz(_cbuf(key), _cbuf(data), len(data), ctypes.byref(h)))
+    return h.value
+
+
+def dbg_hmac_sha1(key20: bytes, msg: bytes) -> bytes:
+    out = ctypes.create_string_buffer(20)
+    _check(lib.nfc_dbg_hmac_sha1(_cbuf(key20), _cbuf(msg), len(msg), out))
+    return out.raw
 
 
 def version() -> str:

@@ -1,0 +1,201 @@
+"""CPU tests of the product's table builders (include/nfc_debug.h): each device
+image is walked on the host with the kernel's algorithm and compared with the
+oracle, plus the paper's structural claims (IPv4 lookup takes two
+memory accesses, IPv6 up to 7)."""
+import math
+import random
+
+import numpy as np
+import pytest
+
+import nfcgen
+import oracle
+from tests.conftest import golden_rows
+
+
+@pytest.fixture(scope="module")
+def nfc():
+    from paper_conf_hpca_hul18_b200 import build
+    build.build()
+    from paper_conf_hpca_hul18_b200 import nfc as m
+    return m
+
+
+def _pattern_tables(pats, acts=None):
+    t = nfcgen.Tables()
+    off = np.zeros(len(pats) + 1, dtype=np.uint32)
+    off[1:] = np.cumsum([len(p) for p in pats])
+    t.pat_blob = np.frombuffer(b"".join(pats), dtype=np.uint8).copy()
+    t.pat_off = off
+    t.pat_action = np.array(acts if acts is not None else [0] * len(pats), dtype=np.uint8)
+    return t
+
+
+@pytest.mark.parametrize("case", ["c1", "c4", "allbytes", "tiny"])
+def test_dfa_image_vs_oracle(nfc, case):
+    rng = random.Random(hash(case) & 0xFFFF)
+    if case == "c1":
+        t = nfcgen.workload("C1").tables
+    elif case == "c4":
+        t = nfcgen.workload("C4").tables
+    elif case == "allbytes":  # every byte value occurs in some pattern: 256 classes, no "other" class
+        pats = [bytes([b, (b * 7) & 255]) for b in range(256)] + [b"\x00\x01\x02"]
+        t = _pattern_tables(pats, [rng.random() < 0.1 for _ in pats])
+    else:
+        pats = [bytes(rng.choice(b"ab") for _ in range(rng.randrange(1, 5))) for _ in range(12)]
+        t = _pattern_tables(pats)
+    img = nfc.HostImage("DPI", blob=t.pat_blob, off=t.pat_off, action=t.pat_action)
+    ns, ncls, wide = img.dpi_shape()
+    assert ncls <= 256
+    orc = oracle.OracleChain(["DPI"], t)
+    pats = t.patterns()
+    for k in range(400):
+        n = rng.randrange(0, 200)
+        alpha = b"ab" if case == "tiny" else None
+        text = bytes(rng.choice(alpha) if alpha else rng.randrange(256) for _ in range(n))
+        for _ in range(rng.randrange(0, 4)):
+            p = rng.choice(pats)
+            i = rng.randrange(0, len(text) + 1)
+            text = text[:i] + p + text[i:]
+        ids, drop = img.dpi(text)
+        assert ids == orc.ac_match(text)
+        assert drop == any(t.pat_action[j] for j in ids)
+
+
+def test_dir24_8_vs_oracle_and_two_accesses(nfc):
+    w = nfcgen.workload("C1")
+    t = w.tables
+    # add /25../32 routes so TBLlong is exercised
+    rng = np.random.default_rng(5)
+    extra = nfcgen.gen_routes4(rng, 300, len(t.nh4), default_route=False)
+    extra = extra[extra["len"] > 24]
+    routes = np.concatenate([t.routes4, extra])
+    _, idx = np.unique(np.stack([routes["prefix"].astype(np.int64), routes["len"].astype(np.int64)], 1),
+                       axis=0, return_index=True)
+    routes = routes[np.sort(idx)]
+    t2 = nfcgen.Tables(routes4=routes, nh4=t.nh4, pmac4=t.pmac4)
+    img = nfc.HostImage("LPM4", routes=routes, nexthops=t.nh4, port_macs=t.pmac4)
+    orc = oracle.OracleChain(["LPM4"], t2)
+    r = random.Random(1)
+    reads_seen = set()
+    max_reads = int(golden_rows("paper_facts.txt")[1][1])
+    for k in range(20000):
+        if k % 2:
+            rt = routes[r.randrange(len(routes))]
+            L = int(rt["len"])
+            a = int(rt["prefix"]) | (r.getrandbits(32) & ((1 << (32 - L)) - 1))
+        else:
+            a = r.getrandbits(32)
+        nh, reads = img.lpm4(a)
+        want = orc.lpm4(a)
+        assert nh == (0x7FFF if want < 0 else want)
+        assert reads <= max_reads  # "two memory accesses"
+        reads_seen.add(reads)
+    assert reads_seen == {1, 2}
+
+
+def test_lpm6_waldvogel_vs_oracle_full_c4(nfc):
+    """200K IPv6 prefixes: binary search on prefix lengths, <= 7 hash-level probes."""
+    t = nfcgen.workload("C4").tables
+    img = nfc.HostImage("LPM6", routes=t.routes6, nexthops=t.nh6, port_macs=t.pmac6)
+    orc = oracle.OracleChain(["LPM6"], t)
+    levels = img.lpm6_levels()
+    bound = math.ceil(math.log2(levels + 1))
+    assert bound <= int(golden_rows("paper_facts.txt")[2][1])
+    r = random.Random(2)
+    worst = 0
+    for k in range(20000):
+        if k % 4:
+            rt = t.routes6[r.randrange(len(t.routes6))]
+            L = int(rt["len"])
+            a = int.from_bytes(bytes(rt["prefix"]), "big") | (r.getrandbits(128) & ((1 << (128 - L)) - 1))
+        else:
+            a = r.getrandbits(128)
+        dst = a.to_bytes(16, "big")
+        nh, probes, _ = img.lpm6(dst)
+        want = orc.lpm6(dst)
+        assert nh == (0x7FFF if want < 0 else want), k
+        worst = max(worst, probes)
+    assert worst <= bound
+
+
+def test_lpm6_adversarial_nesting(nfc):
+    """Nested prefixes at many lengths (markers with and without a best-matching prefix)."""
+    r = random.Random(9)
+    base = r.getrandbits(128)
+    routes = []
+    seen = set()
+    for L in [1, 3, 8, 16, 17, 31, 32, 33, 47, 48, 63, 64, 65, 96, 127, 128]:
+        for j in range(3):
+            v = base ^ (r.getrandbits(4) << (128 - L)) if j else base
+            v &= ((1 << L) - 1) << (128 - L)
+            if (v, L) in seen:
+                continue
+            seen.add((v, L))
+            routes.append((v, L))
+    rt = np.zeros(len(routes), dtype=nfcgen.ROUTE6)
+    for i, (v, L) in enumerate(routes):
+        rt[i]["prefix"] = np.frombuffer(v.to_bytes(16, "big"), dtype=np.uint8)
+        rt[i]["len"] = L
+        rt[i]["nh"] = i % 7
+    nh, pm = nfcgen.gen_nexthops(np.random.default_rng(1), 7, 2)
+    t = nfcgen.Tables(routes6=rt, nh6=nh, pmac6=pm)
+    img = nfc.HostImage("LPM6", routes=rt, nexthops=nh, port_macs=pm)
+    orc = oracle.OracleChain(["LPM6"], t)
+    for k in range(5000):
+        a = base ^ (r.getrandbits(128) >> r.randrange(0, 128))
+        dst = a.to_bytes(16, "big")
+        want = orc.lpm6(dst)
+        assert img.lpm6(dst)[0] == (0x7FFF if want < 0 else want)
+
+
+@pytest.mark.parametrize("fam", [4, 6])
+def test_acl_image_vs_oracle(nfc, fam):
+    rng = np.random.default_rng(40 + fam)
+    rules = np.concatenate([nfcgen.gen_acl(rng, 40, 4), nfcgen.gen_acl(rng, 40, 6)])
+    rng.shuffle(rules)
+    t = nfcgen.Tables(acl_rules=rules, acl_default=1)
+    img = nfc.HostImage("ACL", rules=rules, default_action=1)
+    orc = oracle.OracleChain(["ACL"], t)
+    r = random.Random(fam)
+    nb = 4 if fam == 4 else 16
+    fam_idx = [i for i in range(len(rules)) if rules[i]["family"] == fam]
+    for _ in range(3000):
+        src = bytearray(r.getrandbits(8) for _ in range(nb))
+        dst = bytearray(r.getrandbits(8) for _ in range(nb))
+        sp, dp, proto = r.getrandbits(16), r.getrandbits(16), r.choice([1, 6, 17])
+        if r.random() < 0.7:
+            ru = rules[r.choice(fam_idx)]
+            for arr, p, L in ((src, ru["src"], int(ru["slen"])), (dst, ru["dst"], int(ru["dlen"]))):
+                for k in range(nb):
+                    keep = L - 8 * k
+                    m = 0xFF if keep >= 8 else 0 if keep <= 0 else (0xFF << (8 - keep)) & 0xFF
+                    arr[k] = (int(p[k]) & m) | (arr[k] & ~m & 0xFF)
+            sp = r.randint(int(ru["sp_lo"]), int(ru["sp_hi"]))
+            dp = r.randint(int(ru["dp_lo"]), int(ru["dp_hi"]))
+            proto = int(ru["proto"]) if not ru["proto_any"] else proto
+        rule, act = img.acl(fam, bytes(src), bytes(dst), sp, dp, proto)
+        want = orc.acl(fam, bytes(src), bytes(dst), sp, dp, proto)
+        assert rule == (0xFFFF if want < 0 else want)
+        assert act == (1 if want < 0 else int(rules[want]["action"]))
+
+
+@pytest.mark.parametrize("row", golden_rows("fips197_aes128.txt"))
+def test_ttable_aes_fips197(nfc, row):
+    key, pt, ct = (bytes.fromhex(x) for x in row)
+    assert nfc.dbg_aes128_block(key, pt) == ct
+
+
+@pytest.mark.parametrize("row", golden_rows("ms_rss_toeplitz.txt"))
+def test_nibble_toeplitz_ms_rss(nfc, row):
+    import ipaddress
+    src, sp, dst, dp, h_ip, h_l4 = row
+    a = ipaddress.ip_address(src).packed + ipaddress.ip_address(dst).packed
+    assert nfc.dbg_toeplitz(oracle.MS_RSS_KEY, a) == int(h_ip, 16)
+    assert nfc.dbg_toeplitz(oracle.MS_RSS_KEY, a + int(sp).to_bytes(2, "big") + int(dp).to_bytes(2, "big")) == int(h_l4, 16)
+
+
+@pytest.mark.parametrize("row", [r for r in golden_rows("rfc2202_hmac_sha1.txt") if len(r[0]) <= 40])
+def test_ipad_opad_hmac_rfc2202(nfc, row):
+    key = bytes.fromhex(row[0]).ljust(20, b"\x00")  # HMAC zero-pads keys shorter than the block
+    assert nfc.dbg_hmac_sha1(key, bytes.fromhex(row[1])).hex() == row[2]

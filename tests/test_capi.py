@@ -21,8 +21,8 @@ def nfc():
     return m
 
 
-def _declared():
-    src = open(os.path.join(ROOT, "include", "nfc.h")).read()
+def _declared(headers=("nfc.h", "nfc_debug.h")):
+    src = "".join(open(os.path.join(ROOT, "include", h)).read() for h in headers)
     return sorted(set(re.findall(r"NFC_API\s+[\w\s\*]*?\b(nfc_\w+)\s*\(", src)))
 
 
@@ -36,7 +36,8 @@ def test_library_exports_every_declared_symbol(nfc):
     lib = ctypes.CDLL(nfc.LIB_PATH)
     for name in _declared():
         assert hasattr(lib, name), name
-    assert set(_declared()) == set(nfc.EXPORTS)
+    assert set(_declared(('nfc.h',))) == set(nfc.EXPORTS)
+    assert set(_declared(('nfc_debug.h',))) == set(nfc.DEBUG_EXPORTS)
 
 
 def test_ctypes_layouts_match_header(nfc):
