@@ -1,0 +1,395 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the fused B200 SFC kernel (BASELINE.json metric).
+
+A step is one nfc_process_batch call (one persistent kernel launch) over a
+ring of synthetic packets resident in HBM that is much larger than the 126 MB
+L2.  Default workload: BASELINE config C1's chain ACL(64)->DPI(100)->LPM4(1K)
+on 64-B packets -- the DPI+LPM chain the north-star's HBM-roofline target is
+stated on.  Other configs: --config C2..C5.
+
+    python bench.py [--gpus N --steps K --warmup W] [--config C1] [--impl reference]
+
+Multi-GPU: one process per GPU (torchrun), flows sharded across ranks, no
+data-path collective (weak scaling); the per-rank counters are summed with
+one NCCL all-reduce after the timed region.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+RESTORE_KINDS = {"IPSEC"}    # chains whose in-place rewrite changes the next step's work
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C1")
+    ap.add_argument("--pkt-len", type=int, default=None, help="frame length (0 = IMIX)")
+    ap.add_argument("--k", type=int, default=None, help="C5 chain length")
+    ap.add_argument("--ring-mb", type=int, default=1024, help="HBM ring size per GPU (>> 126 MB L2)")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ workload
+def make_workload(args):
+    import nfcgen
+    w = nfcgen.workload(args.config, pkt_len=args.pkt_len, k=args.k)
+    w.traffic.ttl = 255  # steps re-process the same ring: keep TTL/hop limit from expiring
+    return w
+
+
+def ring_packets(w, ring_mb):
+    import nfcgen
+    probe = nfcgen.generate(w.traffic, w.tables, 0, 4096)
+    slot = (len(probe.arena) - 64) / 4096.0
+    n = int(ring_mb * (1 << 20) / slot)
+    return max(4096, (n // 4096) * 4096)
+
+
+def alg_bytes_per_step(kinds, lens, fam, rec):
+    """Algorithmic HBM bytes of one pass: per packet
+    off+len (10 B) + header sector(s) min(len,64) [+ the rest of the frame if a payload
+    NF (DPI/IPSEC) is reached in original order] + 16 B record + 32 B header rewrite if a
+    forwarder rewrote it + the ESP output frame if IPsec ran; + 6 B per match pair."""
+    lens = lens.astype(np.int64)
+    n = len(lens)
+    drop = rec["drop_nf"].astype(np.int64)
+    parsed = drop != 0xFE
+
+    def reached(p):
+        return parsed & ((drop == 0xFF) | (drop >= p))
+
+    def passed(p):
+        return parsed & ((drop == 0xFF) | (drop > p))
+
+    payload = np.zeros(n, dtype=bool)
+    rewritten = np.zeros(n, dtype=bool)
+    for p, k in enumerate(kinds):
+        if k in ("DPI", "IPSEC"):
+            payload |= reached(p)
+        if k == "LPM4":
+            rewritten |= passed(p) & (fam == 4)
+        if k == "LPM6":
+            rewritten |= passed(p) & (fam == 6)
+    rd = 10 * n + int(np.where(payload, lens, np.minimum(lens, 64)).sum())
+    wr = 16 * n + 32 * int(rewritten.sum())
+    esp = rec["esp_sa"] != 0xFF
+    wr += int(rec["out_len"][esp].astype(np.int64).sum())
+    wr += 6 * int(rec["dpi_nmatch"].astype(np.int64).sum())
+    return rd + wr, rd, wr
+
+
+def frame_family(b):
+    et = b.arena[b.off.astype(np.int64) + 12].astype(np.int64) << 8 | b.arena[b.off.astype(np.int64) + 13]
+    return np.where(et == 0x86DD, 6, np.where(et == 0x0800, 4, 0))
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks",
+               0x10: "sync_boost"}
+
+    def __init__(self, torch_dev: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            import torch
+            pr = torch.cuda.get_device_properties(torch_dev)
+            h = None
+            try:
+                bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+                h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+            except Exception:
+                h = pynvml.nvmlDeviceGetHandleByIndex(torch_dev)
+            self.h, self.nv = h, pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # noqa: BLE001
+            self.err = repr(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "note": getattr(self, "err", "")}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ oracle baseline
+def oracle_rate(w, first, budget_s, chunk=8192, max_chunks=100000):
+    """Plain C oracle, single-threaded, on consecutive chunks of the same workload."""
+    import nfcgen
+    import oracle
+    orc = oracle.OracleChain(w.kinds, w.tables)
+    t_work, pk, by = 0.0, 0, 0
+    i = 0
+    while t_work < budget_s and i < max_chunks:
+        b = nfcgen.generate(w.traffic, w.tables, first + pk, chunk)
+        t0 = time.perf_counter()
+        orc.run(b, match_cap=1 << 20)
+        t_work += time.perf_counter() - t0
+        pk += b.n
+        by += int(b.len.astype(np.int64).sum())
+        i += 1
+    return pk / t_work / 1e6, by * 8 / t_work / 1e9, pk, t_work
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    w = make_workload(args)
+    # calibrate a per-step sample of ~1 s of oracle work
+    rate, _, _, _ = oracle_rate(w, 0, 0.5, chunk=2048, max_chunks=50)
+    per_step = max(2048, int(rate * 1e6 * 1.0) // 2048 * 2048)
+    ts, pk, by = [], 0, 0
+    import nfcgen
+    import oracle
+    orc = oracle.OracleChain(w.kinds, w.tables)
+    for s in range(args.warmup + args.steps):
+        b = nfcgen.generate(w.traffic, w.tables, s * per_step, per_step)
+        t0 = time.perf_counter()
+        orc.run(b, match_cap=1 << 20)
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            ts.append(dt)
+            pk += b.n
+            by += int(b.len.astype(np.int64).sum())
+    tot = sum(ts)
+    mpps = pk / tot / 1e6
+    sample = f"{args.steps} steps x {per_step} packets of {w.name} (same generator/tables), 1 thread"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": round(mpps, 6), "unit": "Mpps",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "gbps": round(by * 8 / tot / 1e9, 6),
+        "config": {"workload": f"{w.name}: {w.note}", "chain": w.kinds, "packets_per_step": per_step},
+        "cpu_baseline": {"value": round(mpps, 6), "unit": "Mpps", "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(mpps, 6), "unit": "Mpps", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    import nfcgen
+    from paper_conf_hpca_hul18_b200 import nfc
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    w = make_workload(args)
+    n = ring_packets(w, args.ring_mb)
+    first = rank * n                       # flows of rank r: its own slice of the global stream
+    b = nfcgen.generate(w.traffic, w.tables, first, n)
+    chain = nfc.Chain(w.kinds, device=local)
+    chain.load_tables(w.tables)
+    hr, tr = chain.room()
+    assert hr <= w.traffic.headroom and tr <= w.traffic.tailroom
+
+    arena = torch.from_numpy(b.arena).to(dev)
+    off = torch.from_numpy(b.off.view(np.int64)).to(dev)
+    ln = torch.from_numpy(b.len.view(np.int16)).to(dev)
+    restore = bool(RESTORE_KINDS & set(w.kinds))
+    pristine = arena.clone() if restore else None
+    rec = torch.empty((n, 16), dtype=torch.uint8, device=dev)
+    cap = 1 << 22
+    mp = torch.empty(cap, dtype=torch.int32, device=dev)
+    mq = torch.empty(cap, dtype=torch.int16, device=dev)
+    mc = torch.zeros(1, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    desc = [(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), n, first)]
+
+    def step():
+        mc.zero_()
+        chain.process(desc, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+
+    for _ in range(args.warmup):
+        if restore:
+            arena.copy_(pristine)
+        step()
+    torch.cuda.synchronize(dev)
+    chain.stats(reset=True)
+    launches0 = chain.launches()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    t_wall0 = time.perf_counter()
+    with ClockSampler(local) as clk:
+        if restore:   # restore the pristine ring between steps, outside the timed intervals
+            for s in range(args.steps):
+                arena.copy_(pristine)
+                ev[s][0].record(stream)
+                step()
+                ev[s][1].record(stream)
+        else:         # back-to-back launches; the 1 GiB ring evicts L2 between passes
+            ev[0][0].record(stream)
+            for s in range(args.steps):
+                step()
+            ev[-1][1].record(stream)
+        torch.cuda.synchronize(dev)
+    t_wall = time.perf_counter() - t_wall0
+    if world > 1:
+        dist.barrier()
+    if restore:
+        ms = sum(a.elapsed_time(b_) for a, b_ in ev)
+    else:
+        ms = ev[0][0].elapsed_time(ev[-1][1])
+    launches = chain.launches() - launches0
+    stats = chain.stats(reset=True)
+    ms_t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    st_t = torch.from_numpy(stats.view(np.int64)).to(dev)
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(st_t, op=dist.ReduceOp.SUM)   # the only collective: counters
+    ms_max = float(ms_t.item())
+    tot_pkts = n * args.steps * world
+    tot_bytes = int(b.len.astype(np.int64).sum()) * args.steps * world
+    mpps = tot_pkts / (ms_max / 1e3) / 1e6
+    gbps = tot_bytes * 8 / (ms_max / 1e3) / 1e9
+
+    # roofline of the (only) kernel: algorithmic bytes per launch / avg launch duration
+    rec_h = rec.cpu().numpy().view(nfcgen.RESULT).reshape(n)
+    alg, rd, wr = alg_bytes_per_step(w.kinds, b.len, frame_family(b), rec_h)
+    launch_ms = ms / args.steps
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    peak = peaks.get("hbm_gbs", 6650.0)
+    achieved = alg / (launch_ms / 1e3) / 1e9
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tfile):
+        tj = json.load(open(tfile)).get(w.name)
+        if tj and tj.get("packets"):
+            traffic = int(tj["dram_bytes_per_launch"] * n / tj["packets"])
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": traffic,
+            "alg_bytes_per_launch": alg, "alg_bytes_per_packet": round(alg / n, 2),
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING fallback"}
+
+    # end to end through the host-buffer C-ABI call (H2D + kernel + D2H every step)
+    e2e = None
+    if not args.no_e2e:
+        host = torch.empty(len(b.arena), dtype=torch.uint8, pin_memory=True)
+        hnp = host.numpy()
+        hoff = torch.from_numpy(b.off.view(np.int64)).pin_memory()
+        hlen = torch.from_numpy(b.len.view(np.int16)).pin_memory()
+        hrec = torch.empty((n, 16), dtype=torch.uint8, pin_memory=True)
+        hmp = torch.empty(cap, dtype=torch.int32, pin_memory=True)
+        hmq = torch.empty(cap, dtype=torch.int16, pin_memory=True)
+        e2e_steps = max(2, min(args.steps, 5))
+        times = []
+        npairs = 0
+        for s in range(1 + e2e_steps):
+            hnp[:] = b.arena
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            npairs = chain.process_host_ptr(host.data_ptr(), len(b.arena), hoff.data_ptr(), hlen.data_ptr(), n,
+                                            hrec.data_ptr(), hmp.data_ptr(), hmq.data_ptr(), cap, first,
+                                            stream.cuda_stream)
+            dt = time.perf_counter() - t0
+            if s:
+                times.append(dt)
+        e2e_t = torch.tensor([sum(times)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        e2e = {"value": round(n * len(times) * world / float(e2e_t.item()) / 1e6, 3), "unit": "Mpps",
+               "h2d_bytes_per_step": len(b.arena) + n * 10,
+               "d2h_bytes_per_step": len(b.arena) + n * 16 + 4 + min(npairs, cap) * 6,
+               "steps": len(times), "api": "nfc_process_host (pinned host buffers)"}
+        chain.stats(reset=True)
+
+    cpu = None
+    if not args.no_cpu and rank == 0 and world == 1:
+        r_mpps, r_gbps, r_pk, r_t = oracle_rate(w, first, args.cpu_seconds)
+        cpu = {"value": round(r_mpps, 6), "unit": "Mpps", "cores": 1, "kind": "oracle",
+               "sample": f"{r_pk} packets of {w.name} (same generator and tables), {r_t:.1f} s, 1 thread",
+               "gbps": round(r_gbps, 6)}
+
+    if rank == 0:
+        st = st_t.cpu().numpy().view(np.uint64)
+        out = {
+            "metric": METRIC, "value": round(mpps, 3), "unit": "Mpps", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "gbps": round(gbps, 2),
+            "config": {"workload": f"{w.name}: {w.note}", "chain": w.kinds,
+                       "pkt_len": "IMIX" if w.traffic.pkt_len == 0 else w.traffic.pkt_len,
+                       "packets_per_step_per_gpu": n, "ring_bytes_per_gpu": len(b.arena),
+                       "l2": "ring >> 126 MB L2 (no flush needed)" if not restore else
+                             "pristine ring restored between steps (1 GiB-class copy, evicts L2), outside timed intervals",
+                       "timing": "CUDA events on the launch stream; max over ranks",
+                       "parallelism": f"flow-sharded x{world}, no data-path collective",
+                       "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4)},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            "wall_s_timed_region": round(t_wall, 4),
+        }
+        print(json.dumps(out))
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

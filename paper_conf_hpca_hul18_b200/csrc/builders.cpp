@@ -29,12 +29,50 @@ static void mask128(const uint8_t *a, int len, uint32_t w[4])
 }
 
 // ---------------------------------------------------------------- ACL
-std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector<uint4> &r6)
+// Bit-vector classification (Lakshman & Stiliadis style), one image per address
+// family.  Each of the fields src, dst, sport, dport is cut into elementary
+// intervals at the rule boundaries; interval j carries the bitset of rules whose
+// range contains it; proto has a direct 256-entry bitset table.  The lookup ANDs
+// the five bitsets and takes the lowest set bit = the first matching rule.
+// Blob layout (u32 words): see AclBv in nfc_internal.h.
+namespace {
+typedef unsigned __int128 u128;
+static u128 key128(const uint8_t *a)
+{
+    u128 k = 0;
+    for (int i = 0; i < 16; i++) k = (k << 8) | a[i];
+    return k;
+}
+static u128 mask128v(int len) { return len <= 0 ? (u128)0 : len >= 128 ? ~(u128)0 : ~(u128)0 << (128 - len); }
+
+struct FieldIv {
+    std::vector<u128> b;                  // interval starts, b[0] = 0
+    std::vector<uint64_t> bv;             // b.size() x W words
+};
+
+static void build_field(const std::vector<std::pair<u128, u128>> &rng, u128 maxv, uint32_t W, FieldIv &f)
+{
+    std::vector<u128> pts{0};
+    for (auto &r : rng) {
+        pts.push_back(r.first);
+        if (r.second != maxv) pts.push_back(r.second + 1);
+    }
+    std::sort(pts.begin(), pts.end());
+    pts.erase(std::unique(pts.begin(), pts.end()), pts.end());
+    f.b = pts;
+    f.bv.assign(pts.size() * W, 0);
+    for (size_t r = 0; r < rng.size(); r++) {
+        size_t j0 = std::lower_bound(pts.begin(), pts.end(), rng[r].first) - pts.begin();
+        for (size_t j = j0; j < pts.size() && pts[j] <= rng[r].second; j++) f.bv[j * W + r / 64] |= 1ull << (r % 64);
+    }
+}
+} // namespace
+
+std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6)
 {
     if (s.n_rules > 65534) return "acl: too many rules (max 65534)";
     if (s.n_rules && !s.rules) return "acl: rules == NULL";
     if (s.default_action > 1) return "acl: default_action must be 0 or 1";
-    r4.clear(); r6.clear();
     for (uint32_t i = 0; i < s.n_rules; i++) {
         const nfc_acl_rule &r = s.rules[i];
         int maxl = r.family == 4 ? 32 : 128;
@@ -42,22 +80,64 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector
         if (r.slen > maxl || r.dlen > maxl) return "acl: prefix length out of range";
         if (r.sp_lo > r.sp_hi || r.dp_lo > r.dp_hi) return "acl: port range lo > hi";
         if (r.action > 1 || r.proto_any > 1) return "acl: bad action/proto_any";
-        uint4 tail = make_uint4((uint32_t)r.sp_lo | (uint32_t)r.sp_hi << 16, (uint32_t)r.dp_lo | (uint32_t)r.dp_hi << 16,
-                                (uint32_t)r.proto | (uint32_t)r.proto_any << 8 | (uint32_t)r.action << 16, i);
-        if (r.family == 4) {
-            uint32_t sm = mask32(r.slen), dm = mask32(r.dlen);
-            r4.push_back(make_uint4(be32(r.src) & sm, sm, be32(r.dst) & dm, dm));
-            r4.push_back(tail);
-        } else {
-            uint32_t sw[4], dw[4];
-            mask128(r.src, r.slen, sw);
-            mask128(r.dst, r.dlen, dw);
-            r6.push_back(make_uint4(sw[0], sw[1], sw[2], sw[3]));
-            r6.push_back(make_uint4(mask32(r.slen), mask32(r.slen - 32), mask32(r.slen - 64), mask32(r.slen - 96)));
-            r6.push_back(make_uint4(dw[0], dw[1], dw[2], dw[3]));
-            r6.push_back(make_uint4(mask32(r.dlen), mask32(r.dlen - 32), mask32(r.dlen - 64), mask32(r.dlen - 96)));
-            r6.push_back(tail);
+    }
+    for (int fam : {4, 6}) {
+        std::vector<uint32_t> &blob = fam == 4 ? blob4 : blob6;
+        std::vector<uint32_t> gidx;
+        for (uint32_t i = 0; i < s.n_rules; i++)
+            if (s.rules[i].family == fam) gidx.push_back(i);
+        const uint32_t n = (uint32_t)gidx.size(), W = (n + 63) / 64, kw = fam == 4 ? 1 : 4;
+        const int bits = fam == 4 ? 32 : 128;
+        const u128 amax = fam == 4 ? (u128)0xFFFFFFFFu : ~(u128)0;
+        std::vector<std::pair<u128, u128>> rs, rd, rsp, rdp;
+        for (uint32_t g : gidx) {
+            const nfc_acl_rule &r = s.rules[g];
+            u128 sk = fam == 4 ? (u128)be32(r.src) : key128(r.src), dk = fam == 4 ? (u128)be32(r.dst) : key128(r.dst);
+            u128 sm = mask128v(r.slen) >> (128 - bits), dm = mask128v(r.dlen) >> (128 - bits);
+            if (fam == 4) { sm &= 0xFFFFFFFFu; dm &= 0xFFFFFFFFu; }
+            rs.push_back({sk & sm, (sk & sm) | (amax & ~sm)});
+            rd.push_back({dk & dm, (dk & dm) | (amax & ~dm)});
+            rsp.push_back({r.sp_lo, r.sp_hi});
+            rdp.push_back({r.dp_lo, r.dp_hi});
         }
+        FieldIv F[4];
+        build_field(rs, amax, W ? W : 1, F[0]);
+        build_field(rd, amax, W ? W : 1, F[1]);
+        build_field(rsp, 0xFFFF, W ? W : 1, F[2]);
+        build_field(rdp, 0xFFFF, W ? W : 1, F[3]);
+        const uint32_t Wd = W ? W : 1;
+        std::vector<uint64_t> vproto(256 * Wd, 0);
+        for (uint32_t r = 0; r < n; r++) {
+            const nfc_acl_rule &ru = s.rules[gidx[r]];
+            for (int p = 0; p < 256; p++)
+                if (ru.proto_any || ru.proto == p) vproto[p * Wd + r / 64] |= 1ull << (r % 64);
+        }
+        blob.assign(ACLBV_HDR, 0);
+        blob[0] = n; blob[1] = Wd; blob[2] = (uint32_t)F[0].b.size(); blob[3] = (uint32_t)F[1].b.size();
+        blob[4] = (uint32_t)F[2].b.size(); blob[5] = (uint32_t)F[3].b.size(); blob[6] = kw;
+        auto align2 = [&]() { if (blob.size() & 1) blob.push_back(0); };
+        auto put_keys = [&](const FieldIv &f, uint32_t kwords) {
+            uint32_t o = (uint32_t)blob.size();
+            for (u128 k : f.b)
+                for (int q = (int)kwords - 1; q >= 0; q--) blob.push_back((uint32_t)(k >> (32 * q)));
+            return o;
+        };
+        auto put_bv = [&](const std::vector<uint64_t> &v) {
+            align2();
+            uint32_t o = (uint32_t)blob.size();
+            for (uint64_t x : v) { blob.push_back((uint32_t)x); blob.push_back((uint32_t)(x >> 32)); }
+            return o;
+        };
+        uint32_t offs[10];
+        offs[0] = put_keys(F[0], kw); offs[1] = put_bv(F[0].bv);
+        offs[2] = put_keys(F[1], kw); offs[3] = put_bv(F[1].bv);
+        offs[4] = put_keys(F[2], 1);  offs[5] = put_bv(F[2].bv);
+        offs[6] = put_keys(F[3], 1);  offs[7] = put_bv(F[3].bv);
+        offs[8] = put_bv(vproto);
+        offs[9] = (uint32_t)blob.size();
+        for (uint32_t r = 0; r < n; r++) blob.push_back(gidx[r] | (uint32_t)s.rules[gidx[r]].action << 31);
+        while (blob.size() & 3) blob.push_back(0);   // 16-B multiple for staging copies
+        for (int k = 0; k < 10; k++) blob[8 + k] = offs[k];
     }
     return "";
 }

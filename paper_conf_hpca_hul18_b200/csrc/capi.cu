@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdio>
+#include <algorithm>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -179,13 +180,13 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
     case NFC_ACL: {
         if (spec_bytes != sizeof(nfc_acl_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_acl_spec)");
         const nfc_acl_spec &s = *static_cast<const nfc_acl_spec *>(spec);
-        std::vector<uint4> r4, r6;
-        err = build_acl(s, r4, r6);
+        std::vector<uint32_t> b4, b6;
+        err = build_acl(s, b4, b6);
         if (!err.empty()) return fail(NFC_EINVAL, err);
-        CK(c->acl_r4.upload(r4));
-        CK(c->acl_r6.upload(r6));
-        c->acl = AclImg{c->acl_r4.as<uint4>(), (uint32_t)(r4.size() / 2), c->acl_r6.as<uint4>(),
-                        (uint32_t)(r6.size() / 5), s.n_rules, s.default_action};
+        CK(c->acl_r4.upload(b4));
+        CK(c->acl_r6.upload(b6));
+        c->acl = AclImg{c->acl_r4.as<uint32_t>(), c->acl_r6.as<uint32_t>(), (uint32_t)b4.size(),
+                        (uint32_t)b6.size(), s.n_rules, s.default_action, 0};
         c->n_acl_rules = s.n_rules;
         break;
     }
@@ -352,6 +353,25 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         p.epoch = c->epoch;
         p.seq_in = c->esp_seq[c->seq_parity].as<uint32_t>();
         p.seq_out = c->esp_seq[c->seq_parity ^ 1].as<uint32_t>();
+    }
+    // shared-memory budget per CTA for the target occupancy: stage the ACL image
+    // when it fits and give the rest to full-row DFA hot states
+    {
+        int smem_sm = 0;
+        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device);
+        const int target = (c->mask & MASK_IPSEC) ? 2 : 4;
+        const size_t budget = (size_t)smem_sm / target - 1024 - 64;
+        p.acl.smem_words = 0;
+        p.dpi.hot_states = 0;
+        if (c->mask & MASK_ACL) {
+            p.acl.smem_words = 1;
+            if (sfc_smem_bytes(c->mask, p) > budget / 2) p.acl.smem_words = 0;
+        }
+        if ((c->mask & MASK_DPI) && !c->dpi.wide) {
+            size_t base = sfc_smem_bytes(c->mask, p);
+            size_t h = base < budget ? (budget - base) / 512 : 0;
+            p.dpi.hot_states = (uint32_t)std::min<size_t>(h, c->dpi.n_states);
+        }
     }
     if (c->mask & MASK_DPI) {
         LaunchCfg q{};

@@ -14,7 +14,7 @@ using namespace nfc;
 
 struct nfc_dbg {
     uint32_t kind = 0;
-    std::vector<uint4> r4, r6;
+    std::vector<uint32_t> r4, r6;
     uint32_t n_rules = 0, default_action = 0;
     DpiHost dpi;
     std::vector<uint16_t> tbl24, tbllong;
@@ -152,39 +152,50 @@ int nfc_dbg_lpm6(nfc_dbg *d, const uint8_t dst[16], uint32_t *nh, uint32_t *prob
     return NFC_OK;
 }
 
+static uint32_t bs32(const uint32_t *B, uint32_t m, uint32_t key)
+{
+    uint32_t lo = 0;
+    while (m > 1) { uint32_t h = m >> 1; if (B[lo + h] <= key) lo += h; m -= h; }
+    return lo;
+}
+static bool le128h(const uint32_t *b, const uint32_t *k)
+{
+    for (int q = 0; q < 3; q++) if (b[q] != k[q]) return b[q] < k[q];
+    return b[3] <= k[3];
+}
+static uint32_t bs128(const uint32_t *B, uint32_t m, const uint32_t *k)
+{
+    uint32_t lo = 0;
+    while (m > 1) { uint32_t h = m >> 1; if (le128h(B + 4 * (lo + h), k)) lo += h; m -= h; }
+    return lo;
+}
+
 int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *dst, uint16_t sport,
                 uint16_t dport, uint8_t proto, uint32_t *rule, uint32_t *action)
 {
     if (!d || d->kind != NFC_ACL) return NFC_EINVAL;
-    auto tail_ok = [&](const uint4 &t) {
-        if (sport < (t.x & 0xFFFF) || sport > (t.x >> 16)) return false;
-        if (dport < (t.y & 0xFFFF) || dport > (t.y >> 16)) return false;
-        if (!((t.z >> 8) & 1) && (t.z & 0xFF) != proto) return false;
-        return true;
-    };
+    const uint32_t *A = family == 4 ? d->r4.data() : d->r6.data();
     *rule = 0xFFFF;
     *action = d->default_action;
-    if (family == 4) {
-        uint32_t s = be32(src), t = be32(dst);
-        for (size_t i = 0; i + 1 < d->r4.size(); i += 2) {
-            const uint4 &r = d->r4[i];
-            if ((s & r.y) != r.x || (t & r.w) != r.z || !tail_ok(d->r4[i + 1])) continue;
-            *rule = d->r4[i + 1].w;
-            *action = (d->r4[i + 1].z >> 16) & 1;
-            return NFC_OK;
-        }
-    } else {
-        uint32_t s[4], t[4];
-        for (int k = 0; k < 4; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
-        for (size_t i = 0; i + 4 < d->r6.size(); i += 5) {
-            const uint4 *r = &d->r6[i];
-            const uint32_t sv[4] = {r[0].x, r[0].y, r[0].z, r[0].w}, sm[4] = {r[1].x, r[1].y, r[1].z, r[1].w};
-            const uint32_t dv[4] = {r[2].x, r[2].y, r[2].z, r[2].w}, dm[4] = {r[3].x, r[3].y, r[3].z, r[3].w};
-            bool ok = true;
-            for (int k = 0; k < 4; k++) ok &= (s[k] & sm[k]) == sv[k] && (t[k] & dm[k]) == dv[k];
-            if (!ok || !tail_ok(r[4])) continue;
-            *rule = r[4].w;
-            *action = (r[4].z >> 16) & 1;
+    if (A[0] == 0) return NFC_OK;
+    uint32_t s[4], t[4];
+    int nb = family == 4 ? 1 : 4;
+    for (int k = 0; k < nb; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
+    const uint32_t W = A[1];
+    uint32_t js = nb == 1 ? bs32(A + A[8], A[2], s[0]) : bs128(A + A[8], A[2], s);
+    uint32_t jd = nb == 1 ? bs32(A + A[10], A[3], t[0]) : bs128(A + A[10], A[3], t);
+    uint32_t jsp = bs32(A + A[12], A[4], sport), jdp = bs32(A + A[14], A[5], dport);
+    auto bv = [&](uint32_t off, uint32_t j, uint32_t w) {
+        uint64_t x;
+        memcpy(&x, A + off + 2 * ((size_t)j * W + w), 8);
+        return x;
+    };
+    for (uint32_t w = 0; w < W; w++) {
+        uint64_t x = bv(A[9], js, w) & bv(A[11], jd, w) & bv(A[13], jsp, w) & bv(A[15], jdp, w) & bv(A[16], proto, w);
+        if (x) {
+            uint32_t e = A[A[17] + 64 * w + __builtin_ctzll(x)];
+            *rule = e & 0xFFFF;
+            *action = e >> 31;
             return NFC_OK;
         }
     }

@@ -13,16 +13,18 @@
 namespace nfc {
 
 // ---------------------------------------------------------------- ACL
-// Linear first-match image, rules of one family in priority order.
-// IPv4 rule = 2 x uint4:  {src, smask, dst, dmask}, {sp_lo|sp_hi<<16, dp_lo|dp_hi<<16,
-//                          proto | proto_any<<8 | action<<16, global rule index}
-// IPv6 rule = 5 x uint4:  src[4], smask[4], dst[4], dmask[4] (BE-value words), then the
-//                          same tail word group.
+// Bit-vector image per family (u32 blob):
+//   [0] n rules of the family  [1] W = 64-bit words per bitset  [2..5] interval counts
+//   m_src, m_dst, m_sport, m_dport  [6] key words per address (1 v4, 4 v6)
+//   [8..17] word offsets: keys_src, bv_src, keys_dst, bv_dst, keys_sp, bv_sp, keys_dp, bv_dp,
+//   bv_proto (256 x W), ridx (global rule index | action << 31).  Bitsets are u64 at even offsets.
+static const uint32_t ACLBV_HDR = 20;
 struct AclImg {
-    const uint4 *r4; uint32_t n4;
-    const uint4 *r6; uint32_t n6;
+    const uint32_t *bv4, *bv6;        // device blobs
+    uint32_t words4, words6;          // blob sizes (u32 words)
     uint32_t n_rules;
     uint32_t default_action;
+    uint32_t smem_words;              // words staged in shared memory (0 = read from global)
 };
 
 // ---------------------------------------------------------------- DPI
@@ -40,7 +42,7 @@ struct DpiImg {
     uint32_t n_pat;
     uint32_t *ovf_bitmap;        // per resident thread scratch for > DPI_LIST distinct matches
     uint32_t bitmap_words;       // words per thread
-    uint32_t smem_states;        // rows of trans staged in shared memory (0 = none)
+    uint32_t hot_states;         // states whose full 256-byte rows are staged in shared memory
 };
 
 // ---------------------------------------------------------------- LPM4 (DIR-24-8)
@@ -142,7 +144,7 @@ struct KParams {
 
 // host-side builders (builders.cpp); return "" on success or an error message
 struct HostImage { std::vector<uint8_t> bytes; };
-std::string build_acl(const nfc_acl_spec &s, std::vector<uint4> &r4, std::vector<uint4> &r6);
+std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
 struct DpiHost {
     std::vector<uint8_t> cls;
     std::vector<uint8_t> trans;   // raw bytes (u16 or u32 entries)

@@ -1,17 +1,21 @@
 // sfc_kernel.cu -- the fused, persistent SFC kernel for sm_100a.
 //
-// One launch drains all packets of an nfc_process_batch call.  Each CTA of
-// TILE threads repeatedly claims a tile of TILE consecutive packets from a
-// global atomic counter (persistent kernel, P:L112, P:L235 [SIV]) and every
-// thread carries one packet through the whole chain in registers:
+// One launch drains all packets of an nfc_process_batch call.  Every thread
+// carries one packet through the whole chain in registers:
 //   parse once (the de-duplicated header classifier)
 //   -> NFs in original SFC order, a dropped packet skipping every later NF
-//      (early drop; no batch re-split between NFs)
-//   -> ESP sequence numbers per SA in global packet order via a decoupled
-//      look-back across tiles (the only cross-packet dependency)
-//   -> one 16 B result record, counters aggregated per warp / CTA.
-// Packet bytes are read from HBM once and rewritten in place.  No tensor
-// cores: nothing here is a dense contraction (integer / table-lookup work).
+//      (early drop; no batch re-split or per-NF launch)
+//   -> one 16 B result record; counters in per-warp private shared memory.
+// Scheduling (persistent kernel, P:L112, P:L235 [SIV]): without IPsec each warp
+// claims 32-packet chunks from a global atomic counter (no CTA barriers); with
+// IPsec each CTA claims TILE-packet tiles in order and assigns per-SA ESP
+// sequence numbers in global packet order by a decoupled look-back.
+// Tables stay on chip where they fit: the ACL bit-vector image, the hot rows
+// of the Aho-Corasick DFA, AES T-tables and Toeplitz nibble tables live in
+// shared memory; DIR-24-8 / IPv6 hash levels are read through L2 with an
+// evict-last policy while the packet stream is evict-first.  Packet bytes are
+// read from HBM once and rewritten in place.  No tensor cores: nothing here is
+// a dense contraction.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -19,24 +23,32 @@
 
 namespace nfc {
 
-static constexpr int TILE = 256;        // threads per CTA == packets per tile
+static constexpr int TILE = 256;        // threads per CTA (== packets per IPsec tile)
 static constexpr int NWARP = TILE / 32;
-static constexpr int DPI_LIST = 16;     // distinct matches kept in registers before the bitmap path
+static constexpr int DPI_LIST = 16;     // distinct matches kept in a list before the bitmap path
+static constexpr int NFIX = ST_VAR_BASE;
 
 // ---------------------------------------------------------------- shared memory layout
 struct SmemLayout {
-    uint32_t te, ms_nib, lb_nib, cls, stats, wcnt, prefix, total;
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, acl4, acl6, wcnt, prefix, total;
 };
 __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, const KParams &p)
 {
     SmemLayout L{};
     uint32_t o = 0;
+    L.wst = o; o += NWARP * NFIX * 8;                              // per-warp private counters (u64)
+    L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
+    o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 5 * 256 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
-    if (mask & MASK_DPI) { L.cls = o; o += 256; }
+    if (mask & MASK_DPI) { L.cls = o; o += 256; L.hot = o; o += p.dpi.hot_states * 256 * 2; }
     o = (o + 15) & ~15u;
-    L.stats = o;
-    o += (p.smem_stats ? p.stats_len : ST_VAR_BASE) * 8;
+    if (mask & MASK_ACL) {
+        const uint32_t s4 = p.acl.smem_words ? p.acl.words4 : 0, s6 = p.acl.smem_words ? p.acl.words6 : 0;
+        L.acl4 = o; o += s4 * 4;
+        L.acl6 = o; o += s6 * 4;
+    }
+    o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += NWARP * 256 * 2;
         L.prefix = o; o += 256 * 4;
@@ -59,22 +71,43 @@ __device__ __forceinline__ void st_release(uint32_t *p, uint32_t v)
 }
 __device__ __forceinline__ uint32_t mask32d(int len) { return len <= 0 ? 0u : len >= 32 ? 0xFFFFFFFFu : 0xFFFFFFFFu << (32 - len); }
 
+// L2 eviction policies: the packet stream is touched once (evict-first); lookup
+// tables are re-used by every packet (evict-last).
+__device__ __forceinline__ uint64_t pol_first()
+{
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_last()
+{
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint4 ld_stream16(const void *a, uint64_t pol)
+{
+    uint4 v;
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void st_stream16(void *a, uint4 v, uint64_t pol)
+{
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;"
+                 ::"l"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_tab16(const uint16_t *a, uint64_t pol)
+{
+    uint16_t v;
+    asm("ld.global.nc.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(a), "l"(pol));
+    return v;
+}
+
 // byte k (0..63) of the 64 B header cache; k compile-time in hot paths
 __device__ __forceinline__ uint32_t hbyte(const uint32_t h[16], uint32_t k) { return (h[k >> 2] >> ((k & 3) * 8)) & 0xFF; }
 __device__ __forceinline__ uint32_t hbe16(const uint32_t h[16], uint32_t k) { return hbyte(h, k) << 8 | hbyte(h, k + 1); }
 __device__ __forceinline__ uint32_t hbe32(const uint32_t h[16], uint32_t k) { return hbe16(h, k) << 16 | hbe16(h, k + 2); }
-// dynamic byte index: header cache if < 64 else global memory
-__device__ __forceinline__ uint32_t dbyte(const uint32_t h[16], const uint8_t *f, uint32_t k)
-{
-    if (k < 64) {
-        uint32_t w = 0;
-#pragma unroll
-        for (int j = 0; j < 16; j++) w = (j == (int)(k >> 2)) ? h[j] : w;
-        return (w >> ((k & 3) * 8)) & 0xFF;
-    }
-    return f[k];
-}
-
 // ---------------------------------------------------------------- per-packet state
 struct PV {
     uint32_t fam;                 // 4 or 6
@@ -83,19 +116,18 @@ struct PV {
     uint32_t src[4], dst[4];      // big-endian-valued words
 };
 
-__device__ __forceinline__ void load_header(const uint8_t *f, uint32_t flen, uint32_t h[16])
+__device__ __forceinline__ void load_header(const uint8_t *f, uint32_t flen, uint32_t h[16], uint64_t pol)
 {
-    const uint4 *q = reinterpret_cast<const uint4 *>(f);
-    uint32_t nch = min(4u, (flen + 15) >> 4);
+    const uint32_t nch = min(4u, (flen + 15) >> 4);
 #pragma unroll
     for (int c = 0; c < 4; c++) {
-        uint4 v = c < (int)nch ? q[c] : make_uint4(0, 0, 0, 0);
+        uint4 v = c < (int)nch ? ld_stream16(f + 16 * c, pol) : make_uint4(0, 0, 0, 0);
         h[4 * c] = v.x; h[4 * c + 1] = v.y; h[4 * c + 2] = v.z; h[4 * c + 3] = v.w;
     }
 }
 
 // Parse (P:L87 validity check): Ethernet -> IPv4/IPv6 -> UDP/TCP.
-__device__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV &v)
+__device__ __forceinline__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV &v)
 {
     if (flen < 14) return false;
     uint32_t et = hbe16(h, 12);
@@ -140,15 +172,16 @@ __device__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV 
             l4len = 8;
         } else {
             if (l4 + 20 > v.ip_end) return false;
-            uint32_t doff = dbyte(h, f, l4 + 12) >> 4;
+            // data offset: byte 46 sits in the header cache; other offsets are rare -> memory
+            uint32_t doff = (l4 == 34 ? hbyte(h, 46) : (uint32_t)f[l4 + 12]) >> 4;
             if (doff < 5 || l4 + 4 * doff > v.ip_end) return false;
             l4len = 4 * doff;
         }
         if (l4 == 34) { v.sport = hbe16(h, 34); v.dport = hbe16(h, 36); }
         else if (l4 == 54) { v.sport = hbe16(h, 54); v.dport = hbe16(h, 56); }
         else {
-            v.sport = dbyte(h, f, l4) << 8 | dbyte(h, f, l4 + 1);
-            v.dport = dbyte(h, f, l4 + 2) << 8 | dbyte(h, f, l4 + 3);
+            v.sport = (uint32_t)f[l4] << 8 | f[l4 + 1];      // IPv4 options: rare, from memory
+            v.dport = (uint32_t)f[l4 + 2] << 8 | f[l4 + 3];
         }
     }
     v.pl_off = v.l4_off + l4len;
@@ -156,132 +189,199 @@ __device__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV 
 }
 
 // ---------------------------------------------------------------- ACL
-// First-match linear scan over the packet's family (rules kept in priority order).
-__device__ uint32_t nf_acl(const AclImg &a, const PV &v)
+// Bit-vector first match: five interval lookups (binary search over the
+// elementary-interval starts), AND of the five rule bitsets, lowest set bit.
+__device__ __forceinline__ uint32_t bsearch32(const uint32_t *B, uint32_t m, uint32_t key)
 {
-    uint32_t ports = v.sport << 16 | v.dport;
-    (void)ports;
-    if (v.fam == 4) {
-        for (uint32_t i = 0; i < a.n4; i++) {
-            uint4 r = __ldg(a.r4 + 2 * i);
-            if (((v.src[0] & r.y) != r.x) | ((v.dst[0] & r.w) != r.z)) continue;
-            uint4 t = __ldg(a.r4 + 2 * i + 1);
-            if (v.sport < (t.x & 0xFFFF) || v.sport > (t.x >> 16)) continue;
-            if (v.dport < (t.y & 0xFFFF) || v.dport > (t.y >> 16)) continue;
-            if (!((t.z >> 8) & 1) && (t.z & 0xFF) != v.proto) continue;
-            return t.w | ((t.z >> 16) & 1) << 31;
-        }
-    } else {
-        for (uint32_t i = 0; i < a.n6; i++) {
-            const uint4 *r = a.r6 + 5 * i;
-            uint4 s = __ldg(r), sm = __ldg(r + 1);
-            if (((v.src[0] & sm.x) != s.x) | ((v.src[1] & sm.y) != s.y) | ((v.src[2] & sm.z) != s.z) |
-                ((v.src[3] & sm.w) != s.w)) continue;
-            uint4 d = __ldg(r + 2), dm = __ldg(r + 3);
-            if (((v.dst[0] & dm.x) != d.x) | ((v.dst[1] & dm.y) != d.y) | ((v.dst[2] & dm.z) != d.z) |
-                ((v.dst[3] & dm.w) != d.w)) continue;
-            uint4 t = __ldg(r + 4);
-            if (v.sport < (t.x & 0xFFFF) || v.sport > (t.x >> 16)) continue;
-            if (v.dport < (t.y & 0xFFFF) || v.dport > (t.y >> 16)) continue;
-            if (!((t.z >> 8) & 1) && (t.z & 0xFF) != v.proto) continue;
-            return t.w | ((t.z >> 16) & 1) << 31;
-        }
+    uint32_t lo = 0;
+    while (m > 1) {
+        const uint32_t half = m >> 1;
+        lo = (B[lo + half] <= key) ? lo + half : lo;
+        m -= half;
     }
-    return 0xFFFFu | a.default_action << 31;   // no match
+    return lo;
+}
+__device__ __forceinline__ bool le128(const uint32_t *b, const uint32_t k[4])
+{
+    if (b[0] != k[0]) return b[0] < k[0];
+    if (b[1] != k[1]) return b[1] < k[1];
+    if (b[2] != k[2]) return b[2] < k[2];
+    return b[3] <= k[3];
+}
+__device__ __forceinline__ uint32_t bsearch128(const uint32_t *B, uint32_t m, const uint32_t k[4])
+{
+    uint32_t lo = 0;
+    while (m > 1) {
+        const uint32_t half = m >> 1;
+        lo = le128(B + 4 * (lo + half), k) ? lo + half : lo;
+        m -= half;
+    }
+    return lo;
+}
+
+// returns global rule index (0xFFFF none) | action << 31
+__device__ __forceinline__ uint32_t nf_acl(const uint32_t *A, uint32_t default_action, const PV &v)
+{
+    const uint32_t n = A[0];
+    if (n == 0) return 0xFFFFu | default_action << 31;
+    const uint32_t W = A[1];
+    uint32_t js, jd;
+    if (A[6] == 1) {
+        js = bsearch32(A + A[8], A[2], v.src[0]);
+        jd = bsearch32(A + A[10], A[3], v.dst[0]);
+    } else {
+        js = bsearch128(A + A[8], A[2], v.src);
+        jd = bsearch128(A + A[10], A[3], v.dst);
+    }
+    const uint32_t jsp = bsearch32(A + A[12], A[4], v.sport);
+    const uint32_t jdp = bsearch32(A + A[14], A[5], v.dport);
+    const uint64_t *vs = reinterpret_cast<const uint64_t *>(A + A[9]) + (size_t)js * W;
+    const uint64_t *vd = reinterpret_cast<const uint64_t *>(A + A[11]) + (size_t)jd * W;
+    const uint64_t *vsp = reinterpret_cast<const uint64_t *>(A + A[13]) + (size_t)jsp * W;
+    const uint64_t *vdp = reinterpret_cast<const uint64_t *>(A + A[15]) + (size_t)jdp * W;
+    const uint64_t *vpr = reinterpret_cast<const uint64_t *>(A + A[16]) + (size_t)v.proto * W;
+    for (uint32_t w = 0; w < W; w++) {
+        const uint64_t x = vs[w] & vd[w] & vsp[w] & vdp[w] & vpr[w];
+        if (x) return A[A[17] + 64 * w + (__ffsll((long long)x) - 1)];
+    }
+    return 0xFFFFu | default_action << 31;
 }
 
 // ---------------------------------------------------------------- DPI
-struct DpiOut { uint32_t nmatch; bool drop; uint16_t ids[DPI_LIST]; bool ovf; };
+// Aho-Corasick DFA walk.  States below hot_states use full 256-byte rows staged
+// in shared memory; the rest read the global class-compressed table.
+struct DpiCtx {
+    const uint8_t *cls;     // smem
+    const uint16_t *hot;    // smem
+    uint32_t H, ncls, wide;
+    const void *trans;
+    const uint32_t *out_off;
+    const uint16_t *out_ids;
+    const uint8_t *pat_action;
+};
 
-__device__ __forceinline__ uint32_t dfa_step(const DpiImg &d, const uint8_t *cls, uint32_t s, uint32_t b, bool &acc)
+__device__ __forceinline__ uint32_t dfa_step(const DpiCtx &c, uint32_t s, uint32_t b, bool &acc)
 {
-    uint32_t c = cls[b];
     uint32_t e;
-    if (d.wide) { e = __ldg(reinterpret_cast<const uint32_t *>(d.trans) + s * d.ncls + c); acc = e >> 31; e &= 0x7FFFFFFFu; }
-    else { e = __ldg(reinterpret_cast<const uint16_t *>(d.trans) + s * d.ncls + c); acc = e >> 15; e &= 0x7FFFu; }
-    return e;
+    if (s < c.H) {
+        e = c.hot[(s << 8) | b];
+        acc = e >> 15;
+        return e & 0x7FFFu;
+    }
+    const uint32_t k = s * c.ncls + c.cls[b];
+    if (c.wide) { e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k); acc = e >> 31; return e & 0x7FFFFFFFu; }
+    e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
+    acc = e >> 15;
+    return e & 0x7FFFu;
 }
 
-// Walk the DFA over payload [pl_off, ip_end).  Distinct ids go to a register list;
-// more than DPI_LIST distinct ids switch to an exact per-thread bitmap rescan.
+// walk payload [a, b): bytes < 64 from the header cache, the rest from memory
 template <typename F>
-__device__ __forceinline__ void dpi_scan(const uint8_t *f, uint32_t a, uint32_t b, F &&on_byte)
+__device__ __forceinline__ void dpi_walk(const uint32_t h[16], const uint8_t *f, uint32_t a, uint32_t b, uint64_t pol,
+                                         F &&on_byte)
 {
-    if (a >= b) return;
-    uint32_t c0 = a & ~15u;
-    for (uint32_t c = c0; c < b; c += 16) {
-        uint4 q = *reinterpret_cast<const uint4 *>(f + c);
-        uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+    for (int c = 0; c < 64; c += 16) {
+        if ((uint32_t)c + 16 > a && (uint32_t)c < b) {
+#pragma unroll
+            for (int k = 0; k < 16; k++) {
+                const uint32_t idx = c + k;
+                if (idx >= a && idx < b) on_byte((h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF);
+            }
+        }
+    }
+    for (uint32_t c = max(64u, a & ~15u); c < b; c += 16) {
+        const uint4 q = ld_stream16(f + c, pol);
+        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
         for (int k = 0; k < 16; k++) {
-            uint32_t idx = c + k;
+            const uint32_t idx = c + k;
             if (idx >= a && idx < b) on_byte((w[k >> 2] >> ((k & 3) * 8)) & 0xFF);
         }
     }
 }
 
-__device__ void nf_dpi(const DpiImg &d, const uint8_t *cls, const uint8_t *f, const PV &v, uint32_t gtid,
-                       DpiOut &o)
+// Exact match set of a packet whose walk hit an accepting state (rare path, not
+// inlined): re-walk the payload from memory collecting distinct pattern ids in a
+// register list, or -- beyond DPI_LIST ids -- in a per-thread global bitmap; emit
+// the (packet, pattern) pairs.  Returns nmatch | any_drop << 31.
+struct DpiOvf {
+    uint32_t *bitmap;
+    uint32_t words;
+    uint32_t *match_count, *match_pkt;
+    uint16_t *match_pat;
+    uint32_t match_cap;
+    unsigned long long *stats;
+};
+__device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a, uint32_t b, uint32_t gtid,
+                                          DpiOvf o, uint32_t pkt_id)
 {
-    o.nmatch = 0; o.drop = false; o.ovf = false;
+    uint16_t ids[DPI_LIST];
+    uint32_t n = 0, drop = 0;
+    bool ovf = false;
     uint32_t s = 0;
-    dpi_scan(f, v.pl_off, v.ip_end, [&](uint32_t byte) {
+    for (uint32_t i = a; i < b && !ovf; i++) {
         bool acc;
-        s = dfa_step(d, cls, s, byte, acc);
-        if (acc) {
-            uint32_t e = __ldg(d.out_off + s + 1);
-            for (uint32_t x = __ldg(d.out_off + s); x < e; x++) {
-                uint32_t id = __ldg(d.out_ids + x);
-                o.drop |= __ldg(d.pat_action + id) != 0;
-                if (o.ovf) continue;
-                bool seen = false;
-                for (uint32_t k = 0; k < o.nmatch; k++) seen |= o.ids[k] == id;
-                if (!seen) {
-                    if (o.nmatch < DPI_LIST) o.ids[o.nmatch++] = (uint16_t)id;
-                    else o.ovf = true;
-                }
-            }
+        s = dfa_step(c, s, f[i], acc);
+        if (!acc) continue;
+        const uint32_t e = __ldg(c.out_off + s + 1);
+        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+            const uint32_t id = __ldg(c.out_ids + x);
+            drop |= __ldg(c.pat_action + id);
+            bool seen = false;
+            for (uint32_t k = 0; k < n; k++) seen |= ids[k] == id;
+            if (seen) continue;
+            if (n == DPI_LIST) { ovf = true; break; }
+            ids[n++] = (uint16_t)id;
         }
-    });
-}
-
-// exact distinct set with a per-thread bitmap (rare path), emitting pairs directly
-__device__ uint32_t dpi_bitmap_pass(const DpiImg &d, const uint8_t *cls, const uint8_t *f, const PV &v,
-                                    uint32_t gtid, const KParams &P, uint32_t pkt_id)
-{
-    uint32_t *bm = d.ovf_bitmap + (size_t)gtid * d.bitmap_words;
-    for (uint32_t k = 0; k < d.bitmap_words; k++) bm[k] = 0;
-    uint32_t s = 0, cnt = 0;
-    dpi_scan(f, v.pl_off, v.ip_end, [&](uint32_t byte) {
+    }
+    if (!ovf) {
+        if (n) {
+            const uint32_t slot = atomicAdd(o.match_count, n);
+            for (uint32_t q = 0; q < n; q++)
+                if (slot + q < o.match_cap) { o.match_pkt[slot + q] = pkt_id; o.match_pat[slot + q] = ids[q]; }
+            if (slot + n > o.match_cap)
+                atomicAdd(&o.stats[ST_MATCH_OVF], (unsigned long long)(slot + n - max(slot, o.match_cap)));
+        }
+        return n | drop << 31;
+    }
+    // more than DPI_LIST distinct ids: exact bitmap pass
+    atomicAdd(&o.stats[ST_DPI_OVF_PKTS], 1ull);
+    uint32_t *bm = o.bitmap + (size_t)gtid * o.words;
+    for (uint32_t k = 0; k < o.words; k++) bm[k] = 0;
+    uint32_t cnt = 0;
+    s = 0;
+    drop = 0;
+    for (uint32_t i = a; i < b; i++) {
         bool acc;
-        s = dfa_step(d, cls, s, byte, acc);
-        if (acc) {
-            uint32_t e = __ldg(d.out_off + s + 1);
-            for (uint32_t x = __ldg(d.out_off + s); x < e; x++) {
-                uint32_t id = __ldg(d.out_ids + x);
-                uint32_t bit = 1u << (id & 31);
-                if (!(bm[id >> 5] & bit)) {
-                    bm[id >> 5] |= bit;
-                    cnt++;
-                    uint32_t slot = atomicAdd(P.match_count, 1u);
-                    if (slot < P.match_cap) { P.match_pkt[slot] = pkt_id; P.match_pat[slot] = (uint16_t)id; }
-                    else atomicAdd(&P.stats[ST_MATCH_OVF], 1ull);
-                }
-            }
+        s = dfa_step(c, s, f[i], acc);
+        if (!acc) continue;
+        const uint32_t e = __ldg(c.out_off + s + 1);
+        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+            const uint32_t id = __ldg(c.out_ids + x);
+            drop |= __ldg(c.pat_action + id);
+            const uint32_t bit = 1u << (id & 31);
+            if (bm[id >> 5] & bit) continue;
+            bm[id >> 5] |= bit;
+            cnt++;
+            const uint32_t slot = atomicAdd(o.match_count, 1u);
+            if (slot < o.match_cap) { o.match_pkt[slot] = pkt_id; o.match_pat[slot] = (uint16_t)id; }
+            else atomicAdd(&o.stats[ST_MATCH_OVF], 1ull);
         }
-    });
-    return cnt;
+    }
+    return cnt | drop << 31;
 }
 
 // ---------------------------------------------------------------- LPM
-__device__ __forceinline__ uint32_t lpm4_lookup(const Lpm4Img &t, uint32_t dst)
+// DIR-24-8: at most two dependent table reads ("two memory accesses")
+__device__ __forceinline__ uint32_t lpm4_lookup(const Lpm4Img &t, uint32_t dst, uint64_t pol)
 {
-    uint32_t e = __ldg(t.tbl24 + (dst >> 8));
-    if (e & 0x8000) e = __ldg(t.tbllong + ((e & 0x7FFF) << 8) + (dst & 0xFF));
+    uint32_t e = ld_tab16(t.tbl24 + (dst >> 8), pol);
+    if (e & 0x8000) e = ld_tab16(t.tbllong + ((e & 0x7FFF) << 8) + (dst & 0xFF), pol);
     return e;
 }
 
-__device__ uint32_t lpm6_lookup(const Lpm6Img &t, const uint32_t dst[4])
+__device__ __forceinline__ uint32_t lpm6_lookup(const Lpm6Img &t, const uint32_t dst[4])
 {
     uint32_t best = t.def_nh;
     int lo = 0, hi = (int)t.n_levels - 1;
@@ -315,7 +415,7 @@ __device__ uint32_t lpm6_lookup(const Lpm6Img &t, const uint32_t dst[4])
 // L2/L3 rewrite after an LPM hit (R#6): dst MAC = nh MAC, src MAC = port MAC,
 // TTL / hop limit - 1, IPv4 header checksum recomputed (RFC 1071, byte-order independent
 // sum over little-endian halves).  Writes the first 32 B of the frame.
-__device__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm)
+__device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm, uint64_t pol)
 {
     h[0] = nh.x;
     h[1] = (nh.y & 0xFFFF) | (pm.x << 16);
@@ -327,12 +427,10 @@ __device__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 n
         if (v.l4_off == 34) {
             sum = (h[3] >> 16) + (h[4] & 0xFFFF) + (h[4] >> 16) + (h[5] & 0xFFFF) + (h[5] >> 16) +
                   (h[6] >> 16) + (h[7] & 0xFFFF) + (h[7] >> 16) + (h[8] & 0xFFFF);
-        } else {                              // IPv4 options: header beyond the cache
-            sum = (h[3] >> 16);
-            for (uint32_t k = 16; k < v.l4_off; k += 2) {
-                uint32_t lo = dbyte(h, f, k), hi = dbyte(h, f, k + 1);
-                if (k != 24) sum += lo | hi << 8;
-            }
+        } else {                              // IPv4 options (rare): bytes >= 32 from memory
+            sum = (h[3] >> 16) + (h[4] & 0xFFFF) + (h[4] >> 16) + (h[5] & 0xFFFF) + (h[5] >> 16) +
+                  (h[6] >> 16) + (h[7] & 0xFFFF) + (h[7] >> 16);
+            for (uint32_t k = 32; k < v.l4_off; k += 2) sum += (uint32_t)f[k] | (uint32_t)f[k + 1] << 8;
         }
         sum = (sum & 0xFFFF) + (sum >> 16);
         sum = (sum & 0xFFFF) + (sum >> 16);
@@ -340,9 +438,8 @@ __device__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 n
     } else {
         h[5] -= 1u << 8;                      // hop limit: byte 21
     }
-    uint4 *q = reinterpret_cast<uint4 *>(f);
-    q[0] = make_uint4(h[0], h[1], h[2], h[3]);
-    q[1] = make_uint4(h[4], h[5], h[6], h[7]);
+    st_stream16(f, make_uint4(h[0], h[1], h[2], h[3]), pol);
+    st_stream16(f + 16, make_uint4(h[4], h[5], h[6], h[7]), pol);
 }
 
 // ---------------------------------------------------------------- Toeplitz flow hash
@@ -542,270 +639,340 @@ __device__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t s
 }
 
 // ---------------------------------------------------------------- the kernel
+struct Pkt {
+    uint8_t *f;
+    uint32_t flen, orig_len;
+    uint64_t gidx;
+    uint32_t h[16];
+    PV v;
+    uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
+    bool alive;
+};
+
+struct Ctx {
+    const uint32_t *acl4, *acl6;
+    DpiCtx dpi;
+    const uint32_t *te, *ms_nib, *lb_nib;
+    uint32_t *vst;            // smem u32 hit counters (nullptr: global atomics)
+    uint64_t pol_f, pol_l;
+    uint32_t gtid;
+};
+
+__device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_t idx)
+{
+    if (C.vst) atomicAdd(&C.vst[idx - NFIX], 1u);
+    else atomicAdd(&P.stats[idx], 1ull);
+}
+
+__device__ __forceinline__ void pkt_begin(const KParams &P, const Ctx &C, uint32_t g, bool valid, Pkt &k)
+{
+    k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.flen = 0; k.orig_len = 0;
+    k.f = nullptr; k.gidx = 0;
+    if (!valid) return;
+    uint32_t bi = 0;
+    if (P.n_batches > 1) {
+        uint32_t lo = 0, hi = P.n_batches - 1;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi + 1) >> 1;
+            if (P.batches[mid].start <= g) lo = mid; else hi = mid - 1;
+        }
+        bi = lo;
+    }
+    const BatchDev &B = P.batches[bi];
+    const uint32_t li = g - B.start;
+    k.f = B.arena + B.off[li];
+    k.flen = k.orig_len = B.len[li];
+    k.gidx = B.first + li;
+    load_header(k.f, k.flen, k.h, C.pol_f);
+    k.alive = parse(k.h, k.f, k.flen, k.v);
+    if (!k.alive) k.drop = 0xFE;
+    k.out_len = k.flen;
+}
+
 template <uint32_t MASK>
-__global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 1 : 2) sfc_kernel(const KParams P)
+__device__ __forceinline__ void run_nf(const KParams &P, const Ctx &C, Pkt &k, uint32_t pos)
+{
+    const uint32_t kind = P.kind[pos];
+    bool dropped = false;
+    if ((MASK & MASK_ACL) && kind == NFC_ACL) {
+        const uint32_t r = nf_acl(k.v.fam == 4 ? C.acl4 : C.acl6, P.acl.default_action, k.v);
+        const uint32_t rule = r & 0xFFFF;
+        k.acl_rule = rule;
+        var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
+        dropped = (r >> 31) != 0;
+    } else if ((MASK & MASK_DPI) && kind == NFC_DPI) {
+        uint32_t s = 0;
+        bool any = false;
+        dpi_walk(k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, [&](uint32_t byte) {
+            bool acc;
+            s = dfa_step(C.dpi, s, byte, acc);
+            any |= acc;
+        });
+        if (any) {
+            const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
+                            P.match_cap, P.stats};
+            const uint32_t r = dpi_slow(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+            k.nmatch = r & 0x7FFFFFFFu;
+            dropped = (r >> 31) != 0;
+        }
+    } else if ((MASK & MASK_LPM4) && kind == NFC_LPM4) {
+        if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
+        const uint32_t nh = lpm4_lookup(P.l4, k.v.dst[0], C.pol_l);
+        if (nh == 0x7FFF || hbyte(k.h, 22) <= 1) dropped = true;
+        else {
+            const uint2 n = __ldg(P.l4.nh + nh);
+            const uint32_t pt = n.y >> 16;
+            forward_rewrite(k.f, k.h, k.v, n, __ldg(P.l4.pmac + pt), C.pol_f);
+            k.port = pt;
+        }
+    } else if ((MASK & MASK_LPM6) && kind == NFC_LPM6) {
+        if (k.v.fam != 6) { k.passmask |= 1u << pos; return; }
+        const uint32_t nh = lpm6_lookup(P.l6, k.v.dst);
+        if (nh == 0x7FFF || hbyte(k.h, 21) <= 1) dropped = true;
+        else {
+            const uint2 n = __ldg(P.l6.nh + nh);
+            const uint32_t pt = n.y >> 16;
+            forward_rewrite(k.f, k.h, k.v, n, __ldg(P.l6.pmac + pt), C.pol_f);
+            k.port = pt;
+        }
+    } else if ((MASK & MASK_IPSEC) && kind == NFC_IPSEC) {
+        const uint32_t nl = nf_esp(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te);
+        k.esp_bytes = nl - 28 - k.v.l4_off;      // ciphertext bytes |C|
+        k.f -= 16;
+        k.flen = nl;
+        k.out_len = nl;
+        load_header(k.f, k.flen, k.h, C.pol_f);
+        parse(k.h, k.f, k.flen, k.v);             // later NFs see proto 50, ports 0
+    } else if ((MASK & MASK_LB) && kind == NFC_LB) {
+        const uint32_t hsh = toeplitz(C.lb_nib, k.v);
+        const uint32_t b = (uint32_t)(((uint64_t)hsh * P.lb.n_backends) >> 32);
+        k.lb_b = b;
+        k.port = __ldg(P.lb.port + b);
+        var_stat(P, C, P.st_lb + b);
+    }
+    if (dropped) { k.drop = pos; k.alive = false; }
+}
+
+// record store + counters of one warp's 32 packets into the warp's private slot
+__device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, bool valid, uint32_t g,
+                                        unsigned long long *ws, uint32_t lane)
+{
+    if (valid) {
+        if (k.drop != 0xFF) k.port = 0xFFFF;
+        const uint4 rec = make_uint4(k.drop | k.esp_sa << 8 | k.port << 16, k.acl_rule | k.lb_b << 16,
+                                     k.nmatch | k.out_len << 16, k.esp_seq);
+        st_stream16(reinterpret_cast<uint4 *>(P.rec) + g, rec, C.pol_f);
+    }
+    const uint32_t FULL = 0xFFFFFFFFu;
+    const bool esp = k.esp_sa != 0xFF;
+    const uint32_t nv = __popc(__ballot_sync(FULL, valid));
+    const uint32_t nparse = __popc(__ballot_sync(FULL, valid && k.drop == 0xFE));
+    const uint32_t nfwd = __popc(__ballot_sync(FULL, valid && k.drop == 0xFF));
+    const uint32_t bin = __reduce_add_sync(FULL, k.orig_len);
+    const uint32_t bout = __reduce_add_sync(FULL, (valid && k.drop == 0xFF) ? k.out_len : 0u);
+    const uint32_t pairs = __reduce_add_sync(FULL, k.nmatch);
+    const uint32_t nesp = __popc(__ballot_sync(FULL, esp));
+    const uint32_t eb = __reduce_add_sync(FULL, esp ? k.esp_bytes : 0u);
+    const uint32_t eblk = __reduce_add_sync(FULL, esp ? (k.esp_bytes + 15) >> 4 : 0u);
+    uint32_t pc[NFC_MAX_CHAIN][3];
+#pragma unroll
+    for (int p = 0; p < NFC_MAX_CHAIN; p++) {
+        const bool reached = valid && k.drop != 0xFE && (k.drop == 0xFF || k.drop >= (uint32_t)p);
+        pc[p][0] = __popc(__ballot_sync(FULL, reached));
+        pc[p][1] = __popc(__ballot_sync(FULL, valid && k.drop == (uint32_t)p));
+        pc[p][2] = __popc(__ballot_sync(FULL, reached && ((k.passmask >> p) & 1)));
+    }
+    if (lane == 0 && nv) {
+        ws[ST_PKTS] += nv;
+        ws[ST_FWD] += nfwd;
+        ws[ST_DROP] += nv - nfwd;
+        ws[ST_PARSE_DROP] += nparse;
+        ws[ST_BYTES_IN] += bin;
+        ws[ST_BYTES_OUT] += bout;
+        ws[ST_DPI_PAIRS] += pairs;
+        ws[ST_ESP_PKTS] += nesp;
+        ws[ST_ESP_BYTES] += eb;
+        ws[ST_ESP_BLOCKS] += eblk;
+#pragma unroll
+        for (int p = 0; p < NFC_MAX_CHAIN; p++) {
+            if ((uint32_t)p >= P.n_nf) break;
+            ws[ST_POS_BASE + 4 * p] += pc[p][0];
+            ws[ST_POS_BASE + 4 * p + 1] += pc[p][1];
+            ws[ST_POS_BASE + 4 * p + 2] += pc[p][2];
+            ws[ST_POS_BASE + 4 * p + 3] += pc[p][0] - pc[p][1] - pc[p][2];
+        }
+    }
+}
+
+// ESP sequence numbers for one CTA tile: per SA, global packet order (decoupled look-back)
+__device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8_t *smem, const SmemLayout &L, uint32_t tile,
+                           Pkt &k)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t nsa = P.esp.n_sa;
+    uint16_t *wcnt = reinterpret_cast<uint16_t *>(smem + L.wcnt);
+    uint32_t *pref = reinterpret_cast<uint32_t *>(smem + L.prefix);
+    for (uint32_t i = tid; i < NWARP * 256; i += TILE) wcnt[i] = 0;
+    uint32_t sa = 0xFFFF;
+    if (k.alive) sa = toeplitz(C.ms_nib, k.v) % nsa;
+    __syncthreads();
+    const uint32_t key = k.alive ? sa : (0x10000u + lane);
+    const uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
+    const uint32_t rank = __popc(grp & ((1u << lane) - 1));
+    if (k.alive && rank == 0) wcnt[warp * 256 + sa] = (uint16_t)__popc(grp);
+    __syncthreads();
+    if (warp == 0) {
+        uint32_t *vec = P.tile_vec + (size_t)tile * 2 * nsa;
+        for (uint32_t s = lane; s < nsa; s += 32) {
+            uint32_t run = 0;
+#pragma unroll
+            for (int w = 0; w < NWARP; w++) { const uint32_t c = wcnt[w * 256 + s]; wcnt[w * 256 + s] = (uint16_t)run; run += c; }
+            vec[s] = run;
+            pref[s] = 0;
+        }
+        __syncwarp();
+        if (tile > 0) {
+            if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 1u); }
+            int pt = (int)tile - 1;
+            for (;;) {
+                uint32_t fl;
+                do { fl = ld_acquire(P.tile_flag + pt); } while ((fl >> 2) != P.epoch || (fl & 3) == 0);
+                const uint32_t *pv = P.tile_vec + (size_t)pt * 2 * nsa;
+                const bool incl = (fl & 3) == 2;
+                for (uint32_t s = lane; s < nsa; s += 32) pref[s] += __ldcg(pv + (incl ? nsa : 0) + s);
+                if (incl) break;
+                pt--;
+            }
+        }
+        __syncwarp();
+        for (uint32_t s = lane; s < nsa; s += 32) vec[nsa + s] = pref[s] + vec[s];
+        __syncwarp();
+        if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 2u); }
+        if (tile == P.n_tiles - 1)
+            for (uint32_t s = lane; s < nsa; s += 32) P.seq_out[s] = P.seq_in[s] + pref[s] + vec[s];
+    }
+    __syncthreads();
+    if (k.alive) {
+        k.esp_sa = sa;
+        k.esp_seq = __ldg(P.seq_in + sa) + pref[sa] + wcnt[warp * 256 + sa] + rank + 1;
+        var_stat(P, C, P.st_sa + sa);
+    }
+}
+
+template <uint32_t MASK>
+__global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(const KParams P)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t s_tile;
     const SmemLayout L = smem_layout(MASK, P);
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t gtid = blockIdx.x * TILE + tid;
-    unsigned long long *sst = reinterpret_cast<unsigned long long *>(smem + L.stats);
-    const uint32_t n_sst = P.smem_stats ? P.stats_len : ST_VAR_BASE;
-    for (uint32_t i = tid; i < n_sst; i += TILE) sst[i] = 0;
-    uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te);
-    uint32_t *ms_nib = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
-    uint32_t *lb_nib = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
-    uint8_t *cls = smem + L.cls;
+    unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
+    uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
+    const uint32_t n_var = P.stats_len - NFIX;
+    for (uint32_t i = tid; i < NWARP * NFIX; i += TILE) wst[i] = 0;
+    if (P.smem_stats)
+        for (uint32_t i = tid; i < n_var; i += TILE) vst[i] = 0;
+
+    Ctx C;
+    C.gtid = blockIdx.x * TILE + tid;
+    C.vst = P.smem_stats ? vst : nullptr;
+    C.pol_f = pol_first();
+    C.pol_l = pol_last();
+    C.acl4 = C.acl6 = nullptr;
+    C.te = C.ms_nib = C.lb_nib = nullptr;
+    C.dpi.cls = smem + L.cls;
+    C.dpi.ncls = P.dpi.ncls;
+    C.dpi.wide = P.dpi.wide;
+    C.dpi.trans = P.dpi.trans;
+    C.dpi.out_off = P.dpi.out_off;
+    C.dpi.out_ids = P.dpi.out_ids;
+    C.dpi.pat_action = P.dpi.pat_action;
+    C.dpi.hot = reinterpret_cast<const uint16_t *>(smem + L.hot);
+    C.dpi.H = 0;
     // NFs compiled into this variant but absent from the chain are skipped at run time
     const bool has_esp = (MASK & MASK_IPSEC) && P.esp_pos < P.n_nf;
-    if ((MASK & MASK_IPSEC) && has_esp) {
-        for (uint32_t i = tid; i < 5 * 256; i += TILE) te[i] = __ldg(P.esp.te + i);
-        for (uint32_t i = tid; i < 72 * 16; i += TILE) ms_nib[i] = __ldg(P.esp.rss_nib + i);
+    if ((MASK & MASK_ACL) && (P.present & MASK_ACL)) {
+        if (P.acl.smem_words) {
+            uint4 *d4 = reinterpret_cast<uint4 *>(smem + L.acl4);
+            uint4 *d6 = reinterpret_cast<uint4 *>(smem + L.acl6);
+            for (uint32_t i = tid; i < P.acl.words4 / 4; i += TILE) d4[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv4) + i);
+            for (uint32_t i = tid; i < P.acl.words6 / 4; i += TILE) d6[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv6) + i);
+            C.acl4 = reinterpret_cast<const uint32_t *>(d4);
+            C.acl6 = reinterpret_cast<const uint32_t *>(d6);
+        } else {
+            C.acl4 = P.acl.bv4;
+            C.acl6 = P.acl.bv6;
+        }
     }
-    if ((MASK & MASK_LB) && (P.present & MASK_LB))
-        for (uint32_t i = tid; i < 72 * 16; i += TILE) lb_nib[i] = __ldg(P.lb.nib + i);
-    if ((MASK & MASK_DPI) && (P.present & MASK_DPI))
+    if ((MASK & MASK_DPI) && (P.present & MASK_DPI)) {
+        uint8_t *cls = smem + L.cls;
         for (uint32_t i = tid; i < 256; i += TILE) cls[i] = __ldg(P.dpi.cls + i);
-    // variable stats live in smem or go straight to global memory
-    auto stat_add = [&](uint32_t idx, unsigned long long v) {
-        if (P.smem_stats) atomicAdd(&sst[idx], v);
-        else atomicAdd(&P.stats[idx], v);
-    };
+        const uint32_t H = P.dpi.wide ? 0 : P.dpi.hot_states;
+        uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
+        const uint16_t *tr = reinterpret_cast<const uint16_t *>(P.dpi.trans);
+        for (uint32_t i = tid; i < H * 256; i += TILE) hot[i] = __ldg(tr + (i >> 8) * P.dpi.ncls + __ldg(P.dpi.cls + (i & 255)));
+        C.dpi.H = H;
+    }
+    if ((MASK & MASK_IPSEC) && has_esp) {
+        uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
+        for (uint32_t i = tid; i < 5 * 256; i += TILE) te[i] = __ldg(P.esp.te + i);
+        for (uint32_t i = tid; i < 72 * 16; i += TILE) mn[i] = __ldg(P.esp.rss_nib + i);
+        C.te = te;
+        C.ms_nib = mn;
+    }
+    if ((MASK & MASK_LB) && (P.present & MASK_LB)) {
+        uint32_t *ln = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
+        for (uint32_t i = tid; i < 72 * 16; i += TILE) ln[i] = __ldg(P.lb.nib + i);
+        C.lb_nib = ln;
+    }
     __syncthreads();
+    unsigned long long *ws = wst + warp * NFIX;
 
-    for (;;) {
-        if (tid == 0) s_tile = atomicAdd(P.tile_counter, 1u);
-        __syncthreads();
-        const uint32_t tile = s_tile;
-        __syncthreads();
-        if (tile >= P.n_tiles) break;
-        const uint32_t g = tile * TILE + tid;
-        const bool valid = g < P.n_pkts;
-        // ---- locate the packet
-        uint32_t bi = 0;
-        if (P.n_batches > 1 && valid) {
-            uint32_t lo = 0, hi = P.n_batches - 1;
-            while (lo < hi) {
-                uint32_t mid = (lo + hi + 1) >> 1;
-                if (P.batches[mid].start <= g) lo = mid; else hi = mid - 1;
-            }
-            bi = lo;
+    if (!has_esp) {
+        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA barriers
+        for (;;) {
+            uint32_t base = 0;
+            if (lane == 0) base = atomicAdd(P.tile_counter, 32u);
+            base = __shfl_sync(0xFFFFFFFFu, base, 0);
+            if (base >= P.n_pkts) break;
+            const uint32_t g = base + lane;
+            const bool valid = g < P.n_pkts;
+            Pkt k;
+            pkt_begin(P, C, g, valid, k);
+            for (uint32_t pos = 0; pos < P.n_nf && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
+            pkt_end(P, C, k, valid, g, ws, lane);
         }
-        uint8_t *f = nullptr;
-        uint32_t flen = 0;
-        uint64_t gidx = 0;
-        if (valid) {
-            const BatchDev &B = P.batches[bi];
-            uint32_t li = g - B.start;
-            f = B.arena + B.off[li];
-            flen = B.len[li];
-            gidx = B.first + li;
-        }
-        // ---- per-packet state
-        uint32_t h[16];
-        PV v{};
-        uint32_t drop = 0xFF, esp_sa = 0xFF, port = 0, acl_rule = 0xFFFF, lb_b = 0xFFFF, nmatch = 0, esp_seq = 0;
-        uint32_t passmask = 0, esp_bytes = 0;
-        bool ok = false;
-        if (valid) {
-            load_header(f, flen, h);
-            ok = parse(h, f, flen, v);
-            if (!ok) drop = 0xFE;
-        }
-        bool alive = ok;
-        uint32_t out_len = flen;
-
-        auto run_nf = [&](uint32_t pos) {
-            const uint32_t kind = P.kind[pos];
-            bool dropped = false;
-            if ((MASK & MASK_ACL) && kind == NFC_ACL) {
-                uint32_t r = nf_acl(P.acl, v);
-                uint32_t rule = r & 0xFFFF;
-                acl_rule = rule;
-                stat_add(P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule), 1ull);
-                dropped = (r >> 31) != 0;
-            } else if ((MASK & MASK_DPI) && kind == NFC_DPI) {
-                DpiOut o;
-                nf_dpi(P.dpi, cls, f, v, gtid, o);
-                const uint32_t pkt_id = (uint32_t)gidx;
-                if (!o.ovf) {
-                    nmatch = o.nmatch;
-                    if (o.nmatch) {
-                        uint32_t slot = atomicAdd(P.match_count, o.nmatch);
-                        for (uint32_t k = 0; k < o.nmatch; k++)
-                            if (slot + k < P.match_cap) { P.match_pkt[slot + k] = pkt_id; P.match_pat[slot + k] = o.ids[k]; }
-                        if (slot + o.nmatch > P.match_cap)
-                            stat_add(ST_MATCH_OVF, (unsigned long long)(slot + o.nmatch - max(slot, P.match_cap)));
-                    }
-                } else {
-                    nmatch = dpi_bitmap_pass(P.dpi, cls, f, v, gtid, P, pkt_id);
-                    stat_add(ST_DPI_OVF_PKTS, 1ull);
-                }
-                dropped = o.drop;
-            } else if ((MASK & MASK_LPM4) && kind == NFC_LPM4) {
-                if (v.fam != 4) { passmask |= 1u << pos; return; }
-                uint32_t nh = lpm4_lookup(P.l4, v.dst[0]);
-                uint32_t ttl = hbyte(h, 22);
-                if (nh == 0x7FFF || ttl <= 1) { dropped = true; }
-                else {
-                    uint2 n = __ldg(P.l4.nh + nh);
-                    uint32_t pt = n.y >> 16;
-                    forward_rewrite(f, h, v, n, __ldg(P.l4.pmac + pt));
-                    port = pt;
-                }
-            } else if ((MASK & MASK_LPM6) && kind == NFC_LPM6) {
-                if (v.fam != 6) { passmask |= 1u << pos; return; }
-                uint32_t nh = lpm6_lookup(P.l6, v.dst);
-                uint32_t hl = hbyte(h, 21);
-                if (nh == 0x7FFF || hl <= 1) { dropped = true; }
-                else {
-                    uint2 n = __ldg(P.l6.nh + nh);
-                    uint32_t pt = n.y >> 16;
-                    forward_rewrite(f, h, v, n, __ldg(P.l6.pmac + pt));
-                    port = pt;
-                }
-            } else if ((MASK & MASK_IPSEC) && kind == NFC_IPSEC) {
-                uint32_t nl = nf_esp(f, v, P.esp.sa + esp_sa, esp_seq, te);
-                esp_bytes = nl - 28 - v.l4_off;          // == clen (ciphertext bytes)
-                f -= 16;
-                flen = nl;
-                out_len = nl;
-                load_header(f, flen, h);
-                parse(h, f, flen, v);                    // later NFs see proto 50, ports 0
-            } else if ((MASK & MASK_LB) && kind == NFC_LB) {
-                uint32_t hsh = toeplitz(lb_nib, v);
-                uint32_t b = (uint32_t)(((uint64_t)hsh * P.lb.n_backends) >> 32);
-                lb_b = b;
-                port = __ldg(P.lb.port + b);
-                stat_add(P.st_lb + b, 1ull);
-            }
-            if (dropped) { drop = pos; alive = false; }
-        };
-
-        const uint32_t n_pre = has_esp ? P.esp_pos : P.n_nf;
-        for (uint32_t pos = 0; pos < n_pre && alive; pos++) run_nf(pos);
-
-        if ((MASK & MASK_IPSEC) && has_esp) {   // uniform across the CTA
-            // ---- ESP sequence numbers: per SA, global packet order (decoupled look-back)
-            const uint32_t nsa = P.esp.n_sa;
-            uint16_t *wcnt = reinterpret_cast<uint16_t *>(smem + L.wcnt);
-            uint32_t *pref = reinterpret_cast<uint32_t *>(smem + L.prefix);
-            for (uint32_t i = tid; i < NWARP * 256; i += TILE) wcnt[i] = 0;
-            uint32_t sa = 0xFFFF;
-            if (alive) sa = toeplitz(ms_nib, v) % nsa;
+    } else if constexpr ((MASK & MASK_IPSEC) != 0) {
+        // CTA tiles claimed in global order (ESP sequence numbers need the order)
+        for (;;) {
+            if (tid == 0) s_tile = atomicAdd(P.tile_counter, 1u);
             __syncthreads();
-            const uint32_t key = alive ? sa : (0x10000u + lane);
-            const uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
-            const uint32_t rank = __popc(grp & ((1u << lane) - 1));
-            if (alive && rank == 0) wcnt[warp * 256 + sa] = (uint16_t)__popc(grp);
+            const uint32_t tile = s_tile;
             __syncthreads();
-            if (warp == 0) {
-                uint32_t *vec = P.tile_vec + (size_t)tile * 2 * nsa;
-                for (uint32_t s = lane; s < nsa; s += 32) {
-                    uint32_t run = 0;
-#pragma unroll
-                    for (int w = 0; w < NWARP; w++) { uint32_t c = wcnt[w * 256 + s]; wcnt[w * 256 + s] = (uint16_t)run; run += c; }
-                    vec[s] = run;                                   // aggregate
-                    pref[s] = 0;
-                }
-                __syncwarp();
-                if (tile > 0) {
-                    if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 1u); }
-                    int pt = (int)tile - 1;
-                    for (;;) {
-                        uint32_t fl;
-                        do { fl = ld_acquire(P.tile_flag + pt); } while ((fl >> 2) != P.epoch || (fl & 3) == 0);
-                        const uint32_t *pv = P.tile_vec + (size_t)pt * 2 * nsa;
-                        const bool incl = (fl & 3) == 2;
-                        for (uint32_t s = lane; s < nsa; s += 32) pref[s] += __ldcg(pv + (incl ? nsa : 0) + s);
-                        if (incl) break;
-                        pt--;
-                    }
-                }
-                __syncwarp();
-                for (uint32_t s = lane; s < nsa; s += 32) vec[nsa + s] = pref[s] + vec[s];
-                __syncwarp();
-                if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 2u); }
-                if (tile == P.n_tiles - 1)
-                    for (uint32_t s = lane; s < nsa; s += 32) P.seq_out[s] = P.seq_in[s] + pref[s] + vec[s];
-            }
-            __syncthreads();
-            if (alive) {
-                esp_sa = sa;
-                esp_seq = __ldg(P.seq_in + sa) + pref[sa] + wcnt[warp * 256 + sa] + rank + 1;
-                stat_add(P.st_sa + sa, 1ull);
-            }
-            for (uint32_t pos = P.esp_pos; pos < P.n_nf && alive; pos++) run_nf(pos);
-        }
-
-        // ---- result record + counters (warp-aggregated)
-        if (valid) {
-            if (drop != 0xFF) port = 0xFFFF;
-            uint4 rec;
-            rec.x = drop | esp_sa << 8 | port << 16;
-            rec.y = acl_rule | lb_b << 16;
-            rec.z = nmatch | out_len << 16;
-            rec.w = esp_seq;
-            reinterpret_cast<uint4 *>(P.rec)[g] = rec;
-        }
-        const uint32_t FULL = 0xFFFFFFFFu;
-        const uint32_t b_valid = __ballot_sync(FULL, valid);
-        const uint32_t b_parse = __ballot_sync(FULL, valid && drop == 0xFE);
-        const uint32_t b_fwd = __ballot_sync(FULL, valid && drop == 0xFF);
-        const uint32_t out_bytes = __reduce_add_sync(FULL, (valid && drop == 0xFF) ? out_len : 0u);
-        const uint32_t pairs = __reduce_add_sync(FULL, valid ? nmatch : 0u);
-        const uint32_t eb = __reduce_add_sync(FULL, esp_sa != 0xFF ? esp_bytes : 0u);
-        const uint32_t eblk = __reduce_add_sync(FULL, esp_sa != 0xFF ? (esp_bytes + 15) >> 4 : 0u);
-        const uint32_t ep = __ballot_sync(FULL, esp_sa != 0xFF);
-        uint32_t pos_cnt[NFC_MAX_CHAIN][3];
-#pragma unroll
-        for (int p = 0; p < NFC_MAX_CHAIN; p++) {
-            const bool reached = valid && drop != 0xFE && (drop == 0xFF || drop >= (uint32_t)p);
-            pos_cnt[p][0] = __popc(__ballot_sync(FULL, reached));
-            pos_cnt[p][1] = __popc(__ballot_sync(FULL, valid && drop == (uint32_t)p));
-            pos_cnt[p][2] = __popc(__ballot_sync(FULL, reached && ((passmask >> p) & 1)));
-        }
-        if (lane == 0) {
-            const uint32_t nv = __popc(b_valid);
-            if (nv) {
-                atomicAdd(&sst[ST_PKTS], (unsigned long long)nv);
-                atomicAdd(&sst[ST_FWD], (unsigned long long)__popc(b_fwd));
-                atomicAdd(&sst[ST_DROP], (unsigned long long)(nv - __popc(b_fwd)));
-                atomicAdd(&sst[ST_PARSE_DROP], (unsigned long long)__popc(b_parse));
-                atomicAdd(&sst[ST_BYTES_OUT], (unsigned long long)out_bytes);
-                atomicAdd(&sst[ST_DPI_PAIRS], (unsigned long long)pairs);
-                if (ep) {
-                    atomicAdd(&sst[ST_ESP_PKTS], (unsigned long long)__popc(ep));
-                    atomicAdd(&sst[ST_ESP_BYTES], (unsigned long long)eb);
-                    atomicAdd(&sst[ST_ESP_BLOCKS], (unsigned long long)eblk);
-                }
-                for (uint32_t p = 0; p < P.n_nf; p++) {
-                    const uint32_t base = ST_POS_BASE + 4 * p;
-                    atomicAdd(&sst[base], (unsigned long long)pos_cnt[p][0]);
-                    atomicAdd(&sst[base + 1], (unsigned long long)pos_cnt[p][1]);
-                    atomicAdd(&sst[base + 2], (unsigned long long)pos_cnt[p][2]);
-                    atomicAdd(&sst[base + 3], (unsigned long long)(pos_cnt[p][0] - pos_cnt[p][1] - pos_cnt[p][2]));
-                }
-            }
-        }
-        // bytes_in: original frame length (before ESP growth)
-        {
-            uint32_t orig = 0;
-            if (valid) {
-                const BatchDev &B = P.batches[bi];
-                orig = B.len[g - B.start];
-            }
-            const uint32_t bi_sum = __reduce_add_sync(FULL, orig);
-            if (lane == 0 && bi_sum) atomicAdd(&sst[ST_BYTES_IN], (unsigned long long)bi_sum);
+            if (tile >= P.n_tiles) break;
+            const uint32_t g = tile * TILE + tid;
+            const bool valid = g < P.n_pkts;
+            Pkt k;
+            pkt_begin(P, C, g, valid, k);
+            for (uint32_t pos = 0; pos < P.esp_pos && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
+            esp_assign(P, C, smem, L, tile, k);
+            for (uint32_t pos = P.esp_pos; pos < P.n_nf && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
+            pkt_end(P, C, k, valid, g, ws, lane);
         }
     }
     // ---- flush CTA counters
     __syncthreads();
-    for (uint32_t i = tid; i < n_sst; i += TILE)
-        if (sst[i]) atomicAdd(&P.stats[i], sst[i]);
+    for (uint32_t i = tid; i < NFIX; i += TILE) {
+        unsigned long long s = 0;
+#pragma unroll
+        for (int w = 0; w < NWARP; w++) s += wst[w * NFIX + i];
+        if (s) atomicAdd(&P.stats[i], s);
+    }
+    if (P.smem_stats)
+        for (uint32_t i = tid; i < n_var; i += TILE)
+            if (vst[i]) atomicAdd(&P.stats[NFIX + i], (unsigned long long)vst[i]);
 }
-
 
 // ---------------------------------------------------------------- host launch
 template <uint32_t M>
