@@ -128,7 +128,19 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
             for (uint64_t x : v) { blob.push_back((uint32_t)x); blob.push_back((uint32_t)(x >> 32)); }
             return o;
         };
-        uint32_t offs[10];
+        // 257-entry bucket index per field on the top 8 key bits: bucket[t] = interval
+        // containing the first key of bucket t; the search is confined to [bk[t], bk[t+1]]
+        auto put_buckets = [&](const FieldIv &f, int kbits) {
+            uint32_t o = (uint32_t)blob.size();
+            std::vector<uint32_t> bk(257);
+            for (int t = 0; t <= 256; t++) {
+                u128 first = t == 256 ? (kbits == 128 ? ~(u128)0 : (((u128)1 << kbits) - 1)) : (u128)t << (kbits - 8);
+                bk[t] = (uint32_t)(std::upper_bound(f.b.begin(), f.b.end(), first) - f.b.begin() - 1);
+            }
+            for (int t = 0; t < 257; t++) blob.push_back(bk[t]);
+            return o;
+        };
+        uint32_t offs[14];
         offs[0] = put_keys(F[0], kw); offs[1] = put_bv(F[0].bv);
         offs[2] = put_keys(F[1], kw); offs[3] = put_bv(F[1].bv);
         offs[4] = put_keys(F[2], 1);  offs[5] = put_bv(F[2].bv);
@@ -136,8 +148,12 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
         offs[8] = put_bv(vproto);
         offs[9] = (uint32_t)blob.size();
         for (uint32_t r = 0; r < n; r++) blob.push_back(gidx[r] | (uint32_t)s.rules[gidx[r]].action << 31);
+        offs[10] = put_buckets(F[0], bits);
+        offs[11] = put_buckets(F[1], bits);
+        offs[12] = put_buckets(F[2], 16);
+        offs[13] = put_buckets(F[3], 16);
         while (blob.size() & 3) blob.push_back(0);   // 16-B multiple for staging copies
-        for (int k = 0; k < 10; k++) blob[8 + k] = offs[k];
+        for (int k = 0; k < 14; k++) blob[8 + k] = offs[k];
     }
     return "";
 }

@@ -369,7 +369,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         }
         if ((c->mask & MASK_DPI) && !c->dpi.wide) {
             size_t base = sfc_smem_bytes(c->mask, p);
-            size_t h = base < budget ? (budget - base) / 512 : 0;
+            size_t h = base < budget ? (budget - base) / (2 * c->dpi.ncls + 1) : 0;
             p.dpi.hot_states = (uint32_t)std::min<size_t>(h, c->dpi.n_states);
         }
     }

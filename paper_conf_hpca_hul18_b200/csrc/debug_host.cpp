@@ -182,9 +182,17 @@ int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *
     int nb = family == 4 ? 1 : 4;
     for (int k = 0; k < nb; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
     const uint32_t W = A[1];
-    uint32_t js = nb == 1 ? bs32(A + A[8], A[2], s[0]) : bs128(A + A[8], A[2], s);
-    uint32_t jd = nb == 1 ? bs32(A + A[10], A[3], t[0]) : bs128(A + A[10], A[3], t);
-    uint32_t jsp = bs32(A + A[12], A[4], sport), jdp = bs32(A + A[14], A[5], dport);
+    auto iv32 = [&](uint32_t ok, uint32_t ob, uint32_t key, int kbits) {
+        uint32_t tb = key >> (kbits - 8), lo = A[ob + tb], hi = A[ob + tb + 1];
+        return lo + bs32(A + ok + lo, hi - lo + 1, key);
+    };
+    auto iv128 = [&](uint32_t ok, uint32_t ob, const uint32_t *k) {
+        uint32_t tb = k[0] >> 24, lo = A[ob + tb], hi = A[ob + tb + 1];
+        return lo + bs128(A + ok + 4 * lo, hi - lo + 1, k);
+    };
+    uint32_t js = nb == 1 ? iv32(A[8], A[18], s[0], 32) : iv128(A[8], A[18], s);
+    uint32_t jd = nb == 1 ? iv32(A[10], A[19], t[0], 32) : iv128(A[10], A[19], t);
+    uint32_t jsp = iv32(A[12], A[20], sport, 16), jdp = iv32(A[14], A[21], dport, 16);
     auto bv = [&](uint32_t off, uint32_t j, uint32_t w) {
         uint64_t x;
         memcpy(&x, A + off + 2 * ((size_t)j * W + w), 8);

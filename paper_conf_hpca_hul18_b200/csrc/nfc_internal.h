@@ -17,8 +17,10 @@ namespace nfc {
 //   [0] n rules of the family  [1] W = 64-bit words per bitset  [2..5] interval counts
 //   m_src, m_dst, m_sport, m_dport  [6] key words per address (1 v4, 4 v6)
 //   [8..17] word offsets: keys_src, bv_src, keys_dst, bv_dst, keys_sp, bv_sp, keys_dp, bv_dp,
-//   bv_proto (256 x W), ridx (global rule index | action << 31).  Bitsets are u64 at even offsets.
-static const uint32_t ACLBV_HDR = 20;
+//   bv_proto (256 x W), ridx (global rule index | action << 31),  [18..21] bucket tables
+//   (257 u32 per field) on the top 8 key bits.  Bitsets are u64 at
+//   even offsets.
+static const uint32_t ACLBV_HDR = 24;
 struct AclImg {
     const uint32_t *bv4, *bv6;        // device blobs
     uint32_t words4, words6;          // blob sizes (u32 words)

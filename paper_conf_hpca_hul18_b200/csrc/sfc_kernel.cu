@@ -41,7 +41,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, const KParams &
     o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 5 * 256 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
-    if (mask & MASK_DPI) { L.cls = o; o += 256; L.hot = o; o += p.dpi.hot_states * 256 * 2; }
+    if (mask & MASK_DPI) { L.cls = o; o += 256; L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u; }
     o = (o + 15) & ~15u;
     if (mask & MASK_ACL) {
         const uint32_t s4 = p.acl.smem_words ? p.acl.words4 : 0, s6 = p.acl.smem_words ? p.acl.words6 : 0;
@@ -219,6 +219,20 @@ __device__ __forceinline__ uint32_t bsearch128(const uint32_t *B, uint32_t m, co
     return lo;
 }
 
+// interval of key: bucket on the top 8 bits bounds the binary search to [bk[t], bk[t+1]]
+__device__ __forceinline__ uint32_t iv32(const uint32_t *A, uint32_t okeys, uint32_t obk, uint32_t key, int kbits)
+{
+    const uint32_t t = key >> (kbits - 8);
+    const uint32_t lo = A[obk + t], hi = A[obk + t + 1];
+    return lo + bsearch32(A + okeys + lo, hi - lo + 1, key);
+}
+__device__ __forceinline__ uint32_t iv128(const uint32_t *A, uint32_t okeys, uint32_t obk, const uint32_t k[4])
+{
+    const uint32_t t = k[0] >> 24;
+    const uint32_t lo = A[obk + t], hi = A[obk + t + 1];
+    return lo + bsearch128(A + okeys + 4 * lo, hi - lo + 1, k);
+}
+
 // returns global rule index (0xFFFF none) | action << 31
 __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A, uint32_t default_action, const PV &v)
 {
@@ -227,14 +241,14 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A, uint32_t default_a
     const uint32_t W = A[1];
     uint32_t js, jd;
     if (A[6] == 1) {
-        js = bsearch32(A + A[8], A[2], v.src[0]);
-        jd = bsearch32(A + A[10], A[3], v.dst[0]);
+        js = iv32(A, A[8], A[18], v.src[0], 32);
+        jd = iv32(A, A[10], A[19], v.dst[0], 32);
     } else {
-        js = bsearch128(A + A[8], A[2], v.src);
-        jd = bsearch128(A + A[10], A[3], v.dst);
+        js = iv128(A, A[8], A[18], v.src);
+        jd = iv128(A, A[10], A[19], v.dst);
     }
-    const uint32_t jsp = bsearch32(A + A[12], A[4], v.sport);
-    const uint32_t jdp = bsearch32(A + A[14], A[5], v.dport);
+    const uint32_t jsp = iv32(A, A[12], A[20], v.sport, 16);
+    const uint32_t jdp = iv32(A, A[14], A[21], v.dport, 16);
     const uint64_t *vs = reinterpret_cast<const uint64_t *>(A + A[9]) + (size_t)js * W;
     const uint64_t *vd = reinterpret_cast<const uint64_t *>(A + A[11]) + (size_t)jd * W;
     const uint64_t *vsp = reinterpret_cast<const uint64_t *>(A + A[13]) + (size_t)jsp * W;
@@ -253,52 +267,80 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A, uint32_t default_a
 struct DpiCtx {
     const uint8_t *cls;     // smem
     const uint16_t *hot;    // smem
-    uint32_t H, ncls, wide;
+    uint32_t H, ncls, wide, HK1;
     const void *trans;
     const uint32_t *out_off;
     const uint16_t *out_ids;
     const uint8_t *pat_action;
 };
 
+// One DFA step.  Hot rows (the first H states in BFS order, class-compressed) are
+// staged in shared memory with the same layout as the global table.
 __device__ __forceinline__ uint32_t dfa_step(const DpiCtx &c, uint32_t s, uint32_t b, bool &acc)
 {
-    uint32_t e;
-    if (s < c.H) {
-        e = c.hot[(s << 8) | b];
-        acc = e >> 15;
-        return e & 0x7FFFu;
-    }
     const uint32_t k = s * c.ncls + c.cls[b];
-    if (c.wide) { e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k); acc = e >> 31; return e & 0x7FFFFFFFu; }
-    e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
-    acc = e >> 15;
+    uint32_t e;
+    if (c.wide) {
+        e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k);
+        acc = e >> 31;
+        return e & 0x7FFFFFFFu;
+    }
+    e = s < c.H ? (uint32_t)c.hot[k] : (uint32_t)__ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
+    acc = (e >> 15) & 1;
     return e & 0x7FFFu;
 }
 
-// walk payload [a, b): bytes < 64 from the header cache, the rest from memory
-template <typename F>
-__device__ __forceinline__ void dpi_walk(const uint32_t h[16], const uint8_t *f, uint32_t a, uint32_t b, uint64_t pol,
-                                         F &&on_byte)
+// Fast DFA walk over payload [a, b) that only ORs the accept bits (exact match sets
+// are recomputed by dpi_slow for the rare packets that hit an accepting state).
+// Branch-free step: class lookup, hot-row lookup at a clamped index (shared memory),
+// predicated global load for cold states, predicated state update for bytes outside
+// the payload.  Bytes 32..63 come from the header cache (a payload never starts
+// before byte 34), the rest from memory in 16-B chunks.
+template <bool WIDE>
+__device__ __forceinline__ uint32_t dfa_byte(const DpiCtx &c, uint32_t s, uint32_t byte, uint32_t &any)
 {
-#pragma unroll
-    for (int c = 0; c < 64; c += 16) {
-        if ((uint32_t)c + 16 > a && (uint32_t)c < b) {
-#pragma unroll
-            for (int k = 0; k < 16; k++) {
-                const uint32_t idx = c + k;
-                if (idx >= a && idx < b) on_byte((h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF);
-            }
-        }
+    const uint32_t k = s * c.ncls + c.cls[byte];
+    uint32_t e;
+    if (WIDE) {
+        e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k);
+        any |= e >> 16;
+        return e & 0x7FFFFFFFu;
     }
-    for (uint32_t c = max(64u, a & ~15u); c < b; c += 16) {
-        const uint4 q = ld_stream16(f + c, pol);
+    e = c.hot[min(k, c.HK1)];
+    if (s >= c.H) e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
+    any |= e;
+    return e & 0x7FFFu;
+}
+
+template <bool WIDE>
+__device__ __forceinline__ bool dpi_fast(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
+                                         uint32_t b, uint64_t pol)
+{
+    uint32_t s = 0, any = 0;
+    const uint32_t n = b - a;
+#pragma unroll
+    for (int idx = 32; idx < 64; idx++) {
+        const uint32_t byte = (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF;
+        uint32_t an = 0;
+        const uint32_t ns = dfa_byte<WIDE>(c, s, byte, an);
+        const bool act = (uint32_t)idx - a < n;
+        s = act ? ns : s;
+        any |= act ? an : 0u;
+    }
+    for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
+        const uint4 q = ld_stream16(f + ch, pol);
         const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
         for (int k = 0; k < 16; k++) {
-            const uint32_t idx = c + k;
-            if (idx >= a && idx < b) on_byte((w[k >> 2] >> ((k & 3) * 8)) & 0xFF);
+            const uint32_t byte = (w[k >> 2] >> ((k & 3) * 8)) & 0xFF;
+            uint32_t an = 0;
+            const uint32_t ns = dfa_byte<WIDE>(c, s, byte, an);
+            const bool act = ch + k - a < n;
+            s = act ? ns : s;
+            any |= act ? an : 0u;
         }
     }
+    return (any >> 15) & 1;
 }
 
 // Exact match set of a packet whose walk hit an accepting state (rare path, not
@@ -320,9 +362,12 @@ __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a
     uint32_t n = 0, drop = 0;
     bool ovf = false;
     uint32_t s = 0;
+    uint4 q = make_uint4(0, 0, 0, 0);
     for (uint32_t i = a; i < b && !ovf; i++) {
+        if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
+        const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
         bool acc;
-        s = dfa_step(c, s, f[i], acc);
+        s = dfa_step(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
         const uint32_t e = __ldg(c.out_off + s + 1);
         for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
@@ -353,8 +398,10 @@ __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a
     s = 0;
     drop = 0;
     for (uint32_t i = a; i < b; i++) {
+        if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
+        const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
         bool acc;
-        s = dfa_step(c, s, f[i], acc);
+        s = dfa_step(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
         const uint32_t e = __ldg(c.out_off + s + 1);
         for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
@@ -702,13 +749,8 @@ __device__ __forceinline__ void run_nf(const KParams &P, const Ctx &C, Pkt &k, u
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
         dropped = (r >> 31) != 0;
     } else if ((MASK & MASK_DPI) && kind == NFC_DPI) {
-        uint32_t s = 0;
-        bool any = false;
-        dpi_walk(k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, [&](uint32_t byte) {
-            bool acc;
-            s = dfa_step(C.dpi, s, byte, acc);
-            any |= acc;
-        });
+        const bool any = C.dpi.wide ? dpi_fast<true>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f)
+                                    : dpi_fast<false>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
         if (any) {
             const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                             P.match_cap, P.stats};
@@ -890,6 +932,7 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(
     C.dpi.pat_action = P.dpi.pat_action;
     C.dpi.hot = reinterpret_cast<const uint16_t *>(smem + L.hot);
     C.dpi.H = 0;
+    C.dpi.HK1 = 0;
     // NFs compiled into this variant but absent from the chain are skipped at run time
     const bool has_esp = (MASK & MASK_IPSEC) && P.esp_pos < P.n_nf;
     if ((MASK & MASK_ACL) && (P.present & MASK_ACL)) {
@@ -911,8 +954,9 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(
         const uint32_t H = P.dpi.wide ? 0 : P.dpi.hot_states;
         uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
         const uint16_t *tr = reinterpret_cast<const uint16_t *>(P.dpi.trans);
-        for (uint32_t i = tid; i < H * 256; i += TILE) hot[i] = __ldg(tr + (i >> 8) * P.dpi.ncls + __ldg(P.dpi.cls + (i & 255)));
+        for (uint32_t i = tid; i < H * P.dpi.ncls; i += TILE) hot[i] = __ldg(tr + i);
         C.dpi.H = H;
+        C.dpi.HK1 = H ? H * P.dpi.ncls - 1 : 0;
     }
     if ((MASK & MASK_IPSEC) && has_esp) {
         uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
