@@ -297,35 +297,41 @@ __device__ __forceinline__ uint32_t dfa_step(const DpiCtx &c, uint32_t s, uint32
 // the payload.  Bytes 32..63 come from the header cache (a payload never starts
 // before byte 34), the rest from memory in 16-B chunks.
 template <bool WIDE>
-__device__ __forceinline__ uint32_t dfa_byte(const DpiCtx &c, uint32_t s, uint32_t byte, uint32_t &any)
+__device__ __forceinline__ uint32_t dfa_byte(const DpiCtx &c, uint32_t s, uint32_t byte, uint32_t &acc)
 {
     const uint32_t k = s * c.ncls + c.cls[byte];
     uint32_t e;
     if (WIDE) {
         e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k);
-        any |= e >> 16;
+        acc = e >> 31;
         return e & 0x7FFFFFFFu;
     }
     e = c.hot[min(k, c.HK1)];
     if (s >= c.H) e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
-    any |= e;
+    acc = (e >> 15) & 1;
     return e & 0x7FFFu;
 }
 
+// Returns the number of accept events; *first = state after the first one.  One
+// accept event (the common matching case) means the match set is exactly the
+// output closure of that state; more need the exact re-walk.
 template <bool WIDE>
-__device__ __forceinline__ bool dpi_fast(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
-                                         uint32_t b, uint64_t pol)
+__device__ __forceinline__ uint32_t dpi_fast(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
+                                             uint32_t b, uint64_t pol, uint32_t &first)
 {
-    uint32_t s = 0, any = 0;
+    uint32_t s = 0, cnt = 0;
+    first = 0;
     const uint32_t n = b - a;
 #pragma unroll
     for (int idx = 32; idx < 64; idx++) {
         const uint32_t byte = (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF;
-        uint32_t an = 0;
-        const uint32_t ns = dfa_byte<WIDE>(c, s, byte, an);
+        uint32_t acc;
+        const uint32_t ns = dfa_byte<WIDE>(c, s, byte, acc);
         const bool act = (uint32_t)idx - a < n;
         s = act ? ns : s;
-        any |= act ? an : 0u;
+        acc = act ? acc : 0u;
+        first = (acc && cnt == 0) ? ns : first;
+        cnt += acc;
     }
     for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
         const uint4 q = ld_stream16(f + ch, pol);
@@ -333,14 +339,16 @@ __device__ __forceinline__ bool dpi_fast(const DpiCtx &c, const uint32_t h[16], 
 #pragma unroll
         for (int k = 0; k < 16; k++) {
             const uint32_t byte = (w[k >> 2] >> ((k & 3) * 8)) & 0xFF;
-            uint32_t an = 0;
-            const uint32_t ns = dfa_byte<WIDE>(c, s, byte, an);
+            uint32_t acc;
+            const uint32_t ns = dfa_byte<WIDE>(c, s, byte, acc);
             const bool act = ch + k - a < n;
             s = act ? ns : s;
-            any |= act ? an : 0u;
+            acc = act ? acc : 0u;
+            first = (acc && cnt == 0) ? ns : first;
+            cnt += acc;
         }
     }
-    return (any >> 15) & 1;
+    return cnt;
 }
 
 // Exact match set of a packet whose walk hit an accepting state (rare path, not
@@ -711,12 +719,12 @@ __device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_
     else atomicAdd(&P.stats[idx], 1ull);
 }
 
-__device__ __forceinline__ void pkt_begin(const KParams &P, const Ctx &C, uint32_t g, bool valid, Pkt &k)
+struct Loc { uint8_t *f; uint32_t len; uint64_t gidx; };
+
+__device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
 {
-    k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
-    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.flen = 0; k.orig_len = 0;
-    k.f = nullptr; k.gidx = 0;
-    if (!valid) return;
+    Loc l{nullptr, 0, 0};
+    if (!valid) return l;
     uint32_t bi = 0;
     if (P.n_batches > 1) {
         uint32_t lo = 0, hi = P.n_batches - 1;
@@ -728,13 +736,22 @@ __device__ __forceinline__ void pkt_begin(const KParams &P, const Ctx &C, uint32
     }
     const BatchDev &B = P.batches[bi];
     const uint32_t li = g - B.start;
-    k.f = B.arena + B.off[li];
-    k.flen = k.orig_len = B.len[li];
-    k.gidx = B.first + li;
+    l.f = B.arena + B.off[li];
+    l.len = B.len[li];
+    l.gidx = B.first + li;
+    return l;
+}
+
+__device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid, Pkt &k)
+{
+    k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false;
+    k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
+    k.out_len = k.flen;
+    if (!valid) return;
     load_header(k.f, k.flen, k.h, C.pol_f);
     k.alive = parse(k.h, k.f, k.flen, k.v);
     if (!k.alive) k.drop = 0xFE;
-    k.out_len = k.flen;
 }
 
 template <uint32_t MASK>
@@ -749,9 +766,25 @@ __device__ __forceinline__ void run_nf(const KParams &P, const Ctx &C, Pkt &k, u
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
         dropped = (r >> 31) != 0;
     } else if ((MASK & MASK_DPI) && kind == NFC_DPI) {
-        const bool any = C.dpi.wide ? dpi_fast<true>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f)
-                                    : dpi_fast<false>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
-        if (any) {
+        uint32_t first;
+        const uint32_t cnt = C.dpi.wide ? dpi_fast<true>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, first)
+                                        : dpi_fast<false>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, first);
+        if (cnt == 1) {
+            // exactly one accept event: match set = output closure of that state (distinct, sorted)
+            const uint32_t o0 = __ldg(P.dpi.out_off + first), o1 = __ldg(P.dpi.out_off + first + 1);
+            const uint32_t nm = o1 - o0;
+            const uint32_t slot = atomicAdd(P.match_count, nm);
+            uint32_t drop = 0;
+            for (uint32_t q = 0; q < nm; q++) {
+                const uint32_t id = __ldg(P.dpi.out_ids + o0 + q);
+                drop |= __ldg(P.dpi.pat_action + id);
+                if (slot + q < P.match_cap) { P.match_pkt[slot + q] = (uint32_t)k.gidx; P.match_pat[slot + q] = (uint16_t)id; }
+            }
+            if (slot + nm > P.match_cap)
+                atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
+            k.nmatch = nm;
+            dropped = drop != 0;
+        } else if (cnt > 1) {
             const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                             P.match_cap, P.stats};
             const uint32_t r = dpi_slow(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
@@ -974,18 +1007,29 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(
     unsigned long long *ws = wst + warp * NFIX;
 
     if (!has_esp) {
-        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA barriers
-        for (;;) {
-            uint32_t base = 0;
-            if (lane == 0) base = atomicAdd(P.tile_counter, 32u);
-            base = __shfl_sync(0xFFFFFFFFu, base, 0);
-            if (base >= P.n_pkts) break;
+        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA
+        // barriers; the next chunk is claimed and located (off/len loads, L2 prefetch
+        // of its headers) before the current one is processed
+        auto claim = [&]() {
+            uint32_t b = 0;
+            if (lane == 0) b = atomicAdd(P.tile_counter, 32u);
+            return __shfl_sync(0xFFFFFFFFu, b, 0);
+        };
+        uint32_t base = claim();
+        Loc loc = pkt_locate(P, base + lane, base + lane < P.n_pkts);
+        while (base < P.n_pkts) {
+            const uint32_t nbase = claim();
+            const bool nvalid = nbase + lane < P.n_pkts;
+            const Loc nloc = pkt_locate(P, nbase + lane, nvalid);
+            if (nvalid) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(nloc.f));
             const uint32_t g = base + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;
-            pkt_begin(P, C, g, valid, k);
+            pkt_begin(C, loc, valid, k);
             for (uint32_t pos = 0; pos < P.n_nf && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
             pkt_end(P, C, k, valid, g, ws, lane);
+            base = nbase;
+            loc = nloc;
         }
     } else if constexpr ((MASK & MASK_IPSEC) != 0) {
         // CTA tiles claimed in global order (ESP sequence numbers need the order)
@@ -998,7 +1042,7 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(
             const uint32_t g = tile * TILE + tid;
             const bool valid = g < P.n_pkts;
             Pkt k;
-            pkt_begin(P, C, g, valid, k);
+            pkt_begin(C, pkt_locate(P, g, valid), valid, k);
             for (uint32_t pos = 0; pos < P.esp_pos && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
             esp_assign(P, C, smem, L, tile, k);
             for (uint32_t pos = P.esp_pos; pos < P.n_nf && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
