@@ -23,12 +23,14 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out=None) -> str:
+    """Build libnfc.so; `defines`/`out` build an experimental variant elsewhere."""
+    if out is None and not force and not _stale():
         return LIB
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
            "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"),
-           "-Xptxas", "-v" if verbose else "-O3", "-o", LIB + ".tmp",
+           *[f"-D{d}" for d in defines],
+           "-Xptxas", "-v" if verbose else "-O3", "-o", (out or LIB) + ".tmp",
            *[os.path.join(CSRC, s) for s in SOURCES]]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
@@ -36,8 +38,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed building libnfc.so")
     if verbose:
         sys.stderr.write(res.stderr)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace((out or LIB) + ".tmp", out or LIB)
+    return out or LIB
 
 
 if __name__ == "__main__":

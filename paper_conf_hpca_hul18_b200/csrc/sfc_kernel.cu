@@ -28,6 +28,17 @@ static constexpr int NWARP = TILE / 32;
 static constexpr int DPI_LIST = 16;     // distinct matches kept in a list before the bitmap path
 static constexpr int NFIX = ST_VAR_BASE;
 
+// tuning knobs (compile-time; defaults are the measured best)
+#ifndef NFC_PIPE
+#define NFC_PIPE 1            // 1: one-chunk lookahead, 3: three-stage pipeline
+#endif
+#ifndef NFC_EARLY_T24
+#define NFC_EARLY_T24 0       // issue the TBL24 read right after parse
+#endif
+#ifndef NFC_MINB
+#define NFC_MINB 3            // min resident CTAs per SM for chains without IPsec
+#endif
+
 // ---------------------------------------------------------------- shared memory layout
 struct SmemLayout {
     uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, acl4, acl6, wcnt, prefix, total;
@@ -312,40 +323,63 @@ __device__ __forceinline__ uint32_t dfa_byte(const DpiCtx &c, uint32_t s, uint32
     return e & 0x7FFFu;
 }
 
-// Returns the number of accept events; *first = state after the first one.  One
+// Returns the number of accept events and the state after the last one.  One
 // accept event (the common matching case) means the match set is exactly the
 // output closure of that state; more need the exact re-walk.
 template <bool WIDE>
+__device__ __forceinline__ void dfa_log(const DpiCtx &c, uint32_t &s, uint32_t byte, uint32_t &cnt, uint32_t &last)
+{
+    uint32_t acc;
+    s = dfa_byte<WIDE>(c, s, byte, acc);
+    if (acc) { cnt++; last = s; }
+}
+
+// payload bytes [A, 64) of the header cache, A compile-time: no per-byte guards
+template <bool WIDE, int A>
+__device__ __forceinline__ void walk_cached(const DpiCtx &c, const uint32_t h[16], uint32_t &s, uint32_t &cnt,
+                                            uint32_t &last)
+{
+#pragma unroll
+    for (int idx = A; idx < 64; idx++) dfa_log<WIDE>(c, s, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, cnt, last);
+}
+
+template <bool WIDE>
 __device__ __forceinline__ uint32_t dpi_fast(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
-                                             uint32_t b, uint64_t pol, uint32_t &first)
+                                             uint32_t b, uint64_t pol, uint32_t &last)
 {
     uint32_t s = 0, cnt = 0;
-    first = 0;
-    const uint32_t n = b - a;
+    last = 0;
+    if (b >= 64 && a == 42) walk_cached<WIDE, 42>(c, h, s, cnt, last);        // IPv4 UDP
+    else if (b >= 64 && a == 62) walk_cached<WIDE, 62>(c, h, s, cnt, last);   // IPv6 UDP
+    else if (b >= 64 && a == 54) walk_cached<WIDE, 54>(c, h, s, cnt, last);   // IPv4 TCP
+    else {
+        const uint32_t n = b - a;
 #pragma unroll
-    for (int idx = 32; idx < 64; idx++) {
-        const uint32_t byte = (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF;
-        uint32_t acc;
-        const uint32_t ns = dfa_byte<WIDE>(c, s, byte, acc);
-        const bool act = (uint32_t)idx - a < n;
-        s = act ? ns : s;
-        acc = act ? acc : 0u;
-        first = (acc && cnt == 0) ? ns : first;
-        cnt += acc;
+        for (int idx = 32; idx < 64; idx++) {
+            uint32_t acc;
+            const uint32_t ns = dfa_byte<WIDE>(c, s, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, acc);
+            if ((uint32_t)idx - a < n) {
+                s = ns;
+                if (acc) { cnt++; last = ns; }
+            }
+        }
     }
     for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
         const uint4 q = ld_stream16(f + ch, pol);
         const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+        if (ch >= a && ch + 16 <= b) {
 #pragma unroll
-        for (int k = 0; k < 16; k++) {
-            const uint32_t byte = (w[k >> 2] >> ((k & 3) * 8)) & 0xFF;
-            uint32_t acc;
-            const uint32_t ns = dfa_byte<WIDE>(c, s, byte, acc);
-            const bool act = ch + k - a < n;
-            s = act ? ns : s;
-            acc = act ? acc : 0u;
-            first = (acc && cnt == 0) ? ns : first;
-            cnt += acc;
+            for (int k = 0; k < 16; k++) dfa_log<WIDE>(c, s, (w[k >> 2] >> ((k & 3) * 8)) & 0xFF, cnt, last);
+        } else {
+#pragma unroll
+            for (int k = 0; k < 16; k++) {
+                uint32_t acc;
+                const uint32_t ns = dfa_byte<WIDE>(c, s, (w[k >> 2] >> ((k & 3) * 8)) & 0xFF, acc);
+                if (ch + k - a < b - a) {
+                    s = ns;
+                    if (acc) { cnt++; last = ns; }
+                }
+            }
         }
     }
     return cnt;
@@ -701,6 +735,7 @@ struct Pkt {
     uint32_t h[16];
     PV v;
     uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
+    uint32_t t24;             // TBL24 entry read right after parse (0xFFFFFFFF: not read)
     bool alive;
 };
 
@@ -721,10 +756,12 @@ __device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_
 
 struct Loc { uint8_t *f; uint32_t len; uint64_t gidx; };
 
-__device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
+// stage 1 of the packet pipeline: find the batch, issue the off/len loads
+struct Raw { uint8_t *arena; uint64_t off; uint32_t len; uint64_t gidx; };
+__device__ __forceinline__ Raw pkt_raw(const KParams &P, uint32_t g, bool valid)
 {
-    Loc l{nullptr, 0, 0};
-    if (!valid) return l;
+    Raw r{nullptr, 0, 0, 0};
+    if (!valid) return r;
     uint32_t bi = 0;
     if (P.n_batches > 1) {
         uint32_t lo = 0, hi = P.n_batches - 1;
@@ -736,16 +773,19 @@ __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool val
     }
     const BatchDev &B = P.batches[bi];
     const uint32_t li = g - B.start;
-    l.f = B.arena + B.off[li];
-    l.len = B.len[li];
-    l.gidx = B.first + li;
-    return l;
+    r.arena = B.arena;
+    r.off = B.off[li];
+    r.len = B.len[li];
+    r.gidx = B.first + li;
+    return r;
 }
+__device__ __forceinline__ Loc pkt_loc(const Raw &r) { return Loc{r.arena + r.off, r.len, r.gidx}; }
+__device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid) { return pkt_loc(pkt_raw(P, g, valid)); }
 
 __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid, Pkt &k)
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
-    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu;
     k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
     k.out_len = k.flen;
     if (!valid) return;
@@ -766,7 +806,7 @@ __device__ __forceinline__ void run_nf(const KParams &P, const Ctx &C, Pkt &k, u
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
         dropped = (r >> 31) != 0;
     } else if ((MASK & MASK_DPI) && kind == NFC_DPI) {
-        uint32_t first;
+        uint32_t first;   // state after the (only) accept event when cnt == 1
         const uint32_t cnt = C.dpi.wide ? dpi_fast<true>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, first)
                                         : dpi_fast<false>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f, first);
         if (cnt == 1) {
@@ -793,7 +833,8 @@ __device__ __forceinline__ void run_nf(const KParams &P, const Ctx &C, Pkt &k, u
         }
     } else if ((MASK & MASK_LPM4) && kind == NFC_LPM4) {
         if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
-        const uint32_t nh = lpm4_lookup(P.l4, k.v.dst[0], C.pol_l);
+        uint32_t nh = k.t24 != 0xFFFFFFFFu ? k.t24 : ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+        if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
         if (nh == 0x7FFF || hbyte(k.h, 22) <= 1) dropped = true;
         else {
             const uint2 n = __ldg(P.l4.nh + nh);
@@ -936,7 +977,7 @@ __device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8
 }
 
 template <uint32_t MASK>
-__global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(const KParams P)
+__global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : NFC_MINB) sfc_kernel(const KParams P)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     __shared__ uint32_t s_tile;
@@ -1007,29 +1048,51 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : 3) sfc_kernel(
     unsigned long long *ws = wst + warp * NFIX;
 
     if (!has_esp) {
-        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA
-        // barriers; the next chunk is claimed and located (off/len loads, L2 prefetch
-        // of its headers) before the current one is processed
+        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA barriers
         auto claim = [&]() {
             uint32_t b = 0;
             if (lane == 0) b = atomicAdd(P.tile_counter, 32u);
             return __shfl_sync(0xFFFFFFFFu, b, 0);
         };
-        uint32_t base = claim();
-        Loc loc = pkt_locate(P, base + lane, base + lane < P.n_pkts);
-        while (base < P.n_pkts) {
-            const uint32_t nbase = claim();
-            const bool nvalid = nbase + lane < P.n_pkts;
-            const Loc nloc = pkt_locate(P, nbase + lane, nvalid);
-            if (nvalid) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(nloc.f));
-            const uint32_t g = base + lane;
+#if NFC_PIPE == 3
+        // three-stage software pipeline, one iteration of distance each:
+        // claim chunk c+3 | load off/len of c+2 | locate c+1, prefetch its headers | process c
+        uint32_t c0 = claim(), c1 = claim(), c2 = claim();
+        Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
+        Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
+        while (c0 < P.n_pkts) {
+            uint32_t c3 = 0;
+            if (lane == 0) c3 = atomicAdd(P.tile_counter, 32u);
+            const Raw raw2 = pkt_raw(P, c2 + lane, c2 + lane < P.n_pkts);
+            const Loc loc1 = pkt_loc(raw1);
+            if (c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(loc1.f));
+#else
+        // next chunk claimed and located before the current one is processed
+        uint32_t c0 = claim();
+        Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
+        while (c0 < P.n_pkts) {
+            const uint32_t c1 = claim();
+            const Loc loc1 = pkt_locate(P, c1 + lane, c1 + lane < P.n_pkts);
+            if (c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(loc1.f));
+#endif
+            const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;
             pkt_begin(C, loc, valid, k);
+#if NFC_EARLY_T24
+            if ((MASK & MASK_LPM4) && (P.present & MASK_LPM4) && k.alive && k.v.fam == 4)
+                k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);   // header-phase lookup, used later
+#endif
             for (uint32_t pos = 0; pos < P.n_nf && k.alive; pos++) run_nf<MASK>(P, C, k, pos);
             pkt_end(P, C, k, valid, g, ws, lane);
-            base = nbase;
-            loc = nloc;
+#if NFC_PIPE == 3
+            c0 = c1; c1 = c2; c2 = __shfl_sync(0xFFFFFFFFu, c3, 0);
+            loc = loc1;
+            raw1 = raw2;
+#else
+            c0 = c1;
+            loc = loc1;
+#endif
         }
     } else if constexpr ((MASK & MASK_IPSEC) != 0) {
         // CTA tiles claimed in global order (ESP sequence numbers need the order)

@@ -13,7 +13,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libnfc.so")
+LIB_PATH = os.environ.get("NFC_LIB") or os.path.join(HERE, "libnfc.so")
 
 NFC_OK, NFC_EINVAL, NFC_ENOMEM, NFC_ECUDA, NFC_ESTATE, NFC_ECAP, NFC_EUNSUP = 0, -1, -2, -3, -4, -5, -6
 ACL, DPI, LPM4, LPM6, IPSEC, LB = 1, 2, 3, 4, 5, 6
