@@ -219,6 +219,14 @@ NFC_API int nfc_stats_len(const nfc_chain *c, size_t *len);
  * (one all-reduce of this vector over NCCL). */
 NFC_API int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags);
 
+/* Receive Side Steering for multi-GPU sharding (P:L87 RSS model): shard[i] =
+ * RETA[Toeplitz(MS default key, src|dst|sport|dport of frame i) & 127], RETA[j] =
+ * j mod n_shards (1..128); frames that fail to parse go to shard 0.  With n_shards
+ * dividing 64 and 64 ESP SAs, every SA lives on exactly one shard, so per-SA ESP
+ * sequence numbers of a sharded run equal the single-GPU run.  b and shard (u8 x n)
+ * are device pointers on `device`; asynchronous on `stream`. */
+NFC_API int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uint8_t *shard, void *stream);
+
 /* Number of kernel launches the library issued on this chain so far. */
 NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 

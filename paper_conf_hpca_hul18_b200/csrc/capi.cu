@@ -456,6 +456,23 @@ int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags)
     return NFC_OK;
 }
 
+int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uint8_t *shard, void *stream)
+{
+    if (!b || !shard || n_shards == 0 || n_shards > 128) return fail(NFC_EINVAL, "bad rss_shard arguments");
+    if (b->n && (!b->arena || !b->off || !b->len)) return fail(NFC_EINVAL, "batch pointers NULL");
+    CK(cudaSetDevice(device));
+    static thread_local DBuf nib_dev[16];
+    DBuf &nb = nib_dev[device & 15];
+    if (!nb.p) {
+        std::vector<uint32_t> nib;
+        build_toeplitz_nibbles(MS_RSS_KEY, nib);
+        CK(nb.upload(nib));
+    }
+    std::string err;
+    int rc = rss_shard_launch(b->arena, b->off, b->len, b->n, nb.as<uint32_t>(), n_shards, shard, stream, err);
+    return rc ? fail(rc, err) : NFC_OK;
+}
+
 int nfc_launch_count(const nfc_chain *c, uint64_t *count)
 {
     if (!c || !count) return fail(NFC_EINVAL, "NULL argument");

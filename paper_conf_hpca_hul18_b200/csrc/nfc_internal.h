@@ -191,5 +191,7 @@ struct LaunchCfg { int grid, block; size_t smem; };
 int sfc_launch(uint32_t mask, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
 size_t sfc_smem_bytes(uint32_t mask, const KParams &p);
 int sfc_query(uint32_t mask, const KParams &p, int device, LaunchCfg *cfg_out);  // grid for full occupancy
+int rss_shard_launch(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n, const uint32_t *nib,
+                     uint32_t n_shards, uint8_t *out, void *stream, std::string &err);
 
 } // namespace nfc

@@ -1125,6 +1125,40 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : NFC_MINB) sfc_
             if (vst[i]) atomicAdd(&P.stats[NFIX + i], (unsigned long long)vst[i]);
 }
 
+// ---------------------------------------------------------------- RSS steering
+// Receive Side Steering: shard = RETA[Toeplitz(MS key, src|dst|sport|dport) & 127]
+// with RETA[i] = i mod n_shards.  For n_shards | 64 every ESP SA (hash mod n_sa, n_sa = 64)
+// maps to exactly one shard.  Frames that fail to parse go to shard 0.
+__global__ void rss_shard_kernel(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n,
+                                 const uint32_t *nib, uint32_t n_shards, uint8_t *out)
+{
+    __shared__ uint32_t snib[72 * 16];
+    for (uint32_t i = threadIdx.x; i < 72 * 16; i += blockDim.x) snib[i] = __ldg(nib + i);
+    __syncthreads();
+    const uint64_t pol = pol_first();
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const uint8_t *f = arena + off[i];
+        const uint32_t fl = len[i];
+        uint32_t h[16];
+        load_header(f, fl, h, pol);
+        PV v;
+        uint32_t hsh = 0;
+        if (parse(h, f, fl, v)) hsh = toeplitz(snib, v);
+        out[i] = (uint8_t)((hsh & 127) % n_shards);
+    }
+}
+
+int rss_shard_launch(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n, const uint32_t *nib,
+                     uint32_t n_shards, uint8_t *out, void *stream, std::string &err)
+{
+    if (!n) return NFC_OK;
+    const uint32_t grid = min((n + 255) / 256, 148u * 8u);
+    rss_shard_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(arena, off, len, n, nib, n_shards, out);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { err = cudaGetErrorString(e); return NFC_ECUDA; }
+    return NFC_OK;
+}
+
 // ---------------------------------------------------------------- host launch
 template <uint32_t M>
 static int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCfg *cfg, bool query_only)

@@ -76,7 +76,7 @@ class Result(ctypes.Structure):
 
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
-           "nfc_launch_count", "nfc_last_error", "nfc_version"]
+           "nfc_launch_count", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
                  "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
@@ -98,6 +98,7 @@ def _load_lib():
     L.nfc_stats_len.argtypes = [_P, ctypes.POINTER(ctypes.c_size_t)]
     L.nfc_collect_stats.argtypes = [_P, _P, ctypes.c_size_t, _u32]
     L.nfc_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64)]
+    L.nfc_rss_shard.argtypes = [ctypes.c_int, ctypes.POINTER(Batch), _u32, _P, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
     P32 = ctypes.POINTER(_u32)
@@ -263,6 +264,13 @@ class Chain:
         c = ctypes.c_uint64()
         _check(lib.nfc_launch_count(self.h, ctypes.byref(c)))
         return c.value
+
+
+def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,
+              stream: int = 0):
+    """Device-side RSS steering: out[i] = shard of frame i (u8)."""
+    b = Batch(arena_ptr, off_ptr, len_ptr, n, 0, 0)
+    return _check(lib.nfc_rss_shard(device, ctypes.byref(b), n_shards, out_ptr, stream or None))
 
 
 def _cbuf(b: bytes):
