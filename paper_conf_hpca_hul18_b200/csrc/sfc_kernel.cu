@@ -50,7 +50,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, const KParams &
     L.wst = o; o += NWARP * NFIX * 8;                              // per-warp private counters (u64)
     L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
     o = (o + 15) & ~15u;
-    if (mask & MASK_IPSEC) { L.te = o; o += 5 * 256 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
+    if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_DPI) { L.cls = o; o += 256; L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u; }
     o = (o + 15) & ~15u;
@@ -555,23 +555,34 @@ __device__ __forceinline__ uint32_t toeplitz(const uint32_t *nib, const PV &v)
 }
 
 // ---------------------------------------------------------------- AES-128 / SHA-1
-__device__ __forceinline__ void aes128_encrypt(const uint32_t *te, const uint32_t rk[44], uint32_t in0, uint32_t in1,
+// AES-128 encryption with one T-table replicated 32 times in shared memory: lane l
+// reads copy l, which lives in bank l, so the 160 random lookups per block are free
+// of bank conflicts.  T1..T3 are byte rotations of T0; the S-box is byte 1 of T0.
+// tl = this lane's column of the replicated table (tl[x * 32] = T0[x]).
+__device__ __forceinline__ uint32_t T(const uint32_t *tl, uint32_t x) { return tl[x << 5]; }
+__device__ __forceinline__ uint32_t ror8(uint32_t x) { return __funnelshift_r(x, x, 8); }
+__device__ __forceinline__ uint32_t ror16(uint32_t x) { return __funnelshift_r(x, x, 16); }
+__device__ __forceinline__ uint32_t ror24(uint32_t x) { return __funnelshift_r(x, x, 24); }
+
+__device__ __forceinline__ void aes128_encrypt(const uint32_t *tl, const uint32_t rk[44], uint32_t in0, uint32_t in1,
                                                uint32_t in2, uint32_t in3, uint32_t out[4])
 {
-    const uint32_t *T0 = te, *T1 = te + 256, *T2 = te + 512, *T3 = te + 768, *S = te + 1024;
     uint32_t s0 = in0 ^ rk[0], s1 = in1 ^ rk[1], s2 = in2 ^ rk[2], s3 = in3 ^ rk[3];
 #pragma unroll
     for (int r = 1; r < 10; r++) {
-        uint32_t t0 = T0[s0 >> 24] ^ T1[(s1 >> 16) & 255] ^ T2[(s2 >> 8) & 255] ^ T3[s3 & 255] ^ rk[4 * r];
-        uint32_t t1 = T0[s1 >> 24] ^ T1[(s2 >> 16) & 255] ^ T2[(s3 >> 8) & 255] ^ T3[s0 & 255] ^ rk[4 * r + 1];
-        uint32_t t2 = T0[s2 >> 24] ^ T1[(s3 >> 16) & 255] ^ T2[(s0 >> 8) & 255] ^ T3[s1 & 255] ^ rk[4 * r + 2];
-        uint32_t t3 = T0[s3 >> 24] ^ T1[(s0 >> 16) & 255] ^ T2[(s1 >> 8) & 255] ^ T3[s2 & 255] ^ rk[4 * r + 3];
+        const uint32_t t0 = T(tl, s0 >> 24) ^ ror8(T(tl, (s1 >> 16) & 255)) ^ ror16(T(tl, (s2 >> 8) & 255)) ^ ror24(T(tl, s3 & 255)) ^ rk[4 * r];
+        const uint32_t t1 = T(tl, s1 >> 24) ^ ror8(T(tl, (s2 >> 16) & 255)) ^ ror16(T(tl, (s3 >> 8) & 255)) ^ ror24(T(tl, s0 & 255)) ^ rk[4 * r + 1];
+        const uint32_t t2 = T(tl, s2 >> 24) ^ ror8(T(tl, (s3 >> 16) & 255)) ^ ror16(T(tl, (s0 >> 8) & 255)) ^ ror24(T(tl, s1 & 255)) ^ rk[4 * r + 2];
+        const uint32_t t3 = T(tl, s3 >> 24) ^ ror8(T(tl, (s0 >> 16) & 255)) ^ ror16(T(tl, (s1 >> 8) & 255)) ^ ror24(T(tl, s2 & 255)) ^ rk[4 * r + 3];
         s0 = t0; s1 = t1; s2 = t2; s3 = t3;
     }
-    out[0] = (S[s0 >> 24] << 24 | S[(s1 >> 16) & 255] << 16 | S[(s2 >> 8) & 255] << 8 | S[s3 & 255]) ^ rk[40];
-    out[1] = (S[s1 >> 24] << 24 | S[(s2 >> 16) & 255] << 16 | S[(s3 >> 8) & 255] << 8 | S[s0 & 255]) ^ rk[41];
-    out[2] = (S[s2 >> 24] << 24 | S[(s3 >> 16) & 255] << 16 | S[(s0 >> 8) & 255] << 8 | S[s1 & 255]) ^ rk[42];
-    out[3] = (S[s3 >> 24] << 24 | S[(s0 >> 16) & 255] << 16 | S[(s1 >> 8) & 255] << 8 | S[s2 & 255]) ^ rk[43];
+    // final round: S[x] = byte 1 of T0[x]
+#define SB(x) ((T(tl, (x)) >> 8) & 255u)
+    out[0] = (SB(s0 >> 24) << 24 | SB((s1 >> 16) & 255) << 16 | SB((s2 >> 8) & 255) << 8 | SB(s3 & 255)) ^ rk[40];
+    out[1] = (SB(s1 >> 24) << 24 | SB((s2 >> 16) & 255) << 16 | SB((s3 >> 8) & 255) << 8 | SB(s0 & 255)) ^ rk[41];
+    out[2] = (SB(s2 >> 24) << 24 | SB((s3 >> 16) & 255) << 16 | SB((s0 >> 8) & 255) << 8 | SB(s1 & 255)) ^ rk[42];
+    out[3] = (SB(s3 >> 24) << 24 | SB((s0 >> 16) & 255) << 16 | SB((s1 >> 8) & 255) << 8 | SB(s2 & 255)) ^ rk[43];
+#undef SB
 }
 
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int n) { return __funnelshift_l(x, x, n); }
@@ -1034,9 +1045,9 @@ __global__ void __launch_bounds__(TILE, (MASK & MASK_IPSEC) ? 2 : NFC_MINB) sfc_
     }
     if ((MASK & MASK_IPSEC) && has_esp) {
         uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
-        for (uint32_t i = tid; i < 5 * 256; i += TILE) te[i] = __ldg(P.esp.te + i);
+        for (uint32_t i = tid; i < 256 * 32; i += TILE) te[i] = __ldg(P.esp.te + (i >> 5));   // T0 x 32 lanes
         for (uint32_t i = tid; i < 72 * 16; i += TILE) mn[i] = __ldg(P.esp.rss_nib + i);
-        C.te = te;
+        C.te = te + lane;         // this lane's bank column
         C.ms_nib = mn;
     }
     if ((MASK & MASK_LB) && (P.present & MASK_LB)) {
