@@ -229,16 +229,23 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % max(1, ndev)     # == local on a real N-GPU node
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
+    backend = os.environ.get("NFC_DIST_BACKEND", "nccl")   # gloo: test the N>1 path on fewer GPUs
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+    cdev = dev if backend == "nccl" else torch.device("cpu")   # where collectives run
 
     w = make_workload(args)
     n = ring_packets(w, args.ring_mb)
     first = rank * n                       # flows of rank r: its own slice of the global stream
     b = nfcgen.generate(w.traffic, w.tables, first, n)
-    chain = nfc.Chain(w.kinds, device=local)
+    chain = nfc.Chain(w.kinds, device=local_dev)
     chain.load_tables(w.tables)
     hr, tr = chain.room()
     assert hr <= w.traffic.headroom and tr <= w.traffic.tailroom
@@ -273,7 +280,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize(dev)
     t_wall0 = time.perf_counter()
-    with ClockSampler(local) as clk:
+    with ClockSampler(local_dev) as clk:
         if restore:   # restore the pristine ring between steps, outside the timed intervals
             for s in range(args.steps):
                 arena.copy_(pristine)
@@ -295,8 +302,8 @@ def main():
         ms = ev[0][0].elapsed_time(ev[-1][1])
     launches = chain.launches() - launches0
     stats = chain.stats(reset=True)
-    ms_t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    st_t = torch.from_numpy(stats.view(np.int64)).to(dev)
+    ms_t = torch.tensor([ms], dtype=torch.float64, device=cdev)
+    st_t = torch.from_numpy(stats.view(np.int64).copy()).to(cdev)
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
         dist.all_reduce(st_t, op=dist.ReduceOp.SUM)   # the only collective: counters
@@ -348,7 +355,7 @@ def main():
             dt = time.perf_counter() - t0
             if s:
                 times.append(dt)
-        e2e_t = torch.tensor([sum(times)], dtype=torch.float64, device=dev)
+        e2e_t = torch.tensor([sum(times)], dtype=torch.float64, device=cdev)
         if world > 1:
             dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         e2e = {"value": round(n * len(times) * world / float(e2e_t.item()) / 1e6, 3), "unit": "Mpps",
