@@ -10,6 +10,12 @@ if ROOT not in sys.path:
 GOLDEN = os.path.join(ROOT, "tests", "golden")
 
 
+def pytest_sessionstart(session):
+    """Build libnfc.so / libnfcgen.so / liboracle.so if missing or stale (nvcc cross-compiles here)."""
+    import __graft_entry__
+    __graft_entry__.build()
+
+
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a CUDA B200 (run with -m gpu on the GPU box)")
     config.addinivalue_line("markers", "slow: long-running CPU test")
