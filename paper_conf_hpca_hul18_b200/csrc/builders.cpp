@@ -115,43 +115,63 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
         blob.assign(ACLBV_HDR, 0);
         blob[0] = n; blob[1] = Wd; blob[2] = (uint32_t)F[0].b.size(); blob[3] = (uint32_t)F[1].b.size();
         blob[4] = (uint32_t)F[2].b.size(); blob[5] = (uint32_t)F[3].b.size(); blob[6] = kw;
-        auto align2 = [&]() { if (blob.size() & 1) blob.push_back(0); };
-        auto put_keys = [&](const FieldIv &f, uint32_t kwords) {
-            uint32_t o = (uint32_t)blob.size();
-            for (u128 k : f.b)
-                for (int q = (int)kwords - 1; q >= 0; q--) blob.push_back((uint32_t)(k >> (32 * q)));
-            return o;
-        };
-        auto put_bv = [&](const std::vector<uint64_t> &v) {
-            align2();
-            uint32_t o = (uint32_t)blob.size();
-            for (uint64_t x : v) { blob.push_back((uint32_t)x); blob.push_back((uint32_t)(x >> 32)); }
-            return o;
-        };
+        auto align_to = [&](size_t a) { while (blob.size() % a) blob.push_back(0); };
         // 257-entry bucket index per field on the top 8 key bits: bucket[t] = interval
-        // containing the first key of bucket t; the search is confined to [bk[t], bk[t+1]]
-        auto put_buckets = [&](const FieldIv &f, int kbits) {
-            uint32_t o = (uint32_t)blob.size();
+        // containing the first key of bucket t; the answer lies in [bk[t], bk[t+1]]
+        auto buckets = [&](const FieldIv &f, int kbits) {
             std::vector<uint32_t> bk(257);
             for (int t = 0; t <= 256; t++) {
                 u128 first = t == 256 ? (kbits == 128 ? ~(u128)0 : (((u128)1 << kbits) - 1)) : (u128)t << (kbits - 8);
                 bk[t] = (uint32_t)(std::upper_bound(f.b.begin(), f.b.end(), first) - f.b.begin() - 1);
             }
+            return bk;
+        };
+        // fixed-depth search: `steps` halvings cover the widest bucket window, so the
+        // device loop has a table-wide (warp-uniform) trip count instead of a per-key one
+        auto steps_of = [](const std::vector<uint32_t> &bk) {
+            uint32_t mmax = 1, st = 0;
+            for (int t = 0; t < 256; t++) mmax = std::max(mmax, bk[t + 1] - bk[t] + 1);
+            while ((1u << st) < mmax) st++;
+            return st;
+        };
+        const int fbits[4] = {bits, bits, 16, 16};
+        std::vector<uint32_t> BK[4];
+        uint32_t steps = 0;
+        for (int q = 0; q < 4; q++) {
+            BK[q] = buckets(F[q], fbits[q]);
+            steps |= steps_of(BK[q]) << (8 * q);
+        }
+        // keys (16-B aligned so an IPv6 key is one 128-bit load), followed by 2^steps
+        // all-ones pad keys: the window may run past the last interval start
+        auto put_keys = [&](const FieldIv &f, uint32_t kwords, uint32_t st) {
+            align_to(4);
+            uint32_t o = (uint32_t)blob.size();
+            for (u128 k : f.b)
+                for (int q = (int)kwords - 1; q >= 0; q--) blob.push_back((uint32_t)(k >> (32 * q)));
+            for (uint32_t i = 0; i < (1u << st) * kwords; i++) blob.push_back(0xFFFFFFFFu);
+            return o;
+        };
+        auto put_bv = [&](const std::vector<uint64_t> &v) {
+            align_to(2);
+            uint32_t o = (uint32_t)blob.size();
+            for (uint64_t x : v) { blob.push_back((uint32_t)x); blob.push_back((uint32_t)(x >> 32)); }
+            return o;
+        };
+        auto put_bk = [&](const std::vector<uint32_t> &bk) {
+            uint32_t o = (uint32_t)blob.size();
             for (int t = 0; t < 257; t++) blob.push_back(bk[t]);
             return o;
         };
         uint32_t offs[14];
-        offs[0] = put_keys(F[0], kw); offs[1] = put_bv(F[0].bv);
-        offs[2] = put_keys(F[1], kw); offs[3] = put_bv(F[1].bv);
-        offs[4] = put_keys(F[2], 1);  offs[5] = put_bv(F[2].bv);
-        offs[6] = put_keys(F[3], 1);  offs[7] = put_bv(F[3].bv);
+        offs[0] = put_keys(F[0], kw, steps & 255); offs[1] = put_bv(F[0].bv);
+        offs[2] = put_keys(F[1], kw, (steps >> 8) & 255); offs[3] = put_bv(F[1].bv);
+        offs[4] = put_keys(F[2], 1, (steps >> 16) & 255);  offs[5] = put_bv(F[2].bv);
+        offs[6] = put_keys(F[3], 1, steps >> 24);  offs[7] = put_bv(F[3].bv);
         offs[8] = put_bv(vproto);
         offs[9] = (uint32_t)blob.size();
         for (uint32_t r = 0; r < n; r++) blob.push_back(gidx[r] | (uint32_t)s.rules[gidx[r]].action << 31);
-        offs[10] = put_buckets(F[0], bits);
-        offs[11] = put_buckets(F[1], bits);
-        offs[12] = put_buckets(F[2], 16);
-        offs[13] = put_buckets(F[3], 16);
+        for (int q = 0; q < 4; q++) offs[10 + q] = put_bk(BK[q]);
+        blob[22] = steps;
         while (blob.size() & 3) blob.push_back(0);   // 16-B multiple for staging copies
         for (int k = 0; k < 14; k++) blob[8 + k] = offs[k];
     }

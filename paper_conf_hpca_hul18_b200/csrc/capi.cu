@@ -186,7 +186,9 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
         CK(c->acl_r4.upload(b4));
         CK(c->acl_r6.upload(b6));
         c->acl = AclImg{c->acl_r4.as<uint32_t>(), c->acl_r6.as<uint32_t>(), (uint32_t)b4.size(),
-                        (uint32_t)b6.size(), s.n_rules, s.default_action, 0};
+                        (uint32_t)b6.size(), s.n_rules, s.default_action, 0, {}, {}};
+        std::copy(b4.begin(), b4.begin() + ACLBV_HDR, c->acl.hdr4);
+        std::copy(b6.begin(), b6.begin() + ACLBV_HDR, c->acl.hdr6);
         c->n_acl_rules = s.n_rules;
         break;
     }
@@ -354,35 +356,47 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         p.seq_in = c->esp_seq[c->seq_parity].as<uint32_t>();
         p.seq_out = c->esp_seq[c->seq_parity ^ 1].as<uint32_t>();
     }
-    // shared-memory budget per CTA for the target occupancy: stage the ACL image
-    // when it fits and give the rest to full-row DFA hot states
+    // Shared memory: with a DM_FULL variant the whole DFA is staged per CTA (one CTA
+    // per SM) when it fits next to the rest; otherwise a budget per CTA for the
+    // target occupancy stages the ACL image and gives the rest to hot DFA rows.
+    Variant v = sfc_variant(c->kind, c->n_nf, false);
     {
-        int smem_sm = 0;
-        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device);
-        const int target = (c->mask & MASK_IPSEC) ? 2 : 4;
-        const size_t budget = (size_t)smem_sm / target - 1024 - 64;
-        p.acl.smem_words = 0;
+        const size_t limit = sfc_smem_limit(c->device);
+        p.acl.smem_words = (c->mask & MASK_ACL) ? 1 : 0;
         p.dpi.hot_states = 0;
-        if (c->mask & MASK_ACL) {
-            p.acl.smem_words = 1;
-            if (sfc_smem_bytes(c->mask, p) > budget / 2) p.acl.smem_words = 0;
-        }
+        bool full = false;
         if ((c->mask & MASK_DPI) && !c->dpi.wide) {
-            size_t base = sfc_smem_bytes(c->mask, p);
-            size_t h = base < budget ? (budget - base) / (2 * c->dpi.ncls + 1) : 0;
-            p.dpi.hot_states = (uint32_t)std::min<size_t>(h, c->dpi.n_states);
+            Variant vf = sfc_variant(c->kind, c->n_nf, true);
+            if (vf.dm == DM_FULL) {
+                p.dpi.hot_states = c->dpi.n_states;
+                if (sfc_smem_bytes(vf, p) + 1024 <= limit) { v = vf; full = true; }
+                else p.dpi.hot_states = 0;
+            }
+        }
+        if (!full) {
+            int smem_sm = 0;
+            cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device);
+            const int target = (c->mask & MASK_IPSEC) ? 2 : 4;
+            const size_t budget = std::min((size_t)smem_sm / target - 1024 - 64, limit);
+            if (c->mask & MASK_ACL)
+                if (sfc_smem_bytes(v, p) > budget / 2) p.acl.smem_words = 0;
+            if ((c->mask & MASK_DPI) && !c->dpi.wide) {
+                size_t base = sfc_smem_bytes(v, p);
+                size_t h = base < budget ? (budget - base) / (2 * c->dpi.ncls + 1) : 0;
+                p.dpi.hot_states = (uint32_t)std::min<size_t>(h, c->dpi.n_states);
+            }
         }
     }
     if (c->mask & MASK_DPI) {
         LaunchCfg q{};
-        if (sfc_query(c->mask, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");
+        if (sfc_query(v, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");
         size_t need = (size_t)q.grid * q.block * c->dpi.bitmap_words * 4;
         CK(c->dpi_bitmap.reserve(need));
         c->dpi.ovf_bitmap = c->dpi_bitmap.as<uint32_t>();
         p.dpi.ovf_bitmap = c->dpi.ovf_bitmap;
     }
     std::string err;
-    rc = sfc_launch(c->mask, p, c->device, st, err, nullptr);
+    rc = sfc_launch(v, p, c->device, st, err, nullptr);
     if (rc) return fail(rc, err);
     c->launches++;
     if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;

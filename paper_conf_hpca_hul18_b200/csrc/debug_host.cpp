@@ -152,22 +152,22 @@ int nfc_dbg_lpm6(nfc_dbg *d, const uint8_t dst[16], uint32_t *nh, uint32_t *prob
     return NFC_OK;
 }
 
-static uint32_t bs32(const uint32_t *B, uint32_t m, uint32_t key)
+// the kernel's fixed-depth window search (sfc_kernel.cu iv_search): `st` halvings from
+// the bucket start, clamped to the last real interval
+static uint32_t bs32(const uint32_t *B, uint32_t lo, uint32_t st, uint32_t m, uint32_t key)
 {
-    uint32_t lo = 0;
-    while (m > 1) { uint32_t h = m >> 1; if (B[lo + h] <= key) lo += h; m -= h; }
-    return lo;
+    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) if (B[lo + h] <= key) lo += h;
+    return std::min(lo, m - 1);
 }
 static bool le128h(const uint32_t *b, const uint32_t *k)
 {
     for (int q = 0; q < 3; q++) if (b[q] != k[q]) return b[q] < k[q];
     return b[3] <= k[3];
 }
-static uint32_t bs128(const uint32_t *B, uint32_t m, const uint32_t *k)
+static uint32_t bs128(const uint32_t *B, uint32_t lo, uint32_t st, uint32_t m, const uint32_t *k)
 {
-    uint32_t lo = 0;
-    while (m > 1) { uint32_t h = m >> 1; if (le128h(B + 4 * (lo + h), k)) lo += h; m -= h; }
-    return lo;
+    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) if (le128h(B + 4 * (lo + h), k)) lo += h;
+    return std::min(lo, m - 1);
 }
 
 int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *dst, uint16_t sport,
@@ -182,17 +182,15 @@ int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *
     int nb = family == 4 ? 1 : 4;
     for (int k = 0; k < nb; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
     const uint32_t W = A[1];
-    auto iv32 = [&](uint32_t ok, uint32_t ob, uint32_t key, int kbits) {
-        uint32_t tb = key >> (kbits - 8), lo = A[ob + tb], hi = A[ob + tb + 1];
-        return lo + bs32(A + ok + lo, hi - lo + 1, key);
+    auto iv32 = [&](int q, uint32_t key, int kbits) {
+        return bs32(A + A[8 + 2 * q], A[A[18 + q] + (key >> (kbits - 8))], (A[22] >> (8 * q)) & 255, A[2 + q], key);
     };
-    auto iv128 = [&](uint32_t ok, uint32_t ob, const uint32_t *k) {
-        uint32_t tb = k[0] >> 24, lo = A[ob + tb], hi = A[ob + tb + 1];
-        return lo + bs128(A + ok + 4 * lo, hi - lo + 1, k);
+    auto iv128 = [&](int q, const uint32_t *k) {
+        return bs128(A + A[8 + 2 * q], A[A[18 + q] + (k[0] >> 24)], (A[22] >> (8 * q)) & 255, A[2 + q], k);
     };
-    uint32_t js = nb == 1 ? iv32(A[8], A[18], s[0], 32) : iv128(A[8], A[18], s);
-    uint32_t jd = nb == 1 ? iv32(A[10], A[19], t[0], 32) : iv128(A[10], A[19], t);
-    uint32_t jsp = iv32(A[12], A[20], sport, 16), jdp = iv32(A[14], A[21], dport, 16);
+    uint32_t js = nb == 1 ? iv32(0, s[0], 32) : iv128(0, s);
+    uint32_t jd = nb == 1 ? iv32(1, t[0], 32) : iv128(1, t);
+    uint32_t jsp = iv32(2, sport, 16), jdp = iv32(3, dport, 16);
     auto bv = [&](uint32_t off, uint32_t j, uint32_t w) {
         uint64_t x;
         memcpy(&x, A + off + 2 * ((size_t)j * W + w), 8);

@@ -18,8 +18,9 @@ namespace nfc {
 //   m_src, m_dst, m_sport, m_dport  [6] key words per address (1 v4, 4 v6)
 //   [8..17] word offsets: keys_src, bv_src, keys_dst, bv_dst, keys_sp, bv_sp, keys_dp, bv_dp,
 //   bv_proto (256 x W), ridx (global rule index | action << 31),  [18..21] bucket tables
-//   (257 u32 per field) on the top 8 key bits.  Bitsets are u64 at
-//   even offsets.
+//   (257 u32 per field) on the top 8 key bits,  [22] search steps per field (8 bits each).
+//   Key arrays are 16-B aligned and followed by 2^steps all-ones pad keys.  Bitsets are
+//   u64 at even offsets.
 static const uint32_t ACLBV_HDR = 24;
 struct AclImg {
     const uint32_t *bv4, *bv6;        // device blobs
@@ -27,6 +28,7 @@ struct AclImg {
     uint32_t n_rules;
     uint32_t default_action;
     uint32_t smem_words;              // words staged in shared memory (0 = read from global)
+    uint32_t hdr4[ACLBV_HDR], hdr6[ACLBV_HDR];   // image headers, read from the constant bank
 };
 
 // ---------------------------------------------------------------- DPI
@@ -186,11 +188,18 @@ inline uint32_t l6_hash(uint32_t k0, uint32_t k1, uint32_t k2, uint32_t k3)
     return h ^ (h >> 15);
 }
 
-// kernel launch (sfc_kernel.cu)
+// kernel launch (sfc_kernel.cu).  The variant is chosen from the chain kinds and
+// the DFA placement (dfa_full: the whole DFA is staged in shared memory).
 struct LaunchCfg { int grid, block; size_t smem; };
-int sfc_launch(uint32_t mask, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
-size_t sfc_smem_bytes(uint32_t mask, const KParams &p);
-int sfc_query(uint32_t mask, const KParams &p, int device, LaunchCfg *cfg_out);  // grid for full occupancy
+// DFA placement: DM_HOT = hot rows in shared memory, the rest read through L2;
+// DM_FULL = the whole DFA in shared memory (one CTA per SM).
+enum { DM_HOT = 1, DM_FULL = 2 };
+struct Variant { uint32_t sig; int dm; int threads; bool esp; };
+Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full);
+int sfc_launch(const Variant &v, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
+size_t sfc_smem_bytes(const Variant &v, const KParams &p);
+size_t sfc_smem_limit(int device);      // max dynamic shared memory per CTA (opt-in)
+int sfc_query(const Variant &v, const KParams &p, int device, LaunchCfg *cfg_out);  // grid for full occupancy
 int rss_shard_launch(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n, const uint32_t *nib,
                      uint32_t n_shards, uint8_t *out, void *stream, std::string &err);
 

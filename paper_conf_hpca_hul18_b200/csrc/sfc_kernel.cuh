@@ -1,0 +1,1286 @@
+// sfc_kernel.cuh -- the fused, persistent SFC kernel for sm_100a (device code and
+// the launch template; instantiated per chain signature in sfc_inst_*.cu).
+//
+// One launch drains all packets of an nfc_process_batch call.  Every thread
+// carries one packet through the whole chain in registers:
+//   parse once (the de-duplicated header classifier)
+//   -> NFs in original SFC order, a dropped packet skipping every later NF
+//      (early drop; no batch re-split or per-NF launch)
+//   -> one 16 B result record; counters in per-warp private shared memory.
+// NF synthesis is done at compile time: the chain's kinds are a
+// template "signature", so the NF sequence is straight-line code with no
+// per-packet dispatch; one SIG_ANY instantiation interprets any other chain.
+// Scheduling (persistent kernel, P:L112, P:L235 [SIV]): without IPsec each warp
+// claims 32-packet chunks from a global atomic counter (no CTA barriers); with
+// IPsec each CTA claims tiles in order and assigns per-SA ESP sequence numbers
+// in global packet order by a decoupled look-back.
+// Tables stay on chip where they fit: the ACL bit-vector image, the Aho-Corasick
+// DFA (entirely, DM_FULL; or its hot rows, DM_HOT), AES T-tables and Toeplitz
+// nibble tables live in shared memory; DIR-24-8 / IPv6 hash levels are read
+// through L2 with an evict-last policy while the packet stream is evict-first.
+// Packet bytes are read from HBM once and rewritten in place.  No tensor cores:
+// nothing here is a dense contraction.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "nfc_internal.h"
+
+namespace nfc {
+
+static constexpr int DPI_LIST = 16;     // distinct matches kept in a list before the bitmap path
+static constexpr int NFIX = ST_VAR_BASE;
+static constexpr int NWS = ST_POS_BASE + 4 * NFC_MAX_CHAIN;   // per-warp counter slots
+
+// ---------------------------------------------------------------- chain signatures
+// n_nf in bits 28..31, the NF kind of position p in bits 4p..4p+3; SIG_ANY = 0
+// interprets P.kind at run time.
+static constexpr uint32_t SIG_ANY = 0;
+__host__ __device__ constexpr uint32_t sig_n(uint32_t s) { return s >> 28; }
+__host__ __device__ constexpr uint32_t sig_kind(uint32_t s, int p) { return (s >> (4 * p)) & 15u; }
+__host__ __device__ constexpr uint32_t sig_mask(uint32_t s)
+{
+    if (s == SIG_ANY) return (1u << NFC_ACL) | (1u << NFC_DPI) | (1u << NFC_LPM4) | (1u << NFC_LPM6) |
+                             (1u << NFC_IPSEC) | (1u << NFC_LB);
+    uint32_t m = 0;
+    for (int p = 0; p < (int)sig_n(s); p++) m |= 1u << sig_kind(s, p);
+    return m;
+}
+__host__ __device__ constexpr uint32_t sig_pos(uint32_t s, uint32_t kind)
+{
+    for (int p = 0; p < (int)sig_n(s); p++)
+        if (sig_kind(s, p) == kind) return (uint32_t)p;
+    return 0xFF;
+}
+__host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_t k1 = 0, uint32_t k2 = 0, uint32_t k3 = 0, uint32_t k4 = 0,
+                            uint32_t k5 = 0)
+{
+    return n << 28 | k0 | k1 << 4 | k2 << 8 | k3 << 12 | k4 << 16 | k5 << 20;
+}
+
+
+template <uint32_t S, int DM> struct KCfg {
+    static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
+    static constexpr int threads = (DM == DM_FULL && (S != SIG_ANY) && !esp) ? 768 : 256;
+    static constexpr int minb = esp ? 2 : (DM == DM_FULL ? 1 : 3);
+    static constexpr int nwarp = threads / 32;
+};
+
+// ---------------------------------------------------------------- shared memory layout
+struct SmemLayout {
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, acl4, acl6, wcnt, prefix, total;
+};
+__host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, const KParams &p)
+{
+    SmemLayout L{};
+    uint32_t o = 0;
+    L.wst = o; o += nwarp * NWS * 8;                                // per-warp private counters (u64)
+    L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
+    o = (o + 15) & ~15u;
+    if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
+    if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
+    if (mask & MASK_DPI) { L.cls = o; o += 256 * 4; L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u; }
+    o = (o + 15) & ~15u;
+    if (mask & MASK_ACL) {
+        const uint32_t s4 = p.acl.smem_words ? p.acl.words4 : 0, s6 = p.acl.smem_words ? p.acl.words6 : 0;
+        L.acl4 = o; o += s4 * 4;
+        L.acl6 = o; o += s6 * 4;
+    }
+    o = (o + 15) & ~15u;
+    if (mask & MASK_IPSEC) {
+        L.wcnt = o; o += nwarp * 256 * 2;
+        L.prefix = o; o += 256 * 4;
+    }
+    L.total = o;
+    return L;
+}
+
+// ---------------------------------------------------------------- small helpers
+__device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t mask32d(int len) { return len <= 0 ? 0u : len >= 32 ? 0xFFFFFFFFu : 0xFFFFFFFFu << (32 - len); }
+
+// L2 eviction policies: the packet stream is touched once (evict-first); lookup
+// tables are re-used by every packet (evict-last).
+__device__ __forceinline__ uint64_t pol_first()
+{
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_last()
+{
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint4 ld_stream16(const void *a, uint64_t pol)
+{
+    uint4 v;
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void st_stream16(void *a, uint4 v, uint64_t pol)
+{
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;"
+                 ::"l"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_tab16(const uint16_t *a, uint64_t pol)
+{
+    uint16_t v;
+    asm("ld.global.nc.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(a), "l"(pol));
+    return v;
+}
+// predicated read-only u16 load: returns `dflt` when !p (no memory access)
+__device__ __forceinline__ uint32_t ld_u16_if(bool p, const uint16_t *a, uint32_t dflt)
+{
+    uint32_t v = dflt;
+    asm("{\n\t.reg .pred q;\n\t.reg .u16 t;\n\tsetp.ne.u32 q, %2, 0;\n\t@q ld.global.nc.u16 t, [%1];\n\t@q cvt.u32.u16 %0, t;\n\t}"
+        : "+r"(v) : "l"(a), "r"((uint32_t)p));
+    return v;
+}
+
+// byte k (0..63) of the 64 B header cache; k compile-time in hot paths
+__device__ __forceinline__ uint32_t hbyte(const uint32_t h[16], uint32_t k) { return (h[k >> 2] >> ((k & 3) * 8)) & 0xFF; }
+__device__ __forceinline__ uint32_t hbe16(const uint32_t h[16], uint32_t k) { return hbyte(h, k) << 8 | hbyte(h, k + 1); }
+__device__ __forceinline__ uint32_t hbe32(const uint32_t h[16], uint32_t k) { return hbe16(h, k) << 16 | hbe16(h, k + 2); }
+// ---------------------------------------------------------------- per-packet state
+struct PV {
+    uint32_t fam;                 // 4 or 6
+    uint32_t l4_off, ip_end, pl_off;
+    uint32_t proto, sport, dport;
+    uint32_t src[4], dst[4];      // big-endian-valued words
+};
+
+__device__ __forceinline__ void load_header(const uint8_t *f, uint32_t flen, uint32_t h[16], uint64_t pol)
+{
+    const uint32_t nch = min(4u, (flen + 15) >> 4);
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+        uint4 v = c < (int)nch ? ld_stream16(f + 16 * c, pol) : make_uint4(0, 0, 0, 0);
+        h[4 * c] = v.x; h[4 * c + 1] = v.y; h[4 * c + 2] = v.z; h[4 * c + 3] = v.w;
+    }
+}
+
+// L4 fields outside the 64-B header cache (IPv4 options): rare, from memory
+static __device__ __noinline__ uint32_t l4_fields_mem(const uint8_t *f, uint32_t l4, uint32_t tcp)
+{
+    const uint32_t ports = (uint32_t)f[l4] << 24 | (uint32_t)f[l4 + 1] << 16 | (uint32_t)f[l4 + 2] << 8 | f[l4 + 3];
+    (void)tcp;
+    return ports;
+}
+static __device__ __noinline__ uint32_t tcp_doff_mem(const uint8_t *f, uint32_t l4) { return (uint32_t)f[l4 + 12] >> 4; }
+
+// Parse (P:L87 validity check): Ethernet -> IPv4/IPv6 -> UDP/TCP.
+__device__ __forceinline__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV &v)
+{
+    if (flen < 14) return false;
+    const uint32_t et = hbe16(h, 12);
+    bool frag = false;
+    if (et == 0x0800) {
+        if (flen < 34) return false;
+        const uint32_t vi = hbyte(h, 14);
+        if ((vi >> 4) != 4) return false;
+        const uint32_t ihl = vi & 15;
+        if (ihl < 5) return false;
+        const uint32_t tot = hbe16(h, 16);
+        if (tot < 4 * ihl || 14 + tot > flen) return false;
+        v.fam = 4;
+        v.l4_off = 14 + 4 * ihl;
+        v.ip_end = 14 + tot;
+        v.proto = hbyte(h, 23);
+        v.src[0] = hbe32(h, 26);
+        v.dst[0] = hbe32(h, 30);
+        v.src[1] = v.src[2] = v.src[3] = v.dst[1] = v.dst[2] = v.dst[3] = 0;
+        const uint32_t fo = hbe16(h, 20);
+        frag = (fo & 0x3FFF) != 0;       // MF set or non-zero offset
+    } else if (et == 0x86DD) {
+        if (flen < 54) return false;
+        if ((hbyte(h, 14) >> 4) != 6) return false;
+        const uint32_t pl = hbe16(h, 18);
+        if (54 + pl > flen) return false;
+        v.fam = 6;
+        v.l4_off = 54;
+        v.ip_end = 54 + pl;
+        v.proto = hbyte(h, 20);
+#pragma unroll
+        for (int k = 0; k < 4; k++) { v.src[k] = hbe32(h, 22 + 4 * k); v.dst[k] = hbe32(h, 38 + 4 * k); }
+    } else {
+        return false;
+    }
+    uint32_t l4len = 0;
+    v.sport = v.dport = 0;
+    if (!frag && (v.proto == 17 || v.proto == 6)) {
+        const uint32_t l4 = v.l4_off;
+        const bool tcp = v.proto == 6;
+        if (l4 + (tcp ? 20u : 8u) > v.ip_end) return false;
+        l4len = 8;
+        if (tcp) {
+            // data offset: byte 46 sits in the header cache; other offsets are rare -> memory
+            const uint32_t doff = l4 == 34 ? hbyte(h, 46) >> 4 : tcp_doff_mem(f, l4);
+            if (doff < 5 || l4 + 4 * doff > v.ip_end) return false;
+            l4len = 4 * doff;
+        }
+        uint32_t ports;
+        if (l4 == 34) ports = hbe32(h, 34);
+        else if (l4 == 54) ports = hbe32(h, 54);
+        else ports = l4_fields_mem(f, l4, tcp);
+        v.sport = ports >> 16;
+        v.dport = ports & 0xFFFF;
+    }
+    v.pl_off = v.l4_off + l4len;
+    return true;
+}
+
+// ---------------------------------------------------------------- ACL
+// Bit-vector first match: five interval lookups, AND of the five rule bitsets,
+// lowest set bit.  Each interval lookup is a bucket read on the top 8 key bits
+// followed by a fixed-depth window search whose depth is a table property
+// (warp-uniform trip count, no per-key divergence).  Header words come from the
+// kernel parameters (constant bank), not from the image.
+__device__ __forceinline__ uint32_t iv32(const uint32_t *A, const uint32_t *hd, int q, uint32_t key, int kbits)
+{
+    const uint32_t *B = A + hd[8 + 2 * q];
+    uint32_t lo = A[hd[18 + q] + (key >> (kbits - 8))];
+    const uint32_t st = (hd[22] >> (8 * q)) & 255;
+    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) lo = (B[lo + h] <= key) ? lo + h : lo;
+    return min(lo, hd[2 + q] - 1);
+}
+__device__ __forceinline__ bool le128(const uint4 b, const uint32_t k[4])
+{
+    if (b.x != k[0]) return b.x < k[0];
+    if (b.y != k[1]) return b.y < k[1];
+    if (b.z != k[2]) return b.z < k[2];
+    return b.w <= k[3];
+}
+__device__ __forceinline__ uint32_t iv128(const uint32_t *A, const uint32_t *hd, int q, const uint32_t k[4])
+{
+    const uint4 *B = reinterpret_cast<const uint4 *>(A + hd[8 + 2 * q]);
+    uint32_t lo = A[hd[18 + q] + (k[0] >> 24)];
+    const uint32_t st = (hd[22] >> (8 * q)) & 255;
+    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) lo = le128(B[lo + h], k) ? lo + h : lo;
+    return min(lo, hd[2 + q] - 1);
+}
+
+// returns global rule index (0xFFFF none) | action << 31
+__device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t *hd, uint32_t default_action,
+                                              uint32_t js, uint32_t jd, const PV &v)
+{
+    const uint32_t W = hd[1];
+    const uint32_t jsp = iv32(A, hd, 2, v.sport, 16);
+    const uint32_t jdp = iv32(A, hd, 3, v.dport, 16);
+    const uint64_t *vs = reinterpret_cast<const uint64_t *>(A + hd[9]) + (size_t)js * W;
+    const uint64_t *vd = reinterpret_cast<const uint64_t *>(A + hd[11]) + (size_t)jd * W;
+    const uint64_t *vsp = reinterpret_cast<const uint64_t *>(A + hd[13]) + (size_t)jsp * W;
+    const uint64_t *vdp = reinterpret_cast<const uint64_t *>(A + hd[15]) + (size_t)jdp * W;
+    const uint64_t *vpr = reinterpret_cast<const uint64_t *>(A + hd[16]) + (size_t)v.proto * W;
+    for (uint32_t w = 0; w < W; w++) {
+        const uint64_t x = vs[w] & vd[w] & vsp[w] & vdp[w] & vpr[w];
+        if (x) return A[hd[17] + 64 * w + (__ffsll((long long)x) - 1)];
+    }
+    return 0xFFFFu | default_action << 31;
+}
+
+__device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A6, const AclImg &ai, const PV &v)
+{
+    if (v.fam == 4) {
+        const uint32_t *hd = ai.hdr4;
+        if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
+        const uint32_t js = iv32(A4, hd, 0, v.src[0], 32);
+        const uint32_t jd = iv32(A4, hd, 1, v.dst[0], 32);
+        return acl_match(A4, hd, ai.default_action, js, jd, v);
+    }
+    const uint32_t *hd = ai.hdr6;
+    if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
+    const uint32_t js = iv128(A6, hd, 0, v.src);
+    const uint32_t jd = iv128(A6, hd, 1, v.dst);
+    return acl_match(A6, hd, ai.default_action, js, jd, v);
+}
+
+// ---------------------------------------------------------------- DPI
+// Aho-Corasick DFA walk over byte classes.  Transition entries are u16: next
+// state | ACCEPT << 15 (ACCEPT: the next state has a non-empty output set); u32
+// with ACCEPT << 31 above 32K states ("wide").
+//   DM_FULL: all rows in shared memory; cls[b] = smem byte offset of column
+//            class(b) in row 0, so a step is IMAD + LDS.
+//   DM_HOT:  the first H states (BFS order) in shared memory, cls[b] = 2*class(b);
+//            cold states read the global table (predicated load).
+// A walk keeps three registers: s (state), cnt (accept events), mx (max entry
+// seen).  Accept entries are >= 0x8000 > any other entry, so when cnt == 1 the
+// state after the only accept event is mx & 0x7FFF and the match set is its
+// output closure; cnt > 1 takes the exact re-walk (dpi_slow).
+struct DpiCtx {
+    const uint32_t *cls;    // smem, 256 entries
+    const uint8_t *gcls;    // global byte -> class table (exact re-walk)
+    const uint8_t *sm;      // smem base (DM_FULL addressing)
+    const uint8_t *hot;     // smem hot rows (DM_HOT)
+    uint32_t row2;          // bytes per row = 2 * ncls
+    uint32_t H, HK2;        // DM_HOT: hot states, byte offset of the last hot entry
+    uint32_t ncls, wide;
+    const void *trans;
+    const uint32_t *out_off;
+    const uint16_t *out_ids;
+    const uint8_t *pat_action;
+};
+
+struct Walk { uint32_t s, cnt, mx; };
+
+template <int DM>
+__device__ __forceinline__ uint32_t dfa_entry(const DpiCtx &c, uint32_t s, uint32_t byte)
+{
+    const uint32_t cv = c.cls[byte];
+    if (DM == DM_FULL) return *reinterpret_cast<const uint16_t *>(c.sm + (s * c.row2 + cv));
+    const uint32_t k2 = s * c.row2 + cv;
+    const uint32_t e = *reinterpret_cast<const uint16_t *>(c.hot + min(k2, c.HK2));
+    return ld_u16_if(s >= c.H, reinterpret_cast<const uint16_t *>(reinterpret_cast<const uint8_t *>(c.trans) + k2), e);
+}
+template <int DM>
+__device__ __forceinline__ void dfa_step(const DpiCtx &c, Walk &w, uint32_t byte)
+{
+    const uint32_t e = dfa_entry<DM>(c, w.s, byte);
+    w.s = e & 0x7FFFu;
+    w.cnt += e >> 15;
+    w.mx = max(w.mx, e);
+}
+// step only if `in` (bytes outside the payload leave the walk unchanged: s <= mx always)
+template <int DM>
+__device__ __forceinline__ void dfa_step_if(const DpiCtx &c, Walk &w, uint32_t byte, bool in)
+{
+    const uint32_t e = in ? dfa_entry<DM>(c, w.s, byte) : w.s;
+    w.s = e & 0x7FFFu;
+    w.cnt += e >> 15;
+    w.mx = max(w.mx, e);
+}
+__device__ __forceinline__ void dfa_step_wide(const DpiCtx &c, Walk &w, uint32_t byte, bool in)
+{
+    const uint32_t k = w.s * c.ncls + (c.cls[byte] >> 1);
+    const uint32_t e = in ? __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k) : w.s;
+    w.s = e & 0x7FFFFFFFu;
+    w.cnt += e >> 31;
+    w.mx = max(w.mx, e);
+}
+
+// payload bytes [A, 64) of the header cache, A compile-time: no per-byte guards
+template <int DM, int A>
+__device__ __forceinline__ void walk_cached(const DpiCtx &c, const uint32_t h[16], Walk &w)
+{
+#pragma unroll
+    for (int idx = A; idx < 64; idx++) dfa_step<DM>(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF);
+}
+
+// walk of a DFA with > 32K states (u32 entries, all rows in global memory); not inlined
+static __device__ __noinline__ Walk dpi_walk_wide(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
+                                                  uint32_t b, uint64_t pol)
+{
+    Walk w{0, 0, 0};
+#pragma unroll
+    for (int idx = 32; idx < 64; idx++) dfa_step_wide(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, (uint32_t)idx - a < b - a);
+    for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
+        const uint4 q = ld_stream16(f + ch, pol);
+        const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+        for (int k = 0; k < 16; k++) dfa_step_wide(c, w, (wd[k >> 2] >> ((k & 3) * 8)) & 0xFF, ch + k - a < b - a);
+    }
+    return w;
+}
+
+// Fast walk over payload [a, b): counts accept events (see DpiCtx).  Bytes 32..63
+// come from the header cache (a payload never starts before byte 34), the rest
+// from memory in 16-B chunks.
+template <int DM>
+__device__ __forceinline__ Walk dpi_walk(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
+                                         uint32_t b, uint64_t pol)
+{
+    if (DM != DM_FULL && c.wide) return dpi_walk_wide(c, h, f, a, b, pol);
+    Walk w{0, 0, 0};
+    if (b >= 64 && a == 42) walk_cached<DM, 42>(c, h, w);        // IPv4 UDP
+    else if (b >= 64 && a == 62) walk_cached<DM, 62>(c, h, w);   // IPv6 UDP
+    else if (b >= 64 && a == 54) walk_cached<DM, 54>(c, h, w);   // IPv4 TCP
+    else {
+#pragma unroll
+        for (int idx = 32; idx < 64; idx++)
+            dfa_step_if<DM>(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, (uint32_t)idx - a < b - a);
+    }
+    for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
+        const uint4 q = ld_stream16(f + ch, pol);
+        const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+        if (ch >= a && ch + 16 <= b) {
+#pragma unroll
+            for (int k = 0; k < 16; k++) dfa_step<DM>(c, w, (wd[k >> 2] >> ((k & 3) * 8)) & 0xFF);
+        } else {
+#pragma unroll
+            for (int k = 0; k < 16; k++) dfa_step_if<DM>(c, w, (wd[k >> 2] >> ((k & 3) * 8)) & 0xFF, ch + k - a < b - a);
+        }
+    }
+    return w;
+}
+
+// Exact match set of a packet whose walk hit more than one accept event (rare
+// path, not inlined): re-walk the payload from memory collecting distinct pattern
+// ids in a register list, or -- beyond DPI_LIST ids -- in a per-thread global
+// bitmap; emit the (packet, pattern) pairs.  Returns nmatch | any_drop << 31.
+struct DpiOvf {
+    uint32_t *bitmap;
+    uint32_t words;
+    uint32_t *match_count, *match_pkt;
+    uint16_t *match_pat;
+    uint32_t match_cap;
+    unsigned long long *stats;
+};
+// one exact DFA step from the global table (state -> next, accept flag)
+__device__ __forceinline__ uint32_t dfa_step_global(const DpiCtx &c, uint32_t s, uint32_t b, bool &acc)
+{
+    const uint32_t k = s * c.ncls + __ldg(c.gcls + b);
+    if (c.wide) {
+        const uint32_t e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k);
+        acc = e >> 31;
+        return e & 0x7FFFFFFFu;
+    }
+    const uint32_t e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + k);
+    acc = (e >> 15) & 1;
+    return e & 0x7FFFu;
+}
+static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a, uint32_t b, uint32_t gtid,
+                                          DpiOvf o, uint32_t pkt_id)
+{
+    uint16_t ids[DPI_LIST];
+    uint32_t n = 0, drop = 0;
+    bool ovf = false;
+    uint32_t s = 0;
+    uint4 q = make_uint4(0, 0, 0, 0);
+    for (uint32_t i = a; i < b && !ovf; i++) {
+        if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
+        const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
+        bool acc;
+        s = dfa_step_global(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
+        if (!acc) continue;
+        const uint32_t e = __ldg(c.out_off + s + 1);
+        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+            const uint32_t id = __ldg(c.out_ids + x);
+            drop |= __ldg(c.pat_action + id);
+            bool seen = false;
+            for (uint32_t k = 0; k < n; k++) seen |= ids[k] == id;
+            if (seen) continue;
+            if (n == DPI_LIST) { ovf = true; break; }
+            ids[n++] = (uint16_t)id;
+        }
+    }
+    if (!ovf) {
+        if (n) {
+            const uint32_t slot = atomicAdd(o.match_count, n);
+            for (uint32_t k = 0; k < n; k++)
+                if (slot + k < o.match_cap) { o.match_pkt[slot + k] = pkt_id; o.match_pat[slot + k] = ids[k]; }
+            if (slot + n > o.match_cap)
+                atomicAdd(&o.stats[ST_MATCH_OVF], (unsigned long long)(slot + n - max(slot, o.match_cap)));
+        }
+        return n | drop << 31;
+    }
+    // more than DPI_LIST distinct ids: exact bitmap pass
+    atomicAdd(&o.stats[ST_DPI_OVF_PKTS], 1ull);
+    uint32_t *bm = o.bitmap + (size_t)gtid * o.words;
+    for (uint32_t k = 0; k < o.words; k++) bm[k] = 0;
+    uint32_t cnt = 0;
+    s = 0;
+    drop = 0;
+    for (uint32_t i = a; i < b; i++) {
+        if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
+        const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
+        bool acc;
+        s = dfa_step_global(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
+        if (!acc) continue;
+        const uint32_t e = __ldg(c.out_off + s + 1);
+        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+            const uint32_t id = __ldg(c.out_ids + x);
+            drop |= __ldg(c.pat_action + id);
+            const uint32_t bit = 1u << (id & 31);
+            if (bm[id >> 5] & bit) continue;
+            bm[id >> 5] |= bit;
+            cnt++;
+            const uint32_t slot = atomicAdd(o.match_count, 1u);
+            if (slot < o.match_cap) { o.match_pkt[slot] = pkt_id; o.match_pat[slot] = (uint16_t)id; }
+            else atomicAdd(&o.stats[ST_MATCH_OVF], 1ull);
+        }
+    }
+    return cnt | drop << 31;
+}
+
+// ---------------------------------------------------------------- LPM
+__device__ __forceinline__ uint32_t lpm6_lookup(const Lpm6Img &t, const uint32_t dst[4])
+{
+    uint32_t best = t.def_nh;
+    int lo = 0, hi = (int)t.n_levels - 1;
+    while (lo <= hi) {
+        int mid = (lo + hi) >> 1;
+        int L = __ldg(t.lens + mid);
+        uint32_t k0 = dst[0] & mask32d(L), k1 = dst[1] & mask32d(L - 32);
+        uint32_t k2 = dst[2] & mask32d(L - 64), k3 = dst[3] & mask32d(L - 96);
+        uint32_t m = __ldg(t.mask + mid), base = __ldg(t.base + mid);
+        uint32_t hsh = l6_hash(k0, k1, k2, k3) & m;
+        bool found = false;
+        uint32_t info = 0;
+        for (;;) {
+            const uint4 *e = t.ent + 2 * (size_t)(base + hsh);
+            uint4 key = __ldg(e);
+            uint32_t inf = __ldg(reinterpret_cast<const uint32_t *>(e + 1));
+            if (!(inf & L6_VALID)) break;
+            if (key.x == k0 && key.y == k1 && key.z == k2 && key.w == k3) { found = true; info = inf; break; }
+            hsh = (hsh + 1) & m;
+        }
+        if (found) {
+            if ((info & 0xFFFF) != 0x7FFF) best = info & 0xFFFF;
+            lo = mid + 1;
+        } else {
+            hi = mid - 1;
+        }
+    }
+    return best;
+}
+
+// L2/L3 rewrite after an LPM hit (R#6): dst MAC = nh MAC, src MAC = port MAC,
+// TTL / hop limit - 1, IPv4 header checksum recomputed (RFC 1071, byte-order independent
+// sum over little-endian halves).  Writes the first 32 B of the frame.
+__device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm, uint64_t pol)
+{
+    h[0] = nh.x;
+    h[1] = (nh.y & 0xFFFF) | (pm.x << 16);
+    h[2] = (pm.x >> 16) | (pm.y << 16);
+    if (v.fam == 4) {
+        h[5] -= 1u << 16;                     // TTL: byte 22
+        h[6] &= 0xFFFF0000u;                  // checksum bytes 24..25 := 0
+        uint32_t sum;
+        if (v.l4_off == 34) {
+            sum = (h[3] >> 16) + (h[4] & 0xFFFF) + (h[4] >> 16) + (h[5] & 0xFFFF) + (h[5] >> 16) +
+                  (h[6] >> 16) + (h[7] & 0xFFFF) + (h[7] >> 16) + (h[8] & 0xFFFF);
+        } else {                              // IPv4 options (rare): bytes >= 32 from memory
+            sum = (h[3] >> 16) + (h[4] & 0xFFFF) + (h[4] >> 16) + (h[5] & 0xFFFF) + (h[5] >> 16) +
+                  (h[6] >> 16) + (h[7] & 0xFFFF) + (h[7] >> 16);
+            for (uint32_t k = 32; k < v.l4_off; k += 2) sum += (uint32_t)f[k] | (uint32_t)f[k + 1] << 8;
+        }
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        h[6] |= (~sum) & 0xFFFF;
+    } else {
+        h[5] -= 1u << 8;                      // hop limit: byte 21
+    }
+    st_stream16(f, make_uint4(h[0], h[1], h[2], h[3]), pol);
+    st_stream16(f + 16, make_uint4(h[4], h[5], h[6], h[7]), pol);
+}
+
+// ---------------------------------------------------------------- Toeplitz flow hash
+__device__ __forceinline__ uint32_t toeplitz(const uint32_t *nib, const PV &v)
+{
+    uint32_t w[9];
+    uint32_t nw;
+    if (v.fam == 4) { w[0] = v.src[0]; w[1] = v.dst[0]; w[2] = v.sport << 16 | v.dport; nw = 3; }
+    else {
+#pragma unroll
+        for (int k = 0; k < 4; k++) { w[k] = v.src[k]; w[4 + k] = v.dst[k]; }
+        w[8] = v.sport << 16 | v.dport;
+        nw = 9;
+    }
+    uint32_t hsh = 0;
+#pragma unroll
+    for (int i = 0; i < 9; i++) {
+        if (i < (int)nw) {
+#pragma unroll
+            for (int n = 0; n < 8; n++) hsh ^= nib[(8 * i + n) * 16 + ((w[i] >> (28 - 4 * n)) & 15)];
+        }
+    }
+    return hsh;
+}
+
+// ---------------------------------------------------------------- AES-128 / SHA-1
+// AES-128 encryption with one T-table replicated 32 times in shared memory: lane l
+// reads copy l, which lives in bank l, so the 160 random lookups per block are free
+// of bank conflicts.  T1..T3 are byte rotations of T0; the S-box is byte 1 of T0.
+// tl = this lane's column of the replicated table (tl[x * 32] = T0[x]).
+__device__ __forceinline__ uint32_t T(const uint32_t *tl, uint32_t x) { return tl[x << 5]; }
+__device__ __forceinline__ uint32_t ror8(uint32_t x) { return __funnelshift_r(x, x, 8); }
+__device__ __forceinline__ uint32_t ror16(uint32_t x) { return __funnelshift_r(x, x, 16); }
+__device__ __forceinline__ uint32_t ror24(uint32_t x) { return __funnelshift_r(x, x, 24); }
+
+__device__ __forceinline__ void aes128_encrypt(const uint32_t *tl, const uint32_t rk[44], uint32_t in0, uint32_t in1,
+                                               uint32_t in2, uint32_t in3, uint32_t out[4])
+{
+    uint32_t s0 = in0 ^ rk[0], s1 = in1 ^ rk[1], s2 = in2 ^ rk[2], s3 = in3 ^ rk[3];
+#pragma unroll
+    for (int r = 1; r < 10; r++) {
+        const uint32_t t0 = T(tl, s0 >> 24) ^ ror8(T(tl, (s1 >> 16) & 255)) ^ ror16(T(tl, (s2 >> 8) & 255)) ^ ror24(T(tl, s3 & 255)) ^ rk[4 * r];
+        const uint32_t t1 = T(tl, s1 >> 24) ^ ror8(T(tl, (s2 >> 16) & 255)) ^ ror16(T(tl, (s3 >> 8) & 255)) ^ ror24(T(tl, s0 & 255)) ^ rk[4 * r + 1];
+        const uint32_t t2 = T(tl, s2 >> 24) ^ ror8(T(tl, (s3 >> 16) & 255)) ^ ror16(T(tl, (s0 >> 8) & 255)) ^ ror24(T(tl, s1 & 255)) ^ rk[4 * r + 2];
+        const uint32_t t3 = T(tl, s3 >> 24) ^ ror8(T(tl, (s0 >> 16) & 255)) ^ ror16(T(tl, (s1 >> 8) & 255)) ^ ror24(T(tl, s2 & 255)) ^ rk[4 * r + 3];
+        s0 = t0; s1 = t1; s2 = t2; s3 = t3;
+    }
+    // final round: S[x] = byte 1 of T0[x]
+#define SB(x) ((T(tl, (x)) >> 8) & 255u)
+    out[0] = (SB(s0 >> 24) << 24 | SB((s1 >> 16) & 255) << 16 | SB((s2 >> 8) & 255) << 8 | SB(s3 & 255)) ^ rk[40];
+    out[1] = (SB(s1 >> 24) << 24 | SB((s2 >> 16) & 255) << 16 | SB((s3 >> 8) & 255) << 8 | SB(s0 & 255)) ^ rk[41];
+    out[2] = (SB(s2 >> 24) << 24 | SB((s3 >> 16) & 255) << 16 | SB((s0 >> 8) & 255) << 8 | SB(s1 & 255)) ^ rk[42];
+    out[3] = (SB(s3 >> 24) << 24 | SB((s0 >> 16) & 255) << 16 | SB((s1 >> 8) & 255) << 8 | SB(s2 & 255)) ^ rk[43];
+#undef SB
+}
+
+__device__ __forceinline__ uint32_t rotl(uint32_t x, int n) { return __funnelshift_l(x, x, n); }
+
+__device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16])
+{
+    uint32_t a = H[0], b = H[1], c = H[2], d = H[3], e = H[4];
+#pragma unroll
+    for (int t = 0; t < 80; t++) {
+        uint32_t w;
+        if (t < 16) w = W[t];
+        else {
+            w = rotl(W[(t - 3) & 15] ^ W[(t - 8) & 15] ^ W[(t - 14) & 15] ^ W[t & 15], 1);
+            W[t & 15] = w;
+        }
+        uint32_t f, k;
+        if (t < 20) { f = d ^ (b & (c ^ d)); k = 0x5a827999u; }
+        else if (t < 40) { f = b ^ c ^ d; k = 0x6ed9eba1u; }
+        else if (t < 60) { f = (b & c) | (d & (b | c)); k = 0x8f1bbcdcu; }
+        else { f = b ^ c ^ d; k = 0xca62c1d6u; }
+        uint32_t tmp = rotl(a, 5) + f + e + k + w;
+        e = d; d = c; c = rotl(b, 30); b = a; a = tmp;
+    }
+    H[0] += a; H[1] += b; H[2] += c; H[3] += d; H[4] += e;
+}
+
+// IPsec ESP transport mode (RFC 4303 + RFC 3686 + RFC 2404; R#8), in place:
+// the header [0,l4) moves to f-16, ESP header + IV fill [l4-16, l4) of the new frame,
+// the L4 bytes are encrypted where they lie, trailer and ICV are appended.
+// Returns the new frame length.  Stream bytes are handled as 32-bit words; memory
+// words are 4-B aligned and related to stream words by a funnel shift of r = A & 3.
+__device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t seq, const uint32_t *te)
+{
+    const uint32_t l4 = v.l4_off, plen = v.ip_end - l4;
+    const uint32_t p = (4 - ((plen + 2) & 3)) & 3;
+    const uint32_t clen = plen + p + 2;          // multiple of 4
+    const uint32_t nK = clen >> 2;
+    uint32_t rk[44];
+    {
+        const uint4 *q = reinterpret_cast<const uint4 *>(sap->rk);
+#pragma unroll
+        for (int i = 0; i < 11; i++) { uint4 x = __ldg(q + i); rk[4 * i] = x.x; rk[4 * i + 1] = x.y; rk[4 * i + 2] = x.z; rk[4 * i + 3] = x.w; }
+    }
+    const uint32_t spi = __ldg(&sap->spi), nonce = __ldg(&sap->nonce);
+    // 1. move the header 16 B left and fix up the IP header
+    {
+        uint32_t *src = reinterpret_cast<uint32_t *>(f);
+        uint32_t *dst = reinterpret_cast<uint32_t *>(f - 16);
+        uint32_t nw = (l4 + 3) >> 2;
+        for (uint32_t i = 0; i < nw; i++) dst[i] = src[i];
+        uint8_t *g = f - 16;
+        if (v.fam == 4) {
+            g[23] = 50;
+            uint32_t tot = ((uint32_t)g[16] << 8 | g[17]) + 30 + p;
+            g[16] = (uint8_t)(tot >> 8); g[17] = (uint8_t)tot;
+            g[24] = 0; g[25] = 0;
+            uint32_t sum = 0;
+            for (uint32_t k = 14; k < l4; k += 2) sum += (uint32_t)g[k] << 8 | g[k + 1];
+            sum = (sum & 0xFFFF) + (sum >> 16);
+            sum = (sum & 0xFFFF) + (sum >> 16);
+            sum = ~sum;
+            g[24] = (uint8_t)(sum >> 8); g[25] = (uint8_t)sum;
+        } else {
+            g[20] = 50;
+            uint32_t pl = ((uint32_t)g[18] << 8 | g[19]) + 30 + p;
+            g[18] = (uint8_t)(pl >> 8); g[19] = (uint8_t)pl;
+        }
+        // the new frame starts at f-16, so its ESP header bytes [l4, l4+16) are f+[l4-16, l4)
+        uint8_t *e = f + l4 - 16;
+        const uint32_t hw[4] = {spi, seq, 0u, seq};
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            e[4 * i] = (uint8_t)(hw[i] >> 24); e[4 * i + 1] = (uint8_t)(hw[i] >> 16);
+            e[4 * i + 2] = (uint8_t)(hw[i] >> 8); e[4 * i + 3] = (uint8_t)hw[i];
+        }
+    }
+    // 2. encrypt [A, A+clen) in place and MAC [A-16, A+clen), A = f + l4
+    uint8_t *A = f + l4;
+    const uint32_t r = (uint32_t)(reinterpret_cast<uintptr_t>(A) & 3);
+    uint32_t *W0 = reinterpret_cast<uint32_t *>(A - r);   // aligned word 0 (contains stream bytes -r..3-r)
+    const uint32_t sh = 32 - 8 * r;                       // funnel amount memory<-stream
+    uint32_t Mcur = W0[0];                                // memory word k (plaintext side)
+    uint32_t Cprev = r ? (Mcur << (8 * (4 - r))) : 0u;    // carries the IV bytes below A
+    uint32_t H[5];
+#pragma unroll
+    for (int i = 0; i < 5; i++) H[i] = __ldg(&sap->ipad[i]);
+    uint32_t W[16];
+    const uint32_t nmsg = 4 + nK;                         // message words (ESP hdr + C)
+    const uint32_t total_bits = (64u + 4u * nmsg) * 8u;
+    const uint32_t nblk = (4 * nmsg + 9 + 63) / 64;       // SHA blocks after the ipad block
+    const uint32_t trailer_nh = v.proto;
+    uint32_t ks[4] = {0, 0, 0, 0};
+    for (uint32_t blk = 0; blk < nblk; blk++) {
+#pragma unroll
+        for (int w = 0; w < 16; w++) {
+            const uint32_t i = blk * 16 + w;              // message word index
+            uint32_t m;
+            if (i < 4) {
+                m = (w == 0) ? spi : (w == 2) ? 0u : seq;
+            } else if (i < nmsg) {
+                const uint32_t k = i - 4;                 // stream word
+                if ((w & 3) == 0) {                       // new AES counter block every 4 words
+                    uint32_t o[4];
+                    aes128_encrypt(te, rk, nonce, 0u, seq, (k >> 2) + 1, o);
+                    ks[0] = bswap32(o[0]); ks[1] = bswap32(o[1]); ks[2] = bswap32(o[2]); ks[3] = bswap32(o[3]);
+                }
+                uint32_t Mnext = W0[k + 1];
+                uint32_t P = __funnelshift_rc(Mcur, Mnext, 8 * r);   // stream bytes 4k..4k+3 (LE)
+                if (4 * k + 4 > plen) {                   // trailer: pad 1..p, p, next header
+                    uint32_t pw = 0;
+#pragma unroll
+                    for (int b = 0; b < 4; b++) {
+                        uint32_t s = 4 * k + b, byte;
+                        if (s < plen) byte = (P >> (8 * b)) & 0xFF;
+                        else if (s < plen + p) byte = s - plen + 1;
+                        else if (s == plen + p) byte = p;
+                        else byte = trailer_nh;
+                        pw |= byte << (8 * b);
+                    }
+                    P = pw;
+                }
+                uint32_t C = P ^ ks[w & 3];
+                W0[k] = __funnelshift_rc(Cprev, C, sh);   // memory word k (LE)
+                Cprev = C;
+                Mcur = Mnext;
+                m = bswap32(C);
+            } else if (i == nmsg) {
+                m = 0x80000000u;
+            } else if (i == nblk * 16 - 1) {
+                m = total_bits;
+            } else {
+                m = 0;
+            }
+            W[w] = m;
+        }
+        sha1_compress(H, W);
+    }
+    // outer hash: opad state, message = inner digest (20 B)
+    uint32_t G[5];
+#pragma unroll
+    for (int i = 0; i < 5; i++) G[i] = __ldg(&sap->opad[i]);
+#pragma unroll
+    for (int i = 0; i < 16; i++) W[i] = i < 5 ? H[i] : (i == 5 ? 0x80000000u : (i == 15 ? (64u + 20u) * 8u : 0u));
+    sha1_compress(G, W);
+    // 3. ICV = first 12 bytes; memory words nK .. nK+3
+    const uint32_t icv[3] = {bswap32(G[0]), bswap32(G[1]), bswap32(G[2])};
+    W0[nK] = __funnelshift_rc(Cprev, icv[0], sh);
+    W0[nK + 1] = __funnelshift_rc(icv[0], icv[1], sh);
+    W0[nK + 2] = __funnelshift_rc(icv[1], icv[2], sh);
+    if (r) W0[nK + 3] = __funnelshift_rc(icv[2], 0u, sh);
+    return v.ip_end + 30 + p;
+}
+
+// ---------------------------------------------------------------- the kernel
+struct Pkt {
+    uint8_t *f;
+    uint32_t flen, orig_len;
+    uint64_t gidx;
+    uint32_t h[16];
+    PV v;
+    uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
+    bool alive;
+};
+
+struct Ctx {
+    const uint32_t *acl4, *acl6;
+    DpiCtx dpi;
+    const uint32_t *te, *ms_nib, *lb_nib;
+    uint32_t *vst;            // smem u32 hit counters (nullptr: global atomics)
+    uint64_t pol_f, pol_l;
+    uint32_t gtid;
+};
+
+__device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_t idx)
+{
+    if (C.vst) atomicAdd(&C.vst[idx - NFIX], 1u);
+    else atomicAdd(&P.stats[idx], 1ull);
+}
+
+struct Loc { uint8_t *f; uint32_t len; uint64_t gidx; };
+
+// locate packet g of the call: batch (binary search over batch starts), off/len loads
+__device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
+{
+    Loc r{nullptr, 0, 0};
+    if (!valid) return r;
+    uint32_t bi = 0;
+    if (P.n_batches > 1) {
+        uint32_t lo = 0, hi = P.n_batches - 1;
+        while (lo < hi) {
+            const uint32_t mid = (lo + hi + 1) >> 1;
+            if (P.batches[mid].start <= g) lo = mid; else hi = mid - 1;
+        }
+        bi = lo;
+    }
+    const BatchDev &B = P.batches[bi];
+    const uint32_t li = g - B.start;
+    r.f = B.arena + B.off[li];
+    r.len = B.len[li];
+    r.gidx = B.first + li;
+    return r;
+}
+
+__device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid, Pkt &k)
+{
+    k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false;
+    k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
+    k.out_len = k.flen;
+    if (!valid) return;
+    load_header(k.f, k.flen, k.h, C.pol_f);
+    k.alive = parse(k.h, k.f, k.flen, k.v);
+    if (!k.alive) k.drop = 0xFE;
+}
+
+// one NF of kind KIND at chain position pos (KIND compile-time)
+template <uint32_t KIND, int DM>
+__device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k, uint32_t pos)
+{
+    bool dropped = false;
+    if constexpr (KIND == NFC_ACL) {
+        const uint32_t r = nf_acl(C.acl4, C.acl6, P.acl, k.v);
+        const uint32_t rule = r & 0xFFFF;
+        k.acl_rule = rule;
+        var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
+        dropped = (r >> 31) != 0;
+    } else if constexpr (KIND == NFC_DPI) {
+        const Walk w = dpi_walk<DM>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
+        if (w.cnt == 1) {
+            // exactly one accept event: match set = output closure of that state (distinct, sorted)
+            const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
+            const uint32_t o0 = __ldg(P.dpi.out_off + st), o1 = __ldg(P.dpi.out_off + st + 1);
+            const uint32_t nm = o1 - o0;
+            const uint32_t slot = atomicAdd(P.match_count, nm);
+            uint32_t drop = 0;
+            for (uint32_t q = 0; q < nm; q++) {
+                const uint32_t id = __ldg(P.dpi.out_ids + o0 + q);
+                drop |= __ldg(P.dpi.pat_action + id);
+                if (slot + q < P.match_cap) { P.match_pkt[slot + q] = (uint32_t)k.gidx; P.match_pat[slot + q] = (uint16_t)id; }
+            }
+            if (slot + nm > P.match_cap)
+                atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
+            k.nmatch = nm;
+            dropped = drop != 0;
+        } else if (w.cnt > 1) {
+            const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
+                            P.match_cap, P.stats};
+            const uint32_t r = dpi_slow(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+            k.nmatch = r & 0x7FFFFFFFu;
+            dropped = (r >> 31) != 0;
+        }
+    } else if constexpr (KIND == NFC_LPM4) {
+        // DIR-24-8: at most two dependent table reads ("two memory accesses")
+        if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
+        uint32_t nh = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+        if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
+        if (nh == 0x7FFF || hbyte(k.h, 22) <= 1) dropped = true;
+        else {
+            const uint2 n = __ldg(P.l4.nh + nh);
+            const uint32_t pt = n.y >> 16;
+            forward_rewrite(k.f, k.h, k.v, n, __ldg(P.l4.pmac + pt), C.pol_f);
+            k.port = pt;
+        }
+    } else if constexpr (KIND == NFC_LPM6) {
+        if (k.v.fam != 6) { k.passmask |= 1u << pos; return; }
+        const uint32_t nh = lpm6_lookup(P.l6, k.v.dst);
+        if (nh == 0x7FFF || hbyte(k.h, 21) <= 1) dropped = true;
+        else {
+            const uint2 n = __ldg(P.l6.nh + nh);
+            const uint32_t pt = n.y >> 16;
+            forward_rewrite(k.f, k.h, k.v, n, __ldg(P.l6.pmac + pt), C.pol_f);
+            k.port = pt;
+        }
+    } else if constexpr (KIND == NFC_IPSEC) {
+        const uint32_t nl = nf_esp(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te);
+        k.esp_bytes = nl - 28 - k.v.l4_off;      // ciphertext bytes |C|
+        k.f -= 16;
+        k.flen = nl;
+        k.out_len = nl;
+        load_header(k.f, k.flen, k.h, C.pol_f);
+        parse(k.h, k.f, k.flen, k.v);             // later NFs see proto 50, ports 0
+    } else if constexpr (KIND == NFC_LB) {
+        const uint32_t hsh = toeplitz(C.lb_nib, k.v);
+        const uint32_t b = (uint32_t)(((uint64_t)hsh * P.lb.n_backends) >> 32);
+        k.lb_b = b;
+        k.port = __ldg(P.lb.port + b);
+        var_stat(P, C, P.st_lb + b);
+    }
+    if (dropped) { k.drop = pos; k.alive = false; }
+}
+
+// positions [POS, END) of a compile-time chain; SIG_ANY interprets P.kind
+template <uint32_t S, int DM, int POS, int END>
+__device__ __forceinline__ void run_fixed(const KParams &P, const Ctx &C, Pkt &k)
+{
+    if constexpr (POS < END) {
+        if (k.alive) nf_apply<sig_kind(S, POS), DM>(P, C, k, POS);
+        run_fixed<S, DM, POS + 1, END>(P, C, k);
+    }
+}
+template <int DM>
+__device__ __forceinline__ void run_any(const KParams &P, const Ctx &C, Pkt &k, uint32_t from, uint32_t to)
+{
+    for (uint32_t pos = from; pos < to && k.alive; pos++) {
+        switch (P.kind[pos]) {
+        case NFC_ACL: nf_apply<NFC_ACL, DM>(P, C, k, pos); break;
+        case NFC_DPI: nf_apply<NFC_DPI, DM>(P, C, k, pos); break;
+        case NFC_LPM4: nf_apply<NFC_LPM4, DM>(P, C, k, pos); break;
+        case NFC_LPM6: nf_apply<NFC_LPM6, DM>(P, C, k, pos); break;
+        case NFC_IPSEC: nf_apply<NFC_IPSEC, DM>(P, C, k, pos); break;
+        case NFC_LB: nf_apply<NFC_LB, DM>(P, C, k, pos); break;
+        }
+    }
+}
+// chain positions [0, esp) or [esp, n) (esp = n for chains without IPsec)
+template <uint32_t S, int DM, bool HEAD>
+__device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
+{
+    if constexpr (S == SIG_ANY) {
+        const uint32_t e = min(P.esp_pos, P.n_nf);
+        if (HEAD) run_any<DM>(P, C, k, 0, e);
+        else run_any<DM>(P, C, k, e, P.n_nf);
+    } else {
+        constexpr int N = (int)sig_n(S);
+        constexpr int E = sig_pos(S, NFC_IPSEC) == 0xFF ? N : (int)sig_pos(S, NFC_IPSEC);
+        if constexpr (HEAD) run_fixed<S, DM, 0, E>(P, C, k);
+        else run_fixed<S, DM, E, N>(P, C, k);
+    }
+}
+
+// Record store + counters of one warp's 32 packets into the warp's private slot.
+// Only independent counts are kept per warp (chain-position "in", "applied" and
+// the total drop count are derived at the flush).
+template <uint32_t S>
+__device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, bool valid, uint32_t g,
+                                        unsigned long long *ws, uint32_t lane)
+{
+    constexpr uint32_t M = sig_mask(S);
+    if (valid) {
+        if (k.drop != 0xFF) k.port = 0xFFFF;
+        const uint4 rec = make_uint4(k.drop | k.esp_sa << 8 | k.port << 16, k.acl_rule | k.lb_b << 16,
+                                     k.nmatch | k.out_len << 16, k.esp_seq);
+        st_stream16(reinterpret_cast<uint4 *>(P.rec) + g, rec, C.pol_f);
+    }
+    const uint32_t FULL = 0xFFFFFFFFu;
+    const bool fwd = valid && k.drop == 0xFF;
+    const uint32_t nv = __popc(__ballot_sync(FULL, valid));
+    const uint32_t nparse = __popc(__ballot_sync(FULL, valid && k.drop == 0xFE));
+    const uint32_t nfwd = __popc(__ballot_sync(FULL, fwd));
+    const uint32_t bin = __reduce_add_sync(FULL, valid ? k.orig_len : 0u);
+    const uint32_t bout = __reduce_add_sync(FULL, fwd ? k.out_len : 0u);
+    uint32_t pairs = 0, nesp = 0, eb = 0, eblk = 0;
+    if constexpr ((M & MASK_DPI) != 0) pairs = __reduce_add_sync(FULL, k.nmatch);
+    if constexpr ((M & MASK_IPSEC) != 0) {
+        const bool esp = k.esp_sa != 0xFF;
+        nesp = __popc(__ballot_sync(FULL, esp));
+        eb = __reduce_add_sync(FULL, esp ? k.esp_bytes : 0u);
+        eblk = __reduce_add_sync(FULL, esp ? (k.esp_bytes + 15) >> 4 : 0u);
+    }
+    if (lane == 0) {
+        ws[ST_PKTS] += nv;
+        ws[ST_FWD] += nfwd;
+        ws[ST_PARSE_DROP] += nparse;
+        ws[ST_BYTES_IN] += bin;
+        ws[ST_BYTES_OUT] += bout;
+        if constexpr ((M & MASK_DPI) != 0) ws[ST_DPI_PAIRS] += pairs;
+        if constexpr ((M & MASK_IPSEC) != 0) {
+            ws[ST_ESP_PKTS] += nesp;
+            ws[ST_ESP_BYTES] += eb;
+            ws[ST_ESP_BLOCKS] += eblk;
+        }
+    }
+    constexpr int NP = S == SIG_ANY ? NFC_MAX_CHAIN : (int)sig_n(S);
+#pragma unroll
+    for (int p = 0; p < NP; p++) {
+        if (S == SIG_ANY && (uint32_t)p >= P.n_nf) break;          // uniform
+        const uint32_t nd = __popc(__ballot_sync(FULL, valid && k.drop == (uint32_t)p));
+        const uint32_t kd = S == SIG_ANY ? P.kind[p] : sig_kind(S, p);
+        uint32_t np = 0;
+        if (kd == NFC_LPM4 || kd == NFC_LPM6) np = __popc(__ballot_sync(FULL, (k.passmask >> p) & 1));
+        if (lane == 0) {
+            ws[ST_POS_BASE + 4 * p + 1] += nd;
+            ws[ST_POS_BASE + 4 * p + 2] += np;
+        }
+    }
+}
+
+// ESP sequence numbers for one CTA tile: per SA, global packet order (decoupled look-back)
+template <int NW>
+__device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8_t *smem, const SmemLayout &L,
+                                           uint32_t tile, Pkt &k)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t nsa = P.esp.n_sa;
+    uint16_t *wcnt = reinterpret_cast<uint16_t *>(smem + L.wcnt);
+    uint32_t *pref = reinterpret_cast<uint32_t *>(smem + L.prefix);
+    for (uint32_t i = tid; i < NW * 256; i += NW * 32) wcnt[i] = 0;
+    uint32_t sa = 0xFFFF;
+    if (k.alive) sa = toeplitz(C.ms_nib, k.v) % nsa;
+    __syncthreads();
+    const uint32_t key = k.alive ? sa : (0x10000u + lane);
+    const uint32_t grp = __match_any_sync(0xFFFFFFFFu, key);
+    const uint32_t rank = __popc(grp & ((1u << lane) - 1));
+    if (k.alive && rank == 0) wcnt[warp * 256 + sa] = (uint16_t)__popc(grp);
+    __syncthreads();
+    if (warp == 0) {
+        uint32_t *vec = P.tile_vec + (size_t)tile * 2 * nsa;
+        for (uint32_t s = lane; s < nsa; s += 32) {
+            uint32_t run = 0;
+#pragma unroll
+            for (int w = 0; w < NW; w++) { const uint32_t c = wcnt[w * 256 + s]; wcnt[w * 256 + s] = (uint16_t)run; run += c; }
+            vec[s] = run;
+            pref[s] = 0;
+        }
+        __syncwarp();
+        if (tile > 0) {
+            if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 1u); }
+            int pt = (int)tile - 1;
+            for (;;) {
+                uint32_t fl;
+                do { fl = ld_acquire(P.tile_flag + pt); } while ((fl >> 2) != P.epoch || (fl & 3) == 0);
+                const uint32_t *pv = P.tile_vec + (size_t)pt * 2 * nsa;
+                const bool incl = (fl & 3) == 2;
+                for (uint32_t s = lane; s < nsa; s += 32) pref[s] += __ldcg(pv + (incl ? nsa : 0) + s);
+                if (incl) break;
+                pt--;
+            }
+        }
+        __syncwarp();
+        for (uint32_t s = lane; s < nsa; s += 32) vec[nsa + s] = pref[s] + vec[s];
+        __syncwarp();
+        if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 2u); }
+        if (tile == P.n_tiles - 1)
+            for (uint32_t s = lane; s < nsa; s += 32) P.seq_out[s] = P.seq_in[s] + pref[s] + vec[s];
+    }
+    __syncthreads();
+    if (k.alive) {
+        k.esp_sa = sa;
+        k.esp_seq = __ldg(P.seq_in + sa) + pref[sa] + wcnt[warp * 256 + sa] + rank + 1;
+        var_stat(P, C, P.st_sa + sa);
+    }
+}
+
+template <uint32_t S, int DM>
+__global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
+{
+    constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp;
+    extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ uint32_t s_tile;
+    const uint32_t mask = P.present & sig_mask(S);
+    const SmemLayout L = smem_layout(mask, NW, P);
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
+    uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
+    const uint32_t n_var = P.stats_len - NFIX;
+    for (uint32_t i = tid; i < NW * NWS; i += NT) wst[i] = 0;
+    if (P.smem_stats)
+        for (uint32_t i = tid; i < n_var; i += NT) vst[i] = 0;
+
+    Ctx C;
+    C.gtid = blockIdx.x * NT + tid;
+    C.vst = P.smem_stats ? vst : nullptr;
+    C.pol_f = pol_first();
+    C.pol_l = pol_last();
+    C.acl4 = C.acl6 = nullptr;
+    C.te = C.ms_nib = C.lb_nib = nullptr;
+    C.dpi.cls = reinterpret_cast<const uint32_t *>(smem + L.cls);
+    C.dpi.gcls = P.dpi.cls;
+    C.dpi.sm = smem;
+    C.dpi.hot = smem + L.hot;
+    C.dpi.row2 = 2 * P.dpi.ncls;
+    C.dpi.ncls = P.dpi.ncls;
+    C.dpi.wide = DM == DM_FULL ? 0 : P.dpi.wide;
+    C.dpi.trans = P.dpi.trans;
+    C.dpi.out_off = P.dpi.out_off;
+    C.dpi.out_ids = P.dpi.out_ids;
+    C.dpi.pat_action = P.dpi.pat_action;
+    C.dpi.H = 0;
+    C.dpi.HK2 = 0;
+    const bool has_esp = (sig_mask(S) & MASK_IPSEC) && P.esp_pos < P.n_nf;
+    if ((sig_mask(S) & MASK_ACL) && (mask & MASK_ACL)) {
+        if (P.acl.smem_words) {
+            uint4 *d4 = reinterpret_cast<uint4 *>(smem + L.acl4);
+            uint4 *d6 = reinterpret_cast<uint4 *>(smem + L.acl6);
+            for (uint32_t i = tid; i < P.acl.words4 / 4; i += NT) d4[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv4) + i);
+            for (uint32_t i = tid; i < P.acl.words6 / 4; i += NT) d6[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv6) + i);
+            C.acl4 = reinterpret_cast<const uint32_t *>(d4);
+            C.acl6 = reinterpret_cast<const uint32_t *>(d6);
+        } else {
+            C.acl4 = P.acl.bv4;
+            C.acl6 = P.acl.bv6;
+        }
+    }
+    if ((sig_mask(S) & MASK_DPI) && (mask & MASK_DPI)) {
+        uint32_t *cls = reinterpret_cast<uint32_t *>(smem + L.cls);
+        // DM_FULL: smem byte offset of the class column in row 0; DM_HOT: 2 * class
+        for (uint32_t i = tid; i < 256; i += NT) cls[i] = (DM == DM_FULL ? L.hot : 0u) + 2u * __ldg(P.dpi.cls + i);
+        const uint32_t H = C.dpi.wide ? 0 : P.dpi.hot_states;
+        uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
+        const uint16_t *tr = reinterpret_cast<const uint16_t *>(P.dpi.trans);
+        const uint32_t nh = H * P.dpi.ncls;
+        if ((nh & 7) == 0) {
+            for (uint32_t i = tid; i < nh / 8; i += NT) reinterpret_cast<uint4 *>(hot)[i] = __ldg(reinterpret_cast<const uint4 *>(tr) + i);
+        } else {
+            for (uint32_t i = tid; i < nh; i += NT) hot[i] = __ldg(tr + i);
+        }
+        C.dpi.H = H;
+        C.dpi.HK2 = H ? 2 * (H * P.dpi.ncls - 1) : 0;
+    }
+    if ((sig_mask(S) & MASK_IPSEC) && has_esp) {
+        uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
+        for (uint32_t i = tid; i < 256 * 32; i += NT) te[i] = __ldg(P.esp.te + (i >> 5));   // T0 x 32 lanes
+        for (uint32_t i = tid; i < 72 * 16; i += NT) mn[i] = __ldg(P.esp.rss_nib + i);
+        C.te = te + lane;         // this lane's bank column
+        C.ms_nib = mn;
+    }
+    if ((sig_mask(S) & MASK_LB) && (mask & MASK_LB)) {
+        uint32_t *ln = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
+        for (uint32_t i = tid; i < 72 * 16; i += NT) ln[i] = __ldg(P.lb.nib + i);
+        C.lb_nib = ln;
+    }
+    __syncthreads();
+    unsigned long long *ws = wst + warp * NWS;
+
+    if (!KCfg<S, DM>::esp || (S == SIG_ANY && !has_esp)) {
+        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA
+        // barriers; the next chunk is claimed and located (off/len loads, header
+        // prefetch to L2) before the current one is processed
+        auto claim = [&]() {
+            uint32_t b = 0;
+            if (lane == 0) b = atomicAdd(P.tile_counter, 32u);
+            return __shfl_sync(0xFFFFFFFFu, b, 0);
+        };
+        uint32_t c0 = claim();
+        Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
+        while (c0 < P.n_pkts) {
+            const uint32_t c1 = claim();
+            const Loc loc1 = pkt_locate(P, c1 + lane, c1 + lane < P.n_pkts);
+            if (c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(loc1.f));
+            const uint32_t g = c0 + lane;
+            const bool valid = g < P.n_pkts;
+            Pkt k;
+            pkt_begin(C, loc, valid, k);
+            run_part<S, DM, true>(P, C, k);
+            run_part<S, DM, false>(P, C, k);
+            pkt_end<S>(P, C, k, valid, g, ws, lane);
+            c0 = c1;
+            loc = loc1;
+        }
+    } else if constexpr (KCfg<S, DM>::esp) {
+        // CTA tiles claimed in global order (ESP sequence numbers need the order)
+        for (;;) {
+            if (tid == 0) s_tile = atomicAdd(P.tile_counter, 1u);
+            __syncthreads();
+            const uint32_t tile = s_tile;
+            __syncthreads();
+            if (tile >= P.n_tiles) break;
+            const uint32_t g = tile * NT + tid;
+            const bool valid = g < P.n_pkts;
+            Pkt k;
+            pkt_begin(C, pkt_locate(P, g, valid), valid, k);
+            run_part<S, DM, true>(P, C, k);
+            esp_assign<NW>(P, C, smem, L, tile, k);
+            run_part<S, DM, false>(P, C, k);
+            pkt_end<S>(P, C, k, valid, g, ws, lane);
+        }
+    }
+    // ---- flush CTA counters; derive drop total and per-position in / applied
+    __syncthreads();
+    if (warp == 0) {
+        unsigned long long t[2] = {0, 0};
+        const uint32_t i = lane;     // slots 0..31 by lane, 32..NWS-1 by lanes 0..NWS-33
+#pragma unroll
+        for (int r = 0; r < 2; r++) {
+            const uint32_t idx = i + 32 * r;
+            if (idx < NWS)
+                for (int w = 0; w < NW; w++) t[r] += wst[w * NWS + idx];
+        }
+        __syncwarp();
+        wst[i] = t[0];
+        if (i + 32 < NWS) wst[i + 32] = t[1];
+        __syncwarp();
+        if (lane == 0) {
+            wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
+            unsigned long long in = wst[ST_PKTS] - wst[ST_PARSE_DROP];
+            for (uint32_t p = 0; p < P.n_nf; p++) {
+                const unsigned long long d = wst[ST_POS_BASE + 4 * p + 1], ps = wst[ST_POS_BASE + 4 * p + 2];
+                wst[ST_POS_BASE + 4 * p] = in;
+                wst[ST_POS_BASE + 4 * p + 3] = in - d - ps;
+                in -= d;
+            }
+        }
+        __syncwarp();
+        for (uint32_t idx = lane; idx < NWS; idx += 32)
+            if (wst[idx]) atomicAdd(&P.stats[idx], wst[idx]);
+    }
+    if (P.smem_stats)
+        for (uint32_t i = tid; i < n_var; i += NT)
+            if (vst[i]) atomicAdd(&P.stats[NFIX + i], (unsigned long long)vst[i]);
+}
+
+// ---------------------------------------------------------------- host launch
+template <uint32_t S, int DM>
+int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCfg *cfg, bool query_only)
+{
+    constexpr int NT = KCfg<S, DM>::threads;
+    const size_t smem = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p).total;
+    static int attr_smem[64] = {0};   // per device: dynamic smem size already granted
+    static int per_sm_cache[64] = {0};
+    static size_t per_sm_smem[64] = {0};
+    const int d = dev & 63;
+    if ((int)smem > attr_smem[d]) {
+        if (cudaFuncSetAttribute(sfc_kernel<S, DM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+            err = "cudaFuncSetAttribute failed (shared memory " + std::to_string(smem) + " B)";
+            return NFC_ECUDA;
+        }
+        attr_smem[d] = (int)smem;
+    }
+    int per_sm = per_sm_cache[d];
+    if (!per_sm || per_sm_smem[d] != smem) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sfc_kernel<S, DM>, NT, smem);
+        if (per_sm < 1) per_sm = 1;
+        per_sm_cache[d] = per_sm;
+        per_sm_smem[d] = smem;
+    }
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    int grid = sms * per_sm;
+    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + 31) / 32 / KCfg<S, DM>::nwarp + 1;
+    if (!query_only && (uint32_t)grid > units) grid = (int)units;
+    if (grid < 1) grid = 1;
+    if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }
+    if (query_only) return NFC_OK;
+    sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(p);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { err = std::string("sfc_kernel launch: ") + cudaGetErrorString(e); return NFC_ECUDA; }
+    return NFC_OK;
+}
+
+// chain signatures with dedicated instantiations (sfc_inst_*.cu)
+static constexpr uint32_t SIG_C1 = make_sig(3, NFC_ACL, NFC_DPI, NFC_LPM4);                       // also C5 k=3
+static constexpr uint32_t SIG_C2 = make_sig(1, NFC_IPSEC);
+static constexpr uint32_t SIG_C3 = make_sig(3, NFC_ACL, NFC_DPI, NFC_LB);
+static constexpr uint32_t SIG_C4 = make_sig(5, NFC_ACL, NFC_LPM6, NFC_DPI, NFC_IPSEC, NFC_LB);
+static constexpr uint32_t SIG_K1 = make_sig(1, NFC_ACL);
+static constexpr uint32_t SIG_K2 = make_sig(2, NFC_ACL, NFC_DPI);
+static constexpr uint32_t SIG_K4 = make_sig(4, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6);
+static constexpr uint32_t SIG_K5 = make_sig(5, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6, NFC_IPSEC);
+static constexpr uint32_t SIG_K6 = make_sig(6, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6, NFC_IPSEC, NFC_LB);
+
+#define NFC_DECLARE_LAUNCH(S, DM)                                                                   \
+    extern template int launch_t<S, DM>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+#define NFC_INSTANTIATE_LAUNCH(S, DM)                                                               \
+    template int launch_t<S, DM>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+
+} // namespace nfc
