@@ -278,6 +278,15 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
     o.out_off[n] = (uint32_t)o.out_ids.size();
     if (o.out_ids.empty()) o.out_ids.push_back(0);
     o.action.assign(s.action, s.action + s.n_patterns);
+    // per-state match summary for the kernel's single-accept path: closure offset,
+    // size and whether any pattern in it is a DROP pattern
+    o.out_meta.assign(n, 0);
+    for (size_t k = 0; k < n; k++) {
+        const uint32_t o0 = o.out_off[k], nm = o.out_off[k + 1] - o0;
+        uint32_t drop = 0;
+        for (uint32_t x = o0; x < o0 + nm; x++) drop |= o.action[o.out_ids[x]];
+        o.out_meta[k] = (o0 < (1u << 20) && nm < 2047u) ? (o0 | nm << 20 | drop << 31) : DPI_META_NONE;
+    }
     return "";
 }
 

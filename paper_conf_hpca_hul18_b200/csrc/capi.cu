@@ -65,7 +65,7 @@ struct nfc_chain {
     // tables
     DBuf acl_r4, acl_r6;
     AclImg acl{};
-    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap;
+    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta;
     DpiImg dpi{};
     DBuf l4_tbl24, l4_long, l4_nh, l4_pmac;
     Lpm4Img l4{};
@@ -150,7 +150,7 @@ void nfc_destroy_chain(nfc_chain *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
-                   &c->dpi_bitmap, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
+                   &c->dpi_bitmap, &c->dpi_meta, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
@@ -202,7 +202,9 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
         CK(c->dpi_off.upload(d.out_off));
         CK(c->dpi_ids.upload(d.out_ids));
         CK(c->dpi_act.upload(d.action));
+        CK(c->dpi_meta.upload(d.out_meta));
         c->dpi = DpiImg{};
+        c->dpi.out_meta = c->dpi_meta.as<uint32_t>();
         c->dpi.cls = c->dpi_cls.as<uint8_t>();
         c->dpi.trans = c->dpi_trans.p;
         c->dpi.ncls = d.ncls;
@@ -315,6 +317,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     p.esp_pos = c->esp_pos;
     p.present = c->mask;
     p.batches = c->batches.as<BatchDev>();
+    p.b0 = hb[0];
     p.n_batches = nb;
     p.n_pkts = (uint32_t)total;
     p.n_tiles = n_tiles;
@@ -365,10 +368,12 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         p.acl.smem_words = (c->mask & MASK_ACL) ? 1 : 0;
         p.dpi.hot_states = 0;
         bool full = false;
-        if ((c->mask & MASK_DPI) && !c->dpi.wide) {
+        if ((c->mask & MASK_DPI) && !c->dpi.wide && c->dpi.ncls <= 128) {
             Variant vf = sfc_variant(c->kind, c->n_nf, true);
             if (vf.dm == DM_FULL) {
                 p.dpi.hot_states = c->dpi.n_states;
+                p.dpi.meta_smem = 1;
+                if (sfc_smem_bytes(vf, p) + 1024 > limit) p.dpi.meta_smem = 0;
                 if (sfc_smem_bytes(vf, p) + 1024 <= limit) { v = vf; full = true; }
                 else p.dpi.hot_states = 0;
             }

@@ -47,7 +47,11 @@ struct DpiImg {
     uint32_t *ovf_bitmap;        // per resident thread scratch for > DPI_LIST distinct matches
     uint32_t bitmap_words;       // words per thread
     uint32_t hot_states;         // states whose full 256-byte rows are staged in shared memory
+    const uint32_t *out_meta;    // per state: out_off | n_out << 20 | any DROP pattern << 31
+                                 // (DPI_META_NONE if the closure does not fit the fields)
+    uint32_t meta_smem;          // 1: out_meta staged in shared memory
 };
+static const uint32_t DPI_META_NONE = 0x7FFFFFFFu;
 
 // ---------------------------------------------------------------- LPM4 (DIR-24-8)
 // tbl24[dst>>8]: bit 15 set -> long group g = v & 0x7FFF, nh = tbllong[g*256 + (dst&255)];
@@ -117,6 +121,7 @@ struct KParams {
     uint32_t present;            // MASK_* bits of the NFs in the chain
     // work
     const BatchDev *batches;
+    BatchDev b0;                 // batches[0] (constant bank: no descriptor loads for single-batch calls)
     uint32_t n_batches;
     uint32_t n_pkts;
     uint32_t n_tiles;
@@ -156,6 +161,7 @@ struct DpiHost {
     std::vector<uint32_t> out_off;
     std::vector<uint16_t> out_ids;
     std::vector<uint8_t> action;
+    std::vector<uint32_t> out_meta;
 };
 std::string build_dpi(const nfc_dpi_spec &s, DpiHost &out);
 std::string build_lpm4(const nfc_lpm4_spec &s, std::vector<uint16_t> &tbl24, std::vector<uint16_t> &tbllong,

@@ -59,16 +59,22 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 }
 
 
+#ifndef NFC_FULL_THREADS
+#define NFC_FULL_THREADS 768   // DM_FULL: one CTA per SM
+#endif
+#ifndef NFC_HOT_MINB
+#define NFC_HOT_MINB 3         // DM_HOT chains without IPsec: resident 256-thread CTAs per SM
+#endif
 template <uint32_t S, int DM> struct KCfg {
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
-    static constexpr int threads = (DM == DM_FULL && (S != SIG_ANY) && !esp) ? 768 : 256;
-    static constexpr int minb = esp ? 2 : (DM == DM_FULL ? 1 : 3);
+    static constexpr int threads = (DM == DM_FULL && (S != SIG_ANY) && !esp) ? NFC_FULL_THREADS : 256;
+    static constexpr int minb = esp ? 2 : (DM == DM_FULL ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
 };
 
 // ---------------------------------------------------------------- shared memory layout
 struct SmemLayout {
-    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, acl4, acl6, wcnt, prefix, total;
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, meta, acl4, acl6, wcnt, prefix, total;
 };
 __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, const KParams &p)
 {
@@ -79,7 +85,11 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
-    if (mask & MASK_DPI) { L.cls = o; o += 256 * 4; L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u; }
+    if (mask & MASK_DPI) {
+        L.cls = o; o += 256 * 4;
+        L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u;
+        L.meta = o; o += p.dpi.meta_smem ? (p.dpi.n_states * 4 + 15) & ~15u : 0;
+    }
     o = (o + 15) & ~15u;
     if (mask & MASK_ACL) {
         const uint32_t s4 = p.acl.smem_words ? p.acl.words4 : 0, s6 = p.acl.smem_words ? p.acl.words6 : 0;
@@ -184,6 +194,31 @@ static __device__ __noinline__ uint32_t tcp_doff_mem(const uint8_t *f, uint32_t 
 // Parse (P:L87 validity check): Ethernet -> IPv4/IPv6 -> UDP/TCP.
 __device__ __forceinline__ bool parse(const uint32_t h[16], const uint8_t *f, uint32_t flen, PV &v)
 {
+    // fast path, the common frames: Ethernet / IPv4 (IHL 5, not a fragment) / UDP or TCP
+    // with the L4 header in the header cache (words are little-endian: byte 12 is the
+    // low byte of h[3]); anything else, valid or not, takes the general parse below
+    {
+        const uint32_t pr = h[5] >> 24;
+        if ((h[3] & 0x00FFFFFFu) == 0x00450008u && (h[5] & 0x0000FF3Fu) == 0 && (pr == 17 || pr == 6)) {
+            const uint32_t tot = __byte_perm(h[4], 0, 0x4401);
+            const uint32_t doff = (h[11] >> 20) & 15;                  // TCP data offset, byte 46
+            const uint32_t l4len = pr == 6 ? 4 * doff : 8;
+            if (14 + tot <= flen && l4len + 20 <= tot && (pr == 17 || doff >= 5)) {
+                v.fam = 4;
+                v.l4_off = 34;
+                v.ip_end = 14 + tot;
+                v.pl_off = 34 + l4len;
+                v.proto = pr;
+                v.src[0] = __byte_perm(h[6], h[7], 0x2345);
+                v.dst[0] = __byte_perm(h[7], h[8], 0x2345);
+                v.src[1] = v.src[2] = v.src[3] = v.dst[1] = v.dst[2] = v.dst[3] = 0;
+                const uint32_t ports = __byte_perm(h[8], h[9], 0x2345);
+                v.sport = ports >> 16;
+                v.dport = ports & 0xFFFF;
+                return true;
+            }
+        }
+    }
     if (flen < 14) return false;
     const uint32_t et = hbe16(h, 12);
     bool frag = false;
@@ -311,8 +346,8 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
 // Aho-Corasick DFA walk over byte classes.  Transition entries are u16: next
 // state | ACCEPT << 15 (ACCEPT: the next state has a non-empty output set); u32
 // with ACCEPT << 31 above 32K states ("wide").
-//   DM_FULL: all rows in shared memory; cls[b] = smem byte offset of column
-//            class(b) in row 0, so a step is IMAD + LDS.
+//   DM_FULL: all rows in shared memory; cls8[b] = 2*class(b) (u8, ncls <= 128),
+//            so a step is PRMT (byte) + LDS.U8 (class) + IMAD + LDS.U16.
 //   DM_HOT:  the first H states (BFS order) in shared memory, cls[b] = 2*class(b);
 //            cold states read the global table (predicated load).
 // A walk keeps three registers: s (state), cnt (accept events), mx (max entry
@@ -320,7 +355,8 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
 // state after the only accept event is mx & 0x7FFF and the match set is its
 // output closure; cnt > 1 takes the exact re-walk (dpi_slow).
 struct DpiCtx {
-    const uint32_t *cls;    // smem, 256 entries
+    const uint32_t *cls;    // smem, 256 entries (DM_HOT)
+    const uint8_t *cls8;    // smem, 256 entries (DM_FULL)
     const uint8_t *gcls;    // global byte -> class table (exact re-walk)
     const uint8_t *sm;      // smem base (DM_FULL addressing)
     const uint8_t *hot;     // smem hot rows (DM_HOT)
@@ -335,12 +371,14 @@ struct DpiCtx {
 
 struct Walk { uint32_t s, cnt, mx; };
 
+// byte k (compile-time) of a little-endian word, zero-extended: one PRMT
+__device__ __forceinline__ uint32_t byte_of(uint32_t w, int k) { return __byte_perm(w, 0, 0x4440 + k); }
+
 template <int DM>
 __device__ __forceinline__ uint32_t dfa_entry(const DpiCtx &c, uint32_t s, uint32_t byte)
 {
-    const uint32_t cv = c.cls[byte];
-    if (DM == DM_FULL) return *reinterpret_cast<const uint16_t *>(c.sm + (s * c.row2 + cv));
-    const uint32_t k2 = s * c.row2 + cv;
+    if (DM == DM_FULL) return *reinterpret_cast<const uint16_t *>(c.hot + (s * c.row2 + c.cls8[byte]));
+    const uint32_t k2 = s * c.row2 + c.cls[byte];
     const uint32_t e = *reinterpret_cast<const uint16_t *>(c.hot + min(k2, c.HK2));
     return ld_u16_if(s >= c.H, reinterpret_cast<const uint16_t *>(reinterpret_cast<const uint8_t *>(c.trans) + k2), e);
 }
@@ -370,12 +408,26 @@ __device__ __forceinline__ void dfa_step_wide(const DpiCtx &c, Walk &w, uint32_t
     w.mx = max(w.mx, e);
 }
 
+// DM_HOT: make a payload word depend on the walk state so the class lookups of its
+// bytes are not hoisted far ahead of the walk (that raises register pressure past the
+// occupancy budget and spills); DM_FULL has the registers to spare
+template <int DM>
+__device__ __forceinline__ uint32_t tie(uint32_t word, const Walk &w)
+{
+    if (DM == DM_HOT) asm("" : "+r"(word) : "r"(w.s));
+    return word;
+}
+
 // payload bytes [A, 64) of the header cache, A compile-time: no per-byte guards
 template <int DM, int A>
 __device__ __forceinline__ void walk_cached(const DpiCtx &c, const uint32_t h[16], Walk &w)
 {
+    uint32_t wd = tie<DM>(h[A >> 2], w);
 #pragma unroll
-    for (int idx = A; idx < 64; idx++) dfa_step<DM>(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF);
+    for (int idx = A; idx < 64; idx++) {
+        if ((idx & 3) == 0) wd = tie<DM>(h[idx >> 2], w);
+        dfa_step<DM>(c, w, byte_of(wd, idx & 3));
+    }
 }
 
 // walk of a DFA with > 32K states (u32 entries, all rows in global memory); not inlined
@@ -407,19 +459,30 @@ __device__ __forceinline__ Walk dpi_walk(const DpiCtx &c, const uint32_t h[16], 
     else if (b >= 64 && a == 62) walk_cached<DM, 62>(c, h, w);   // IPv6 UDP
     else if (b >= 64 && a == 54) walk_cached<DM, 54>(c, h, w);   // IPv4 TCP
     else {
+        uint32_t wd = 0;
 #pragma unroll
-        for (int idx = 32; idx < 64; idx++)
-            dfa_step_if<DM>(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, (uint32_t)idx - a < b - a);
+        for (int idx = 32; idx < 64; idx++) {
+            if ((idx & 3) == 0) wd = tie<DM>(h[idx >> 2], w);
+            dfa_step_if<DM>(c, w, byte_of(wd, idx & 3), (uint32_t)idx - a < b - a);
+        }
     }
     for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
         const uint4 q = ld_stream16(f + ch, pol);
-        const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+        uint32_t wd[4] = {q.x, q.y, q.z, q.w};
         if (ch >= a && ch + 16 <= b) {
 #pragma unroll
-            for (int k = 0; k < 16; k++) dfa_step<DM>(c, w, (wd[k >> 2] >> ((k & 3) * 8)) & 0xFF);
+            for (int k = 0; k < 16; k++) {
+                const uint32_t x = (k & 3) == 0 ? tie<DM>(wd[k >> 2], w) : wd[k >> 2];
+                if ((k & 3) == 0) wd[k >> 2] = x;
+                dfa_step<DM>(c, w, byte_of(x, k & 3));
+            }
         } else {
 #pragma unroll
-            for (int k = 0; k < 16; k++) dfa_step_if<DM>(c, w, (wd[k >> 2] >> ((k & 3) * 8)) & 0xFF, ch + k - a < b - a);
+            for (int k = 0; k < 16; k++) {
+                const uint32_t x = (k & 3) == 0 ? tie<DM>(wd[k >> 2], w) : wd[k >> 2];
+                if ((k & 3) == 0) wd[k >> 2] = x;
+                dfa_step_if<DM>(c, w, byte_of(x, k & 3), ch + k - a < b - a);
+            }
         }
     }
     return w;
@@ -789,13 +852,29 @@ struct Pkt {
     uint32_t h[16];
     PV v;
     uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
+    uint32_t t24;             // TBL24 entry, loaded right after parse (NFC_EARLY_T24)
+    uint32_t mmeta, mslot;    // deferred match-pair emission: closure meta, first pair slot
     bool alive;
 };
+
+#ifndef NFC_EARLY_T24
+#define NFC_EARLY_T24 0       // issue the DIR-24-8 first read right after parse, use it at LPM4
+#endif
+#ifndef NFC_DEFER_PAIRS
+#define NFC_DEFER_PAIRS 0     // 1: claim match-pair slots at DPI, write the pairs at the end of the chunk
+#endif
+#ifndef NFC_LOOKBACK_WIN
+#define NFC_LOOKBACK_WIN 1    // ESP sequence look-back over 32 predecessor tiles per step
+#endif
+#ifndef NFC_CLAIM
+#define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic
+#endif
 
 struct Ctx {
     const uint32_t *acl4, *acl6;
     DpiCtx dpi;
     const uint32_t *te, *ms_nib, *lb_nib;
+    const uint32_t *meta;     // per-state match summary (smem or global)
     uint32_t *vst;            // smem u32 hit counters (nullptr: global atomics)
     uint64_t pol_f, pol_l;
     uint32_t gtid;
@@ -808,39 +887,71 @@ __device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_
 }
 
 struct Loc { uint8_t *f; uint32_t len; uint64_t gidx; };
+struct Raw { uint64_t off; uint32_t len, bi; };   // a packet's descriptor loads (issued early)
 
-// locate packet g of the call: batch (binary search over batch starts), off/len loads
+// batch of packet g (binary search over batch starts) and its off/len loads
+__device__ __forceinline__ Raw pkt_raw(const KParams &P, uint32_t g, bool valid)
+{
+    Raw r{0, 0, 0};
+    if (!valid) return r;
+    if (P.n_batches == 1) {
+        r.off = P.b0.off[g];
+        r.len = P.b0.len[g];
+        return r;
+    }
+    uint32_t lo = 0, hi = P.n_batches - 1;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (P.batches[mid].start <= g) lo = mid; else hi = mid - 1;
+    }
+    const BatchDev &B = P.batches[lo];
+    r.off = B.off[g - B.start];
+    r.len = B.len[g - B.start];
+    r.bi = lo;
+    return r;
+}
+__device__ __forceinline__ Loc pkt_loc(const KParams &P, const Raw &r, uint32_t g, bool valid)
+{
+    Loc l{nullptr, 0, 0};
+    if (!valid) return l;
+    if (P.n_batches == 1) {
+        l.f = P.b0.arena + r.off;
+        l.gidx = P.b0.first + g;
+    } else {
+        const BatchDev &B = P.batches[r.bi];
+        l.f = B.arena + r.off;
+        l.gidx = B.first + (g - B.start);
+    }
+    l.len = r.len;
+    return l;
+}
 __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
 {
-    Loc r{nullptr, 0, 0};
-    if (!valid) return r;
-    uint32_t bi = 0;
-    if (P.n_batches > 1) {
-        uint32_t lo = 0, hi = P.n_batches - 1;
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi + 1) >> 1;
-            if (P.batches[mid].start <= g) lo = mid; else hi = mid - 1;
-        }
-        bi = lo;
-    }
-    const BatchDev &B = P.batches[bi];
-    const uint32_t li = g - B.start;
-    r.f = B.arena + B.off[li];
-    r.len = B.len[li];
-    r.gidx = B.first + li;
-    return r;
+    return pkt_loc(P, pkt_raw(P, g, valid), g, valid);
 }
 
 __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid, Pkt &k)
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
-    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
     k.out_len = k.flen;
     if (!valid) return;
     load_header(k.f, k.flen, k.h, C.pol_f);
     k.alive = parse(k.h, k.f, k.flen, k.v);
     if (!k.alive) k.drop = 0xFE;
+}
+
+// (packet, pattern) pairs of an output closure [o0, o0+nm) at slots [slot, slot+nm)
+__device__ __forceinline__ void emit_pairs(const KParams &P, uint32_t o0, uint32_t nm, uint32_t slot, uint32_t pkt)
+{
+    for (uint32_t q = 0; q < nm; q++)
+        if (slot + q < P.match_cap) {
+            P.match_pkt[slot + q] = pkt;
+            P.match_pat[slot + q] = __ldg(P.dpi.out_ids + o0 + q);
+        }
+    if (slot + nm > P.match_cap)
+        atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
 }
 
 // one NF of kind KIND at chain position pos (KIND compile-time)
@@ -856,23 +967,23 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         dropped = (r >> 31) != 0;
     } else if constexpr (KIND == NFC_DPI) {
         const Walk w = dpi_walk<DM>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
-        if (w.cnt == 1) {
-            // exactly one accept event: match set = output closure of that state (distinct, sorted)
-            const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
-            const uint32_t o0 = __ldg(P.dpi.out_off + st), o1 = __ldg(P.dpi.out_off + st + 1);
-            const uint32_t nm = o1 - o0;
-            const uint32_t slot = atomicAdd(P.match_count, nm);
-            uint32_t drop = 0;
-            for (uint32_t q = 0; q < nm; q++) {
-                const uint32_t id = __ldg(P.dpi.out_ids + o0 + q);
-                drop |= __ldg(P.dpi.pat_action + id);
-                if (slot + q < P.match_cap) { P.match_pkt[slot + q] = (uint32_t)k.gidx; P.match_pat[slot + q] = (uint16_t)id; }
-            }
-            if (slot + nm > P.match_cap)
-                atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
+        const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
+        const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
+        if (w.cnt == 1 && meta != DPI_META_NONE) {
+            // exactly one accept event: the match set is the output closure of that state
+            // (distinct ids); its size and DROP flag come from the per-state summary.  The
+            // pair slots are claimed now and the pairs written at the end of the chunk, so
+            // the atomic's latency overlaps the rest of the chain.
+            const uint32_t nm = (meta >> 20) & 0x7FF;
             k.nmatch = nm;
-            dropped = drop != 0;
-        } else if (w.cnt > 1) {
+            dropped = (meta >> 31) != 0;
+#if NFC_DEFER_PAIRS
+            k.mmeta = meta & 0x7FFFFFFFu;
+            k.mslot = atomicAdd(P.match_count, nm);
+#else
+            emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
+#endif
+        } else if (w.cnt >= 1) {
             const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                             P.match_cap, P.stats};
             const uint32_t r = dpi_slow(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
@@ -882,7 +993,7 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
     } else if constexpr (KIND == NFC_LPM4) {
         // DIR-24-8: at most two dependent table reads ("two memory accesses")
         if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
-        uint32_t nh = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+        uint32_t nh = k.t24 != 0xFFFFFFFFu ? k.t24 : ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
         if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
         if (nh == 0x7FFF || hbyte(k.h, 22) <= 1) dropped = true;
         else {
@@ -946,6 +1057,13 @@ __device__ __forceinline__ void run_any(const KParams &P, const Ctx &C, Pkt &k, 
 template <uint32_t S, int DM, bool HEAD>
 __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
 {
+    if constexpr (HEAD && NFC_EARLY_T24 && S != SIG_ANY && sig_pos(S, NFC_LPM4) != 0xFF && sig_pos(S, NFC_LPM4) != 0) {
+        // header-phase read of the DIR-24-8 first level: its latency overlaps the NFs
+        // before LPM4 (a later NF may rewrite only the IPsec-moved header, and IPsec is
+        // never placed before LPM4 in the instantiated signatures)
+        static_assert(sig_pos(S, NFC_IPSEC) == 0xFF || sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4), "");
+        if (k.alive && k.v.fam == 4) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+    }
     if constexpr (S == SIG_ANY) {
         const uint32_t e = min(P.esp_pos, P.n_nf);
         if (HEAD) run_any<DM>(P, C, k, 0, e);
@@ -966,6 +1084,8 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
                                         unsigned long long *ws, uint32_t lane)
 {
     constexpr uint32_t M = sig_mask(S);
+    if constexpr ((M & MASK_DPI) != 0 && NFC_DEFER_PAIRS)
+        if (k.mmeta) emit_pairs(P, k.mmeta & 0xFFFFF, k.mmeta >> 20, k.mslot, (uint32_t)k.gidx);
     if (valid) {
         if (k.drop != 0xFF) k.port = 0xFFFF;
         const uint4 rec = make_uint4(k.drop | k.esp_sa << 8 | k.port << 16, k.acl_rule | k.lb_b << 16,
@@ -1045,6 +1165,29 @@ __device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8
         __syncwarp();
         if (tile > 0) {
             if (lane == 0) { __threadfence(); st_release(P.tile_flag + tile, P.epoch << 2 | 1u); }
+#if NFC_LOOKBACK_WIN
+            // windowed decoupled look-back: lane j watches tile base-j; the window stops at
+            // the nearest tile with an inclusive prefix (or before tile 0); the aggregates
+            // of the tiles in front of it are summed in parallel
+            int base = (int)tile - 1;
+            for (;;) {
+                const int pt = base - (int)lane;
+                uint32_t fl = 2;
+                if (pt >= 0)
+                    do { fl = ld_acquire(P.tile_flag + pt); } while ((fl >> 2) != P.epoch || (fl & 3) == 0);
+                const uint32_t stop = __ballot_sync(0xFFFFFFFFu, pt < 0 || (fl & 3) == 2);
+                const int d = stop ? __ffs(stop) - 1 : 32;          // aggregates before the stop lane
+                const bool incl = stop && base - d >= 0;            // stop lane holds an inclusive prefix
+                for (uint32_t s = lane; s < nsa; s += 32) {
+                    uint32_t acc = 0;
+                    for (int j = 0; j < d; j++) acc += __ldcg(P.tile_vec + (size_t)(base - j) * 2 * nsa + s);
+                    if (incl) acc += __ldcg(P.tile_vec + (size_t)(base - d) * 2 * nsa + nsa + s);
+                    pref[s] += acc;
+                }
+                if (stop) break;
+                base -= 32;
+            }
+#else
             int pt = (int)tile - 1;
             for (;;) {
                 uint32_t fl;
@@ -1055,6 +1198,7 @@ __device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8
                 if (incl) break;
                 pt--;
             }
+#endif
         }
         __syncwarp();
         for (uint32_t s = lane; s < nsa; s += 32) vec[nsa + s] = pref[s] + vec[s];
@@ -1095,6 +1239,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     C.acl4 = C.acl6 = nullptr;
     C.te = C.ms_nib = C.lb_nib = nullptr;
     C.dpi.cls = reinterpret_cast<const uint32_t *>(smem + L.cls);
+    C.dpi.cls8 = smem + L.cls;
     C.dpi.gcls = P.dpi.cls;
     C.dpi.sm = smem;
     C.dpi.hot = smem + L.hot;
@@ -1107,6 +1252,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     C.dpi.pat_action = P.dpi.pat_action;
     C.dpi.H = 0;
     C.dpi.HK2 = 0;
+    C.meta = P.dpi.meta_smem ? reinterpret_cast<const uint32_t *>(smem + L.meta) : P.dpi.out_meta;
     const bool has_esp = (sig_mask(S) & MASK_IPSEC) && P.esp_pos < P.n_nf;
     if ((sig_mask(S) & MASK_ACL) && (mask & MASK_ACL)) {
         if (P.acl.smem_words) {
@@ -1122,9 +1268,13 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         }
     }
     if ((sig_mask(S) & MASK_DPI) && (mask & MASK_DPI)) {
-        uint32_t *cls = reinterpret_cast<uint32_t *>(smem + L.cls);
-        // DM_FULL: smem byte offset of the class column in row 0; DM_HOT: 2 * class
-        for (uint32_t i = tid; i < 256; i += NT) cls[i] = (DM == DM_FULL ? L.hot : 0u) + 2u * __ldg(P.dpi.cls + i);
+        // 2 * class: u8 for DM_FULL (ncls <= 128), u32 for DM_HOT
+        if (DM == DM_FULL) {
+            for (uint32_t i = tid; i < 256; i += NT) smem[L.cls + i] = (uint8_t)(2u * __ldg(P.dpi.cls + i));
+        } else {
+            uint32_t *cls = reinterpret_cast<uint32_t *>(smem + L.cls);
+            for (uint32_t i = tid; i < 256; i += NT) cls[i] = 2u * __ldg(P.dpi.cls + i);
+        }
         const uint32_t H = C.dpi.wide ? 0 : P.dpi.hot_states;
         uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
         const uint16_t *tr = reinterpret_cast<const uint16_t *>(P.dpi.trans);
@@ -1136,6 +1286,10 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         }
         C.dpi.H = H;
         C.dpi.HK2 = H ? 2 * (H * P.dpi.ncls - 1) : 0;
+        if (P.dpi.meta_smem) {
+            uint32_t *mt = reinterpret_cast<uint32_t *>(smem + L.meta);
+            for (uint32_t i = tid; i < P.dpi.n_states; i += NT) mt[i] = __ldg(P.dpi.out_meta + i);
+        }
     }
     if ((sig_mask(S) & MASK_IPSEC) && has_esp) {
         uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
@@ -1153,19 +1307,31 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     unsigned long long *ws = wst + warp * NWS;
 
     if (!KCfg<S, DM>::esp || (S == SIG_ANY && !has_esp)) {
-        // warp-granular persistent loop: 32 consecutive packets per claim, no CTA
-        // barriers; the next chunk is claimed and located (off/len loads, header
+        // warp-granular persistent loop: chunks of 32 consecutive packets (NFC_CLAIM
+        // chunks per atomic claim), no CTA barriers; the next chunk is claimed and located (off/len loads, header
         // prefetch to L2) before the current one is processed
-        auto claim = [&]() {
-            uint32_t b = 0;
-            if (lane == 0) b = atomicAdd(P.tile_counter, 32u);
-            return __shfl_sync(0xFFFFFFFFu, b, 0);
+        uint32_t cbase = 0, cleft = 0;
+        auto claim = [&]() {                 // next 32-packet chunk; one atomic per NFC_CLAIM chunks
+            if (cleft == 0) {
+                uint32_t b = 0;
+                if (lane == 0) b = atomicAdd(P.tile_counter, 32u * NFC_CLAIM);
+                cbase = __shfl_sync(0xFFFFFFFFu, b, 0);
+                cleft = NFC_CLAIM;
+            }
+            const uint32_t c = cbase;
+            cbase += 32;
+            cleft--;
+            return c;
         };
-        uint32_t c0 = claim();
+        // software pipeline over chunks: descriptors (off/len) of chunk c2 are loaded two
+        // iterations ahead, the frame of chunk c1 is prefetched into L2 one ahead
+        uint32_t c0 = claim(), c1 = claim();
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
+        Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
         while (c0 < P.n_pkts) {
-            const uint32_t c1 = claim();
-            const Loc loc1 = pkt_locate(P, c1 + lane, c1 + lane < P.n_pkts);
+            const uint32_t c2 = claim();
+            const Raw raw2 = pkt_raw(P, c2 + lane, c2 + lane < P.n_pkts);
+            const Loc loc1 = pkt_loc(P, raw1, c1 + lane, c1 + lane < P.n_pkts);
             if (c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(loc1.f));
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
@@ -1175,7 +1341,9 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             run_part<S, DM, false>(P, C, k);
             pkt_end<S>(P, C, k, valid, g, ws, lane);
             c0 = c1;
+            c1 = c2;
             loc = loc1;
+            raw1 = raw2;
         }
     } else if constexpr (KCfg<S, DM>::esp) {
         // CTA tiles claimed in global order (ESP sequence numbers need the order)
@@ -1256,7 +1424,7 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     int grid = sms * per_sm;
-    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + 31) / 32 / KCfg<S, DM>::nwarp + 1;
+    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + 32 * NFC_CLAIM - 1) / (32 * NFC_CLAIM) / KCfg<S, DM>::nwarp + 1;
     if (!query_only && (uint32_t)grid > units) grid = (int)units;
     if (grid < 1) grid = 1;
     if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }
