@@ -45,6 +45,8 @@ def parse_args():
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-unfused", action="store_true", help="skip the NEXT-1 unfused baseline timing")
+    ap.add_argument("--unfused", action="store_true", help="time the unfused baseline as the main arm")
     return ap.parse_args()
 
 
@@ -275,7 +277,7 @@ def main():
     n = ring_packets(w, args.ring_mb)
     first = rank * n                       # flows of rank r: its own slice of the global stream
     b = nfcgen.generate(w.traffic, w.tables, first, n)
-    chain = nfc.Chain(w.kinds, device=local_dev)
+    chain = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_UNFUSED if args.unfused else 0)
     chain.load_tables(w.tables)
     hr, tr = chain.room()
     assert hr <= w.traffic.headroom and tr <= w.traffic.tailroom
@@ -407,6 +409,37 @@ def main():
                "steps": len(times), "api": "nfc_process_host (pinned host buffers)"}
         chain.stats(reset=True)
 
+    # NEXT-1: the same chain as one kernel per NF with a device-side
+    # re-split between NFs, timed on the same ring -- the fusion benefit on B200
+    unfused = None
+    if not args.no_unfused and not args.unfused and "IPSEC" not in w.kinds:
+        uch = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_UNFUSED)
+        uch.load_tables(w.tables)
+
+        def ustep():
+            mc.zero_()
+            uch.process(desc, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+        for _ in range(args.warmup):
+            ustep()
+        torch.cuda.synchronize(dev)
+        l0 = uch.launches()
+        ue0, ue1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ue0.record(stream)
+        for _ in range(args.steps):
+            ustep()
+        ue1.record(stream)
+        torch.cuda.synchronize(dev)
+        ums = ue0.elapsed_time(ue1)
+        u_t = torch.tensor([ums], dtype=torch.float64, device=cdev)
+        if world > 1:
+            dist.all_reduce(u_t, op=dist.ReduceOp.MAX)
+        u_mpps = n * args.steps * world / (float(u_t.item()) / 1e3) / 1e6
+        unfused = {"value": round(u_mpps, 3), "unit": "Mpps",
+                   "kernels_per_step": (uch.launches() - l0) // args.steps,
+                   "fused_speedup": round(mpps / u_mpps, 3),
+                   "what": "NFC_F_UNFUSED: one kernel per NF + device-side re-split, same ring and tables"}
+        uch.close()
+
     cpu = None
     if not args.no_cpu and rank == 0 and world == 1:
         r_mpps, r_gbps, r_pk, r_t = oracle_rate(w, first, args.cpu_seconds)
@@ -431,6 +464,7 @@ def main():
                        "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4)},
             "roofline": roof,
             "cpu_baseline": cpu,
+            "unfused_baseline": unfused,
             "e2e": e2e,
             "gpu_launches": int(launches),
             "clocks": clk.summary(),

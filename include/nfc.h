@@ -63,9 +63,16 @@ extern "C" {
 
 typedef struct nfc_chain nfc_chain; /* opaque; owned by the library */
 
+/* nfc_chain_opts.flags */
+#define NFC_F_UNFUSED 1u     /* baseline: one kernel per NF with a
+                              * device-side re-split of surviving packets between NFs and
+                              * a per-NF header re-read/re-parse -- the per-element
+                              * pipeline of P:L142-171.  Identical results; chains with
+                              * NFC_IPSEC are rejected with NFC_EUNSUP.                  */
+
 typedef struct {
     int device;              /* CUDA device ordinal                                   */
-    uint32_t flags;          /* reserved, must be 0                                   */
+    uint32_t flags;          /* 0 (fused, the product) or NFC_F_UNFUSED               */
     uint32_t max_batch_pkts; /* hint: largest packet count per nfc_process_batch call */
 } nfc_chain_opts;
 

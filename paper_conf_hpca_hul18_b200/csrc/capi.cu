@@ -61,6 +61,8 @@ struct nfc_chain {
     uint32_t kind[NFC_MAX_CHAIN] = {0};
     uint32_t mask = 0;
     uint32_t esp_pos = 0xFF;
+    uint32_t flags = 0;
+    DBuf uf_list[2], uf_cnt, uf_pass;     // NFC_F_UNFUSED scratch
     bool loaded[8] = {false};
     // tables
     DBuf acl_r4, acl_r6;
@@ -119,10 +121,13 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
         if (mask & (1u << kinds[i])) return fail(NFC_EUNSUP, "repeated NF kind in chain");
         mask |= 1u << kinds[i];
     }
-    if (opts && opts->flags) return fail(NFC_EINVAL, "opts->flags must be 0");
+    const uint32_t flags = opts ? opts->flags : 0;
+    if (flags & ~NFC_F_UNFUSED) return fail(NFC_EINVAL, "opts->flags: unknown bits");
+    if ((flags & NFC_F_UNFUSED) && (mask & (1u << NFC_IPSEC))) return fail(NFC_EUNSUP, "NFC_F_UNFUSED: IPsec chains are not offered");
     nfc_chain *c = new (std::nothrow) nfc_chain();
     if (!c) return fail(NFC_ENOMEM, "out of host memory");
     c->device = opts ? opts->device : 0;
+    c->flags = flags;
     c->n_nf = n;
     c->mask = mask;
     for (uint32_t i = 0; i < n; i++) {
@@ -150,7 +155,7 @@ void nfc_destroy_chain(nfc_chain *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
-                   &c->dpi_bitmap, &c->dpi_meta, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
+                   &c->dpi_bitmap, &c->dpi_meta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
@@ -395,12 +400,31 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     if (c->mask & MASK_DPI) {
         LaunchCfg q{};
         if (sfc_query(v, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");
-        size_t need = (size_t)q.grid * q.block * c->dpi.bitmap_words * 4;
+        size_t threads = (size_t)q.grid * q.block;
+        if (c->flags & NFC_F_UNFUSED) {          // stage kernels may keep more threads resident
+            int sms = 0;
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
+            threads = std::max(threads, (size_t)sms * 2048);
+        }
+        size_t need = threads * c->dpi.bitmap_words * 4;
         CK(c->dpi_bitmap.reserve(need));
         c->dpi.ovf_bitmap = c->dpi_bitmap.as<uint32_t>();
         p.dpi.ovf_bitmap = c->dpi.ovf_bitmap;
     }
     std::string err;
+    if (c->flags & NFC_F_UNFUSED) {
+        CK(c->uf_list[0].reserve((size_t)total * 4));
+        CK(c->uf_list[1].reserve((size_t)total * 4));
+        CK(c->uf_cnt.reserve((NFC_MAX_CHAIN + 1) * 4));
+        CK(c->uf_pass.reserve((size_t)total));
+        CK(cudaMemsetAsync(c->uf_cnt.p, 0, (NFC_MAX_CHAIN + 1) * 4, st));
+        uint32_t nl = 0;
+        rc = uf_launch(c->kind, c->n_nf, v.dm, p, c->uf_list[0].as<uint32_t>(), c->uf_list[1].as<uint32_t>(),
+                       c->uf_cnt.as<uint32_t>(), c->uf_pass.as<uint8_t>(), c->device, st, err, &nl);
+        if (rc) return fail(rc, err);
+        c->launches += nl;
+        return NFC_OK;
+    }
     rc = sfc_launch(v, p, c->device, st, err, nullptr);
     if (rc) return fail(rc, err);
     c->launches++;

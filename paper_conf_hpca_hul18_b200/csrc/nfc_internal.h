@@ -206,6 +206,9 @@ int sfc_launch(const Variant &v, const KParams &p, int device, void *stream, std
 size_t sfc_smem_bytes(const Variant &v, const KParams &p);
 size_t sfc_smem_limit(int device);      // max dynamic shared memory per CTA (opt-in)
 int sfc_query(const Variant &v, const KParams &p, int device, LaunchCfg *cfg_out);  // grid for full occupancy
+// NFC_F_UNFUSED baseline (unfused.cu): parse stage, one stage kernel per NF, stats stage
+int uf_launch(const uint32_t *kinds, uint32_t n_nf, int dm, const KParams &p, uint32_t *list0, uint32_t *list1,
+              uint32_t *counts, uint8_t *passmask, int device, void *stream, std::string &err, uint32_t *n_launch);
 int rss_shard_launch(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n, const uint32_t *nib,
                      uint32_t n_shards, uint8_t *out, void *stream, std::string &err);
 

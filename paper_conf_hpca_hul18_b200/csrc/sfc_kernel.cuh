@@ -59,6 +59,22 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 }
 
 
+// ---------------------------------------------------------------- tuning knobs (compile-time; defaults = measured best)
+#ifndef NFC_EARLY_T24
+#define NFC_EARLY_T24 0       // issue the DIR-24-8 first read right after parse, use it at LPM4
+#endif
+#ifndef NFC_DEFER_PAIRS
+#define NFC_DEFER_PAIRS 0     // 1: claim match-pair slots at DPI, write the pairs at the end of the chunk
+#endif
+#ifndef NFC_LOOKBACK_WIN
+#define NFC_LOOKBACK_WIN 1    // ESP sequence look-back over 32 predecessor tiles per step
+#endif
+#ifndef NFC_TIE
+#define NFC_TIE 1             // DM_HOT: order class lookups after the walk state (register pressure)
+#endif
+#ifndef NFC_CLAIM
+#define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic (DM_FULL; DM_HOT: 1)
+#endif
 #ifndef NFC_FULL_THREADS
 #define NFC_FULL_THREADS 768   // DM_FULL: one CTA per SM
 #endif
@@ -70,6 +86,7 @@ template <uint32_t S, int DM> struct KCfg {
     static constexpr int threads = (DM == DM_FULL && (S != SIG_ANY) && !esp) ? NFC_FULL_THREADS : 256;
     static constexpr int minb = esp ? 2 : (DM == DM_FULL ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
+    static constexpr uint32_t claim = DM == DM_FULL ? NFC_CLAIM : 1;   // chunks per warp claim
 };
 
 // ---------------------------------------------------------------- shared memory layout
@@ -414,7 +431,7 @@ __device__ __forceinline__ void dfa_step_wide(const DpiCtx &c, Walk &w, uint32_t
 template <int DM>
 __device__ __forceinline__ uint32_t tie(uint32_t word, const Walk &w)
 {
-    if (DM == DM_HOT) asm("" : "+r"(word) : "r"(w.s));
+    if (DM == DM_HOT && NFC_TIE) asm("" : "+r"(word) : "r"(w.s));
     return word;
 }
 
@@ -857,18 +874,6 @@ struct Pkt {
     bool alive;
 };
 
-#ifndef NFC_EARLY_T24
-#define NFC_EARLY_T24 0       // issue the DIR-24-8 first read right after parse, use it at LPM4
-#endif
-#ifndef NFC_DEFER_PAIRS
-#define NFC_DEFER_PAIRS 0     // 1: claim match-pair slots at DPI, write the pairs at the end of the chunk
-#endif
-#ifndef NFC_LOOKBACK_WIN
-#define NFC_LOOKBACK_WIN 1    // ESP sequence look-back over 32 predecessor tiles per step
-#endif
-#ifndef NFC_CLAIM
-#define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic
-#endif
 
 struct Ctx {
     const uint32_t *acl4, *acl6;
@@ -1215,23 +1220,13 @@ __device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8
     }
 }
 
-template <uint32_t S, int DM>
-__global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
+// Per-CTA context: pointers into the tables, staged into shared memory for the NFs of
+// SMASK (compile-time) that the chain uses (mask).  No barrier: the caller syncs.
+template <uint32_t SMASK, int DM, int NT>
+__device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const SmemLayout &L, uint32_t mask,
+                                          bool has_esp, uint32_t *vst, Ctx &C)
 {
-    constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp;
-    extern __shared__ __align__(16) uint8_t smem[];
-    __shared__ uint32_t s_tile;
-    const uint32_t mask = P.present & sig_mask(S);
-    const SmemLayout L = smem_layout(mask, NW, P);
-    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
-    uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
-    const uint32_t n_var = P.stats_len - NFIX;
-    for (uint32_t i = tid; i < NW * NWS; i += NT) wst[i] = 0;
-    if (P.smem_stats)
-        for (uint32_t i = tid; i < n_var; i += NT) vst[i] = 0;
-
-    Ctx C;
+    const uint32_t tid = threadIdx.x, lane = tid & 31;
     C.gtid = blockIdx.x * NT + tid;
     C.vst = P.smem_stats ? vst : nullptr;
     C.pol_f = pol_first();
@@ -1253,8 +1248,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     C.dpi.H = 0;
     C.dpi.HK2 = 0;
     C.meta = P.dpi.meta_smem ? reinterpret_cast<const uint32_t *>(smem + L.meta) : P.dpi.out_meta;
-    const bool has_esp = (sig_mask(S) & MASK_IPSEC) && P.esp_pos < P.n_nf;
-    if ((sig_mask(S) & MASK_ACL) && (mask & MASK_ACL)) {
+    if ((SMASK & MASK_ACL) && (mask & MASK_ACL)) {
         if (P.acl.smem_words) {
             uint4 *d4 = reinterpret_cast<uint4 *>(smem + L.acl4);
             uint4 *d6 = reinterpret_cast<uint4 *>(smem + L.acl6);
@@ -1267,7 +1261,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             C.acl6 = P.acl.bv6;
         }
     }
-    if ((sig_mask(S) & MASK_DPI) && (mask & MASK_DPI)) {
+    if ((SMASK & MASK_DPI) && (mask & MASK_DPI)) {
         // 2 * class: u8 for DM_FULL (ncls <= 128), u32 for DM_HOT
         if (DM == DM_FULL) {
             for (uint32_t i = tid; i < 256; i += NT) smem[L.cls + i] = (uint8_t)(2u * __ldg(P.dpi.cls + i));
@@ -1291,18 +1285,39 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             for (uint32_t i = tid; i < P.dpi.n_states; i += NT) mt[i] = __ldg(P.dpi.out_meta + i);
         }
     }
-    if ((sig_mask(S) & MASK_IPSEC) && has_esp) {
+    if ((SMASK & MASK_IPSEC) && has_esp) {
         uint32_t *te = reinterpret_cast<uint32_t *>(smem + L.te), *mn = reinterpret_cast<uint32_t *>(smem + L.ms_nib);
         for (uint32_t i = tid; i < 256 * 32; i += NT) te[i] = __ldg(P.esp.te + (i >> 5));   // T0 x 32 lanes
         for (uint32_t i = tid; i < 72 * 16; i += NT) mn[i] = __ldg(P.esp.rss_nib + i);
         C.te = te + lane;         // this lane's bank column
         C.ms_nib = mn;
     }
-    if ((sig_mask(S) & MASK_LB) && (mask & MASK_LB)) {
+    if ((SMASK & MASK_LB) && (mask & MASK_LB)) {
         uint32_t *ln = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
         for (uint32_t i = tid; i < 72 * 16; i += NT) ln[i] = __ldg(P.lb.nib + i);
         C.lb_nib = ln;
     }
+}
+
+template <uint32_t S, int DM>
+__global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
+{
+    constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp;
+    extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ uint32_t s_tile;
+    const uint32_t mask = P.present & sig_mask(S);
+    const SmemLayout L = smem_layout(mask, NW, P);
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
+    uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
+    const uint32_t n_var = P.stats_len - NFIX;
+    for (uint32_t i = tid; i < NW * NWS; i += NT) wst[i] = 0;
+    if (P.smem_stats)
+        for (uint32_t i = tid; i < n_var; i += NT) vst[i] = 0;
+
+    const bool has_esp = (sig_mask(S) & MASK_IPSEC) && P.esp_pos < P.n_nf;
+    Ctx C;
+    setup_ctx<sig_mask(S), DM, NT>(P, smem, L, mask, has_esp, vst, C);
     __syncthreads();
     unsigned long long *ws = wst + warp * NWS;
 
@@ -1312,11 +1327,12 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // prefetch to L2) before the current one is processed
         uint32_t cbase = 0, cleft = 0;
         auto claim = [&]() {                 // next 32-packet chunk; one atomic per NFC_CLAIM chunks
+            constexpr uint32_t CL = KCfg<S, DM>::claim;
             if (cleft == 0) {
                 uint32_t b = 0;
-                if (lane == 0) b = atomicAdd(P.tile_counter, 32u * NFC_CLAIM);
+                if (lane == 0) b = atomicAdd(P.tile_counter, 32u * CL);
                 cbase = __shfl_sync(0xFFFFFFFFu, b, 0);
-                cleft = NFC_CLAIM;
+                cleft = CL;
             }
             const uint32_t c = cbase;
             cbase += 32;
@@ -1424,7 +1440,8 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     int grid = sms * per_sm;
-    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + 32 * NFC_CLAIM - 1) / (32 * NFC_CLAIM) / KCfg<S, DM>::nwarp + 1;
+    constexpr uint32_t CLW = 32u * KCfg<S, DM>::claim;   // packets per warp claim
+    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + CLW - 1) / CLW / KCfg<S, DM>::nwarp + 1;
     if (!query_only && (uint32_t)grid > units) grid = (int)units;
     if (grid < 1) grid = 1;
     if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }

@@ -19,6 +19,7 @@ NFC_OK, NFC_EINVAL, NFC_ENOMEM, NFC_ECUDA, NFC_ESTATE, NFC_ECAP, NFC_EUNSUP = 0,
 ACL, DPI, LPM4, LPM6, IPSEC, LB = 1, 2, 3, 4, 5, 6
 KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB}
 STATS_RESET = 1
+F_UNFUSED = 1   # nfc_chain_opts.flags: per-NF kernels with re-split (NEXT-1 baseline)
 
 # stats vector layout
 ST_PKTS, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP = 0, 1, 2, 3, 4, 5
@@ -134,11 +135,11 @@ def _np(a, dtype=None):
 class Chain:
     """A service function chain bound to one CUDA device (original SFC order)."""
 
-    def __init__(self, kinds: Sequence, device: int = 0, max_batch_pkts: int = 0):
+    def __init__(self, kinds: Sequence, device: int = 0, max_batch_pkts: int = 0, flags: int = 0):
         ks = [KINDS[k] if isinstance(k, str) else int(k) for k in kinds]
         arr = (_u32 * len(ks))(*ks)
         h = _P()
-        opts = ChainOpts(device, 0, max_batch_pkts)
+        opts = ChainOpts(device, flags, max_batch_pkts)
         _check(lib.nfc_build_chain(arr, len(ks), ctypes.byref(opts), ctypes.byref(h)))
         self.h = h
         self.kinds = ks

@@ -68,6 +68,16 @@ def test_validation_before_cuda(nfc):
     assert nfc.version().startswith("nfc-b200")
 
 
+def test_flags_validation_before_cuda(nfc):
+    # NFC_F_UNFUSED (NEXT-1 baseline) does not offer IPsec chains; unknown flag bits are rejected
+    lib = nfc.lib
+    h = ctypes.c_void_p()
+    esp = (ctypes.c_uint32 * 2)(nfc.ACL, nfc.IPSEC)
+    assert lib.nfc_build_chain(esp, 2, ctypes.byref(nfc.ChainOpts(0, nfc.F_UNFUSED, 0)), ctypes.byref(h)) == nfc.NFC_EUNSUP
+    one = (ctypes.c_uint32 * 1)(nfc.ACL)
+    assert lib.nfc_build_chain(one, 1, ctypes.byref(nfc.ChainOpts(0, 0x80, 0)), ctypes.byref(h)) == nfc.NFC_EINVAL
+
+
 def test_no_oracle_in_product():
     # the product path never imports, includes or links the oracle
     pkg = os.path.join(ROOT, "paper_conf_hpca_hul18_b200")

@@ -190,3 +190,13 @@ def test_malformed_specs_rejected(nfc):
         ch.load_lpm(nfc.LPM4, r, w.tables.nh4, w.tables.pmac4)
     with pytest.raises(nfc.NfcError):
         ch.load_dpi(np.zeros(0, np.uint8), np.zeros(2, np.uint32), np.zeros(1, np.uint8))
+
+
+@pytest.mark.parametrize("cfg,k", [("C1", None), ("C3", None), ("C5", 4)])
+def test_unfused_baseline_parity(nfc, cfg, k):
+    """NEXT-1: the per-NF kernel pipeline with device-side re-split gives the oracle's
+    results exactly (records, bytes, pairs, stats), like the fused kernel."""
+    w = nfcgen.workload(cfg, k=k, small=(cfg == "C3"))
+    ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_UNFUSED)
+    ch.load_tables(w.tables)
+    check_parity(w, ch, 3001)
