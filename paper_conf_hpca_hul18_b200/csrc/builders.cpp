@@ -136,19 +136,21 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
         };
         const int fbits[4] = {bits, bits, 16, 16};
         std::vector<uint32_t> BK[4];
-        uint32_t steps = 0;
+        uint32_t steps = 0, maxst = 0;
         for (int q = 0; q < 4; q++) {
             BK[q] = buckets(F[q], fbits[q]);
             steps |= steps_of(BK[q]) << (8 * q);
+            maxst = std::max(maxst, steps_of(BK[q]));
         }
-        // keys (16-B aligned so an IPv6 key is one 128-bit load), followed by 2^steps
-        // all-ones pad keys: the window may run past the last interval start
-        auto put_keys = [&](const FieldIv &f, uint32_t kwords, uint32_t st) {
+        // keys (16-B aligned so an IPv6 key is one 128-bit load), followed by 2^maxst
+        // all-ones pad keys: the window may run past the last interval start (the kernel
+        // runs the four searches jointly for the largest depth)
+        auto put_keys = [&](const FieldIv &f, uint32_t kwords, uint32_t) {
             align_to(4);
             uint32_t o = (uint32_t)blob.size();
             for (u128 k : f.b)
                 for (int q = (int)kwords - 1; q >= 0; q--) blob.push_back((uint32_t)(k >> (32 * q)));
-            for (uint32_t i = 0; i < (1u << st) * kwords; i++) blob.push_back(0xFFFFFFFFu);
+            for (uint32_t i = 0; i < (1u << maxst) * kwords; i++) blob.push_back(0xFFFFFFFFu);
             return o;
         };
         auto put_bv = [&](const std::vector<uint64_t> &v) {
@@ -172,6 +174,7 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
         for (uint32_t r = 0; r < n; r++) blob.push_back(gidx[r] | (uint32_t)s.rules[gidx[r]].action << 31);
         for (int q = 0; q < 4; q++) offs[10 + q] = put_bk(BK[q]);
         blob[22] = steps;
+        blob[23] = maxst;
         while (blob.size() & 3) blob.push_back(0);   // 16-B multiple for staging copies
         for (int k = 0; k < 14; k++) blob[8 + k] = offs[k];
     }

@@ -386,8 +386,9 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         if (!full) {
             int smem_sm = 0;
             cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device);
-            const int target = (c->mask & MASK_IPSEC) ? 2 : 4;
-            const size_t budget = std::min((size_t)smem_sm / target - 1024 - 64, limit);
+            // CTAs resident per SM: 1 for the big-CTA DPI variants, else the launch-bounds target
+            const int target = v.threads > 256 ? 1 : (c->mask & MASK_IPSEC) ? 2 : 4;
+            const size_t budget = std::min((size_t)smem_sm / target - 1024 - 64, limit - 1024);
             if (c->mask & MASK_ACL)
                 if (sfc_smem_bytes(v, p) > budget / 2) p.acl.smem_words = 0;
             if ((c->mask & MASK_DPI) && !c->dpi.wide) {
@@ -397,6 +398,8 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
             }
         }
     }
+    p.dpi.row2 = 2 * c->dpi.ncls;
+    p.dpi.hk2 = p.dpi.hot_states ? 2 * (p.dpi.hot_states * c->dpi.ncls - 1) : 0;
     if (c->mask & MASK_DPI) {
         LaunchCfg q{};
         if (sfc_query(v, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");

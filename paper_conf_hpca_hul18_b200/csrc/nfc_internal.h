@@ -18,8 +18,8 @@ namespace nfc {
 //   m_src, m_dst, m_sport, m_dport  [6] key words per address (1 v4, 4 v6)
 //   [8..17] word offsets: keys_src, bv_src, keys_dst, bv_dst, keys_sp, bv_sp, keys_dp, bv_dp,
 //   bv_proto (256 x W), ridx (global rule index | action << 31),  [18..21] bucket tables
-//   (257 u32 per field) on the top 8 key bits,  [22] search steps per field (8 bits each).
-//   Key arrays are 16-B aligned and followed by 2^steps all-ones pad keys.  Bitsets are
+//   (257 u32 per field) on the top 8 key bits,  [22] search steps per field (8 bits each),
+//   [23] max steps.  Key arrays are 16-B aligned and followed by 2^maxsteps all-ones pad keys.  Bitsets are
 //   u64 at even offsets.
 static const uint32_t ACLBV_HDR = 24;
 struct AclImg {
@@ -47,6 +47,7 @@ struct DpiImg {
     uint32_t *ovf_bitmap;        // per resident thread scratch for > DPI_LIST distinct matches
     uint32_t bitmap_words;       // words per thread
     uint32_t hot_states;         // states whose full 256-byte rows are staged in shared memory
+    uint32_t row2, hk2;          // per launch: bytes per DFA row (2 ncls); byte offset of the last hot entry
     const uint32_t *out_meta;    // per state: out_off | n_out << 20 | any DROP pattern << 31
                                  // (DPI_META_NONE if the closure does not fit the fields)
     uint32_t meta_smem;          // 1: out_meta staged in shared memory
@@ -114,7 +115,14 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
        ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS,
        ST_POS_BASE = 16, ST_VAR_BASE = 64 };
 
+// byte offsets of the kernel's dynamic shared-memory regions (computed on the host per
+// launch, read by the kernel from the constant bank)
+struct SmemLayout {
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, meta, acl4, acl6, wcnt, prefix, total;
+};
+
 struct KParams {
+    SmemLayout lay;
     uint32_t n_nf;
     uint32_t kind[NFC_MAX_CHAIN];
     uint32_t esp_pos;            // chain position of IPSEC or 0xFF

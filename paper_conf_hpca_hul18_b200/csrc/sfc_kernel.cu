@@ -40,8 +40,7 @@ Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full)
     v.sig = sig;
     v.dm = (dfa_full && has_full(sig)) ? DM_FULL : DM_HOT;
     v.esp = esp;
-    if (sig == SIG_ANY) v.threads = KCfg<SIG_ANY, DM_HOT>::threads;
-    else v.threads = (v.dm == DM_FULL && !esp) ? KCfg<SIG_C1, DM_FULL>::threads : 256;
+    v.threads = kcfg_threads(sig);
     return v;
 }
 

@@ -76,23 +76,31 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic (DM_FULL; DM_HOT: 1)
 #endif
 #ifndef NFC_FULL_THREADS
-#define NFC_FULL_THREADS 768   // DM_FULL: one CTA per SM
+#define NFC_FULL_THREADS 768   // DPI chains without IPsec: one CTA per SM
 #endif
 #ifndef NFC_HOT_MINB
 #define NFC_HOT_MINB 3         // DM_HOT chains without IPsec: resident 256-thread CTAs per SM
 #endif
+// Launch shape: DPI chains without IPsec run one big CTA per SM (the DFA -- all of it,
+// or as many hot rows as fit -- is staged once per SM); IPsec chains run 256-thread
+// tiles (ESP sequence order), the rest 256-thread CTAs at NFC_HOT_MINB per SM.
+__host__ __device__ constexpr bool kcfg_big(uint32_t S)
+{
+    return S != SIG_ANY && !(sig_mask(S) & (1u << NFC_IPSEC)) && (sig_mask(S) & (1u << NFC_DPI));
+}
+__host__ __device__ constexpr int kcfg_threads(uint32_t S) { return kcfg_big(S) ? NFC_FULL_THREADS : 256; }
 template <uint32_t S, int DM> struct KCfg {
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
-    static constexpr int threads = (DM == DM_FULL && (S != SIG_ANY) && !esp) ? NFC_FULL_THREADS : 256;
-    static constexpr int minb = esp ? 2 : (DM == DM_FULL ? 1 : NFC_HOT_MINB);
+    static constexpr int threads = kcfg_threads(S);
+    static constexpr int minb = esp ? 2 : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
     static constexpr uint32_t claim = DM == DM_FULL ? NFC_CLAIM : 1;   // chunks per warp claim
 };
 
 // ---------------------------------------------------------------- shared memory layout
-struct SmemLayout {
-    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, meta, acl4, acl6, wcnt, prefix, total;
-};
+// the kernels' dynamic shared memory (one symbol: device functions address it directly,
+// with region offsets from P.lay in the constant bank -- no per-thread base registers)
+extern __shared__ __align__(16) uint8_t nfc_smem[];
 __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, const KParams &p)
 {
     SmemLayout L{};
@@ -300,14 +308,6 @@ __device__ __forceinline__ bool parse(const uint32_t h[16], const uint8_t *f, ui
 // followed by a fixed-depth window search whose depth is a table property
 // (warp-uniform trip count, no per-key divergence).  Header words come from the
 // kernel parameters (constant bank), not from the image.
-__device__ __forceinline__ uint32_t iv32(const uint32_t *A, const uint32_t *hd, int q, uint32_t key, int kbits)
-{
-    const uint32_t *B = A + hd[8 + 2 * q];
-    uint32_t lo = A[hd[18 + q] + (key >> (kbits - 8))];
-    const uint32_t st = (hd[22] >> (8 * q)) & 255;
-    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) lo = (B[lo + h] <= key) ? lo + h : lo;
-    return min(lo, hd[2 + q] - 1);
-}
 __device__ __forceinline__ bool le128(const uint4 b, const uint32_t k[4])
 {
     if (b.x != k[0]) return b.x < k[0];
@@ -315,27 +315,21 @@ __device__ __forceinline__ bool le128(const uint4 b, const uint32_t k[4])
     if (b.z != k[2]) return b.z < k[2];
     return b.w <= k[3];
 }
-__device__ __forceinline__ uint32_t iv128(const uint32_t *A, const uint32_t *hd, int q, const uint32_t k[4])
-{
-    const uint4 *B = reinterpret_cast<const uint4 *>(A + hd[8 + 2 * q]);
-    uint32_t lo = A[hd[18 + q] + (k[0] >> 24)];
-    const uint32_t st = (hd[22] >> (8 * q)) & 255;
-    for (uint32_t h = (1u << st) >> 1; h; h >>= 1) lo = le128(B[lo + h], k) ? lo + h : lo;
-    return min(lo, hd[2 + q] - 1);
-}
 
 // returns global rule index (0xFFFF none) | action << 31
 __device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t *hd, uint32_t default_action,
-                                              uint32_t js, uint32_t jd, const PV &v)
+                                              uint32_t js, uint32_t jd, uint32_t jsp, uint32_t jdp, uint32_t proto)
 {
     const uint32_t W = hd[1];
-    const uint32_t jsp = iv32(A, hd, 2, v.sport, 16);
-    const uint32_t jdp = iv32(A, hd, 3, v.dport, 16);
+    js = min(js, hd[2] - 1);
+    jd = min(jd, hd[3] - 1);
+    jsp = min(jsp, hd[4] - 1);
+    jdp = min(jdp, hd[5] - 1);
     const uint64_t *vs = reinterpret_cast<const uint64_t *>(A + hd[9]) + (size_t)js * W;
     const uint64_t *vd = reinterpret_cast<const uint64_t *>(A + hd[11]) + (size_t)jd * W;
     const uint64_t *vsp = reinterpret_cast<const uint64_t *>(A + hd[13]) + (size_t)jsp * W;
     const uint64_t *vdp = reinterpret_cast<const uint64_t *>(A + hd[15]) + (size_t)jdp * W;
-    const uint64_t *vpr = reinterpret_cast<const uint64_t *>(A + hd[16]) + (size_t)v.proto * W;
+    const uint64_t *vpr = reinterpret_cast<const uint64_t *>(A + hd[16]) + (size_t)proto * W;
     for (uint32_t w = 0; w < W; w++) {
         const uint64_t x = vs[w] & vd[w] & vsp[w] & vdp[w] & vpr[w];
         if (x) return A[hd[17] + 64 * w + (__ffsll((long long)x) - 1)];
@@ -343,20 +337,42 @@ __device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t 
     return 0xFFFFu | default_action << 31;
 }
 
+// The four interval lookups (src, dst, sport, dport) run jointly: one bucket read
+// each on the top 8 key bits, then one loop of the image's max window depth
+// (a table property: warp-uniform trip count) with four independent compare
+// steps per iteration.  Header words come from the constant bank.
 __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A6, const AclImg &ai, const PV &v)
 {
     if (v.fam == 4) {
         const uint32_t *hd = ai.hdr4;
         if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
-        const uint32_t js = iv32(A4, hd, 0, v.src[0], 32);
-        const uint32_t jd = iv32(A4, hd, 1, v.dst[0], 32);
-        return acl_match(A4, hd, ai.default_action, js, jd, v);
+        const uint32_t *A = A4;
+        const uint32_t *Bs = A + hd[8], *Bd = A + hd[10], *Bsp = A + hd[12], *Bdp = A + hd[14];
+        const uint32_t ks = v.src[0], kd = v.dst[0];
+        uint32_t js = A[hd[18] + (ks >> 24)], jd = A[hd[19] + (kd >> 24)];
+        uint32_t jsp = A[hd[20] + (v.sport >> 8)], jdp = A[hd[21] + (v.dport >> 8)];
+        for (uint32_t h = (1u << hd[23]) >> 1; h; h >>= 1) {
+            js = Bs[js + h] <= ks ? js + h : js;
+            jd = Bd[jd + h] <= kd ? jd + h : jd;
+            jsp = Bsp[jsp + h] <= v.sport ? jsp + h : jsp;
+            jdp = Bdp[jdp + h] <= v.dport ? jdp + h : jdp;
+        }
+        return acl_match(A, hd, ai.default_action, js, jd, jsp, jdp, v.proto);
     }
     const uint32_t *hd = ai.hdr6;
     if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
-    const uint32_t js = iv128(A6, hd, 0, v.src);
-    const uint32_t jd = iv128(A6, hd, 1, v.dst);
-    return acl_match(A6, hd, ai.default_action, js, jd, v);
+    const uint32_t *A = A6;
+    const uint4 *Bs = reinterpret_cast<const uint4 *>(A + hd[8]), *Bd = reinterpret_cast<const uint4 *>(A + hd[10]);
+    const uint32_t *Bsp = A + hd[12], *Bdp = A + hd[14];
+    uint32_t js = A[hd[18] + (v.src[0] >> 24)], jd = A[hd[19] + (v.dst[0] >> 24)];
+    uint32_t jsp = A[hd[20] + (v.sport >> 8)], jdp = A[hd[21] + (v.dport >> 8)];
+    for (uint32_t h = (1u << hd[23]) >> 1; h; h >>= 1) {
+        js = le128(Bs[js + h], v.src) ? js + h : js;
+        jd = le128(Bd[jd + h], v.dst) ? jd + h : jd;
+        jsp = Bsp[jsp + h] <= v.sport ? jsp + h : jsp;
+        jdp = Bdp[jdp + h] <= v.dport ? jdp + h : jdp;
+    }
+    return acl_match(A, hd, ai.default_action, js, jd, jsp, jdp, v.proto);
 }
 
 // ---------------------------------------------------------------- DPI
@@ -392,26 +408,28 @@ struct Walk { uint32_t s, cnt, mx; };
 __device__ __forceinline__ uint32_t byte_of(uint32_t w, int k) { return __byte_perm(w, 0, 0x4440 + k); }
 
 template <int DM>
-__device__ __forceinline__ uint32_t dfa_entry(const DpiCtx &c, uint32_t s, uint32_t byte)
+__device__ __forceinline__ uint32_t dfa_entry(const KParams &P, uint32_t s, uint32_t byte)
 {
-    if (DM == DM_FULL) return *reinterpret_cast<const uint16_t *>(c.hot + (s * c.row2 + c.cls8[byte]));
-    const uint32_t k2 = s * c.row2 + c.cls[byte];
-    const uint32_t e = *reinterpret_cast<const uint16_t *>(c.hot + min(k2, c.HK2));
-    return ld_u16_if(s >= c.H, reinterpret_cast<const uint16_t *>(reinterpret_cast<const uint8_t *>(c.trans) + k2), e);
+    if (DM == DM_FULL)
+        return *reinterpret_cast<const uint16_t *>(nfc_smem + P.lay.hot + (s * P.dpi.row2 + nfc_smem[P.lay.cls + byte]));
+    const uint32_t k2 = s * P.dpi.row2 + reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.cls)[byte];
+    uint32_t e = *reinterpret_cast<const uint16_t *>(nfc_smem + P.lay.hot + min(k2, P.dpi.hk2));
+    if (s >= P.dpi.hot_states) e = __ldg(reinterpret_cast<const uint16_t *>(reinterpret_cast<const uint8_t *>(P.dpi.trans) + k2));
+    return e;
 }
 template <int DM>
-__device__ __forceinline__ void dfa_step(const DpiCtx &c, Walk &w, uint32_t byte)
+__device__ __forceinline__ void dfa_step(const KParams &P, Walk &w, uint32_t byte)
 {
-    const uint32_t e = dfa_entry<DM>(c, w.s, byte);
+    const uint32_t e = dfa_entry<DM>(P, w.s, byte);
     w.s = e & 0x7FFFu;
     w.cnt += e >> 15;
     w.mx = max(w.mx, e);
 }
 // step only if `in` (bytes outside the payload leave the walk unchanged: s <= mx always)
 template <int DM>
-__device__ __forceinline__ void dfa_step_if(const DpiCtx &c, Walk &w, uint32_t byte, bool in)
+__device__ __forceinline__ void dfa_step_if(const KParams &P, Walk &w, uint32_t byte, bool in)
 {
-    const uint32_t e = in ? dfa_entry<DM>(c, w.s, byte) : w.s;
+    const uint32_t e = in ? dfa_entry<DM>(P, w.s, byte) : w.s;
     w.s = e & 0x7FFFu;
     w.cnt += e >> 15;
     w.mx = max(w.mx, e);
@@ -437,24 +455,23 @@ __device__ __forceinline__ uint32_t tie(uint32_t word, const Walk &w)
 
 // payload bytes [A, 64) of the header cache, A compile-time: no per-byte guards
 template <int DM, int A>
-__device__ __forceinline__ void walk_cached(const DpiCtx &c, const uint32_t h[16], Walk &w)
+__device__ __forceinline__ void walk_cached(const KParams &P, const uint32_t h[16], Walk &w)
 {
     uint32_t wd = tie<DM>(h[A >> 2], w);
 #pragma unroll
     for (int idx = A; idx < 64; idx++) {
         if ((idx & 3) == 0) wd = tie<DM>(h[idx >> 2], w);
-        dfa_step<DM>(c, w, byte_of(wd, idx & 3));
+        dfa_step<DM>(P, w, byte_of(wd, idx & 3));
     }
 }
 
 // walk of a DFA with > 32K states (u32 entries, all rows in global memory); not inlined
-static __device__ __noinline__ Walk dpi_walk_wide(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
-                                                  uint32_t b, uint64_t pol)
+static __device__ __noinline__ Walk dpi_walk_wide(const DpiCtx &c, const uint8_t *f, uint32_t a, uint32_t b,
+                                                  uint64_t pol)
 {
+    // payload bytes come from memory here (the header cache stays in registers in the caller)
     Walk w{0, 0, 0};
-#pragma unroll
-    for (int idx = 32; idx < 64; idx++) dfa_step_wide(c, w, (h[idx >> 2] >> ((idx & 3) * 8)) & 0xFF, (uint32_t)idx - a < b - a);
-    for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
+    for (uint32_t ch = a & ~15u; ch < b; ch += 16) {
         const uint4 q = ld_stream16(f + ch, pol);
         const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
@@ -467,20 +484,20 @@ static __device__ __noinline__ Walk dpi_walk_wide(const DpiCtx &c, const uint32_
 // come from the header cache (a payload never starts before byte 34), the rest
 // from memory in 16-B chunks.
 template <int DM>
-__device__ __forceinline__ Walk dpi_walk(const DpiCtx &c, const uint32_t h[16], const uint8_t *f, uint32_t a,
-                                         uint32_t b, uint64_t pol)
+__device__ __forceinline__ Walk dpi_walk(const KParams &P, const DpiCtx &c, const uint32_t h[16], const uint8_t *f,
+                                         uint32_t a, uint32_t b, uint64_t pol)
 {
-    if (DM != DM_FULL && c.wide) return dpi_walk_wide(c, h, f, a, b, pol);
+    if (DM != DM_FULL && P.dpi.wide) return dpi_walk_wide(c, f, a, b, pol);
     Walk w{0, 0, 0};
-    if (b >= 64 && a == 42) walk_cached<DM, 42>(c, h, w);        // IPv4 UDP
-    else if (b >= 64 && a == 62) walk_cached<DM, 62>(c, h, w);   // IPv6 UDP
-    else if (b >= 64 && a == 54) walk_cached<DM, 54>(c, h, w);   // IPv4 TCP
+    if (b >= 64 && a == 42) walk_cached<DM, 42>(P, h, w);        // IPv4 UDP
+    else if (b >= 64 && a == 62) walk_cached<DM, 62>(P, h, w);   // IPv6 UDP
+    else if (b >= 64 && a == 54) walk_cached<DM, 54>(P, h, w);   // IPv4 TCP
     else {
         uint32_t wd = 0;
 #pragma unroll
         for (int idx = 32; idx < 64; idx++) {
             if ((idx & 3) == 0) wd = tie<DM>(h[idx >> 2], w);
-            dfa_step_if<DM>(c, w, byte_of(wd, idx & 3), (uint32_t)idx - a < b - a);
+            dfa_step_if<DM>(P, w, byte_of(wd, idx & 3), (uint32_t)idx - a < b - a);
         }
     }
     for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
@@ -491,14 +508,14 @@ __device__ __forceinline__ Walk dpi_walk(const DpiCtx &c, const uint32_t h[16], 
             for (int k = 0; k < 16; k++) {
                 const uint32_t x = (k & 3) == 0 ? tie<DM>(wd[k >> 2], w) : wd[k >> 2];
                 if ((k & 3) == 0) wd[k >> 2] = x;
-                dfa_step<DM>(c, w, byte_of(x, k & 3));
+                dfa_step<DM>(P, w, byte_of(x, k & 3));
             }
         } else {
 #pragma unroll
             for (int k = 0; k < 16; k++) {
                 const uint32_t x = (k & 3) == 0 ? tie<DM>(wd[k >> 2], w) : wd[k >> 2];
                 if ((k & 3) == 0) wd[k >> 2] = x;
-                dfa_step_if<DM>(c, w, byte_of(x, k & 3), ch + k - a < b - a);
+                dfa_step_if<DM>(P, w, byte_of(x, k & 3), ch + k - a < b - a);
             }
         }
     }
@@ -971,7 +988,7 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
         dropped = (r >> 31) != 0;
     } else if constexpr (KIND == NFC_DPI) {
-        const Walk w = dpi_walk<DM>(C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
+        const Walk w = dpi_walk<DM>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
         const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
         const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
         if (w.cnt == 1 && meta != DPI_META_NONE) {
@@ -1303,10 +1320,10 @@ template <uint32_t S, int DM>
 __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
 {
     constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp;
-    extern __shared__ __align__(16) uint8_t smem[];
+    uint8_t *smem = nfc_smem;
     __shared__ uint32_t s_tile;
     const uint32_t mask = P.present & sig_mask(S);
-    const SmemLayout L = smem_layout(mask, NW, P);
+    const SmemLayout &L = P.lay;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
     uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
@@ -1446,7 +1463,9 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     if (grid < 1) grid = 1;
     if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }
     if (query_only) return NFC_OK;
-    sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(p);
+    KParams q = p;
+    q.lay = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p);
+    sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(q);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { err = std::string("sfc_kernel launch: ") + cudaGetErrorString(e); return NFC_ECUDA; }
     return NFC_OK;

@@ -58,9 +58,9 @@ __global__ void __launch_bounds__(NT, DM == DM_FULL ? 1 : 2)
     uf_nf_kernel(const KParams P, uint32_t pos, const uint32_t *in_list, const uint32_t *in_count, uint32_t *out_list,
                  uint32_t *out_count, uint8_t *passmask)
 {
-    extern __shared__ __align__(16) uint8_t smem[];
+    uint8_t *smem = nfc_smem;
     const uint32_t mask = 1u << KIND;
-    const SmemLayout L = smem_layout(mask, NT / 32, P);
+    const SmemLayout &L = P.lay;
     const uint32_t tid = threadIdx.x, lane = tid & 31;
     uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
     const uint32_t n_var = P.stats_len - NFIX;
@@ -173,7 +173,9 @@ static int uf_stage(const KParams &p, uint32_t pos, const uint32_t *in, const ui
     int per_sm = 1;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, uf_nf_kernel<KIND, DM, NT>, NT, smem);
     if (per_sm < 1) per_sm = 1;
-    uf_nf_kernel<KIND, DM, NT><<<sms * per_sm, NT, smem, st>>>(p, pos, in, in_n, out, out_n, pm);
+    KParams q = p;
+    q.lay = smem_layout(1u << KIND, NT / 32, p);
+    uf_nf_kernel<KIND, DM, NT><<<sms * per_sm, NT, smem, st>>>(q, pos, in, in_n, out, out_n, pm);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { err = std::string("unfused stage: ") + cudaGetErrorString(e); return NFC_ECUDA; }
     return NFC_OK;
