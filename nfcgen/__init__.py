@@ -267,8 +267,16 @@ def gen_acl(rng: np.random.Generator, n: int, family: int = 4, deny_frac: float 
         pk = int(rng.integers(0, 3))
         r[i]["proto_any"] = 1 if pk == 2 else 0
         r[i]["proto"] = (6, 17, 0)[pk]
-        r[i]["action"] = 1 if rng.random() < deny_frac else 0
-    return r
+        # a DENY rule names at least one address prefix (no wildcard-address deny that
+        # would shadow the whole set; R#28)
+        deny = rng.random() < deny_frac
+        r[i]["action"] = 1 if deny and int(r[i]["slen"]) + int(r[i]["dlen"]) > 0 else 0
+    # ClassBench filter sets list specific filters before general ones (a catch-all
+    # last); order by specificity so a broad rule does not shadow the set (R#28)
+    spec = (r["slen"].astype(np.int64) + r["dlen"]) * 2 ** 20 \
+        - (r["sp_hi"].astype(np.int64) - r["sp_lo"]) - (r["dp_hi"].astype(np.int64) - r["dp_lo"]) \
+        + (1 - r["proto_any"].astype(np.int64)) * 2 ** 18
+    return r[np.argsort(-spec, kind="stable")].copy()
 
 
 def gen_patterns(rng: np.random.Generator, n: int, lmin=4, lmax=16, printable_frac=1.0,
