@@ -333,6 +333,7 @@ def main():
     else:
         ms = ev[0][0].elapsed_time(ev[-1][1])
     launches = chain.launches() - launches0
+    launch_info = chain.last_launch()
     stats = chain.stats(reset=True)
     ms_t = torch.tensor([ms], dtype=torch.float64, device=cdev)
     st_t = torch.from_numpy(stats.view(np.int64).copy()).to(cdev)
@@ -461,7 +462,8 @@ def main():
                              "pristine ring restored between steps (1 GiB-class copy, evicts L2), outside timed intervals",
                        "timing": "CUDA events on the launch stream; max over ranks",
                        "parallelism": f"flow-sharded x{world}, no data-path collective",
-                       "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4)},
+                       "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4),
+                       "launch": launch_info},
             "roofline": roof,
             "cpu_baseline": cpu,
             "unfused_baseline": unfused,

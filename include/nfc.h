@@ -237,6 +237,15 @@ NFC_API int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uin
 /* Number of kernel launches the library issued on this chain so far. */
 NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 
+/* Shape of the chain's last fused-kernel launch (diagnostics; all zero before the first
+   nfc_process_batch): grid and block size, dynamic shared memory (bytes), DFA placement
+   (0 none, 1 tiered: dense rows + sparse records + global, 2 every row in shared memory),
+   DFA states with dense rows and with sparse records in shared memory. */
+typedef struct {
+    uint32_t grid, block, smem, dfa_mode, dfa_dense, dfa_sparse;
+} nfc_launch_info;
+NFC_API int nfc_last_launch(const nfc_chain *c, nfc_launch_info *out);
+
 NFC_API const char *nfc_last_error(void);
 NFC_API const char *nfc_version(void);
 

@@ -27,6 +27,14 @@ NFC_API int nfc_dbg_dpi(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids,
                         uint32_t *count, uint32_t *drop);
 /* DPI image shape: states, byte classes, 1 if 32-bit entries. */
 NFC_API int nfc_dbg_dpi_shape(nfc_dbg *d, uint32_t *n_states, uint32_t *n_classes, uint32_t *wide);
+/* DPI, tiered placement as the kernel's DM_HOT mode walks it: rows of states [0, hot) dense,
+   states [hot, hot + sparse) by their sparse record (base row + <= 2 exceptions), the rest
+   from the full table.  Same outputs as nfc_dbg_dpi; tier_steps (3 u32, may be NULL) counts
+   steps taken from dense rows, sparse records and the full table. */
+NFC_API int nfc_dbg_dpi_tier(nfc_dbg *d, uint32_t hot, uint32_t sparse, const uint8_t *buf, size_t n,
+                             uint16_t *ids, uint32_t cap, uint32_t *count, uint32_t *drop, uint32_t *tier_steps);
+/* DPI tier shape: states of depth <= 1, states with a representable sparse record. */
+NFC_API int nfc_dbg_dpi_tier_shape(nfc_dbg *d, uint32_t *n_d1, uint32_t *n_sparse_ok);
 /* LPM4: next-hop index (0x7FFF = miss) and number of table reads (1 or 2). */
 NFC_API int nfc_dbg_lpm4(nfc_dbg *d, uint32_t dst, uint32_t *nh, uint32_t *reads);
 /* LPM6: next-hop index (0x7FFF = miss), hash-level probes and hash-slot reads. */

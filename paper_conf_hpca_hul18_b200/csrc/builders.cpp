@@ -188,6 +188,7 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
 std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
 {
     if (s.n_patterns == 0 || s.n_patterns > 65535) return "dpi: n_patterns must be 1..65535";
+    o.maxlen = 0;
     if (!s.blob || !s.off || !s.action) return "dpi: NULL pointer";
     // byte classes
     std::array<int, 256> cls{};
@@ -195,6 +196,7 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
     for (uint32_t j = 0; j < s.n_patterns; j++) {
         if (s.off[j + 1] <= s.off[j]) return "dpi: empty pattern";
         if (s.action[j] > 1) return "dpi: action must be 0 or 1";
+        o.maxlen = std::max(o.maxlen, s.off[j + 1] - s.off[j]);
         for (uint32_t k = s.off[j]; k < s.off[j + 1]; k++) cls[s.blob[k]] = 1;
     }
     // used bytes get classes 0..u-1; all unused bytes share class u (if any) -> ncls <= 256
@@ -281,6 +283,37 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
     o.out_off[n] = (uint32_t)o.out_ids.size();
     if (o.out_ids.empty()) o.out_ids.push_back(0);
     o.action.assign(s.action, s.action + s.n_patterns);
+    // tier records (DpiImg::sparse): base = first depth <= 1 state on the failure chain,
+    // exceptions = the classes where the row differs from the base row (at most 2)
+    {
+        std::vector<int> depth(n, 0);
+        for (int u : order)
+            for (auto &kc : kids[u]) depth[kc.second] = depth[u] + 1;
+        uint32_t nd1 = 0;
+        for (size_t u = 0; u < n; u++) nd1 += depth[u] <= 1;
+        o.n_d1 = nd1;                      // BFS order: exactly the ids [0, nd1)
+        o.sparse.assign(n, make_uint2(0xFFFFFFFFu, 0));
+        auto entry = [&](int v) {
+            uint32_t e = (uint32_t)newid[v];
+            if (!outc[v].empty()) e |= 0x8000u;
+            return e;
+        };
+        if (!o.wide) {
+            for (int u : order) {
+                if (depth[u] <= 1) continue;
+                int b = fail[u];
+                while (depth[b] > 1) b = fail[b];
+                int ex[3], nx = 0;
+                for (int c = 0; c < ncls && nx < 3; c++)
+                    if (delta[(size_t)u * ncls + c] != delta[(size_t)b * ncls + c]) ex[nx++] = c;
+                if (nx > 2) continue;      // cold
+                int c0 = nx ? ex[0] : 0, c1 = nx > 1 ? ex[1] : c0;
+                uint32_t e0 = entry(delta[(size_t)u * ncls + c0]), e1 = entry(delta[(size_t)u * ncls + c1]);
+                o.sparse[newid[u]] = make_uint2((uint32_t)newid[b] | (uint32_t)c0 << 16 | (uint32_t)c1 << 24,
+                                                e0 | e1 << 16);
+            }
+        }
+    }
     // per-state match summary for the kernel's single-accept path: closure offset,
     // size and whether any pattern in it is a DROP pattern
     o.out_meta.assign(n, 0);

@@ -62,12 +62,13 @@ struct nfc_chain {
     uint32_t mask = 0;
     uint32_t esp_pos = 0xFF;
     uint32_t flags = 0;
+    nfc_launch_info last{};               // shape of the last fused launch
     DBuf uf_list[2], uf_cnt, uf_pass;     // NFC_F_UNFUSED scratch
     bool loaded[8] = {false};
     // tables
     DBuf acl_r4, acl_r6;
     AclImg acl{};
-    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta;
+    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta, dpi_sparse;
     DpiImg dpi{};
     DBuf l4_tbl24, l4_long, l4_nh, l4_pmac;
     Lpm4Img l4{};
@@ -155,7 +156,7 @@ void nfc_destroy_chain(nfc_chain *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
-                   &c->dpi_bitmap, &c->dpi_meta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
+                   &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
@@ -208,8 +209,12 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
         CK(c->dpi_ids.upload(d.out_ids));
         CK(c->dpi_act.upload(d.action));
         CK(c->dpi_meta.upload(d.out_meta));
+        CK(c->dpi_sparse.upload(d.sparse));
         c->dpi = DpiImg{};
         c->dpi.out_meta = c->dpi_meta.as<uint32_t>();
+        c->dpi.sparse = c->dpi_sparse.as<uint2>();
+        c->dpi.n_d1 = d.n_d1;
+        c->dpi.maxlen = d.maxlen;
         c->dpi.cls = c->dpi_cls.as<uint8_t>();
         c->dpi.trans = c->dpi_trans.p;
         c->dpi.ncls = d.ncls;
@@ -372,6 +377,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         const size_t limit = sfc_smem_limit(c->device);
         p.acl.smem_words = (c->mask & MASK_ACL) ? 1 : 0;
         p.dpi.hot_states = 0;
+        p.dpi.sparse_states = 0;
         bool full = false;
         if ((c->mask & MASK_DPI) && !c->dpi.wide && c->dpi.ncls <= 128) {
             Variant vf = sfc_variant(c->kind, c->n_nf, true);
@@ -392,9 +398,19 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
             if (c->mask & MASK_ACL)
                 if (sfc_smem_bytes(v, p) > budget / 2) p.acl.smem_words = 0;
             if ((c->mask & MASK_DPI) && !c->dpi.wide) {
-                size_t base = sfc_smem_bytes(v, p);
-                size_t h = base < budget ? (budget - base) / (2 * c->dpi.ncls + 1) : 0;
-                p.dpi.hot_states = (uint32_t)std::min<size_t>(h, c->dpi.n_states);
+                // tiered DFA: every row dense if it fits; else the depth <= 1 rows dense
+                // and as many sparse records (8 B) as fit after them (DpiImg::sparse)
+                p.dpi.sparse_states = 0;
+                const size_t base = sfc_smem_bytes(v, p), row = 2 * c->dpi.ncls;
+                const size_t room = base < budget ? budget - base : 0;
+                if ((size_t)c->dpi.n_states * row <= room) {
+                    p.dpi.hot_states = c->dpi.n_states;
+                } else {
+                    const size_t h = std::min<size_t>(c->dpi.n_d1, room / row);
+                    p.dpi.hot_states = (uint32_t)h;
+                    const size_t left = room - h * row;
+                    p.dpi.sparse_states = (uint32_t)std::min<size_t>(c->dpi.n_states - h, left / 8);
+                }
             }
         }
     }
@@ -428,8 +444,11 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         c->launches += nl;
         return NFC_OK;
     }
-    rc = sfc_launch(v, p, c->device, st, err, nullptr);
+    LaunchCfg lc{};
+    rc = sfc_launch(v, p, c->device, st, err, &lc);
     if (rc) return fail(rc, err);
+    c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
+                              (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states};
     c->launches++;
     if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;
     return NFC_OK;
@@ -517,6 +536,13 @@ int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uint8_t *sh
     std::string err;
     int rc = rss_shard_launch(b->arena, b->off, b->len, b->n, nb.as<uint32_t>(), n_shards, shard, stream, err);
     return rc ? fail(rc, err) : NFC_OK;
+}
+
+int nfc_last_launch(const nfc_chain *c, nfc_launch_info *out)
+{
+    if (!c || !out) return fail(NFC_EINVAL, "NULL argument");
+    *out = c->last;
+    return NFC_OK;
 }
 
 int nfc_launch_count(const nfc_chain *c, uint64_t *count)

@@ -101,6 +101,58 @@ int nfc_dbg_dpi(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids, uint32_
     return NFC_OK;
 }
 
+int nfc_dbg_dpi_tier(nfc_dbg *d, uint32_t hot, uint32_t sparse, const uint8_t *buf, size_t n, uint16_t *ids,
+                     uint32_t cap, uint32_t *count, uint32_t *drop, uint32_t *tier_steps)
+{
+    if (!d || d->kind != NFC_DPI) return NFC_EINVAL;
+    const DpiHost &D = d->dpi;
+    if (D.wide || hot == 0 || hot > D.n_states) return NFC_EINVAL;
+    std::vector<uint8_t> seen(D.action.size(), 0);
+    std::vector<uint16_t> got;
+    uint32_t s = 0, dr = 0, ts[3] = {0, 0, 0};
+    auto row = [&](uint32_t st, uint32_t c) {
+        uint16_t x;
+        memcpy(&x, &D.trans[((size_t)st * D.ncls + c) * 2], 2);
+        return (uint32_t)x;
+    };
+    for (size_t i = 0; i < n; i++) {
+        // the kernel's DM_HOT step (sfc_kernel.cuh dfa_entry): dense / sparse / cold
+        const uint32_t c = D.cls[buf[i]];
+        const bool sp = s >= hot;
+        uint32_t rx = 0xFFFFFFFFu, ry = 0;
+        if (sp && s - hot < sparse) { rx = D.sparse[s].x; ry = D.sparse[s].y; }
+        const uint32_t b = sp ? (rx & 0xFFFF) : s;
+        uint32_t e = b < hot ? row(b, c) : 0;
+        if (sp && c == ((rx >> 16) & 0xFF)) e = ry & 0xFFFF;
+        if (sp && c == (rx >> 24)) e = ry >> 16;
+        if (b >= hot) e = row(s, c);
+        ts[b >= hot ? 2 : sp ? 1 : 0]++;
+        s = e & 0x7FFF;
+        if (e >> 15)
+            for (uint32_t k = D.out_off[s]; k < D.out_off[s + 1]; k++) {
+                uint16_t id = D.out_ids[k];
+                dr |= D.action[id];
+                if (!seen[id]) { seen[id] = 1; got.push_back(id); }
+            }
+    }
+    std::sort(got.begin(), got.end());
+    for (uint32_t k = 0; k < got.size() && k < cap; k++) ids[k] = got[k];
+    *count = (uint32_t)got.size();
+    *drop = dr;
+    if (tier_steps) memcpy(tier_steps, ts, sizeof(ts));
+    return NFC_OK;
+}
+
+int nfc_dbg_dpi_tier_shape(nfc_dbg *d, uint32_t *n_d1, uint32_t *n_sparse_ok)
+{
+    if (!d || d->kind != NFC_DPI) return NFC_EINVAL;
+    *n_d1 = d->dpi.n_d1;
+    uint32_t k = 0;
+    for (size_t s = d->dpi.n_d1; s < d->dpi.sparse.size(); s++) k += (d->dpi.sparse[s].x & 0xFFFF) != 0xFFFF;
+    *n_sparse_ok = k;
+    return NFC_OK;
+}
+
 int nfc_dbg_lpm4(nfc_dbg *d, uint32_t dst, uint32_t *nh, uint32_t *reads)
 {
     if (!d || d->kind != NFC_LPM4) return NFC_EINVAL;

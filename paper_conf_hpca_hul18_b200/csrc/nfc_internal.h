@@ -51,6 +51,18 @@ struct DpiImg {
     const uint32_t *out_meta;    // per state: out_off | n_out << 20 | any DROP pattern << 31
                                  // (DPI_META_NONE if the closure does not fit the fields)
     uint32_t meta_smem;          // 1: out_meta staged in shared memory
+    // Tiered placement (DM_HOT): rows of states [0, hot_states) are dense in shared
+    // memory; states [hot_states, hot_states + sparse_states) are sparse records in
+    // shared memory; the rest are read from `trans` (cold).  A sparse record describes
+    // a state s by a dense base state b (the first state of depth <= 1 on s's failure
+    // chain) and the <= 2 classes where s's row differs from b's row:
+    //   x = b | c0 << 16 | c1 << 24,  y = e0 | e1 << 16   (b = 0xFFFF: not representable, cold)
+    // next(s, c) = c == c0 ? e0 : c == c1 ? e1 : row(b)[c].
+    const uint2 *sparse;         // n_states records (entries [0, n_d1) unused)
+    uint32_t n_d1;               // states of depth <= 1
+    uint32_t maxlen;             // longest pattern (bytes): a walk started maxlen - 1 bytes
+                                 // early is in the exact state (warp-split payload walks)
+    uint32_t sparse_states;      // per launch: records staged in shared memory
 };
 static const uint32_t DPI_META_NONE = 0x7FFFFFFFu;
 
@@ -118,7 +130,7 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
 // byte offsets of the kernel's dynamic shared-memory regions (computed on the host per
 // launch, read by the kernel from the constant bank)
 struct SmemLayout {
-    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, meta, acl4, acl6, wcnt, prefix, total;
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, total;
 };
 
 struct KParams {
@@ -170,6 +182,9 @@ struct DpiHost {
     std::vector<uint16_t> out_ids;
     std::vector<uint8_t> action;
     std::vector<uint32_t> out_meta;
+    uint32_t n_d1 = 0;               // states of depth <= 1 (BFS ids [0, n_d1))
+    uint32_t maxlen = 0;             // longest pattern
+    std::vector<uint2> sparse;       // per state: tier record (see DpiImg::sparse)
 };
 std::string build_dpi(const nfc_dpi_spec &s, DpiHost &out);
 std::string build_lpm4(const nfc_lpm4_spec &s, std::vector<uint16_t> &tbl24, std::vector<uint16_t> &tbllong,

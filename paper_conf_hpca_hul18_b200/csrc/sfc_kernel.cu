@@ -40,13 +40,13 @@ Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full)
     v.sig = sig;
     v.dm = (dfa_full && has_full(sig)) ? DM_FULL : DM_HOT;
     v.esp = esp;
-    v.threads = kcfg_threads(sig);
+    v.threads = kcfg_threads(sig, v.dm);
     return v;
 }
 
 size_t sfc_smem_bytes(const Variant &v, const KParams &p)
 {
-    return smem_layout(p.present & sig_mask(v.sig), v.threads / 32, p).total;
+    return smem_layout(p.present & sig_mask(v.sig), v.threads / 32, p, kcfg_nws(v.sig), v.dm).total;
 }
 
 size_t sfc_smem_limit(int device)

@@ -78,6 +78,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_FULL_THREADS
 #define NFC_FULL_THREADS 768   // DPI chains without IPsec: one CTA per SM
 #endif
+#ifndef NFC_HOTBIG_THREADS
+#define NFC_HOTBIG_THREADS 768 // DPI chains without IPsec whose DFA is tiered (DM_HOT)
+#endif
 #ifndef NFC_HOT_MINB
 #define NFC_HOT_MINB 3         // DM_HOT chains without IPsec: resident 256-thread CTAs per SM
 #endif
@@ -88,10 +91,13 @@ __host__ __device__ constexpr bool kcfg_big(uint32_t S)
 {
     return S != SIG_ANY && !(sig_mask(S) & (1u << NFC_IPSEC)) && (sig_mask(S) & (1u << NFC_DPI));
 }
-__host__ __device__ constexpr int kcfg_threads(uint32_t S) { return kcfg_big(S) ? NFC_FULL_THREADS : 256; }
+__host__ __device__ constexpr int kcfg_threads(uint32_t S, int dm) { return kcfg_big(S) ? (dm == DM_FULL ? NFC_FULL_THREADS : NFC_HOTBIG_THREADS) : 256; }
+// per-warp counter slots: the fixed counters + 4 per chain position
+__host__ __device__ constexpr int kcfg_nws(uint32_t S) { return ST_POS_BASE + 4 * (S == SIG_ANY ? NFC_MAX_CHAIN : (int)sig_n(S)); }
 template <uint32_t S, int DM> struct KCfg {
+    static constexpr int nws = kcfg_nws(S);
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
-    static constexpr int threads = kcfg_threads(S);
+    static constexpr int threads = kcfg_threads(S, DM);
     static constexpr int minb = esp ? 2 : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
     static constexpr uint32_t claim = DM == DM_FULL ? NFC_CLAIM : 1;   // chunks per warp claim
@@ -101,19 +107,21 @@ template <uint32_t S, int DM> struct KCfg {
 // the kernels' dynamic shared memory (one symbol: device functions address it directly,
 // with region offsets from P.lay in the constant bank -- no per-thread base registers)
 extern __shared__ __align__(16) uint8_t nfc_smem[];
-__host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, const KParams &p)
+__host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, const KParams &p, int nws = NWS, int dm = DM_HOT)
 {
     SmemLayout L{};
     uint32_t o = 0;
-    L.wst = o; o += nwarp * NWS * 8;                                // per-warp private counters (u64)
+    L.wst = o; o += nwarp * nws * 8;                                // per-warp private counters (u64)
     L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
     o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_DPI) {
-        L.cls = o; o += 256 * 4;
+        L.cls = o; o += dm == DM_FULL ? 256 : 256 * 4;               // byte -> 2 * class (u8 / u32)
         L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u;
+        L.sp = o; o += p.dpi.sparse_states * 8;
         L.meta = o; o += p.dpi.meta_smem ? (p.dpi.n_states * 4 + 15) & ~15u : 0;
+        L.seg = o; o += nwarp * 64 * 4;                             // split-walk accumulators (cnt, mx) x 32
     }
     o = (o + 15) & ~15u;
     if (mask & MASK_ACL) {
@@ -184,6 +192,13 @@ __device__ __forceinline__ uint32_t ld_u16_if(bool p, const uint16_t *a, uint32_
         : "+r"(v) : "l"(a), "r"((uint32_t)p));
     return v;
 }
+
+// A DPI walk is a dependent chain of shared-memory lookups, so the bytes ahead of it are
+// prefetched into L2 (NFC_PF_DIST bytes ahead, one 128-B line at a time).
+#ifndef NFC_PF_DIST
+#define NFC_PF_DIST 512
+#endif
+__device__ __forceinline__ void prefetch_l2(const void *a) { asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a)); }
 
 // byte k (0..63) of the 64 B header cache; k compile-time in hot paths
 __device__ __forceinline__ uint32_t hbyte(const uint32_t h[16], uint32_t k) { return (h[k >> 2] >> ((k & 3) * 8)) & 0xFF; }
@@ -393,8 +408,9 @@ struct DpiCtx {
     const uint8_t *gcls;    // global byte -> class table (exact re-walk)
     const uint8_t *sm;      // smem base (DM_FULL addressing)
     const uint8_t *hot;     // smem hot rows (DM_HOT)
+    const uint2 *sp;        // smem sparse records (DM_HOT), states [H, H + S)
     uint32_t row2;          // bytes per row = 2 * ncls
-    uint32_t H, HK2;        // DM_HOT: hot states, byte offset of the last hot entry
+    uint32_t H, HK2, S;     // DM_HOT: hot states, byte offset of the last hot entry, sparse records
     uint32_t ncls, wide;
     const void *trans;
     const uint32_t *out_off;
@@ -412,9 +428,37 @@ __device__ __forceinline__ uint32_t dfa_entry(const KParams &P, uint32_t s, uint
 {
     if (DM == DM_FULL)
         return *reinterpret_cast<const uint16_t *>(nfc_smem + P.lay.hot + (s * P.dpi.row2 + nfc_smem[P.lay.cls + byte]));
-    const uint32_t k2 = s * P.dpi.row2 + reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.cls)[byte];
-    uint32_t e = *reinterpret_cast<const uint16_t *>(nfc_smem + P.lay.hot + min(k2, P.dpi.hk2));
-    if (s >= P.dpi.hot_states) e = __ldg(reinterpret_cast<const uint16_t *>(reinterpret_cast<const uint8_t *>(P.dpi.trans) + k2));
+    // tiered rows (DpiImg::sparse): dense row, or a sparse record's base row with <= 2
+    // exceptions, or (cold) the global table.  Branch-free: the sparse-record, dense-row
+    // and cold loads are predicated.  cls[byte] = class (u32).
+    const uint32_t c = reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.cls)[byte];
+    const uint32_t H = P.dpi.hot_states;
+    uint32_t rx, ry;
+    {
+        const uint32_t ra = (uint32_t)__cvta_generic_to_shared(nfc_smem + P.lay.sp) + 8u * (s - H);
+        asm("{\n\t.reg .pred q;\n\tsetp.lt.u32 q, %2, %3;\n\tmov.b32 %0, -1;\n\tmov.b32 %1, 0;\n\t"
+            "@q ld.shared.v2.u32 {%0, %1}, [%4];\n\t}"
+            : "=r"(rx), "=r"(ry) : "r"(s - H), "r"(P.dpi.sparse_states), "r"(ra));
+    }
+    const bool sp = s >= H;
+    const uint32_t b = sp ? (rx & 0xFFFFu) : s;
+    uint32_t e;
+    {
+        const uint32_t da = (uint32_t)__cvta_generic_to_shared(nfc_smem + P.lay.hot) + 2u * (b * P.dpi.ncls + c);
+        asm("{\n\t.reg .pred q;\n\tsetp.lt.u32 q, %1, %2;\n\tmov.b32 %0, 0;\n\t@q ld.shared.u16 %0, [%3];\n\t}"
+            : "=r"(e) : "r"(b), "r"(H), "r"(da));
+    }
+    e = (sp && c == __byte_perm(rx, 0, 0x4442)) ? (ry & 0xFFFFu) : e;
+    e = (sp && c == __byte_perm(rx, 0, 0x4443)) ? (ry >> 16) : e;
+    // cold rows (deep states beyond the on-chip tiers): predicated load
+    const bool cold = b >= H;
+    {
+        const uint16_t *ga = reinterpret_cast<const uint16_t *>(P.dpi.trans) + (s * P.dpi.ncls + c);
+        uint32_t o;
+        asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\tmov.b32 %0, %2;\n\t@q ld.global.nc.u16 %0, [%3];\n\t}"
+            : "=r"(o) : "r"((uint32_t)cold), "r"(e), "l"(ga));
+        e = o;
+    }
     return e;
 }
 template <int DM>
@@ -429,14 +473,18 @@ __device__ __forceinline__ void dfa_step(const KParams &P, Walk &w, uint32_t byt
 template <int DM>
 __device__ __forceinline__ void dfa_step_if(const KParams &P, Walk &w, uint32_t byte, bool in)
 {
-    const uint32_t e = in ? dfa_entry<DM>(P, w.s, byte) : w.s;
+    // branch-free: the entry is looked up for any state (all loads stay in bounds) and
+    // discarded when the byte is outside the span
+    uint32_t e = dfa_entry<DM>(P, w.s, byte);
+    asm("" : "+r"(e));
+    e = in ? e : w.s;
     w.s = e & 0x7FFFu;
     w.cnt += e >> 15;
     w.mx = max(w.mx, e);
 }
 __device__ __forceinline__ void dfa_step_wide(const DpiCtx &c, Walk &w, uint32_t byte, bool in)
 {
-    const uint32_t k = w.s * c.ncls + (c.cls[byte] >> 1);
+    const uint32_t k = w.s * c.ncls + c.cls[byte];
     const uint32_t e = in ? __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k) : w.s;
     w.s = e & 0x7FFFFFFFu;
     w.cnt += e >> 31;
@@ -488,6 +536,7 @@ __device__ __forceinline__ Walk dpi_walk(const KParams &P, const DpiCtx &c, cons
                                          uint32_t a, uint32_t b, uint64_t pol)
 {
     if (DM != DM_FULL && P.dpi.wide) return dpi_walk_wide(c, f, a, b, pol);
+    for (uint32_t l = 128; l < min(b, 64u + NFC_PF_DIST); l += 128) prefetch_l2(f + l);
     Walk w{0, 0, 0};
     if (b >= 64 && a == 42) walk_cached<DM, 42>(P, h, w);        // IPv4 UDP
     else if (b >= 64 && a == 62) walk_cached<DM, 62>(P, h, w);   // IPv6 UDP
@@ -501,6 +550,7 @@ __device__ __forceinline__ Walk dpi_walk(const KParams &P, const DpiCtx &c, cons
         }
     }
     for (uint32_t ch = max(64u, a & ~15u); ch < b; ch += 16) {
+        if ((ch & 127) == 0 && ch + NFC_PF_DIST < b) prefetch_l2(f + ch + NFC_PF_DIST);
         const uint4 q = ld_stream16(f + ch, pol);
         uint32_t wd[4] = {q.x, q.y, q.z, q.w};
         if (ch >= a && ch + 16 <= b) {
@@ -522,6 +572,25 @@ __device__ __forceinline__ Walk dpi_walk(const KParams &P, const DpiCtx &c, cons
     return w;
 }
 
+// Payload bytes [a, min(b, 64)) from the header cache (the owner lane's registers).
+template <int DM>
+__device__ __forceinline__ Walk dpi_walk_head(const KParams &P, const uint32_t h[16], uint32_t a, uint32_t b)
+{
+    Walk w{0, 0, 0};
+    if (b >= 64 && a == 42) walk_cached<DM, 42>(P, h, w);        // IPv4 UDP
+    else if (DM == DM_FULL && b >= 64 && a == 62) walk_cached<DM, 62>(P, h, w);   // IPv6 UDP
+    else if (DM == DM_FULL && b >= 64 && a == 54) walk_cached<DM, 54>(P, h, w);   // IPv4 TCP
+    else if (a < 64) {
+        uint32_t wd = 0;
+#pragma unroll
+        for (int idx = 32; idx < 64; idx++) {
+            if ((idx & 3) == 0) wd = tie<DM>(h[idx >> 2], w);
+            dfa_step_if<DM>(P, w, byte_of(wd, idx & 3), (uint32_t)idx - a < b - a);
+        }
+    }
+    return w;
+}
+
 // Exact match set of a packet whose walk hit more than one accept event (rare
 // path, not inlined): re-walk the payload from memory collecting distinct pattern
 // ids in a register list, or -- beyond DPI_LIST ids -- in a per-thread global
@@ -534,9 +603,30 @@ struct DpiOvf {
     uint32_t match_cap;
     unsigned long long *stats;
 };
-// one exact DFA step from the global table (state -> next, accept flag)
+// one exact DFA step (state -> next, accept flag): the on-chip tiers as in dfa_entry
+// (DM_FULL: all rows; DM_HOT: dense rows / sparse records / global), or the global
+// table for > 32K-state DFAs
+template <int DM>
 __device__ __forceinline__ uint32_t dfa_step_global(const DpiCtx &c, uint32_t s, uint32_t b, bool &acc)
 {
+    if (!c.wide) {
+        uint32_t e;
+        if (DM == DM_FULL) {
+            e = *reinterpret_cast<const uint16_t *>(c.hot + s * c.row2 + c.cls8[b]);
+        } else {
+            const uint32_t cl = c.cls[b];
+            const bool sp = s >= c.H;
+            uint2 r = make_uint2(0xFFFFFFFFu, 0u);
+            if (sp && s - c.H < c.S) r = c.sp[s - c.H];
+            const uint32_t bs = sp ? (r.x & 0xFFFFu) : s;
+            e = bs < c.H ? *reinterpret_cast<const uint16_t *>(c.hot + 2 * (bs * c.ncls + cl)) : 0u;
+            if (sp && cl == ((r.x >> 16) & 0xFFu)) e = r.y & 0xFFFFu;
+            if (sp && cl == (r.x >> 24)) e = r.y >> 16;
+            if (bs >= c.H) e = __ldg(reinterpret_cast<const uint16_t *>(c.trans) + s * c.ncls + cl);
+        }
+        acc = (e >> 15) & 1;
+        return e & 0x7FFFu;
+    }
     const uint32_t k = s * c.ncls + __ldg(c.gcls + b);
     if (c.wide) {
         const uint32_t e = __ldg(reinterpret_cast<const uint32_t *>(c.trans) + k);
@@ -547,6 +637,7 @@ __device__ __forceinline__ uint32_t dfa_step_global(const DpiCtx &c, uint32_t s,
     acc = (e >> 15) & 1;
     return e & 0x7FFFu;
 }
+template <int DM>
 static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a, uint32_t b, uint32_t gtid,
                                           DpiOvf o, uint32_t pkt_id)
 {
@@ -559,7 +650,7 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
         const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
         bool acc;
-        s = dfa_step_global(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
+        s = dfa_step_global<DM>(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
         const uint32_t e = __ldg(c.out_off + s + 1);
         for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
@@ -593,7 +684,7 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         if (i == a || (i & 15) == 0) q = *reinterpret_cast<const uint4 *>(f + (i & ~15u));
         const uint32_t wd = (i & 8) ? ((i & 4) ? q.w : q.z) : ((i & 4) ? q.y : q.x);
         bool acc;
-        s = dfa_step_global(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
+        s = dfa_step_global<DM>(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
         const uint32_t e = __ldg(c.out_off + s + 1);
         for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
@@ -976,6 +1067,159 @@ __device__ __forceinline__ void emit_pairs(const KParams &P, uint32_t o0, uint32
         atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
 }
 
+// DPI result of a packet from its walk summary (R#9/R#10): no accept
+// event -> no match; exactly one -> the output closure of that state (per-state summary:
+// size + DROP flag); more -> exact re-walk (dpi_slow).  Returns true if a DROP pattern matched.
+template <int DM>
+__device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &k, const Walk w)
+{
+    bool dropped = false;
+    const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
+    const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
+    if (w.cnt == 1 && meta != DPI_META_NONE) {
+        // exactly one accept event: the match set is the output closure of that state
+        // (distinct ids); its size and DROP flag come from the per-state summary.  The
+        // pair slots are claimed now and the pairs written at the end of the chunk, so
+        // the atomic's latency overlaps the rest of the chain.
+        const uint32_t nm = (meta >> 20) & 0x7FF;
+        k.nmatch = nm;
+        dropped = (meta >> 31) != 0;
+#if NFC_DEFER_PAIRS
+        k.mmeta = meta & 0x7FFFFFFFu;
+        k.mslot = atomicAdd(P.match_count, nm);
+#else
+        emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
+#endif
+    } else if (w.cnt >= 1) {
+        const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
+                        P.match_cap, P.stats};
+        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+        k.nmatch = r & 0x7FFFFFFFu;
+        dropped = (r >> 31) != 0;
+    }
+    return dropped;
+}
+
+// DPI for the 32 packets of a warp, called by all lanes (compile-time chains).  With
+// the whole DFA on chip (DM_FULL) each lane first walks its own packet's payload bytes
+// below 64 from the header cache.  The rest of the 32 payloads ([base, b) per packet,
+// base = 64 or the 16-B line of the payload start, padded to 16 B) is concatenated into one virtual byte stream and cut
+// into 32 equal 16-B-aligned ranges, one per lane, so IMIX lengths do not leave lanes
+// idle.  All lanes advance one 16-B chunk per iteration (a convergent loop); a lane
+// whose piece ends fetches the next piece's packet by warp shuffles.  A piece that
+// starts inside a payload re-walks the maxlen - 1 bytes before it from the root
+// without counting (the Aho-Corasick state depends only on the last maxlen bytes, so
+// the state at the piece start is exact); a piece at the start of a remainder
+// continues the owner's walk.  Piece results (accept-event count, largest entry) are
+// combined into the owner's summary through shared memory, so the owner ends with
+// exactly the (cnt, mx) of a sequential walk, evaluated by dpi_finish.
+template <int DM>
+__device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt &k)
+{
+    const uint32_t FULL = 0xFFFFFFFFu, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (DM != DM_FULL && P.dpi.wide)          // > 32K states: per-lane walk from L2
+        return k.alive ? dpi_finish<DM>(P, C, k, dpi_walk<DM>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f))
+                       : false;
+    const bool act = k.alive;
+    const uint32_t a = k.v.pl_off, b = k.v.ip_end;
+    Walk w{0, 0, 0};
+    // DM_FULL: bytes below 64 from the header cache (registers); DM_HOT: everything
+    // through the stream (one copy of the walk loop keeps the kernel's code small)
+    if (DM == DM_FULL && act) w = dpi_walk_head<DM>(P, k.h, a, b);
+    const uint32_t base = (DM != DM_FULL || a >= 64) ? (a & ~15u) : 64u;
+    const uint32_t rem = act && b > base ? (b - base + 15) & ~15u : 0u;
+    uint32_t incl = rem;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, d);
+        if (lane >= (uint32_t)d) incl += y;
+    }
+    const uint32_t total = __shfl_sync(FULL, incl, 31);
+    if (total) {                              // warp-uniform
+        const uint32_t excl = incl - rem;
+        uint32_t *acc = reinterpret_cast<uint32_t *>(nfc_smem + P.lay.seg) + warp * 64;
+        acc[lane] = 0;
+        acc[32 + lane] = 0;
+        __syncwarp();
+        const uint32_t per = ((total + 31) / 32 + 15) & ~15u;
+        uint32_t lo = min(lane * per, total);
+        const uint32_t hi = min(lo + per, total);
+        const uint32_t O = P.dpi.maxlen - 1;
+        const uint64_t fa = reinterpret_cast<uint64_t>(k.f);
+        uint32_t x = 0, e0 = 0, v0 = 0, sc = 0, own = 0;
+        const uint8_t *f = nullptr;
+        Walk pw{0, 0, 0};
+        for (;;) {
+            const bool need = x >= e0 && lo < hi;
+            if (__any_sync(FULL, need)) {
+                // next piece: the packet owning virtual byte lo (the last whose range starts at or before it)
+                uint32_t p = 0;
+#pragma unroll
+                for (uint32_t bit = 16; bit; bit >>= 1)
+                    if (__shfl_sync(FULL, excl, p + bit) <= lo) p += bit;
+                const uint32_t pe = __shfl_sync(FULL, incl, p), px = __shfl_sync(FULL, excl, p);
+                const uint32_t pb = __shfl_sync(FULL, base, p), pa = __shfl_sync(FULL, a, p);
+                const uint32_t pend = __shfl_sync(FULL, b, p), ps = __shfl_sync(FULL, w.s, p);
+                const uint64_t pf = __shfl_sync(FULL, fa, p);
+                if (need) {
+                    const uint32_t ev = min(hi, pe);
+                    const uint32_t s0 = pb + (lo - px);
+                    e0 = min(pb + (ev - px), pend);
+                    own = p;
+                    f = reinterpret_cast<const uint8_t *>(pf);
+                    if (s0 == pb) {               // continues the owner's walk
+                        pw = Walk{ps, 0, 0};
+                        v0 = max(pa, s0);
+                        x = s0;
+                        sc = s0;
+                    } else {                      // warm-up from the root, counting from s0
+                        pw = Walk{0, 0, 0};
+                        v0 = max(pa, s0 - min(O, s0));
+                        x = v0 & ~15u;
+                        sc = s0;
+                    }
+                    for (uint32_t l = x & ~127u; l < min(e0, x + NFC_PF_DIST); l += 128) prefetch_l2(f + l);
+                    lo = ev;
+                }
+            }
+            const bool run = x < e0;
+            if (!__any_sync(FULL, run)) break;
+            if (run) {
+                if (x == sc) { pw.cnt = 0; pw.mx = 0; }
+                if ((x & 127) == 0 && x + NFC_PF_DIST < e0) prefetch_l2(f + x + NFC_PF_DIST);
+                const uint4 q = ld_stream16(f + x, C.pol_f);
+                uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+                if (DM == DM_FULL && x >= v0 && x + 16 <= e0) {
+#pragma unroll
+                    for (int kk = 0; kk < 16; kk++) {
+                        const uint32_t y = (kk & 3) == 0 ? tie<DM>(wd[kk >> 2], pw) : wd[kk >> 2];
+                        if ((kk & 3) == 0) wd[kk >> 2] = y;
+                        dfa_step<DM>(P, pw, byte_of(y, kk & 3));
+                    }
+                } else {
+#pragma unroll
+                    for (int kk = 0; kk < 16; kk++) {
+                        const uint32_t y = (kk & 3) == 0 ? tie<DM>(wd[kk >> 2], pw) : wd[kk >> 2];
+                        if ((kk & 3) == 0) wd[kk >> 2] = y;
+                        dfa_step_if<DM>(P, pw, byte_of(y, kk & 3), x + kk - v0 < e0 - v0);
+                    }
+                }
+                x += 16;
+                if (x >= e0 && pw.cnt) {          // piece done: into the owner's summary
+                    atomicAdd(&acc[own], pw.cnt);
+                    atomicMax(&acc[32 + own], pw.mx);
+                }
+            }
+        }
+        __syncwarp();
+        if (rem) {
+            w.cnt += acc[lane];
+            w.mx = max(w.mx, acc[32 + lane]);
+        }
+    }
+    return act ? dpi_finish<DM>(P, C, k, w) : false;
+}
+
 // one NF of kind KIND at chain position pos (KIND compile-time)
 template <uint32_t KIND, int DM>
 __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k, uint32_t pos)
@@ -988,30 +1232,7 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
         dropped = (r >> 31) != 0;
     } else if constexpr (KIND == NFC_DPI) {
-        const Walk w = dpi_walk<DM>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
-        const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
-        const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
-        if (w.cnt == 1 && meta != DPI_META_NONE) {
-            // exactly one accept event: the match set is the output closure of that state
-            // (distinct ids); its size and DROP flag come from the per-state summary.  The
-            // pair slots are claimed now and the pairs written at the end of the chunk, so
-            // the atomic's latency overlaps the rest of the chain.
-            const uint32_t nm = (meta >> 20) & 0x7FF;
-            k.nmatch = nm;
-            dropped = (meta >> 31) != 0;
-#if NFC_DEFER_PAIRS
-            k.mmeta = meta & 0x7FFFFFFFu;
-            k.mslot = atomicAdd(P.match_count, nm);
-#else
-            emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
-#endif
-        } else if (w.cnt >= 1) {
-            const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
-                            P.match_cap, P.stats};
-            const uint32_t r = dpi_slow(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
-            k.nmatch = r & 0x7FFFFFFFu;
-            dropped = (r >> 31) != 0;
-        }
+        dropped = dpi_finish<DM>(P, C, k, dpi_walk<DM>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f));
     } else if constexpr (KIND == NFC_LPM4) {
         // DIR-24-8: at most two dependent table reads ("two memory accesses")
         if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
@@ -1057,7 +1278,12 @@ template <uint32_t S, int DM, int POS, int END>
 __device__ __forceinline__ void run_fixed(const KParams &P, const Ctx &C, Pkt &k)
 {
     if constexpr (POS < END) {
-        if (k.alive) nf_apply<sig_kind(S, POS), DM>(P, C, k, POS);
+        if constexpr (sig_kind(S, POS) == NFC_DPI) {
+            // warp-cooperative (all lanes): payload bytes split evenly over the lanes
+            if (nf_dpi_warp<DM>(P, C, k)) { k.drop = POS; k.alive = false; }
+        } else {
+            if (k.alive) nf_apply<sig_kind(S, POS), DM>(P, C, k, POS);
+        }
         run_fixed<S, DM, POS + 1, END>(P, C, k);
     }
 }
@@ -1279,12 +1505,12 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         }
     }
     if ((SMASK & MASK_DPI) && (mask & MASK_DPI)) {
-        // 2 * class: u8 for DM_FULL (ncls <= 128), u32 for DM_HOT
+        // 2 * class as u8 for DM_FULL (ncls <= 128), class as u32 for DM_HOT
         if (DM == DM_FULL) {
             for (uint32_t i = tid; i < 256; i += NT) smem[L.cls + i] = (uint8_t)(2u * __ldg(P.dpi.cls + i));
         } else {
             uint32_t *cls = reinterpret_cast<uint32_t *>(smem + L.cls);
-            for (uint32_t i = tid; i < 256; i += NT) cls[i] = 2u * __ldg(P.dpi.cls + i);
+            for (uint32_t i = tid; i < 256; i += NT) cls[i] = __ldg(P.dpi.cls + i);
         }
         const uint32_t H = C.dpi.wide ? 0 : P.dpi.hot_states;
         uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
@@ -1297,6 +1523,13 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         }
         C.dpi.H = H;
         C.dpi.HK2 = H ? 2 * (H * P.dpi.ncls - 1) : 0;
+        C.dpi.sp = reinterpret_cast<const uint2 *>(smem + L.sp);
+        C.dpi.S = 0;
+        if (DM != DM_FULL && !C.dpi.wide) {
+            uint2 *sp = reinterpret_cast<uint2 *>(smem + L.sp);
+            for (uint32_t i = tid; i < P.dpi.sparse_states; i += NT) sp[i] = __ldg(P.dpi.sparse + H + i);
+            C.dpi.S = P.dpi.sparse_states;
+        }
         if (P.dpi.meta_smem) {
             uint32_t *mt = reinterpret_cast<uint32_t *>(smem + L.meta);
             for (uint32_t i = tid; i < P.dpi.n_states; i += NT) mt[i] = __ldg(P.dpi.out_meta + i);
@@ -1319,7 +1552,7 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
 template <uint32_t S, int DM>
 __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
 {
-    constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp;
+    constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp, WS = KCfg<S, DM>::nws;
     uint8_t *smem = nfc_smem;
     __shared__ uint32_t s_tile;
     const uint32_t mask = P.present & sig_mask(S);
@@ -1328,7 +1561,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
     uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
     const uint32_t n_var = P.stats_len - NFIX;
-    for (uint32_t i = tid; i < NW * NWS; i += NT) wst[i] = 0;
+    for (uint32_t i = tid; i < NW * WS; i += NT) wst[i] = 0;
     if (P.smem_stats)
         for (uint32_t i = tid; i < n_var; i += NT) vst[i] = 0;
 
@@ -1336,7 +1569,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     Ctx C;
     setup_ctx<sig_mask(S), DM, NT>(P, smem, L, mask, has_esp, vst, C);
     __syncthreads();
-    unsigned long long *ws = wst + warp * NWS;
+    unsigned long long *ws = wst + warp * WS;
 
     if (!KCfg<S, DM>::esp || (S == SIG_ANY && !has_esp)) {
         // warp-granular persistent loop: chunks of 32 consecutive packets (NFC_CLAIM
@@ -1404,12 +1637,12 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 #pragma unroll
         for (int r = 0; r < 2; r++) {
             const uint32_t idx = i + 32 * r;
-            if (idx < NWS)
-                for (int w = 0; w < NW; w++) t[r] += wst[w * NWS + idx];
+            if (idx < WS)
+                for (int w = 0; w < NW; w++) t[r] += wst[w * WS + idx];
         }
         __syncwarp();
         wst[i] = t[0];
-        if (i + 32 < NWS) wst[i + 32] = t[1];
+        if (i + 32 < WS) wst[i + 32] = t[1];
         __syncwarp();
         if (lane == 0) {
             wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
@@ -1422,7 +1655,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             }
         }
         __syncwarp();
-        for (uint32_t idx = lane; idx < NWS; idx += 32)
+        for (uint32_t idx = lane; idx < WS; idx += 32)
             if (wst[idx]) atomicAdd(&P.stats[idx], wst[idx]);
     }
     if (P.smem_stats)
@@ -1435,7 +1668,7 @@ template <uint32_t S, int DM>
 int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCfg *cfg, bool query_only)
 {
     constexpr int NT = KCfg<S, DM>::threads;
-    const size_t smem = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p).total;
+    const size_t smem = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p, KCfg<S, DM>::nws, DM).total;
     static int attr_smem[64] = {0};   // per device: dynamic smem size already granted
     static int per_sm_cache[64] = {0};
     static size_t per_sm_smem[64] = {0};
@@ -1464,7 +1697,7 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }
     if (query_only) return NFC_OK;
     KParams q = p;
-    q.lay = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p);
+    q.lay = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p, KCfg<S, DM>::nws, DM);
     sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(q);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { err = std::string("sfc_kernel launch: ") + cudaGetErrorString(e); return NFC_ECUDA; }

@@ -164,7 +164,7 @@ static int uf_stage(const KParams &p, uint32_t pos, const uint32_t *in, const ui
                     uint32_t *out_n, uint8_t *pm, int sms, cudaStream_t st, std::string &err)
 {
     constexpr int NT = DM == DM_FULL ? 768 : 256;
-    const size_t smem = smem_layout(1u << KIND, NT / 32, p).total;
+    const size_t smem = smem_layout(1u << KIND, NT / 32, p, NWS, DM).total;
     if (cudaFuncSetAttribute(uf_nf_kernel<KIND, DM, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
         cudaSuccess) {
         err = "cudaFuncSetAttribute (unfused stage) failed";
@@ -174,7 +174,7 @@ static int uf_stage(const KParams &p, uint32_t pos, const uint32_t *in, const ui
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, uf_nf_kernel<KIND, DM, NT>, NT, smem);
     if (per_sm < 1) per_sm = 1;
     KParams q = p;
-    q.lay = smem_layout(1u << KIND, NT / 32, p);
+    q.lay = smem_layout(1u << KIND, NT / 32, p, NWS, DM);
     uf_nf_kernel<KIND, DM, NT><<<sms * per_sm, NT, smem, st>>>(q, pos, in, in_n, out, out_n, pm);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { err = std::string("unfused stage: ") + cudaGetErrorString(e); return NFC_ECUDA; }

@@ -77,8 +77,9 @@ class Result(ctypes.Structure):
 
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
-           "nfc_launch_count", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
-DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_lpm4",
+           "nfc_launch_count", "nfc_last_launch", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
+DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
+                 "nfc_dbg_dpi_tier_shape", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
                  "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
 
@@ -99,6 +100,7 @@ def _load_lib():
     L.nfc_stats_len.argtypes = [_P, ctypes.POINTER(ctypes.c_size_t)]
     L.nfc_collect_stats.argtypes = [_P, _P, ctypes.c_size_t, _u32]
     L.nfc_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64)]
+    L.nfc_last_launch.argtypes = [_P, _P]
     L.nfc_rss_shard.argtypes = [ctypes.c_int, ctypes.POINTER(Batch), _u32, _P, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
@@ -108,6 +110,8 @@ def _load_lib():
     L.nfc_dbg_destroy.restype = None
     L.nfc_dbg_dpi.argtypes = [_P, _P, ctypes.c_size_t, _P, _u32, P32, P32]
     L.nfc_dbg_dpi_shape.argtypes = [_P, P32, P32, P32]
+    L.nfc_dbg_dpi_tier.argtypes = [_P, _u32, _u32, _P, ctypes.c_size_t, _P, _u32, P32, P32, _P]
+    L.nfc_dbg_dpi_tier_shape.argtypes = [_P, P32, P32]
     L.nfc_dbg_lpm4.argtypes = [_P, _u32, P32, P32]
     L.nfc_dbg_lpm6.argtypes = [_P, _P, P32, P32, P32]
     L.nfc_dbg_lpm6_levels.argtypes = [_P, P32]
@@ -266,6 +270,12 @@ class Chain:
         _check(lib.nfc_launch_count(self.h, ctypes.byref(c)))
         return c.value
 
+    def last_launch(self) -> dict:
+        """Shape of the last fused launch (nfc_last_launch)."""
+        a = np.zeros(6, dtype=np.uint32)
+        _check(lib.nfc_last_launch(self.h, a.ctypes.data))
+        return dict(zip(("grid", "block", "smem", "dfa_mode", "dfa_dense", "dfa_sparse"), (int(x) for x in a)))
+
 
 def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,
               stream: int = 0):
@@ -319,6 +329,20 @@ class HostImage:
         a, b, c = _u32(), _u32(), _u32()
         _check(lib.nfc_dbg_dpi_shape(self.h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
         return a.value, b.value, c.value
+
+    def dpi_tier(self, data: bytes, hot: int, sparse: int, cap: int = 65536):
+        """The kernel's tiered DFA walk (dense / sparse / cold); returns (ids, drop, tier_steps)."""
+        ids = np.zeros(cap, dtype=np.uint16)
+        ts = np.zeros(3, dtype=np.uint32)
+        c, d = _u32(), _u32()
+        _check(lib.nfc_dbg_dpi_tier(self.h, hot, sparse, _cbuf(data), len(data), ids.ctypes.data, cap,
+                                    ctypes.byref(c), ctypes.byref(d), ts.ctypes.data))
+        return [int(x) for x in ids[:min(c.value, cap)]], bool(d.value), [int(x) for x in ts]
+
+    def dpi_tier_shape(self):
+        a, b = _u32(), _u32()
+        _check(lib.nfc_dbg_dpi_tier_shape(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
 
     def lpm4(self, dst: int):
         nh, r = _u32(), _u32()

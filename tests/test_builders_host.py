@@ -62,6 +62,48 @@ def test_dfa_image_vs_oracle(nfc, case):
         assert drop == any(t.pat_action[j] for j in ids)
 
 
+@pytest.mark.parametrize("case", ["c3", "c1", "tiny", "allbytes"])
+def test_dfa_tiered_walk_vs_oracle(nfc, case):
+    """The kernel's tiered DFA placement (dense rows / sparse records / cold rows,
+    DpiImg::sparse) gives the oracle's match sets for every split of the states,
+    including splits where records fall back to the full table."""
+    rng = random.Random(7 + len(case))
+    if case == "c3":
+        t = nfcgen.workload("C3").tables
+    elif case == "c1":
+        t = nfcgen.workload("C1").tables
+    elif case == "allbytes":
+        pats = [bytes([b, (b * 7) & 255, b ^ 0x55]) for b in range(256)] + [b"\x00\x01\x02"]
+        t = _pattern_tables(pats, [rng.random() < 0.1 for _ in pats])
+    else:
+        pats = [bytes(rng.choice(b"ab") for _ in range(rng.randrange(1, 6))) for _ in range(16)]
+        t = _pattern_tables(pats)
+    img = nfc.HostImage("DPI", blob=t.pat_blob, off=t.pat_off, action=t.pat_action)
+    ns, ncls, wide = img.dpi_shape()
+    nd1, nok = img.dpi_tier_shape()
+    assert 1 <= nd1 <= min(ns, 257)
+    orc = oracle.OracleChain(["DPI"], t)
+    pats = t.patterns()
+    splits = [(nd1, ns - nd1), (nd1, (ns - nd1) // 3), (max(1, nd1 // 2), ns), (1, 0), (ns, 0)]
+    used = [0, 0, 0]
+    for k in range(150):
+        n = rng.randrange(0, 300)
+        text = bytes(rng.choice(b"ab") if case == "tiny" else rng.randrange(256) for _ in range(n))
+        for _ in range(rng.randrange(0, 6)):
+            p = rng.choice(pats)
+            i = rng.randrange(0, len(text) + 1)
+            text = text[:i] + p + text[i:]
+        want = orc.ac_match(text)
+        for hot, sparse in splits:
+            ids, drop, ts = img.dpi_tier(text, hot, sparse)
+            assert ids == want, (hot, sparse)
+            assert drop == any(t.pat_action[j] for j in ids)
+            used = [a + b for a, b in zip(used, ts)]
+    assert used[1] > 0 and used[2] > 0          # sparse and cold paths both exercised
+    if case in ("c3", "c1"):
+        assert nok >= 0.99 * (ns - nd1)         # nearly every deep state has <= 2 exceptions
+
+
 def test_dir24_8_vs_oracle_and_two_accesses(nfc):
     w = nfcgen.workload("C1")
     t = w.tables
