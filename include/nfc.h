@@ -105,7 +105,7 @@ typedef struct {                 /* 48 B */
 } nfc_acl_rule;
 
 typedef struct {
-    uint32_t n_rules;            /* <= 65534                                      */
+    uint32_t n_rules;            /* <= 32767                                      */
     uint32_t default_action;     /* action when no rule matches: 0/1              */
     const nfc_acl_rule *rules;   /* host; rule i has priority i (first match)     */
 } nfc_acl_spec;
@@ -240,9 +240,10 @@ NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 /* Shape of the chain's last fused-kernel launch (diagnostics; all zero before the first
    nfc_process_batch): grid and block size, dynamic shared memory (bytes), DFA placement
    (0 none, 1 tiered: dense rows + sparse records + global, 2 every row in shared memory),
-   DFA states with dense rows and with sparse records in shared memory. */
+   DFA states with dense rows and with sparse records in shared memory, 1 if the per-state
+   match summary is in shared memory, bytes of the ACL images in shared memory. */
 typedef struct {
-    uint32_t grid, block, smem, dfa_mode, dfa_dense, dfa_sparse;
+    uint32_t grid, block, smem, dfa_mode, dfa_dense, dfa_sparse, dfa_meta_smem, acl_smem;
 } nfc_launch_info;
 NFC_API int nfc_last_launch(const nfc_chain *c, nfc_launch_info *out);
 

@@ -70,7 +70,7 @@ static void build_field(const std::vector<std::pair<u128, u128>> &rng, u128 maxv
 
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6)
 {
-    if (s.n_rules > 65534) return "acl: too many rules (max 65534)";
+    if (s.n_rules > 32767) return "acl: too many rules (max 32767)";
     if (s.n_rules && !s.rules) return "acl: rules == NULL";
     if (s.default_action > 1) return "acl: default_action must be 0 or 1";
     for (uint32_t i = 0; i < s.n_rules; i++) {
@@ -159,9 +159,9 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
             for (uint64_t x : v) { blob.push_back((uint32_t)x); blob.push_back((uint32_t)(x >> 32)); }
             return o;
         };
-        auto put_bk = [&](const std::vector<uint32_t> &bk) {
+        auto put_bk = [&](const std::vector<uint32_t> &bk) {   // 257 u16 (interval indices < 2^16)
             uint32_t o = (uint32_t)blob.size();
-            for (int t = 0; t < 257; t++) blob.push_back(bk[t]);
+            for (int t = 0; t < 258; t += 2) blob.push_back(bk[t] | (t + 1 < 257 ? bk[t + 1] << 16 : 0u));
             return o;
         };
         uint32_t offs[14];

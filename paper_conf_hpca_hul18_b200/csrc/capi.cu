@@ -448,7 +448,8 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     rc = sfc_launch(v, p, c->device, st, err, &lc);
     if (rc) return fail(rc, err);
     c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
-                              (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states};
+                              (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states,
+                              p.dpi.meta_smem, p.acl.smem_words ? 4 * (p.acl.words4 + p.acl.words6) : 0u};
     c->launches++;
     if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;
     return NFC_OK;

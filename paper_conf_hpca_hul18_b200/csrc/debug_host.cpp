@@ -235,10 +235,10 @@ int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *
     for (int k = 0; k < nb; k++) { s[k] = be32(src + 4 * k); t[k] = be32(dst + 4 * k); }
     const uint32_t W = A[1];
     auto iv32 = [&](int q, uint32_t key, int kbits) {
-        return bs32(A + A[8 + 2 * q], A[A[18 + q] + (key >> (kbits - 8))], A[23], A[2 + q], key);
+        return bs32(A + A[8 + 2 * q], reinterpret_cast<const uint16_t *>(A + A[18 + q])[key >> (kbits - 8)], A[23], A[2 + q], key);
     };
     auto iv128 = [&](int q, const uint32_t *k) {
-        return bs128(A + A[8 + 2 * q], A[A[18 + q] + (k[0] >> 24)], A[23], A[2 + q], k);
+        return bs128(A + A[8 + 2 * q], reinterpret_cast<const uint16_t *>(A + A[18 + q])[k[0] >> 24], A[23], A[2 + q], k);
     };
     uint32_t js = nb == 1 ? iv32(0, s[0], 32) : iv128(0, s);
     uint32_t jd = nb == 1 ? iv32(1, t[0], 32) : iv128(1, t);

@@ -18,7 +18,7 @@ namespace nfc {
 //   m_src, m_dst, m_sport, m_dport  [6] key words per address (1 v4, 4 v6)
 //   [8..17] word offsets: keys_src, bv_src, keys_dst, bv_dst, keys_sp, bv_sp, keys_dp, bv_dp,
 //   bv_proto (256 x W), ridx (global rule index | action << 31),  [18..21] bucket tables
-//   (257 u32 per field) on the top 8 key bits,  [22] search steps per field (8 bits each),
+//   (257 u16 per field) on the top 8 key bits,  [22] search steps per field (8 bits each),
 //   [23] max steps.  Key arrays are 16-B aligned and followed by 2^maxsteps all-ones pad keys.  Bitsets are
 //   u64 at even offsets.
 static const uint32_t ACLBV_HDR = 24;

@@ -331,6 +331,12 @@ __device__ __forceinline__ bool le128(const uint4 b, const uint32_t k[4])
     return b.w <= k[3];
 }
 
+// bucket t of a field's 257-entry u16 bucket table at word offset o
+__device__ __forceinline__ uint32_t acl_bucket(const uint32_t *A, uint32_t o, uint32_t t)
+{
+    return reinterpret_cast<const uint16_t *>(A + o)[t];
+}
+
 // returns global rule index (0xFFFF none) | action << 31
 __device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t *hd, uint32_t default_action,
                                               uint32_t js, uint32_t jd, uint32_t jsp, uint32_t jdp, uint32_t proto)
@@ -364,8 +370,8 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
         const uint32_t *A = A4;
         const uint32_t *Bs = A + hd[8], *Bd = A + hd[10], *Bsp = A + hd[12], *Bdp = A + hd[14];
         const uint32_t ks = v.src[0], kd = v.dst[0];
-        uint32_t js = A[hd[18] + (ks >> 24)], jd = A[hd[19] + (kd >> 24)];
-        uint32_t jsp = A[hd[20] + (v.sport >> 8)], jdp = A[hd[21] + (v.dport >> 8)];
+        uint32_t js = acl_bucket(A, hd[18], ks >> 24), jd = acl_bucket(A, hd[19], kd >> 24);
+        uint32_t jsp = acl_bucket(A, hd[20], v.sport >> 8), jdp = acl_bucket(A, hd[21], v.dport >> 8);
         for (uint32_t h = (1u << hd[23]) >> 1; h; h >>= 1) {
             js = Bs[js + h] <= ks ? js + h : js;
             jd = Bd[jd + h] <= kd ? jd + h : jd;
@@ -379,8 +385,8 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
     const uint32_t *A = A6;
     const uint4 *Bs = reinterpret_cast<const uint4 *>(A + hd[8]), *Bd = reinterpret_cast<const uint4 *>(A + hd[10]);
     const uint32_t *Bsp = A + hd[12], *Bdp = A + hd[14];
-    uint32_t js = A[hd[18] + (v.src[0] >> 24)], jd = A[hd[19] + (v.dst[0] >> 24)];
-    uint32_t jsp = A[hd[20] + (v.sport >> 8)], jdp = A[hd[21] + (v.dport >> 8)];
+    uint32_t js = acl_bucket(A, hd[18], v.src[0] >> 24), jd = acl_bucket(A, hd[19], v.dst[0] >> 24);
+    uint32_t jsp = acl_bucket(A, hd[20], v.sport >> 8), jdp = acl_bucket(A, hd[21], v.dport >> 8);
     for (uint32_t h = (1u << hd[23]) >> 1; h; h >>= 1) {
         js = le128(Bs[js + h], v.src) ? js + h : js;
         jd = le128(Bd[jd + h], v.dst) ? jd + h : jd;
@@ -1128,14 +1134,14 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
     if (DM == DM_FULL && act) w = dpi_walk_head<DM>(P, k.h, a, b);
     const uint32_t base = (DM != DM_FULL || a >= 64) ? (a & ~15u) : 64u;
     const uint32_t rem = act && b > base ? (b - base + 15) & ~15u : 0u;
-    uint32_t incl = rem;
+    if (__any_sync(FULL, rem != 0)) {         // warp-uniform (64-B frames: never)
+        uint32_t incl = rem;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, incl, d);
-        if (lane >= (uint32_t)d) incl += y;
-    }
-    const uint32_t total = __shfl_sync(FULL, incl, 31);
-    if (total) {                              // warp-uniform
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        const uint32_t total = __shfl_sync(FULL, incl, 31);
         const uint32_t excl = incl - rem;
         uint32_t *acc = reinterpret_cast<uint32_t *>(nfc_smem + P.lay.seg) + warp * 64;
         acc[lane] = 0;

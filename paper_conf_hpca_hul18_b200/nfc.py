@@ -272,9 +272,10 @@ class Chain:
 
     def last_launch(self) -> dict:
         """Shape of the last fused launch (nfc_last_launch)."""
-        a = np.zeros(6, dtype=np.uint32)
+        a = np.zeros(8, dtype=np.uint32)
         _check(lib.nfc_last_launch(self.h, a.ctypes.data))
-        return dict(zip(("grid", "block", "smem", "dfa_mode", "dfa_dense", "dfa_sparse"), (int(x) for x in a)))
+        return dict(zip(("grid", "block", "smem", "dfa_mode", "dfa_dense", "dfa_sparse", "dfa_meta_smem", "acl_smem"),
+                        (int(x) for x in a)))
 
 
 def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,
