@@ -234,6 +234,16 @@ NFC_API int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t 
  * are device pointers on `device`; asynchronous on `stream`. */
 NFC_API int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uint8_t *shard, void *stream);
 
+/* SFC parallelization plan (Tables II-III): cuts
+ * the chain kinds[0..n) into groups of consecutive NFs that may run on copies of
+ * the same packet and be merged by XOR with a result identical to the
+ * sequential chain.  group[p] (n bytes, host memory) receives the group index of
+ * position p (0, 1, ... non-decreasing).  Greedy maximal groups under the
+ * field-level rule of DESIGN.md R#16 (no read-after-write, no write-after-write on
+ * a packet field, per packet family); IPsec always stands alone.  NFC_EINVAL for
+ * NULL pointers, n outside 1..6 or an unknown kind. */
+NFC_API int nfc_plan_parallel(const uint32_t *kinds, uint32_t n, uint8_t *group);
+
 /* Number of kernel launches the library issued on this chain so far. */
 NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 

@@ -55,6 +55,9 @@ def lib():
         L.oracle_destroy.argtypes = [_P]
         L.oracle_stats_len.restype = ctypes.c_size_t
         L.oracle_stats_len.argtypes = [_P]
+        L.oracle_run_reorg.restype = ctypes.c_uint64
+        L.oracle_run_reorg.argtypes = [_P, _P, _P, _P, _P, ctypes.c_uint32, ctypes.c_uint64, _P, _P, _P,
+                                       ctypes.c_uint64, _P]
         L.oracle_run.restype = ctypes.c_uint64
         L.oracle_run.argtypes = [_P, _P, _P, _P, ctypes.c_uint32, ctypes.c_uint64, _P, _P, _P,
                                  ctypes.c_uint64, _P, _P]
@@ -202,6 +205,28 @@ class OracleChain:
         npairs = lib().oracle_run(self.h, arena.ctypes.data, off.ctypes.data, ln.ctypes.data, n, first,
                                   res.ctypes.data, mp.ctypes.data, mq.ctypes.data, match_cap,
                                   self.stats.ctypes.data, None if so is None else so.ctypes.data)
+        k = min(int(npairs), match_cap)
+        return res, arena, (mp[:k].copy(), mq[:k].copy()), int(npairs)
+
+    def run_reorg(self, b: nfcgen.Batch, group, arena: Optional[np.ndarray] = None, match_cap: int = 1 << 20):
+        """The chain re-organized into parallel groups (oracle_run_reorg: per-NF packet
+        copies + XOR merge).  group[p] = group index of chain position p.
+        Returns like run(); raises ValueError for an invalid grouping."""
+        if arena is None:
+            arena = b.arena.copy()
+        off = np.ascontiguousarray(b.off, dtype=np.uint64)
+        ln = np.ascontiguousarray(b.len, dtype=np.uint16)
+        n = len(off)
+        g = np.zeros(8, dtype=np.uint8)
+        g[:len(group)] = group
+        res = np.zeros(n, dtype=nfcgen.RESULT)
+        mp = np.zeros(max(1, match_cap), dtype=np.uint32)
+        mq = np.zeros(max(1, match_cap), dtype=np.uint16)
+        npairs = lib().oracle_run_reorg(self.h, g.ctypes.data, arena.ctypes.data, off.ctypes.data, ln.ctypes.data, n,
+                                        b.first_index, res.ctypes.data, mp.ctypes.data, mq.ctypes.data, match_cap,
+                                        self.stats.ctypes.data)
+        if npairs == (1 << 64) - 1:
+            raise ValueError(f"invalid grouping {list(group)}")
         k = min(int(npairs), match_cap)
         return res, arena, (mp[:k].copy(), mq[:k].copy()), int(npairs)
 

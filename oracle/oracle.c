@@ -704,3 +704,184 @@ uint64_t oracle_run(or_chain *c, uint8_t *arena, const uint64_t *off, const uint
     free(ids);
     return n_pairs;
 }
+
+/* ======================================================================
+ * SFC parallelization with packet copies and XOR merge (P:L243-263
+ * [SIV.B.1]; semantics in oracle.h).  Written independently of oracle_run
+ * above (which stays the definition): each NF here acts on a private copy
+ * and reports its effects, which the group merge then commits.
+ * ==================================================================== */
+typedef struct {
+    int dropped, pass;              /* verdict of this NF on its copy */
+    int set_port; uint16_t port;
+    int acl; uint16_t acl_rule; uint32_t acl_hit;
+    int lb; uint16_t lb_backend;
+    int dpi; uint32_t n_ids; uint32_t *ids;
+} nf_eff;
+
+static void nf_on_copy(or_chain *c, uint32_t p, uint8_t *f, const pview *v, nf_eff *e)
+{
+    const or_spec *s = &c->s;
+    switch (s->kind[p]) {
+    case OR_ACL: {                       /* first matching rule */
+        int32_t rule = or_acl(c, (uint8_t)v->family, v->src, v->dst, v->sport, v->dport, v->proto);
+        uint32_t act;
+        e->acl = 1;
+        if (rule >= 0) { e->acl_rule = (uint16_t)rule; e->acl_hit = (uint32_t)rule; act = s->acl[rule].action; }
+        else { e->acl_rule = 0xFFFF; e->acl_hit = s->n_acl; act = s->acl_default; }
+        e->dropped = act == 1;
+        break;
+    }
+    case OR_DPI: {                       /* distinct pattern set of the payload */
+        int any_drop = 0;
+        e->dpi = 1;
+        e->n_ids = s->n_pat ? ac_scan(c, f + v->pl_off, (size_t)(v->ip_end - v->pl_off), e->ids, s->n_pat, &any_drop) : 0;
+        qsort(e->ids, e->n_ids, sizeof(uint32_t), cmp_u32);
+        e->dropped = any_drop;
+        break;
+    }
+    case OR_LPM4:
+    case OR_LPM6: {
+        int want = s->kind[p] == OR_LPM4 ? 4 : 6;
+        if (v->family != want) { e->pass = 1; break; }
+        int32_t nh;
+        const or_nexthop *tab;
+        if (want == 4) {
+            uint32_t d = ((uint32_t)v->dst[0] << 24) | ((uint32_t)v->dst[1] << 16) | ((uint32_t)v->dst[2] << 8) | v->dst[3];
+            nh = or_lpm4(c, d); tab = s->nh4;
+        } else {
+            nh = or_lpm6(c, v->dst); tab = s->nh6;
+        }
+        int ttl = want == 4 ? f[22] : f[21];
+        if (nh < 0 || ttl <= 1) { e->dropped = 1; break; }       /* R#12 */
+        forward_rewrite(f, v, &tab[nh], want == 4 ? s->pmac4 : s->pmac6, want == 4 ? s->n_port4 : s->n_port6);
+        e->set_port = 1;
+        e->port = tab[nh].port;
+        break;
+    }
+    case OR_LB: {                        /* flow hash -> backend */
+        uint8_t t[36];
+        size_t tl = tuple_bytes(v, t);
+        uint32_t h = or_toeplitz(s->lb_key, t, tl);
+        uint32_t b = (uint32_t)(((uint64_t)h * s->n_lb) >> 32);
+        e->lb = 1;
+        e->lb_backend = (uint16_t)b;
+        e->set_port = 1;
+        e->port = s->lb_port[b];
+        break;
+    }
+    default:
+        break;
+    }
+}
+
+uint64_t oracle_run_reorg(or_chain *c, const uint8_t *group, uint8_t *arena, const uint64_t *off,
+                          const uint16_t *len, uint32_t n, uint64_t first_global, or_result *res,
+                          uint32_t *match_pkt, uint16_t *match_pat, uint64_t match_cap, uint64_t *stats)
+{
+    const or_spec *s = &c->s;
+    /* grouping must be consecutive from 0; IPSEC alone in its group */
+    if (s->n_nf == 0 || group[0] != 0) return UINT64_MAX;
+    for (uint32_t p = 1; p < s->n_nf; p++)
+        if (group[p] != group[p - 1] && group[p] != group[p - 1] + 1) return UINT64_MAX;
+    for (uint32_t p = 0; p < s->n_nf; p++)
+        if (s->kind[p] == OR_IPSEC && ((p > 0 && group[p - 1] == group[p]) || (p + 1 < s->n_nf && group[p + 1] == group[p])))
+            return UINT64_MAX;
+    uint64_t n_pairs = 0;
+    uint64_t *acl_hits = stats + OR_ST_VAR_BASE;
+    uint64_t *lb_hits = acl_hits + s->n_acl + 1;
+    uint64_t *sa_pkts = lb_hits + s->n_lb;
+    uint32_t *idbuf = (uint32_t *)malloc((size_t)8 * (s->n_pat + 1) * sizeof(uint32_t));
+    uint8_t *orig = (uint8_t *)malloc(65536), *copy = (uint8_t *)malloc((size_t)8 * 65536);
+    for (uint32_t i = 0; i < n; i++) {
+        uint8_t *f = arena + off[i];
+        int flen = len[i];
+        or_result r = {0xFF, 0xFF, 0, 0xFFFF, 0xFFFF, 0, (uint16_t)flen, 0};
+        stats[OR_ST_PKTS]++;
+        stats[OR_ST_BYTES_IN] += (uint64_t)flen;
+        pview v;
+        int dropped = 0;
+        if (!parse(f, flen, &v)) {
+            r.drop_nf = 0xFE;
+            stats[OR_ST_PARSE_DROP]++;
+            dropped = 1;
+        }
+        uint32_t p0 = 0;
+        while (!dropped && p0 < s->n_nf) {
+            uint32_t p1 = p0;
+            while (p1 + 1 < s->n_nf && group[p1 + 1] == group[p0]) p1++;
+            if (s->kind[p0] == OR_IPSEC) {             /* singleton: applied to the packet itself */
+                uint64_t *ps = stats + OR_ST_POS_BASE + 4 * p0;
+                ps[0]++;
+                uint8_t t[36];
+                size_t tl = tuple_bytes(&v, t);
+                uint32_t sa = or_toeplitz(MS_RSS_KEY, t, tl) % s->n_sa;
+                uint32_t seq = ++c->seq[sa];
+                int ol = esp_apply(c, f, flen, &v, sa, seq, stats);
+                f -= 16;
+                flen = ol;
+                r.esp_sa = (uint8_t)sa;
+                r.esp_seq = seq;
+                r.out_len = (uint16_t)ol;
+                sa_pkts[sa]++;
+                ps[3]++;
+                parse(f, flen, &v);
+                p0 = p1 + 1;
+                continue;
+            }
+            /* duplicate the packet entering the group, run every member on its copy */
+            memcpy(orig, f, (size_t)flen);
+            nf_eff eff[8];
+            uint32_t m = p1 - p0 + 1;
+            for (uint32_t j = 0; j < m; j++) {
+                memset(&eff[j], 0, sizeof(nf_eff));
+                eff[j].ids = idbuf + (size_t)j * (s->n_pat + 1);
+                memcpy(copy + (size_t)j * 65536, orig, (size_t)flen);
+                nf_on_copy(c, p0 + j, copy + (size_t)j * 65536, &v, &eff[j]);
+            }
+            /* XOR merge: out = orig ^ OR_j (orig ^ copy_j) */
+            for (int k = 0; k < flen; k++) {
+                uint8_t acc = 0;
+                for (uint32_t j = 0; j < m; j++) acc |= (uint8_t)(orig[k] ^ copy[(size_t)j * 65536 + k]);
+                f[k] = (uint8_t)(orig[k] ^ acc);
+            }
+            /* commit in original order up to the earliest dropper */
+            for (uint32_t j = 0; j < m; j++) {
+                const uint32_t p = p0 + j;
+                uint64_t *ps = stats + OR_ST_POS_BASE + 4 * p;
+                nf_eff *e = &eff[j];
+                ps[0]++;
+                if (e->acl) { r.acl_rule = e->acl_rule; acl_hits[e->acl_hit]++; }
+                if (e->dpi) {
+                    r.dpi_nmatch = (uint16_t)e->n_ids;
+                    for (uint32_t q = 0; q < e->n_ids; q++) {
+                        if (n_pairs < match_cap) {
+                            match_pkt[n_pairs] = (uint32_t)(first_global + i);
+                            match_pat[n_pairs] = (uint16_t)e->ids[q];
+                        }
+                        n_pairs++;
+                    }
+                    stats[OR_ST_DPI_PAIRS] += e->n_ids;
+                }
+                if (e->lb) { r.lb_backend = e->lb_backend; lb_hits[e->lb_backend]++; }
+                if (e->set_port) r.port = e->port;
+                if (e->dropped) { ps[1]++; r.drop_nf = (uint8_t)p; dropped = 1; break; }
+                if (e->pass) ps[2]++;
+                else ps[3]++;
+            }
+            if (!dropped) parse(f, flen, &v);          /* the merged packet enters the next group */
+            p0 = p1 + 1;
+        }
+        if (dropped) {
+            r.port = 0xFFFF;
+            stats[OR_ST_DROP]++;
+        } else {
+            stats[OR_ST_FWD]++;
+            stats[OR_ST_BYTES_OUT] += r.out_len;
+        }
+        res[i] = r;
+    }
+    if (n_pairs > match_cap) stats[OR_ST_MATCH_OVF] += n_pairs - match_cap;
+    free(idbuf); free(orig); free(copy);
+    return n_pairs;
+}

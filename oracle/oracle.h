@@ -110,6 +110,22 @@ uint64_t oracle_run(or_chain *c, uint8_t *arena, const uint64_t *off, const uint
                     uint32_t *match_pkt, uint16_t *match_pat, uint64_t match_cap,
                     uint64_t *stats, const uint32_t *seq_override);
 
+/* SFC parallelization (P:L243-263 [SIV.B.1], Figs. 13-14): the chain is cut into
+ * groups of consecutive positions (group[p], non-decreasing from 0, consecutive);
+ * every NF of a group receives its own copy of the packet entering the group
+ * ("creates the copy of network packets and distributes them"), and the
+ * copies are merged by the paper's XOR rule: out = orig ^ OR_f (orig ^
+ * f(orig)).  Verdict: dropped iff some member dropped, at the smallest such
+ * position; side effects of members after that position are discarded ("the
+ * alert or log operation should be executed in the same packet state",
+ * P:L269).  Egress port: last setter in original order (R#19).  A group holding
+ * IPSEC must hold only IPSEC (it grows the packet, Table II "Add/Rm").
+ * Returns the number of match pairs, or UINT64_MAX if the grouping is invalid.
+ * Same outputs as oracle_run exactly when every group is parallel-legal. */
+uint64_t oracle_run_reorg(or_chain *c, const uint8_t *group, uint8_t *arena, const uint64_t *off,
+                          const uint16_t *len, uint32_t n, uint64_t first_global, or_result *res,
+                          uint32_t *match_pkt, uint16_t *match_pat, uint64_t match_cap, uint64_t *stats);
+
 /* ---- individual primitives, exported for the pin tests ---- */
 void or_aes128_encrypt_block(const uint8_t key[16], const uint8_t in[16], uint8_t out[16]);
 void or_aes128_ctr(const uint8_t key[16], const uint8_t ctr_block0[16], const uint8_t *in,

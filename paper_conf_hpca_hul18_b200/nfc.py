@@ -77,7 +77,7 @@ class Result(ctypes.Structure):
 
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
-           "nfc_launch_count", "nfc_last_launch", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
+           "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
@@ -101,6 +101,7 @@ def _load_lib():
     L.nfc_collect_stats.argtypes = [_P, _P, ctypes.c_size_t, _u32]
     L.nfc_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64)]
     L.nfc_last_launch.argtypes = [_P, _P]
+    L.nfc_plan_parallel.argtypes = [_P, _u32, _P]
     L.nfc_rss_shard.argtypes = [ctypes.c_int, ctypes.POINTER(Batch), _u32, _P, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
@@ -276,6 +277,14 @@ class Chain:
         _check(lib.nfc_last_launch(self.h, a.ctypes.data))
         return dict(zip(("grid", "block", "smem", "dfa_mode", "dfa_dense", "dfa_sparse", "dfa_meta_smem", "acl_smem"),
                         (int(x) for x in a)))
+
+
+def plan_parallel(kinds) -> list:
+    """nfc_plan_parallel: group index per chain position (SFC parallelization, NEXT-2)."""
+    k = np.array([KINDS[x] if isinstance(x, str) else int(x) for x in kinds], dtype=np.uint32)
+    g = np.zeros(max(1, len(k)), dtype=np.uint8)
+    _check(lib.nfc_plan_parallel(k.ctypes.data, len(k), g.ctypes.data))
+    return [int(x) for x in g[:len(k)]]
 
 
 def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,
