@@ -30,6 +30,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
 RESTORE_KINDS = {"IPSEC"}    # chains whose in-place rewrite changes the next step's work
+BATCH = 4096                  # one batch (C1: "one batch of 4,096 synthetic 64-B packets")
 
 
 def parse_args():
@@ -441,6 +442,55 @@ def main():
                    "what": "NFC_F_UNFUSED: one kernel per NF + device-side re-split, same ring and tables"}
         uch.close()
 
+    # NEXT-2: SFC parallelization -- the chain's NFs on different warps,
+    # each on its own packet copy, XOR-merged -- on the same ring, and the
+    # latency of ONE batch (the paper's Fig. 14 metric) for fused / parallel / unfused
+    parallel = None
+    if not args.no_unfused and not args.unfused and "IPSEC" not in w.kinds:
+        pch = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_PARALLEL)
+        pch.load_tables(w.tables)
+
+        def pstep():
+            mc.zero_()
+            pch.process(desc, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+        for _ in range(args.warmup):
+            pstep()
+        torch.cuda.synchronize(dev)
+        pe0, pe1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pe0.record(stream)
+        for _ in range(args.steps):
+            pstep()
+        pe1.record(stream)
+        torch.cuda.synchronize(dev)
+        p_t = torch.tensor([pe0.elapsed_time(pe1)], dtype=torch.float64, device=cdev)
+        if world > 1:
+            dist.all_reduce(p_t, op=dist.ReduceOp.MAX)
+        p_mpps = n * args.steps * world / (float(p_t.item()) / 1e3) / 1e6
+        # one batch of BATCH packets (C1's 4,096): median of 30 launches per arm
+        nb = min(n, BATCH)
+        bdesc = [(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), nb, first)]
+        uch2 = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_UNFUSED)
+        uch2.load_tables(w.tables)
+        lat = {}
+        for name, ch in (("fused", chain), ("parallel", pch), ("unfused", uch2)):
+            ts = []
+            for it in range(40):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                mc.zero_()
+                e0.record(stream)
+                ch.process(bdesc, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+                e1.record(stream)
+                torch.cuda.synchronize(dev)
+                if it >= 10:
+                    ts.append(e0.elapsed_time(e1) * 1e3)
+            lat[name + "_us"] = round(float(np.median(ts)), 2)
+        parallel = {"value": round(p_mpps, 3), "unit": "Mpps", "groups": nfc.plan_parallel(w.kinds),
+                    "fused_speedup": round(mpps / p_mpps, 3), "batch_pkts": nb, "batch_latency": lat,
+                    "what": "NFC_F_PARALLEL: NFs on different warps of a team, per-warp packet copies, XOR merge"}
+        uch2.close()
+        pch.close()
+        chain.stats(reset=True)
+
     cpu = None
     if not args.no_cpu and rank == 0 and world == 1:
         r_mpps, r_gbps, r_pk, r_t = oracle_rate(w, first, args.cpu_seconds)
@@ -467,6 +517,7 @@ def main():
             "roofline": roof,
             "cpu_baseline": cpu,
             "unfused_baseline": unfused,
+            "sfc_parallel": parallel,
             "e2e": e2e,
             "gpu_launches": int(launches),
             "clocks": clk.summary(),

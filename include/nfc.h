@@ -70,9 +70,16 @@ typedef struct nfc_chain nfc_chain; /* opaque; owned by the library */
                               * pipeline of P:L142-171.  Identical results; chains with
                               * NFC_IPSEC are rejected with NFC_EUNSUP.                  */
 
+#define NFC_F_PARALLEL 2u    /* SFC parallelization: the
+                              * chain's NFs (one parallel-legal group, nfc_plan_parallel)
+                              * run at once on different warps, each on its own copy of
+                              * a 32-packet chunk, merged by XOR with the earliest
+                              * dropper's later side effects discarded.  Identical
+                              * results; chains with NFC_IPSEC are rejected (NFC_EUNSUP). */
+
 typedef struct {
     int device;              /* CUDA device ordinal                                   */
-    uint32_t flags;          /* 0 (fused, the product) or NFC_F_UNFUSED               */
+    uint32_t flags;          /* 0 (fused, the product), NFC_F_UNFUSED or NFC_F_PARALLEL */
     uint32_t max_batch_pkts; /* hint: largest packet count per nfc_process_batch call */
 } nfc_chain_opts;
 

@@ -123,8 +123,10 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
         mask |= 1u << kinds[i];
     }
     const uint32_t flags = opts ? opts->flags : 0;
-    if (flags & ~NFC_F_UNFUSED) return fail(NFC_EINVAL, "opts->flags: unknown bits");
+    if (flags & ~(NFC_F_UNFUSED | NFC_F_PARALLEL)) return fail(NFC_EINVAL, "opts->flags: unknown bits");
+    if ((flags & NFC_F_UNFUSED) && (flags & NFC_F_PARALLEL)) return fail(NFC_EINVAL, "opts->flags: UNFUSED and PARALLEL are exclusive");
     if ((flags & NFC_F_UNFUSED) && (mask & (1u << NFC_IPSEC))) return fail(NFC_EUNSUP, "NFC_F_UNFUSED: IPsec chains are not offered");
+    if ((flags & NFC_F_PARALLEL) && (mask & (1u << NFC_IPSEC))) return fail(NFC_EUNSUP, "NFC_F_PARALLEL: IPsec chains are not offered");
     nfc_chain *c = new (std::nothrow) nfc_chain();
     if (!c) return fail(NFC_ENOMEM, "out of host memory");
     c->device = opts ? opts->device : 0;
@@ -373,13 +375,17 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     // per SM) when it fits next to the rest; otherwise a budget per CTA for the
     // target occupancy stages the ACL image and gives the rest to hot DFA rows.
     Variant v = sfc_variant(c->kind, c->n_nf, false);
+    const bool par = (c->flags & NFC_F_PARALLEL) != 0;
+    uint32_t n_fwd = 0;
+    for (uint32_t q = 0; q < c->n_nf; q++) n_fwd += (c->kind[q] == NFC_LPM4 || c->kind[q] == NFC_LPM6);
+    if (par) { v.sig = 0; v.dm = DM_HOT; v.threads = 768; }
     {
         const size_t limit = sfc_smem_limit(c->device);
         p.acl.smem_words = (c->mask & MASK_ACL) ? 1 : 0;
         p.dpi.hot_states = 0;
         p.dpi.sparse_states = 0;
         bool full = false;
-        if ((c->mask & MASK_DPI) && !c->dpi.wide && c->dpi.ncls <= 128) {
+        if (!par && (c->mask & MASK_DPI) && !c->dpi.wide && c->dpi.ncls <= 128) {
             Variant vf = sfc_variant(c->kind, c->n_nf, true);
             if (vf.dm == DM_FULL) {
                 p.dpi.hot_states = c->dpi.n_states;
@@ -401,7 +407,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
                 // tiered DFA: every row dense if it fits; else the depth <= 1 rows dense
                 // and as many sparse records (8 B) as fit after them (DpiImg::sparse)
                 p.dpi.sparse_states = 0;
-                const size_t base = sfc_smem_bytes(v, p), row = 2 * c->dpi.ncls;
+                const size_t base = par ? par_smem_bytes(p, n_fwd) + 16 : sfc_smem_bytes(v, p), row = 2 * c->dpi.ncls;
                 const size_t room = base < budget ? budget - base : 0;
                 if ((size_t)c->dpi.n_states * row <= room) {
                     p.dpi.hot_states = c->dpi.n_states;
@@ -420,7 +426,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         LaunchCfg q{};
         if (sfc_query(v, p, c->device, &q) != NFC_OK) return fail(NFC_ECUDA, "occupancy query failed");
         size_t threads = (size_t)q.grid * q.block;
-        if (c->flags & NFC_F_UNFUSED) {          // stage kernels may keep more threads resident
+        if (c->flags & (NFC_F_UNFUSED | NFC_F_PARALLEL)) {   // other kernels may keep more threads resident
             int sms = 0;
             cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
             threads = std::max(threads, (size_t)sms * 2048);
@@ -445,7 +451,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         return NFC_OK;
     }
     LaunchCfg lc{};
-    rc = sfc_launch(v, p, c->device, st, err, &lc);
+    rc = par ? par_launch(p, c->device, st, err, &lc) : sfc_launch(v, p, c->device, st, err, &lc);
     if (rc) return fail(rc, err);
     c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
                               (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states,

@@ -130,7 +130,7 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
 // byte offsets of the kernel's dynamic shared-memory regions (computed on the host per
 // launch, read by the kernel from the constant bank)
 struct SmemLayout {
-    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, total;
+    uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, par, total;
 };
 
 struct KParams {
@@ -145,6 +145,7 @@ struct KParams {
     uint32_t n_batches;
     uint32_t n_pkts;
     uint32_t n_tiles;
+    uint32_t claim;              // 32-packet chunks per work claim (set by the launcher)
     uint32_t *tile_counter;
     // outputs
     nfc_pkt_result *rec;
@@ -232,6 +233,9 @@ int sfc_query(const Variant &v, const KParams &p, int device, LaunchCfg *cfg_out
 // NFC_F_UNFUSED baseline (unfused.cu): parse stage, one stage kernel per NF, stats stage
 int uf_launch(const uint32_t *kinds, uint32_t n_nf, int dm, const KParams &p, uint32_t *list0, uint32_t *list1,
               uint32_t *counts, uint8_t *passmask, int device, void *stream, std::string &err, uint32_t *n_launch);
+// NFC_F_PARALLEL (parallel.cu): the chain's NFs on different warps of a team, XOR merge
+size_t par_smem_bytes(const KParams &p, uint32_t n_fwd);
+int par_launch(const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg);
 int rss_shard_launch(const uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n, const uint32_t *nib,
                      uint32_t n_shards, uint8_t *out, void *stream, std::string &err);
 

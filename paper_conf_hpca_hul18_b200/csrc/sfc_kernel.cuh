@@ -608,6 +608,7 @@ struct DpiOvf {
     uint16_t *match_pat;
     uint32_t match_cap;
     unsigned long long *stats;
+    uint32_t emit;          // 0: count ids and the DROP flag only (no pairs, no counters)
 };
 // one exact DFA step (state -> next, accept flag): the on-chip tiers as in dfa_entry
 // (DM_FULL: all rows; DM_HOT: dense rows / sparse records / global), or the global
@@ -670,7 +671,7 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         }
     }
     if (!ovf) {
-        if (n) {
+        if (n && o.emit) {
             const uint32_t slot = atomicAdd(o.match_count, n);
             for (uint32_t k = 0; k < n; k++)
                 if (slot + k < o.match_cap) { o.match_pkt[slot + k] = pkt_id; o.match_pat[slot + k] = ids[k]; }
@@ -680,7 +681,7 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         return n | drop << 31;
     }
     // more than DPI_LIST distinct ids: exact bitmap pass
-    atomicAdd(&o.stats[ST_DPI_OVF_PKTS], 1ull);
+    if (o.emit) atomicAdd(&o.stats[ST_DPI_OVF_PKTS], 1ull);
     uint32_t *bm = o.bitmap + (size_t)gtid * o.words;
     for (uint32_t k = 0; k < o.words; k++) bm[k] = 0;
     uint32_t cnt = 0;
@@ -700,6 +701,7 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
             if (bm[id >> 5] & bit) continue;
             bm[id >> 5] |= bit;
             cnt++;
+            if (!o.emit) continue;
             const uint32_t slot = atomicAdd(o.match_count, 1u);
             if (slot < o.match_cap) { o.match_pkt[slot] = pkt_id; o.match_pat[slot] = (uint16_t)id; }
             else atomicAdd(&o.stats[ST_MATCH_OVF], 1ull);
@@ -743,7 +745,7 @@ __device__ __forceinline__ uint32_t lpm6_lookup(const Lpm6Img &t, const uint32_t
 // L2/L3 rewrite after an LPM hit (R#6): dst MAC = nh MAC, src MAC = port MAC,
 // TTL / hop limit - 1, IPv4 header checksum recomputed (RFC 1071, byte-order independent
 // sum over little-endian halves).  Writes the first 32 B of the frame.
-__device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm, uint64_t pol)
+__device__ __forceinline__ void forward_words(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm)
 {
     h[0] = nh.x;
     h[1] = (nh.y & 0xFFFF) | (pm.x << 16);
@@ -766,6 +768,10 @@ __device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], cons
     } else {
         h[5] -= 1u << 8;                      // hop limit: byte 21
     }
+}
+__device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm, uint64_t pol)
+{
+    forward_words(f, h, v, nh, pm);
     st_stream16(f, make_uint4(h[0], h[1], h[2], h[3]), pol);
     st_stream16(f + 16, make_uint4(h[4], h[5], h[6], h[7]), pol);
 }
@@ -1098,7 +1104,7 @@ __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &
 #endif
     } else if (w.cnt >= 1) {
         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
-                        P.match_cap, P.stats};
+                        P.match_cap, P.stats, 1u};
         const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
         k.nmatch = r & 0x7FFFFFFFu;
         dropped = (r >> 31) != 0;
@@ -1582,8 +1588,8 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // chunks per atomic claim), no CTA barriers; the next chunk is claimed and located (off/len loads, header
         // prefetch to L2) before the current one is processed
         uint32_t cbase = 0, cleft = 0;
-        auto claim = [&]() {                 // next 32-packet chunk; one atomic per NFC_CLAIM chunks
-            constexpr uint32_t CL = KCfg<S, DM>::claim;
+        auto claim = [&]() {                 // next 32-packet chunk; one atomic per P.claim chunks
+            const uint32_t CL = P.claim;
             if (cleft == 0) {
                 uint32_t b = 0;
                 if (lane == 0) b = atomicAdd(P.tile_counter, 32u * CL);
@@ -1696,13 +1702,18 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     int grid = sms * per_sm;
-    constexpr uint32_t CLW = 32u * KCfg<S, DM>::claim;   // packets per warp claim
-    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (p.n_pkts + CLW - 1) / CLW / KCfg<S, DM>::nwarp + 1;
+    // chunks per claim: NFC_CLAIM (DM_FULL) when every warp gets many claims, else 1 (large
+    // frames or small batches: the tail of the last claims would dominate)
+    const uint32_t chunks = (p.n_pkts + 31) / 32;
+    uint32_t claim = KCfg<S, DM>::claim;
+    if ((uint64_t)chunks < 16ull * claim * (uint64_t)grid * KCfg<S, DM>::nwarp) claim = 1;
+    const uint32_t units = KCfg<S, DM>::esp ? p.n_tiles : (chunks + claim - 1) / claim / KCfg<S, DM>::nwarp + 1;
     if (!query_only && (uint32_t)grid > units) grid = (int)units;
     if (grid < 1) grid = 1;
     if (cfg) { cfg->grid = grid; cfg->block = NT; cfg->smem = smem; }
     if (query_only) return NFC_OK;
     KParams q = p;
+    q.claim = claim;
     q.lay = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p, KCfg<S, DM>::nws, DM);
     sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(q);
     cudaError_t e = cudaGetLastError();

@@ -20,6 +20,7 @@ ACL, DPI, LPM4, LPM6, IPSEC, LB = 1, 2, 3, 4, 5, 6
 KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB}
 STATS_RESET = 1
 F_UNFUSED = 1   # nfc_chain_opts.flags: per-NF kernels with re-split (NEXT-1 baseline)
+F_PARALLEL = 2  # nfc_chain_opts.flags: the chain's NFs on different warps + XOR merge (NEXT-2)
 
 # stats vector layout
 ST_PKTS, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP = 0, 1, 2, 3, 4, 5

@@ -200,3 +200,25 @@ def test_unfused_baseline_parity(nfc, cfg, k):
     ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_UNFUSED)
     ch.load_tables(w.tables)
     check_parity(w, ch, 3001)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("cfg,k,pl", [("C1", None, None), ("C3", None, None), ("C5", 4, None), ("C5", 3, 0),
+                                      ("C5", 2, 1500)])
+def test_parallel_sfc_parity(nfc, cfg, k, pl):
+    """NEXT-2: the chain's NFs on different warps, each on its own packet copy, merged
+    by XOR with the earliest dropper's later side effects discarded (P:L243-263,
+    P:L269) -- the oracle's sequential results exactly (records, bytes, pairs, stats)."""
+    w = nfcgen.workload(cfg, k=k, pkt_len=pl, small=(cfg == "C3"))
+    w.traffic.ttl1_ppm = 10_000
+    w.traffic.malformed_ppm = 5_000
+    assert max(nfc.plan_parallel(w.kinds)) == 0          # one parallel-legal group
+    ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_PARALLEL)
+    ch.load_tables(w.tables)
+    check_parity(w, ch, 2999)
+
+
+@pytest.mark.gpu
+def test_parallel_rejects_ipsec(nfc):
+    with pytest.raises(nfc.NfcError):
+        nfc.Chain(["ACL", "IPSEC"], device=0, flags=nfc.F_PARALLEL)
