@@ -33,6 +33,12 @@ NFC_API int nfc_dbg_dpi_shape(nfc_dbg *d, uint32_t *n_states, uint32_t *n_classe
    steps taken from dense rows, sparse records and the full table. */
 NFC_API int nfc_dbg_dpi_tier(nfc_dbg *d, uint32_t hot, uint32_t sparse, const uint8_t *buf, size_t n,
                              uint16_t *ids, uint32_t cap, uint32_t *count, uint32_t *drop, uint32_t *tier_steps);
+/* DPI, slot image as the kernel's DM_FULL mode walks it (DpiImg::frows: signed slots,
+   accepting states negative).  Same outputs as nfc_dbg_dpi; events = accept events of the
+   walk; summary = the per-slot match summary the kernel reads when events == 1
+   (closure offset | size << 20 | DROP << 31), else 0.  events/summary may be NULL. */
+NFC_API int nfc_dbg_dpi_slot(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids, uint32_t cap,
+                             uint32_t *count, uint32_t *drop, uint32_t *events, uint32_t *summary);
 /* DPI tier shape: states of depth <= 1, states with a representable sparse record. */
 NFC_API int nfc_dbg_dpi_tier_shape(nfc_dbg *d, uint32_t *n_d1, uint32_t *n_sparse_ok);
 /* LPM4: next-hop index (0x7FFF = miss) and number of table reads (1 or 2). */

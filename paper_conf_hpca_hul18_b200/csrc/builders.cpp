@@ -323,6 +323,27 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
         for (uint32_t x = o0; x < o0 + nm; x++) drop |= o.action[o.out_ids[x]];
         o.out_meta[k] = (o0 < (1u << 20) && nm < 2047u) ? (o0 | nm << 20 | drop << 31) : DPI_META_NONE;
     }
+    // slot image (DpiImg::frows): non-accepting states 0.., accepting -1.. (BFS order);
+    // physical row of slot x = n_acc + x
+    o.frows.clear();
+    o.acc_id.clear();
+    o.acc_meta.clear();
+    o.n_acc = 0;
+    if (!o.wide) {
+        std::vector<int32_t> slot(n);
+        int32_t na = 0, nn = 0;
+        for (size_t k = 0; k < n; k++) slot[k] = outc[order[k]].empty() ? nn++ : -(++na);
+        o.n_acc = (uint32_t)na;
+        o.acc_id.assign(na, 0);
+        o.acc_meta.assign(na, 0);
+        for (size_t k = 0; k < n; k++)
+            if (slot[k] < 0) { o.acc_id[-slot[k] - 1] = (uint32_t)k; o.acc_meta[-slot[k] - 1] = o.out_meta[k]; }
+        o.frows.assign(n * ncls, 0);
+        for (size_t u = 0; u < n; u++) {
+            const size_t row = (size_t)(na + slot[newid[u]]);
+            for (int c = 0; c < ncls; c++) o.frows[row * ncls + c] = (int16_t)slot[newid[delta[u * ncls + c]]];
+        }
+    }
     return "";
 }
 

@@ -68,7 +68,7 @@ struct nfc_chain {
     // tables
     DBuf acl_r4, acl_r6;
     AclImg acl{};
-    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta, dpi_sparse;
+    DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta, dpi_sparse, dpi_frows, dpi_accid, dpi_accmeta;
     DpiImg dpi{};
     DBuf l4_tbl24, l4_long, l4_nh, l4_pmac;
     Lpm4Img l4{};
@@ -158,7 +158,7 @@ void nfc_destroy_chain(nfc_chain *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
-                   &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
+                   &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->dpi_frows, &c->dpi_accid, &c->dpi_accmeta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
@@ -212,7 +212,14 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
         CK(c->dpi_act.upload(d.action));
         CK(c->dpi_meta.upload(d.out_meta));
         CK(c->dpi_sparse.upload(d.sparse));
+        CK(c->dpi_frows.upload(d.frows));
+        CK(c->dpi_accid.upload(d.acc_id));
+        CK(c->dpi_accmeta.upload(d.acc_meta));
         c->dpi = DpiImg{};
+        c->dpi.frows = c->dpi_frows.as<int16_t>();
+        c->dpi.acc_id = c->dpi_accid.as<uint32_t>();
+        c->dpi.acc_meta = c->dpi_accmeta.as<uint32_t>();
+        c->dpi.n_acc = d.n_acc;
         c->dpi.out_meta = c->dpi_meta.as<uint32_t>();
         c->dpi.sparse = c->dpi_sparse.as<uint2>();
         c->dpi.n_d1 = d.n_d1;

@@ -143,6 +143,41 @@ int nfc_dbg_dpi_tier(nfc_dbg *d, uint32_t hot, uint32_t sparse, const uint8_t *b
     return NFC_OK;
 }
 
+int nfc_dbg_dpi_slot(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t *ids, uint32_t cap, uint32_t *count,
+                     uint32_t *drop, uint32_t *events, uint32_t *summary)
+{
+    if (!d || d->kind != NFC_DPI) return NFC_EINVAL;
+    const DpiHost &D = d->dpi;
+    if (D.wide || D.frows.empty()) return NFC_EINVAL;
+    std::vector<uint8_t> seen(D.action.size(), 0);
+    std::vector<uint16_t> got;
+    uint32_t s = 0, dr = 0, cnt = 0, mx = 0;
+    for (size_t i = 0; i < n; i++) {
+        // the kernel's DM_FULL step (sfc_kernel.cuh dfa_entry / dfa_step): the row of slot
+        // s is physical row n_acc + s; the entry is the next slot, sign-extended
+        const int32_t e = D.frows[(size_t)((int32_t)D.n_acc + (int32_t)s) * D.ncls + D.cls[buf[i]]];
+        s = (uint32_t)e;
+        cnt += s >> 31;
+        mx = std::max(mx, s);
+        if (e < 0) {
+            const uint32_t st = D.acc_id[~s];
+            for (uint32_t k = D.out_off[st]; k < D.out_off[st + 1]; k++) {
+                uint16_t id = D.out_ids[k];
+                dr |= D.action[id];
+                if (!seen[id]) { seen[id] = 1; got.push_back(id); }
+            }
+        }
+    }
+    std::sort(got.begin(), got.end());
+    for (uint32_t k = 0; k < got.size() && k < cap; k++) ids[k] = got[k];
+    *count = (uint32_t)got.size();
+    *drop = dr;
+    if (events) *events = cnt;
+    // the kernel's single-accept summary: acc_meta[~mx] (0 without exactly one event)
+    if (summary) *summary = cnt == 1 ? D.acc_meta[~mx] : 0u;
+    return NFC_OK;
+}
+
 int nfc_dbg_dpi_tier_shape(nfc_dbg *d, uint32_t *n_d1, uint32_t *n_sparse_ok)
 {
     if (!d || d->kind != NFC_DPI) return NFC_EINVAL;

@@ -63,6 +63,17 @@ struct DpiImg {
     uint32_t maxlen;             // longest pattern (bytes): a walk started maxlen - 1 bytes
                                  // early is in the exact state (warp-split payload walks)
     uint32_t sparse_states;      // per launch: records staged in shared memory
+    // Slot image (DM_FULL, the whole DFA in shared memory).  A state is named by a
+    // signed slot: non-accepting states 0, 1, 2, ... (root = 0), accepting states
+    // -1, -2, ... (both in BFS order).  Rows are stored so that the row of slot x
+    // starts x * row2 bytes from the row of slot 0 (accepting rows below it), and an
+    // entry is the next state's slot (s16).  A step is then one multiply-add and one
+    // sign-extending load, the accept test is the sign bit, and the unique accepting
+    // entry of a walk with one accept event is its largest entry as u32.
+    const int16_t *frows;        // n_states * ncls entries, physical row order
+    const uint32_t *acc_id;      // n_acc: BFS state id of accepting slot -(q+1)
+    const uint32_t *acc_meta;    // n_acc: out_meta of accepting slot -(q+1)
+    uint32_t n_acc;
 };
 static const uint32_t DPI_META_NONE = 0x7FFFFFFFu;
 
@@ -131,6 +142,7 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
 // launch, read by the kernel from the constant bank)
 struct SmemLayout {
     uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, par, total;
+    uint32_t frow0;               // DM_FULL: row of slot 0 (DpiImg::frows)
 };
 
 struct KParams {
@@ -186,6 +198,11 @@ struct DpiHost {
     uint32_t n_d1 = 0;               // states of depth <= 1 (BFS ids [0, n_d1))
     uint32_t maxlen = 0;             // longest pattern
     std::vector<uint2> sparse;       // per state: tier record (see DpiImg::sparse)
+    // slot image (DpiImg::frows), u16 DFAs only
+    std::vector<int16_t> frows;      // n_states rows of ncls signed slots, physical order
+    std::vector<uint32_t> acc_id;    // accept slot q (slot -(q+1)) -> BFS state id
+    std::vector<uint32_t> acc_meta;  // out_meta of accept slot q
+    uint32_t n_acc = 0;
 };
 std::string build_dpi(const nfc_dpi_spec &s, DpiHost &out);
 std::string build_lpm4(const nfc_lpm4_spec &s, std::vector<uint16_t> &tbl24, std::vector<uint16_t> &tbllong,

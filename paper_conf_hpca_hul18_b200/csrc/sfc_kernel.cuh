@@ -76,7 +76,7 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic (DM_FULL; DM_HOT: 1)
 #endif
 #ifndef NFC_FULL_THREADS
-#define NFC_FULL_THREADS 768   // DPI chains without IPsec: one CTA per SM
+#define NFC_FULL_THREADS 640   // DPI chains without IPsec: one CTA per SM (640: no spills at 96 regs)
 #endif
 #ifndef NFC_HOTBIG_THREADS
 #define NFC_HOTBIG_THREADS 768 // DPI chains without IPsec whose DFA is tiered (DM_HOT)
@@ -111,16 +111,20 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
 {
     SmemLayout L{};
     uint32_t o = 0;
+    // the DPI byte-class table first: offset 0 is a compile-time address for the walk
+    if (mask & MASK_DPI) { L.cls = o; o += dm == DM_FULL ? 256 : 256 * 4; }
     L.wst = o; o += nwarp * nws * 8;                                // per-warp private counters (u64)
     L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
     o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_DPI) {
-        L.cls = o; o += dm == DM_FULL ? 256 : 256 * 4;               // byte -> 2 * class (u8 / u32)
+        // L.cls (byte -> 2 * class, u8 / u32) sits at offset 0 (above)
         L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u;
+        L.frow0 = L.hot + p.dpi.n_acc * p.dpi.ncls * 2;            // DM_FULL slot rows
         L.sp = o; o += p.dpi.sparse_states * 8;
-        L.meta = o; o += p.dpi.meta_smem ? (p.dpi.n_states * 4 + 15) & ~15u : 0;
+        // match summaries: DM_FULL of the accepting slots only, else of every state
+        L.meta = o; o += p.dpi.meta_smem ? ((dm == DM_FULL ? p.dpi.n_acc : p.dpi.n_states) * 4 + 15) & ~15u : 0;
         L.seg = o; o += nwarp * 64 * 4;                             // split-walk accumulators (cnt, mx) x 32
     }
     o = (o + 15) & ~15u;
@@ -361,7 +365,8 @@ __device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t 
 // The four interval lookups (src, dst, sport, dport) run jointly: one bucket read
 // each on the top 8 key bits, then one loop of the image's max window depth
 // (a table property: warp-uniform trip count) with four independent compare
-// steps per iteration.  Header words come from the constant bank.
+// steps per iteration.  Header words come from the constant bank.  Generic version
+// (any image pointer; used by the unfused and parallel kernels).
 __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A6, const AclImg &ai, const PV &v)
 {
     if (v.fam == 4) {
@@ -396,6 +401,134 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
     return acl_match(A, hd, ai.default_action, js, jd, jsp, jdp, v.proto);
 }
 
+// Fused-kernel version: the image is addressed in one known space -- shared memory
+// (SM: 32-bit shared addresses, the image base a compile-time symbol plus a
+// constant-bank offset) or global (read-only path, 32-bit byte offsets from one
+// base) -- never through generic pointers.  The window search keeps byte offsets
+// into the key arrays and is unrolled up to 8 halvings, each guarded by the image
+// depth (constant bank, warp-uniform): a step is one load at a constant offset, a
+// compare and a predicated add.
+template <bool SM> struct AclMem {
+    const uint8_t *g;     // global image (SM == false)
+    uint32_t s;           // shared-memory byte offset of the image (SM == true)
+    template <typename T> __device__ __forceinline__ T at(uint32_t o) const
+    {
+        if constexpr (SM) return *reinterpret_cast<const T *>(nfc_smem + s + o);
+        else return __ldg(reinterpret_cast<const T *>(g + o));
+    }
+};
+template <bool SM>
+__device__ __forceinline__ uint32_t acl_match_w(const AclMem<SM> &M, const uint32_t *hd, uint32_t default_action,
+                                                uint32_t js, uint32_t jd, uint32_t jsp, uint32_t jdp, uint32_t proto)
+{
+    js = min(js, hd[2] - 1);
+    jd = min(jd, hd[3] - 1);
+    jsp = min(jsp, hd[4] - 1);
+    jdp = min(jdp, hd[5] - 1);
+    const uint32_t W = hd[1];
+    for (uint32_t w = 0; w < W; w++) {      // W == 1 up to 64 rules of the family
+        const uint2 a = M.template at<uint2>(4 * hd[9] + 8 * (js * W + w));
+        const uint2 b = M.template at<uint2>(4 * hd[11] + 8 * (jd * W + w));
+        const uint2 c = M.template at<uint2>(4 * hd[13] + 8 * (jsp * W + w));
+        const uint2 d = M.template at<uint2>(4 * hd[15] + 8 * (jdp * W + w));
+        const uint2 e = M.template at<uint2>(4 * hd[16] + 8 * (proto * W + w));
+        const uint32_t lo = a.x & b.x & c.x & d.x & e.x, hi = a.y & b.y & c.y & d.y & e.y;
+        if (lo | hi) return M.template at<uint32_t>(4 * (hd[17] + 64 * w + (lo ? __ffs(lo) - 1 : 31 + __ffs(hi))));
+    }
+    return 0xFFFFu | default_action << 31;
+}
+// shared-memory window search over absolute 32-bit shared addresses: D halvings
+// (compile-time), each a load at an immediate offset, a compare and a predicated add
+template <uint32_t H4>
+__device__ __forceinline__ void acl_step_s(uint32_t &a, uint32_t key)
+{
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(H4));
+    a += v <= key ? H4 : 0u;
+}
+template <int D>
+__device__ __forceinline__ void acl_search4_s(uint32_t &as, uint32_t &ad, uint32_t &asp, uint32_t &adp, const PV &v)
+{
+    if constexpr (D > 0) {
+        constexpr uint32_t H4 = 4u << (D - 1);
+        acl_step_s<H4>(as, v.src[0]);
+        acl_step_s<H4>(ad, v.dst[0]);
+        acl_step_s<H4>(asp, v.sport);
+        acl_step_s<H4>(adp, v.dport);
+        acl_search4_s<D - 1>(as, ad, asp, adp, v);
+    }
+}
+template <bool SM>
+__device__ __forceinline__ uint32_t acl_core(const AclMem<SM> &M4, const AclMem<SM> &M6, const AclImg &ai, const PV &v)
+{
+    if (v.fam == 4) {
+        const uint32_t *hd = ai.hdr4;
+        if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
+        const AclMem<SM> &M = M4;
+        const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport, kdp = v.dport;
+        // window starts (bucket reads on the top 8 key bits), as byte offsets
+        uint32_t os = 4 * hd[8] + 4 * M.template at<uint16_t>(4 * hd[18] + 2 * (ks >> 24));
+        uint32_t od = 4 * hd[10] + 4 * M.template at<uint16_t>(4 * hd[19] + 2 * (kd >> 24));
+        uint32_t osp = 4 * hd[12] + 4 * M.template at<uint16_t>(4 * hd[20] + 2 * (ksp >> 8));
+        uint32_t odp = 4 * hd[14] + 4 * M.template at<uint16_t>(4 * hd[21] + 2 * (kdp >> 8));
+        const uint32_t D = hd[23];
+        if constexpr (SM) {
+            // absolute shared addresses; one straight-line search per image depth
+            const uint32_t base = (uint32_t)__cvta_generic_to_shared(nfc_smem) + M.s;
+            uint32_t as = base + os, ad = base + od, asp = base + osp, adp = base + odp;
+            // (a uniform if-chain, not a switch: no indexed jump per packet)
+            if (D == 3) acl_search4_s<3>(as, ad, asp, adp, v);
+            else if (D == 2) acl_search4_s<2>(as, ad, asp, adp, v);
+            else if (D == 4) acl_search4_s<4>(as, ad, asp, adp, v);
+            else if (D == 1) acl_search4_s<1>(as, ad, asp, adp, v);
+            else if (D == 5) acl_search4_s<5>(as, ad, asp, adp, v);
+            else if (D > 5) {
+                for (int i = (int)D - 1; i >= 5; i--) {
+                    const uint32_t h4 = 4u << i;
+                    as += M.template at<uint32_t>(as - base + h4) <= ks ? h4 : 0u;
+                    ad += M.template at<uint32_t>(ad - base + h4) <= kd ? h4 : 0u;
+                    asp += M.template at<uint32_t>(asp - base + h4) <= ksp ? h4 : 0u;
+                    adp += M.template at<uint32_t>(adp - base + h4) <= kdp ? h4 : 0u;
+                }
+                acl_search4_s<5>(as, ad, asp, adp, v);
+            }
+            os = as - base; od = ad - base; osp = asp - base; odp = adp - base;
+        } else {
+            for (int i = (int)D - 1; i >= 0; i--) {
+                const uint32_t h4 = 4u << i;
+                os += M.template at<uint32_t>(os + h4) <= ks ? h4 : 0u;
+                od += M.template at<uint32_t>(od + h4) <= kd ? h4 : 0u;
+                osp += M.template at<uint32_t>(osp + h4) <= ksp ? h4 : 0u;
+                odp += M.template at<uint32_t>(odp + h4) <= kdp ? h4 : 0u;
+            }
+        }
+        return acl_match_w<SM>(M, hd, ai.default_action, (os >> 2) - hd[8], (od >> 2) - hd[10], (osp >> 2) - hd[12],
+                               (odp >> 2) - hd[14], v.proto);
+    }
+    const uint32_t *hd = ai.hdr6;
+    if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
+    const AclMem<SM> &M = M6;
+    uint32_t js = M.template at<uint16_t>(4 * hd[18] + 2 * (v.src[0] >> 24));
+    uint32_t jd = M.template at<uint16_t>(4 * hd[19] + 2 * (v.dst[0] >> 24));
+    uint32_t jsp = M.template at<uint16_t>(4 * hd[20] + 2 * (v.sport >> 8));
+    uint32_t jdp = M.template at<uint16_t>(4 * hd[21] + 2 * (v.dport >> 8));
+    for (uint32_t h = (1u << hd[23]) >> 1; h; h >>= 1) {
+        js = le128(M.template at<uint4>(4 * hd[8] + 16 * (js + h)), v.src) ? js + h : js;
+        jd = le128(M.template at<uint4>(4 * hd[10] + 16 * (jd + h)), v.dst) ? jd + h : jd;
+        jsp = M.template at<uint32_t>(4 * hd[12] + 4 * (jsp + h)) <= v.sport ? jsp + h : jsp;
+        jdp = M.template at<uint32_t>(4 * hd[14] + 4 * (jdp + h)) <= v.dport ? jdp + h : jdp;
+    }
+    return acl_match_w<SM>(M, hd, ai.default_action, js, jd, jsp, jdp, v.proto);
+}
+// the fused kernel's entry: image staged in shared memory (P.lay offsets) or global
+__device__ __forceinline__ uint32_t nf_acl_fused(const KParams &P, const PV &v)
+{
+    if (P.acl.smem_words)
+        return acl_core<true>(AclMem<true>{nullptr, P.lay.acl4}, AclMem<true>{nullptr, P.lay.acl6}, P.acl, v);
+    return acl_core<false>(AclMem<false>{reinterpret_cast<const uint8_t *>(P.acl.bv4), 0u},
+                           AclMem<false>{reinterpret_cast<const uint8_t *>(P.acl.bv6), 0u}, P.acl, v);
+}
+
 // ---------------------------------------------------------------- DPI
 // Aho-Corasick DFA walk over byte classes.  Transition entries are u16: next
 // state | ACCEPT << 15 (ACCEPT: the next state has a non-empty output set); u32
@@ -408,6 +541,11 @@ __device__ __forceinline__ uint32_t nf_acl(const uint32_t *A4, const uint32_t *A
 // seen).  Accept entries are >= 0x8000 > any other entry, so when cnt == 1 the
 // state after the only accept event is mx & 0x7FFF and the match set is its
 // output closure; cnt > 1 takes the exact re-walk (dpi_slow).
+// DM_FULL walks the slot image (DpiImg::frows) instead: s is a signed slot, an
+// entry is the next slot sign-extended to 32 bits, cnt += e >> 31, and the
+// accepting entries (negative) are the largest as u32, so with cnt == 1 the only
+// accepting slot is mx and ~mx indexes the accept tables.  The class table sits
+// at shared offset 0: a step is PRMT + LDS.U8 + IMAD + LDS.S16 (+ 2 ALU).
 struct DpiCtx {
     const uint32_t *cls;    // smem, 256 entries (DM_HOT)
     const uint8_t *cls8;    // smem, 256 entries (DM_FULL)
@@ -422,6 +560,7 @@ struct DpiCtx {
     const uint32_t *out_off;
     const uint16_t *out_ids;
     const uint8_t *pat_action;
+    const uint32_t *acc_id;   // DM_FULL: accepting slot -> state id
 };
 
 struct Walk { uint32_t s, cnt, mx; };
@@ -432,8 +571,14 @@ __device__ __forceinline__ uint32_t byte_of(uint32_t w, int k) { return __byte_p
 template <int DM>
 __device__ __forceinline__ uint32_t dfa_entry(const KParams &P, uint32_t s, uint32_t byte)
 {
-    if (DM == DM_FULL)
-        return *reinterpret_cast<const uint16_t *>(nfc_smem + P.lay.hot + (s * P.dpi.row2 + nfc_smem[P.lay.cls + byte]));
+    if (DM == DM_FULL) {     // slot image; class table at shared offset 0
+        // (uniform row base) + (per-lane offset): one LDS [R + UR] after the IMAD
+        const uint32_t rb = (uint32_t)__cvta_generic_to_shared(nfc_smem) + P.lay.frow0;
+        const uint32_t t = s * P.dpi.row2 + nfc_smem[byte];
+        int32_t e;
+        asm("{\n\t.reg .s16 h;\n\tld.shared.s16 h, [%1];\n\tcvt.s32.s16 %0, h;\n\t}" : "=r"(e) : "r"(rb + t));
+        return (uint32_t)e;
+    }
     // tiered rows (DpiImg::sparse): dense row, or a sparse record's base row with <= 2
     // exceptions, or (cold) the global table.  Branch-free: the sparse-record, dense-row
     // and cold loads are predicated.  cls[byte] = class (u32).
@@ -471,8 +616,13 @@ template <int DM>
 __device__ __forceinline__ void dfa_step(const KParams &P, Walk &w, uint32_t byte)
 {
     const uint32_t e = dfa_entry<DM>(P, w.s, byte);
-    w.s = e & 0x7FFFu;
-    w.cnt += e >> 15;
+    if (DM == DM_FULL) {
+        w.s = e;
+        w.cnt += e >> 31;
+    } else {
+        w.s = e & 0x7FFFu;
+        w.cnt += e >> 15;
+    }
     w.mx = max(w.mx, e);
 }
 // step only if `in` (bytes outside the payload leave the walk unchanged: s <= mx always)
@@ -483,9 +633,15 @@ __device__ __forceinline__ void dfa_step_if(const KParams &P, Walk &w, uint32_t 
     // discarded when the byte is outside the span
     uint32_t e = dfa_entry<DM>(P, w.s, byte);
     asm("" : "+r"(e));
-    e = in ? e : w.s;
-    w.s = e & 0x7FFFu;
-    w.cnt += e >> 15;
+    if (DM == DM_FULL) {     // the state keeps its sign: count only bytes inside the span
+        w.cnt += in ? e >> 31 : 0u;
+        e = in ? e : w.s;
+        w.s = e;
+    } else {
+        e = in ? e : w.s;
+        w.s = e & 0x7FFFu;
+        w.cnt += e >> 15;
+    }
     w.mx = max(w.mx, e);
 }
 __device__ __forceinline__ void dfa_step_wide(const DpiCtx &c, Walk &w, uint32_t byte, bool in)
@@ -618,8 +774,10 @@ __device__ __forceinline__ uint32_t dfa_step_global(const DpiCtx &c, uint32_t s,
 {
     if (!c.wide) {
         uint32_t e;
-        if (DM == DM_FULL) {
-            e = *reinterpret_cast<const uint16_t *>(c.hot + s * c.row2 + c.cls8[b]);
+        if (DM == DM_FULL) {     // slot image: s and the result are slots (c.hot = row of slot 0)
+            const int32_t x = *reinterpret_cast<const int16_t *>(c.hot + (int32_t)s * (int32_t)c.row2 + c.cls8[b]);
+            acc = x < 0;
+            return (uint32_t)x;
         } else {
             const uint32_t cl = c.cls[b];
             const bool sp = s >= c.H;
@@ -644,6 +802,13 @@ __device__ __forceinline__ uint32_t dfa_step_global(const DpiCtx &c, uint32_t s,
     acc = (e >> 15) & 1;
     return e & 0x7FFFu;
 }
+// BFS state id of an accepting walk state (DM_FULL walks slots)
+template <int DM>
+__device__ __forceinline__ uint32_t dfa_out_state(const DpiCtx &c, uint32_t s)
+{
+    if (DM == DM_FULL && !c.wide) return __ldg(c.acc_id + ~s);
+    return s;
+}
 template <int DM>
 static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uint32_t a, uint32_t b, uint32_t gtid,
                                           DpiOvf o, uint32_t pkt_id)
@@ -659,8 +824,9 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         bool acc;
         s = dfa_step_global<DM>(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
-        const uint32_t e = __ldg(c.out_off + s + 1);
-        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+        const uint32_t so = dfa_out_state<DM>(c, s);
+        const uint32_t e = __ldg(c.out_off + so + 1);
+        for (uint32_t x = __ldg(c.out_off + so); x < e; x++) {
             const uint32_t id = __ldg(c.out_ids + x);
             drop |= __ldg(c.pat_action + id);
             bool seen = false;
@@ -693,8 +859,9 @@ static __device__ __noinline__ uint32_t dpi_slow(DpiCtx c, const uint8_t *f, uin
         bool acc;
         s = dfa_step_global<DM>(c, s, (wd >> ((i & 3) * 8)) & 0xFF, acc);
         if (!acc) continue;
-        const uint32_t e = __ldg(c.out_off + s + 1);
-        for (uint32_t x = __ldg(c.out_off + s); x < e; x++) {
+        const uint32_t so = dfa_out_state<DM>(c, s);
+        const uint32_t e = __ldg(c.out_off + so + 1);
+        for (uint32_t x = __ldg(c.out_off + so); x < e; x++) {
             const uint32_t id = __ldg(c.out_ids + x);
             drop |= __ldg(c.pat_action + id);
             const uint32_t bit = 1u << (id & 31);
@@ -1086,7 +1253,8 @@ template <int DM>
 __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &k, const Walk w)
 {
     bool dropped = false;
-    const uint32_t st = C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
+    // DM_FULL: C.meta holds the accepting slots' summaries (index ~slot)
+    const uint32_t st = DM == DM_FULL ? ~w.mx : C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
     const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
     if (w.cnt == 1 && meta != DPI_META_NONE) {
         // exactly one accept event: the match set is the output closure of that state
@@ -1238,7 +1406,7 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
 {
     bool dropped = false;
     if constexpr (KIND == NFC_ACL) {
-        const uint32_t r = nf_acl(C.acl4, C.acl6, P.acl, k.v);
+        const uint32_t r = nf_acl_fused(P, k.v);
         const uint32_t rule = r & 0xFFFF;
         k.acl_rule = rule;
         var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
@@ -1492,7 +1660,7 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
     C.dpi.cls8 = smem + L.cls;
     C.dpi.gcls = P.dpi.cls;
     C.dpi.sm = smem;
-    C.dpi.hot = smem + L.hot;
+    C.dpi.hot = smem + (DM == DM_FULL ? L.frow0 : L.hot);   // DM_FULL: row of slot 0
     C.dpi.row2 = 2 * P.dpi.ncls;
     C.dpi.ncls = P.dpi.ncls;
     C.dpi.wide = DM == DM_FULL ? 0 : P.dpi.wide;
@@ -1500,9 +1668,11 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
     C.dpi.out_off = P.dpi.out_off;
     C.dpi.out_ids = P.dpi.out_ids;
     C.dpi.pat_action = P.dpi.pat_action;
+    C.dpi.acc_id = P.dpi.acc_id;
     C.dpi.H = 0;
     C.dpi.HK2 = 0;
-    C.meta = P.dpi.meta_smem ? reinterpret_cast<const uint32_t *>(smem + L.meta) : P.dpi.out_meta;
+    C.meta = P.dpi.meta_smem ? reinterpret_cast<const uint32_t *>(smem + L.meta)
+                             : DM == DM_FULL ? P.dpi.acc_meta : P.dpi.out_meta;
     if ((SMASK & MASK_ACL) && (mask & MASK_ACL)) {
         if (P.acl.smem_words) {
             uint4 *d4 = reinterpret_cast<uint4 *>(smem + L.acl4);
@@ -1526,7 +1696,9 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         }
         const uint32_t H = C.dpi.wide ? 0 : P.dpi.hot_states;
         uint16_t *hot = reinterpret_cast<uint16_t *>(smem + L.hot);
-        const uint16_t *tr = reinterpret_cast<const uint16_t *>(P.dpi.trans);
+        // DM_FULL stages the slot image (DpiImg::frows), DM_HOT the BFS-ordered table
+        const uint16_t *tr = DM == DM_FULL ? reinterpret_cast<const uint16_t *>(P.dpi.frows)
+                                           : reinterpret_cast<const uint16_t *>(P.dpi.trans);
         const uint32_t nh = H * P.dpi.ncls;
         if ((nh & 7) == 0) {
             for (uint32_t i = tid; i < nh / 8; i += NT) reinterpret_cast<uint4 *>(hot)[i] = __ldg(reinterpret_cast<const uint4 *>(tr) + i);
@@ -1544,7 +1716,10 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         }
         if (P.dpi.meta_smem) {
             uint32_t *mt = reinterpret_cast<uint32_t *>(smem + L.meta);
-            for (uint32_t i = tid; i < P.dpi.n_states; i += NT) mt[i] = __ldg(P.dpi.out_meta + i);
+            if (DM == DM_FULL)
+                for (uint32_t i = tid; i < P.dpi.n_acc; i += NT) mt[i] = __ldg(P.dpi.acc_meta + i);
+            else
+                for (uint32_t i = tid; i < P.dpi.n_states; i += NT) mt[i] = __ldg(P.dpi.out_meta + i);
         }
     }
     if ((SMASK & MASK_IPSEC) && has_esp) {

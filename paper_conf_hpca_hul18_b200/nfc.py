@@ -80,7 +80,7 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
-                 "nfc_dbg_dpi_tier_shape", "nfc_dbg_lpm4",
+                 "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
                  "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
 
@@ -114,6 +114,7 @@ def _load_lib():
     L.nfc_dbg_dpi_shape.argtypes = [_P, P32, P32, P32]
     L.nfc_dbg_dpi_tier.argtypes = [_P, _u32, _u32, _P, ctypes.c_size_t, _P, _u32, P32, P32, _P]
     L.nfc_dbg_dpi_tier_shape.argtypes = [_P, P32, P32]
+    L.nfc_dbg_dpi_slot.argtypes = [_P, _P, ctypes.c_size_t, _P, _u32, P32, P32, P32, P32]
     L.nfc_dbg_lpm4.argtypes = [_P, _u32, P32, P32]
     L.nfc_dbg_lpm6.argtypes = [_P, _P, P32, P32, P32]
     L.nfc_dbg_lpm6_levels.argtypes = [_P, P32]
@@ -349,6 +350,14 @@ class HostImage:
         _check(lib.nfc_dbg_dpi_tier(self.h, hot, sparse, _cbuf(data), len(data), ids.ctypes.data, cap,
                                     ctypes.byref(c), ctypes.byref(d), ts.ctypes.data))
         return [int(x) for x in ids[:min(c.value, cap)]], bool(d.value), [int(x) for x in ts]
+
+    def dpi_slot(self, data: bytes, cap: int = 65536):
+        """The kernel's DM_FULL walk over the slot image; returns (ids, drop, events, summary)."""
+        ids = np.zeros(cap, dtype=np.uint16)
+        c, d, ev, sm = _u32(), _u32(), _u32(), _u32()
+        _check(lib.nfc_dbg_dpi_slot(self.h, _cbuf(data), len(data), ids.ctypes.data, cap, ctypes.byref(c),
+                                    ctypes.byref(d), ctypes.byref(ev), ctypes.byref(sm)))
+        return [int(x) for x in ids[:min(c.value, cap)]], bool(d.value), ev.value, sm.value
 
     def dpi_tier_shape(self):
         a, b = _u32(), _u32()

@@ -104,6 +104,46 @@ def test_dfa_tiered_walk_vs_oracle(nfc, case):
         assert nok >= 0.99 * (ns - nd1)         # nearly every deep state has <= 2 exceptions
 
 
+@pytest.mark.parametrize("case", ["c1", "c5", "tiny", "allbytes"])
+def test_dfa_slot_walk_vs_oracle(nfc, case):
+    """The kernel's DM_FULL slot image (DpiImg::frows: signed slots, accepting states
+    negative, rows addressed relative to slot 0) gives the oracle's match sets, the
+    accept-event count of a brute-force scan, and -- for walks with exactly one accept
+    event -- a match summary (size, DROP flag) equal to the oracle's result."""
+    rng = random.Random(11 + len(case))
+    if case in ("c1", "c5"):
+        t = nfcgen.workload(case.upper()).tables
+    elif case == "allbytes":
+        pats = [bytes([b, (b * 7) & 255, b ^ 0x55]) for b in range(256)] + [b"\x00\x01\x02"]
+        t = _pattern_tables(pats, [rng.random() < 0.1 for _ in pats])
+    else:
+        pats = [bytes(rng.choice(b"ab") for _ in range(rng.randrange(1, 6))) for _ in range(16)]
+        t = _pattern_tables(pats)
+    img = nfc.HostImage("DPI", blob=t.pat_blob, off=t.pat_off, action=t.pat_action)
+    orc = oracle.OracleChain(["DPI"], t)
+    pats = t.patterns()
+    singles = 0
+    for k in range(200):
+        n = rng.randrange(0, 300)
+        text = bytes(rng.choice(b"ab") if case == "tiny" else rng.randrange(256) for _ in range(n))
+        for _ in range(rng.randrange(0, 3)):
+            p = rng.choice(pats)
+            i = rng.randrange(0, len(text) + 1)
+            text = text[:i] + p + text[i:]
+        want = orc.ac_match(text)
+        ids, drop, events, summary = img.dpi_slot(text)
+        assert ids == want
+        assert drop == any(t.pat_action[j] for j in ids)
+        # accept events = end positions at which some pattern occurs (brute force)
+        ends = sum(1 for e in range(1, len(text) + 1) if any(text[:e].endswith(p) for p in pats))
+        assert events == ends
+        if events == 1:
+            singles += 1
+            assert (summary >> 20) & 0x7FF == len(want)
+            assert bool(summary >> 31) == drop
+    assert singles > 0 or case == "tiny"     # binary texts always hit several patterns
+
+
 def test_dir24_8_vs_oracle_and_two_accesses(nfc):
     w = nfcgen.workload("C1")
     t = w.tables
