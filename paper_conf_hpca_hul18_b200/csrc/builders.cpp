@@ -175,6 +175,24 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
         for (int q = 0; q < 4; q++) offs[10 + q] = put_bk(BK[q]);
         blob[22] = steps;
         blob[23] = maxst;
+        // aggregate level (ABV, Baboescu & Varghese): per row, bit w of aggregate word
+        // w / 64 is set iff the row's bitset word w is non-zero.  The lookup ANDs the
+        // five aggregate rows first and examines only the candidate words, in order
+        // (first match = lowest rule index), so large rule sets need not scan W words.
+        const uint32_t WA = (Wd + 63) / 64;
+        auto put_agg = [&](const std::vector<uint64_t> &v) {
+            std::vector<uint64_t> ag(v.size() / Wd * WA, 0);
+            for (size_t j = 0; j < v.size() / Wd; j++)
+                for (uint32_t w = 0; w < Wd; w++)
+                    if (v[j * Wd + w]) ag[j * WA + w / 64] |= 1ull << (w % 64);
+            return put_bv(ag);
+        };
+        blob[24] = put_agg(F[0].bv);
+        blob[25] = put_agg(F[1].bv);
+        blob[26] = put_agg(F[2].bv);
+        blob[27] = put_agg(F[3].bv);
+        blob[28] = put_agg(vproto);
+        blob[29] = WA;
         while (blob.size() & 3) blob.push_back(0);   // 16-B multiple for staging copies
         for (int k = 0; k < 14; k++) blob[8 + k] = offs[k];
     }

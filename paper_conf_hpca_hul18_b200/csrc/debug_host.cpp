@@ -283,13 +283,25 @@ int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *
         memcpy(&x, A + off + 2 * ((size_t)j * W + w), 8);
         return x;
     };
-    for (uint32_t w = 0; w < W; w++) {
-        uint64_t x = bv(A[9], js, w) & bv(A[11], jd, w) & bv(A[13], jsp, w) & bv(A[15], jdp, w) & bv(A[16], proto, w);
-        if (x) {
-            uint32_t e = A[A[17] + 64 * w + __builtin_ctzll(x)];
-            *rule = e & 0xFFFF;
-            *action = e >> 31;
-            return NFC_OK;
+    // as the kernel (acl_match_w): W == 1 directly, else candidate words from the
+    // aggregate rows (ABV) in increasing order
+    const uint32_t WA = A[29];
+    for (uint32_t a = 0; a < (W == 1 ? 1u : WA); a++) {
+        uint64_t cand = 1;
+        if (W > 1) {   // aggregate rows: WA words per row
+            auto ag = [&](uint32_t off, uint32_t j) { uint64_t x; memcpy(&x, A + off + 2 * ((size_t)j * WA + a), 8); return x; };
+            cand = ag(A[24], js) & ag(A[25], jd) & ag(A[26], jsp) & ag(A[27], jdp) & ag(A[28], proto);
+        }
+        while (cand) {
+            const uint32_t w = 64 * a + __builtin_ctzll(cand);
+            uint64_t x = bv(A[9], js, w) & bv(A[11], jd, w) & bv(A[13], jsp, w) & bv(A[15], jdp, w) & bv(A[16], proto, w);
+            if (x) {
+                uint32_t e = A[A[17] + 64 * w + __builtin_ctzll(x)];
+                *rule = e & 0xFFFF;
+                *action = e >> 31;
+                return NFC_OK;
+            }
+            cand &= cand - 1;
         }
     }
     return NFC_OK;

@@ -21,7 +21,7 @@ namespace nfc {
 //   (257 u16 per field) on the top 8 key bits,  [22] search steps per field (8 bits each),
 //   [23] max steps.  Key arrays are 16-B aligned and followed by 2^maxsteps all-ones pad keys.  Bitsets are
 //   u64 at even offsets.
-static const uint32_t ACLBV_HDR = 24;
+static const uint32_t ACLBV_HDR = 32;   // [24..28] aggregate-row offsets, [29] WA
 struct AclImg {
     const uint32_t *bv4, *bv6;        // device blobs
     uint32_t words4, words6;          // blob sizes (u32 words)

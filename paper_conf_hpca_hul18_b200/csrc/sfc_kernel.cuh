@@ -75,6 +75,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_CLAIM
 #define NFC_CLAIM 4           // 32-packet chunks a warp claims per atomic (DM_FULL; DM_HOT: 1)
 #endif
+#ifndef NFC_SPEC
+#define NFC_SPEC 1            // speculative ACL || DPI head walk || TBL24 block (spec_ok)
+#endif
 #ifndef NFC_FULL_THREADS
 #define NFC_FULL_THREADS 640   // DPI chains without IPsec: one CTA per SM (640: no spills at 96 regs)
 #endif
@@ -355,9 +358,25 @@ __device__ __forceinline__ uint32_t acl_match(const uint32_t *A, const uint32_t 
     const uint64_t *vsp = reinterpret_cast<const uint64_t *>(A + hd[13]) + (size_t)jsp * W;
     const uint64_t *vdp = reinterpret_cast<const uint64_t *>(A + hd[15]) + (size_t)jdp * W;
     const uint64_t *vpr = reinterpret_cast<const uint64_t *>(A + hd[16]) + (size_t)proto * W;
-    for (uint32_t w = 0; w < W; w++) {
-        const uint64_t x = vs[w] & vd[w] & vsp[w] & vdp[w] & vpr[w];
-        if (x) return A[hd[17] + 64 * w + (__ffsll((long long)x) - 1)];
+    if (W == 1) {
+        const uint64_t x = vs[0] & vd[0] & vsp[0] & vdp[0] & vpr[0];
+        return x ? A[hd[17] + (__ffsll((long long)x) - 1)] : 0xFFFFu | default_action << 31;
+    }
+    // aggregate level: only words whose five rows are all non-zero are examined, in order
+    const uint32_t WA = hd[29];
+    const uint64_t *as = reinterpret_cast<const uint64_t *>(A + hd[24]) + (size_t)js * WA;
+    const uint64_t *ad = reinterpret_cast<const uint64_t *>(A + hd[25]) + (size_t)jd * WA;
+    const uint64_t *asp = reinterpret_cast<const uint64_t *>(A + hd[26]) + (size_t)jsp * WA;
+    const uint64_t *adp = reinterpret_cast<const uint64_t *>(A + hd[27]) + (size_t)jdp * WA;
+    const uint64_t *apr = reinterpret_cast<const uint64_t *>(A + hd[28]) + (size_t)proto * WA;
+    for (uint32_t a = 0; a < WA; a++) {
+        uint64_t cand = as[a] & ad[a] & asp[a] & adp[a] & apr[a];
+        while (cand) {
+            const uint32_t w = 64 * a + (__ffsll((long long)cand) - 1);
+            const uint64_t x = vs[w] & vd[w] & vsp[w] & vdp[w] & vpr[w];
+            if (x) return A[hd[17] + 64 * w + (__ffsll((long long)x) - 1)];
+            cand &= cand - 1;
+        }
     }
     return 0xFFFFu | default_action << 31;
 }
@@ -426,14 +445,36 @@ __device__ __forceinline__ uint32_t acl_match_w(const AclMem<SM> &M, const uint3
     jsp = min(jsp, hd[4] - 1);
     jdp = min(jdp, hd[5] - 1);
     const uint32_t W = hd[1];
-    for (uint32_t w = 0; w < W; w++) {      // W == 1 up to 64 rules of the family
+    auto word = [&](uint32_t w, uint32_t &lo, uint32_t &hi) {
         const uint2 a = M.template at<uint2>(4 * hd[9] + 8 * (js * W + w));
         const uint2 b = M.template at<uint2>(4 * hd[11] + 8 * (jd * W + w));
         const uint2 c = M.template at<uint2>(4 * hd[13] + 8 * (jsp * W + w));
         const uint2 d = M.template at<uint2>(4 * hd[15] + 8 * (jdp * W + w));
         const uint2 e = M.template at<uint2>(4 * hd[16] + 8 * (proto * W + w));
-        const uint32_t lo = a.x & b.x & c.x & d.x & e.x, hi = a.y & b.y & c.y & d.y & e.y;
-        if (lo | hi) return M.template at<uint32_t>(4 * (hd[17] + 64 * w + (lo ? __ffs(lo) - 1 : 31 + __ffs(hi))));
+        lo = a.x & b.x & c.x & d.x & e.x;
+        hi = a.y & b.y & c.y & d.y & e.y;
+    };
+    uint32_t lo, hi;
+    if (W == 1) {                 // up to 64 rules of the family
+        word(0, lo, hi);
+        if (lo | hi) return M.template at<uint32_t>(4 * (hd[17] + (lo ? __ffs(lo) - 1 : 31 + __ffs(hi))));
+        return 0xFFFFu | default_action << 31;
+    }
+    // aggregate level (builders.cpp "ABV"): only words whose five rows are non-zero
+    const uint32_t WA = hd[29];
+    for (uint32_t a = 0; a < WA; a++) {
+        const uint2 s0 = M.template at<uint2>(4 * hd[24] + 8 * (js * WA + a));
+        const uint2 s1 = M.template at<uint2>(4 * hd[25] + 8 * (jd * WA + a));
+        const uint2 s2 = M.template at<uint2>(4 * hd[26] + 8 * (jsp * WA + a));
+        const uint2 s3 = M.template at<uint2>(4 * hd[27] + 8 * (jdp * WA + a));
+        const uint2 s4 = M.template at<uint2>(4 * hd[28] + 8 * (proto * WA + a));
+        uint64_t cand = (uint64_t)(s0.x & s1.x & s2.x & s3.x & s4.x) | (uint64_t)(s0.y & s1.y & s2.y & s3.y & s4.y) << 32;
+        while (cand) {
+            const uint32_t w = 64 * a + (__ffsll((long long)cand) - 1);
+            word(w, lo, hi);
+            if (lo | hi) return M.template at<uint32_t>(4 * (hd[17] + 64 * w + (lo ? __ffs(lo) - 1 : 31 + __ffs(hi))));
+            cand &= cand - 1;
+        }
     }
     return 0xFFFFu | default_action << 31;
 }
@@ -1294,7 +1335,7 @@ __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &
 // combined into the owner's summary through shared memory, so the owner ends with
 // exactly the (cnt, mx) of a sequential walk, evaluated by dpi_finish.
 template <int DM>
-__device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt &k)
+__device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt &k, const Walk *head = nullptr)
 {
     const uint32_t FULL = 0xFFFFFFFFu, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (DM != DM_FULL && P.dpi.wide)          // > 32K states: per-lane walk from L2
@@ -1305,7 +1346,8 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
     Walk w{0, 0, 0};
     // DM_FULL: bytes below 64 from the header cache (registers); DM_HOT: everything
     // through the stream (one copy of the walk loop keeps the kernel's code small)
-    if (DM == DM_FULL && act) w = dpi_walk_head<DM>(P, k.h, a, b);
+    if (DM == DM_FULL && head) w = *head;     // walked speculatively with the ACL (spec_acl_dpi)
+    else if (DM == DM_FULL && act) w = dpi_walk_head<DM>(P, k.h, a, b);
     const uint32_t base = (DM != DM_FULL || a >= 64) ? (a & ~15u) : 64u;
     const uint32_t rem = act && b > base ? (b - base + 15) & ~15u : 0u;
     if (__any_sync(FULL, rem != 0)) {         // warp-uniform (64-B frames: never)
@@ -1400,6 +1442,83 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
     return act ? dpi_finish<DM>(P, C, k, w) : false;
 }
 
+// ---------------------------------------------------------------- speculative ACL || DPI || TBL24
+// Chains that open with ACL -> DPI (C1, C3, the C5 prefixes) on a whole-DFA launch:
+// the ACL classification, the DPI walk over the payload bytes in the header cache
+// and (if LPM4 follows) the DIR-24-8 first-level read are pure functions of the
+// parsed packet, so they are computed together in ONE basic block -- no branches,
+// the ACL window search with predicated steps -- and the scheduler interleaves the
+// ACL's shared-memory chain and the TBL24 read with the DFA chain.  Their effects are
+// then applied in chain order (nf_apply / nf_dpi_warp), so results equal the
+// sequential chain (effects in original-order packet state).  Taken when
+// warp-uniformly: IPv4 ACL image with rules, <= 64 rules, depth <= 3, staged in
+// shared memory; otherwise the sequential path runs.
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a)
+{
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u16z(uint32_t a)
+{
+    uint32_t v;
+    asm("{\n\t.reg .u16 t;\n\tld.shared.u16 t, [%1];\n\tcvt.u32.u16 %0, t;\n\t}" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds_u64(uint32_t a)
+{
+    uint2 v;
+    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+// IPv4 ACL, W == 1 image in shared memory, depth <= 3: straight-line (returns as acl_core)
+__device__ __forceinline__ uint32_t acl4_spec(const KParams &P, const PV &v)
+{
+    const uint32_t *hd = P.acl.hdr4;
+    const uint32_t B = (uint32_t)__cvta_generic_to_shared(nfc_smem) + P.lay.acl4;
+    // (lanes whose parse failed carry arbitrary fields: every index below stays in bounds)
+    const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport & 0xFFFF, kdp = v.dport & 0xFFFF;
+    uint32_t as = B + 4 * hd[8] + 4 * lds_u16z(B + 4 * hd[18] + 2 * (ks >> 24));
+    uint32_t ad = B + 4 * hd[10] + 4 * lds_u16z(B + 4 * hd[19] + 2 * (kd >> 24));
+    uint32_t asp = B + 4 * hd[12] + 4 * lds_u16z(B + 4 * hd[20] + 2 * (ksp >> 8));
+    uint32_t adp = B + 4 * hd[14] + 4 * lds_u16z(B + 4 * hd[21] + 2 * (kdp >> 8));
+    const uint32_t D = hd[23];
+#pragma unroll
+    for (int i = 2; i >= 0; i--) {
+        const uint32_t h4 = (uint32_t)i < D ? 4u << i : 0u;    // steps beyond the depth are no-ops
+        as += lds_u32(as + h4) <= ks ? h4 : 0u;
+        ad += lds_u32(ad + h4) <= kd ? h4 : 0u;
+        asp += lds_u32(asp + h4) <= ksp ? h4 : 0u;
+        adp += lds_u32(adp + h4) <= kdp ? h4 : 0u;
+    }
+    const uint32_t js = min((as - B) / 4 - hd[8], hd[2] - 1), jd = min((ad - B) / 4 - hd[10], hd[3] - 1);
+    const uint32_t jsp = min((asp - B) / 4 - hd[12], hd[4] - 1), jdp = min((adp - B) / 4 - hd[14], hd[5] - 1);
+    const uint2 a = lds_u64(B + 4 * hd[9] + 8 * js), b = lds_u64(B + 4 * hd[11] + 8 * jd);
+    const uint2 c = lds_u64(B + 4 * hd[13] + 8 * jsp), d = lds_u64(B + 4 * hd[15] + 8 * jdp);
+    const uint2 e = lds_u64(B + 4 * hd[16] + 8 * (v.proto & 255));   // (dead lanes: any value, in bounds)
+    const uint32_t lo = a.x & b.x & c.x & d.x & e.x, hi = a.y & b.y & c.y & d.y & e.y;
+    const uint32_t bit = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
+    uint32_t r = 0xFFFFu | P.acl.default_action << 31;
+    if (lo | hi) r = lds_u32(B + 4 * (hd[17] + bit));
+    return r;
+}
+// DPI walk of payload bytes [a, min(b, 64)) from the header cache for a >= 42, every
+// step predicated (UDP and TCP payload starts in one code path)
+__device__ __forceinline__ Walk dpi_head_spec(const KParams &P, const uint32_t h[16], uint32_t a, uint32_t b)
+{
+    Walk w{0, 0, 0};
+#pragma unroll
+    for (int idx = 42; idx < 64; idx++)
+        dfa_step_if<DM_FULL>(P, w, byte_of(h[idx >> 2], idx & 3), (uint32_t)idx - a < b - a);
+    return w;
+}
+template <uint32_t S>
+__device__ __forceinline__ bool spec_ok(const KParams &P)
+{
+    return S != SIG_ANY && sig_kind(S, 0) == NFC_ACL && sig_n(S) >= 2 && sig_kind(S, 1) == NFC_DPI &&
+           P.acl.smem_words && P.acl.hdr4[0] != 0 && P.acl.hdr4[1] == 1 && P.acl.hdr4[23] <= 3;
+}
+
 // one NF of kind KIND at chain position pos (KIND compile-time)
 template <uint32_t KIND, int DM>
 __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k, uint32_t pos)
@@ -1491,6 +1610,28 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
         // never placed before LPM4 in the instantiated signatures)
         static_assert(sig_pos(S, NFC_IPSEC) == 0xFF || sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4), "");
         if (k.alive && k.v.fam == 4) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+    }
+    if constexpr (NFC_SPEC && HEAD && S != SIG_ANY && DM == DM_FULL && sig_n(S) >= 2 && sig_kind(S, 0) == NFC_ACL &&
+                  sig_kind(S, 1) == NFC_DPI) {
+        // speculative ACL || DPI head walk || TBL24 (see spec_ok), warp-uniform choice
+        const bool v4 = !k.alive || (k.v.fam == 4 && k.v.pl_off >= 42);   // payload starts inside [42, 64) or later
+        if (spec_ok<S>(P) && __all_sync(0xFFFFFFFFu, v4)) {
+            const uint32_t r = acl4_spec(P, k.v);
+            const Walk wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
+            if constexpr (sig_pos(S, NFC_LPM4) != 0xFF && (sig_pos(S, NFC_IPSEC) == 0xFF ||
+                                                            sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4)))
+                k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+            if (k.alive) {                     // ACL effects (position 0)
+                const uint32_t rule = r & 0xFFFF;
+                k.acl_rule = rule;
+                var_stat(P, C, P.st_acl + (rule == 0xFFFF ? P.acl.n_rules : rule));
+                if (r >> 31) { k.drop = 0; k.alive = false; }
+            }
+            if (nf_dpi_warp<DM>(P, C, k, &wh)) { k.drop = 1; k.alive = false; }
+            constexpr int E = sig_pos(S, NFC_IPSEC) == 0xFF ? (int)sig_n(S) : (int)sig_pos(S, NFC_IPSEC);
+            run_fixed<S, DM, 2, E>(P, C, k);
+            return;
+        }
     }
     if constexpr (S == SIG_ANY) {
         const uint32_t e = min(P.esp_pos, P.n_nf);
@@ -1782,10 +1923,13 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
         Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
         while (c0 < P.n_pkts) {
-            const uint32_t c2 = claim();
-            const Raw raw2 = pkt_raw(P, c2 + lane, c2 + lane < P.n_pkts);
+            // locate chunk c1 (its descriptors arrived during the last chunk) BEFORE issuing
+            // the descriptor loads of c2: an address add that consumed a just-issued load's
+            // scoreboard slot would wait for that DRAM read and undo the two-ahead pipeline
             const Loc loc1 = pkt_loc(P, raw1, c1 + lane, c1 + lane < P.n_pkts);
             if (c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(loc1.f));
+            const uint32_t c2 = claim();
+            const Raw raw2 = pkt_raw(P, c2 + lane, c2 + lane < P.n_pkts);
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;

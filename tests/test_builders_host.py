@@ -231,18 +231,21 @@ def test_lpm6_adversarial_nesting(nfc):
         assert img.lpm6(dst)[0] == (0x7FFF if want < 0 else want)
 
 
-@pytest.mark.parametrize("fam", [4, 6])
-def test_acl_image_vs_oracle(nfc, fam):
-    rng = np.random.default_rng(40 + fam)
-    rules = np.concatenate([nfcgen.gen_acl(rng, 40, 4), nfcgen.gen_acl(rng, 40, 6)])
+@pytest.mark.parametrize("fam,n", [(4, 40), (6, 40), (4, 1000), (4, 10000), (6, 1000)])
+def test_acl_image_vs_oracle(nfc, fam, n):
+    """Bit-vector image (one 64-bit word per field for <= 64 rules, else the aggregate
+    level picks candidate words, ABV) == linear first-match scan, up to the paper's
+    10K-rule ACL."""
+    rng = np.random.default_rng(40 + fam + n)
+    rules = np.concatenate([nfcgen.gen_acl(rng, n, 4), nfcgen.gen_acl(rng, n if fam == 6 else 40, 6)])
     rng.shuffle(rules)
     t = nfcgen.Tables(acl_rules=rules, acl_default=1)
     img = nfc.HostImage("ACL", rules=rules, default_action=1)
     orc = oracle.OracleChain(["ACL"], t)
-    r = random.Random(fam)
+    r = random.Random(fam + n)
     nb = 4 if fam == 4 else 16
     fam_idx = [i for i in range(len(rules)) if rules[i]["family"] == fam]
-    for _ in range(3000):
+    for _ in range(3000 if n <= 1000 else 600):
         src = bytearray(r.getrandbits(8) for _ in range(nb))
         dst = bytearray(r.getrandbits(8) for _ in range(nb))
         sp, dp, proto = r.getrandbits(16), r.getrandbits(16), r.choice([1, 6, 17])
