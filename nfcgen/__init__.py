@@ -37,10 +37,14 @@ SA = np.dtype([("spi", "<u4"), ("seq0", "<u4"), ("aes_key", "u1", (16,)), ("nonc
 RESULT = np.dtype([("drop_nf", "u1"), ("esp_sa", "u1"), ("port", "<u2"), ("acl_rule", "<u2"),
                    ("lb_backend", "<u2"), ("dpi_nmatch", "<u2"), ("out_len", "<u2"),
                    ("esp_seq", "<u4")])
+NAT_PREFIX = np.dtype([("prefix", "<u4"), ("len", "u1"), ("pad", "u1", (3,))])
+NAT_DNAT = np.dtype([("ext_addr", "<u4"), ("ext_port", "<u2"), ("proto", "u1"), ("pad", "u1"),
+                     ("int_addr", "<u4"), ("int_port", "<u2"), ("pad2", "<u2")])
+assert NAT_PREFIX.itemsize == 8 and NAT_DNAT.itemsize == 16
 assert ACL_RULE.itemsize == 48 and ROUTE4.itemsize == 8 and ROUTE6.itemsize == 20
 assert NEXTHOP.itemsize == 8 and SA.itemsize == 48 and RESULT.itemsize == 16
 
-KINDS = {"ACL": 1, "DPI": 2, "LPM4": 3, "LPM6": 4, "IPSEC": 5, "LB": 6}
+KINDS = {"ACL": 1, "DPI": 2, "LPM4": 3, "LPM6": 4, "IPSEC": 5, "LB": 6, "NAT": 7}
 KIND_NAMES = {v: k for k, v in KINDS.items()}
 
 
@@ -60,6 +64,13 @@ class Tables:
     sas: Optional[np.ndarray] = None
     lb_ports: Optional[np.ndarray] = None      # u16
     lb_key: Optional[np.ndarray] = None        # u8[40]
+    nat_inside: Optional[np.ndarray] = None    # NAT_PREFIX
+    nat_pool: Optional[np.ndarray] = None      # u32 public addresses (host-order values)
+    nat_port_lo: int = 1024
+    nat_port_hi: int = 65535
+    nat_dnat: Optional[np.ndarray] = None      # NAT_DNAT
+    nat_ext_ports: int = 0                     # bit p: egress port p faces the Internet
+    nat_key: Optional[np.ndarray] = None       # u8[40]
 
     @property
     def n_pat(self) -> int:
@@ -87,6 +98,7 @@ class TrafficParams:
     printable: int = 1
     headroom: int = 0
     tailroom: int = 0
+    l4csum: int = 0             # 1: arbitrary TCP/UDP checksum values (NAT updates them)
 
 
 @dataclass
@@ -103,7 +115,8 @@ class Workload:
 class _GenParams(ctypes.Structure):
     _fields_ = [("seed", ctypes.c_uint64), ("n_flows", ctypes.c_uint64)] + [
         (n, ctypes.c_uint32) for n in ("v6_bp", "pkt_len", "match_ppm", "in_acl_pct", "tcp_pct", "ttl",
-                                       "ttl1_ppm", "malformed_ppm", "printable", "headroom", "tailroom")]
+                                       "ttl1_ppm", "malformed_ppm", "printable", "headroom", "tailroom",
+                                       "l4csum")]
 
 
 _P = ctypes.c_void_p
@@ -139,6 +152,9 @@ def _load():
         _lib.nfcgen_fill.restype = None
         _lib.nfcgen_fill.argtypes = [ctypes.POINTER(_GenParams), ctypes.POINTER(_GenTables),
                                      ctypes.c_uint64, ctypes.c_uint32, _P, _P, _P]
+        _lib.nfcgen_flow.restype = None
+        _lib.nfcgen_flow.argtypes = [ctypes.POINTER(_GenParams), ctypes.POINTER(_GenTables), ctypes.c_uint64,
+                                     _P, _P, _P, _P, _P, _P]
         _lib.nfcgen_rnd.restype = ctypes.c_uint64
         _lib.nfcgen_rnd.argtypes = [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint64]
     return _lib
@@ -165,7 +181,7 @@ def _gen_structs(tp: TrafficParams, t: Tables):
     keep = _Keep()
     gp = _GenParams(tp.seed, tp.n_flows, tp.v6_bp, tp.pkt_len, tp.match_ppm, tp.in_acl_pct,
                     tp.tcp_pct, tp.ttl, tp.ttl1_ppm, tp.malformed_ppm, tp.printable,
-                    tp.headroom, tp.tailroom)
+                    tp.headroom, tp.tailroom, tp.l4csum)
     gt = _GenTables()
     if t.routes4 is not None and len(t.routes4):
         r4p = keep(t.routes4["prefix"].astype(np.uint32))
@@ -220,6 +236,20 @@ def generate(tp: TrafficParams, t: Tables, first: int, n: int) -> Batch:
         lib.nfcgen_fill(ctypes.byref(gp), ctypes.byref(gt), first, n, _ptr(arena), _ptr(off), _ptr(ln))
     del keep
     return Batch(arena, off, ln, first, tp.headroom, tp.tailroom)
+
+
+def flow(tp: TrafficParams, t: Tables, f: int):
+    """The 5-tuple of flow f: (family, src bytes, dst bytes, sport, dport, proto)."""
+    lib = _load()
+    gp, gt, keep = _gen_structs(tp, t)
+    fam = ctypes.c_uint32()
+    src, dst = (ctypes.c_uint8 * 16)(), (ctypes.c_uint8 * 16)()
+    sp, dp, pr = ctypes.c_uint16(), ctypes.c_uint16(), ctypes.c_uint8()
+    lib.nfcgen_flow(ctypes.byref(gp), ctypes.byref(gt), f, ctypes.byref(fam), src, dst, ctypes.byref(sp),
+                    ctypes.byref(dp), ctypes.byref(pr))
+    del keep
+    nb = 4 if fam.value == 4 else 16
+    return fam.value, bytes(src)[:nb], bytes(dst)[:nb], sp.value, dp.value, pr.value
 
 
 def rnd(seed: int, stream: int, idx: int) -> int:
@@ -387,6 +417,42 @@ def gen_lb(rng, n_backends: int, n_ports: int = 16):
             rng.integers(0, 256, 40, dtype=np.uint8))
 
 
+def gen_nat(rng, tp: "TrafficParams", t: Tables, n_dnat: int = 1000, n_inside: int = 8, n_pool: int = 64,
+            hit_frac: float = 0.5, n_ports: int = 16):
+    """NAT44 tables (R#30): n_inside distinct /4 inside prefixes (half of all source
+    addresses), a pool of public addresses, source ports 1024..65535, the upper half of
+    the router's ports Internet-facing, and n_dnat static DNAT entries of which
+    hit_frac are (proto, dst, dport) of real flows of the traffic."""
+    firsts = rng.choice(16, size=min(n_inside, 16), replace=False)
+    t.nat_inside = np.zeros(len(firsts), dtype=NAT_PREFIX)
+    t.nat_inside["prefix"] = firsts.astype(np.uint32) << 28
+    t.nat_inside["len"] = 4
+    t.nat_pool = rng.integers(0, 1 << 32, n_pool, dtype=np.uint64).astype(np.uint32)
+    t.nat_port_lo, t.nat_port_hi = 1024, 65535
+    t.nat_ext_ports = sum(1 << p for p in range(n_ports // 2, n_ports))
+    t.nat_key = rng.integers(0, 256, 40, dtype=np.uint8)
+    d = np.zeros(n_dnat, dtype=NAT_DNAT)
+    seen = set()
+    k = 0
+    while k < n_dnat:
+        if rng.random() < hit_frac:
+            fam, src, dst, sp, dpt, pr = flow(tp, t, int(rng.integers(0, tp.n_flows)))
+            if fam != 4 or pr not in (6, 17):
+                continue
+            key = (pr, int.from_bytes(dst, "big"), dpt)
+        else:
+            key = (int(rng.choice([6, 17])), int(rng.integers(0, 1 << 32)), int(rng.integers(0, 1 << 16)))
+        if key in seen:
+            continue
+        seen.add(key)
+        d[k]["proto"], d[k]["ext_addr"], d[k]["ext_port"] = key
+        d[k]["int_addr"] = (10 << 24) | int(rng.integers(0, 1 << 24))
+        d[k]["int_port"] = int(rng.integers(1, 1 << 16))
+        k += 1
+    t.nat_dnat = d
+    return t
+
+
 def make_tables(seed: int, kinds: List[str], n_acl=64, acl_family=4, n_pat=100, pat_kw=None,
                 n_r4=1000, n_r6=0, n_sa=64, n_lb=64, n_nh=64, n_ports=16,
                 acl_deny=0.10, acl6_extra=0) -> Tables:
@@ -418,7 +484,7 @@ C6_CHAIN = ["ACL", "DPI", "LPM4", "LPM6", "IPSEC", "LB"]   # DESIGN.md R#20
 
 
 def workload(name: str, pkt_len: Optional[int] = None, k: Optional[int] = None,
-             small: bool = False, seed: Optional[int] = None) -> Workload:
+             small: bool = False, seed: Optional[int] = None, acl_rules: Optional[int] = None) -> Workload:
     """BASELINE.json configs C1..C5; small=True shrinks tables for fast tests."""
     name = name.upper()
     if name == "C1":
@@ -466,4 +532,15 @@ def workload(name: str, pkt_len: Optional[int] = None, k: Optional[int] = None,
                            headroom=16 if esp else 0, tailroom=32 if esp else 0)
         return Workload(f"C5k{kk}", kinds, t, tp,
                         note=f"C6 chain prefix k={kk}, dual-stack 75/25")
+    if name == "N3":
+        # SURVEY 8(f) NEXT-3 (Figs. 16-17): FW -> router -> NAT with the
+        # paper's ACL sizes (200 / 1K / 10K rules) at 64 / 128 / 1500 B
+        kinds = ["ACL", "LPM4", "NAT"]
+        sd = 6 if seed is None else seed
+        n_acl = acl_rules or (200 if small else 1000)
+        t = make_tables(sd, kinds, n_acl=n_acl, n_r4=1000)
+        tp = TrafficParams(seed=sd, pkt_len=64 if pkt_len is None else pkt_len, match_ppm=0, tcp_pct=30,
+                           l4csum=1)
+        gen_nat(np.random.default_rng(np.random.PCG64(sd + 1000)), tp, t, n_dnat=1000 if not small else 200)
+        return Workload("N3", kinds, t, tp, note=f"FW({n_acl})->IPv4 router(1K)->NAT44, SNAT+DNAT")
     raise ValueError(name)

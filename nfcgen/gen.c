@@ -29,6 +29,7 @@ typedef struct {
     uint32_t malformed_ppm;  /* malformed frames (edge case), per million */
     uint32_t printable;      /* payload bytes drawn from 0x20..0x7e */
     uint32_t headroom, tailroom;
+    uint32_t l4csum;         /* 1: arbitrary (random) TCP/UDP checksum fields, 1/8 of UDP 0 = none */
 } gen_params;
 
 typedef struct {
@@ -41,7 +42,7 @@ typedef struct {
 } gen_tables;
 
 enum { S_FLOW = 1, S_FAM, S_INACL, S_RULE, S_SRC, S_DST, S_DST2, S_SP, S_DP, S_ROUTE, S_PROTO, S_LEN,
-       S_PAY, S_MATCH, S_PAT, S_POFF, S_TTL, S_BAD, S_BADK, S_SRC2 };
+       S_PAY, S_MATCH, S_PAT, S_POFF, S_TTL, S_BAD, S_BADK, S_SRC2, S_CSUM };
 
 static inline uint64_t mix64(uint64_t z)
 {
@@ -111,6 +112,20 @@ static void make_flow(const gen_params *p, const gen_tables *t, uint64_t f, flow
         fl->dp = (uint16_t)R(S_DP, f);
         fl->proto = (R(S_PROTO, f) % 100) < p->tcp_pct ? 6 : 17;
     }
+}
+
+/* The 5-tuple of flow f (table generators use it to draw entries real flows hit). */
+void nfcgen_flow(const gen_params *p, const gen_tables *t, uint64_t f, uint32_t *fam, uint8_t *src, uint8_t *dst,
+                 uint16_t *sp, uint16_t *dp, uint8_t *proto)
+{
+    flow_t fl;
+    make_flow(p, t, f, &fl);
+    *fam = (uint32_t)fl.fam;
+    memcpy(src, fl.src, 16);
+    memcpy(dst, fl.dst, 16);
+    *sp = fl.sp;
+    *dp = fl.dp;
+    *proto = fl.proto;
 }
 
 static uint32_t frame_len(const gen_params *p, uint64_t i, int fam, uint8_t proto)
@@ -183,16 +198,19 @@ void nfcgen_fill(const gen_params *p, const gen_tables *t, uint64_t first, uint3
             l4 = 54;
         }
         uint32_t pl = l4;
+        /* checksum fields: 0, or (l4csum) an arbitrary value -- never computed here */
+        const uint64_t rc = R(S_CSUM, i);
+        const uint32_t ck = p->l4csum ? (uint32_t)(rc & 0xffff) : 0;
         if (fl.proto == 17) {
             put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
-            put16(f + l4 + 4, L - l4); put16(f + l4 + 6, 0);
+            put16(f + l4 + 4, L - l4); put16(f + l4 + 6, ((rc >> 16) & 7) == 0 ? 0 : ck);
             pl = l4 + 8;
         } else if (fl.proto == 6) {
             put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
             uint64_t r = R(S_SP, i);
             for (int b = 0; b < 8; b++) f[l4 + 4 + b] = (uint8_t)(r >> (8 * b));
             f[l4 + 12] = 0x50; f[l4 + 13] = 0x18;
-            put16(f + l4 + 14, 0xffff); put16(f + l4 + 16, 0); put16(f + l4 + 18, 0);
+            put16(f + l4 + 14, 0xffff); put16(f + l4 + 16, ck); put16(f + l4 + 18, 0);
             pl = l4 + 20;
         }
         /* payload */

@@ -39,7 +39,12 @@ class OrSpec(ctypes.Structure):
                 ("r6", _P), ("n_r6", ctypes.c_uint32), ("nh6", _P), ("n_nh6", ctypes.c_uint32),
                 ("pmac6", _P), ("n_port6", ctypes.c_uint32),
                 ("sa", _P), ("n_sa", ctypes.c_uint32),
-                ("lb_port", _P), ("n_lb", ctypes.c_uint32), ("lb_key", _P)]
+                ("lb_port", _P), ("n_lb", ctypes.c_uint32), ("lb_key", _P),
+                ("nat_inside", _P), ("n_nat_inside", ctypes.c_uint32),
+                ("nat_pool", _P), ("n_nat_pool", ctypes.c_uint32),
+                ("nat_port_lo", ctypes.c_uint32), ("nat_port_hi", ctypes.c_uint32),
+                ("nat_dnat", _P), ("n_nat_dnat", ctypes.c_uint32),
+                ("nat_ext_ports", ctypes.c_uint32), ("nat_key", _P)]
 
 
 _lib = None
@@ -69,6 +74,8 @@ def lib():
         L.or_toeplitz.argtypes = [_P, _P, ctypes.c_size_t]
         L.or_ipv4_checksum.restype = ctypes.c_uint16
         L.or_ipv4_checksum.argtypes = [_P, ctypes.c_size_t]
+        L.or_csum_update.restype = ctypes.c_uint16
+        L.or_csum_update.argtypes = [ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint16]
         L.or_ac_match.restype = ctypes.c_uint32
         L.or_ac_match.argtypes = [_P, _P, ctypes.c_size_t, _P, ctypes.c_uint32]
         L.or_lpm4.restype = ctypes.c_int32
@@ -118,6 +125,11 @@ def ipv4_checksum(hdr: bytes) -> int:
     return int(lib().or_ipv4_checksum(_buf(hdr), len(hdr)))
 
 
+def csum_update(hc: int, m: int, m1: int) -> int:
+    """RFC 1624 eqn. 3 incremental checksum update (one 16-bit field m -> m1)."""
+    return int(lib().or_csum_update(hc, m, m1))
+
+
 MS_RSS_KEY = bytes.fromhex("6d5a56da255b0ec24167253d43a38fb0d0ca2bcbae7b30b477cb2da38030f20c"
                            "6a42b73bbeac01fa")
 
@@ -160,6 +172,12 @@ class OracleChain:
             s.sa, s.n_sa = P(t.sas), len(t.sas)
         if "LB" in ks and t.lb_ports is not None:
             s.lb_port, s.n_lb, s.lb_key = P(t.lb_ports), len(t.lb_ports), P(t.lb_key)
+        if "NAT" in ks and t.nat_pool is not None:
+            s.nat_inside, s.n_nat_inside = P(t.nat_inside), len(t.nat_inside)
+            s.nat_pool, s.n_nat_pool = P(t.nat_pool), len(t.nat_pool)
+            s.nat_port_lo, s.nat_port_hi = t.nat_port_lo, t.nat_port_hi
+            s.nat_dnat, s.n_nat_dnat = P(t.nat_dnat), len(t.nat_dnat)
+            s.nat_ext_ports, s.nat_key = t.nat_ext_ports, P(t.nat_key)
         self.spec = s
         self.kinds = list(kinds)
         self.tables = t

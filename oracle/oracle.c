@@ -587,6 +587,87 @@ static void forward_rewrite(uint8_t *f, const pview *v, const or_nexthop *nh, co
     }
 }
 
+/* RFC 1624 eqn. 3: HC' = ~(~HC + ~m + m'), one's complement 16-bit sums. */
+static uint32_t oc_add16(uint32_t a, uint32_t b)
+{
+    uint32_t x = a + b;
+    return (x & 0xFFFF) + (x >> 16);
+}
+uint16_t or_csum_update(uint16_t hc, uint16_t m, uint16_t m1)
+{
+    uint32_t x = oc_add16(oc_add16((uint16_t)~hc, (uint16_t)~m), m1);
+    return (uint16_t)~x;
+}
+
+/* NAT44 ("For traffics to Internet, the NAT network function performs
+ * source and destination NAT"; Table II row NAT: header read + write, no drop;
+ * reading R#30).  Applies to IPv4 TCP/UDP packets (L4 header parsed) whose
+ * egress port, as set by the NFs before it, is marked as Internet-facing.
+ *   h    = Toeplitz(nat_key, src | dst | sport | dport) of the packet as it arrives;
+ *   DNAT : the first entry with (proto, ext_addr, ext_port) == (proto, dst, dport)
+ *          rewrites dst, dport to (int_addr, int_port);
+ *   SNAT : if src lies in one of the inside prefixes (first match), src := pool[(h
+ *          & 0xFFFF) mod n_pool], sport := port_lo + ((h >> 16) mod (port_hi -
+ *          port_lo + 1))  (deterministic NAPT: a pure function of the flow);
+ *   the IPv4 header checksum is recomputed (RFC 1071), the TCP / UDP checksum is
+ *   updated per changed 16-bit word by RFC 1624 eqn. 3 (pseudo-header addresses
+ *   and ports); a UDP checksum of 0 ("none", RFC 768) stays 0, and an updated
+ *   UDP checksum of 0 is sent as 0xFFFF.
+ * Returns 1 if the NAT applied, 0 for pass-through. */
+static uint32_t be32p(const uint8_t *p) { return (uint32_t)p[0] << 24 | (uint32_t)p[1] << 16 | (uint32_t)p[2] << 8 | p[3]; }
+static void put32p(uint8_t *p, uint32_t v) { p[0] = (uint8_t)(v >> 24); p[1] = (uint8_t)(v >> 16); p[2] = (uint8_t)(v >> 8); p[3] = (uint8_t)v; }
+static int nat_apply(const or_spec *s, uint8_t *f, pview *v, uint32_t port)
+{
+    if (v->family != 4 || (v->proto != 6 && v->proto != 17) || v->pl_off == v->l4_off) return 0;
+    if (port >= 32 || !((s->nat_ext_ports >> port) & 1)) return 0;
+    uint8_t t[12];
+    tuple_bytes(v, t);
+    const uint32_t h = or_toeplitz(s->nat_key, t, 12);
+    const uint32_t src = be32p(v->src), dst = be32p(v->dst);
+    uint32_t nsrc = src, ndst = dst;
+    uint16_t nsp = v->sport, ndp = v->dport;
+    for (uint32_t k = 0; k < s->n_nat_dnat; k++) {
+        const or_nat_dnat *e = &s->nat_dnat[k];
+        if (e->proto == v->proto && e->ext_addr == dst && e->ext_port == v->dport) {
+            ndst = e->int_addr;
+            ndp = e->int_port;
+            break;
+        }
+    }
+    for (uint32_t k = 0; k < s->n_nat_inside; k++) {
+        const or_nat_prefix *q = &s->nat_inside[k];
+        const uint32_t m = q->len == 0 ? 0u : 0xFFFFFFFFu << (32 - q->len);
+        if ((src & m) == (q->prefix & m)) {
+            nsrc = s->nat_pool[(h & 0xFFFF) % s->n_nat_pool];
+            nsp = (uint16_t)(s->nat_port_lo + (h >> 16) % (s->nat_port_hi - s->nat_port_lo + 1));
+            break;
+        }
+    }
+    const int l4 = v->l4_off, ck_at = v->proto == 6 ? l4 + 16 : l4 + 6;
+    uint16_t ck = be16(f + ck_at);
+    if (!(v->proto == 17 && ck == 0)) {
+        const uint16_t m[6] = {(uint16_t)(src >> 16), (uint16_t)src, (uint16_t)(dst >> 16), (uint16_t)dst, v->sport, v->dport};
+        const uint16_t m1[6] = {(uint16_t)(nsrc >> 16), (uint16_t)nsrc, (uint16_t)(ndst >> 16), (uint16_t)ndst, nsp, ndp};
+        for (int k = 0; k < 6; k++)
+            if (m[k] != m1[k]) ck = or_csum_update(ck, m[k], m1[k]);
+        if (v->proto == 17 && ck == 0) ck = 0xFFFF;
+        f[ck_at] = (uint8_t)(ck >> 8);
+        f[ck_at + 1] = (uint8_t)ck;
+    }
+    put32p(f + 26, nsrc);
+    put32p(f + 30, ndst);
+    f[l4] = (uint8_t)(nsp >> 8); f[l4 + 1] = (uint8_t)nsp;
+    f[l4 + 2] = (uint8_t)(ndp >> 8); f[l4 + 3] = (uint8_t)ndp;
+    f[24] = f[25] = 0;
+    const uint16_t ipck = or_ipv4_checksum(f + 14, (size_t)(l4 - 14));
+    f[24] = (uint8_t)(ipck >> 8); f[25] = (uint8_t)ipck;
+    put32p(v->src, nsrc);
+    put32p(v->dst, ndst);
+    v->sport = nsp;
+    v->dport = ndp;
+    return 1;
+}
+
 uint64_t oracle_run(or_chain *c, uint8_t *arena, const uint64_t *off, const uint16_t *len, uint32_t n,
                     uint64_t first_global, or_result *res, uint32_t *match_pkt, uint16_t *match_pat,
                     uint64_t match_cap, uint64_t *stats, const uint32_t *seq_override)
@@ -684,6 +765,9 @@ uint64_t oracle_run(or_chain *c, uint8_t *arena, const uint64_t *off, const uint
                 lb_hits[b]++;
                 break;
             }
+            case OR_NAT:
+                pass = !nat_apply(s, f, &v, r.port);
+                break;
             default:
                 break;
             }
@@ -785,8 +869,9 @@ uint64_t oracle_run_reorg(or_chain *c, const uint8_t *group, uint8_t *arena, con
     for (uint32_t p = 1; p < s->n_nf; p++)
         if (group[p] != group[p - 1] && group[p] != group[p - 1] + 1) return UINT64_MAX;
     for (uint32_t p = 0; p < s->n_nf; p++)
-        if (s->kind[p] == OR_IPSEC && ((p > 0 && group[p - 1] == group[p]) || (p + 1 < s->n_nf && group[p + 1] == group[p])))
-            return UINT64_MAX;
+        if ((s->kind[p] == OR_IPSEC || s->kind[p] == OR_NAT) &&
+            ((p > 0 && group[p - 1] == group[p]) || (p + 1 < s->n_nf && group[p + 1] == group[p])))
+            return UINT64_MAX;   /* IPSEC and NAT stand alone (R#29, R#30) */
     uint64_t n_pairs = 0;
     uint64_t *acl_hits = stats + OR_ST_VAR_BASE;
     uint64_t *lb_hits = acl_hits + s->n_acl + 1;
@@ -810,6 +895,14 @@ uint64_t oracle_run_reorg(or_chain *c, const uint8_t *group, uint8_t *arena, con
         while (!dropped && p0 < s->n_nf) {
             uint32_t p1 = p0;
             while (p1 + 1 < s->n_nf && group[p1 + 1] == group[p0]) p1++;
+            if (s->kind[p0] == OR_NAT) {               /* singleton: applied to the packet itself */
+                uint64_t *ps = stats + OR_ST_POS_BASE + 4 * p0;
+                ps[0]++;
+                if (nat_apply(s, f, &v, r.port)) ps[3]++;
+                else ps[2]++;
+                p0 = p1 + 1;
+                continue;
+            }
             if (s->kind[p0] == OR_IPSEC) {             /* singleton: applied to the packet itself */
                 uint64_t *ps = stats + OR_ST_POS_BASE + 4 * p0;
                 ps[0]++;

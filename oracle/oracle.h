@@ -24,7 +24,7 @@ extern "C" {
 #endif
 
 /* NF kinds, in the numbering of the logical chain spec. */
-enum { OR_ACL = 1, OR_DPI = 2, OR_LPM4 = 3, OR_LPM6 = 4, OR_IPSEC = 5, OR_LB = 6 };
+enum { OR_ACL = 1, OR_DPI = 2, OR_LPM4 = 3, OR_LPM6 = 4, OR_IPSEC = 5, OR_LB = 6, OR_NAT = 7 };
 
 /* 48 B ACL rule (P:L219 firewall; P:L383 ClassBench-style 5-tuple rules). */
 typedef struct {
@@ -48,6 +48,14 @@ typedef struct {                                                                
     uint8_t auth_key[20];
 } or_sa;
 
+/* NAT44 tables ("the NAT network function performs source and destination
+ * NAT"; Table II row NAT: reads and writes the header, never drops; R#30). */
+typedef struct { uint32_t prefix; uint8_t len; uint8_t pad[3]; } or_nat_prefix;          /* 8 B  */
+typedef struct {                                                                          /* 16 B */
+    uint32_t ext_addr; uint16_t ext_port; uint8_t proto; uint8_t pad;
+    uint32_t int_addr; uint16_t int_port; uint16_t pad2;
+} or_nat_dnat;
+
 typedef struct {
     uint32_t n_nf;
     uint8_t kind[8];           /* kind[p] for chain position p (original SFC order) */
@@ -65,6 +73,13 @@ typedef struct {
     const or_sa *sa; uint32_t n_sa;
     /* LB */
     const uint16_t *lb_port; uint32_t n_lb; const uint8_t *lb_key; /* 40 B Toeplitz key */
+    /* NAT (R#30): addresses are host-order u32 values */
+    const or_nat_prefix *nat_inside; uint32_t n_nat_inside;
+    const uint32_t *nat_pool; uint32_t n_nat_pool;
+    uint32_t nat_port_lo, nat_port_hi;
+    const or_nat_dnat *nat_dnat; uint32_t n_nat_dnat;
+    uint32_t nat_ext_ports;    /* bit p: egress port p faces the Internet */
+    const uint8_t *nat_key;    /* 40 B Toeplitz key of the translation hash */
 } or_spec;
 
 /* 16 B per-packet record (identical layout on both sides). */
@@ -134,6 +149,8 @@ void or_sha1(const uint8_t *msg, size_t n, uint8_t out[20]);
 void or_hmac_sha1(const uint8_t *key, size_t klen, const uint8_t *msg, size_t n, uint8_t out[20]);
 uint32_t or_toeplitz(const uint8_t key[40], const uint8_t *in, size_t n);
 uint16_t or_ipv4_checksum(const uint8_t *hdr, size_t hlen);
+/* RFC 1624 eqn. 3: checksum after one 16-bit field changes from m to m1 */
+uint16_t or_csum_update(uint16_t hc, uint16_t m, uint16_t m1);
 /* DPI: distinct pattern set of one byte string; returns |M|, writes sorted IDs into ids (cap). */
 uint32_t or_ac_match(or_chain *c, const uint8_t *buf, size_t n, uint32_t *ids, uint32_t cap);
 /* LPM: next hop index or -1 */
