@@ -42,6 +42,7 @@ def parse_args():
     ap.add_argument("--config", default="C1")
     ap.add_argument("--pkt-len", type=int, default=None, help="frame length (0 = IMIX)")
     ap.add_argument("--k", type=int, default=None, help="C5 chain length")
+    ap.add_argument("--acl-rules", type=int, default=None, help="N3 (NEXT-3) ACL size: 200 / 1000 / 10000")
     ap.add_argument("--ring-mb", type=int, default=1024, help="HBM ring size per GPU (>> 126 MB L2)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
     ap.add_argument("--no-e2e", action="store_true")
@@ -54,7 +55,7 @@ def parse_args():
 # ------------------------------------------------------------------ workload
 def make_workload(args):
     import nfcgen
-    w = nfcgen.workload(args.config, pkt_len=args.pkt_len, k=args.k)
+    w = nfcgen.workload(args.config, pkt_len=args.pkt_len, k=args.k, acl_rules=getattr(args, "acl_rules", None))
     w.traffic.ttl = 255  # steps re-process the same ring: keep TTL/hop limit from expiring
     return w
 
@@ -92,8 +93,12 @@ def alg_bytes_per_step(kinds, lens, fam, rec):
             rewritten |= passed(p) & (fam == 4)
         if k == "LPM6":
             rewritten |= passed(p) & (fam == 6)
+        if k == "NAT":      # address/port/checksum sector [32, 64) of IPv4 packets past the NAT
+            natw = passed(p) & (fam == 4)
     rd = 10 * n + int(np.where(payload, lens, np.minimum(lens, 64)).sum())
     wr = 16 * n + 32 * int(rewritten.sum())
+    if "NAT" in kinds:
+        wr += 32 * int(natw.sum())
     esp = rec["esp_sa"] != 0xFF
     wr += int(rec["out_len"][esp].astype(np.int64).sum())
     wr += 6 * int(rec["dpi_nmatch"].astype(np.int64).sum())
@@ -446,7 +451,7 @@ def main():
     # each on its own packet copy, XOR-merged -- on the same ring, and the
     # latency of ONE batch (the paper's Fig. 14 metric) for fused / parallel / unfused
     parallel = None
-    if not args.no_unfused and not args.unfused and "IPSEC" not in w.kinds:
+    if not args.no_unfused and not args.unfused and "IPSEC" not in w.kinds and "NAT" not in w.kinds:
         pch = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_PARALLEL)
         pch.load_tables(w.tables)
 

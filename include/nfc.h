@@ -58,6 +58,7 @@ extern "C" {
 #define NFC_LPM6 4  /* IPv6 forwarder, longest-prefix match (Waldvogel levels)    */
 #define NFC_IPSEC 5 /* IPsec ESP gateway: AES-128-CTR + HMAC-SHA1-96              */
 #define NFC_LB 6    /* load balancer: flow hash -> backend -> egress port         */
+#define NFC_NAT 7   /* NAT44: source NAPT + static destination NAT (R#30)  */
 
 #define NFC_MAX_CHAIN 6
 
@@ -155,6 +156,31 @@ typedef struct {
     const uint16_t *backend_port;/* host; egress port per backend                  */
     const uint8_t *key;          /* host; 40 B Toeplitz key                        */
 } nfc_lb_spec;
+
+/* NAT44 ("For traffics to Internet, the NAT network
+ * function performs source and destination NAT"; Table II: header read+write, no
+ * drop; R#30).  Applies to IPv4 TCP/UDP packets whose egress port (set by
+ * the NFs before it; 0 if none) has its bit set in ext_ports.  With h =
+ * Toeplitz(key, src|dst|sport|dport) of the arriving packet: DNAT rewrites (dst,
+ * dport) of the first entry matching (proto, dst, dport); SNAT, for sources inside
+ * one of the prefixes, sets src = pool[(h & 0xFFFF) % n_pool] and sport = port_lo +
+ * (h >> 16) % (port_hi - port_lo + 1).  The IPv4 header checksum is recomputed and the
+ * TCP/UDP checksum updated per RFC 1624 eqn. 3 (a UDP checksum of 0 stays 0; an
+ * updated UDP checksum of 0 becomes 0xFFFF).  Addresses are host-order u32 values. */
+typedef struct { uint32_t prefix; uint8_t len; uint8_t pad[3]; } nfc_nat_prefix;        /* 8 B  */
+typedef struct {                                                                         /* 16 B */
+    uint32_t ext_addr; uint16_t ext_port; uint8_t proto; uint8_t pad;
+    uint32_t int_addr; uint16_t int_port; uint16_t pad2;
+} nfc_nat_dnat;
+
+typedef struct {
+    uint32_t n_inside;  const nfc_nat_prefix *inside; /* host; <= 64 prefixes (SNAT sources)     */
+    uint32_t n_pool;    const uint32_t *pool;         /* host; 1..65536 public addresses          */
+    uint32_t port_lo, port_hi;                        /* SNAT source port range, lo <= hi < 65536 */
+    uint32_t n_dnat;    const nfc_nat_dnat *dnat;     /* host; distinct (proto, ext_addr, ext_port) */
+    uint32_t ext_ports;                               /* bit p: egress port p faces the Internet   */
+    const uint8_t *key;                               /* host; 40 B Toeplitz key                   */
+} nfc_nat_spec;
 
 /* Build the device image of one NF's tables on the host and copy it to the
  * device (synchronous).  spec points to the nfc_*_spec matching kind;

@@ -339,7 +339,9 @@ std::string build_dpi(const nfc_dpi_spec &s, DpiHost &o)
         const uint32_t o0 = o.out_off[k], nm = o.out_off[k + 1] - o0;
         uint32_t drop = 0;
         for (uint32_t x = o0; x < o0 + nm; x++) drop |= o.action[o.out_ids[x]];
-        o.out_meta[k] = (o0 < (1u << 20) && nm < 2047u) ? (o0 | nm << 20 | drop << 31) : DPI_META_NONE;
+        // a one-pattern closure carries the pattern id itself (no CSR read when emitting)
+        const uint32_t lo = nm == 1 ? o.out_ids[o0] : o0;
+        o.out_meta[k] = (lo < (1u << 20) && nm < 2047u) ? (lo | nm << 20 | drop << 31) : DPI_META_NONE;
     }
     // slot image (DpiImg::frows): non-accepting states 0.., accepting -1.. (BFS order);
     // physical row of slot x = n_acc + x
@@ -650,6 +652,46 @@ void build_toeplitz_nibbles(const uint8_t key[40], std::vector<uint32_t> &nib)
                 if ((v >> (3 - j)) & 1) h ^= window(4 * k + j);
             nib[k * 16 + v] = h;
         }
+}
+
+// ---------------------------------------------------------------- NAT44 (R#30)
+std::string build_nat(const nfc_nat_spec &s, NatHost &o)
+{
+    if (s.n_inside > NAT_MAX_INSIDE || (s.n_inside && !s.inside)) return "nat: n_inside must be <= 64 (with prefixes)";
+    if (s.n_pool == 0 || s.n_pool > 65536 || !s.pool) return "nat: n_pool must be 1..65536";
+    if (s.port_lo > s.port_hi || s.port_hi > 65535) return "nat: port range must satisfy lo <= hi <= 65535";
+    if (s.n_dnat && !s.dnat) return "nat: dnat == NULL";
+    if (!s.key) return "nat: key == NULL";
+    o.img = NatImg{};
+    o.img.n_inside = s.n_inside;
+    for (uint32_t k = 0; k < s.n_inside; k++) {
+        if (s.inside[k].len > 32) return "nat: inside prefix length > 32";
+        const uint32_t m = s.inside[k].len ? 0xFFFFFFFFu << (32 - s.inside[k].len) : 0u;
+        o.img.in_mask[k] = m;
+        o.img.in_pref[k] = s.inside[k].prefix & m;
+    }
+    o.pool.assign(s.pool, s.pool + s.n_pool);
+    o.img.n_pool = s.n_pool;
+    o.img.port_lo = s.port_lo;
+    o.img.port_range = s.port_hi - s.port_lo + 1;
+    o.img.ext_ports = s.ext_ports;
+    uint32_t cap = 16;
+    while (cap < 2 * s.n_dnat) cap <<= 1;
+    o.dnat.assign(cap, make_uint4(0, 0, 0, 0));
+    for (uint32_t k = 0; k < s.n_dnat; k++) {
+        const nfc_nat_dnat &e = s.dnat[k];
+        if (e.proto != 6 && e.proto != 17) return "nat: dnat proto must be 6 or 17";
+        const uint32_t key1 = (uint32_t)e.ext_port | (uint32_t)e.proto << 16;
+        uint32_t h = nat_slot(e.ext_addr, key1) & (cap - 1);
+        while (o.dnat[h].y & NAT_VALID) {
+            if (o.dnat[h].x == e.ext_addr && (o.dnat[h].y & 0xFFFFFF) == key1) return "nat: duplicate dnat entry";
+            h = (h + 1) & (cap - 1);
+        }
+        o.dnat[h] = make_uint4(e.ext_addr, key1 | NAT_VALID, e.int_addr, e.int_port);
+    }
+    o.img.dnat_mask = cap - 1;
+    build_toeplitz_nibbles(s.key, o.nib);
+    return "";
 }
 
 } // namespace nfc

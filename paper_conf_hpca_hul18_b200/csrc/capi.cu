@@ -79,6 +79,8 @@ struct nfc_chain {
     uint32_t seq_parity = 0;
     DBuf lb_port, lb_nib;
     LbImg lb{};
+    NatImg nat{};
+    DBuf nat_pool, nat_dnat, nat_nib;
     // stats
     DBuf stats;
     uint32_t stats_len = ST_VAR_BASE;
@@ -118,7 +120,7 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
     if (n < 1 || n > NFC_MAX_CHAIN) return fail(NFC_EUNSUP, "chain length must be 1..6");
     uint32_t mask = 0;
     for (uint32_t i = 0; i < n; i++) {
-        if (kinds[i] < NFC_ACL || kinds[i] > NFC_LB) return fail(NFC_EINVAL, "unknown NF kind");
+        if (kinds[i] < NFC_ACL || kinds[i] > NFC_NAT) return fail(NFC_EINVAL, "unknown NF kind");
         if (mask & (1u << kinds[i])) return fail(NFC_EUNSUP, "repeated NF kind in chain");
         mask |= 1u << kinds[i];
     }
@@ -126,7 +128,8 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
     if (flags & ~(NFC_F_UNFUSED | NFC_F_PARALLEL)) return fail(NFC_EINVAL, "opts->flags: unknown bits");
     if ((flags & NFC_F_UNFUSED) && (flags & NFC_F_PARALLEL)) return fail(NFC_EINVAL, "opts->flags: UNFUSED and PARALLEL are exclusive");
     if ((flags & NFC_F_UNFUSED) && (mask & (1u << NFC_IPSEC))) return fail(NFC_EUNSUP, "NFC_F_UNFUSED: IPsec chains are not offered");
-    if ((flags & NFC_F_PARALLEL) && (mask & (1u << NFC_IPSEC))) return fail(NFC_EUNSUP, "NFC_F_PARALLEL: IPsec chains are not offered");
+    if ((flags & NFC_F_PARALLEL) && (mask & ((1u << NFC_IPSEC) | (1u << NFC_NAT))))
+        return fail(NFC_EUNSUP, "NFC_F_PARALLEL: IPsec and NAT chains are not offered");
     nfc_chain *c = new (std::nothrow) nfc_chain();
     if (!c) return fail(NFC_ENOMEM, "out of host memory");
     c->device = opts ? opts->device : 0;
@@ -160,7 +163,8 @@ void nfc_destroy_chain(nfc_chain *c)
     DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
                    &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->dpi_frows, &c->dpi_accid, &c->dpi_accmeta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
-                   &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->stats, &c->counter,
+                   &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->nat_pool, &c->nat_dnat, &c->nat_nib,
+                   &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
                    &c->h_mp, &c->h_mq, &c->h_mc};
     for (DBuf *b : all) b->release();
@@ -179,7 +183,7 @@ int nfc_chain_room(const nfc_chain *c, uint32_t *headroom, uint32_t *tailroom)
 int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_bytes)
 {
     if (!c || !spec) return fail(NFC_EINVAL, "NULL argument");
-    if (kind < NFC_ACL || kind > NFC_LB) return fail(NFC_EINVAL, "unknown NF kind");
+    if (kind < NFC_ACL || kind > NFC_NAT) return fail(NFC_EINVAL, "unknown NF kind");
     int rc = set_device(c);
     if (rc) return rc;
     cudaDeviceSynchronize();   // tables are replaced atomically w.r.t. later launches
@@ -300,6 +304,20 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
         c->n_lb = s.n_backends;
         break;
     }
+    case NFC_NAT: {
+        if (spec_bytes != sizeof(nfc_nat_spec)) return fail(NFC_EINVAL, "spec_bytes != sizeof(nfc_nat_spec)");
+        NatHost h;
+        err = build_nat(*static_cast<const nfc_nat_spec *>(spec), h);
+        if (!err.empty()) return fail(NFC_EINVAL, err);
+        CK(c->nat_pool.upload(h.pool));
+        CK(c->nat_dnat.upload(h.dnat));
+        CK(c->nat_nib.upload(h.nib));
+        c->nat = h.img;
+        c->nat.pool = c->nat_pool.as<uint32_t>();
+        c->nat.dnat = c->nat_dnat.as<uint4>();
+        c->nat.nib = c->nat_nib.as<uint32_t>();
+        break;
+    }
     }
     c->loaded[kind] = true;
     return realloc_stats(c);
@@ -358,6 +376,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     p.l6 = c->l6;
     p.esp = c->esp;
     p.lb = c->lb;
+    p.nat = c->nat;
     if (c->mask & MASK_IPSEC) {
         if (n_tiles > c->tile_cap) {
             uint32_t cap = n_tiles + n_tiles / 4 + 64;

@@ -48,7 +48,7 @@ struct DpiImg {
     uint32_t bitmap_words;       // words per thread
     uint32_t hot_states;         // states whose full 256-byte rows are staged in shared memory
     uint32_t row2, hk2;          // per launch: bytes per DFA row (2 ncls); byte offset of the last hot entry
-    const uint32_t *out_meta;    // per state: out_off | n_out << 20 | any DROP pattern << 31
+    const uint32_t *out_meta;    // per state: out_off (the pattern id if n_out == 1) | n_out << 20 | any DROP << 31
                                  // (DPI_META_NONE if the closure does not fit the fields)
     uint32_t meta_smem;          // 1: out_meta staged in shared memory
     // Tiered placement (DM_HOT): rows of states [0, hot_states) are dense in shared
@@ -127,11 +127,35 @@ struct LbImg {
     const uint32_t *nib;         // Toeplitz nibble table of the LB key (72 x 16)
 };
 
+// ---------------------------------------------------------------- NAT44 (R#30)
+// Inside prefixes in the constant bank (uniform loop); DNAT entries in an
+// open-addressing table: {ext_addr, ext_port | proto << 16 | NAT_VALID, int_addr,
+// int_port}, slot = nat_slot(ext_addr, ext_port | proto << 16) & mask, linear probing.
+static const uint32_t NAT_MAX_INSIDE = 64, NAT_VALID = 0x80000000u;
+__host__ __device__ inline uint32_t nat_slot(uint32_t a, uint32_t b)
+{
+    uint32_t x = a * 0x9E3779B1u ^ (b + 0x7F4A7C15u) * 0x85EBCA77u;
+    x ^= x >> 15;
+    x *= 0x2C1B3C6Du;
+    return x ^ (x >> 13);
+}
+struct NatImg {
+    uint32_t n_inside;
+    uint32_t in_pref[NAT_MAX_INSIDE], in_mask[NAT_MAX_INSIDE];
+    const uint32_t *pool;
+    uint32_t n_pool, port_lo, port_range;
+    const uint4 *dnat;
+    uint32_t dnat_mask;
+    uint32_t ext_ports;
+    const uint32_t *nib;         // Toeplitz nibble table of the NAT key (72 x 16)
+};
+
 // ---------------------------------------------------------------- launch
 struct BatchDev { uint8_t *arena; const uint64_t *off; const uint16_t *len; uint32_t n; uint32_t start; uint64_t first; };
 
 enum { MASK_ACL = 1u << NFC_ACL, MASK_DPI = 1u << NFC_DPI, MASK_LPM4 = 1u << NFC_LPM4,
-       MASK_LPM6 = 1u << NFC_LPM6, MASK_IPSEC = 1u << NFC_IPSEC, MASK_LB = 1u << NFC_LB };
+       MASK_LPM6 = 1u << NFC_LPM6, MASK_IPSEC = 1u << NFC_IPSEC, MASK_LB = 1u << NFC_LB,
+       MASK_NAT = 1u << NFC_NAT };
 
 // stats vector layout
 enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, ST_DPI_PAIRS,
@@ -142,7 +166,8 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
 // launch, read by the kernel from the constant bank)
 struct SmemLayout {
     uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, par, total;
-    uint32_t frow0;               // DM_FULL: row of slot 0 (DpiImg::frows)
+    uint32_t frow0;
+    uint32_t nat_nib;             // NAT Toeplitz nibbles               // DM_FULL: row of slot 0 (DpiImg::frows)
 };
 
 struct KParams {
@@ -182,6 +207,7 @@ struct KParams {
     Lpm6Img l6;
     EspImg esp;
     LbImg lb;
+    NatImg nat;
 };
 
 // host-side builders (builders.cpp); return "" on success or an error message
@@ -218,6 +244,13 @@ std::string build_lpm6(const nfc_lpm6_spec &s, Lpm6Host &out);
 std::string build_ipsec(const nfc_ipsec_spec &s, std::vector<EspSa> &sa);
 void build_aes_tables(std::vector<uint32_t> &te);           // Te0..3 + sbox
 void build_toeplitz_nibbles(const uint8_t key[40], std::vector<uint32_t> &nib);
+struct NatHost {
+    NatImg img{};                    // scalars + inside prefixes (pointers set by the caller)
+    std::vector<uint32_t> pool;
+    std::vector<uint4> dnat;         // power-of-two open-addressing table
+    std::vector<uint32_t> nib;
+};
+std::string build_nat(const nfc_nat_spec &s, NatHost &out);
 extern const uint8_t MS_RSS_KEY[40];
 void aes_expand(const uint8_t key[16], uint32_t rk[44]);
 void sha1_compress(uint32_t h[5], const uint8_t blk[64]);

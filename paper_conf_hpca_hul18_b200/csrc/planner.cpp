@@ -37,6 +37,8 @@ RW rw_of(uint32_t kind, int fam)
         return fam == 6 ? RW{F_DST | F_TTL, F_ETH_DST | F_ETH_SRC | F_TTL} : RW{0, 0};
     case NFC_IPSEC: return {F_ALL, F_ALL};                                 // encrypts, adds bytes
     case NFC_LB: return {F_SRC | F_DST | F_PORTS | F_PROTO, 0};            // flow hash
+    case NFC_NAT:                                                          // P:L383, Table II: NAT44 (R#30)
+        return fam == 4 ? RW{F_SRC | F_DST | F_PORTS | F_PROTO, F_SRC | F_DST | F_PORTS | F_CSUM} : RW{0, 0};
     }
     return {F_ALL, F_ALL};
 }
@@ -44,7 +46,9 @@ RW rw_of(uint32_t kind, int fam)
 // earlier NF a, later NF b: legal in one group (no RAW, no WAW on any family)
 bool legal_pair(uint32_t a, uint32_t b)
 {
-    if (a == NFC_IPSEC || b == NFC_IPSEC) return false;
+    // IPsec rewrites everything; NAT decides on the egress port an earlier forwarder set
+    // (a read of merge-resolved metadata) and rewrites the 5-tuple: both stand alone (R#30)
+    if (a == NFC_IPSEC || b == NFC_IPSEC || a == NFC_NAT || b == NFC_NAT) return false;
     for (int fam : {4, 6}) {
         const RW x = rw_of(a, fam), y = rw_of(b, fam);
         if (x.w & y.r) return false;     // read after write
@@ -58,7 +62,7 @@ extern "C" NFC_API int nfc_plan_parallel(const uint32_t *kinds, uint32_t n, uint
 {
     if (!kinds || !group || n == 0 || n > NFC_MAX_CHAIN) return NFC_EINVAL;
     for (uint32_t p = 0; p < n; p++)
-        if (kinds[p] < NFC_ACL || kinds[p] > NFC_LB) return NFC_EINVAL;
+        if (kinds[p] < NFC_ACL || kinds[p] > NFC_NAT) return NFC_EINVAL;
     // greedy: extend the current group while the next NF is legal with every member
     uint32_t g = 0, start = 0;
     group[0] = 0;

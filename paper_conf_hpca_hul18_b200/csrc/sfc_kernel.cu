@@ -17,6 +17,7 @@ NFC_DECLARE_LAUNCH(SIG_K1, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_C4, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_K5, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_K6, DM_HOT)
+NFC_DECLARE_LAUNCH(SIG_N3, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_ANY, DM_HOT)
 
 // chains with a DM_FULL instantiation (no IPsec: the DFA takes the whole CTA's shared memory)
@@ -24,7 +25,7 @@ static bool has_full(uint32_t sig) { return sig == SIG_C1 || sig == SIG_K2 || si
 static bool known(uint32_t sig)
 {
     return has_full(sig) || sig == SIG_C2 || sig == SIG_C3 || sig == SIG_K1 || sig == SIG_C4 || sig == SIG_K5 ||
-           sig == SIG_K6;
+           sig == SIG_K6 || sig == SIG_N3;
 }
 
 Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full)
@@ -73,6 +74,7 @@ static int dispatch(const Variant &v, const KParams &p, int dev, void *stream, s
     NFC_CASE(SIG_C4)
     NFC_CASE(SIG_K5)
     NFC_CASE(SIG_K6)
+    NFC_CASE(SIG_N3)
 #undef NFC_CASE
     return launch_t<SIG_ANY, DM_HOT>(p, dev, stream, err, cfg, q);
 }

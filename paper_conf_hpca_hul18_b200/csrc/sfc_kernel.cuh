@@ -41,7 +41,7 @@ __host__ __device__ constexpr uint32_t sig_kind(uint32_t s, int p) { return (s >
 __host__ __device__ constexpr uint32_t sig_mask(uint32_t s)
 {
     if (s == SIG_ANY) return (1u << NFC_ACL) | (1u << NFC_DPI) | (1u << NFC_LPM4) | (1u << NFC_LPM6) |
-                             (1u << NFC_IPSEC) | (1u << NFC_LB);
+                             (1u << NFC_IPSEC) | (1u << NFC_LB) | (1u << NFC_NAT);
     uint32_t m = 0;
     for (int p = 0; p < (int)sig_n(s); p++) m |= 1u << sig_kind(s, p);
     return m;
@@ -121,6 +121,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     o = (o + 15) & ~15u;
     if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
+    if (mask & MASK_NAT) { L.nat_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_DPI) {
         // L.cls (byte -> 2 * class, u8 / u32) sits at offset 0 (above)
         L.hot = o; o += (p.dpi.hot_states * p.dpi.ncls * 2 + 15) & ~15u;
@@ -1007,6 +1008,103 @@ __device__ __forceinline__ uint32_t toeplitz(const uint32_t *nib, const PV &v)
     return hsh;
 }
 
+// ---------------------------------------------------------------- NAT44 (Table II; R#30)
+// The translation as values: DNAT by the open-addressing table, SNAT by the inside
+// prefixes (constant bank) and the flow hash h; the L4 checksum updated per changed
+// 16-bit word (RFC 1624 eqn. 3).  Returns the new (src, dst, ports, l4 checksum).
+struct NatOut { uint32_t src, dst, ports, ck; };
+__device__ __forceinline__ uint32_t oc_add16(uint32_t a, uint32_t b)
+{
+    const uint32_t x = a + b;
+    return (x & 0xFFFF) + (x >> 16);
+}
+// RFC 1624 eqn. 3 for one field m -> m1 (identity when m == m1: ~(~HC + ~m + m) = HC
+// except that 0xFFFF and 0x0000 are the two zeros -- skipped explicitly)
+__device__ __forceinline__ uint32_t csum_upd(uint32_t hc, uint32_t m, uint32_t m1)
+{
+    const uint32_t x = oc_add16(oc_add16(~hc & 0xFFFF, ~m & 0xFFFF), m1);
+    return m == m1 ? hc : (~x & 0xFFFF);
+}
+__device__ __forceinline__ NatOut nat_values(const KParams &P, const uint32_t *nat_nib, const PV &v, uint32_t ck)
+{
+    const NatImg &N = P.nat;
+    const uint32_t h = toeplitz(nat_nib, v);
+    const uint32_t src = v.src[0], dst = v.dst[0], sp = v.sport, dp = v.dport;
+    uint32_t nsrc = src, ndst = dst, nsp = sp, ndp = dp;
+    // DNAT: (proto, dst, dport) exact match, linear probing
+    const uint32_t key1 = dp | v.proto << 16;
+    for (uint32_t slot = nat_slot(dst, key1) & N.dnat_mask;; slot = (slot + 1) & N.dnat_mask) {
+        const uint4 e = __ldg(N.dnat + slot);
+        if (!(e.y & NAT_VALID)) break;
+        if (e.x == dst && (e.y & 0xFFFFFF) == key1) { ndst = e.z; ndp = e.w; break; }
+    }
+    // SNAT: first inside prefix (constant bank, uniform loop)
+    for (uint32_t q = 0; q < N.n_inside; q++)
+        if ((src & N.in_mask[q]) == N.in_pref[q]) {
+            nsrc = __ldg(N.pool + (h & 0xFFFF) % N.n_pool);
+            nsp = N.port_lo + (h >> 16) % N.port_range;
+            break;
+        }
+    if (!(v.proto == 17 && ck == 0)) {
+        ck = csum_upd(ck, src >> 16, nsrc >> 16);
+        ck = csum_upd(ck, src & 0xFFFF, nsrc & 0xFFFF);
+        ck = csum_upd(ck, dst >> 16, ndst >> 16);
+        ck = csum_upd(ck, dst & 0xFFFF, ndst & 0xFFFF);
+        ck = csum_upd(ck, sp, nsp);
+        ck = csum_upd(ck, dp, ndp);
+        if (v.proto == 17 && ck == 0) ck = 0xFFFF;
+    }
+    return NatOut{nsrc, ndst, nsp << 16 | ndp, ck};
+}
+__device__ __forceinline__ uint32_t bswap16w(uint32_t x) { return __byte_perm(x, 0, 0x4401); }   // 16-bit value <-> 2 LE bytes
+// Applies the NAT to a packet (v.fam == 4, TCP/UDP, egress port Internet-facing):
+// header-cache fast path for a 20-B IPv4 header (bytes 24..63 written back), memory
+// path otherwise.  Updates v (and h) for the NFs after it.
+__device__ __forceinline__ void nf_nat(const KParams &P, const uint32_t *nat_nib, uint8_t *f, uint32_t h[16], PV &v,
+                                       uint64_t pol)
+{
+    const bool tcp = v.proto == 6;
+    if (v.l4_off == 34) {
+        // UDP checksum: bytes 40..41 (h[10] low half); TCP: bytes 50..51 (h[12] high half)
+        const uint32_t ckw = tcp ? h[12] >> 16 : h[10] & 0xFFFF;
+        const NatOut o = nat_values(P, nat_nib, v, bswap16w(ckw));
+        const uint32_t sb = bswap32(o.src), db = bswap32(o.dst), pb = bswap32(o.ports);   // network-order words
+        // bytes 26..29 src, 30..33 dst, 34..37 ports (word-straddling: byte_perm)
+        h[6] = __byte_perm(h[6], sb, 0x5410);            // bytes 24,25 keep; 26,27 = src[0..1]
+        h[7] = __byte_perm(sb, db, 0x5432);              // 28,29 = src[2..3]; 30,31 = dst[0..1]
+        h[8] = __byte_perm(db, pb, 0x5432);              // 32,33 = dst[2..3]; 34,35 = sport
+        h[9] = __byte_perm(pb, h[9], 0x7632);            // 36,37 = dport; 38,39 keep
+        if (tcp) h[12] = (h[12] & 0xFFFFu) | bswap16w(o.ck) << 16;
+        else h[10] = (h[10] & 0xFFFF0000u) | bswap16w(o.ck);
+        // IPv4 header checksum (RFC 1071 over bytes 14..33, field 24..25 zeroed)
+        h[6] &= 0xFFFF0000u;
+        uint32_t sum = (h[3] >> 16) + (h[4] & 0xFFFF) + (h[4] >> 16) + (h[5] & 0xFFFF) + (h[5] >> 16) +
+                       (h[6] >> 16) + (h[7] & 0xFFFF) + (h[7] >> 16) + (h[8] & 0xFFFF);
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        h[6] |= (~sum) & 0xFFFF;
+        st_stream16(f + 16, make_uint4(h[4], h[5], h[6], h[7]), pol);
+        st_stream16(f + 32, make_uint4(h[8], h[9], h[10], h[11]), pol);
+        if (tcp) st_stream16(f + 48, make_uint4(h[12], h[13], h[14], h[15]), pol);
+        v.src[0] = o.src; v.dst[0] = o.dst; v.sport = o.ports >> 16; v.dport = o.ports & 0xFFFF;
+        return;
+    }
+    // IPv4 options (rare): bytes from memory
+    const uint32_t l4 = v.l4_off, ca = l4 + (tcp ? 16 : 6);
+    const NatOut o = nat_values(P, nat_nib, v, (uint32_t)f[ca] << 8 | f[ca + 1]);
+    for (int k = 0; k < 4; k++) { f[26 + k] = (uint8_t)(o.src >> (24 - 8 * k)); f[30 + k] = (uint8_t)(o.dst >> (24 - 8 * k)); }
+    for (int k = 0; k < 4; k++) f[l4 + k] = (uint8_t)(o.ports >> (24 - 8 * k));
+    f[ca] = (uint8_t)(o.ck >> 8); f[ca + 1] = (uint8_t)o.ck;
+    f[24] = f[25] = 0;
+    uint32_t sum = 0;
+    for (uint32_t k = 14; k < l4; k += 2) sum += (uint32_t)f[k] << 8 | f[k + 1];
+    sum = (sum & 0xFFFF) + (sum >> 16);
+    sum = (sum & 0xFFFF) + (sum >> 16);
+    f[24] = (uint8_t)(~sum >> 8); f[25] = (uint8_t)~sum;
+    load_header(f, 64, h, pol);     // refresh the cache (frames here are >= 64 B: IHL > 5 + L4)
+    v.src[0] = o.src; v.dst[0] = o.dst; v.sport = o.ports >> 16; v.dport = o.ports & 0xFFFF;
+}
+
 // ---------------------------------------------------------------- AES-128 / SHA-1
 // AES-128 encryption with one T-table replicated 32 times in shared memory: lane l
 // reads copy l, which lives in bank l, so the 160 random lookups per block are free
@@ -1206,7 +1304,7 @@ struct Pkt {
 struct Ctx {
     const uint32_t *acl4, *acl6;
     DpiCtx dpi;
-    const uint32_t *te, *ms_nib, *lb_nib;
+    const uint32_t *te, *ms_nib, *lb_nib, *nat_nib;
     const uint32_t *meta;     // per-state match summary (smem or global)
     uint32_t *vst;            // smem u32 hit counters (nullptr: global atomics)
     uint64_t pol_f, pol_l;
@@ -1278,10 +1376,11 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
 // (packet, pattern) pairs of an output closure [o0, o0+nm) at slots [slot, slot+nm)
 __device__ __forceinline__ void emit_pairs(const KParams &P, uint32_t o0, uint32_t nm, uint32_t slot, uint32_t pkt)
 {
+    // o0: CSR offset of the closure, or (nm == 1) the pattern id itself (DpiHost::out_meta)
     for (uint32_t q = 0; q < nm; q++)
         if (slot + q < P.match_cap) {
             P.match_pkt[slot + q] = pkt;
-            P.match_pat[slot + q] = __ldg(P.dpi.out_ids + o0 + q);
+            P.match_pat[slot + q] = nm == 1 ? o0 : __ldg(P.dpi.out_ids + o0 + q);
         }
     if (slot + nm > P.match_cap)
         atomicAdd(&P.stats[ST_MATCH_OVF], (unsigned long long)(slot + nm - max(slot, P.match_cap)));
@@ -1312,6 +1411,53 @@ __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &
         emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
 #endif
     } else if (w.cnt >= 1) {
+        const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
+                        P.match_cap, P.stats, 1u};
+        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+        k.nmatch = r & 0x7FFFFFFFu;
+        dropped = (r >> 31) != 0;
+    }
+    return dropped;
+}
+
+// dpi_finish for a whole warp (all lanes call it): the match-pair slots of the lanes whose
+// walk had exactly one accept event are claimed with ONE atomic per warp (sum of the
+// closure sizes, exclusive prefix by ballot/popc when every closure has one pattern, else
+// by a shuffle scan); lanes with several events take the exact re-walk as in dpi_finish.
+template <int DM>
+__device__ __forceinline__ bool dpi_finish_warp(const KParams &P, const Ctx &C, Pkt &k, const Walk w, bool act)
+{
+    const uint32_t FULL = 0xFFFFFFFFu, lane = threadIdx.x & 31;
+    const uint32_t st = DM == DM_FULL ? ~w.mx : C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
+    const uint32_t meta = act && w.cnt == 1 ? C.meta[st] : DPI_META_NONE;
+    const bool single = meta != DPI_META_NONE;
+    const uint32_t nm = single ? (meta >> 20) & 0x7FF : 0u;
+    bool dropped = false;
+    if (__any_sync(FULL, nm != 0)) {
+        uint32_t excl, total;
+        if (__all_sync(FULL, nm <= 1)) {
+            const uint32_t b = __ballot_sync(FULL, nm != 0);
+            excl = __popc(b & ((1u << lane) - 1));
+            total = __popc(b);
+        } else {
+            uint32_t incl = nm;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULL, incl, d);
+                if (lane >= (uint32_t)d) incl += y;
+            }
+            total = __shfl_sync(FULL, incl, 31);
+            excl = incl - nm;
+        }
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(P.match_count, total);
+        base = __shfl_sync(FULL, base, 0);
+        if (nm) emit_pairs(P, meta & 0xFFFFF, nm, base + excl, (uint32_t)k.gidx);
+    }
+    if (single) {
+        k.nmatch = nm;
+        dropped = (meta >> 31) != 0;
+    } else if (act && w.cnt >= 1) {
         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                         P.match_cap, P.stats, 1u};
         const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
@@ -1439,7 +1585,7 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
             w.mx = max(w.mx, acc[32 + lane]);
         }
     }
-    return act ? dpi_finish<DM>(P, C, k, w) : false;
+    return dpi_finish_warp<DM>(P, C, k, w, act);
 }
 
 // ---------------------------------------------------------------- speculative ACL || DPI || TBL24
@@ -1562,6 +1708,10 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         k.out_len = nl;
         load_header(k.f, k.flen, k.h, C.pol_f);
         parse(k.h, k.f, k.flen, k.v);             // later NFs see proto 50, ports 0
+    } else if constexpr (KIND == NFC_NAT) {
+        const bool l4 = k.v.fam == 4 && (k.v.proto == 6 || k.v.proto == 17) && k.v.pl_off != k.v.l4_off;
+        if (!l4 || k.port >= 32 || !((P.nat.ext_ports >> k.port) & 1)) { k.passmask |= 1u << pos; return; }
+        nf_nat(P, C.nat_nib, k.f, k.h, k.v, C.pol_f);
     } else if constexpr (KIND == NFC_LB) {
         const uint32_t hsh = toeplitz(C.lb_nib, k.v);
         const uint32_t b = (uint32_t)(((uint64_t)hsh * P.lb.n_backends) >> 32);
@@ -1597,6 +1747,7 @@ __device__ __forceinline__ void run_any(const KParams &P, const Ctx &C, Pkt &k, 
         case NFC_LPM6: nf_apply<NFC_LPM6, DM>(P, C, k, pos); break;
         case NFC_IPSEC: nf_apply<NFC_IPSEC, DM>(P, C, k, pos); break;
         case NFC_LB: nf_apply<NFC_LB, DM>(P, C, k, pos); break;
+        case NFC_NAT: nf_apply<NFC_NAT, DM>(P, C, k, pos); break;
         }
     }
 }
@@ -1696,7 +1847,7 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
         const uint32_t nd = __popc(__ballot_sync(FULL, valid && k.drop == (uint32_t)p));
         const uint32_t kd = S == SIG_ANY ? P.kind[p] : sig_kind(S, p);
         uint32_t np = 0;
-        if (kd == NFC_LPM4 || kd == NFC_LPM6) np = __popc(__ballot_sync(FULL, (k.passmask >> p) & 1));
+        if (kd == NFC_LPM4 || kd == NFC_LPM6 || kd == NFC_NAT) np = __popc(__ballot_sync(FULL, (k.passmask >> p) & 1));
         if (lane == 0) {
             ws[ST_POS_BASE + 4 * p + 1] += nd;
             ws[ST_POS_BASE + 4 * p + 2] += np;
@@ -1869,6 +2020,12 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         for (uint32_t i = tid; i < 72 * 16; i += NT) mn[i] = __ldg(P.esp.rss_nib + i);
         C.te = te + lane;         // this lane's bank column
         C.ms_nib = mn;
+    }
+    C.nat_nib = nullptr;
+    if ((SMASK & MASK_NAT) && (mask & MASK_NAT)) {
+        uint32_t *nn = reinterpret_cast<uint32_t *>(smem + L.nat_nib);
+        for (uint32_t i = tid; i < 72 * 16; i += NT) nn[i] = __ldg(P.nat.nib + i);
+        C.nat_nib = nn;
     }
     if ((SMASK & MASK_LB) && (mask & MASK_LB)) {
         uint32_t *ln = reinterpret_cast<uint32_t *>(smem + L.lb_nib);
@@ -2050,6 +2207,7 @@ static constexpr uint32_t SIG_K2 = make_sig(2, NFC_ACL, NFC_DPI);
 static constexpr uint32_t SIG_K4 = make_sig(4, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6);
 static constexpr uint32_t SIG_K5 = make_sig(5, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6, NFC_IPSEC);
 static constexpr uint32_t SIG_K6 = make_sig(6, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6, NFC_IPSEC, NFC_LB);
+static constexpr uint32_t SIG_N3 = make_sig(3, NFC_ACL, NFC_LPM4, NFC_NAT);                       // NEXT-3
 
 #define NFC_DECLARE_LAUNCH(S, DM)                                                                   \
     extern template int launch_t<S, DM>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);

@@ -205,6 +205,7 @@ int uf_launch(const uint32_t *kinds, uint32_t n_nf, int dm, const KParams &p, ui
         case NFC_LPM4: rc = uf_stage<NFC_LPM4, DM_HOT>(p, pos, in, in_n, out, out_n, passmask, sms, st, err); break;
         case NFC_LPM6: rc = uf_stage<NFC_LPM6, DM_HOT>(p, pos, in, in_n, out, out_n, passmask, sms, st, err); break;
         case NFC_LB: rc = uf_stage<NFC_LB, DM_HOT>(p, pos, in, in_n, out, out_n, passmask, sms, st, err); break;
+        case NFC_NAT: rc = uf_stage<NFC_NAT, DM_HOT>(p, pos, in, in_n, out, out_n, passmask, sms, st, err); break;
         default: err = "unfused mode does not run IPsec"; return NFC_EUNSUP;
         }
         if (rc) return rc;

@@ -16,8 +16,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("NFC_LIB") or os.path.join(HERE, "libnfc.so")
 
 NFC_OK, NFC_EINVAL, NFC_ENOMEM, NFC_ECUDA, NFC_ESTATE, NFC_ECAP, NFC_EUNSUP = 0, -1, -2, -3, -4, -5, -6
-ACL, DPI, LPM4, LPM6, IPSEC, LB = 1, 2, 3, 4, 5, 6
-KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB}
+ACL, DPI, LPM4, LPM6, IPSEC, LB, NAT = 1, 2, 3, 4, 5, 6, 7
+KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB, "NAT": NAT}
 STATS_RESET = 1
 F_UNFUSED = 1   # nfc_chain_opts.flags: per-NF kernels with re-split (NEXT-1 baseline)
 F_PARALLEL = 2  # nfc_chain_opts.flags: the chain's NFs on different warps + XOR merge (NEXT-2)
@@ -64,6 +64,11 @@ class IpsecSpec(ctypes.Structure):
 
 class LbSpec(ctypes.Structure):
     _fields_ = [("n_backends", _u32), ("backend_port", _P), ("key", _P)]
+
+
+class NatSpec(ctypes.Structure):
+    _fields_ = [("n_inside", _u32), ("inside", _P), ("n_pool", _u32), ("pool", _P), ("port_lo", _u32),
+                ("port_hi", _u32), ("n_dnat", _u32), ("dnat", _P), ("ext_ports", _u32), ("key", _P)]
 
 
 class Batch(ctypes.Structure):
@@ -194,6 +199,17 @@ class Chain:
         p, k = _np(ports, np.uint16), _np(key, np.uint8)
         return self._load(LB, LbSpec(len(p), p.ctypes.data, k.ctypes.data))
 
+    def load_nat(self, inside: np.ndarray, pool: np.ndarray, port_lo: int, port_hi: int, dnat: np.ndarray,
+                 ext_ports: int, key: np.ndarray):
+        """NAT44 tables (nfc_nat_spec): inside prefixes (8-B records), public pool (u32),
+        SNAT port range, DNAT entries (16-B records), Internet-facing port mask, 40-B key."""
+        i, d = np.ascontiguousarray(inside), np.ascontiguousarray(dnat)     # 8-B / 16-B records
+        assert i.itemsize == 8 and d.itemsize == 16
+        p, k = _np(pool, np.uint32), _np(key, np.uint8)
+        return self._load(NAT, NatSpec(len(inside), i.ctypes.data if i.size else None, len(p), p.ctypes.data,
+                                       port_lo, port_hi, len(dnat), d.ctypes.data if d.size else None,
+                                       ext_ports, k.ctypes.data))
+
     def load_tables(self, t):
         """Load every NF of the chain from an object with the nfcgen.Tables fields."""
         for k in self.kinds:
@@ -209,6 +225,9 @@ class Chain:
                 self.load_ipsec(t.sas)
             elif k == LB:
                 self.load_lb(t.lb_ports, t.lb_key)
+            elif k == NAT:
+                self.load_nat(t.nat_inside, t.nat_pool, t.nat_port_lo, t.nat_port_hi, t.nat_dnat,
+                              t.nat_ext_ports, t.nat_key)
 
     # ------------------------------------------------------------ processing
     def process(self, batches, rec_ptr: int, match_pkt_ptr: int = 0, match_pat_ptr: int = 0,

@@ -222,3 +222,35 @@ def test_parallel_sfc_parity(nfc, cfg, k, pl):
 def test_parallel_rejects_ipsec(nfc):
     with pytest.raises(nfc.NfcError):
         nfc.Chain(["ACL", "IPSEC"], device=0, flags=nfc.F_PARALLEL)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("n_acl,pl", [(200, 64), (1000, 128), (10000, 1500), (1000, 1), (200, 0)])
+def test_n3_fw_router_nat_parity(nfc, n_acl, pl):
+    """NEXT-3 (Figs. 16-17): FW(200 / 1K / 10K rules) -> IPv4 router -> NAT44
+    at 64 / 128 / 1500 B (and ragged / IMIX): records, rewritten bytes (SNAT / DNAT,
+    IPv4 and TCP/UDP checksums) and stats equal the oracle's."""
+    w = nfcgen.workload("N3", acl_rules=n_acl, pkt_len=pl)
+    w.traffic.ttl1_ppm = 5_000
+    w.traffic.malformed_ppm = 5_000
+    ch = _chain(nfc, w)
+    got, _ = check_parity(w, ch, 3001)
+    assert (got["drop_nf"] == 0xFF).sum() > 2500
+
+
+@pytest.mark.gpu
+def test_n3_unfused_and_nat_only(nfc):
+    """The unfused baseline runs the NAT stage too; a NAT-only chain (egress port 0)
+    and a chain with every port Internet-facing match the oracle."""
+    w = nfcgen.workload("N3", acl_rules=1000, pkt_len=1)
+    ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_UNFUSED)
+    ch.load_tables(w.tables)
+    check_parity(w, ch, 2001)
+    w2 = nfcgen.workload("N3", acl_rules=200, pkt_len=1)
+    w2.tables.nat_ext_ports = 1
+    w2.kinds = ["NAT"]
+    ch2 = _chain(nfc, w2)
+    check_parity(w2, ch2, 2001)
+    w3 = nfcgen.workload("N3", acl_rules=200, pkt_len=64)
+    w3.tables.nat_ext_ports = 0xFFFFFFFF
+    check_parity(w3, _chain(nfc, w3), 2001)

@@ -143,7 +143,7 @@ def _rw(kind, fam):
 
 
 def _legal(a, b_):
-    if "IPSEC" in (a, b_):
+    if "IPSEC" in (a, b_) or "NAT" in (a, b_):   # R#29, R#30: stand alone
         return False
     for fam in (4, 6):
         ra, wa = _rw(a, fam)
