@@ -78,6 +78,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_SPEC
 #define NFC_SPEC 1            // speculative ACL || DPI head walk || TBL24 block (spec_ok)
 #endif
+#ifndef NFC_HDR_AHEAD
+#define NFC_HDR_AHEAD 0       // 1: load the next chunk's header at the tail of the current one
+#endif
 #ifndef NFC_FULL_THREADS
 #define NFC_FULL_THREADS 640   // DPI chains without IPsec: one CTA per SM (640: no spills at 96 regs)
 #endif
@@ -1373,6 +1376,20 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
     if (!k.alive) k.drop = 0xFE;
 }
 
+// pkt_begin with the header words already loaded (NFC_HDR_AHEAD)
+__device__ __forceinline__ void pkt_begin_h(const Loc &l, bool valid, Pkt &k, const uint32_t hn[16])
+{
+    k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0;
+    k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
+    k.out_len = k.flen;
+    if (!valid) return;
+#pragma unroll
+    for (int i = 0; i < 16; i++) k.h[i] = hn[i];
+    k.alive = parse(k.h, k.f, k.flen, k.v);
+    if (!k.alive) k.drop = 0xFE;
+}
+
 // (packet, pattern) pairs of an output closure [o0, o0+nm) at slots [slot, slot+nm)
 __device__ __forceinline__ void emit_pairs(const KParams &P, uint32_t o0, uint32_t nm, uint32_t slot, uint32_t pkt)
 {
@@ -2079,6 +2096,12 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         uint32_t c0 = claim(), c1 = claim();
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
         Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
+#if NFC_HDR_AHEAD
+        // the next chunk's header words are loaded at the tail of the current chunk (after
+        // its last NF, before the record store and counters), so the L2 read overlaps them
+        uint32_t hn[16];
+        if (c0 + lane < P.n_pkts) load_header(loc.f, loc.len, hn, C.pol_f);
+#endif
         while (c0 < P.n_pkts) {
             // locate chunk c1 (its descriptors arrived during the last chunk) BEFORE issuing
             // the descriptor loads of c2: an address add that consumed a just-issued load's
@@ -2090,9 +2113,16 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;
+#if NFC_HDR_AHEAD
+            pkt_begin_h(loc, valid, k, hn);
+#else
             pkt_begin(C, loc, valid, k);
+#endif
             run_part<S, DM, true>(P, C, k);
             run_part<S, DM, false>(P, C, k);
+#if NFC_HDR_AHEAD
+            if (c1 + lane < P.n_pkts) load_header(loc1.f, loc1.len, hn, C.pol_f);
+#endif
             pkt_end<S>(P, C, k, valid, g, ws, lane);
             c0 = c1;
             c1 = c2;
