@@ -41,6 +41,11 @@ NFC_API int nfc_dbg_dpi_slot(nfc_dbg *d, const uint8_t *buf, size_t n, uint16_t 
                              uint32_t *count, uint32_t *drop, uint32_t *events, uint32_t *summary);
 /* DPI tier shape: states of depth <= 1, states with a representable sparse record. */
 NFC_API int nfc_dbg_dpi_tier_shape(nfc_dbg *d, uint32_t *n_d1, uint32_t *n_sparse_ok);
+/* NAT44 translation as the kernel computes it from the device image (nat_values):
+   out = {src, dst, sport, dport, tcp/udp checksum} for a packet the NAT applies to;
+   probes (may be NULL) = DNAT hash-table slots read. */
+NFC_API int nfc_dbg_nat(nfc_dbg *d, uint8_t proto, uint32_t src, uint32_t dst, uint16_t sport, uint16_t dport,
+                        uint16_t ck, uint32_t out[5], uint32_t *probes);
 /* LPM4: next-hop index (0x7FFF = miss) and number of table reads (1 or 2). */
 NFC_API int nfc_dbg_lpm4(nfc_dbg *d, uint32_t dst, uint32_t *nh, uint32_t *reads);
 /* LPM6: next-hop index (0x7FFF = miss), hash-level probes and hash-slot reads. */

@@ -20,6 +20,7 @@ struct nfc_dbg {
     std::vector<uint16_t> tbl24, tbllong;
     std::vector<uint2> nh, pmac;
     Lpm6Host l6;
+    NatHost nat;
 };
 
 static inline uint32_t be32(const uint8_t *p) { return (uint32_t)p[0] << 24 | (uint32_t)p[1] << 16 | (uint32_t)p[2] << 8 | p[3]; }
@@ -52,6 +53,10 @@ int nfc_dbg_build(uint32_t kind, const void *spec, size_t spec_bytes, nfc_dbg **
     case NFC_LPM6:
         if (spec_bytes != sizeof(nfc_lpm6_spec)) break;
         err = build_lpm6(*static_cast<const nfc_lpm6_spec *>(spec), d->l6);
+        break;
+    case NFC_NAT:
+        if (spec_bytes != sizeof(nfc_nat_spec)) break;
+        err = build_nat(*static_cast<const nfc_nat_spec *>(spec), d->nat);
         break;
     }
     if (!err.empty()) {
@@ -342,6 +347,51 @@ int nfc_dbg_toeplitz(const uint8_t key[40], const uint8_t *in, size_t n, uint32_
     uint32_t x = 0;
     for (size_t i = 0; i < n; i++) x ^= nib[(2 * i) * 16 + (in[i] >> 4)] ^ nib[(2 * i + 1) * 16 + (in[i] & 15)];
     *h = x;
+    return NFC_OK;
+}
+
+int nfc_dbg_nat(nfc_dbg *d, uint8_t proto, uint32_t src, uint32_t dst, uint16_t sport, uint16_t dport, uint16_t ck,
+                uint32_t out[5], uint32_t *probes)
+{
+    if (!d || d->kind != NFC_NAT || !out) return NFC_EINVAL;
+    const NatHost &N = d->nat;
+    // the kernel's nat_values (sfc_kernel.cuh): Toeplitz over src|dst|sport|dport by the
+    // nibble tables, DNAT open-addressing probe, SNAT by the inside prefixes, RFC 1624
+    uint8_t t[12];
+    for (int k = 0; k < 4; k++) { t[k] = (uint8_t)(src >> (24 - 8 * k)); t[4 + k] = (uint8_t)(dst >> (24 - 8 * k)); }
+    t[8] = (uint8_t)(sport >> 8); t[9] = (uint8_t)sport; t[10] = (uint8_t)(dport >> 8); t[11] = (uint8_t)dport;
+    uint32_t h = 0;
+    for (int i = 0; i < 12; i++) h ^= N.nib[(2 * i) * 16 + (t[i] >> 4)] ^ N.nib[(2 * i + 1) * 16 + (t[i] & 15)];
+    uint32_t nsrc = src, ndst = dst, nsp = sport, ndp = dport, np = 0;
+    const uint32_t key1 = (uint32_t)dport | (uint32_t)proto << 16;
+    for (uint32_t slot = nat_slot(dst, key1) & N.img.dnat_mask;; slot = (slot + 1) & N.img.dnat_mask) {
+        np++;
+        const uint4 e = N.dnat[slot];
+        if (!(e.y & NAT_VALID)) break;
+        if (e.x == dst && (e.y & 0xFFFFFF) == key1) { ndst = e.z; ndp = e.w; break; }
+    }
+    for (uint32_t q = 0; q < N.img.n_inside; q++)
+        if ((src & N.img.in_mask[q]) == N.img.in_pref[q]) {
+            nsrc = N.pool[(h & 0xFFFF) % N.img.n_pool];
+            nsp = N.img.port_lo + (h >> 16) % N.img.port_range;
+            break;
+        }
+    uint32_t c = ck;
+    if (!(proto == 17 && c == 0)) {
+        auto upd = [](uint32_t hc, uint32_t m, uint32_t m1) {
+            auto add = [](uint32_t a, uint32_t b) { uint32_t x = a + b; return (x & 0xFFFF) + (x >> 16); };
+            return m == m1 ? hc : (~add(add(~hc & 0xFFFF, ~m & 0xFFFF), m1) & 0xFFFF);
+        };
+        c = upd(c, src >> 16, nsrc >> 16);
+        c = upd(c, src & 0xFFFF, nsrc & 0xFFFF);
+        c = upd(c, dst >> 16, ndst >> 16);
+        c = upd(c, dst & 0xFFFF, ndst & 0xFFFF);
+        c = upd(c, sport, nsp);
+        c = upd(c, dport, ndp);
+        if (proto == 17 && c == 0) c = 0xFFFF;
+    }
+    out[0] = nsrc; out[1] = ndst; out[2] = nsp; out[3] = ndp; out[4] = c;
+    if (probes) *probes = np;
     return NFC_OK;
 }
 

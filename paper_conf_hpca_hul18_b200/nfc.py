@@ -85,7 +85,7 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
-                 "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_lpm4",
+                 "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
                  "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
 
@@ -120,6 +120,8 @@ def _load_lib():
     L.nfc_dbg_dpi_tier.argtypes = [_P, _u32, _u32, _P, ctypes.c_size_t, _P, _u32, P32, P32, _P]
     L.nfc_dbg_dpi_tier_shape.argtypes = [_P, P32, P32]
     L.nfc_dbg_dpi_slot.argtypes = [_P, _P, ctypes.c_size_t, _P, _u32, P32, P32, P32, P32]
+    L.nfc_dbg_nat.argtypes = [_P, ctypes.c_uint8, _u32, _u32, ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint16,
+                              _P, P32]
     L.nfc_dbg_lpm4.argtypes = [_P, _u32, P32, P32]
     L.nfc_dbg_lpm6.argtypes = [_P, _P, P32, P32, P32]
     L.nfc_dbg_lpm6_levels.argtypes = [_P, P32]
@@ -338,6 +340,13 @@ class HostImage:
             r, n, p = _np(tables["routes"]), _np(tables["nexthops"]), _np(tables["port_macs"], np.uint8)
             self._keep += [r, n, p]
             spec = LpmSpec(len(r), r.ctypes.data, len(n), n.ctypes.data, len(p), p.ctypes.data)
+        elif kind == NAT:
+            i, d = np.ascontiguousarray(tables["inside"]), np.ascontiguousarray(tables["dnat"])
+            p, k = _np(tables["pool"], np.uint32), _np(tables["key"], np.uint8)
+            self._keep += [i, d, p, k]
+            spec = NatSpec(len(i), i.ctypes.data if i.size else None, len(p), p.ctypes.data, tables["port_lo"],
+                           tables["port_hi"], len(d), d.ctypes.data if d.size else None, tables.get("ext_ports", 0),
+                           k.ctypes.data)
         else:
             raise ValueError(kind)
         h = _P()
@@ -349,6 +358,13 @@ class HostImage:
         if getattr(self, "h", None):
             lib.nfc_dbg_destroy(self.h)
             self.h = None
+
+    def nat(self, proto: int, src: int, dst: int, sport: int, dport: int, ck: int):
+        """The kernel's NAT translation: ((src, dst, sport, dport, checksum), DNAT probes)."""
+        out = np.zeros(5, dtype=np.uint32)
+        pr = _u32()
+        _check(lib.nfc_dbg_nat(self.h, proto, src, dst, sport, dport, ck, out.ctypes.data, ctypes.byref(pr)))
+        return tuple(int(x) for x in out), pr.value
 
     def dpi(self, data: bytes, cap: int = 65536):
         ids = np.zeros(cap, dtype=np.uint16)

@@ -284,3 +284,39 @@ def test_nibble_toeplitz_ms_rss(nfc, row):
 def test_ipad_opad_hmac_rfc2202(nfc, row):
     key = bytes.fromhex(row[0]).ljust(20, b"\x00")  # HMAC zero-pads keys shorter than the block
     assert nfc.dbg_hmac_sha1(key, bytes.fromhex(row[1])).hex() == row[2]
+
+
+def test_nat_image_vs_oracle(nfc):
+    """The NAT device image (DNAT open-addressing table, inside prefixes, pool, Toeplitz
+    nibbles) walked with the kernel's nat_values gives the oracle's translated header
+    for every packet of an N3 sample, and rejects malformed specs."""
+    w = nfcgen.workload("N3", acl_rules=200, small=True, pkt_len=1)
+    t = w.tables
+    t.nat_ext_ports = 1
+    img = nfc.HostImage("NAT", inside=t.nat_inside, pool=t.nat_pool, port_lo=t.nat_port_lo, port_hi=t.nat_port_hi,
+                        dnat=t.nat_dnat, ext_ports=1, key=t.nat_key)
+    orc = oracle.OracleChain(["NAT"], t)
+    b = nfcgen.generate(w.traffic, t, 0, 1500)
+    max_probes = 0
+    for i in range(b.n):
+        fr = b.frame(i)
+        if fr[12:14] != b"\x08\x00" or fr[23] not in (6, 17):
+            continue
+        l4 = 14 + 4 * (fr[14] & 15)
+        ca = l4 + (16 if fr[23] == 6 else 6)
+        r, out, _ = orc.run_one(fr, i, headroom=0)
+        got, probes = img.nat(fr[23], int.from_bytes(fr[26:30], "big"), int.from_bytes(fr[30:34], "big"),
+                              int.from_bytes(fr[l4:l4 + 2], "big"), int.from_bytes(fr[l4 + 2:l4 + 4], "big"),
+                              int.from_bytes(fr[ca:ca + 2], "big"))
+        want = (int.from_bytes(out[26:30], "big"), int.from_bytes(out[30:34], "big"),
+                int.from_bytes(out[l4:l4 + 2], "big"), int.from_bytes(out[l4 + 2:l4 + 4], "big"),
+                int.from_bytes(out[ca:ca + 2], "big"))
+        assert got == want, i
+        max_probes = max(max_probes, probes)
+    assert max_probes <= 16                      # load factor <= 1/2
+    dup = np.concatenate([t.nat_dnat, t.nat_dnat[:1]])
+    with pytest.raises(Exception):
+        nfc.HostImage("NAT", inside=t.nat_inside, pool=t.nat_pool, port_lo=1, port_hi=2, dnat=dup, key=t.nat_key)
+    with pytest.raises(Exception):
+        nfc.HostImage("NAT", inside=t.nat_inside, pool=t.nat_pool, port_lo=9, port_hi=2, dnat=t.nat_dnat,
+                      key=t.nat_key)
