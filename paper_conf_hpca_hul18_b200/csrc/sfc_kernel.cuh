@@ -78,6 +78,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_SPEC
 #define NFC_SPEC 1            // speculative ACL || DPI head walk || TBL24 block (spec_ok)
 #endif
+#ifndef NFC_DESC_L1
+#define NFC_DESC_L1 0         // 1: descriptors prefetched into L1 two chunks ahead instead of registers
+#endif
 #ifndef NFC_HDR_AHEAD
 #define NFC_HDR_AHEAD 0       // 1: load the next chunk's header at the tail of the current one
 #endif
@@ -2094,6 +2097,35 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // software pipeline over chunks: descriptors (off/len) of chunk c2 are loaded two
         // iterations ahead, the frame of chunk c1 is prefetched into L2 one ahead
         uint32_t c0 = claim(), c1 = claim();
+#if NFC_DESC_L1
+        // descriptors (off/len) are prefetched into L1 two chunks ahead -- no registers held
+        // across a chunk -- and re-loaded (L1 hits) when the frame prefetch and the chunk need them
+        auto desc_l1 = [&](uint32_t g) {
+            if (P.n_batches == 1 && g < P.n_pkts) {
+                asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.off + g));
+                asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.len + g));
+            }
+        };
+        desc_l1(c0 + lane);
+        desc_l1(c1 + lane);
+        while (c0 < P.n_pkts) {
+            if (c1 + lane < P.n_pkts) {
+                const Loc l1 = pkt_locate(P, c1 + lane, true);
+                asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
+            }
+            const uint32_t c2 = claim();
+            desc_l1(c2 + lane);
+            const uint32_t g = c0 + lane;
+            const bool valid = g < P.n_pkts;
+            Pkt k;
+            pkt_begin(C, pkt_locate(P, g, valid), valid, k);
+            run_part<S, DM, true>(P, C, k);
+            run_part<S, DM, false>(P, C, k);
+            pkt_end<S>(P, C, k, valid, g, ws, lane);
+            c0 = c1;
+            c1 = c2;
+        }
+#else
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
         Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
 #if NFC_HDR_AHEAD
@@ -2129,6 +2161,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             loc = loc1;
             raw1 = raw2;
         }
+#endif
     } else if constexpr (KCfg<S, DM>::esp) {
         // CTA tiles claimed in global order (ESP sequence numbers need the order)
         for (;;) {
