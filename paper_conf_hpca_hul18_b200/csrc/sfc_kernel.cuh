@@ -79,7 +79,7 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #define NFC_SPEC 1            // speculative ACL || DPI head walk || TBL24 block (spec_ok)
 #endif
 #ifndef NFC_DESC_L1
-#define NFC_DESC_L1 0         // 1: descriptors prefetched into L1 two chunks ahead instead of registers
+#define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
 #endif
 #ifndef NFC_HDR_AHEAD
 #define NFC_HDR_AHEAD 0       // 1: load the next chunk's header at the tail of the current one
@@ -2108,9 +2108,14 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         };
         desc_l1(c0 + lane);
         desc_l1(c1 + lane);
+#if NFC_HDR_AHEAD
+        uint32_t hn[16];
+        if (c0 + lane < P.n_pkts) { const Loc l0 = pkt_locate(P, c0 + lane, true); load_header(l0.f, l0.len, hn, C.pol_f); }
+#endif
         while (c0 < P.n_pkts) {
+            Loc l1{nullptr, 0, 0};
             if (c1 + lane < P.n_pkts) {
-                const Loc l1 = pkt_locate(P, c1 + lane, true);
+                l1 = pkt_locate(P, c1 + lane, true);
                 asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
             }
             const uint32_t c2 = claim();
@@ -2118,9 +2123,16 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;
+#if NFC_HDR_AHEAD
+            pkt_begin_h(pkt_locate(P, g, valid), valid, k, hn);
+#else
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
+#endif
             run_part<S, DM, true>(P, C, k);
             run_part<S, DM, false>(P, C, k);
+#if NFC_HDR_AHEAD
+            if (c1 + lane < P.n_pkts) load_header(l1.f, l1.len, hn, C.pol_f);
+#endif
             pkt_end<S>(P, C, k, valid, g, ws, lane);
             c0 = c1;
             c1 = c2;
