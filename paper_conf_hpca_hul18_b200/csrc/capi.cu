@@ -446,6 +446,16 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
             }
         }
     }
+    // LPM4 next-hop records in shared memory when they fit beside everything else
+    p.l4.nh_smem = 0;
+    if (!par && (c->mask & MASK_LPM4) && c->l4.n_nh * 16 <= 8192) {
+        p.l4.nh_smem = 1;
+        int smem_sm = 0;
+        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device);
+        const int per = v.threads > 256 ? 1 : (c->mask & MASK_IPSEC) ? 2 : 4;
+        const size_t cap = std::min(sfc_smem_limit(c->device), (size_t)smem_sm / per) - 1024;
+        if (sfc_smem_bytes(v, p) > cap) p.l4.nh_smem = 0;
+    }
     p.dpi.row2 = 2 * c->dpi.ncls;
     p.dpi.hk2 = p.dpi.hot_states ? 2 * (p.dpi.hot_states * c->dpi.ncls - 1) : 0;
     if (c->mask & MASK_DPI) {

@@ -86,6 +86,7 @@ struct Lpm4Img {
     const uint2 *nh;             // {port | mac0<<16 | mac1<<24, mac2..mac5}
     const uint2 *pmac;           // per port: {mac0..3, mac4|mac5<<8}
     uint32_t n_nh, n_ports;
+    uint32_t nh_smem;            // per launch: 1 = {nh, pmac[port]} records (16 B) staged in shared memory
 };
 
 // ---------------------------------------------------------------- LPM6 (Waldvogel)
@@ -167,7 +168,8 @@ enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, S
 struct SmemLayout {
     uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, par, total;
     uint32_t frow0;
-    uint32_t nat_nib;             // NAT Toeplitz nibbles               // DM_FULL: row of slot 0 (DpiImg::frows)
+    uint32_t nat_nib;             // NAT Toeplitz nibbles
+    uint32_t nh4;                 // LPM4 next-hop records (Lpm4Img::nh_smem)               // DM_FULL: row of slot 0 (DpiImg::frows)
 };
 
 struct KParams {

@@ -78,6 +78,12 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_SPEC
 #define NFC_SPEC 1            // speculative ACL || DPI head walk || TBL24 block (spec_ok)
 #endif
+#ifndef NFC_T24_NA
+#define NFC_T24_NA 1          // DIR-24-8 reads bypass L1
+#endif
+#ifndef NFC_PF_LATE
+#define NFC_PF_LATE 1         // frame L2 prefetch of the next chunk issued after the chain's head part
+#endif
 #ifndef NFC_DESC_L1
 #define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
 #endif
@@ -144,6 +150,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
         L.acl6 = o; o += s6 * 4;
     }
     o = (o + 15) & ~15u;
+    if ((mask & MASK_LPM4) && p.l4.nh_smem) { L.nh4 = o; o += p.l4.n_nh * 16; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
         L.prefix = o; o += 256 * 4;
@@ -195,7 +202,13 @@ __device__ __forceinline__ void st_stream16(void *a, uint4 v, uint64_t pol)
 __device__ __forceinline__ uint32_t ld_tab16(const uint16_t *a, uint64_t pol)
 {
     uint16_t v;
+#if NFC_T24_NA
+    // DIR-24-8 reads are random over 32 MB: keep them out of L1 (the descriptors and the
+    // next-hop records live there)
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(a), "l"(pol));
+#else
     asm("ld.global.nc.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(a), "l"(pol));
+#endif
     return v;
 }
 // predicated read-only u16 load: returns `dflt` when !p (no memory access)
@@ -1303,6 +1316,7 @@ struct Pkt {
     uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
     uint32_t t24;             // TBL24 entry, loaded right after parse (NFC_EARLY_T24)
     uint32_t mmeta, mslot;    // deferred match-pair emission: closure meta, first pair slot
+    uint32_t mbase;           // deferred warp-aggregated claim: base slot (lane 0)
     bool alive;
 };
 
@@ -1370,7 +1384,7 @@ __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool val
 __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid, Pkt &k)
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
-    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
     k.out_len = k.flen;
     if (!valid) return;
@@ -1383,7 +1397,7 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
 __device__ __forceinline__ void pkt_begin_h(const Loc &l, bool valid, Pkt &k, const uint32_t hn[16])
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
-    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0;
+    k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
     k.out_len = k.flen;
     if (!valid) return;
@@ -1424,12 +1438,8 @@ __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &
         const uint32_t nm = (meta >> 20) & 0x7FF;
         k.nmatch = nm;
         dropped = (meta >> 31) != 0;
-#if NFC_DEFER_PAIRS
-        k.mmeta = meta & 0x7FFFFFFFu;
-        k.mslot = atomicAdd(P.match_count, nm);
-#else
+        // (per-lane path: emitted at once -- the unfused and parallel kernels have no pkt_end)
         emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
-#endif
     } else if (w.cnt >= 1) {
         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                         P.match_cap, P.stats, 1u};
@@ -1471,8 +1481,16 @@ __device__ __forceinline__ bool dpi_finish_warp(const KParams &P, const Ctx &C, 
         }
         uint32_t base = 0;
         if (lane == 0) base = atomicAdd(P.match_count, total);
+#if NFC_DEFER_PAIRS
+        // the atomic's result is consumed at the end of the chunk (pkt_end): its round trip
+        // overlaps the NFs after the DPI
+        k.mbase = base;
+        k.mslot = excl;
+        k.mmeta = nm ? meta & 0x7FFFFFFFu : 0u;
+#else
         base = __shfl_sync(FULL, base, 0);
         if (nm) emit_pairs(P, meta & 0xFFFFF, nm, base + excl, (uint32_t)k.gidx);
+#endif
     }
     if (single) {
         k.nmatch = nm;
@@ -1704,7 +1722,11 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         uint32_t nh = k.t24 != 0xFFFFFFFFu ? k.t24 : ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
         if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
         if (nh == 0x7FFF || hbyte(k.h, 22) <= 1) dropped = true;
-        else {
+        else if (P.l4.nh_smem) {          // {nh, pmac[nh.port]} in one shared-memory record
+            const uint4 r = reinterpret_cast<const uint4 *>(nfc_smem + P.lay.nh4)[nh];
+            forward_rewrite(k.f, k.h, k.v, make_uint2(r.x, r.y), make_uint2(r.z, r.w), C.pol_f);
+            k.port = r.y >> 16;
+        } else {
             const uint2 n = __ldg(P.l4.nh + nh);
             const uint32_t pt = n.y >> 16;
             forward_rewrite(k.f, k.h, k.v, n, __ldg(P.l4.pmac + pt), C.pol_f);
@@ -1824,8 +1846,14 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
                                         unsigned long long *ws, uint32_t lane)
 {
     constexpr uint32_t M = sig_mask(S);
-    if constexpr ((M & MASK_DPI) != 0 && NFC_DEFER_PAIRS)
-        if (k.mmeta) emit_pairs(P, k.mmeta & 0xFFFFF, k.mmeta >> 20, k.mslot, (uint32_t)k.gidx);
+    if constexpr ((M & MASK_DPI) != 0 && NFC_DEFER_PAIRS) {
+        // warp-aggregated claims keep the base in lane 0 (k.mbase) and the lane's offset in
+        // k.mslot; per-lane claims keep the absolute slot in k.mslot and k.mbase = 0
+        if (__any_sync(0xFFFFFFFFu, k.mmeta != 0)) {
+            const uint32_t b0 = __shfl_sync(0xFFFFFFFFu, k.mbase, 0);
+            if (k.mmeta) emit_pairs(P, k.mmeta & 0xFFFFF, k.mmeta >> 20, b0 + k.mslot, (uint32_t)k.gidx);
+        }
+    }
     if (valid) {
         if (k.drop != 0xFF) k.port = 0xFFFF;
         const uint4 rec = make_uint4(k.drop | k.esp_sa << 8 | k.port << 16, k.acl_rule | k.lb_b << 16,
@@ -2041,6 +2069,15 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         C.te = te + lane;         // this lane's bank column
         C.ms_nib = mn;
     }
+    if ((SMASK & MASK_LPM4) && (mask & MASK_LPM4) && P.l4.nh_smem) {
+        uint4 *r = reinterpret_cast<uint4 *>(smem + L.nh4);
+        for (uint32_t i = tid; i < P.l4.n_nh; i += NT) {
+            const uint2 n = __ldg(P.l4.nh + i);
+            const uint32_t pt = n.y >> 16;
+            const uint2 m = pt < P.l4.n_ports ? __ldg(P.l4.pmac + pt) : make_uint2(0, 0);
+            r[i] = make_uint4(n.x, n.y, m.x, m.y);
+        }
+    }
     C.nat_nib = nullptr;
     if ((SMASK & MASK_NAT) && (mask & MASK_NAT)) {
         uint32_t *nn = reinterpret_cast<uint32_t *>(smem + L.nat_nib);
@@ -2114,9 +2151,15 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 #endif
         while (c0 < P.n_pkts) {
             Loc l1{nullptr, 0, 0};
+            const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && P.n_batches == 1;   // warp-uniform
+            uint64_t off1 = 0;
             if (c1 + lane < P.n_pkts) {
-                l1 = pkt_locate(P, c1 + lane, true);
-                asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
+                if (late) {
+                    off1 = P.b0.off[c1 + lane];        // consumed after the head part (below)
+                } else {
+                    l1 = pkt_locate(P, c1 + lane, true);
+                    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
+                }
             }
             const uint32_t c2 = claim();
             desc_l1(c2 + lane);
@@ -2129,6 +2172,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #endif
             run_part<S, DM, true>(P, C, k);
+            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(P.b0.arena + off1));
             run_part<S, DM, false>(P, C, k);
 #if NFC_HDR_AHEAD
             if (c1 + lane < P.n_pkts) load_header(l1.f, l1.len, hn, C.pol_f);
