@@ -1696,6 +1696,18 @@ __device__ __forceinline__ Walk dpi_head_spec(const KParams &P, const uint32_t h
         dfa_step_if<DM_FULL>(P, w, byte_of(h[idx >> 2], idx & 3), (uint32_t)idx - a < b - a);
     return w;
 }
+// the same walk when every lane's payload starts at byte 42 (UDP) or 54 (TCP) and runs
+// past byte 64: unconditional steps, a TCP lane restarting from the root at byte 54
+__device__ __forceinline__ Walk dpi_head_fast(const KParams &P, const uint32_t h[16], bool tcp)
+{
+    Walk w{0, 0, 0};
+#pragma unroll
+    for (int idx = 42; idx < 64; idx++) {
+        if (idx == 54 && tcp) w = Walk{0, 0, 0};
+        dfa_step<DM_FULL>(P, w, byte_of(h[idx >> 2], idx & 3));
+    }
+    return w;
+}
 template <uint32_t S>
 __device__ __forceinline__ bool spec_ok(const KParams &P)
 {
@@ -1809,11 +1821,23 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
         // speculative ACL || DPI head walk || TBL24 (see spec_ok), warp-uniform choice
         const bool v4 = !k.alive || (k.v.fam == 4 && k.v.pl_off >= 42);   // payload starts inside [42, 64) or later
         if (spec_ok<S>(P) && __all_sync(0xFFFFFFFFu, v4)) {
-            const uint32_t r = acl4_spec(P, k.v);
-            const Walk wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
-            if constexpr (sig_pos(S, NFC_LPM4) != 0xFF && (sig_pos(S, NFC_IPSEC) == 0xFF ||
-                                                            sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4)))
-                k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+            constexpr bool T24 = sig_pos(S, NFC_LPM4) != 0xFF &&
+                                 (sig_pos(S, NFC_IPSEC) == 0xFF || sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4));
+            // UDP/TCP payloads from byte 42/54 past byte 64 (64-B-class frames): unconditional
+            // DFA steps; else every step predicated.  Each branch is one basic block.
+            const bool fastw = __all_sync(0xFFFFFFFFu, !k.alive || ((k.v.pl_off == 42 || k.v.pl_off == 54) &&
+                                                                    k.v.ip_end >= 64));
+            uint32_t r;
+            Walk wh;
+            if (fastw) {
+                r = acl4_spec(P, k.v);
+                wh = dpi_head_fast(P, k.h, k.v.pl_off == 54);
+                if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+            } else {
+                r = acl4_spec(P, k.v);
+                wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
+                if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+            }
             if (k.alive) {                     // ACL effects (position 0)
                 const uint32_t rule = r & 0xFFFF;
                 k.acl_rule = rule;
