@@ -84,6 +84,12 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_PF_LATE
 #define NFC_PF_LATE 1         // frame L2 prefetch of the next chunk issued after the chain's head part
 #endif
+#ifndef NFC_HOT_FAST
+#define NFC_HOT_FAST 0        // 1: DM_HOT split walk takes the unconditional 16-byte step too
+#endif
+#ifndef NFC_CARRY_DESC
+#define NFC_CARRY_DESC 1      // carry the next chunk's off/len in registers from the loop top (C1 +2 %)
+#endif
 #ifndef NFC_DESC_L1
 #define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
 #endif
@@ -1595,7 +1601,7 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
                 if ((x & 127) == 0 && x + NFC_PF_DIST < e0) prefetch_l2(f + x + NFC_PF_DIST);
                 const uint4 q = ld_stream16(f + x, C.pol_f);
                 uint32_t wd[4] = {q.x, q.y, q.z, q.w};
-                if (DM == DM_FULL && x >= v0 && x + 16 <= e0) {
+                if ((DM == DM_FULL || NFC_HOT_FAST) && x >= v0 && x + 16 <= e0) {
 #pragma unroll
                     for (int kk = 0; kk < 16; kk++) {
                         const uint32_t y = (kk & 3) == 0 ? tie<DM>(wd[kk >> 2], pw) : wd[kk >> 2];
@@ -2173,13 +2179,26 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         uint32_t hn[16];
         if (c0 + lane < P.n_pkts) { const Loc l0 = pkt_locate(P, c0 + lane, true); load_header(l0.f, l0.len, hn, C.pol_f); }
 #endif
+#if NFC_CARRY_DESC
+        // single batch: the next chunk's off/len are read at the top of the current one and
+        // carried into it, so its header loads issue without a descriptor round trip
+        uint64_t off0 = 0;
+        uint32_t len0 = 0;
+        if (P.n_batches == 1 && c0 + lane < P.n_pkts) { off0 = P.b0.off[c0 + lane]; len0 = P.b0.len[c0 + lane]; }
+#endif
         while (c0 < P.n_pkts) {
             Loc l1{nullptr, 0, 0};
             const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && P.n_batches == 1;   // warp-uniform
             uint64_t off1 = 0;
+#if NFC_CARRY_DESC
+            uint32_t len1 = 0;
+#endif
             if (c1 + lane < P.n_pkts) {
                 if (late) {
                     off1 = P.b0.off[c1 + lane];        // consumed after the head part (below)
+#if NFC_CARRY_DESC
+                    len1 = P.b0.len[c1 + lane];
+#endif
                 } else {
                     l1 = pkt_locate(P, c1 + lane, true);
                     asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
@@ -2192,6 +2211,9 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             Pkt k;
 #if NFC_HDR_AHEAD
             pkt_begin_h(pkt_locate(P, g, valid), valid, k, hn);
+#elif NFC_CARRY_DESC
+            if (late) pkt_begin(C, Loc{P.b0.arena + off0, len0, P.b0.first + g}, valid, k);
+            else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #else
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #endif
@@ -2204,6 +2226,10 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             pkt_end<S>(P, C, k, valid, g, ws, lane);
             c0 = c1;
             c1 = c2;
+#if NFC_CARRY_DESC
+            off0 = off1;
+            len0 = len1;
+#endif
         }
 #else
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
