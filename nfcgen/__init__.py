@@ -542,5 +542,5 @@ def workload(name: str, pkt_len: Optional[int] = None, k: Optional[int] = None,
         tp = TrafficParams(seed=sd, pkt_len=64 if pkt_len is None else pkt_len, match_ppm=0, tcp_pct=30,
                            l4csum=1)
         gen_nat(np.random.default_rng(np.random.PCG64(sd + 1000)), tp, t, n_dnat=1000 if not small else 200)
-        return Workload("N3", kinds, t, tp, note=f"FW({n_acl})->IPv4 router(1K)->NAT44, SNAT+DNAT")
+        return Workload(f"N3_{n_acl}", kinds, t, tp, note=f"FW({n_acl})->IPv4 router(1K)->NAT44, SNAT+DNAT")
     raise ValueError(name)
