@@ -115,6 +115,8 @@ struct EspSa {                   // 256 B
     uint32_t pad[8];
 };
 static_assert(sizeof(EspSa) == 256, "EspSa must stay 16-B aligned in arrays");
+// round keys staged in shared memory per SA at an odd word stride (bank spread)
+static const uint32_t ESP_RK_STRIDE = 45;
 struct EspImg {
     const EspSa *sa;
     uint32_t n_sa;
@@ -169,7 +171,8 @@ struct SmemLayout {
     uint32_t wst, vst, te, ms_nib, lb_nib, cls, hot, sp, meta, seg, acl4, acl6, wcnt, prefix, par, total;
     uint32_t frow0;
     uint32_t nat_nib;             // NAT Toeplitz nibbles
-    uint32_t nh4;                 // LPM4 next-hop records (Lpm4Img::nh_smem)               // DM_FULL: row of slot 0 (DpiImg::frows)
+    uint32_t nh4;                 // LPM4 next-hop records (Lpm4Img::nh_smem)
+    uint32_t rk;                  // ESP: AES round keys of every SA, ESP_RK_STRIDE words each               // DM_FULL: row of slot 0 (DpiImg::frows)
 };
 
 struct KParams {

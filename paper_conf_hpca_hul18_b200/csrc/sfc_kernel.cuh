@@ -84,6 +84,15 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_PF_LATE
 #define NFC_PF_LATE 1         // frame L2 prefetch of the next chunk issued after the chain's head part
 #endif
+#ifndef NFC_ESP_PF
+#define NFC_ESP_PF 1          // prefetch the whole frame into L2 when ESP starts on it (+1 %)
+#endif
+#ifndef NFC_ESP_MINB
+#define NFC_ESP_MINB 2        // IPsec chains: resident 256-thread tiles per SM (launch bounds)
+#endif
+#ifndef NFC_ESP_RK_SMEM
+#define NFC_ESP_RK_SMEM 1     // ESP reads AES round keys from shared memory (one out-of-line block cipher; C2 +11 %)
+#endif
 #ifndef NFC_HOT_FAST
 #define NFC_HOT_FAST 0        // 1: DM_HOT split walk takes the unconditional 16-byte step too
 #endif
@@ -119,7 +128,7 @@ template <uint32_t S, int DM> struct KCfg {
     static constexpr int nws = kcfg_nws(S);
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
     static constexpr int threads = kcfg_threads(S, DM);
-    static constexpr int minb = esp ? 2 : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
+    static constexpr int minb = esp ? NFC_ESP_MINB : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
     static constexpr uint32_t claim = DM == DM_FULL ? NFC_CLAIM : 1;   // chunks per warp claim
 };
@@ -137,7 +146,12 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     L.wst = o; o += nwarp * nws * 8;                                // per-warp private counters (u64)
     L.vst = o; o += (p.smem_stats ? p.stats_len - NFIX : 0) * 4;  // ACL/LB/SA hit counters (u32)
     o = (o + 15) & ~15u;
-    if (mask & MASK_IPSEC) { L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4; }
+    if (mask & MASK_IPSEC) {
+        L.te = o; o += 256 * 32 * 4; L.ms_nib = o; o += 72 * 16 * 4;
+#if NFC_ESP_RK_SMEM
+        L.rk = o; o += ((p.esp.n_sa * ESP_RK_STRIDE * 4) + 15) & ~15u;
+#endif
+    }
     if (mask & MASK_LB) { L.lb_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_NAT) { L.nat_nib = o; o += 72 * 16 * 4; }
     if (mask & MASK_DPI) {
@@ -1161,6 +1175,30 @@ __device__ __forceinline__ void aes128_encrypt(const uint32_t *tl, const uint32_
 #undef SB
 }
 
+// the same cipher with round keys in shared memory (rk: this SA's 44 words), out of line:
+// one copy of the 10 rounds in the kernel instead of four inlined per 16-word SHA block
+static __device__ __noinline__ uint4 aes128_encrypt_s(const uint32_t *tl, const uint32_t *rk, uint32_t in0, uint32_t in1,
+                                                      uint32_t in2, uint32_t in3)
+{
+    uint32_t s0 = in0 ^ rk[0], s1 = in1 ^ rk[1], s2 = in2 ^ rk[2], s3 = in3 ^ rk[3];
+#pragma unroll
+    for (int r = 1; r < 10; r++) {
+        const uint32_t t0 = T(tl, s0 >> 24) ^ ror8(T(tl, (s1 >> 16) & 255)) ^ ror16(T(tl, (s2 >> 8) & 255)) ^ ror24(T(tl, s3 & 255)) ^ rk[4 * r];
+        const uint32_t t1 = T(tl, s1 >> 24) ^ ror8(T(tl, (s2 >> 16) & 255)) ^ ror16(T(tl, (s3 >> 8) & 255)) ^ ror24(T(tl, s0 & 255)) ^ rk[4 * r + 1];
+        const uint32_t t2 = T(tl, s2 >> 24) ^ ror8(T(tl, (s3 >> 16) & 255)) ^ ror16(T(tl, (s0 >> 8) & 255)) ^ ror24(T(tl, s1 & 255)) ^ rk[4 * r + 2];
+        const uint32_t t3 = T(tl, s3 >> 24) ^ ror8(T(tl, (s0 >> 16) & 255)) ^ ror16(T(tl, (s1 >> 8) & 255)) ^ ror24(T(tl, s2 & 255)) ^ rk[4 * r + 3];
+        s0 = t0; s1 = t1; s2 = t2; s3 = t3;
+    }
+#define SB(x) ((T(tl, (x)) >> 8) & 255u)
+    uint4 o;
+    o.x = (SB(s0 >> 24) << 24 | SB((s1 >> 16) & 255) << 16 | SB((s2 >> 8) & 255) << 8 | SB(s3 & 255)) ^ rk[40];
+    o.y = (SB(s1 >> 24) << 24 | SB((s2 >> 16) & 255) << 16 | SB((s3 >> 8) & 255) << 8 | SB(s0 & 255)) ^ rk[41];
+    o.z = (SB(s2 >> 24) << 24 | SB((s3 >> 16) & 255) << 16 | SB((s0 >> 8) & 255) << 8 | SB(s1 & 255)) ^ rk[42];
+    o.w = (SB(s3 >> 24) << 24 | SB((s0 >> 16) & 255) << 16 | SB((s1 >> 8) & 255) << 8 | SB(s2 & 255)) ^ rk[43];
+#undef SB
+    return o;
+}
+
 __device__ __forceinline__ uint32_t rotl(uint32_t x, int n) { return __funnelshift_l(x, x, n); }
 
 __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16])
@@ -1190,18 +1228,26 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16])
 // the L4 bytes are encrypted where they lie, trailer and ICV are appended.
 // Returns the new frame length.  Stream bytes are handled as 32-bit words; memory
 // words are 4-B aligned and related to stream words by a funnel shift of r = A & 3.
-__device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t seq, const uint32_t *te)
+__device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t seq, const uint32_t *te,
+                                           const uint32_t *rk_smem)
 {
     const uint32_t l4 = v.l4_off, plen = v.ip_end - l4;
+#if NFC_ESP_PF
+    for (uint32_t o = 128; o < v.ip_end; o += 128) prefetch_l2(f + o);
+#endif
     const uint32_t p = (4 - ((plen + 2) & 3)) & 3;
     const uint32_t clen = plen + p + 2;          // multiple of 4
     const uint32_t nK = clen >> 2;
+#if NFC_ESP_RK_SMEM
+    const uint32_t *rks = rk_smem;
+#else
     uint32_t rk[44];
     {
         const uint4 *q = reinterpret_cast<const uint4 *>(sap->rk);
 #pragma unroll
         for (int i = 0; i < 11; i++) { uint4 x = __ldg(q + i); rk[4 * i] = x.x; rk[4 * i + 1] = x.y; rk[4 * i + 2] = x.z; rk[4 * i + 3] = x.w; }
     }
+#endif
     const uint32_t spi = __ldg(&sap->spi), nonce = __ldg(&sap->nonce);
     // 1. move the header 16 B left and fix up the IP header
     {
@@ -1261,9 +1307,14 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
             } else if (i < nmsg) {
                 const uint32_t k = i - 4;                 // stream word
                 if ((w & 3) == 0) {                       // new AES counter block every 4 words
+#if NFC_ESP_RK_SMEM
+                    const uint4 o = aes128_encrypt_s(te, rks, nonce, 0u, seq, (k >> 2) + 1);
+                    ks[0] = bswap32(o.x); ks[1] = bswap32(o.y); ks[2] = bswap32(o.z); ks[3] = bswap32(o.w);
+#else
                     uint32_t o[4];
                     aes128_encrypt(te, rk, nonce, 0u, seq, (k >> 2) + 1, o);
                     ks[0] = bswap32(o[0]); ks[1] = bswap32(o[1]); ks[2] = bswap32(o[2]); ks[3] = bswap32(o[3]);
+#endif
                 }
                 uint32_t Mnext = W0[k + 1];
                 uint32_t P = __funnelshift_rc(Mcur, Mnext, 8 * r);   // stream bytes 4k..4k+3 (LE)
@@ -1761,7 +1812,8 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
             k.port = pt;
         }
     } else if constexpr (KIND == NFC_IPSEC) {
-        const uint32_t nl = nf_esp(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te);
+        const uint32_t nl = nf_esp(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te,
+                                   reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.rk) + k.esp_sa * ESP_RK_STRIDE);
         k.esp_bytes = nl - 28 - k.v.l4_off;      // ciphertext bytes |C|
         k.f -= 16;
         k.flen = nl;
@@ -2098,6 +2150,10 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         for (uint32_t i = tid; i < 72 * 16; i += NT) mn[i] = __ldg(P.esp.rss_nib + i);
         C.te = te + lane;         // this lane's bank column
         C.ms_nib = mn;
+#if NFC_ESP_RK_SMEM
+        uint32_t *rk = reinterpret_cast<uint32_t *>(smem + L.rk);
+        for (uint32_t i = tid; i < P.esp.n_sa * 44; i += NT) rk[(i / 44) * ESP_RK_STRIDE + i % 44] = __ldg(P.esp.sa[i / 44].rk + i % 44);
+#endif
     }
     if ((SMASK & MASK_LPM4) && (mask & MASK_LPM4) && P.l4.nh_smem) {
         uint4 *r = reinterpret_cast<uint4 *>(smem + L.nh4);
