@@ -93,6 +93,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_ESP_RK_SMEM
 #define NFC_ESP_RK_SMEM 1     // ESP reads AES round keys from shared memory (one out-of-line block cipher; C2 +11 %)
 #endif
+#ifndef NFC_SPEC_V6
+#define NFC_SPEC_V6 0         // 1: dual-stack warps take the speculative block (IPv6 lanes re-classified)
+#endif
 #ifndef NFC_HOT_FAST
 #define NFC_HOT_FAST 0        // 1: DM_HOT split walk takes the unconditional 16-byte step too
 #endif
@@ -1877,7 +1880,9 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
     if constexpr (NFC_SPEC && HEAD && S != SIG_ANY && DM == DM_FULL && sig_n(S) >= 2 && sig_kind(S, 0) == NFC_ACL &&
                   sig_kind(S, 1) == NFC_DPI) {
         // speculative ACL || DPI head walk || TBL24 (see spec_ok), warp-uniform choice
-        const bool v4 = !k.alive || (k.v.fam == 4 && k.v.pl_off >= 42);   // payload starts inside [42, 64) or later
+        // every payload starts at byte 42 or later; IPv6 lanes (dual-stack traffic) take the
+        // IPv4 classification speculatively too and are re-classified below
+        const bool v4 = !k.alive || ((k.v.fam == 4 || NFC_SPEC_V6) && k.v.pl_off >= 42);
         if (spec_ok<S>(P) && __all_sync(0xFFFFFFFFu, v4)) {
             constexpr bool T24 = sig_pos(S, NFC_LPM4) != 0xFF &&
                                  (sig_pos(S, NFC_IPSEC) == 0xFF || sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4));
@@ -1896,6 +1901,7 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
                 wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
                 if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
             }
+            if (NFC_SPEC_V6 && k.alive && k.v.fam != 4) r = nf_acl_fused(P, k.v);   // IPv6 lanes
             if (k.alive) {                     // ACL effects (position 0)
                 const uint32_t rule = r & 0xFFFF;
                 k.acl_rule = rule;
