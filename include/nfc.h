@@ -277,6 +277,46 @@ NFC_API int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uin
  * NULL pointers, n outside 1..6 or an unknown kind. */
 NFC_API int nfc_plan_parallel(const uint32_t *kinds, uint32_t n, uint8_t *group);
 
+/* ---------------------------------------------------------------- stateful DPI
+ * stateful, cross-packet DPI (PAPER.md P:L161 [SIII.B.b]
+ * "in-order processing of packet in the same connection ... resembled as traffic
+ * stream"; P:L132 [SIII.A.2] Aho-Corasick for string matching; R#32).
+ * A flow is the exact (family, proto, src, dst, sport, dport) of a frame that
+ * parses under R#24 (ports 0 for fragments and non-TCP/UDP).  The payloads
+ * [pl_off, ip_end) of a flow's packets, in global order (calls in order, packets
+ * of a call in index order), form one byte stream; every occurrence of a pattern
+ * in that stream (case-sensitive, overlapping) is reported against the packet
+ * holding its LAST byte.  Flow state (the Aho-Corasick DFA state) persists in a
+ * device flow table across calls until nfc_dpi_stream_reset.  Standalone NF: it
+ * is not part of a fused chain. */
+typedef struct nfc_dpi_stream nfc_dpi_stream; /* opaque; owned by the library */
+
+typedef struct {
+    uint32_t *nocc;              /* device; n: occurrences ending in packet i (0 if not inspected) */
+    uint8_t *drop;               /* device; n: 1 iff a DROP pattern occurrence ends in packet i   */
+    uint32_t *occ_pkt;           /* device; occurrence: packet global index                     */
+    uint16_t *occ_pat;           /* device; occurrence: pattern id                              */
+    uint16_t *occ_end;           /* device; occurrence: offset of its last byte in the payload  */
+    uint32_t occ_cap;            /* capacity of occ_*; occurrences beyond it are counted only   */
+    uint32_t reserved;
+    uint32_t *occ_count;         /* device u32, incremented atomically; caller zeroes it        */
+} nfc_stream_result;
+
+/* Builds the Aho-Corasick DFA of `spec` (NFC_EINVAL as nfc_load_tables for a
+ * malformed spec) and a device flow table of the next power of two >= 2 x
+ * max_flows slots (1..2^28) on `device`.  NFC_ENOMEM / NFC_ECUDA on failure. */
+NFC_API int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flows, nfc_dpi_stream **out);
+NFC_API int nfc_dpi_stream_destroy(nfc_dpi_stream *s);
+/* Forgets every flow (asynchronous on `stream`). */
+NFC_API int nfc_dpi_stream_reset(nfc_dpi_stream *s, void *stream);
+/* Inspects one batch (frames are only read) asynchronously on `stream`; results are
+ * valid after the stream syncs.  Occurrences are appended in unspecified order.  A
+ * packet of a new flow that finds the flow table full is not inspected (counted by
+ * nfc_dpi_stream_flows).  Calls on one object must be ordered on one stream. */
+NFC_API int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stream_result *r, void *stream);
+/* Synchronizes the device; flows in the table and packets not placed (table full). */
+NFC_API int nfc_dpi_stream_flows(nfc_dpi_stream *s, uint64_t *n_flows, uint64_t *n_unplaced);
+
 /* Number of kernel launches the library issued on this chain so far. */
 NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 

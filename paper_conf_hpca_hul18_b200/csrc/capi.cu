@@ -21,6 +21,8 @@ static int fail(int code, const std::string &msg)
     return code;
 }
 
+int nfc::set_fail(int code, const std::string &msg) { return fail(code, msg); }
+
 #define CK(call)                                                                                   \
     do {                                                                                           \
         cudaError_t e_ = (call);                                                                   \

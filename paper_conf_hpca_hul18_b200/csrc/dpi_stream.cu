@@ -1,0 +1,349 @@
+// dpi_stream.cu -- stateful (cross-packet) DPI, SURVEY 8(f) NEXT-4 (include/nfc.h
+// "Stateful DPI"; PAPER.md P:L161 [SIII.B.b] in-order processing of the packets of
+// a connection, P:L132 [SIII.A.2] Aho-Corasick DPI; R#32, section 16).
+//
+// Three launches per call, all on the caller's stream:
+//   k_flow  -- one thread per packet: R#24 parse, flow key -> slot of a device
+//              open-addressing flow table (lock-free insert), payload span;
+//   cub radix sort of (slot, packet index) pairs (stable: a flow's packets stay
+//              in index order, i.e. stream order);
+//   k_walk  -- one thread per flow present in the batch: starts from the flow's
+//              carried DFA state, walks its packets' payloads in order through the
+//              Aho-Corasick DFA (the same image builders.cpp makes for the fused
+//              kernel), appends every occurrence, stores the state back.
+// The flow table and the per-flow DFA states persist across calls.
+#include <cuda_runtime.h>
+#include <cub/device/device_radix_sort.cuh>
+
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "nfc_internal.h"
+
+using namespace nfc;
+
+namespace {
+
+constexpr uint32_t KW = 10;   // key words: src[4], dst[4], sport<<16|dport, proto | family<<8
+
+struct StreamDfa {
+    const uint8_t *cls;
+    const void *trans;
+    const uint32_t *out_off;
+    const uint16_t *out_ids;
+    const uint8_t *action;
+    uint32_t ncls, wide;
+};
+
+__device__ __forceinline__ uint32_t be16d(const uint8_t *p) { return (uint32_t)p[0] << 8 | p[1]; }
+
+// R#24 parse: returns false if the frame is not inspected; key[KW], payload [a, b)
+__device__ bool parse_flow(const uint8_t *f, uint32_t flen, uint32_t key[KW], uint32_t &a, uint32_t &b)
+{
+    if (flen < 14) return false;
+    const uint32_t et = be16d(f + 12);
+    uint32_t l4, ip_end, proto, fam;
+    bool frag = false;
+    for (int k = 0; k < (int)KW; k++) key[k] = 0;
+    if (et == 0x0800) {
+        if (flen < 34 || (f[14] >> 4) != 4) return false;
+        const uint32_t ihl = f[14] & 15, tot = be16d(f + 16);
+        if (ihl < 5 || tot < 4 * ihl || 14 + tot > flen) return false;
+        fam = 4; l4 = 14 + 4 * ihl; ip_end = 14 + tot; proto = f[23];
+        key[0] = (uint32_t)f[26] << 24 | (uint32_t)f[27] << 16 | (uint32_t)f[28] << 8 | f[29];
+        key[4] = (uint32_t)f[30] << 24 | (uint32_t)f[31] << 16 | (uint32_t)f[32] << 8 | f[33];
+        const uint32_t fo = be16d(f + 20);
+        frag = (fo & 0x3FFF) != 0;
+    } else if (et == 0x86DD) {
+        if (flen < 54 || (f[14] >> 4) != 6) return false;
+        const uint32_t pl = be16d(f + 18);
+        if (54 + pl > flen) return false;
+        fam = 6; l4 = 54; ip_end = 54 + pl; proto = f[20];
+        for (int w = 0; w < 4; w++) {
+            const uint8_t *s = f + 22 + 4 * w, *d = f + 38 + 4 * w;
+            key[w] = (uint32_t)s[0] << 24 | (uint32_t)s[1] << 16 | (uint32_t)s[2] << 8 | s[3];
+            key[4 + w] = (uint32_t)d[0] << 24 | (uint32_t)d[1] << 16 | (uint32_t)d[2] << 8 | d[3];
+        }
+    } else {
+        return false;
+    }
+    uint32_t hl = 0;
+    if (!frag && proto == 17) {
+        if (l4 + 8 > ip_end) return false;
+        hl = 8;
+    } else if (!frag && proto == 6) {
+        if (l4 + 20 > ip_end) return false;
+        const uint32_t doff = f[l4 + 12] >> 4;
+        if (doff < 5 || l4 + 4 * doff > ip_end) return false;
+        hl = 4 * doff;
+    }
+    if (hl) key[8] = be16d(f + l4) << 16 | be16d(f + l4 + 2);
+    key[9] = proto | fam << 8 | 1u << 16;          // bit 16: never an all-zero key
+    a = l4 + hl;
+    b = ip_end;
+    return true;
+}
+
+__device__ __forceinline__ uint32_t key_hash(const uint32_t key[KW])
+{
+    uint32_t h = 0x9E3779B9u;
+    for (int k = 0; k < (int)KW; k++) {
+        uint32_t x = key[k] * 0xCC9E2D51u;
+        x = (x << 15) | (x >> 17);
+        h ^= x * 0x1B873593u;
+        h = ((h << 13) | (h >> 19)) * 5u + 0xE6546B64u;
+    }
+    h ^= h >> 16; h *= 0x85EBCA6Bu; h ^= h >> 13; h *= 0xC2B2AE35u; h ^= h >> 16;
+    return h;
+}
+
+// Flow table slot of `key` (inserted if new); 0xFFFFFFFF if the table is full.
+// lock[s]: 0 empty, 1 key being written, 2 key published.
+__device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t *n_flows,
+                              const uint32_t key[KW])
+{
+    uint32_t s = key_hash(key) & mask;
+    for (uint32_t probe = 0; probe <= mask; probe++, s = (s + 1) & mask) {
+        uint32_t l = atomicCAS(&lock[s], 0u, 1u);
+        if (l == 0) {
+            for (int k = 0; k < (int)KW; k++) keys[(size_t)s * KW + k] = key[k];
+            __threadfence();
+            atomicExch(&lock[s], 2u);
+            atomicAdd(n_flows, 1u);
+            return s;
+        }
+        while (l == 1) l = *(volatile uint32_t *)&lock[s];
+        __threadfence();
+        bool eq = true;
+        for (int k = 0; k < (int)KW; k++) eq &= __ldcg(&keys[(size_t)s * KW + k]) == key[k];
+        if (eq) return s;
+    }
+    return 0xFFFFFFFFu;
+}
+
+__global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t none,
+                       uint32_t *ctr, uint32_t *fkey, uint32_t *fidx, uint32_t *span,
+                       uint32_t *nocc, uint8_t *drop)
+{
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= b.n) return;
+    nocc[i] = 0;
+    drop[i] = 0;
+    fidx[i] = i;
+    uint32_t key[KW], a, e;
+    uint32_t slot = none;
+    if (parse_flow(b.arena + b.off[i], b.len[i], key, a, e)) {
+        slot = flow_slot(lock, keys, mask, &ctr[0], key);
+        if (slot == 0xFFFFFFFFu) { atomicAdd(&ctr[1], 1u); slot = none; }
+        span[i] = a | e << 16;
+    }
+    fkey[i] = slot;
+}
+
+template <bool WIDE>
+__global__ void __launch_bounds__(128) k_walk(nfc_batch b, StreamDfa d, uint32_t none, const uint32_t *fkey,
+                                              const uint32_t *fidx, const uint32_t *span, uint32_t *fstate,
+                                              nfc_stream_result r)
+{
+    __shared__ uint8_t cls[256];
+    for (int k = threadIdx.x; k < 256; k += blockDim.x) cls[k] = d.cls[k];
+    __syncthreads();
+    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= b.n) return;
+    const uint32_t f = fkey[t];
+    if (f == none || (t > 0 && fkey[t - 1] == f)) return;   // not inspected / not the flow's first packet
+    uint32_t s = fstate[f];
+    const uint32_t first = (uint32_t)b.first_global_index;
+    for (uint32_t u = t; u < b.n && fkey[u] == f; u++) {
+        const uint32_t i = fidx[u], sp = span[i], a = sp & 0xFFFF, e = sp >> 16;
+        const uint8_t *p = b.arena + b.off[i];
+        uint32_t cnt = 0, dr = 0;
+        for (uint32_t x = a; x < e; x++) {
+            const size_t at = (size_t)s * d.ncls + cls[p[x]];
+            uint32_t nx;
+            bool acc;
+            if (WIDE) { nx = __ldg((const uint32_t *)d.trans + at); acc = nx >> 31; s = nx & 0x7FFFFFFFu; }
+            else      { nx = __ldg((const uint16_t *)d.trans + at); acc = nx >> 15; s = nx & 0x7FFFu; }
+            if (acc) {
+                const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
+                for (uint32_t k = o0; k < o1; k++) {
+                    const uint32_t pat = __ldg(d.out_ids + k);
+                    const uint32_t w = atomicAdd(r.occ_count, 1u);
+                    if (w < r.occ_cap) {
+                        r.occ_pkt[w] = first + i;
+                        r.occ_pat[w] = (uint16_t)pat;
+                        r.occ_end[w] = (uint16_t)(x - a);
+                    }
+                    dr |= __ldg(d.action + pat);
+                }
+                cnt += o1 - o0;
+            }
+        }
+        r.nocc[i] = cnt;
+        r.drop[i] = (uint8_t)dr;
+    }
+    fstate[f] = s;
+}
+
+}  // namespace
+
+struct nfc_dpi_stream {
+    int device = 0;
+    uint32_t n_slots = 0, mask = 0, key_bits = 0;
+    uint32_t *lock = nullptr, *keys = nullptr, *fstate = nullptr, *ctr = nullptr;
+    // DFA (device)
+    uint8_t *cls = nullptr, *trans = nullptr, *action = nullptr;
+    uint32_t *out_off = nullptr;
+    uint16_t *out_ids = nullptr;
+    uint32_t ncls = 0, wide = 0, n_states = 0;
+    // per-call scratch
+    uint32_t cap_pkts = 0;
+    uint32_t *fkey = nullptr, *fkey2 = nullptr, *fidx = nullptr, *fidx2 = nullptr, *span = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0;
+    uint64_t launches = 0;
+};
+
+#define SCK(call)                                                                                  \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) return set_fail(NFC_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+    } while (0)
+
+template <class T>
+static cudaError_t dev_copy(T **dst, const T *src, size_t n)
+{
+    cudaError_t e = cudaMalloc((void **)dst, std::max<size_t>(1, n) * sizeof(T));
+    if (e != cudaSuccess) return e;
+    return n ? cudaMemcpy(*dst, src, n * sizeof(T), cudaMemcpyHostToDevice) : cudaSuccess;
+}
+
+static void free_scratch(nfc_dpi_stream *s)
+{
+    cudaFree(s->fkey); cudaFree(s->fkey2); cudaFree(s->fidx); cudaFree(s->fidx2); cudaFree(s->span);
+    cudaFree(s->tmp);
+    s->fkey = s->fkey2 = s->fidx = s->fidx2 = s->span = nullptr;
+    s->tmp = nullptr;
+    s->cap_pkts = 0;
+    s->tmp_bytes = 0;
+}
+
+int nfc_dpi_stream_destroy(nfc_dpi_stream *s)
+{
+    if (!s) return NFC_OK;
+    cudaSetDevice(s->device);
+    free_scratch(s);
+    cudaFree(s->lock); cudaFree(s->keys); cudaFree(s->fstate); cudaFree(s->ctr);
+    cudaFree(s->cls); cudaFree(s->trans); cudaFree(s->action); cudaFree(s->out_off); cudaFree(s->out_ids);
+    delete s;
+    return NFC_OK;
+}
+
+int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flows, nfc_dpi_stream **out)
+{
+    if (!spec || !out) return set_fail(NFC_EINVAL, "dpi_stream_create: NULL pointer");
+    if (max_flows == 0 || max_flows > (1u << 28)) return set_fail(NFC_EINVAL, "dpi_stream_create: max_flows must be 1..2^28");
+    *out = nullptr;
+    DpiHost h;
+    std::string e = build_dpi(*spec, h);
+    if (!e.empty()) return set_fail(NFC_EINVAL, e);
+    SCK(cudaSetDevice(device));
+    nfc_dpi_stream *s = new nfc_dpi_stream;
+    s->device = device;
+    uint32_t lg = 1;
+    while ((1u << lg) < 2 * max_flows) lg++;           // load factor <= 1/2
+    s->n_slots = 1u << lg;
+    s->mask = s->n_slots - 1;
+    s->key_bits = lg + 1;                              // slot ids and the "none" key n_slots
+    s->ncls = h.ncls;
+    s->wide = h.wide;
+    s->n_states = h.n_states;
+    cudaError_t ce = cudaSuccess;
+    auto ok = [&](cudaError_t x) { if (ce == cudaSuccess) ce = x; };
+    ok(cudaMalloc((void **)&s->lock, (size_t)s->n_slots * 4));
+    ok(cudaMalloc((void **)&s->keys, (size_t)s->n_slots * KW * 4));
+    ok(cudaMalloc((void **)&s->fstate, (size_t)s->n_slots * 4));
+    ok(cudaMalloc((void **)&s->ctr, 4 * 4));
+    ok(dev_copy(&s->cls, h.cls.data(), h.cls.size()));
+    ok(dev_copy(&s->trans, h.trans.data(), h.trans.size()));
+    ok(dev_copy(&s->action, h.action.data(), h.action.size()));
+    ok(dev_copy(&s->out_off, h.out_off.data(), h.out_off.size()));
+    ok(dev_copy(&s->out_ids, h.out_ids.data(), h.out_ids.size()));
+    if (ce == cudaSuccess) {
+        ok(cudaMemset(s->lock, 0, (size_t)s->n_slots * 4));
+        ok(cudaMemset(s->fstate, 0, (size_t)s->n_slots * 4));
+        ok(cudaMemset(s->ctr, 0, 16));
+        ok(cudaDeviceSynchronize());
+    }
+    if (ce != cudaSuccess) {
+        nfc_dpi_stream_destroy(s);
+        return set_fail(ce == cudaErrorMemoryAllocation ? NFC_ENOMEM : NFC_ECUDA,
+                        std::string("dpi_stream_create: ") + cudaGetErrorString(ce));
+    }
+    *out = s;
+    return NFC_OK;
+}
+
+int nfc_dpi_stream_reset(nfc_dpi_stream *s, void *stream)
+{
+    if (!s) return set_fail(NFC_EINVAL, "dpi_stream_reset: NULL stream object");
+    SCK(cudaSetDevice(s->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    SCK(cudaMemsetAsync(s->lock, 0, (size_t)s->n_slots * 4, st));
+    SCK(cudaMemsetAsync(s->fstate, 0, (size_t)s->n_slots * 4, st));
+    SCK(cudaMemsetAsync(s->ctr, 0, 16, st));
+    return NFC_OK;
+}
+
+int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stream_result *r, void *stream)
+{
+    if (!s || !b || !r) return set_fail(NFC_EINVAL, "dpi_stream_process: NULL pointer");
+    if (b->n == 0) return NFC_OK;
+    if (!b->arena || !b->off || !b->len || !r->nocc || !r->drop || !r->occ_count ||
+        (r->occ_cap && (!r->occ_pkt || !r->occ_pat || !r->occ_end)))
+        return set_fail(NFC_EINVAL, "dpi_stream_process: NULL device buffer");
+    SCK(cudaSetDevice(s->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    if (b->n > s->cap_pkts) {
+        SCK(cudaStreamSynchronize(st));
+        free_scratch(s);
+        const size_t n = b->n;
+        SCK(cudaMalloc((void **)&s->fkey, n * 4));
+        SCK(cudaMalloc((void **)&s->fkey2, n * 4));
+        SCK(cudaMalloc((void **)&s->fidx, n * 4));
+        SCK(cudaMalloc((void **)&s->fidx2, n * 4));
+        SCK(cudaMalloc((void **)&s->span, n * 4));
+        SCK(cub::DeviceRadixSort::SortPairs(nullptr, s->tmp_bytes, s->fkey, s->fkey2, s->fidx, s->fidx2,
+                                            (int)n, 0, (int)s->key_bits, st));
+        SCK(cudaMalloc(&s->tmp, std::max<size_t>(16, s->tmp_bytes)));
+        s->cap_pkts = b->n;
+    }
+    const uint32_t none = s->n_slots;
+    const uint32_t blocks = (b->n + 255) / 256;
+    k_flow<<<blocks, 256, 0, st>>>(*b, s->lock, s->keys, s->mask, none, s->ctr, s->fkey, s->fidx, s->span,
+                                   r->nocc, r->drop);
+    SCK(cudaGetLastError());
+    size_t tb = s->tmp_bytes;
+    SCK(cub::DeviceRadixSort::SortPairs(s->tmp, tb, s->fkey, s->fkey2, s->fidx, s->fidx2, (int)b->n, 0,
+                                        (int)s->key_bits, st));
+    StreamDfa d{s->cls, s->trans, s->out_off, s->out_ids, s->action, s->ncls, s->wide};
+    const uint32_t wb = (b->n + 127) / 128;
+    if (s->wide) k_walk<true><<<wb, 128, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, *r);
+    else         k_walk<false><<<wb, 128, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, *r);
+    SCK(cudaGetLastError());
+    s->launches += 2;   // k_flow + k_walk (the cub sort launches its own kernels)
+    return NFC_OK;
+}
+
+int nfc_dpi_stream_flows(nfc_dpi_stream *s, uint64_t *n_flows, uint64_t *n_unplaced)
+{
+    if (!s || !n_flows || !n_unplaced) return set_fail(NFC_EINVAL, "dpi_stream_flows: NULL pointer");
+    SCK(cudaSetDevice(s->device));
+    SCK(cudaDeviceSynchronize());
+    uint32_t c[4];
+    SCK(cudaMemcpy(c, s->ctr, 16, cudaMemcpyDeviceToHost));
+    *n_flows = c[0];
+    *n_unplaced = c[1];
+    return NFC_OK;
+}

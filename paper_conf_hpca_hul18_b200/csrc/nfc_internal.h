@@ -216,6 +216,7 @@ struct KParams {
 };
 
 // host-side builders (builders.cpp); return "" on success or an error message
+int set_fail(int code, const std::string &msg);   // capi.cu: nfc_last_error + code
 struct HostImage { std::vector<uint8_t> bytes; };
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
 struct DpiHost {

@@ -76,6 +76,11 @@ class Batch(ctypes.Structure):
                 ("first_global_index", ctypes.c_uint64)]
 
 
+class StreamResult(ctypes.Structure):
+    _fields_ = [("nocc", _P), ("drop", _P), ("occ_pkt", _P), ("occ_pat", _P), ("occ_end", _P),
+                ("occ_cap", _u32), ("reserved", _u32), ("occ_count", _P)]
+
+
 class Result(ctypes.Structure):
     _fields_ = [("rec", _P), ("match_pkt", _P), ("match_pat", _P), ("match_cap", _u32),
                 ("reserved", _u32), ("match_count", _P)]
@@ -83,7 +88,9 @@ class Result(ctypes.Structure):
 
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
-           "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard"]
+           "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard",
+           "nfc_dpi_stream_create", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
+           "nfc_dpi_stream_process", "nfc_dpi_stream_flows"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
@@ -109,6 +116,11 @@ def _load_lib():
     L.nfc_last_launch.argtypes = [_P, _P]
     L.nfc_plan_parallel.argtypes = [_P, _u32, _P]
     L.nfc_rss_shard.argtypes = [ctypes.c_int, ctypes.POINTER(Batch), _u32, _P, _P]
+    L.nfc_dpi_stream_create.argtypes = [ctypes.c_int, ctypes.POINTER(DpiSpec), _u32, ctypes.POINTER(_P)]
+    L.nfc_dpi_stream_destroy.argtypes = [_P]
+    L.nfc_dpi_stream_reset.argtypes = [_P, _P]
+    L.nfc_dpi_stream_process.argtypes = [_P, ctypes.POINTER(Batch), ctypes.POINTER(StreamResult), _P]
+    L.nfc_dpi_stream_flows.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
     P32 = ctypes.POINTER(_u32)
@@ -308,6 +320,58 @@ def plan_parallel(kinds) -> list:
     g = np.zeros(max(1, len(k)), dtype=np.uint8)
     _check(lib.nfc_plan_parallel(k.ctypes.data, len(k), g.ctypes.data))
     return [int(x) for x in g[:len(k)]]
+
+
+class DpiStream:
+    """Stateful cross-packet DPI (include/nfc.h "stateful DPI", NEXT-4, R#32) on one device.
+
+    Argument marshalling only: every step runs in dpi_stream.cu."""
+
+    def __init__(self, blob: np.ndarray, off: np.ndarray, action: np.ndarray, max_flows: int, device: int = 0):
+        b, o, a = _np(blob, np.uint8), _np(off, np.uint32), _np(action, np.uint8)
+        h = _P()
+        _check(lib.nfc_dpi_stream_create(device, ctypes.byref(DpiSpec(len(a), b.ctypes.data, o.ctypes.data,
+                                                                      a.ctypes.data)), max_flows, ctypes.byref(h)))
+        self.h = h
+        self.device = device
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.nfc_dpi_stream_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def reset(self, stream: int = 0):
+        return _check(lib.nfc_dpi_stream_reset(self.h, stream or None))
+
+    def process(self, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, first_global_index: int,
+                nocc_ptr: int, drop_ptr: int, occ_pkt_ptr: int, occ_pat_ptr: int, occ_end_ptr: int,
+                occ_cap: int, occ_count_ptr: int, stream: int = 0):
+        b = Batch(arena_ptr, off_ptr, len_ptr, n, 0, first_global_index)
+        r = StreamResult(nocc_ptr, drop_ptr, occ_pkt_ptr or None, occ_pat_ptr or None, occ_end_ptr or None,
+                         occ_cap, 0, occ_count_ptr)
+        return _check(lib.nfc_dpi_stream_process(self.h, ctypes.byref(b), ctypes.byref(r), stream or None))
+
+    def process_tensors(self, arena, off, ln, nocc, drop, occ_pkt, occ_pat, occ_end, occ_count,
+                        first_global_index: int = 0, stream=None):
+        """torch CUDA tensors: arena u8, off int64, len int16, nocc int32[n], drop u8[n],
+        occ_pkt int32[cap], occ_pat int16[cap], occ_end int16[cap], occ_count int32[1] (zeroed)."""
+        import torch
+        s = stream if stream is not None else torch.cuda.current_stream(arena.device)
+        return self.process(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), int(off.numel()),
+                            first_global_index, nocc.data_ptr(), drop.data_ptr(), occ_pkt.data_ptr(),
+                            occ_pat.data_ptr(), occ_end.data_ptr(), int(occ_pkt.numel()),
+                            occ_count.data_ptr(), s.cuda_stream)
+
+    def flows(self):
+        nf, nu = ctypes.c_uint64(), ctypes.c_uint64()
+        _check(lib.nfc_dpi_stream_flows(self.h, ctypes.byref(nf), ctypes.byref(nu)))
+        return nf.value, nu.value
 
 
 def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,

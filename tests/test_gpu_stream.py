@@ -1,0 +1,159 @@
+"""GPU parity of stateful cross-packet DPI (NEXT-4, R#32): nfc_dpi_stream_* through
+the C ABI against oracle/stream_dpi.py on the same seeded S1 traffic.  Integer
+work: the sorted occurrence list (packet, pattern, end offset), per-packet counts
+and DROP verdicts must be identical."""
+import numpy as np
+import pytest
+
+import nfcgen
+from nfcgen.stream import StreamBatch, stream_batch
+from oracle.stream_dpi import StreamDPI
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def nfc():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_hpca_hul18_b200 import build
+    build.build()
+    from paper_conf_hpca_hul18_b200 import nfc as m
+    return m
+
+
+def _pats(seed, n, lmin=2, lmax=8):
+    rng = np.random.default_rng(seed)
+    blob, off, act = nfcgen.gen_patterns(rng, n, lmin=lmin, lmax=lmax, drop_frac=0.1)
+    return blob, off, act, nfcgen.Tables(pat_blob=blob, pat_off=off, pat_action=act).patterns()
+
+
+def _gpu(ds, sb: StreamBatch, cap=1 << 20):
+    import torch
+    d = torch.device("cuda:0")
+    arena = torch.from_numpy(sb.arena).to(d)
+    off = torch.from_numpy(sb.off.astype(np.int64)).to(d)
+    ln = torch.from_numpy(sb.len.view(np.int16)).to(d)
+    n = len(sb.off)
+    nocc = torch.full((n,), 0x7777, dtype=torch.int32, device=d)
+    drop = torch.full((n,), 7, dtype=torch.uint8, device=d)
+    op = torch.zeros(cap, dtype=torch.int32, device=d)
+    oq = torch.zeros(cap, dtype=torch.int16, device=d)
+    oe = torch.zeros(cap, dtype=torch.int16, device=d)
+    cnt = torch.zeros(1, dtype=torch.int32, device=d)
+    ds.process_tensors(arena, off, ln, nocc, drop, op, oq, oe, cnt, first_global_index=sb.first_index)
+    torch.cuda.synchronize()
+    k = int(cnt.item())
+    m = min(k, cap)
+    occ = sorted(zip(op[:m].cpu().numpy().view(np.uint32).tolist(), oq[:m].cpu().numpy().view(np.uint16).tolist(),
+                     oe[:m].cpu().numpy().view(np.uint16).tolist()))
+    return occ, nocc.cpu().numpy().tolist(), drop.cpu().numpy().tolist(), k
+
+
+def test_stream_parity_multi_call(nfc):
+    blob, off, act, pats = _pats(1, 100)
+    ds = nfc.DpiStream(blob, off, act, max_flows=4096)
+    orc = StreamDPI(pats, list(act))
+    first = 0
+    total_cross = 0
+    for call, n in enumerate([3000, 1, 2500, 4097]):
+        sb = stream_batch(100 + call, n, 60, pats, len_choices=[64, 65, 128, 300, 1500], plant_frac=0.3,
+                          first_index=first, flow_seed=42)
+        want, wn, wd = orc.process(sb.frames(), first)
+        got, gn, gd, k = _gpu(ds, sb)
+        assert k == len(want)
+        assert got == want
+        assert gn == wn and gd == wd
+        total_cross += sum(1 for i, j, e in want if e < len(pats[j]) - 1)
+        first += n
+    assert total_cross > 100
+    assert ds.flows() == (orc.n_flows(), 0)
+    # reset forgets every flow: the next call starts each stream afresh
+    ds.reset()
+    orc2 = StreamDPI(pats, list(act))
+    sb = stream_batch(7, 2000, 60, pats, plant_frac=0.3, first_index=first, flow_seed=42)
+    want, wn, wd = orc2.process(sb.frames(), first)
+    got, gn, gd, _ = _gpu(ds, sb)
+    assert got == want and gn == wn and gd == wd
+
+
+def test_stream_parity_wide_dfa(nfc):
+    """> 32768 DFA states: 32-bit transition entries."""
+    blob, off, act, pats = _pats(2, 2600, lmin=12, lmax=16)
+    ds = nfc.DpiStream(blob, off, act, max_flows=64)
+    orc = StreamDPI(pats, list(act))
+    sb = stream_batch(3, 400, 20, pats, len_choices=[64, 200], plant_frac=0.5)
+    want, wn, wd = orc.process(sb.frames())
+    got, gn, gd, _ = _gpu(ds, sb)
+    assert len(want) > 20
+    assert got == want and gn == wn and gd == wd
+
+
+def _frame_batch(frames, first=0):
+    offs, pos = [], 0
+    for f in frames:
+        offs.append(pos)
+        pos += (len(f) + 15) // 16 * 16
+    arena = np.zeros(pos + 16, dtype=np.uint8)
+    for o, f in zip(offs, frames):
+        arena[o:o + len(f)] = np.frombuffer(f, dtype=np.uint8)
+    return StreamBatch(arena, np.array(offs, dtype=np.uint64), np.array([len(f) for f in frames], dtype=np.uint16),
+                       first)
+
+
+def test_stream_edge_frames(nfc):
+    """IPv6, fragments, TCP options, non-parsing frames, empty payloads, capacity overflow."""
+    from tests.test_oracle_stream import _udp
+    pats = [b"ab", b"abc", b"b", b"cab"]
+    act = [0, 1, 0, 0]
+    blob = np.frombuffer(b"".join(pats), dtype=np.uint8)
+    off = np.cumsum([0] + [len(p) for p in pats]).astype(np.uint32)
+
+    def v6(payload, sport=5):
+        l4 = sport.to_bytes(2, "big") + b"\x00\x35" + (8 + len(payload)).to_bytes(2, "big") + b"\0\0"
+        ip = bytes([0x60, 0, 0, 0]) + (8 + len(payload)).to_bytes(2, "big") + bytes([17, 64]) + \
+            bytes(range(16)) + bytes(range(16, 32))
+        return bytes(12) + b"\x86\xdd" + ip + l4 + payload
+
+    frames = [_udp(b"xxa"), v6(b"ca"), _udp(b"bcab"), v6(b"b"), _udp(b"", sport=9), _udp(b"ab", frag=0x2001),
+              _udp(b"b", frag=0x2001), b"\x00" * 20, _udp(b"a", proto=6), _udp(b"bc", proto=6), v6(b"ab" * 40)]
+    sb = _frame_batch(frames, first=5)
+    ds = nfc.DpiStream(blob, off, np.array(act, dtype=np.uint8), max_flows=16)
+    want, wn, wd = StreamDPI(pats, act).process(sb.frames(), 5)
+    got, gn, gd, k = _gpu(ds, sb)
+    assert got == want and gn == wn and gd == wd
+    # occurrence capacity: counted, first `cap` written
+    ds.reset()
+    got, gn, gd, k = _gpu(ds, sb, cap=3)
+    assert k == len(want) and len(got) == 3 and set(got) <= set(want) and gn == wn
+    # flow table full: 2 slots, more flows -> packets of unplaced flows not inspected
+    small = nfc.DpiStream(blob, off, np.array(act, dtype=np.uint8), max_flows=1)
+    got, gn, gd, k = _gpu(small, sb)
+    nf, nu = small.flows()
+    assert nf == 2 and nu > 0
+
+
+def test_stream_fullsize_sampled_flows(nfc):
+    """2^21 64-B packets over 64 K flows in one call (bench shape); the oracle checks
+    every packet of 300 sampled flows (flows are independent streams, so the
+    sample is exact), and the occurrence total is checked against the count sum."""
+    n, nflows = 1 << 21, 65536
+    blob, off, act, pats = _pats(4, 100, lmin=4, lmax=16)
+    rng = np.random.default_rng(8)
+    flow_of = rng.integers(0, nflows, n)
+    sb = stream_batch(9, n, nflows, pats, plant_frac=0.05, flow_of=flow_of)
+    ds = nfc.DpiStream(blob, off, act, max_flows=1 << 17)
+    got, gn, gd, k = _gpu(ds, sb, cap=1 << 22)
+    assert k == sum(gn) and len(got) == k
+    assert ds.flows() == (len(np.unique(flow_of)), 0)
+    sample = rng.choice(nflows, 300, replace=False)
+    sel = np.nonzero(np.isin(flow_of, sample))[0]
+    orc = StreamDPI(pats, list(act))
+    frames = sb.frames_of(sel) if hasattr(sb, "frames_of") else \
+        [sb.arena[int(sb.off[i]):int(sb.off[i]) + int(sb.len[i])].tobytes() for i in sel]
+    want, wn, wd = orc.process(frames)
+    want = sorted((int(sel[i]), j, e) for i, j, e in want)
+    selset = set(sel.tolist())
+    assert [o for o in got if o[0] in selset] == want
+    assert [gn[i] for i in sel] == wn and [gd[i] for i in sel] == wd
+    assert sum(1 for i, j, e in want if e < len(pats[j]) - 1) > 10
