@@ -7,10 +7,12 @@
 //              open-addressing flow table (lock-free insert), payload span;
 //   cub radix sort of (slot, packet index) pairs (stable: a flow's packets stay
 //              in index order, i.e. stream order);
-//   k_walk  -- one thread per flow present in the batch: starts from the flow's
-//              carried DFA state, walks its packets' payloads in order through the
-//              Aho-Corasick DFA (the same image builders.cpp makes for the fused
-//              kernel), appends every occurrence, stores the state back.
+//   k_walk  -- one thread per packet: rebuilds the packet's start state by
+//              re-walking the last maxlen - 1 bytes of its flow's stream (or from
+//              the state carried from earlier calls), walks its payload through the
+//              Aho-Corasick DFA (the image builders.cpp makes for the fused kernel)
+//              and appends every occurrence ending in it;
+//   k_commit -- stores each flow's final state for the next call.
 // The flow table and the per-flow DFA states persist across calls.
 #include <cuda_runtime.h>
 #include <cub/device/device_radix_sort.cuh>
@@ -105,7 +107,8 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
 {
     uint32_t s = key_hash(key) & mask;
     for (uint32_t probe = 0; probe <= mask; probe++, s = (s + 1) & mask) {
-        uint32_t l = atomicCAS(&lock[s], 0u, 1u);
+        uint32_t l = __ldcg(&lock[s]);               // published slots need no atomic
+        if (l == 0) l = atomicCAS(&lock[s], 0u, 1u);
         if (l == 0) {
             for (int k = 0; k < (int)KW; k++) keys[(size_t)s * KW + k] = key[k];
             __threadfence();
@@ -142,48 +145,84 @@ __global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mas
 }
 
 template <bool WIDE>
-__global__ void __launch_bounds__(128) k_walk(nfc_batch b, StreamDfa d, uint32_t none, const uint32_t *fkey,
-                                              const uint32_t *fidx, const uint32_t *span, uint32_t *fstate,
-                                              nfc_stream_result r)
+__device__ __forceinline__ uint32_t dfa_step(const StreamDfa &d, const uint8_t *cls, uint32_t s, uint32_t byte,
+                                             bool &acc)
+{
+    const size_t at = (size_t)s * d.ncls + cls[byte];
+    uint32_t nx;
+    if (WIDE) { nx = __ldg((const uint32_t *)d.trans + at); acc = nx >> 31; return nx & 0x7FFFFFFFu; }
+    nx = __ldg((const uint16_t *)d.trans + at);
+    acc = nx >> 15;
+    return nx & 0x7FFFu;
+}
+
+// One thread per packet in flow-sorted order (position u).  The packet's start
+// state is rebuilt from the flow's stream: a walk from the root that starts
+// maxlen - 1 bytes before the payload sees every occurrence ending in the payload
+// (an occurrence is at most maxlen bytes long), so the thread re-walks the tail of
+// its predecessors in this batch; if the flow's bytes in this batch are shorter than
+// that, it starts from the state carried from earlier calls.  The flow's last packet
+// leaves its final state in fin[u] (committed by k_commit: readers of fstate and
+// its writer never race).
+template <bool WIDE>
+__global__ void __launch_bounds__(256) k_walk(nfc_batch b, StreamDfa d, uint32_t none, uint32_t need,
+                                              const uint32_t *fkey, const uint32_t *fidx, const uint32_t *span,
+                                              const uint32_t *fstate, uint32_t *fin, nfc_stream_result r)
 {
     __shared__ uint8_t cls[256];
     for (int k = threadIdx.x; k < 256; k += blockDim.x) cls[k] = d.cls[k];
     __syncthreads();
-    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= b.n) return;
-    const uint32_t f = fkey[t];
-    if (f == none || (t > 0 && fkey[t - 1] == f)) return;   // not inspected / not the flow's first packet
-    uint32_t s = fstate[f];
-    const uint32_t first = (uint32_t)b.first_global_index;
-    for (uint32_t u = t; u < b.n && fkey[u] == f; u++) {
-        const uint32_t i = fidx[u], sp = span[i], a = sp & 0xFFFF, e = sp >> 16;
-        const uint8_t *p = b.arena + b.off[i];
-        uint32_t cnt = 0, dr = 0;
-        for (uint32_t x = a; x < e; x++) {
-            const size_t at = (size_t)s * d.ncls + cls[p[x]];
-            uint32_t nx;
-            bool acc;
-            if (WIDE) { nx = __ldg((const uint32_t *)d.trans + at); acc = nx >> 31; s = nx & 0x7FFFFFFFu; }
-            else      { nx = __ldg((const uint16_t *)d.trans + at); acc = nx >> 15; s = nx & 0x7FFFu; }
-            if (acc) {
-                const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
-                for (uint32_t k = o0; k < o1; k++) {
-                    const uint32_t pat = __ldg(d.out_ids + k);
-                    const uint32_t w = atomicAdd(r.occ_count, 1u);
-                    if (w < r.occ_cap) {
-                        r.occ_pkt[w] = first + i;
-                        r.occ_pat[w] = (uint16_t)pat;
-                        r.occ_end[w] = (uint16_t)(x - a);
-                    }
-                    dr |= __ldg(d.action + pat);
-                }
-                cnt += o1 - o0;
-            }
-        }
-        r.nocc[i] = cnt;
-        r.drop[i] = (uint8_t)dr;
+    const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+    if (u >= b.n) return;
+    const uint32_t f = fkey[u];
+    if (f == none) return;
+    // warm-up start: packet v, byte skip within its payload, start state s
+    uint32_t v = u, acc = 0, skip = 0, s = 0;
+    while (acc < need && v > 0 && fkey[v - 1] == f) {
+        v--;
+        const uint32_t sp = span[fidx[v]];
+        acc += (sp >> 16) - (sp & 0xFFFF);
     }
-    fstate[f] = s;
+    if (acc >= need) skip = acc - need;
+    else s = fstate[f];                              // v is the flow's first packet of this call
+    bool hit;
+    for (uint32_t w = v; w < u; w++) {
+        const uint32_t i = fidx[w], sp = span[i];
+        const uint8_t *p = b.arena + b.off[i];
+        for (uint32_t x = (sp & 0xFFFF) + (w == v ? skip : 0); x < (sp >> 16); x++) s = dfa_step<WIDE>(d, cls, s, p[x], hit);
+    }
+    const uint32_t i = fidx[u], sp = span[i], a = sp & 0xFFFF, e = sp >> 16;
+    const uint8_t *p = b.arena + b.off[i];
+    const uint32_t first = (uint32_t)b.first_global_index;
+    uint32_t cnt = 0, dr = 0;
+    for (uint32_t x = a; x < e; x++) {
+        s = dfa_step<WIDE>(d, cls, s, p[x], hit);
+        if (hit) {
+            const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
+            for (uint32_t k = o0; k < o1; k++) {
+                const uint32_t pat = __ldg(d.out_ids + k);
+                const uint32_t w = atomicAdd(r.occ_count, 1u);
+                if (w < r.occ_cap) {
+                    r.occ_pkt[w] = first + i;
+                    r.occ_pat[w] = (uint16_t)pat;
+                    r.occ_end[w] = (uint16_t)(x - a);
+                }
+                dr |= __ldg(d.action + pat);
+            }
+            cnt += o1 - o0;
+        }
+    }
+    r.nocc[i] = cnt;
+    r.drop[i] = (uint8_t)dr;
+    if (u + 1 == b.n || fkey[u + 1] != f) fin[u] = s;
+}
+
+__global__ void k_commit(uint32_t n, uint32_t none, const uint32_t *fkey, const uint32_t *fin, uint32_t *fstate)
+{
+    const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+    if (u >= n) return;
+    const uint32_t f = fkey[u];
+    if (f != none && (u + 1 == n || fkey[u + 1] != f)) fstate[f] = fin[u];
 }
 
 }  // namespace
@@ -196,7 +235,7 @@ struct nfc_dpi_stream {
     uint8_t *cls = nullptr, *trans = nullptr, *action = nullptr;
     uint32_t *out_off = nullptr;
     uint16_t *out_ids = nullptr;
-    uint32_t ncls = 0, wide = 0, n_states = 0;
+    uint32_t ncls = 0, wide = 0, n_states = 0, maxlen = 0;
     // per-call scratch
     uint32_t cap_pkts = 0;
     uint32_t *fkey = nullptr, *fkey2 = nullptr, *fidx = nullptr, *fidx2 = nullptr, *span = nullptr;
@@ -259,6 +298,7 @@ int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flo
     s->ncls = h.ncls;
     s->wide = h.wide;
     s->n_states = h.n_states;
+    s->maxlen = h.maxlen;
     cudaError_t ce = cudaSuccess;
     auto ok = [&](cudaError_t x) { if (ce == cudaSuccess) ce = x; };
     ok(cudaMalloc((void **)&s->lock, (size_t)s->n_slots * 4));
@@ -328,11 +368,14 @@ int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stre
     SCK(cub::DeviceRadixSort::SortPairs(s->tmp, tb, s->fkey, s->fkey2, s->fidx, s->fidx2, (int)b->n, 0,
                                         (int)s->key_bits, st));
     StreamDfa d{s->cls, s->trans, s->out_off, s->out_ids, s->action, s->ncls, s->wide};
-    const uint32_t wb = (b->n + 127) / 128;
-    if (s->wide) k_walk<true><<<wb, 128, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, *r);
-    else         k_walk<false><<<wb, 128, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, *r);
+    const uint32_t wb = (b->n + 255) / 256, need = s->maxlen - 1;
+    // s->fkey (unsorted keys) is dead after the sort: it holds the flows' final states
+    if (s->wide) k_walk<true><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+    else         k_walk<false><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
     SCK(cudaGetLastError());
-    s->launches += 2;   // k_flow + k_walk (the cub sort launches its own kernels)
+    k_commit<<<blocks, 256, 0, st>>>(b->n, none, s->fkey2, s->fkey, s->fstate);
+    SCK(cudaGetLastError());
+    s->launches += 3;   // k_flow + k_walk + k_commit (the cub sort launches its own kernels)
     return NFC_OK;
 }
 
