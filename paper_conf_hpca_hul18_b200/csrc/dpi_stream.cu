@@ -100,6 +100,13 @@ __device__ __forceinline__ uint32_t key_hash(const uint32_t key[KW])
     return h;
 }
 
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
 // Flow table slot of `key` (inserted if new); 0xFFFFFFFF if the table is full.
 // lock[s]: 0 empty, 1 key being written, 2 key published.
 __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t *n_flows,
@@ -107,17 +114,19 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
 {
     uint32_t s = key_hash(key) & mask;
     for (uint32_t probe = 0; probe <= mask; probe++, s = (s + 1) & mask) {
-        uint32_t l = __ldcg(&lock[s]);               // published slots need no atomic
-        if (l == 0) l = atomicCAS(&lock[s], 0u, 1u);
+        uint32_t l = ld_acquire(&lock[s]);           // published slots need no atomic
         if (l == 0) {
-            for (int k = 0; k < (int)KW; k++) keys[(size_t)s * KW + k] = key[k];
-            __threadfence();
-            atomicExch(&lock[s], 2u);
-            atomicAdd(n_flows, 1u);
-            return s;
+            l = atomicCAS(&lock[s], 0u, 1u);
+            if (l == 0) {
+                for (int k = 0; k < (int)KW; k++) keys[(size_t)s * KW + k] = key[k];
+                __threadfence();
+                atomicExch(&lock[s], 2u);
+                atomicAdd(n_flows, 1u);
+                return s;
+            }
+            l = ld_acquire(&lock[s]);                // the CAS is relaxed: re-read with acquire
         }
-        while (l == 1) l = *(volatile uint32_t *)&lock[s];
-        __threadfence();
+        while (l == 1) l = ld_acquire(&lock[s]);     // acquire: the published key is visible
         bool eq = true;
         for (int k = 0; k < (int)KW; k++) eq &= __ldcg(&keys[(size_t)s * KW + k]) == key[k];
         if (eq) return s;
@@ -156,6 +165,47 @@ __device__ __forceinline__ uint32_t dfa_step(const StreamDfa &d, const uint8_t *
     return nx & 0x7FFFu;
 }
 
+// Walks payload bytes [x0, x1) of the frame at p (16-B aligned) from state s.  The
+// bytes are fetched as aligned 16-B words, so a payload costs ceil(len/16) + 1 loads
+// issued ahead of the dependent DFA steps instead of one byte load per step.
+struct Emit {
+    nfc_stream_result r;
+    uint32_t pkt, a, cnt, dr;
+};
+
+template <bool WIDE, bool EMIT>
+__device__ __forceinline__ uint32_t walk(const StreamDfa &d, const uint8_t *cls, const uint8_t *p, uint32_t x0,
+                                         uint32_t x1, uint32_t s, Emit &em)
+{
+    uint32_t x = x0;
+    while (x < x1) {
+        const uint32_t base = x & ~15u;
+        const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p + base));
+        const uint32_t hi = min(x1, base + 16);
+        for (; x < hi; x++) {
+            const uint32_t q = (x >> 2) & 3;
+            const uint32_t wd = q == 0 ? v.x : q == 1 ? v.y : q == 2 ? v.z : v.w;
+            bool hit;
+            s = dfa_step<WIDE>(d, cls, s, (wd >> (8 * (x & 3))) & 0xFF, hit);
+            if (EMIT && hit) {
+                const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
+                for (uint32_t k = o0; k < o1; k++) {
+                    const uint32_t pat = __ldg(d.out_ids + k);
+                    const uint32_t w = atomicAdd(em.r.occ_count, 1u);
+                    if (w < em.r.occ_cap) {
+                        em.r.occ_pkt[w] = em.pkt;
+                        em.r.occ_pat[w] = (uint16_t)pat;
+                        em.r.occ_end[w] = (uint16_t)(x - em.a);
+                    }
+                    em.dr |= __ldg(d.action + pat);
+                }
+                em.cnt += o1 - o0;
+            }
+        }
+    }
+    return s;
+}
+
 // One thread per packet in flow-sorted order (position u).  The packet's start
 // state is rebuilt from the flow's stream: a walk from the root that starts
 // maxlen - 1 bytes before the payload sees every occurrence ending in the payload
@@ -185,35 +235,17 @@ __global__ void __launch_bounds__(256) k_walk(nfc_batch b, StreamDfa d, uint32_t
     }
     if (acc >= need) skip = acc - need;
     else s = fstate[f];                              // v is the flow's first packet of this call
-    bool hit;
+    Emit em{r, (uint32_t)b.first_global_index, 0, 0, 0};
     for (uint32_t w = v; w < u; w++) {
         const uint32_t i = fidx[w], sp = span[i];
-        const uint8_t *p = b.arena + b.off[i];
-        for (uint32_t x = (sp & 0xFFFF) + (w == v ? skip : 0); x < (sp >> 16); x++) s = dfa_step<WIDE>(d, cls, s, p[x], hit);
+        s = walk<WIDE, false>(d, cls, b.arena + b.off[i], (sp & 0xFFFF) + (w == v ? skip : 0), sp >> 16, s, em);
     }
-    const uint32_t i = fidx[u], sp = span[i], a = sp & 0xFFFF, e = sp >> 16;
-    const uint8_t *p = b.arena + b.off[i];
-    const uint32_t first = (uint32_t)b.first_global_index;
-    uint32_t cnt = 0, dr = 0;
-    for (uint32_t x = a; x < e; x++) {
-        s = dfa_step<WIDE>(d, cls, s, p[x], hit);
-        if (hit) {
-            const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
-            for (uint32_t k = o0; k < o1; k++) {
-                const uint32_t pat = __ldg(d.out_ids + k);
-                const uint32_t w = atomicAdd(r.occ_count, 1u);
-                if (w < r.occ_cap) {
-                    r.occ_pkt[w] = first + i;
-                    r.occ_pat[w] = (uint16_t)pat;
-                    r.occ_end[w] = (uint16_t)(x - a);
-                }
-                dr |= __ldg(d.action + pat);
-            }
-            cnt += o1 - o0;
-        }
-    }
-    r.nocc[i] = cnt;
-    r.drop[i] = (uint8_t)dr;
+    const uint32_t i = fidx[u], sp = span[i];
+    em.pkt += i;
+    em.a = sp & 0xFFFF;
+    s = walk<WIDE, true>(d, cls, b.arena + b.off[i], sp & 0xFFFF, sp >> 16, s, em);
+    r.nocc[i] = em.cnt;
+    r.drop[i] = (uint8_t)em.dr;
     if (u + 1 == b.n || fkey[u + 1] != f) fin[u] = s;
 }
 
