@@ -28,6 +28,8 @@ using namespace nfc;
 namespace {
 
 constexpr uint32_t KW = 10;   // key words: src[4], dst[4], sport<<16|dport, proto | family<<8
+constexpr uint32_t KS = 12;   // key words per table slot (48 B: three 16-B loads)
+constexpr uint32_t HB = 96;   // header bytes staged per packet (IPv4 IHL 15 + TCP data offset: 88)
 
 struct StreamDfa {
     const uint8_t *cls;
@@ -41,8 +43,11 @@ struct StreamDfa {
 __device__ __forceinline__ uint32_t be16d(const uint8_t *p) { return (uint32_t)p[0] << 8 | p[1]; }
 
 // R#24 parse: returns false if the frame is not inspected; key[KW], payload [a, b)
-__device__ bool parse_flow(const uint8_t *f, uint32_t flen, uint32_t key[KW], uint32_t &a, uint32_t &b)
+// f holds the frame's first `have` bytes (have = min(flen, HB): every byte the parse
+// reads lies below 88, and each read is guarded by a bound that implies < flen).
+__device__ bool parse_flow(const uint8_t *f, uint32_t have, uint32_t flen, uint32_t key[KW], uint32_t &a, uint32_t &b)
 {
+    (void)have;
     if (flen < 14) return false;
     const uint32_t et = be16d(f + 12);
     uint32_t l4, ip_end, proto, fam;
@@ -118,7 +123,10 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
         if (l == 0) {
             l = atomicCAS(&lock[s], 0u, 1u);
             if (l == 0) {
-                for (int k = 0; k < (int)KW; k++) keys[(size_t)s * KW + k] = key[k];
+                uint4 *kp = reinterpret_cast<uint4 *>(keys + (size_t)s * KS);
+                kp[0] = make_uint4(key[0], key[1], key[2], key[3]);
+                kp[1] = make_uint4(key[4], key[5], key[6], key[7]);
+                kp[2] = make_uint4(key[8], key[9], 0, 0);
                 __threadfence();
                 atomicExch(&lock[s], 2u);
                 atomicAdd(n_flows, 1u);
@@ -127,9 +135,11 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
             l = ld_acquire(&lock[s]);                // the CAS is relaxed: re-read with acquire
         }
         while (l == 1) l = ld_acquire(&lock[s]);     // acquire: the published key is visible
-        bool eq = true;
-        for (int k = 0; k < (int)KW; k++) eq &= __ldcg(&keys[(size_t)s * KW + k]) == key[k];
-        if (eq) return s;
+        const uint4 *kp = reinterpret_cast<const uint4 *>(keys + (size_t)s * KS);
+        const uint4 k0 = __ldcg(kp), k1 = __ldcg(kp + 1), k2 = __ldcg(kp + 2);
+        if (k0.x == key[0] && k0.y == key[1] && k0.z == key[2] && k0.w == key[3] && k1.x == key[4] &&
+            k1.y == key[5] && k1.z == key[6] && k1.w == key[7] && k2.x == key[8] && k2.y == key[9])
+            return s;
     }
     return 0xFFFFFFFFu;
 }
@@ -138,14 +148,23 @@ __global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mas
                        uint32_t *ctr, uint32_t *fkey, uint32_t *fidx, uint32_t *span,
                        uint32_t *nocc, uint8_t *drop)
 {
+    // the first HB bytes of each frame are staged in shared memory with 16-B loads
+    // (frames are 16-B aligned; no load starts beyond the frame), then parsed there
+    __shared__ uint4 hdr[256 * HB / 16];
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= b.n) return;
     nocc[i] = 0;
     drop[i] = 0;
     fidx[i] = i;
+    const uint32_t flen = b.len[i];
+    const uint4 *src = reinterpret_cast<const uint4 *>(b.arena + b.off[i]);
+    uint4 *h = hdr + threadIdx.x * (HB / 16);
+#pragma unroll
+    for (uint32_t k = 0; k < HB / 16; k++)
+        if (16 * k < flen) h[k] = __ldg(src + k);
     uint32_t key[KW], a, e;
     uint32_t slot = none;
-    if (parse_flow(b.arena + b.off[i], b.len[i], key, a, e)) {
+    if (parse_flow(reinterpret_cast<const uint8_t *>(h), min(flen, HB), flen, key, a, e)) {
         slot = flow_slot(lock, keys, mask, &ctr[0], key);
         if (slot == 0xFFFFFFFFu) { atomicAdd(&ctr[1], 1u); slot = none; }
         span[i] = a | e << 16;
@@ -334,7 +353,7 @@ int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flo
     cudaError_t ce = cudaSuccess;
     auto ok = [&](cudaError_t x) { if (ce == cudaSuccess) ce = x; };
     ok(cudaMalloc((void **)&s->lock, (size_t)s->n_slots * 4));
-    ok(cudaMalloc((void **)&s->keys, (size_t)s->n_slots * KW * 4));
+    ok(cudaMalloc((void **)&s->keys, (size_t)s->n_slots * KS * 4));
     ok(cudaMalloc((void **)&s->fstate, (size_t)s->n_slots * 4));
     ok(cudaMalloc((void **)&s->ctr, 4 * 4));
     ok(dev_copy(&s->cls, h.cls.data(), h.cls.size()));
