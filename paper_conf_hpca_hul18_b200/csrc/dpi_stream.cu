@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 #include <cub/device/device_radix_sort.cuh>
 
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -29,6 +30,10 @@ namespace {
 
 constexpr uint32_t KW = 10;   // key words: src[4], dst[4], sport<<16|dport, proto | family<<8
 constexpr uint32_t KS = 12;   // key words per table slot (48 B: three 16-B loads)
+constexpr size_t DFA_SMEM_MAX = 200 * 1024;   // DFA bytes staged in shared memory (k_walk<2>)
+#ifndef WALK_SMEM_THREADS
+#define WALK_SMEM_THREADS 768   // k_walk<2> CTA size (1024 spills at the 64-register cap)
+#endif
 constexpr uint32_t HB = 96;   // header bytes staged per packet (IPv4 IHL 15 + TCP data offset: 88)
 
 struct StreamDfa {
@@ -37,7 +42,7 @@ struct StreamDfa {
     const uint32_t *out_off;
     const uint16_t *out_ids;
     const uint8_t *action;
-    uint32_t ncls, wide;
+    uint32_t ncls, wide, n_states;
 };
 
 __device__ __forceinline__ uint32_t be16d(const uint8_t *p) { return (uint32_t)p[0] << 8 | p[1]; }
@@ -172,14 +177,16 @@ __global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mas
     fkey[i] = slot;
 }
 
-template <bool WIDE>
+// M: 0 = u16 entries read through L1/L2, 1 = u32 entries (> 32768 states), 2 = u16
+// entries staged in shared memory (d.trans points there)
+template <int M>
 __device__ __forceinline__ uint32_t dfa_step(const StreamDfa &d, const uint8_t *cls, uint32_t s, uint32_t byte,
                                              bool &acc)
 {
     const size_t at = (size_t)s * d.ncls + cls[byte];
     uint32_t nx;
-    if (WIDE) { nx = __ldg((const uint32_t *)d.trans + at); acc = nx >> 31; return nx & 0x7FFFFFFFu; }
-    nx = __ldg((const uint16_t *)d.trans + at);
+    if (M == 1) { nx = __ldg((const uint32_t *)d.trans + at); acc = nx >> 31; return nx & 0x7FFFFFFFu; }
+    nx = M == 2 ? ((const uint16_t *)d.trans)[at] : __ldg((const uint16_t *)d.trans + at);
     acc = nx >> 15;
     return nx & 0x7FFFu;
 }
@@ -192,7 +199,7 @@ struct Emit {
     uint32_t pkt, a, cnt, dr;
 };
 
-template <bool WIDE, bool EMIT>
+template <int M, bool EMIT>
 __device__ __forceinline__ uint32_t walk(const StreamDfa &d, const uint8_t *cls, const uint8_t *p, uint32_t x0,
                                          uint32_t x1, uint32_t s, Emit &em)
 {
@@ -205,7 +212,7 @@ __device__ __forceinline__ uint32_t walk(const StreamDfa &d, const uint8_t *cls,
             const uint32_t q = (x >> 2) & 3;
             const uint32_t wd = q == 0 ? v.x : q == 1 ? v.y : q == 2 ? v.z : v.w;
             bool hit;
-            s = dfa_step<WIDE>(d, cls, s, (wd >> (8 * (x & 3))) & 0xFF, hit);
+            s = dfa_step<M>(d, cls, s, (wd >> (8 * (x & 3))) & 0xFF, hit);
             if (EMIT && hit) {
                 const uint32_t o0 = __ldg(d.out_off + s), o1 = __ldg(d.out_off + s + 1);
                 for (uint32_t k = o0; k < o1; k++) {
@@ -233,39 +240,46 @@ __device__ __forceinline__ uint32_t walk(const StreamDfa &d, const uint8_t *cls,
 // that, it starts from the state carried from earlier calls.  The flow's last packet
 // leaves its final state in fin[u] (committed by k_commit: readers of fstate and
 // its writer never race).
-template <bool WIDE>
-__global__ void __launch_bounds__(256) k_walk(nfc_batch b, StreamDfa d, uint32_t none, uint32_t need,
-                                              const uint32_t *fkey, const uint32_t *fidx, const uint32_t *span,
-                                              const uint32_t *fstate, uint32_t *fin, nfc_stream_result r)
+template <int M>
+__global__ void __launch_bounds__(M == 2 ? WALK_SMEM_THREADS : 256) k_walk(nfc_batch b, StreamDfa d, uint32_t none, uint32_t need,
+                                                          const uint32_t *fkey, const uint32_t *fidx,
+                                                          const uint32_t *span, const uint32_t *fstate, uint32_t *fin,
+                                                          nfc_stream_result r)
 {
     __shared__ uint8_t cls[256];
+    extern __shared__ uint4 dyn[];
     for (int k = threadIdx.x; k < 256; k += blockDim.x) cls[k] = d.cls[k];
+    if (M == 2) {   // persistent CTAs: the whole DFA in shared memory, copied once per CTA
+        const uint32_t n16 = (d.ncls * d.n_states * 2 + 15) / 16;
+        for (uint32_t k = threadIdx.x; k < n16; k += blockDim.x) dyn[k] = __ldg((const uint4 *)d.trans + k);
+        d.trans = dyn;
+    }
     __syncthreads();
-    const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
-    if (u >= b.n) return;
-    const uint32_t f = fkey[u];
-    if (f == none) return;
-    // warm-up start: packet v, byte skip within its payload, start state s
-    uint32_t v = u, acc = 0, skip = 0, s = 0;
-    while (acc < need && v > 0 && fkey[v - 1] == f) {
-        v--;
-        const uint32_t sp = span[fidx[v]];
-        acc += (sp >> 16) - (sp & 0xFFFF);
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < b.n; u += gridDim.x * blockDim.x) {
+        const uint32_t f = fkey[u];
+        if (f == none) continue;
+        // warm-up start: packet v, byte skip within its payload, start state s
+        uint32_t v = u, acc = 0, skip = 0, s = 0;
+        while (acc < need && v > 0 && fkey[v - 1] == f) {
+            v--;
+            const uint32_t sp = span[fidx[v]];
+            acc += (sp >> 16) - (sp & 0xFFFF);
+        }
+        if (acc >= need) skip = acc - need;
+        else s = fstate[f];                          // v is the flow's first packet of this call
+        Emit em{r, (uint32_t)b.first_global_index, 0, 0, 0};
+        for (uint32_t w = v; w < u; w++) {
+            const uint32_t i = fidx[w], sp = span[i];
+            s = walk<M, false>(d, cls, b.arena + b.off[i], (sp & 0xFFFF) + (w == v ? skip : 0), sp >> 16, s, em);
+        }
+        const uint32_t i = fidx[u], sp = span[i];
+        em.pkt += i;
+        em.a = sp & 0xFFFF;
+        s = walk<M, true>(d, cls, b.arena + b.off[i], sp & 0xFFFF, sp >> 16, s, em);
+        r.nocc[i] = em.cnt;
+        r.drop[i] = (uint8_t)em.dr;
+        if (u + 1 == b.n || fkey[u + 1] != f) fin[u] = s;
     }
-    if (acc >= need) skip = acc - need;
-    else s = fstate[f];                              // v is the flow's first packet of this call
-    Emit em{r, (uint32_t)b.first_global_index, 0, 0, 0};
-    for (uint32_t w = v; w < u; w++) {
-        const uint32_t i = fidx[w], sp = span[i];
-        s = walk<WIDE, false>(d, cls, b.arena + b.off[i], (sp & 0xFFFF) + (w == v ? skip : 0), sp >> 16, s, em);
-    }
-    const uint32_t i = fidx[u], sp = span[i];
-    em.pkt += i;
-    em.a = sp & 0xFFFF;
-    s = walk<WIDE, true>(d, cls, b.arena + b.off[i], sp & 0xFFFF, sp >> 16, s, em);
-    r.nocc[i] = em.cnt;
-    r.drop[i] = (uint8_t)em.dr;
-    if (u + 1 == b.n || fkey[u + 1] != f) fin[u] = s;
 }
 
 __global__ void k_commit(uint32_t n, uint32_t none, const uint32_t *fkey, const uint32_t *fin, uint32_t *fstate)
@@ -287,6 +301,7 @@ struct nfc_dpi_stream {
     uint32_t *out_off = nullptr;
     uint16_t *out_ids = nullptr;
     uint32_t ncls = 0, wide = 0, n_states = 0, maxlen = 0;
+    uint32_t n_sm = 148, smem_ok = 0;   // k_walk<2>: the DFA fits the opt-in shared memory
     // per-call scratch
     uint32_t cap_pkts = 0;
     uint32_t *fkey = nullptr, *fkey2 = nullptr, *fidx = nullptr, *fidx2 = nullptr, *span = nullptr;
@@ -367,6 +382,16 @@ int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flo
         ok(cudaMemset(s->ctr, 0, 16));
         ok(cudaDeviceSynchronize());
     }
+    if (ce == cudaSuccess && !s->wide && (size_t)s->ncls * s->n_states * 2 <= DFA_SMEM_MAX) {
+        int nsm = 0;
+        ok(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, device));
+        ok(cudaFuncSetAttribute(k_walk<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DFA_SMEM_MAX + 16));
+        s->n_sm = nsm > 0 ? (uint32_t)nsm : 148;
+        s->smem_ok = ce == cudaSuccess;
+        // measured slower (one 768-thread CTA per SM: 491 vs 402 us per 4 M packets with
+        // the rows in L1), so opt-in only
+        if (!getenv("NFC_STREAM_SMEM")) s->smem_ok = 0;
+    }
     if (ce != cudaSuccess) {
         nfc_dpi_stream_destroy(s);
         return set_fail(ce == cudaErrorMemoryAllocation ? NFC_ENOMEM : NFC_ECUDA,
@@ -418,11 +443,18 @@ int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stre
     size_t tb = s->tmp_bytes;
     SCK(cub::DeviceRadixSort::SortPairs(s->tmp, tb, s->fkey, s->fkey2, s->fidx, s->fidx2, (int)b->n, 0,
                                         (int)s->key_bits, st));
-    StreamDfa d{s->cls, s->trans, s->out_off, s->out_ids, s->action, s->ncls, s->wide};
+    StreamDfa d{s->cls, s->trans, s->out_off, s->out_ids, s->action, s->ncls, s->wide, s->n_states};
     const uint32_t wb = (b->n + 255) / 256, need = s->maxlen - 1;
     // s->fkey (unsorted keys) is dead after the sort: it holds the flows' final states
-    if (s->wide) k_walk<true><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
-    else         k_walk<false><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+    const size_t tbytes = (size_t)s->ncls * s->n_states * 2;
+    if (s->wide) {
+        k_walk<1><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+    } else if (s->smem_ok && tbytes <= DFA_SMEM_MAX) {
+        k_walk<2><<<s->n_sm, WALK_SMEM_THREADS, (tbytes + 15) / 16 * 16, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span,
+                                                                s->fstate, s->fkey, *r);
+    } else {
+        k_walk<0><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+    }
     SCK(cudaGetLastError());
     k_commit<<<blocks, 256, 0, st>>>(b->n, none, s->fkey2, s->fkey, s->fstate);
     SCK(cudaGetLastError());

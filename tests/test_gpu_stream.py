@@ -50,7 +50,11 @@ def _gpu(ds, sb: StreamBatch, cap=1 << 20):
     return occ, nocc.cpu().numpy().tolist(), drop.cpu().numpy().tolist(), k
 
 
-def test_stream_parity_multi_call(nfc):
+@pytest.mark.parametrize("smem", [1, 0])
+def test_stream_parity_multi_call(nfc, smem, monkeypatch):
+    """smem=1: the DFA staged in shared memory (k_walk<2>); 0: read through L1/L2 (k_walk<0>)."""
+    if smem:
+        monkeypatch.setenv("NFC_STREAM_SMEM", "1")
     blob, off, act, pats = _pats(1, 100)
     ds = nfc.DpiStream(blob, off, act, max_flows=4096)
     orc = StreamDPI(pats, list(act))
