@@ -87,3 +87,32 @@ def test_no_oracle_in_product():
             if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
                 txt = open(os.path.join(dp, f)).read()
                 assert not bad.search(txt), f
+
+
+def test_stream_dpi_validation_before_cuda(nfc):
+    """nfc_dpi_stream_create: NULL / malformed arguments are NFC_EINVAL before any CUDA
+    call; the struct layout matches the header (8 pointers + 2 u32 = 56 B)."""
+    assert ctypes.sizeof(nfc.StreamResult) == 56
+    L = nfc.lib
+    h = ctypes.c_void_p()
+    good = np.frombuffer(b"abcab", dtype=np.uint8).copy()
+    off = np.array([0, 3, 5], dtype=np.uint32)
+    act = np.zeros(2, dtype=np.uint8)
+    spec = nfc.DpiSpec(2, good.ctypes.data, off.ctypes.data, act.ctypes.data)
+    assert L.nfc_dpi_stream_create(0, None, 16, ctypes.byref(h)) == nfc.NFC_EINVAL
+    assert L.nfc_dpi_stream_create(0, ctypes.byref(spec), 0, ctypes.byref(h)) == nfc.NFC_EINVAL
+    bad_off = np.array([0, 3, 3], dtype=np.uint32)          # empty pattern
+    bad = nfc.DpiSpec(2, good.ctypes.data, bad_off.ctypes.data, act.ctypes.data)
+    assert L.nfc_dpi_stream_create(0, ctypes.byref(bad), 16, ctypes.byref(h)) == nfc.NFC_EINVAL
+    assert b"empty pattern" in L.nfc_last_error()
+    assert L.nfc_dpi_stream_process(None, None, None, None) == nfc.NFC_EINVAL
+    assert L.nfc_dpi_stream_destroy(None) == nfc.NFC_OK
+
+
+def test_stream_dpi_fails_loudly_without_gpu(nfc):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    blob = np.frombuffer(b"abc", dtype=np.uint8).copy()
+    with pytest.raises(nfc.NfcError):
+        nfc.DpiStream(blob, np.array([0, 3], dtype=np.uint32), np.zeros(1, dtype=np.uint8), max_flows=8)
