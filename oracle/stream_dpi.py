@@ -120,3 +120,39 @@ class StreamDPI:
 
     def n_flows(self) -> int:
         return len(self.streams)
+
+
+class StreamRegexDPI(StreamDPI):
+    """Regular-expression variant (P:L132 "for the regular expression we use a DFA";
+    DESIGN.md R#33): an occurrence of expression j ends at stream byte x iff a
+    non-empty substring of the flow's stream ending at x is in L(j).  Written with
+    Python's backtracking `re` (an independent engine, no automaton of ours):
+    re.search(b"(?:R)\\Z", stream[:x + 1]) at every byte, DOTALL so '.' is any byte."""
+
+    def __init__(self, regexes: Sequence[bytes], actions: Sequence[int]):
+        import re
+        super().__init__([b"?"] * len(regexes), actions)
+        self.res = [re.compile(b"(?:" + bytes(r) + b")\\Z", re.DOTALL) for r in regexes]
+
+    def process(self, frames: Sequence[bytes], first_global_index: int = 0):
+        n = len(frames)
+        nocc, drop = [0] * n, [0] * n
+        occ: List[Tuple[int, int, int]] = []
+        for i, fr in enumerate(frames):
+            p = parse(fr)
+            if p is None:
+                continue
+            key, a, b = p
+            st = self.streams.setdefault(key, bytearray())
+            base = len(st)
+            st += fr[a:b]
+            view = bytes(st)
+            for x in range(base, len(st)):
+                for j, rx in enumerate(self.res):
+                    m = rx.search(view, 0, x + 1)
+                    if m is not None and m.end() > m.start():
+                        occ.append((first_global_index + i, j, x - base))
+                        nocc[i] += 1
+                        drop[i] |= self.actions[j]
+        occ.sort()
+        return occ, nocc, drop

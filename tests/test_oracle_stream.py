@@ -145,3 +145,25 @@ def test_generator_plants_cross_packet_occurrences():
     # an occurrence whose end offset is < len - 1 of its pattern started in an earlier packet
     cross = sum(1 for i, j, e in occ if e < len(pats[j]) - 1)
     assert cross > 100
+
+
+def test_regex_oracle_hand_example():
+    from oracle.stream_dpi import StreamRegexDPI
+    o = StreamRegexDPI([b"a[0-9]{2}", b"(xy|z)\\.", b"q.?r"], [0, 1, 0])
+    occ, nocc, drop = o.process([_udp(b"_a1"), _udp(b"2z."), _udp(b"qr q\x00r")], 0)
+    # a12 ends at packet 1 offset 0; z. at packet 1 offset 2; qr at packet 2 offset 1; q\0r at offset 5
+    assert occ == [(1, 0, 0), (1, 1, 2), (2, 2, 1), (2, 2, 5)]
+    assert nocc == [0, 2, 2] and drop == [0, 1, 0]
+
+
+def test_regex_oracle_literals_equal_string_oracle():
+    """A regex set of escaped literals gives exactly the string-pattern oracle's result."""
+    import re
+    from oracle.stream_dpi import StreamRegexDPI
+    r = random.Random(4)
+    pats = list(dict.fromkeys(bytes(r.choice(b"ab.c") for _ in range(r.randrange(1, 5))) for _ in range(8)))
+    frames = [_udp(bytes(r.choice(b"ab.c") for _ in range(r.randrange(0, 12))), sport=r.randrange(3))
+              for _ in range(40)]
+    a = StreamDPI(pats, [0] * len(pats)).process(frames)
+    b = StreamRegexDPI([re.escape(p) for p in pats], [0] * len(pats)).process(frames)
+    assert a == b
