@@ -306,6 +306,17 @@ typedef struct {
  * malformed spec) and a device flow table of the next power of two >= 2 x
  * max_flows slots (1..2^28) on `device`.  NFC_ENOMEM / NFC_ECUDA on failure. */
 NFC_API int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flows, nfc_dpi_stream **out);
+/* Regular-expression variant ("for the regular expression we use a DFA";
+ * DESIGN.md R#33): spec->blob[off[j] .. off[j+1]) is expression j (not NUL-
+ * terminated) over bytes: literals, \xHH, \<punct>, '.', [..] classes with ranges
+ * and '^', (..), '|', '?', {m} and {m,n} with n <= 64.  An occurrence of
+ * expression j ends at byte x iff a non-empty substring of the flow stream ending
+ * at x is in its language (unanchored search); it is reported like a pattern
+ * occurrence.  Every language is finite, so the longest match bounds the re-walk.
+ * NFC_EUNSUP for '*' / '+' / {m,}; NFC_EINVAL for a syntax error, an expression
+ * that matches the empty string, or a DFA over max_states states (0 = 2^20). */
+NFC_API int nfc_dpi_stream_create_regex(int device, const nfc_dpi_spec *spec, uint32_t max_flows,
+                                        uint32_t max_states, nfc_dpi_stream **out);
 NFC_API int nfc_dpi_stream_destroy(nfc_dpi_stream *s);
 /* Forgets every flow (asynchronous on `stream`). */
 NFC_API int nfc_dpi_stream_reset(nfc_dpi_stream *s, void *stream);

@@ -345,6 +345,8 @@ int nfc_dpi_stream_destroy(nfc_dpi_stream *s)
     return NFC_OK;
 }
 
+static int create_from_host(int device, const DpiHost &h, uint32_t max_flows, nfc_dpi_stream **out);
+
 int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flows, nfc_dpi_stream **out)
 {
     if (!spec || !out) return set_fail(NFC_EINVAL, "dpi_stream_create: NULL pointer");
@@ -353,6 +355,23 @@ int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t max_flo
     DpiHost h;
     std::string e = build_dpi(*spec, h);
     if (!e.empty()) return set_fail(NFC_EINVAL, e);
+    return create_from_host(device, h, max_flows, out);
+}
+
+int nfc_dpi_stream_create_regex(int device, const nfc_dpi_spec *spec, uint32_t max_flows, uint32_t max_states,
+                                nfc_dpi_stream **out)
+{
+    if (!spec || !out) return set_fail(NFC_EINVAL, "dpi_stream_create_regex: NULL pointer");
+    if (max_flows == 0 || max_flows > (1u << 28)) return set_fail(NFC_EINVAL, "dpi_stream_create_regex: max_flows must be 1..2^28");
+    *out = nullptr;
+    DpiHost h;
+    std::string e = build_regex_dfa(*spec, h, max_states ? max_states : (1u << 20));
+    if (!e.empty()) return set_fail(e.find("unbounded") != std::string::npos ? NFC_EUNSUP : NFC_EINVAL, e);
+    return create_from_host(device, h, max_flows, out);
+}
+
+static int create_from_host(int device, const DpiHost &h, uint32_t max_flows, nfc_dpi_stream **out)
+{
     SCK(cudaSetDevice(device));
     nfc_dpi_stream *s = new nfc_dpi_stream;
     s->device = device;

@@ -216,7 +216,9 @@ struct KParams {
 };
 
 // host-side builders (builders.cpp); return "" on success or an error message
-int set_fail(int code, const std::string &msg);   // capi.cu: nfc_last_error + code
+int set_fail(int code, const std::string &msg);
+struct DpiHost;
+std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states);   // regex.cpp   // capi.cu: nfc_last_error + code
 struct HostImage { std::vector<uint8_t> bytes; };
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
 struct DpiHost {

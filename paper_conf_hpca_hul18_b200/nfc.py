@@ -89,7 +89,7 @@ class Result(ctypes.Structure):
 EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_tables",
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard",
-           "nfc_dpi_stream_create", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
+           "nfc_dpi_stream_create", "nfc_dpi_stream_create_regex", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
            "nfc_dpi_stream_process", "nfc_dpi_stream_flows"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
@@ -117,6 +117,7 @@ def _load_lib():
     L.nfc_plan_parallel.argtypes = [_P, _u32, _P]
     L.nfc_rss_shard.argtypes = [ctypes.c_int, ctypes.POINTER(Batch), _u32, _P, _P]
     L.nfc_dpi_stream_create.argtypes = [ctypes.c_int, ctypes.POINTER(DpiSpec), _u32, ctypes.POINTER(_P)]
+    L.nfc_dpi_stream_create_regex.argtypes = [ctypes.c_int, ctypes.POINTER(DpiSpec), _u32, _u32, ctypes.POINTER(_P)]
     L.nfc_dpi_stream_destroy.argtypes = [_P]
     L.nfc_dpi_stream_reset.argtypes = [_P, _P]
     L.nfc_dpi_stream_process.argtypes = [_P, ctypes.POINTER(Batch), ctypes.POINTER(StreamResult), _P]
@@ -327,11 +328,16 @@ class DpiStream:
 
     Argument marshalling only: every step runs in dpi_stream.cu."""
 
-    def __init__(self, blob: np.ndarray, off: np.ndarray, action: np.ndarray, max_flows: int, device: int = 0):
+    def __init__(self, blob: np.ndarray, off: np.ndarray, action: np.ndarray, max_flows: int, device: int = 0,
+                 regex: bool = False, max_states: int = 0):
+        """regex=True: blob/off hold regular expressions (nfc_dpi_stream_create_regex)."""
         b, o, a = _np(blob, np.uint8), _np(off, np.uint32), _np(action, np.uint8)
         h = _P()
-        _check(lib.nfc_dpi_stream_create(device, ctypes.byref(DpiSpec(len(a), b.ctypes.data, o.ctypes.data,
-                                                                      a.ctypes.data)), max_flows, ctypes.byref(h)))
+        spec = DpiSpec(len(a), b.ctypes.data, o.ctypes.data, a.ctypes.data)
+        if regex:
+            _check(lib.nfc_dpi_stream_create_regex(device, ctypes.byref(spec), max_flows, max_states, ctypes.byref(h)))
+        else:
+            _check(lib.nfc_dpi_stream_create(device, ctypes.byref(spec), max_flows, ctypes.byref(h)))
         self.h = h
         self.device = device
 

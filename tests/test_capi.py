@@ -116,3 +116,17 @@ def test_stream_dpi_fails_loudly_without_gpu(nfc):
     blob = np.frombuffer(b"abc", dtype=np.uint8).copy()
     with pytest.raises(nfc.NfcError):
         nfc.DpiStream(blob, np.array([0, 3], dtype=np.uint32), np.zeros(1, dtype=np.uint8), max_flows=8)
+
+
+@pytest.mark.parametrize("rx,code", [(b"ab*", "NFC_EUNSUP"), (b"a+", "NFC_EUNSUP"), (b"a{2,}", "NFC_EUNSUP"),
+                                     (b"a?", "NFC_EINVAL"), (b"(a", "NFC_EINVAL"), (b"[ab", "NFC_EINVAL"),
+                                     (b"a)", "NFC_EINVAL"), (b"\\q", "NFC_EINVAL"), (b"a{0}", "NFC_EINVAL")])
+def test_regex_rejected_before_cuda(nfc, rx, code):
+    """Unbounded quantifiers are NFC_EUNSUP, syntax errors and empty-matching expressions
+    NFC_EINVAL -- decided by the host compiler before any CUDA call (R#33)."""
+    blob = np.frombuffer(rx, dtype=np.uint8).copy()
+    off = np.array([0, len(rx)], dtype=np.uint32)
+    act = np.zeros(1, dtype=np.uint8)
+    spec = nfc.DpiSpec(1, blob.ctypes.data, off.ctypes.data, act.ctypes.data)
+    h = ctypes.c_void_p()
+    assert nfc.lib.nfc_dpi_stream_create_regex(0, ctypes.byref(spec), 16, 0, ctypes.byref(h)) == getattr(nfc, code)

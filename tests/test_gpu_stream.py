@@ -161,3 +161,29 @@ def test_stream_fullsize_sampled_flows(nfc):
     assert [o for o in got if o[0] in selset] == want
     assert [gn[i] for i in sel] == wn and [gd[i] for i in sel] == wd
     assert sum(1 for i, j, e in want if e < len(pats[j]) - 1) > 10
+
+
+REGEXES = [b"[a-f][0-9]", b"(ab|cd)[^a-z]", b"\\.[A-Z]{2}", b"q.{3,5}z", b"[0-4]{3}", b"(x|y)?[kK]{2}",
+           b"\\x41\\x42?C", b"G(o|oo|ooo)gle"]
+EXAMPLES = [b"a7", b"cdX", b".QZ", b"q1234z", b"012", b"ykK", b"AC", b"Gooogle"]
+
+
+@pytest.mark.parametrize("calls", [[300, 1, 300]])
+def test_regex_stream_parity(nfc, calls):
+    """Regex DFA (host subset construction) walked by the stream kernels vs Python re."""
+    from oracle.stream_dpi import StreamRegexDPI
+    blob = np.frombuffer(b"".join(REGEXES), dtype=np.uint8).copy()
+    off = np.cumsum([0] + [len(r) for r in REGEXES]).astype(np.uint32)
+    act = np.array([0, 0, 1, 0, 0, 0, 1, 0], dtype=np.uint8)
+    ds = nfc.DpiStream(blob, off, act, max_flows=256, regex=True)
+    orc = StreamRegexDPI(REGEXES, list(act))
+    first = 0
+    for c, n in enumerate(calls):
+        sb = stream_batch(200 + c, n, 40, EXAMPLES, len_choices=[64, 96, 160], plant_frac=0.4,
+                          first_index=first, flow_seed=77)
+        want, wn, wd = orc.process(sb.frames(), first)
+        got, gn, gd, k = _gpu(ds, sb)
+        assert k == len(want) and got == want
+        assert gn == wn and gd == wd
+        first += n
+    assert len(want) > 50
