@@ -277,11 +277,25 @@ def run_stream(args):
     pkt_len = args.pkt_len or 64
     n = (args.ring_mb << 20) // ((pkt_len + 15) // 16 * 16)
     n_flows = 65536
-    rng = np.random.default_rng(4)
-    blob, poff, act = nfcgen.gen_patterns(rng, 100, lmin=4, lmax=16, drop_frac=0.05)
-    pats = nfcgen.Tables(pat_blob=blob, pat_off=poff, pat_action=act).patterns()
-    sb = stream_batch(9 + rank, n, n_flows, pats, pkt_len=pkt_len, plant_frac=0.05, flow_seed=1000 + rank)
-    ds = nfc.DpiStream(blob, poff, act, max_flows=2 * n_flows, device=local_dev)
+    regex = args.config == "S1R"
+    if regex:   # S1R: regular expressions (R#33); plants are example words of each expression
+        rx = [b"[a-f][0-9]{2}", b"(ab|cd)[^a-z]", b"\\.[A-Z]{2}", b"q.{3,5}z", b"[0-4]{4}", b"(x|y)?[kK]{3}",
+              b"\\x41\\x42?C[0-9]", b"G(o|oo|ooo)gle", b"(GET|POST) /[a-z]{1,8}", b"[Uu]ser-[Aa]gent: [A-Z]",
+              b"\\x90{4,8}", b"(cmd|exe)\\.[a-z]{3}", b"id=[0-9]{4,6}&", b"<scr(i|1)pt", b"%[0-9A-F]{2}%",
+              b"pass(wd|word)="]
+        ex = [b"a12", b"cdX", b".QZ", b"q1234z", b"0123", b"ykKk", b"AC7", b"Gooogle", b"GET /index",
+              b"User-Agent: M", b"\x90\x90\x90\x90", b"cmd.exe", b"id=12345&", b"<scr1pt", b"%2F%", b"password="]
+        blob = np.frombuffer(b"".join(rx), dtype=np.uint8).copy()
+        poff = np.cumsum([0] + [len(r) for r in rx]).astype(np.uint32)
+        act = np.array([0] * 13 + [1, 0, 1], dtype=np.uint8)
+        pats, plants = rx, ex
+    else:
+        rng = np.random.default_rng(4)
+        blob, poff, act = nfcgen.gen_patterns(rng, 100, lmin=4, lmax=16, drop_frac=0.05)
+        pats = nfcgen.Tables(pat_blob=blob, pat_off=poff, pat_action=act).patterns()
+        plants = pats
+    sb = stream_batch(9 + rank, n, n_flows, plants, pkt_len=pkt_len, plant_frac=0.05, flow_seed=1000 + rank)
+    ds = nfc.DpiStream(blob, poff, act, max_flows=2 * n_flows, device=local_dev, regex=regex)
     arena = torch.from_numpy(sb.arena).to(dev)
     off = torch.from_numpy(sb.off.astype(np.int64)).to(dev)
     ln = torch.from_numpy(sb.len.view(np.int16)).to(dev)
@@ -358,21 +372,24 @@ def run_stream(args):
                "api": "DpiStream.process_tensors (nfc_dpi_stream_process) + pinned host copies"}
     cpu = None
     if not args.no_cpu and rank == 0 and world == 1:
-        from oracle.stream_dpi import StreamDPI
-        orc = StreamDPI(pats, list(act))
-        frames = [sb.arena[int(o):int(o) + int(l)].tobytes() for o, l in zip(sb.off[:60000], sb.len[:60000])]
+        from oracle.stream_dpi import StreamDPI, StreamRegexDPI
+        orc = StreamRegexDPI(pats, list(act)) if regex else StreamDPI(pats, list(act))
+        ns = 6000 if regex else 60000
+        frames = [sb.arena[int(o):int(o) + int(l)].tobytes() for o, l in zip(sb.off[:ns], sb.len[:ns])]
         t0 = time.perf_counter()
         orc.process(frames)
         t = time.perf_counter() - t0
         cpu = {"value": round(len(frames) / t / 1e6, 6), "unit": "Mpps", "cores": 1, "kind": "oracle",
-               "sample": f"first {len(frames)} packets of S1 (brute-force Python stream oracle), {t:.1f} s, 1 thread"}
+               "sample": f"first {len(frames)} packets of {args.config} (brute-force Python stream oracle{' with re' if regex else ''}), {t:.1f} s, 1 thread"}
     if rank == 0:
         print(json.dumps({
             "metric": METRIC, "value": round(mpps, 3), "unit": "Mpps", "n_gpus": world, "steps": args.steps,
             "warmup": max(3, args.warmup), "ms_per_step": round(ms_max / args.steps, 4), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "gbps": round(n * pkt_len * 8 * args.steps * world / (ms_max / 1e3) / 1e9, 2),
-            "config": {"workload": f"S1: stateful cross-packet DPI (NEXT-4), 100 patterns, {pkt_len} B IPv4 "
+            "config": {"workload": f"S1R: stateful cross-packet regex DPI (NEXT-4, R#33), {len(pats)} expressions, {pkt_len} B IPv4 "
+                                   f"(30 % TCP), {n_flows} flows, 5 % cross-packet plants" if regex else
+                                   f"S1: stateful cross-packet DPI (NEXT-4), 100 patterns, {pkt_len} B IPv4 "
                                    f"(30 % TCP), {n_flows} flows, 5 % cross-packet plants",
                        "packets_per_step_per_gpu": n, "ring_bytes_per_gpu": len(sb.arena),
                        "l2": "ring >> 126 MB L2 (no flush needed)",
@@ -390,7 +407,7 @@ def main():
     args = parse_args()
     if args.impl == "reference":
         return run_reference(args)
-    if args.config == "S1":
+    if args.config in ("S1", "S1R"):
         return run_stream(args)
     import torch
     import torch.distributed as dist
