@@ -106,3 +106,62 @@ def test_merge_by_index_checks_partition():
         pdist.merge_by_index([a], 3, nfcgen.RESULT)
     with pytest.raises(ValueError):
         pdist.merge_by_index([a, a, b], 3, nfcgen.RESULT)
+
+
+def _stream_worker(rank, world, port, n, q):
+    """Stateful DPI sharded by the RSS hash: each rank sees whole flows (in order)."""
+    import torch.distributed as dist
+    from nfcgen.stream import stream_batch
+    from oracle.stream_dpi import StreamDPI
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        rng = np.random.default_rng(6)
+        blob, off, act = nfcgen.gen_patterns(rng, 30, lmin=2, lmax=8)
+        pats = nfcgen.Tables(pat_blob=blob, pat_off=off, pat_action=act).patterns()
+        outs = [None] * world
+        orc = StreamDPI(pats, list(act))
+        mine = []
+        for call in range(2):   # two calls: flow state carried per rank
+            sb = stream_batch(30 + call, n, 50, pats, plant_frac=0.3, first_index=call * n, flow_seed=3)
+            frames = sb.frames()
+            h = np.array([_tuple_hash(f) for f in frames])
+            idx = pdist.shard_indices(pdist.shard_of_hash(h, world), rank)
+            occ, nocc, drop = orc.process([frames[i] for i in idx])
+            mine += [(call * n + int(idx[i]), j, e) for i, j, e in occ]
+        dist.all_gather_object(outs, mine)
+        if rank == 0:
+            q.put(outs)
+    finally:
+        dist.destroy_process_group()
+
+
+def test_stream_dpi_flow_sharded_equals_single():
+    """NEXT-4 multi-GPU rule: sharding packets by the 5-tuple
+    RSS hash keeps every flow's stream on one rank, so the union of the per-rank
+    occurrences equals the single-process result -- no data-path collective."""
+    import torch.multiprocessing as mp
+    from nfcgen.stream import stream_batch
+    from oracle.stream_dpi import StreamDPI
+    n, world = 600, 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_stream_worker, args=(r, world, port, n, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    outs = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    rng = np.random.default_rng(6)
+    blob, off, act = nfcgen.gen_patterns(rng, 30, lmin=2, lmax=8)
+    pats = nfcgen.Tables(pat_blob=blob, pat_off=off, pat_action=act).patterns()
+    orc = StreamDPI(pats, list(act))
+    want = []
+    for call in range(2):
+        sb = stream_batch(30 + call, n, 50, pats, plant_frac=0.3, first_index=call * n, flow_seed=3)
+        occ, _, _ = orc.process(sb.frames(), call * n)
+        want += occ
+    assert all(len(o) > 0 for o in outs)
+    assert sorted(outs[0] + outs[1]) == sorted(want)
