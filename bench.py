@@ -338,8 +338,14 @@ def run_stream(args):
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
     peak = peaks.get("hbm_gbs", 6650.0)
     achieved = alg / (ms / args.steps / 1e3) / 1e9
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tfile) and not regex:
+        tj = json.load(open(tfile)).get("S1")
+        if tj and tj.get("packets"):
+            traffic = int(tj["dram_bytes_per_launch"] * n / tj["packets"])
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": None, "alg_bytes_per_launch": alg,
+            "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes_per_launch": alg,
             "alg_bytes_per_packet": round(alg / n, 2), "scope": "whole call (k_flow + radix sort + k_walk + k_commit)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING fallback"}
     # end to end: pinned host frames -> device, the call, per-packet verdicts + occurrences back
