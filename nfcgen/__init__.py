@@ -99,6 +99,16 @@ class TrafficParams:
     headroom: int = 0
     tailroom: int = 0
     l4csum: int = 0             # 1: arbitrary TCP/UDP checksum values (NAT updates them)
+    # valid edge-case frames (SURVEY 8(c)(i) parse cases), per million packets
+    opt_ppm: int = 0            # IPv4 options (IHL 6..15)
+    frag_ppm: int = 0           # IPv4 fragments (MF and/or offset): ports 0, L4 not parsed
+    tcpopt_ppm: int = 0         # TCP data offset 6..15
+    trailer_ppm: int = 0        # Ethernet trailer after the IP packet (1..46 B)
+
+    def edge(self, ppm: int = 100_000):
+        """Turn on every valid edge-case frame kind at `ppm` each (tests)."""
+        self.opt_ppm = self.frag_ppm = self.tcpopt_ppm = self.trailer_ppm = ppm
+        return self
 
 
 @dataclass
@@ -116,7 +126,7 @@ class _GenParams(ctypes.Structure):
     _fields_ = [("seed", ctypes.c_uint64), ("n_flows", ctypes.c_uint64)] + [
         (n, ctypes.c_uint32) for n in ("v6_bp", "pkt_len", "match_ppm", "in_acl_pct", "tcp_pct", "ttl",
                                        "ttl1_ppm", "malformed_ppm", "printable", "headroom", "tailroom",
-                                       "l4csum")]
+                                       "l4csum", "opt_ppm", "frag_ppm", "tcpopt_ppm", "trailer_ppm")]
 
 
 _P = ctypes.c_void_p
@@ -181,7 +191,8 @@ def _gen_structs(tp: TrafficParams, t: Tables):
     keep = _Keep()
     gp = _GenParams(tp.seed, tp.n_flows, tp.v6_bp, tp.pkt_len, tp.match_ppm, tp.in_acl_pct,
                     tp.tcp_pct, tp.ttl, tp.ttl1_ppm, tp.malformed_ppm, tp.printable,
-                    tp.headroom, tp.tailroom, tp.l4csum)
+                    tp.headroom, tp.tailroom, tp.l4csum, tp.opt_ppm, tp.frag_ppm, tp.tcpopt_ppm,
+                    tp.trailer_ppm)
     gt = _GenTables()
     if t.routes4 is not None and len(t.routes4):
         r4p = keep(t.routes4["prefix"].astype(np.uint32))

@@ -30,6 +30,11 @@ typedef struct {
     uint32_t printable;      /* payload bytes drawn from 0x20..0x7e */
     uint32_t headroom, tailroom;
     uint32_t l4csum;         /* 1: arbitrary (random) TCP/UDP checksum fields, 1/8 of UDP 0 = none */
+    /* valid edge-case frames (SURVEY 8(c)(i) parse cases), per million packets */
+    uint32_t opt_ppm;        /* IPv4 with options: IHL 6..15 */
+    uint32_t frag_ppm;       /* IPv4 fragments: MF set and/or non-zero fragment offset */
+    uint32_t tcpopt_ppm;     /* TCP with options: data offset 6..15 */
+    uint32_t trailer_ppm;    /* Ethernet trailer: IP length ends 1..46 B before the frame end */
 } gen_params;
 
 typedef struct {
@@ -42,7 +47,8 @@ typedef struct {
 } gen_tables;
 
 enum { S_FLOW = 1, S_FAM, S_INACL, S_RULE, S_SRC, S_DST, S_DST2, S_SP, S_DP, S_ROUTE, S_PROTO, S_LEN,
-       S_PAY, S_MATCH, S_PAT, S_POFF, S_TTL, S_BAD, S_BADK, S_SRC2, S_CSUM };
+       S_PAY, S_MATCH, S_PAT, S_POFF, S_TTL, S_BAD, S_BADK, S_SRC2, S_CSUM,
+       S_OPT, S_OPTN, S_FRAG, S_FRAGK, S_TOPT, S_TOPTN, S_TRL, S_TRLN, S_OPTB };
 
 static inline uint64_t mix64(uint64_t z)
 {
@@ -128,7 +134,21 @@ void nfcgen_flow(const gen_params *p, const gen_tables *t, uint64_t f, uint32_t 
     *proto = fl.proto;
 }
 
-static uint32_t frame_len(const gen_params *p, uint64_t i, int fam, uint8_t proto)
+/* Shape of packet i: IPv4 header words, TCP data offset, fragment kind, trailer bytes.
+ * With every edge ppm at 0 this is IHL 5 / data offset 5 / no fragment / no trailer. */
+typedef struct { uint32_t ihl, doff, frag, trailer; } shape_t;
+
+static shape_t pkt_shape(const gen_params *p, uint64_t i, int fam, uint8_t proto)
+{
+    shape_t s = {5, 5, 0, 0};
+    if (fam == 4 && (R(S_OPT, i) % 1000000) < p->opt_ppm) s.ihl = 6 + (uint32_t)(R(S_OPTN, i) % 10);
+    if (fam == 4 && (R(S_FRAG, i) % 1000000) < p->frag_ppm) s.frag = 1 + (uint32_t)(R(S_FRAGK, i) % 3);
+    if (proto == 6 && (R(S_TOPT, i) % 1000000) < p->tcpopt_ppm) s.doff = 6 + (uint32_t)(R(S_TOPTN, i) % 10);
+    if ((R(S_TRL, i) % 1000000) < p->trailer_ppm) s.trailer = 1 + (uint32_t)(R(S_TRLN, i) % 46);
+    return s;
+}
+
+static uint32_t frame_len(const gen_params *p, uint64_t i, int fam, uint8_t proto, shape_t *sh)
 {
     uint32_t L = p->pkt_len;
     if (L == 0) {
@@ -137,8 +157,11 @@ static uint32_t frame_len(const gen_params *p, uint64_t i, int fam, uint8_t prot
     } else if (L == 1) {
         L = 60 + (uint32_t)(R(S_LEN, i) % (1514 - 60 + 1)); /* uniform ragged lengths (tests) */
     }
-    uint32_t hdr = (fam == 4 ? 34 : 54) + (proto == 6 ? 20 : proto == 17 ? 8 : 0);
-    return L < hdr ? hdr : L;
+    *sh = pkt_shape(p, i, fam, proto);
+    uint32_t hdr = (fam == 4 ? 14 + 4 * sh->ihl : 54) + (proto == 6 ? 4 * sh->doff : proto == 17 ? 8 : 0);
+    if (L < hdr) L = hdr;
+    if (sh->trailer > L - hdr) sh->trailer = L - hdr;   /* the IP packet keeps its L4 header */
+    return L;
 }
 
 static uint64_t round16(uint64_t x) { return (x + 15) & ~15ull; }
@@ -152,7 +175,8 @@ uint64_t nfcgen_layout(const gen_params *p, const gen_tables *t, uint64_t first,
         uint64_t i = first + k;
         flow_t fl;
         make_flow(p, t, R(S_FLOW, i) % p->n_flows, &fl);
-        uint32_t L = frame_len(p, i, fl.fam, fl.proto);
+        shape_t sh;
+        uint32_t L = frame_len(p, i, fl.fam, fl.proto, &sh);
         off[k] = pos + p->headroom;
         len[k] = (uint16_t)L;
         pos += round16((uint64_t)p->headroom + L + p->tailroom);
@@ -173,25 +197,31 @@ void nfcgen_fill(const gen_params *p, const gen_tables *t, uint64_t first, uint3
         make_flow(p, t, R(S_FLOW, i) % p->n_flows, &fl);
         uint8_t *f = arena + off[k];
         uint32_t L = len[k];
+        shape_t sh;
+        (void)frame_len(p, i, fl.fam, fl.proto, &sh);
+        const uint32_t ip_end = L - sh.trailer;
         memcpy(f, mac_d, 6);
         memcpy(f + 6, mac_s, 6);
         uint32_t ttl = (R(S_TTL, i) % 1000000) < p->ttl1_ppm ? 1 : p->ttl;
         uint32_t l4;
         if (fl.fam == 4) {
             put16(f + 12, 0x0800);
-            f[14] = 0x45; f[15] = 0;
-            put16(f + 16, L - 14);
+            f[14] = (uint8_t)(0x40 | sh.ihl); f[15] = 0;
+            put16(f + 16, ip_end - 14);
             put16(f + 18, (uint32_t)(i & 0xffff));
-            put16(f + 20, 0x4000); /* DF, not a fragment */
+            /* DF, not a fragment; or a fragment: MF, a non-zero offset, or both */
+            const uint32_t fo = 1 + (uint32_t)(R(S_FRAGK, i) >> 8) % 0x1fff;
+            put16(f + 20, sh.frag == 0 ? 0x4000 : sh.frag == 1 ? 0x2000 : sh.frag == 2 ? fo : 0x2000 | fo);
             f[22] = (uint8_t)ttl; f[23] = fl.proto;
             f[24] = f[25] = 0;
             memcpy(f + 26, fl.src, 4);
             memcpy(f + 30, fl.dst, 4);
-            l4 = 34;
+            l4 = 14 + 4 * sh.ihl;
+            for (uint32_t j = 34; j < l4; j++) f[j] = (uint8_t)(R(S_OPTB, (i << 6) + j) & 0xff); /* options */
         } else {
             put16(f + 12, 0x86DD);
             f[14] = 0x60; f[15] = 0; f[16] = 0; f[17] = 0;
-            put16(f + 18, L - 54);
+            put16(f + 18, ip_end - 54);
             f[20] = fl.proto; f[21] = (uint8_t)ttl;
             memcpy(f + 22, fl.src, 16);
             memcpy(f + 38, fl.dst, 16);
@@ -203,15 +233,16 @@ void nfcgen_fill(const gen_params *p, const gen_tables *t, uint64_t first, uint3
         const uint32_t ck = p->l4csum ? (uint32_t)(rc & 0xffff) : 0;
         if (fl.proto == 17) {
             put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
-            put16(f + l4 + 4, L - l4); put16(f + l4 + 6, ((rc >> 16) & 7) == 0 ? 0 : ck);
+            put16(f + l4 + 4, ip_end - l4); put16(f + l4 + 6, ((rc >> 16) & 7) == 0 ? 0 : ck);
             pl = l4 + 8;
         } else if (fl.proto == 6) {
             put16(f + l4, fl.sp); put16(f + l4 + 2, fl.dp);
             uint64_t r = R(S_SP, i);
             for (int b = 0; b < 8; b++) f[l4 + 4 + b] = (uint8_t)(r >> (8 * b));
-            f[l4 + 12] = 0x50; f[l4 + 13] = 0x18;
+            f[l4 + 12] = (uint8_t)(sh.doff << 4); f[l4 + 13] = 0x18;
             put16(f + l4 + 14, 0xffff); put16(f + l4 + 16, ck); put16(f + l4 + 18, 0);
-            pl = l4 + 20;
+            for (uint32_t j = 20; j < 4 * sh.doff; j++) f[l4 + j] = (uint8_t)(R(S_OPTB, (i << 6) + j) >> 8); /* TCP options */
+            pl = l4 + 4 * sh.doff;
         }
         /* payload */
         for (uint32_t j = pl; j < L; j++) {
@@ -223,8 +254,8 @@ void nfcgen_fill(const gen_params *p, const gen_tables *t, uint64_t first, uint3
         if (t->n_pat && (R(S_MATCH, i) % 1000000) < p->match_ppm) {
             uint64_t pk = R(S_PAT, i) % t->n_pat;
             uint32_t plen = t->pat_off[pk + 1] - t->pat_off[pk];
-            if (pl + plen <= L) {
-                uint32_t o = pl + (uint32_t)(R(S_POFF, i) % (L - pl - plen + 1));
+            if (pl + plen <= ip_end) {
+                uint32_t o = pl + (uint32_t)(R(S_POFF, i) % (ip_end - pl - plen + 1));
                 memcpy(f + o, t->pat_blob + t->pat_off[pk], plen);
             }
         }

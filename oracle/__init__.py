@@ -82,6 +82,8 @@ def lib():
         L.or_lpm4.argtypes = [_P, ctypes.c_uint32]
         L.or_lpm6.restype = ctypes.c_int32
         L.or_lpm6.argtypes = [_P, _P]
+        L.or_parse.restype = ctypes.c_int
+        L.or_parse.argtypes = [_P, ctypes.c_int, _P]
         L.or_acl.restype = ctypes.c_int32
         L.or_acl.argtypes = [_P, ctypes.c_uint8, _P, _P, ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint8]
         _lib = L
@@ -128,6 +130,16 @@ def ipv4_checksum(hdr: bytes) -> int:
 def csum_update(hc: int, m: int, m1: int) -> int:
     """RFC 1624 eqn. 3 incremental checksum update (one 16-bit field m -> m1)."""
     return int(lib().or_csum_update(hc, m, m1))
+
+
+def parse(frame: bytes):
+    """The oracle's packet parse of one frame: None if the frame is
+    dropped by the parse, else dict(family, l4_off, ip_end, pl_off, proto, sport, dport)."""
+    out = (ctypes.c_int32 * 8)()
+    lib().or_parse(_buf(frame), len(frame), out)
+    if not out[0]:
+        return None
+    return dict(zip(("family", "l4_off", "ip_end", "pl_off", "proto", "sport", "dport"), list(out)[1:]))
 
 
 MS_RSS_KEY = bytes.fromhex("6d5a56da255b0ec24167253d43a38fb0d0ca2bcbae7b30b477cb2da38030f20c"

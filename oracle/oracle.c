@@ -507,6 +507,18 @@ static int parse(const uint8_t *f, int flen, pview *v)
     return 1;
 }
 
+/* Test hook: the parse above, exposed so the hand-built-frame pins of SURVEY
+ * 8(c)(i) can check every field.  out = {ok, family, l4_off, ip_end, pl_off,
+ * proto, sport, dport}. */
+int or_parse(const uint8_t *f, int flen, int32_t out[8])
+{
+    pview v;
+    int ok = parse(f, flen, &v);
+    out[0] = ok; out[1] = v.family; out[2] = v.l4_off; out[3] = v.ip_end; out[4] = v.pl_off;
+    out[5] = v.proto; out[6] = v.sport; out[7] = v.dport;
+    return ok;
+}
+
 static size_t tuple_bytes(const pview *v, uint8_t *t)
 {
     int al = v->family == 4 ? 4 : 16;

@@ -160,6 +160,9 @@ int32_t or_lpm6(or_chain *c, const uint8_t dst[16]);
 int32_t or_acl(or_chain *c, uint8_t family, const uint8_t *src, const uint8_t *dst,
                uint16_t sport, uint16_t dport, uint8_t proto);
 
+/* Parse of SURVEY 8(c)(i) 1 (test hook): out = {ok, family, l4_off, ip_end, pl_off, proto, sport, dport}. */
+int or_parse(const uint8_t *f, int flen, int32_t out[8]);
+
 #ifdef __cplusplus
 }
 #endif
