@@ -251,13 +251,37 @@ NFC_API int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes,
  * LB per-backend hits and per-SA ESP packets.  Same sequential semantics as
  * the per-packet records. */
 #define NFC_STATS_RESET 1u
+#define NFC_STATS_ALLREDUCE 2u   /* sum the vector over the ranks of the attached comm  */
 
 NFC_API int nfc_stats_len(const nfc_chain *c, size_t *len);
-/* Synchronizes the device, copies min(cap, len) counters to out (host) and
- * optionally resets them.  Returns NFC_ECAP if match pairs were dropped for
- * capacity since the last reset.  Multi-GPU sums are taken by the caller
- * (one all-reduce of this vector over NCCL). */
+/* Synchronizes the stream of the chain's last nfc_process_batch / nfc_process_host
+ * call (not the whole device), copies min(cap, len) counters to out (host) and
+ * optionally resets this GPU's counters (NFC_STATS_RESET).  With
+ * NFC_STATS_ALLREDUCE the vector written to out is the sum over every rank of the
+ * communicator attached with nfc_attach_comm (one ncclAllReduce(ncclUint64,
+ * ncclSum) on that stream: flows shard by RSS hash, so the
+ * counters are the only exchange); every rank must make the call (collective),
+ * and NFC_ESTATE is returned if no communicator is attached.  Returns NFC_ECAP if
+ * match pairs were dropped for capacity since the last reset (on any rank, with
+ * NFC_STATS_ALLREDUCE). */
 NFC_API int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags);
+
+/* ---------------------------------------------------------------- multi-GPU
+ * One process (or thread) per GPU, one chain per GPU, flows sharded with
+ * nfc_rss_shard (below); the library's only collective is the counter sum of
+ * nfc_collect_stats.  NCCL (libnccl.so.2) is loaded on first use of these calls;
+ * NFC_ESTATE if it cannot be loaded, NFC_ECUDA (message from NCCL) if a call fails. */
+#define NFC_COMM_ID_BYTES 128
+/* Rank 0 creates the communicator id (ncclGetUniqueId) and hands the 128 bytes to
+ * the other ranks out of band (e.g. a torch.distributed broadcast). */
+NFC_API int nfc_comm_unique_id(uint8_t *id, size_t id_bytes);
+/* ncclCommInitRank on `device` (collective over nranks ranks); *comm receives the
+ * ncclComm_t, owned by the caller (nfc_comm_destroy). */
+NFC_API int nfc_comm_init(int device, int nranks, int rank, const uint8_t *id, void **comm);
+NFC_API int nfc_comm_destroy(void *comm);
+/* Attach an ncclComm_t (from nfc_comm_init or the caller's own NCCL) to the chain
+ * for NFC_STATS_ALLREDUCE; NULL detaches.  The chain does not own it. */
+NFC_API int nfc_attach_comm(nfc_chain *c, void *nccl_comm);
 
 /* Receive Side Steering for multi-GPU sharding (P:L87 RSS model): shard[i] =
  * RETA[Toeplitz(MS default key, src|dst|sport|dport of frame i) & 127], RETA[j] =

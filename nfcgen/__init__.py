@@ -143,7 +143,8 @@ class _GenTables(ctypes.Structure):
 
 def build_lib(force: bool = False) -> str:
     src = os.path.join(HERE, "gen.c")
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(src):
+    newest = max(os.path.getmtime(src), os.path.getmtime(os.path.join(HERE, "gen_core.h")))
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < newest:
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", _LIB, src])
     return _LIB
 

@@ -21,7 +21,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
 def sources():
-    s = ["capi.cu", "sfc_kernel.cu", "unfused.cu", "builders.cpp", "debug_host.cpp", "planner.cpp", "parallel.cu", "dpi_stream.cu", "regex.cpp"]
+    s = ["capi.cu", "sfc_kernel.cu", "unfused.cu", "builders.cpp", "debug_host.cpp", "planner.cpp", "parallel.cu", "dpi_stream.cu", "regex.cpp", "comm.cu"]
     s += sorted(os.path.basename(p) for p in glob.glob(os.path.join(CSRC, "sfc_inst_*.cu")))
     return s
 
@@ -63,7 +63,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out=None) -> s
         if verbose:
             sys.stderr.write(f"== {src}\n" + r.stderr)
     objs = [o for _, o, _ in results]
-    link = [NVCC, *ARCH, "-shared", "-o", target + ".tmp", *objs]
+    link = [NVCC, *ARCH, "-shared", "-o", target + ".tmp", *objs, "-ldl"]
     r = subprocess.run(link, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

@@ -88,13 +88,15 @@ struct nfc_chain {
     uint32_t stats_len = ST_VAR_BASE;
     uint32_t n_acl_rules = 0, n_lb = 0, n_sa = 0;
     // scheduling
-    DBuf counter, tile_flag, tile_vec, batches;
+    DBuf counter, tile_flag, tile_vec, batches, crec;
     uint32_t tile_cap = 0;
     uint32_t epoch = 0;
     // host e2e staging
     DBuf h_arena, h_off, h_len, h_rec, h_mp, h_mq, h_mc;
     uint64_t launches = 0;
     cudaStream_t last_stream = nullptr;
+    void *comm = nullptr;                 // attached ncclComm_t (NFC_STATS_ALLREDUCE)
+    DBuf stats_red;                       // all-reduce destination
 };
 
 static int set_device(const nfc_chain *c)
@@ -168,7 +170,7 @@ void nfc_destroy_chain(nfc_chain *c)
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->nat_pool, &c->nat_dnat, &c->nat_nib,
                    &c->stats, &c->counter,
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
-                   &c->h_mp, &c->h_mq, &c->h_mc};
+                   &c->h_mp, &c->h_mq, &c->h_mc, &c->stats_red, &c->crec};
     for (DBuf *b : all) b->release();
     delete c;
 }
@@ -489,6 +491,14 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         return NFC_OK;
     }
     LaunchCfg lc{};
+    if (!par && nb > 1 && !(c->mask & MASK_IPSEC)) {
+        // multi-batch call: per-chunk descriptor records for the pipelined warp loop
+        CK(c->crec.reserve((size_t)((total + 31) / 32) * sizeof(ChunkRec)));
+        rc = chunk_recs_launch(p.batches, nb, (uint32_t)total, c->crec.as<ChunkRec>(), st, err);
+        if (rc) return fail(rc, err);
+        p.crec = c->crec.as<ChunkRec>();
+        c->launches++;
+    }
     rc = par ? par_launch(p, c->device, st, err, &lc) : sfc_launch(v, p, c->device, st, err, &lc);
     if (rc) return fail(rc, err);
     c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
@@ -554,15 +564,34 @@ int nfc_stats_len(const nfc_chain *c, size_t *len)
 int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags)
 {
     if (!c || (!out && cap)) return fail(NFC_EINVAL, "NULL argument");
+    if (flags & ~(NFC_STATS_RESET | NFC_STATS_ALLREDUCE)) return fail(NFC_EINVAL, "unknown stats flags");
+    if ((flags & NFC_STATS_ALLREDUCE) && !c->comm) return fail(NFC_ESTATE, "NFC_STATS_ALLREDUCE without an attached comm");
     int rc = set_device(c);
     if (rc) return rc;
-    CK(cudaDeviceSynchronize());
+    cudaStream_t st = c->last_stream;
+    const size_t bytes = (size_t)c->stats_len * 8;
+    const void *src = c->stats.p;
+    if (flags & NFC_STATS_ALLREDUCE) {
+        CK(c->stats_red.reserve(bytes));
+        CK(cudaMemcpyAsync(c->stats_red.p, c->stats.p, bytes, cudaMemcpyDeviceToDevice, st));
+        rc = comm_allreduce_u64(c->comm, c->stats_red.as<unsigned long long>(), c->stats_len, st);
+        if (rc) return rc;
+        src = c->stats_red.p;
+    }
     std::vector<uint64_t> h(c->stats_len);
-    CK(cudaMemcpy(h.data(), c->stats.p, (size_t)c->stats_len * 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpyAsync(h.data(), src, bytes, cudaMemcpyDeviceToHost, st));
+    if (flags & NFC_STATS_RESET) CK(cudaMemsetAsync(c->stats.p, 0, bytes, st));
+    CK(cudaStreamSynchronize(st));
     size_t k = cap < h.size() ? cap : h.size();
     if (k) memcpy(out, h.data(), k * 8);
-    if (flags & NFC_STATS_RESET) CK(cudaMemset(c->stats.p, 0, (size_t)c->stats_len * 8));
     if (h[ST_MATCH_OVF]) return fail(NFC_ECAP, "match pairs exceeded match_cap");
+    return NFC_OK;
+}
+
+int nfc_attach_comm(nfc_chain *c, void *nccl_comm)
+{
+    if (!c) return fail(NFC_EINVAL, "chain is NULL");
+    c->comm = nccl_comm;
     return NFC_OK;
 }
 

@@ -155,6 +155,13 @@ struct NatImg {
 
 // ---------------------------------------------------------------- launch
 struct BatchDev { uint8_t *arena; const uint64_t *off; const uint16_t *len; uint32_t n; uint32_t start; uint64_t first; };
+// Multi-batch calls: one 32-B record per 32-packet chunk (built on the device by
+// k_chunk_recs before the fused kernel), for the batch of the chunk's first packet:
+// packet g of that batch has off = offp[g], len = lenp[g], bytes at arena + off and
+// global index gb + g.  meta = lane where the next batch starts (0: none) | 1<<5 if
+// the chunk holds more than one batch boundary (those lanes take the binary search).
+struct ChunkRec { const uint64_t *offp; const uint16_t *lenp; uint8_t *arena; uint32_t gb_lo, meta; };  // gb_lo: first - start (diagnostic)
+static_assert(sizeof(ChunkRec) == 32, "ChunkRec is 32 B");
 
 enum { MASK_ACL = 1u << NFC_ACL, MASK_DPI = 1u << NFC_DPI, MASK_LPM4 = 1u << NFC_LPM4,
        MASK_LPM6 = 1u << NFC_LPM6, MASK_IPSEC = 1u << NFC_IPSEC, MASK_LB = 1u << NFC_LB,
@@ -188,6 +195,7 @@ struct KParams {
     uint32_t n_pkts;
     uint32_t n_tiles;
     uint32_t claim;              // 32-packet chunks per work claim (set by the launcher)
+    const ChunkRec *crec;        // n_batches > 1: one record per 32-packet chunk (else nullptr)
     uint32_t *tile_counter;
     // outputs
     nfc_pkt_result *rec;
@@ -217,6 +225,8 @@ struct KParams {
 
 // host-side builders (builders.cpp); return "" on success or an error message
 int set_fail(int code, const std::string &msg);
+// comm.cu: in-place u64 sum across the ranks of an NCCL communicator, on st
+int comm_allreduce_u64(void *comm, unsigned long long *dev, size_t n, cudaStream_t st);
 struct DpiHost;
 std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states);   // regex.cpp   // capi.cu: nfc_last_error + code
 struct HostImage { std::vector<uint8_t> bytes; };
@@ -284,6 +294,9 @@ struct LaunchCfg { int grid, block; size_t smem; };
 enum { DM_HOT = 1, DM_FULL = 2 };
 struct Variant { uint32_t sig; int dm; int threads; bool esp; };
 Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full);
+// records of every 32-packet chunk of a multi-batch call (ChunkRec), on `stream`
+int chunk_recs_launch(const BatchDev *batches, uint32_t n_batches, uint32_t n_pkts, ChunkRec *out, void *stream,
+                      std::string &err);
 int sfc_launch(const Variant &v, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
 size_t sfc_smem_bytes(const Variant &v, const KParams &p);
 size_t sfc_smem_limit(int device);      // max dynamic shared memory per CTA (opt-in)

@@ -96,7 +96,7 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
                     } else if (wk.cnt >= 1) {                             // exact set: DROP flag only
                         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt,
                                         P.match_pat, P.match_cap, P.stats, 0u};
-                        drop = (dpi_slow<DM_HOT>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx) >> 31) != 0;
+                        drop = (dpi_slow<DM_HOT>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, pkt_gidx(P, k.g)) >> 31) != 0;
                     }
                     x = (uint32_t)drop << 16;
                 } else if (kind == NFC_LPM4 || kind == NFC_LPM6) {

@@ -90,6 +90,49 @@ int sfc_query(const Variant &v, const KParams &p, int device, LaunchCfg *cfg_out
     return dispatch(v, p, device, nullptr, err, cfg_out, true);
 }
 
+// ---------------------------------------------------------------- multi-batch chunk records
+// One thread per 32-packet chunk: the batch holding the chunk's first packet (binary
+// search over the batch starts; among equal starts the last batch, i.e. the non-empty
+// one), its descriptor pointers rebased so that packet g of the call indexes them
+// directly, and where the next batch begins inside the chunk (ChunkRec).
+__global__ void k_chunk_recs(const BatchDev *B, uint32_t nb, uint32_t n, ChunkRec *out)
+{
+    const uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t g0 = c * 32;
+    if (g0 >= n) return;
+    uint32_t lo = 0, hi = nb - 1;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (B[mid].start <= g0) lo = mid; else hi = mid - 1;
+    }
+    const BatchDev b = B[lo];
+    const uint32_t end = min(g0 + 32, n);
+    uint32_t split = 0, cnt = 0;
+    for (uint32_t j = lo + 1; j < nb && B[j].start < end; j++)
+        if (B[j].n) {
+            if (!cnt) split = B[j].start - g0;
+            cnt++;
+        }
+    ChunkRec r;
+    r.offp = b.off - b.start;
+    r.lenp = b.len - b.start;
+    r.arena = b.arena;
+    r.gb_lo = (uint32_t)b.first - b.start;
+    r.meta = split | (cnt > 1 ? 32u : 0u);
+    out[c] = r;
+}
+
+int chunk_recs_launch(const BatchDev *batches, uint32_t n_batches, uint32_t n_pkts, ChunkRec *out, void *stream,
+                      std::string &err)
+{
+    const uint32_t chunks = (n_pkts + 31) / 32;
+    if (!chunks) return NFC_OK;
+    k_chunk_recs<<<(chunks + 255) / 256, 256, 0, (cudaStream_t)stream>>>(batches, n_batches, n_pkts, out);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { err = std::string("k_chunk_recs: ") + cudaGetErrorString(e); return NFC_ECUDA; }
+    return NFC_OK;
+}
+
 // ---------------------------------------------------------------- RSS steering
 // Receive Side Steering: shard = RETA[Toeplitz(MS key, src|dst|sport|dport) & 127]
 // with RETA[i] = i mod n_shards.  For n_shards | 64 every ESP SA (hash mod n_sa, n_sa = 64)

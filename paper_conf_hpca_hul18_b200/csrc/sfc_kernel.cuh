@@ -1370,7 +1370,7 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
 struct Pkt {
     uint8_t *f;
     uint32_t flen, orig_len;
-    uint64_t gidx;
+    uint32_t g;               // index of the packet within the call (global index: pkt_gidx)
     uint32_t h[16];
     PV v;
     uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
@@ -1397,7 +1397,7 @@ __device__ __forceinline__ void var_stat(const KParams &P, const Ctx &C, uint32_
     else atomicAdd(&P.stats[idx], 1ull);
 }
 
-struct Loc { uint8_t *f; uint32_t len; uint64_t gidx; };
+struct Loc { uint8_t *f; uint32_t len; uint32_t g; };
 struct Raw { uint64_t off; uint32_t len, bi; };   // a packet's descriptor loads (issued early)
 
 // batch of packet g (binary search over batch starts) and its off/len loads
@@ -1427,14 +1427,62 @@ __device__ __forceinline__ Loc pkt_loc(const KParams &P, const Raw &r, uint32_t 
     if (!valid) return l;
     if (P.n_batches == 1) {
         l.f = P.b0.arena + r.off;
-        l.gidx = P.b0.first + g;
     } else {
         const BatchDev &B = P.batches[r.bi];
         l.f = B.arena + r.off;
-        l.gidx = B.first + (g - B.start);
     }
     l.len = r.len;
+    l.g = g;
     return l;
+}
+// Global packet index (low 32 bits: match-pair packet ids) of packet g of the call;
+// only lanes that emit match pairs ask, so it is looked up instead of carried
+static __device__ __noinline__ uint32_t gidx_search(const BatchDev *bs, uint32_t nb, uint32_t g)
+{
+    uint32_t lo = 0, hi = nb - 1;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (bs[mid].start <= g) lo = mid; else hi = mid - 1;
+    }
+    return (uint32_t)bs[lo].first + (g - bs[lo].start);
+}
+__device__ __forceinline__ uint32_t pkt_gidx(const KParams &P, uint32_t g)
+{
+    return P.n_batches == 1 ? (uint32_t)P.b0.first + g : gidx_search(P.batches, P.n_batches, g);
+}
+
+// arena base of chunk c's descriptors in the pipelined loop (desc_get offsets are relative to it)
+__device__ __forceinline__ uint8_t *chunk_arena(const KParams &P, uint32_t c)
+{
+    if (P.n_batches == 1) return P.b0.arena;
+    return reinterpret_cast<uint8_t *>(__ldg(reinterpret_cast<const unsigned long long *>(&P.crec[c >> 5].arena)));
+}
+
+// descriptors of packet g for the pipelined loop: frame offset relative to chunk_arena
+// of its chunk, and length; single batch from the constant bank, multi-batch from the
+// chunk record (ChunkRec) -- lanes past a batch boundary in the chunk take the binary
+// search and rebase their offset onto the chunk's arena
+__device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t &off, uint32_t &len)
+{
+    if (P.n_batches == 1) {
+        off = P.b0.off[g];
+        len = P.b0.len[g];
+        return;
+    }
+    const uint4 *r = reinterpret_cast<const uint4 *>(P.crec + (g >> 5));
+    const uint4 a = __ldg(r), b = __ldg(r + 1);
+    const uint32_t split = b.w & 31, lane = g & 31;
+    if ((b.w & 32) || (split && lane >= split)) {
+        const Raw w = pkt_raw(P, g, true);
+        const uint64_t base = (uint64_t)b.x | (uint64_t)b.y << 32;
+        off = (uint64_t)P.batches[w.bi].arena + w.off - base;
+        len = w.len;
+        return;
+    }
+    const uint64_t *offp = reinterpret_cast<const uint64_t *>((uint64_t)a.x | (uint64_t)a.y << 32);
+    const uint16_t *lenp = reinterpret_cast<const uint16_t *>((uint64_t)a.z | (uint64_t)a.w << 32);
+    off = offp[g];
+    len = lenp[g];
 }
 __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
 {
@@ -1445,7 +1493,7 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
-    k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
+    k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
     if (!valid) return;
     load_header(k.f, k.flen, k.h, C.pol_f);
@@ -1458,7 +1506,7 @@ __device__ __forceinline__ void pkt_begin_h(const Loc &l, bool valid, Pkt &k, co
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
-    k.f = l.f; k.flen = k.orig_len = l.len; k.gidx = l.gidx;
+    k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
     if (!valid) return;
 #pragma unroll
@@ -1499,11 +1547,11 @@ __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &
         k.nmatch = nm;
         dropped = (meta >> 31) != 0;
         // (per-lane path: emitted at once -- the unfused and parallel kernels have no pkt_end)
-        emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), (uint32_t)k.gidx);
+        emit_pairs(P, meta & 0xFFFFF, nm, atomicAdd(P.match_count, nm), pkt_gidx(P, k.g));
     } else if (w.cnt >= 1) {
         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                         P.match_cap, P.stats, 1u};
-        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, pkt_gidx(P, k.g));
         k.nmatch = r & 0x7FFFFFFFu;
         dropped = (r >> 31) != 0;
     }
@@ -1549,7 +1597,7 @@ __device__ __forceinline__ bool dpi_finish_warp(const KParams &P, const Ctx &C, 
         k.mmeta = nm ? meta & 0x7FFFFFFFu : 0u;
 #else
         base = __shfl_sync(FULL, base, 0);
-        if (nm) emit_pairs(P, meta & 0xFFFFF, nm, base + excl, (uint32_t)k.gidx);
+        if (nm) emit_pairs(P, meta & 0xFFFFF, nm, base + excl, pkt_gidx(P, k.g));
 #endif
     }
     if (single) {
@@ -1558,7 +1606,7 @@ __device__ __forceinline__ bool dpi_finish_warp(const KParams &P, const Ctx &C, 
     } else if (act && w.cnt >= 1) {
         const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt, P.match_pat,
                         P.match_cap, P.stats, 1u};
-        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, (uint32_t)k.gidx);
+        const uint32_t r = dpi_slow<DM>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, pkt_gidx(P, k.g));
         k.nmatch = r & 0x7FFFFFFFu;
         dropped = (r >> 31) != 0;
     }
@@ -1939,7 +1987,7 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
         // k.mslot; per-lane claims keep the absolute slot in k.mslot and k.mbase = 0
         if (__any_sync(0xFFFFFFFFu, k.mmeta != 0)) {
             const uint32_t b0 = __shfl_sync(0xFFFFFFFFu, k.mbase, 0);
-            if (k.mmeta) emit_pairs(P, k.mmeta & 0xFFFFF, k.mmeta >> 20, b0 + k.mslot, (uint32_t)k.gidx);
+            if (k.mmeta) emit_pairs(P, k.mmeta & 0xFFFFF, k.mmeta >> 20, b0 + k.mslot, pkt_gidx(P, k.g));
         }
     }
     if (valid) {
@@ -2230,9 +2278,13 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // descriptors (off/len) are prefetched into L1 two chunks ahead -- no registers held
         // across a chunk -- and re-loaded (L1 hits) when the frame prefetch and the chunk need them
         auto desc_l1 = [&](uint32_t g) {
-            if (P.n_batches == 1 && g < P.n_pkts) {
-                asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.off + g));
-                asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.len + g));
+            if (g < P.n_pkts) {
+                if (P.n_batches == 1) {
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.off + g));
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.len + g));
+                } else if (P.crec && lane == 0) {
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(P.crec + (g >> 5)));
+                }
             }
         };
         desc_l1(c0 + lane);
@@ -2242,24 +2294,26 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         if (c0 + lane < P.n_pkts) { const Loc l0 = pkt_locate(P, c0 + lane, true); load_header(l0.f, l0.len, hn, C.pol_f); }
 #endif
 #if NFC_CARRY_DESC
-        // single batch: the next chunk's off/len are read at the top of the current one and
-        // carried into it, so its header loads issue without a descriptor round trip
+        // the next chunk's descriptors (off/len; multi-batch calls: from its chunk record)
+        // are read at the top of the current one and carried into it, so its header loads
+        // issue without a descriptor round trip
         uint64_t off0 = 0;
         uint32_t len0 = 0;
-        if (P.n_batches == 1 && c0 + lane < P.n_pkts) { off0 = P.b0.off[c0 + lane]; len0 = P.b0.len[c0 + lane]; }
+        const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && (P.n_batches == 1 || P.crec != nullptr);   // warp-uniform
+        if (late && c0 + lane < P.n_pkts) desc_get(P, c0 + lane, off0, len0);
+#else
+        const bool late = false;
 #endif
         while (c0 < P.n_pkts) {
             Loc l1{nullptr, 0, 0};
-            const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && P.n_batches == 1;   // warp-uniform
             uint64_t off1 = 0;
 #if NFC_CARRY_DESC
             uint32_t len1 = 0;
 #endif
             if (c1 + lane < P.n_pkts) {
                 if (late) {
-                    off1 = P.b0.off[c1 + lane];        // consumed after the head part (below)
 #if NFC_CARRY_DESC
-                    len1 = P.b0.len[c1 + lane];
+                    desc_get(P, c1 + lane, off1, len1);   // consumed after the head part (below)
 #endif
                 } else {
                     l1 = pkt_locate(P, c1 + lane, true);
@@ -2274,13 +2328,15 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 #if NFC_HDR_AHEAD
             pkt_begin_h(pkt_locate(P, g, valid), valid, k, hn);
 #elif NFC_CARRY_DESC
-            if (late) pkt_begin(C, Loc{P.b0.arena + off0, len0, P.b0.first + g}, valid, k);
+            if (late) pkt_begin(C, Loc{chunk_arena(P, c0) + off0, len0, g}, valid, k);
             else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #else
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #endif
             run_part<S, DM, true>(P, C, k);
-            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(P.b0.arena + off1));
+#if NFC_CARRY_DESC
+            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(chunk_arena(P, c1) + off1));
+#endif
             run_part<S, DM, false>(P, C, k);
 #if NFC_HDR_AHEAD
             if (c1 + lane < P.n_pkts) load_header(l1.f, l1.len, hn, C.pol_f);

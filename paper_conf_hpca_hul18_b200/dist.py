@@ -57,6 +57,19 @@ def max_over_ranks(x: float, device=None, group=None) -> float:
     return float(t.item())
 
 
+def library_comm(device: int):
+    """The library's own NCCL communicator for this rank (nfc_comm_init): rank 0 makes
+    the id (nfc_comm_unique_id) and torch.distributed broadcasts it.  Attach it to a
+    chain with Chain.attach_comm; Chain.stats(allreduce=True) then sums the counters
+    of every rank with one ncclAllReduce inside the library."""
+    import torch.distributed as dist
+    from paper_conf_hpca_hul18_b200 import nfc
+    rank, world = dist.get_rank(), dist.get_world_size()
+    box = [nfc.comm_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(box, src=0)
+    return nfc.Comm(device, world, rank, box[0])
+
+
 def merge_by_index(parts, n_total: int, dtype) -> np.ndarray:
     """parts = [(global_indices, records)] from every rank -> records in global order."""
     out = np.zeros(n_total, dtype=dtype)

@@ -19,6 +19,8 @@ NFC_OK, NFC_EINVAL, NFC_ENOMEM, NFC_ECUDA, NFC_ESTATE, NFC_ECAP, NFC_EUNSUP = 0,
 ACL, DPI, LPM4, LPM6, IPSEC, LB, NAT = 1, 2, 3, 4, 5, 6, 7
 KINDS = {"ACL": ACL, "DPI": DPI, "LPM4": LPM4, "LPM6": LPM6, "IPSEC": IPSEC, "LB": LB, "NAT": NAT}
 STATS_RESET = 1
+STATS_ALLREDUCE = 2   # nfc_collect_stats: sum over the ranks of the attached NCCL comm
+COMM_ID_BYTES = 128
 F_UNFUSED = 1   # nfc_chain_opts.flags: per-NF kernels with re-split (NEXT-1 baseline)
 F_PARALLEL = 2  # nfc_chain_opts.flags: the chain's NFs on different warps + XOR merge (NEXT-2)
 
@@ -90,7 +92,8 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_process_batch", "nfc_process_host", "nfc_stats_len", "nfc_collect_stats",
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard",
            "nfc_dpi_stream_create", "nfc_dpi_stream_create_regex", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
-           "nfc_dpi_stream_process", "nfc_dpi_stream_flows"]
+           "nfc_dpi_stream_process", "nfc_dpi_stream_flows", "nfc_comm_unique_id", "nfc_comm_init",
+           "nfc_comm_destroy", "nfc_attach_comm"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
@@ -122,6 +125,10 @@ def _load_lib():
     L.nfc_dpi_stream_reset.argtypes = [_P, _P]
     L.nfc_dpi_stream_process.argtypes = [_P, ctypes.POINTER(Batch), ctypes.POINTER(StreamResult), _P]
     L.nfc_dpi_stream_flows.argtypes = [_P, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+    L.nfc_comm_unique_id.argtypes = [_P, ctypes.c_size_t]
+    L.nfc_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, _P, ctypes.POINTER(_P)]
+    L.nfc_comm_destroy.argtypes = [_P]
+    L.nfc_attach_comm.argtypes = [_P, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
     P32 = ctypes.POINTER(_u32)
@@ -294,13 +301,20 @@ class Chain:
                                     rec_ptr, mp_ptr, mq_ptr, match_cap, ctypes.byref(npairs), stream or None))
         return npairs.value
 
-    def stats(self, reset: bool = False, allow_cap: bool = True) -> np.ndarray:
+    def stats(self, reset: bool = False, allow_cap: bool = True, allreduce: bool = False) -> np.ndarray:
+        """nfc_collect_stats; allreduce=True sums over the ranks of the attached comm."""
         n = ctypes.c_size_t()
         _check(lib.nfc_stats_len(self.h, ctypes.byref(n)))
         out = np.zeros(n.value, dtype=np.uint64)
-        _check(lib.nfc_collect_stats(self.h, out.ctypes.data, n.value, STATS_RESET if reset else 0),
+        flags = (STATS_RESET if reset else 0) | (STATS_ALLREDUCE if allreduce else 0)
+        _check(lib.nfc_collect_stats(self.h, out.ctypes.data, n.value, flags),
                allow=(NFC_ECAP,) if allow_cap else ())
         return out
+
+    def attach_comm(self, comm: Optional["Comm"]):
+        """nfc_attach_comm: the NCCL communicator NFC_STATS_ALLREDUCE sums over (None detaches)."""
+        self._comm = comm
+        _check(lib.nfc_attach_comm(self.h, comm.h if comm is not None else None))
 
     def launches(self) -> int:
         c = ctypes.c_uint64()
@@ -378,6 +392,28 @@ class DpiStream:
         nf, nu = ctypes.c_uint64(), ctypes.c_uint64()
         _check(lib.nfc_dpi_stream_flows(self.h, ctypes.byref(nf), ctypes.byref(nu)))
         return nf.value, nu.value
+
+
+def comm_unique_id() -> bytes:
+    """nfc_comm_unique_id (ncclGetUniqueId): rank 0 makes it, the others receive it out of band."""
+    b = ctypes.create_string_buffer(COMM_ID_BYTES)
+    _check(lib.nfc_comm_unique_id(b, COMM_ID_BYTES))
+    return b.raw
+
+
+class Comm:
+    """An NCCL communicator made by the library (nfc_comm_init); one per rank/GPU."""
+
+    def __init__(self, device: int, nranks: int, rank: int, uid: bytes):
+        assert len(uid) == COMM_ID_BYTES
+        h = _P()
+        _check(lib.nfc_comm_init(device, nranks, rank, _cbuf(uid), ctypes.byref(h)))
+        self.h = h.value
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.nfc_comm_destroy(self.h)
+            self.h = None
 
 
 def rss_shard(device: int, arena_ptr: int, off_ptr: int, len_ptr: int, n: int, n_shards: int, out_ptr: int,

@@ -73,3 +73,41 @@ def test_sharded_chains_equal_single_stream(wl, plen):
         for i in range(len(stats)):
             if i != 11:
                 assert stats[i] == orc.stats[i], (N, i)
+
+
+def test_library_nccl_comm_allreduce_one_rank():
+    """nfc_comm_unique_id / nfc_comm_init / nfc_attach_comm / NFC_STATS_ALLREDUCE with a
+    one-rank NCCL communicator (the only shape one GPU allows): the all-reduced vector is
+    the local one, RESET clears the local counters, and ALLREDUCE without a comm is
+    NFC_ESTATE."""
+    import torch
+    from paper_conf_hpca_hul18_b200 import nfc
+    w = nfcgen.workload("C1", small=True)
+    ch = nfc.Chain(w.kinds, device=0)
+    ch.load_tables(w.tables)
+    b = nfcgen.generate(w.traffic, w.tables, 0, 3000)
+    dev = torch.device("cuda", 0)
+    arena = torch.from_numpy(b.arena).to(dev)
+    off = torch.from_numpy(b.off.view(np.int64)).to(dev)
+    ln = torch.from_numpy(b.len.view(np.int16)).to(dev)
+    rec = torch.zeros((b.n, 16), dtype=torch.uint8, device=dev)
+    mp = torch.zeros(1 << 14, dtype=torch.int32, device=dev)
+    mq = torch.zeros(1 << 14, dtype=torch.int16, device=dev)
+    mc = torch.zeros(1, dtype=torch.int32, device=dev)
+    ch.process_tensors(arena, off, ln, rec, mp, mq, mc)
+    with pytest.raises(nfc.NfcError) as e:
+        ch.stats(allreduce=True)
+    assert e.value.code == nfc.NFC_ESTATE
+    comm = nfc.Comm(0, 1, 0, nfc.comm_unique_id())
+    ch.attach_comm(comm)
+    local = ch.stats()
+    red = ch.stats(allreduce=True, reset=True)
+    assert np.array_equal(local, red) and local[0] == b.n
+    assert ch.stats().sum() == 0
+    orc = oracle.OracleChain(w.kinds, w.tables)
+    orc.run(b)
+    for i in range(len(red)):
+        if i != 11:
+            assert red[i] == orc.stats[i], i
+    ch.attach_comm(None)
+    comm.close()

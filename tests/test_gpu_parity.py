@@ -254,3 +254,51 @@ def test_n3_unfused_and_nat_only(nfc):
     w3 = nfcgen.workload("N3", acl_rules=200, pkt_len=64)
     w3.tables.nat_ext_ports = 0xFFFFFFFF
     check_parity(w3, _chain(nfc, w3), 2001)
+
+
+# ---------------------------------------------------------------- valid edge-case frames
+# IPv4 options (IHL 6..15), fragments (ports 0, L4 not parsed), TCP data offsets 6..15 and
+# Ethernet trailers (SURVEY 8(c)(i) parse cases) through the fused kernel's general parse,
+# the options checksum loop, the L4-from-memory paths, the NAT memory path and ESP with
+# IHL > 5.
+EDGE_CASES = [("C1", None, None, False), ("C1", None, 64, False), ("C2", None, 1, False),
+              ("C3", None, None, True), ("C4", None, 1, True), ("N3", None, 1, False),
+              ("N3", None, 64, False), ("C5", 6, 1, True), ("C5", 3, 64, True), ("C5", 4, 0, True)]
+
+
+@pytest.mark.parametrize("cfg,k,pl,small", EDGE_CASES)
+def test_edge_frames_parity(nfc, cfg, k, pl, small):
+    w = nfcgen.workload(cfg, k=k, pkt_len=pl, small=small, acl_rules=200 if cfg == "N3" else None)
+    w.traffic.tcp_pct = 40
+    w.traffic.edge(120_000)
+    w.traffic.malformed_ppm = 10_000
+    w.traffic.ttl1_ppm = 5_000
+    ch = _chain(nfc, w)
+    got, _ = check_parity(w, ch, 3001)
+    assert (got["drop_nf"] == 0xFF).sum() > 1000
+
+
+@pytest.mark.parametrize("flags", ["unfused", "parallel"])
+def test_edge_frames_unfused_parallel(nfc, flags):
+    w = nfcgen.workload("C5", k=4, pkt_len=1, small=True)
+    w.traffic.tcp_pct = 40
+    w.traffic.edge(120_000)
+    ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_UNFUSED if flags == "unfused" else nfc.F_PARALLEL)
+    ch.load_tables(w.tables)
+    check_parity(w, ch, 2501)
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4, 5, 6])
+def test_c5_full_tables(nfc, k):
+    """C5 with its full tables (200K IPv6 routes) at every chain length, IMIX, many batches."""
+    w = nfcgen.workload("C5", k=k, pkt_len=0)
+    ch = _chain(nfc, w)
+    check_parity(w, ch, 6000, split=[4096])
+
+
+def test_c1_many_batches(nfc):
+    """The multi-batch descriptor path: 40 batches of 4,096 packets (ragged last) in one call."""
+    w = nfcgen.workload("C1")
+    ch = _chain(nfc, w)
+    n = 40 * 4096 - 123
+    check_parity(w, ch, n, split=[4096] * 39, match_cap=1 << 20)
