@@ -44,6 +44,8 @@ def parse_args():
     ap.add_argument("--k", type=int, default=None, help="C5 chain length")
     ap.add_argument("--acl-rules", type=int, default=None, help="N3 (NEXT-3) ACL size: 200 / 1000 / 10000")
     ap.add_argument("--ring-mb", type=int, default=1024, help="HBM ring size per GPU (>> 126 MB L2)")
+    ap.add_argument("--batch-pkts", type=int, default=BATCH,
+                    help="packets per nfc_batch descriptor (SURVEY 8(c)(ii)#4: 4,096); 0 = the ring as one batch")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle baseline budget")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -66,6 +68,57 @@ def ring_packets(w, ring_mb):
     slot = (len(probe.arena) - 64) / 4096.0
     n = int(ring_mb * (1 << 20) / slot)
     return max(4096, (n // 4096) * 4096)
+
+
+def prepare_ring(w, ring_mb, rank, world, local_dev, stream):
+    """This rank's packets, resident in HBM: its RSS shard (nfc_rss_shard, the P:L87 Receive
+    Side Steering model: Toeplitz(MS key, 5-tuple) -> RETA) of the global packet stream, in
+    global order, written on the device by the traffic generator (nfcgen.device) one window
+    of the global stream at a time and packed into a dense ring.  World 1: the stream itself.
+    Returns (arena u8, off i64, len i16) device tensors and the packet count."""
+    import torch
+
+    from nfcgen import device as gd
+    from paper_conf_hpca_hul18_b200 import nfc
+    dev = torch.device("cuda", local_dev)
+    n = ring_packets(w, ring_mb)
+    dtab = gd.DeviceTables(w.traffic, w.tables, dev)
+    if world == 1:
+        a, o, l_ = gd.generate(w.traffic, w.tables, 0, n, device=dev, dtab=dtab)
+        return a, o, l_, n
+    hr, tr = w.traffic.headroom, w.traffic.tailroom
+    pieces, have, s0 = [], 0, 0
+    shard = torch.empty(n, dtype=torch.uint8, device=dev)
+    while have < n:
+        a, o, l_ = gd.generate(w.traffic, w.tables, s0, n, device=dev, dtab=dtab)
+        nfc.rss_shard(local_dev, a.data_ptr(), o.data_ptr(), l_.data_ptr(), n, world, shard.data_ptr(),
+                      stream.cuda_stream)
+        idx = torch.nonzero(shard == rank).flatten()[: n - have]
+        pieces.append(gd.gather(a, o, l_, idx, hr, tr))
+        have += int(idx.numel())
+        s0 += n
+        del a, o, l_
+    base, arenas, offs = 0, [], []
+    for a, o, _ in pieces:
+        arenas.append(a[:-64])
+        offs.append(o + base)
+        base += a.numel() - 64
+    arenas.append(torch.zeros(64, dtype=torch.uint8, device=dev))
+    return torch.cat(arenas), torch.cat(offs), torch.cat([p_[2] for p_ in pieces]), n
+
+
+def host_view(arena, off, ln, first, w):
+    """nfcgen.Batch view (host copies) of a device ring, for the byte accounting and the e2e leg."""
+    import nfcgen
+    return nfcgen.Batch(arena.cpu().numpy(), off.cpu().numpy().view(np.uint64), ln.cpu().numpy().view(np.uint16),
+                        first, w.traffic.headroom, w.traffic.tailroom)
+
+
+def batch_descs(arena, off, ln, n, first, bp):
+    """nfc_batch descriptors: the ring cut into batches of bp packets (bp = 0: one batch)."""
+    bp = bp or n
+    return [(arena.data_ptr(), off.data_ptr() + 8 * s_, ln.data_ptr() + 2 * s_, min(bp, n - s_), first + s_)
+            for s_ in range(0, n, bp)]
 
 
 def alg_bytes_per_step(kinds, lens, fam, rec):
@@ -419,6 +472,7 @@ def main():
     import torch.distributed as dist
 
     import nfcgen
+    from paper_conf_hpca_hul18_b200 import dist as pdist
     from paper_conf_hpca_hul18_b200 import nfc
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -437,17 +491,19 @@ def main():
     cdev = dev if backend == "nccl" else torch.device("cpu")   # where collectives run
 
     w = make_workload(args)
-    n = ring_packets(w, args.ring_mb)
-    first = rank * n                       # flows of rank r: its own slice of the global stream
-    b = nfcgen.generate(w.traffic, w.tables, first, n)
+    stream = torch.cuda.current_stream(dev)
+    arena, off, ln, n = prepare_ring(w, args.ring_mb, rank, world, local_dev, stream)
+    first = rank * n                       # match-pair ids: rank-local numbering of the shard
+    b = host_view(arena, off, ln, first, w)
     chain = nfc.Chain(w.kinds, device=local_dev, flags=nfc.F_UNFUSED if args.unfused else 0)
     chain.load_tables(w.tables)
     hr, tr = chain.room()
     assert hr <= w.traffic.headroom and tr <= w.traffic.tailroom
+    comm = None
+    if world > 1 and backend == "nccl":
+        comm = pdist.library_comm(local_dev)      # the library's own NCCL comm: counters only
+        chain.attach_comm(comm)
 
-    arena = torch.from_numpy(b.arena).to(dev)
-    off = torch.from_numpy(b.off.view(np.int64)).to(dev)
-    ln = torch.from_numpy(b.len.view(np.int16)).to(dev)
     restore = bool(RESTORE_KINDS & set(w.kinds))
     pristine = arena.clone() if restore else None
     rec = torch.empty((n, 16), dtype=torch.uint8, device=dev)
@@ -455,8 +511,8 @@ def main():
     mp = torch.empty(cap, dtype=torch.int32, device=dev)
     mq = torch.empty(cap, dtype=torch.int16, device=dev)
     mc = torch.zeros(1, dtype=torch.int32, device=dev)
-    stream = torch.cuda.current_stream(dev)
-    desc = [(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), n, first)]
+    descs = batch_descs(arena, off, ln, n, first, args.batch_pkts)
+    desc = nfc.Chain.batch_array(descs)
 
     def step():
         mc.zero_()
@@ -497,12 +553,15 @@ def main():
         ms = ev[0][0].elapsed_time(ev[-1][1])
     launches = chain.launches() - launches0
     launch_info = chain.last_launch()
-    stats = chain.stats(reset=True)
+    # the only data collective: the counters, summed over ranks inside the library
+    # (nfc_collect_stats(NFC_STATS_ALLREDUCE): one ncclAllReduce on the chain's stream)
+    stats = chain.stats(reset=True, allreduce=comm is not None)
     ms_t = torch.tensor([ms], dtype=torch.float64, device=cdev)
     st_t = torch.from_numpy(stats.view(np.int64).copy()).to(cdev)
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(st_t, op=dist.ReduceOp.SUM)   # the only collective: counters
+        if comm is None:   # gloo test plumbing (several ranks on one GPU): host-side sum
+            dist.all_reduce(st_t, op=dist.ReduceOp.SUM)
     ms_max = float(ms_t.item())
     tot_pkts = n * args.steps * world
     tot_bytes = int(b.len.astype(np.int64).sum()) * args.steps * world
@@ -670,10 +729,14 @@ def main():
             "config": {"workload": f"{w.name}: {w.note}", "chain": w.kinds,
                        "pkt_len": "IMIX" if w.traffic.pkt_len == 0 else w.traffic.pkt_len,
                        "packets_per_step_per_gpu": n, "ring_bytes_per_gpu": len(b.arena),
+                       "batch_pkts": args.batch_pkts or n, "batches_per_step_per_gpu": len(descs),
+                       "sharding": "RSS: nfc_rss_shard (Toeplitz MS key -> RETA) of the global stream, device-generated"
+                                   if world > 1 else "single GPU: the global stream, device-generated",
                        "l2": "ring >> 126 MB L2 (no flush needed)" if not restore else
                              "pristine ring restored between steps (1 GiB-class copy, evicts L2), outside timed intervals",
                        "timing": "CUDA events on the launch stream; max over ranks",
-                       "parallelism": f"flow-sharded x{world}, no data-path collective",
+                       "parallelism": f"RSS flow-sharded x{world}, no data-path collective; counters summed by "
+                                      f"one ncclAllReduce inside the library",
                        "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4),
                        "launch": launch_info},
             "roofline": roof,

@@ -252,15 +252,24 @@ class Chain:
                               t.nat_ext_ports, t.nat_key)
 
     # ------------------------------------------------------------ processing
-    def process(self, batches, rec_ptr: int, match_pkt_ptr: int = 0, match_pat_ptr: int = 0,
-                match_cap: int = 0, match_count_ptr: int = 0, stream: int = 0):
-        """batches: list of (arena_ptr, off_ptr, len_ptr, n, first_global_index) device pointers."""
+    @staticmethod
+    def batch_array(batches):
+        """nfc_batch descriptor array (host) for a list of (arena_ptr, off_ptr, len_ptr, n,
+        first_global_index); pass it to process() to skip rebuilding it every call."""
         arr = (Batch * max(1, len(batches)))()
         for i, (a, o, l, n, fgi) in enumerate(batches):
             arr[i] = Batch(a, o, l, n, 0, fgi)
+        arr.count = len(batches)
+        return arr
+
+    def process(self, batches, rec_ptr: int, match_pkt_ptr: int = 0, match_pat_ptr: int = 0,
+                match_cap: int = 0, match_count_ptr: int = 0, stream: int = 0):
+        """batches: list of (arena_ptr, off_ptr, len_ptr, n, first_global_index) device pointers,
+        or a batch_array() of them."""
+        arr = batches if hasattr(batches, "count") and not isinstance(batches, list) else self.batch_array(batches)
         res = Result(rec_ptr, match_pkt_ptr or None, match_pat_ptr or None, match_cap, 0,
                      match_count_ptr or None)
-        return _check(lib.nfc_process_batch(self.h, arr, len(batches), ctypes.byref(res), stream or None))
+        return _check(lib.nfc_process_batch(self.h, arr, arr.count, ctypes.byref(res), stream or None))
 
     def process_tensors(self, arena, off, ln, rec, match_pkt=None, match_pat=None, match_count=None,
                         first_global_index: int = 0, n: Optional[int] = None, stream=None):
