@@ -68,14 +68,13 @@ GEN_FN uint64_t gen_rnd(uint64_t seed, uint32_t stream, uint64_t idx)
 #define R(st, i) gen_rnd(p->seed, (st), (i))
 
 /* fill addr bits beyond len with random bits (network order, nbytes 4 or 16) */
+GEN_FN uint8_t rnd_byte(uint64_t r0, uint64_t r1, int k) { return (uint8_t)((k < 8 ? r0 : r1) >> (8 * (k & 7))); }
 GEN_FN void host_bits(uint8_t *a, const uint8_t *pref, int len, int nbytes, uint64_t r0, uint64_t r1)
 {
-    uint8_t rb[16];
-    for (int k = 0; k < 8; k++) { rb[k] = (uint8_t)(r0 >> (8 * k)); rb[8 + k] = (uint8_t)(r1 >> (8 * k)); }
     for (int k = 0; k < nbytes; k++) {
-        int keep = len - 8 * k; /* prefix bits in this byte */
-        uint8_t m = keep >= 8 ? 0xFF : keep <= 0 ? 0x00 : (uint8_t)(0xFF << (8 - keep));
-        a[k] = (uint8_t)((pref[k] & m) | (rb[k] & ~m));
+        const int keep = len - 8 * k; /* prefix bits in this byte */
+        const uint32_t m = keep >= 8 ? 0xFFu : keep <= 0 ? 0u : (0xFF00u >> keep) & 0xFFu;
+        a[k] = (uint8_t)(((uint32_t)pref[k] & m) | ((uint32_t)rnd_byte(r0, r1, k) & ~m & 0xFFu));
     }
 }
 
@@ -103,7 +102,7 @@ GEN_FN void make_flow(const gen_params *p, const gen_tables *t, uint64_t f, flow
         uint32_t nr = fl->fam == 4 ? t->n_r4 : t->n_r6;
         if (nr) {
             uint64_t k = R(S_ROUTE, f) % nr;
-            uint8_t pref[16];
+            uint8_t pref[16] = {0};
             int plen;
             if (fl->fam == 4) {
                 uint32_t v = t->r4_prefix[k];

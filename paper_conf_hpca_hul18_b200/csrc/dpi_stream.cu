@@ -16,6 +16,7 @@
 // The flow table and the per-flow DFA states persist across calls.
 #include <cuda_runtime.h>
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
 
 #include <cstdlib>
 #include <cstring>
@@ -117,29 +118,42 @@ __device__ __forceinline__ uint32_t ld_acquire(const uint32_t *p)
     return v;
 }
 
-// Flow table slot of `key` (inserted if new); 0xFFFFFFFF if the table is full.
-// lock[s]: 0 empty, 1 key being written, 2 key published.
-__device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t *n_flows,
+// Flow table slot of `key` (inserted if new); 0xFFFFFFFF if the flow is not in the
+// table and cannot be placed: max_flows flows are already placed (so the load factor
+// stays <= 1/2), or no free slot within PROBE_MAX probes (a bounded probe: a SYN flood
+// of new 5-tuples cannot turn every later miss into a full-table scan).
+// lock[s]: 0 empty, 1 key being written, 2 key published, 3 dead (claimed when the
+// table was already at max_flows: skipped by every probe).  The capacity is counted
+// after the claim, so concurrent packets of one new flow do not over-reserve it.
+constexpr uint32_t PROBE_MAX = 64;
+__device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t *n_flows, uint32_t max_flows,
                               const uint32_t key[KW])
 {
     uint32_t s = key_hash(key) & mask;
-    for (uint32_t probe = 0; probe <= mask; probe++, s = (s + 1) & mask) {
+    const uint32_t probes = min(mask + 1, PROBE_MAX);
+    for (uint32_t probe = 0; probe < probes; probe++, s = (s + 1) & mask) {
         uint32_t l = ld_acquire(&lock[s]);           // published slots need no atomic
         if (l == 0) {
             l = atomicCAS(&lock[s], 0u, 1u);
             if (l == 0) {
+                if (atomicAdd(n_flows, 1u) >= max_flows) {   // table at capacity: no new flow
+                    atomicSub(n_flows, 1u);
+                    __threadfence();
+                    atomicExch(&lock[s], 3u);
+                    return 0xFFFFFFFFu;
+                }
                 uint4 *kp = reinterpret_cast<uint4 *>(keys + (size_t)s * KS);
                 kp[0] = make_uint4(key[0], key[1], key[2], key[3]);
                 kp[1] = make_uint4(key[4], key[5], key[6], key[7]);
                 kp[2] = make_uint4(key[8], key[9], 0, 0);
                 __threadfence();
                 atomicExch(&lock[s], 2u);
-                atomicAdd(n_flows, 1u);
                 return s;
             }
             l = ld_acquire(&lock[s]);                // the CAS is relaxed: re-read with acquire
         }
         while (l == 1) l = ld_acquire(&lock[s]);     // acquire: the published key is visible
+        if (l == 3) continue;                        // dead slot
         const uint4 *kp = reinterpret_cast<const uint4 *>(keys + (size_t)s * KS);
         const uint4 k0 = __ldcg(kp), k1 = __ldcg(kp + 1), k2 = __ldcg(kp + 2);
         if (k0.x == key[0] && k0.y == key[1] && k0.z == key[2] && k0.w == key[3] && k1.x == key[4] &&
@@ -149,7 +163,7 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
     return 0xFFFFFFFFu;
 }
 
-__global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t none,
+__global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mask, uint32_t max_flows, uint32_t none,
                        uint32_t *ctr, uint32_t *fkey, uint32_t *fidx, uint32_t *span,
                        uint32_t *nocc, uint8_t *drop)
 {
@@ -170,7 +184,7 @@ __global__ void k_flow(nfc_batch b, uint32_t *lock, uint32_t *keys, uint32_t mas
     uint32_t key[KW], a, e;
     uint32_t slot = none;
     if (parse_flow(reinterpret_cast<const uint8_t *>(h), min(flen, HB), flen, key, a, e)) {
-        slot = flow_slot(lock, keys, mask, &ctr[0], key);
+        slot = flow_slot(lock, keys, mask, &ctr[0], max_flows, key);
         if (slot == 0xFFFFFFFFu) { atomicAdd(&ctr[1], 1u); slot = none; }
         span[i] = a | e << 16;
     }
@@ -243,8 +257,8 @@ __device__ __forceinline__ uint32_t walk(const StreamDfa &d, const uint8_t *cls,
 template <int M>
 __global__ void __launch_bounds__(M == 2 ? WALK_SMEM_THREADS : 256) k_walk(nfc_batch b, StreamDfa d, uint32_t none, uint32_t need,
                                                           const uint32_t *fkey, const uint32_t *fidx,
-                                                          const uint32_t *span, const uint32_t *fstate, uint32_t *fin,
-                                                          nfc_stream_result r)
+                                                          const uint32_t *span, const unsigned long long *cumx,
+                                                          const uint32_t *fstate, uint32_t *fin, nfc_stream_result r)
 {
     __shared__ uint8_t cls[256];
     extern __shared__ uint4 dyn[];
@@ -258,15 +272,32 @@ __global__ void __launch_bounds__(M == 2 ? WALK_SMEM_THREADS : 256) k_walk(nfc_b
     for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < b.n; u += gridDim.x * blockDim.x) {
         const uint32_t f = fkey[u];
         if (f == none) continue;
-        // warm-up start: packet v, byte skip within its payload, start state s
-        uint32_t v = u, acc = 0, skip = 0, s = 0;
-        while (acc < need && v > 0 && fkey[v - 1] == f) {
-            v--;
-            const uint32_t sp = span[fidx[v]];
-            acc += (sp >> 16) - (sp & 0xFFFF);
+        // warm-up start: packet v, byte skip within its payload, start state s.  v is the
+        // last position before u of the same flow with payload bytes [v, u) >= need
+        // (cumx: exclusive prefix sum of payload lengths in sorted order), found by a
+        // galloping search -- O(log distance), so runs of empty payloads (pure ACKs)
+        // cost no quadratic walk-back; if the flow's bytes before u in this call are
+        // fewer, v is the flow's first packet of the call and s its carried state.
+        const unsigned long long cu = cumx[u];
+        auto stop = [&](uint32_t d) {                // position u - d (d <= u)
+            const uint32_t v = u - d;
+            return fkey[v] != f || cu - cumx[v] >= need;
+        };
+        uint32_t lo = 0, hi = 1;                     // stop(lo) false (lo = 0: none tested), answer in (lo, hi]
+        while (hi <= u && !stop(hi)) { lo = hi; hi *= 2; }
+        if (hi > u) hi = u + 1;                      // position -1: before the call
+        while (hi - lo > 1) {
+            const uint32_t mid = lo + (hi - lo) / 2;
+            if (stop(mid)) hi = mid; else lo = mid;
         }
-        if (acc >= need) skip = acc - need;
-        else s = fstate[f];                          // v is the flow's first packet of this call
+        uint32_t v, skip = 0, s = 0;
+        if (hi <= u && fkey[u - hi] == f) {
+            v = u - hi;
+            skip = (uint32_t)(cu - cumx[v] - need);
+        } else {
+            v = u - lo;                              // the flow's first packet of this call
+            s = fstate[f];
+        }
         Emit em{r, (uint32_t)b.first_global_index, 0, 0, 0};
         for (uint32_t w = v; w < u; w++) {
             const uint32_t i = fidx[w], sp = span[i];
@@ -280,6 +311,20 @@ __global__ void __launch_bounds__(M == 2 ? WALK_SMEM_THREADS : 256) k_walk(nfc_b
         r.drop[i] = (uint8_t)em.dr;
         if (u + 1 == b.n || fkey[u + 1] != f) fin[u] = s;
     }
+}
+
+// payload bytes of each position in flow-sorted order (0 for packets not inspected)
+__global__ void k_plen(uint32_t n, uint32_t none, const uint32_t *fkey, const uint32_t *fidx, const uint32_t *span,
+                       unsigned long long *plen)
+{
+    const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
+    if (u >= n) return;
+    uint32_t l = 0;
+    if (fkey[u] != none) {
+        const uint32_t sp = span[fidx[u]];
+        l = (sp >> 16) - (sp & 0xFFFF);
+    }
+    plen[u] = l;
 }
 
 __global__ void k_commit(uint32_t n, uint32_t none, const uint32_t *fkey, const uint32_t *fin, uint32_t *fstate)
@@ -305,6 +350,8 @@ struct nfc_dpi_stream {
     // per-call scratch
     uint32_t cap_pkts = 0;
     uint32_t *fkey = nullptr, *fkey2 = nullptr, *fidx = nullptr, *fidx2 = nullptr, *span = nullptr;
+    unsigned long long *cumx = nullptr;
+    uint32_t max_flows = 0;
     void *tmp = nullptr;
     size_t tmp_bytes = 0;
     uint64_t launches = 0;
@@ -327,8 +374,10 @@ static cudaError_t dev_copy(T **dst, const T *src, size_t n)
 static void free_scratch(nfc_dpi_stream *s)
 {
     cudaFree(s->fkey); cudaFree(s->fkey2); cudaFree(s->fidx); cudaFree(s->fidx2); cudaFree(s->span);
+    cudaFree(s->cumx);
     cudaFree(s->tmp);
     s->fkey = s->fkey2 = s->fidx = s->fidx2 = s->span = nullptr;
+    s->cumx = nullptr;
     s->tmp = nullptr;
     s->cap_pkts = 0;
     s->tmp_bytes = 0;
@@ -366,7 +415,10 @@ int nfc_dpi_stream_create_regex(int device, const nfc_dpi_spec *spec, uint32_t m
     *out = nullptr;
     DpiHost h;
     std::string e = build_regex_dfa(*spec, h, max_states ? max_states : (1u << 20));
-    if (!e.empty()) return set_fail(e.find("unbounded") != std::string::npos ? NFC_EUNSUP : NFC_EINVAL, e);
+    if (!e.empty())
+        return set_fail(e.find("out of host memory") != std::string::npos ? NFC_ENOMEM
+                        : (e.find("unbounded") != std::string::npos || e.find("not supported") != std::string::npos)
+                            ? NFC_EUNSUP : NFC_EINVAL, e);
     return create_from_host(device, h, max_flows, out);
 }
 
@@ -378,6 +430,7 @@ static int create_from_host(int device, const DpiHost &h, uint32_t max_flows, nf
     uint32_t lg = 1;
     while ((1u << lg) < 2 * max_flows) lg++;           // load factor <= 1/2
     s->n_slots = 1u << lg;
+    s->max_flows = max_flows;
     s->mask = s->n_slots - 1;
     s->key_bits = lg + 1;                              // slot ids and the "none" key n_slots
     s->ncls = h.ncls;
@@ -449,35 +502,43 @@ int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stre
         SCK(cudaMalloc((void **)&s->fidx, n * 4));
         SCK(cudaMalloc((void **)&s->fidx2, n * 4));
         SCK(cudaMalloc((void **)&s->span, n * 4));
+        SCK(cudaMalloc((void **)&s->cumx, (n + 1) * 8));
         SCK(cub::DeviceRadixSort::SortPairs(nullptr, s->tmp_bytes, s->fkey, s->fkey2, s->fidx, s->fidx2,
                                             (int)n, 0, (int)s->key_bits, st));
+        size_t scan_bytes = 0;
+        SCK(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, s->cumx, s->cumx, (int)n, st));
+        s->tmp_bytes = std::max(s->tmp_bytes, scan_bytes);
         SCK(cudaMalloc(&s->tmp, std::max<size_t>(16, s->tmp_bytes)));
         s->cap_pkts = b->n;
     }
     const uint32_t none = s->n_slots;
     const uint32_t blocks = (b->n + 255) / 256;
-    k_flow<<<blocks, 256, 0, st>>>(*b, s->lock, s->keys, s->mask, none, s->ctr, s->fkey, s->fidx, s->span,
+    k_flow<<<blocks, 256, 0, st>>>(*b, s->lock, s->keys, s->mask, s->max_flows, none, s->ctr, s->fkey, s->fidx, s->span,
                                    r->nocc, r->drop);
     SCK(cudaGetLastError());
     size_t tb = s->tmp_bytes;
     SCK(cub::DeviceRadixSort::SortPairs(s->tmp, tb, s->fkey, s->fkey2, s->fidx, s->fidx2, (int)b->n, 0,
                                         (int)s->key_bits, st));
+    k_plen<<<blocks, 256, 0, st>>>(b->n, none, s->fkey2, s->fidx2, s->span, s->cumx);
+    SCK(cudaGetLastError());
+    tb = s->tmp_bytes;
+    SCK(cub::DeviceScan::ExclusiveSum(s->tmp, tb, s->cumx, s->cumx, (int)b->n, st));
     StreamDfa d{s->cls, s->trans, s->out_off, s->out_ids, s->action, s->ncls, s->wide, s->n_states};
     const uint32_t wb = (b->n + 255) / 256, need = s->maxlen - 1;
     // s->fkey (unsorted keys) is dead after the sort: it holds the flows' final states
     const size_t tbytes = (size_t)s->ncls * s->n_states * 2;
     if (s->wide) {
-        k_walk<1><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+        k_walk<1><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->cumx, s->fstate, s->fkey, *r);
     } else if (s->smem_ok && tbytes <= DFA_SMEM_MAX) {
         k_walk<2><<<s->n_sm, WALK_SMEM_THREADS, (tbytes + 15) / 16 * 16, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span,
-                                                                s->fstate, s->fkey, *r);
+                                                                s->cumx, s->fstate, s->fkey, *r);
     } else {
-        k_walk<0><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+        k_walk<0><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->cumx, s->fstate, s->fkey, *r);
     }
     SCK(cudaGetLastError());
     k_commit<<<blocks, 256, 0, st>>>(b->n, none, s->fkey2, s->fkey, s->fstate);
     SCK(cudaGetLastError());
-    s->launches += 3;   // k_flow + k_walk + k_commit (the cub sort launches its own kernels)
+    s->launches += 4;   // k_flow + k_plen + k_walk + k_commit (the cub sort and scan launch their own kernels)
     return NFC_OK;
 }
 

@@ -160,7 +160,7 @@ struct BatchDev { uint8_t *arena; const uint64_t *off; const uint16_t *len; uint
 // packet g of that batch has off = offp[g], len = lenp[g], bytes at arena + off and
 // global index gb + g.  meta = lane where the next batch starts (0: none) | 1<<5 if
 // the chunk holds more than one batch boundary (those lanes take the binary search).
-struct ChunkRec { const uint64_t *offp; const uint16_t *lenp; uint8_t *arena; uint32_t gb_lo, meta; };  // gb_lo: first - start (diagnostic)
+struct ChunkRec { const uint64_t *offp; const uint16_t *lenp; uint8_t *arena; uint32_t gb_lo, meta; };  // gb_lo: (first - start) mod 2^32
 static_assert(sizeof(ChunkRec) == 32, "ChunkRec is 32 B");
 
 enum { MASK_ACL = 1u << NFC_ACL, MASK_DPI = 1u << NFC_DPI, MASK_LPM4 = 1u << NFC_LPM4,

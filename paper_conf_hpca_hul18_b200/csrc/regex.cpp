@@ -17,6 +17,8 @@
 #include <array>
 #include <cstring>
 #include <map>
+#include <new>
+#include <stdexcept>
 #include <string>
 #include <vector>
 
@@ -24,6 +26,11 @@
 
 namespace nfc {
 namespace {
+
+// Bounds: the longest word of an expression, and the NFA size while
+// bounded repeats are expanded (nested {m,n} multiply).  Beyond them: NFC_EUNSUP.
+constexpr long long REGEX_MAXLEN = 1024;
+constexpr size_t REGEX_NFA_MAX = 1u << 20;
 
 struct Nfa {
     struct St { std::array<uint64_t, 4> set{}; int out = -1; std::vector<int> eps; int accept = -1; };
@@ -61,7 +68,7 @@ struct Parser {
         return {a, b};
     }
     // returns fragment and its (min unused) max length in *len
-    bool atom(Frag &f, int &len) {
+    bool atom(Frag &f, long long &len) {
         uint8_t c = *p++;
         std::array<uint64_t, 4> set{};
         auto put = [&](int b) { set[b >> 6] |= 1ull << (b & 63); };
@@ -72,6 +79,7 @@ struct Parser {
             return true;
         }
         if (c == '*' || c == '+') { err = "regex: unbounded quantifier ('*', '+') not supported"; return false; }
+        if (c == '^' || c == '$') { err = "regex: anchors ('^', '$' outside a class) not supported"; return false; }
         if (c == ')' || c == '?' || c == '{' || c == '|') { err = "regex: misplaced metacharacter"; return false; }
         if (c == '.') { for (int b = 0; b < 256; b++) put(b); }
         else if (c == '\\') { uint8_t x; if (!esc(x)) return false; put(x); }
@@ -117,7 +125,7 @@ struct Parser {
         }
         return {f.in + base - lo, f.out + base - lo};
     }
-    bool piece(Frag &f, int &len) {
+    bool piece(Frag &f, long long &len) {
         int lo = (int)n.st.size();
         if (!atom(f, len)) return false;
         int hi = (int)n.st.size();
@@ -132,11 +140,16 @@ struct Parser {
                 if (p >= e || *p != '}' || M < m || M > 64 || M == 0) { err = "regex: bad {m,n} (need 0 <= m <= n <= 64, n > 0)"; return false; }
                 p++;
             }
+            if (len * M > REGEX_MAXLEN) { err = "regex: longest match above 1024 bytes not supported"; return false; }
+            if (n.st.size() + (size_t)(hi - lo) * (size_t)M + 2 * (size_t)M + 2 > REGEX_NFA_MAX) {
+                err = "regex: NFA above 2^20 states not supported";
+                return false;
+            }
             // expand: m mandatory copies, M - m optional copies (all copies are
             // cloned from the untouched fragment before any of them is wired)
             std::vector<Frag> cp{f};
             for (int k = 1; k < M; k++) cp.push_back(clone(lo, hi, f));
-            const int olen = len;
+            const long long olen = len;
             int s0 = n.add(), cur = s0;
             std::vector<int> skips;
             for (int k = 0; k < M; k++) {
@@ -153,27 +166,28 @@ struct Parser {
         }
         return true;
     }
-    bool concat(Frag &f, int &len) {
+    bool concat(Frag &f, long long &len) {
         int s = n.add();
         f = {s, s};
         len = 0;
         while (p < e && *p != '|' && *p != ')') {
             Frag g;
-            int l;
+            long long l;
             if (!piece(g, l)) return false;
             n.st[f.out].eps.push_back(g.in);
             f.out = g.out;
             len += l;
+            if (len > REGEX_MAXLEN) { err = "regex: longest match above 1024 bytes not supported"; return false; }
         }
         return true;
     }
-    bool alt(Frag &f, int &len) {
+    bool alt(Frag &f, long long &len) {
         int s = n.add(), t = n.add();
         f = {s, t};
         len = 0;
         for (;;) {
             Frag g;
-            int l;
+            long long l;
             if (!concat(g, l)) return false;
             n.st[s].eps.push_back(g.in);
             n.st[g.out].eps.push_back(t);
@@ -186,7 +200,21 @@ struct Parser {
 
 }  // namespace
 
+static std::string build_regex_dfa_impl(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states);
+
+// NFC_EUNSUP for messages containing "not supported", NFC_ENOMEM for "out of host memory"
 std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states)
+{
+    try {
+        return build_regex_dfa_impl(s, o, max_states);
+    } catch (const std::bad_alloc &) {
+        return "regex: out of host memory";
+    } catch (const std::length_error &) {
+        return "regex: out of host memory";
+    }
+}
+
+static std::string build_regex_dfa_impl(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states)
 {
     if (s.n_patterns == 0 || s.n_patterns > 65535) return "regex: n_patterns must be 1..65535";
     if (!s.blob || !s.off || !s.action) return "regex: NULL pointer";
@@ -198,7 +226,7 @@ std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_stat
         if (s.action[j] > 1) return "regex: action must be 0 or 1";
         Parser ps(s.blob + s.off[j], s.blob + s.off[j + 1], n);
         Frag f;
-        int len;
+        long long len;
         if (!ps.alt(f, len)) return ps.err + " (expression " + std::to_string(j) + ")";
         if (ps.p != ps.e) return "regex: unbalanced ')' (expression " + std::to_string(j) + ")";
         int acc = n.add();

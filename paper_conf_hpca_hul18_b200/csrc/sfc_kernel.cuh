@@ -1448,7 +1448,13 @@ static __device__ __noinline__ uint32_t gidx_search(const BatchDev *bs, uint32_t
 }
 __device__ __forceinline__ uint32_t pkt_gidx(const KParams &P, uint32_t g)
 {
-    return P.n_batches == 1 ? (uint32_t)P.b0.first + g : gidx_search(P.batches, P.n_batches, g);
+    if (P.n_batches == 1) return (uint32_t)P.b0.first + g;
+    if (P.crec) {   // the chunk record's batch, unless g lies past a batch boundary in the chunk
+        const uint2 m = __ldg(reinterpret_cast<const uint2 *>(&P.crec[g >> 5].gb_lo));
+        const uint32_t split = m.y & 31;
+        if (!(m.y & 32) && !(split && (g & 31) >= split)) return m.x + g;
+    }
+    return gidx_search(P.batches, P.n_batches, g);
 }
 
 // arena base of chunk c's descriptors in the pipelined loop (desc_get offsets are relative to it)

@@ -130,11 +130,11 @@ def test_stream_edge_frames(nfc):
     ds.reset()
     got, gn, gd, k = _gpu(ds, sb, cap=3)
     assert k == len(want) and len(got) == 3 and set(got) <= set(want) and gn == wn
-    # flow table full: 2 slots, more flows -> packets of unplaced flows not inspected
+    # flow table full: max_flows = 1 flow placed, packets of other flows not inspected
     small = nfc.DpiStream(blob, off, np.array(act, dtype=np.uint8), max_flows=1)
     got, gn, gd, k = _gpu(small, sb)
     nf, nu = small.flows()
-    assert nf == 2 and nu > 0
+    assert nf == 1 and nu > 0
 
 
 def test_stream_fullsize_sampled_flows(nfc):
@@ -187,3 +187,90 @@ def test_regex_stream_parity(nfc, calls):
         assert gn == wn and gd == wd
         first += n
     assert len(want) > 50
+
+
+def test_stream_long_empty_payload_runs(nfc):
+    """runs of zero-payload packets in one flow (the ACK direction of a bulk
+    transfer) -- exact results and no quadratic warm-up walk-back: 60 K empty packets
+    of one flow between payload-carrying ones take about as long as 60 K packets of
+    60 K flows."""
+    import time
+    import torch
+    from tests.test_oracle_stream import _udp
+    pats = [b"abcdefgh", b"hab", b"zz"]
+    act = [0, 1, 0]
+    blob = np.frombuffer(b"".join(pats), dtype=np.uint8)
+    off = np.cumsum([0] + [len(p) for p in pats]).astype(np.uint32)
+    rng = np.random.default_rng(3)
+    frames = []
+    for k in range(60000):
+        if k % 20000 == 0:
+            frames.append(_udp(b"xyzabcd"))
+        elif k % 20000 == 1:
+            frames.append(_udp(b"efgh" + bytes(rng.integers(97, 123, 5))))
+        else:
+            frames.append(_udp(b""))
+    frames.append(_udp(b"ab"))
+    sb = _frame_batch(frames, first=3)
+    ds = nfc.DpiStream(blob, off, np.array(act, dtype=np.uint8), max_flows=16)
+    want, wn, wd = StreamDPI(pats, act).process(sb.frames(), 3)
+    got, gn, gd, k = _gpu(ds, sb)
+    assert got == want and gn == wn and gd == wd
+    # timing against the same packet count spread over distinct flows
+    spread = _frame_batch([_udp(b"", sport=1000 + (j % 60000), src=0x0B000000 + j) for j in range(len(frames))])
+    ds2 = nfc.DpiStream(blob, off, np.array(act, dtype=np.uint8), max_flows=1 << 17)
+    ts = []
+    for dsx, sbx in ((ds, sb), (ds2, spread)):
+        dsx.reset()
+        _gpu(dsx, sbx)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(3):
+            _gpu(dsx, sbx)
+        torch.cuda.synchronize()
+        ts.append(time.perf_counter() - t0)
+    assert ts[0] < 3 * ts[1] + 0.05, ts
+
+
+def test_stream_rss_sharded_equals_single(nfc):
+    """the multi-GPU stateful path as N GPUs run it -- frames steered by
+    nfc_rss_shard, one DpiStream (own flow table) per shard, several calls -- equals the
+    single-stream oracle, with fragments, IPv4 options and TCP options in the traffic
+    (a fragment's flow key has ports 0, so all fragments of a (src, dst, proto) share a
+    flow and a shard)."""
+    import torch
+    from oracle.stream_dpi import StreamDPI as SD
+    from paper_conf_hpca_hul18_b200 import dist as pdist
+    blob, off, act, pats = _pats(5, 40, lmin=2, lmax=6)
+    w = nfcgen.workload("C1", small=True)
+    w.traffic.n_flows, w.traffic.tcp_pct, w.traffic.pkt_len = 300, 40, 1
+    w.traffic.edge(150_000)
+    w.traffic.match_ppm = 0
+    d = torch.device("cuda:0")
+    want_all, got_all = [], {}
+    orc = SD(pats, list(act))
+    for N in (2, 4):
+        got_all[N] = []
+        streams = [nfc.DpiStream(blob, off, act, max_flows=1024) for _ in range(N)]
+        for call in range(3):
+            b = nfcgen.generate(w.traffic, w.tables, 2000 * call, 2000)
+            if N == 2:
+                occ, _, _ = orc.process([b.frame(i) for i in range(b.n)], 2000 * call)
+                want_all += occ
+            arena = torch.from_numpy(b.arena).to(d)
+            o_t = torch.from_numpy(b.off.view(np.int64)).to(d)
+            l_t = torch.from_numpy(b.len.view(np.int16)).to(d)
+            sh = torch.zeros(b.n, dtype=torch.uint8, device=d)
+            nfc.rss_shard(0, arena.data_ptr(), o_t.data_ptr(), l_t.data_ptr(), b.n, N, sh.data_ptr())
+            torch.cuda.synchronize()
+            shn = sh.cpu().numpy()
+            for r in range(N):
+                idx = pdist.shard_indices(shn, r)
+                if not len(idx):
+                    continue
+                sub = StreamBatch(b.arena, b.off[idx], b.len[idx], 0)
+                occ, _, _, _ = _gpu(streams[r], sub)
+                got_all[N] += [(int(2000 * call + idx[p]), q, e) for p, q, e in occ]
+    assert len(want_all) > 100
+    for N in (2, 4):
+        assert sorted(got_all[N]) == sorted(want_all), N
