@@ -269,6 +269,94 @@ def oracle_rate(w, first, budget_s, chunk=8192, max_chunks=100000):
     return pk / t_work / 1e6, by * 8 / t_work / 1e9, pk, t_work
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+_ALLCORE = {}
+
+
+def _allcore_worker(p):
+    """One single-threaded oracle process on its RSS shard of the sample (timed alone)."""
+    import oracle
+    w, b, shard = _ALLCORE["w"], _ALLCORE["b"], _ALLCORE["shard"]
+    import nfcgen
+    idx = np.nonzero(shard == p)[0]
+    sub = nfcgen.Batch(b.arena.copy(), b.off[idx], b.len[idx], 0, b.headroom, b.tailroom)
+    orc = oracle.OracleChain(w.kinds, w.tables)
+    t0 = time.perf_counter()
+    orc.run(sub, match_cap=1 << 22)
+    return len(idx), int(b.len[idx].astype(np.int64).sum()), time.perf_counter() - t0
+
+
+def oracle_all_cores(w, local_dev, rate_1core_mpps, budget_s):
+    """All host cores: nproc independent single-threaded oracle processes, each on the RSS
+    shard it would own: the sample's shard ids come from nfc_rss_shard with
+    n_shards = nproc; a sample sized for ~budget_s of work per process."""
+    import multiprocessing as mp
+
+    import torch
+
+    import nfcgen
+    from paper_conf_hpca_hul18_b200 import nfc
+    ncores = os.cpu_count() or 1
+    n = int(max(4096, min(8_000_000, rate_1core_mpps * 1e6 * budget_s * ncores)))
+    b = nfcgen.generate(w.traffic, w.tables, 1 << 40, n)
+    dev = torch.device("cuda", local_dev)
+    a_d = torch.from_numpy(b.arena).to(dev)
+    o_d = torch.from_numpy(b.off.view(np.int64)).to(dev)
+    l_d = torch.from_numpy(b.len.view(np.int16)).to(dev)
+    sh = torch.empty(n, dtype=torch.uint8, device=dev)
+    nfc.rss_shard(local_dev, a_d.data_ptr(), o_d.data_ptr(), l_d.data_ptr(), n, min(ncores, 128), sh.data_ptr(),
+                  torch.cuda.current_stream(dev).cuda_stream)
+    shard = sh.cpu().numpy()
+    del a_d, o_d, l_d
+    _ALLCORE.update(w=w, b=b, shard=shard)
+    ctx = mp.get_context("fork")
+    with ctx.Pool(ncores) as pool:
+        t0 = time.perf_counter()
+        res = pool.map(_allcore_worker, range(min(ncores, 128)))
+        wall = time.perf_counter() - t0
+    _ALLCORE.clear()
+    pk = sum(r[0] for r in res)
+    by = sum(r[1] for r in res)
+    return {"value": round(pk / wall / 1e6, 6), "unit": "Mpps", "cores": ncores, "kind": "oracle",
+            "gbps": round(by * 8 / wall / 1e9, 6),
+            "sample": f"{pk} packets of {w.name}, {ncores} processes of the single-threaded oracle, each on its "
+                      f"RSS shard (nfc_rss_shard, n_shards = nproc); wall {wall:.1f} s, slowest shard "
+                      f"{max(r[2] for r in res):.1f} s"}
+
+
+def payload_bytes(b):
+    """Payload bytes [pl_off, ip_end) per packet by a vectorised read of the headers
+    (bench accounting only: the DPI work per packet; 0 if not parsed)."""
+    o = b.off.astype(np.int64)
+    A = b.arena
+    L = b.len.astype(np.int64)
+    et = A[o + 12].astype(np.int64) << 8 | A[o + 13]
+    v4, v6 = et == 0x0800, et == 0x86DD
+    ihl = (A[o + 14] & 15).astype(np.int64)
+    l4 = np.where(v6, 54, 14 + 4 * ihl)
+    ip_end = np.where(v6, 54 + (A[o + 18].astype(np.int64) << 8 | A[o + 19]),
+                      14 + (A[o + 16].astype(np.int64) << 8 | A[o + 17]))
+    proto = np.where(v6, A[o + 20], A[o + 23]).astype(np.int64)
+    frag = v4 & (((A[o + 20].astype(np.int64) << 8 | A[o + 21]) & 0x3FFF) != 0)
+    lim = np.minimum(o + np.minimum(l4 + 12, L - 1), len(A) - 1)
+    doff = (A[lim] >> 4).astype(np.int64)
+    hl = np.where(frag, 0, np.where(proto == 17, 8, np.where(proto == 6, 4 * doff, 0)))
+    pl = l4 + hl
+    ver = (A[o + 14] >> 4).astype(np.int64)
+    ok = (v4 & (ver == 4) & (ihl >= 5) & (L >= 34) & (ip_end - 14 >= 4 * ihl)) | (v6 & (ver == 6) & (L >= 54))
+    ok &= (ip_end <= L) & (pl <= ip_end) & ~(~frag & (proto == 6) & ((doff < 5) | (l4 + 20 > ip_end)))
+    return np.where(ok, ip_end - pl, 0)
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -568,6 +656,8 @@ def main():
     mpps = tot_pkts / (ms_max / 1e3) / 1e6
     gbps = tot_bytes * 8 / (ms_max / 1e3) / 1e9
 
+    # measured integer / shared-memory / L2 peaks of this GPU (the integer rooflines)
+    mpk = nfc.measure_peaks(local_dev)
     # roofline of the (only) kernel: algorithmic bytes per launch / avg launch duration
     rec_h = rec.cpu().numpy().view(nfcgen.RESULT).reshape(n)
     alg, rd, wr = alg_bytes_per_step(w.kinds, b.len, frame_family(b), rec_h)
@@ -588,17 +678,28 @@ def main():
             "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING fallback"}
     ops = esp_alg_ops(rec_h, l4_offsets(b)) if "IPSEC" in w.kinds else 0
     if ops:
-        # integer-bound chains: issue-limited peak = 148 SMs x 4 schedulers x 32 lanes x max SM clock
-        mhz = peaks.get("sm_max_mhz", 1965.0)
-        alu_peak = 148 * 4 * 32 * mhz * 1e6 / 1e12
+        # integer-bound chains: the measured integer issue peak (nfc_measure_peaks: LOP3/SHF
+        # chains interleaved with IMAD, one instruction per scheduler per clock)
+        alu_peak = mpk["issue_tops"]
         alu_ach = ops / (launch_ms / 1e3) / 1e12
         if alu_ach / alu_peak > achieved / peak:
             roof = {"bound": "alu", "achieved": round(alu_ach, 3), "peak": round(alu_peak, 2), "unit": "Tops/s",
                     "frac": round(alu_ach / alu_peak, 4), "traffic": traffic,
                     "alg_ops_per_launch": ops, "alg_ops_per_packet": round(ops / n, 1),
-                    "peak_source": "derived: 148 SMs x 4 SMSP x 32 lanes x sm_max_mhz (issue limit, DESIGN.md)",
+                    "peak_source": "measured on this GPU: nfc_measure_peaks issue_tops (integer ALU + IMAD issue)",
+                    "alu_pipe_frac": round(alu_ach / mpk["alu_tops"], 4),
                     "hbm": {"achieved": round(achieved, 1), "peak": peak, "frac": round(achieved / peak, 4),
                             "alg_bytes_per_packet": round(alg / n, 2)}}
+    if "DPI" in w.kinds:
+        # DPI work: one dependent DFA lookup per payload byte of every packet reaching DPI
+        # in original order (SURVEY 8(d) "report both fractions")
+        dpos = w.kinds.index("DPI")
+        dr = rec_h["drop_nf"].astype(np.int64)
+        reach = (dr != 0xFE) & ((dr == 0xFF) | (dr >= dpos))
+        lk = int(payload_bytes(b)[reach].sum())
+        roof["dpi_lookups"] = {"per_packet": round(lk / n, 1), "achieved_g_per_s": round(lk / (launch_ms / 1e3) / 1e9, 1),
+                               "smem_peak_g_per_s": round(mpk["smem_glookups"], 1),
+                               "frac": round(lk / (launch_ms / 1e3) / 1e9 / mpk["smem_glookups"], 4)}
 
     # end to end through the host-buffer C-ABI call (H2D + kernel + D2H every step)
     e2e = None
@@ -717,7 +818,11 @@ def main():
         r_mpps, r_gbps, r_pk, r_t = oracle_rate(w, first, args.cpu_seconds)
         cpu = {"value": round(r_mpps, 6), "unit": "Mpps", "cores": 1, "kind": "oracle",
                "sample": f"{r_pk} packets of {w.name} (same generator and tables), {r_t:.1f} s, 1 thread",
-               "gbps": round(r_gbps, 6)}
+               "gbps": round(r_gbps, 6), "cpu_model": cpu_model(), "nproc": os.cpu_count()}
+        try:
+            cpu["all_cores"] = oracle_all_cores(w, local_dev, r_mpps, args.cpu_seconds)
+        except Exception as e:  # noqa: BLE001 -- reported, never fatal to the GPU line
+            cpu["all_cores"] = {"error": repr(e)[:300]}
 
     if rank == 0:
         st = st_t.cpu().numpy().view(np.uint64)
@@ -740,6 +845,7 @@ def main():
                        "fwd_frac": round(float(st[2]) / max(1, float(st[0])), 4),
                        "launch": launch_info},
             "roofline": roof,
+            "measured_peaks": {k_: (round(v_, 2) if isinstance(v_, float) else v_) for k_, v_ in mpk.items()},
             "cpu_baseline": cpu,
             "unfused_baseline": unfused,
             "sfc_parallel": parallel,

@@ -352,6 +352,19 @@ NFC_API int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const 
 /* Synchronizes the device; flows in the table and packets not placed (table full). */
 NFC_API int nfc_dpi_stream_flows(nfc_dpi_stream *s, uint64_t *n_flows, uint64_t *n_unplaced);
 
+/* Measured device peaks, the denominators of the integer-bound rooflines (SURVEY
+ * 8(d): "a repo microbenchmark measures them on the box"): 32-bit ALU-pipe ops/s
+ * (independent LOP3/IADD3/SHF/PRMT chains), integer issue ops/s (the same chains
+ * interleaved with IMAD: ALU + FMA pipes), conflict-free 32-bit shared-memory
+ * lookups/s, and random 32-B L2 sectors/s (64 MiB L2-resident buffer).  Runs ~four
+ * short kernels on `device` (synchronous, about 50 ms); clocks are whatever the
+ * device runs at (sm_clock_mhz is the nominal maximum). */
+typedef struct {
+    double alu_tops, issue_tops, smem_glookups, l2_gsectors;
+    uint32_t sm_count, sm_clock_mhz;
+} nfc_peaks;
+NFC_API int nfc_measure_peaks(int device, nfc_peaks *out);
+
 /* Number of kernel launches the library issued on this chain so far. */
 NFC_API int nfc_launch_count(const nfc_chain *c, uint64_t *count);
 

@@ -21,7 +21,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
 def sources():
-    s = ["capi.cu", "sfc_kernel.cu", "unfused.cu", "builders.cpp", "debug_host.cpp", "planner.cpp", "parallel.cu", "dpi_stream.cu", "regex.cpp", "comm.cu"]
+    s = ["capi.cu", "sfc_kernel.cu", "unfused.cu", "builders.cpp", "debug_host.cpp", "planner.cpp", "parallel.cu", "dpi_stream.cu", "regex.cpp", "comm.cu", "peaks.cu"]
     s += sorted(os.path.basename(p) for p in glob.glob(os.path.join(CSRC, "sfc_inst_*.cu")))
     return s
 

@@ -96,6 +96,8 @@ struct nfc_chain {
     uint64_t launches = 0;
     cudaStream_t last_stream = nullptr;
     void *comm = nullptr;                 // attached ncclComm_t (NFC_STATS_ALLREDUCE)
+    cudaStream_t xs[2] = {nullptr, nullptr};   // nfc_process_host copy/compute streams
+    cudaEvent_t xe[2] = {nullptr, nullptr}, xk = nullptr;
     DBuf stats_red;                       // all-reduce destination
 };
 
@@ -172,6 +174,11 @@ void nfc_destroy_chain(nfc_chain *c)
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
                    &c->h_mp, &c->h_mq, &c->h_mc, &c->stats_red, &c->crec};
     for (DBuf *b : all) b->release();
+    for (int i = 0; i < 2; i++) {
+        if (c->xs[i]) cudaStreamDestroy(c->xs[i]);
+        if (c->xe[i]) cudaEventDestroy(c->xe[i]);
+    }
+    if (c->xk) cudaEventDestroy(c->xk);
     delete c;
 }
 
@@ -515,6 +522,12 @@ int nfc_process_batch(nfc_chain *c, const nfc_batch *batches, uint32_t n_batches
     return process_impl(c, batches, n_batches, r, static_cast<cudaStream_t>(stream));
 }
 
+// End-to-end host path, pipelined: the packets are cut into chunks of consecutive
+// indices; chunk k's bytes [min off - headroom, max off+len + tailroom) go to the same
+// offsets of a device mirror of the arena, its descriptors alongside; copies of chunk
+// k+1 (H2D) and chunk k-1 (D2H) run on the other copy stream while chunk k's kernel
+// runs, so both PCIe directions stay busy.  Kernels run strictly in chunk order (ESP
+// sequence numbers follow global order; the chain's scratch is reused per launch).
 int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const uint64_t *off, const uint16_t *len,
                      uint32_t n, uint64_t first_global_index, nfc_pkt_result *rec, uint32_t *match_pkt,
                      uint16_t *match_pat, uint32_t match_cap, uint32_t *n_pairs, void *stream)
@@ -522,34 +535,84 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
     if (!c || (n && (!arena || !off || !len || !rec))) return fail(NFC_EINVAL, "NULL argument");
     int rc = set_device(c);
     if (rc) return rc;
-    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaStream_t user = static_cast<cudaStream_t>(stream);
+    uint32_t hr = 0, tr = 0;
+    nfc_chain_room(c, &hr, &tr);
     CK(c->h_arena.reserve(arena_bytes + 64));
-    CK(c->h_off.reserve((size_t)n * 8));
-    CK(c->h_len.reserve((size_t)n * 2));
-    CK(c->h_rec.reserve((size_t)n * sizeof(nfc_pkt_result)));
-    CK(c->h_mp.reserve((size_t)match_cap * 4));
-    CK(c->h_mq.reserve((size_t)match_cap * 2));
+    CK(c->h_off.reserve((size_t)n * 8 + 8));
+    CK(c->h_len.reserve((size_t)n * 2 + 8));
+    CK(c->h_rec.reserve((size_t)n * sizeof(nfc_pkt_result) + 16));
+    CK(c->h_mp.reserve((size_t)match_cap * 4 + 4));
+    CK(c->h_mq.reserve((size_t)match_cap * 2 + 4));
     CK(c->h_mc.reserve(4));
-    CK(cudaMemcpyAsync(c->h_arena.p, arena, arena_bytes, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(c->h_off.p, off, (size_t)n * 8, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(c->h_len.p, len, (size_t)n * 2, cudaMemcpyHostToDevice, st));
-    CK(cudaMemsetAsync(c->h_mc.p, 0, 4, st));
-    nfc_batch b{c->h_arena.as<uint8_t>(), c->h_off.as<uint64_t>(), c->h_len.as<uint16_t>(), n, 0, first_global_index};
-    nfc_result r{c->h_rec.as<nfc_pkt_result>(), c->h_mp.as<uint32_t>(), c->h_mq.as<uint16_t>(), match_cap, 0,
-                 c->h_mc.as<uint32_t>()};
-    rc = process_impl(c, &b, 1, &r, st);
-    if (rc) return rc;
-    uint32_t cnt = 0;
-    CK(cudaMemcpyAsync(arena, c->h_arena.p, arena_bytes, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(rec, c->h_rec.p, (size_t)n * sizeof(nfc_pkt_result), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(&cnt, c->h_mc.p, 4, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    uint32_t k = cnt < match_cap ? cnt : match_cap;
-    if (k && match_pkt && match_pat) {
-        CK(cudaMemcpyAsync(match_pkt, c->h_mp.p, (size_t)k * 4, cudaMemcpyDeviceToHost, st));
-        CK(cudaMemcpyAsync(match_pat, c->h_mq.p, (size_t)k * 2, cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
+    if (!c->xs[0]) {
+        for (int i = 0; i < 2; i++) {
+            CK(cudaStreamCreateWithFlags(&c->xs[i], cudaStreamNonBlocking));
+            CK(cudaEventCreateWithFlags(&c->xe[i], cudaEventDisableTiming));
+        }
+        CK(cudaEventCreateWithFlags(&c->xk, cudaEventDisableTiming));
     }
+    // the copy streams start after the caller's prior work
+    CK(cudaEventRecord(c->xk, user));
+    for (int i = 0; i < 2; i++) CK(cudaStreamWaitEvent(c->xs[i], c->xk, 0));
+    CK(cudaMemsetAsync(c->h_mc.p, 0, 4, c->xs[0]));
+    CK(cudaEventRecord(c->xk, c->xs[0]));          // "previous kernel done" starts as: counter zeroed
+    // chunks: about 16 per call, at least 64 K packets each; their byte ranges must be
+    // disjoint and ascending (frames laid out in index order), else one chunk
+    uint32_t per = std::max<uint32_t>(65536, (n + 15) / 16);
+    std::vector<std::pair<uint64_t, uint64_t>> rg;
+    for (int pass = 0; pass < 2; pass++) {
+        rg.clear();
+        bool ok = true;
+        for (uint32_t a0 = 0; a0 < n; a0 += per) {
+            const uint32_t cnt = std::min(per, n - a0);
+            uint64_t lo = ~0ull, hi = 0;
+            for (uint32_t i = a0; i < a0 + cnt; i++) {
+                lo = std::min(lo, off[i]);
+                hi = std::max(hi, off[i] + len[i]);
+            }
+            lo = lo >= hr ? lo - hr : 0;
+            hi = std::min<uint64_t>(hi + tr, arena_bytes);
+            if (lo > arena_bytes || hi < lo) return fail(NFC_EINVAL, "frame outside the arena");
+            if (!rg.empty() && lo < rg.back().second) ok = false;
+            rg.emplace_back(lo, hi);
+        }
+        if (ok) break;
+        per = n;                                    // overlapping chunk ranges: no pipelining
+    }
+    uint8_t *darena = c->h_arena.as<uint8_t>();
+    uint64_t *doff = c->h_off.as<uint64_t>();
+    uint16_t *dlen = c->h_len.as<uint16_t>();
+    uint32_t k = 0;
+    for (uint32_t a0 = 0; a0 < n; a0 += per, k++) {
+        const uint32_t cnt = std::min(per, n - a0);
+        cudaStream_t st = c->xs[k & 1];
+        const uint64_t lo = rg[k].first, hi = rg[k].second;
+        CK(cudaMemcpyAsync(darena + lo, arena + lo, hi - lo, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(doff + a0, off + a0, (size_t)cnt * 8, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(dlen + a0, len + a0, (size_t)cnt * 2, cudaMemcpyHostToDevice, st));
+        CK(cudaStreamWaitEvent(st, c->xk, 0));      // kernels in chunk order
+        nfc_batch b{darena, doff + a0, dlen + a0, cnt, 0, first_global_index + a0};
+        nfc_result r{c->h_rec.as<nfc_pkt_result>() + a0, c->h_mp.as<uint32_t>(), c->h_mq.as<uint16_t>(), match_cap, 0,
+                     c->h_mc.as<uint32_t>()};
+        rc = process_impl(c, &b, 1, &r, st);
+        if (rc) return rc;
+        CK(cudaEventRecord(c->xk, st));
+        CK(cudaMemcpyAsync(arena + lo, darena + lo, hi - lo, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(rec + a0, c->h_rec.as<nfc_pkt_result>() + a0, (size_t)cnt * sizeof(nfc_pkt_result),
+                           cudaMemcpyDeviceToHost, st));
+    }
+    uint32_t cnt = 0;
+    CK(cudaStreamWaitEvent(c->xs[0], c->xk, 0));
+    CK(cudaMemcpyAsync(&cnt, c->h_mc.p, 4, cudaMemcpyDeviceToHost, c->xs[0]));
+    for (int i = 0; i < 2; i++) CK(cudaStreamSynchronize(c->xs[i]));
+    uint32_t m = cnt < match_cap ? cnt : match_cap;
+    if (m && match_pkt && match_pat) {
+        CK(cudaMemcpyAsync(match_pkt, c->h_mp.p, (size_t)m * 4, cudaMemcpyDeviceToHost, c->xs[0]));
+        CK(cudaMemcpyAsync(match_pat, c->h_mq.p, (size_t)m * 2, cudaMemcpyDeviceToHost, c->xs[0]));
+        CK(cudaStreamSynchronize(c->xs[0]));
+    }
+    c->last_stream = c->xs[0];
     if (n_pairs) *n_pairs = cnt;
     return NFC_OK;
 }

@@ -93,7 +93,7 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard",
            "nfc_dpi_stream_create", "nfc_dpi_stream_create_regex", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
            "nfc_dpi_stream_process", "nfc_dpi_stream_flows", "nfc_comm_unique_id", "nfc_comm_init",
-           "nfc_comm_destroy", "nfc_attach_comm"]
+           "nfc_comm_destroy", "nfc_attach_comm", "nfc_measure_peaks"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
@@ -129,6 +129,7 @@ def _load_lib():
     L.nfc_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, _P, ctypes.POINTER(_P)]
     L.nfc_comm_destroy.argtypes = [_P]
     L.nfc_attach_comm.argtypes = [_P, _P]
+    L.nfc_measure_peaks.argtypes = [ctypes.c_int, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
     P32 = ctypes.POINTER(_u32)
@@ -401,6 +402,18 @@ class DpiStream:
         nf, nu = ctypes.c_uint64(), ctypes.c_uint64()
         _check(lib.nfc_dpi_stream_flows(self.h, ctypes.byref(nf), ctypes.byref(nu)))
         return nf.value, nu.value
+
+
+class Peaks(ctypes.Structure):
+    _fields_ = [("alu_tops", ctypes.c_double), ("issue_tops", ctypes.c_double), ("smem_glookups", ctypes.c_double),
+                ("l2_gsectors", ctypes.c_double), ("sm_count", _u32), ("sm_clock_mhz", _u32)]
+
+
+def measure_peaks(device: int = 0) -> dict:
+    """nfc_measure_peaks: measured ALU / issue / shared-memory / L2-gather peaks."""
+    p = Peaks()
+    _check(lib.nfc_measure_peaks(device, ctypes.byref(p)))
+    return {f: getattr(p, f) for f, _ in Peaks._fields_}
 
 
 def comm_unique_id() -> bytes:

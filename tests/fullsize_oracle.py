@@ -18,6 +18,8 @@ from __future__ import annotations
 
 import multiprocessing as mp
 import os
+import sys
+from multiprocessing import shared_memory
 
 import numpy as np
 
@@ -25,6 +27,31 @@ import nfcgen
 import oracle
 
 _G = {}
+_SHM = []
+
+
+def _share(a: np.ndarray):
+    """Put a (large) array into POSIX shared memory for spawned workers."""
+    shm = shared_memory.SharedMemory(create=True, size=max(1, a.nbytes))
+    v = np.ndarray(a.shape, dtype=a.dtype, buffer=shm.buf)
+    v[...] = a
+    _SHM.append(shm)
+    return (shm.name, a.shape, a.dtype.str if a.dtype.names is None else a.dtype.descr)
+
+
+def _attach(spec):
+    name, shape, dt = spec
+    shm = shared_memory.SharedMemory(name=name)
+    _SHM.append(shm)
+    return np.ndarray(shape, dtype=np.dtype(dt), buffer=shm.buf)
+
+
+def _init(w, specs, first, root):
+    """Spawned worker: attach the GPU results (no CUDA, no fork of a threaded parent)."""
+    if root not in sys.path:
+        sys.path.insert(0, root)
+    recs, arena, off, gp, gq = (_attach(x) for x in specs)
+    _G.update(w=w, recs=recs.view(nfcgen.RESULT).reshape(-1), arena=arena, off=off, first=first, pairs=(gp, gq))
 
 
 def _var_layout(kinds, t):
@@ -97,6 +124,16 @@ def _check_pass(job):
     return err, orc.stats.copy(), len(fwd)
 
 
+def _free():
+    while _SHM:
+        shm = _SHM.pop()
+        shm.close()
+        try:
+            shm.unlink()
+        except FileNotFoundError:
+            pass
+
+
 def compare_full(w, recs, arena, off, pairs, n_pairs_total, stats, first=0, workers=None, chunk=None):
     """Compare the GPU pass over packets [0, n) of w's global stream (laid out as
     nfcgen.generate lays them out) with the oracle, element by element.
@@ -108,10 +145,17 @@ def compare_full(w, recs, arena, off, pairs, n_pairs_total, stats, first=0, work
     chunk = chunk or max(4096, -(-n // (4 * workers)))
     ranges = [(a, min(n, a + chunk)) for a in range(0, n, chunk)]
     order = np.lexsort((pairs[1], pairs[0]))
-    _G.update(w=w, recs=recs, arena=arena, off=off, first=first,
-              pairs=(pairs[0][order].astype(np.int64), pairs[1][order]))
-    ctx = mp.get_context("fork")
-    with ctx.Pool(workers) as pool:
+    specs = [_share(np.ascontiguousarray(recs).view(np.uint8)), _share(arena), _share(off),
+             _share(pairs[0][order].astype(np.int64)), _share(pairs[1][order].astype(np.uint16))]
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    # spawn, not fork: the parent holds CUDA and torch threads
+    ctx = mp.get_context("spawn")
+    try:
+        pool = ctx.Pool(workers, initializer=_init, initargs=(w, specs, first, root))
+    except Exception:
+        _free()
+        raise
+    with pool:
         seq = [None] * len(ranges)
         if "IPSEC" in w.kinds:
             counts = pool.map(_count_pass, ranges)
@@ -120,7 +164,7 @@ def compare_full(w, recs, arena, off, pairs, n_pairs_total, stats, first=0, work
                 seq[r] = acc.copy()
                 acc = acc + c
         out = pool.map(_check_pass, list(zip(ranges, seq)))
-    _G.clear()
+    _free()
     errs = [e for o in out for e in o[0]]
     assert not errs, "\n".join(errs[:10])
     tot = sum((o[1].astype(np.uint64) for o in out), np.zeros_like(out[0][1]))

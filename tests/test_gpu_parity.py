@@ -302,3 +302,26 @@ def test_c1_many_batches(nfc):
     ch = _chain(nfc, w)
     n = 40 * 4096 - 123
     check_parity(w, ch, n, split=[4096] * 39, match_cap=1 << 20)
+
+
+@pytest.mark.parametrize("cfg,n,shuffle", [("C1", 300_000, False), ("C2", 70_000, False), ("C1", 100_000, True)])
+def test_process_host_pipelined(nfc, cfg, n, shuffle):
+    """nfc_process_host over many pipeline chunks (H2D / kernel / D2H on two streams,
+    kernels in chunk order: ESP sequence numbers stay global), and with frames NOT laid
+    out in index order (overlapping chunk ranges: one chunk) -- records, bytes and pairs
+    equal the oracle's."""
+    import oracle
+    from tests.gpu_util import compare_bytes, sorted_pairs
+    w = nfcgen.workload(cfg, small=True)
+    w.traffic.pkt_len = 1 if cfg == "C2" else 64
+    b = nfcgen.generate(w.traffic, w.tables, 0, n)
+    if shuffle:
+        perm = np.random.default_rng(1).permutation(n)
+        b = nfcgen.Batch(b.arena, b.off[perm].copy(), b.len[perm].copy(), 0, b.headroom, b.tailroom)
+    ch = _chain(nfc, w)
+    arena = b.arena.copy()
+    rec, (mp, mq), npairs = ch.process_host(arena, b.off, b.len, match_cap=1 << 20)
+    want, want_arena, (wp, wq), wn = oracle.OracleChain(w.kinds, w.tables).run(b)
+    assert np.array_equal(rec.view(np.uint8), want.view(np.uint8))
+    compare_bytes(want, arena, b.off, want_arena, b.off, "host")
+    assert npairs == wn and np.array_equal(sorted_pairs(mp, mq), sorted_pairs(wp, wq))
