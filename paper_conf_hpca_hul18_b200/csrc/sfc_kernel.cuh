@@ -60,6 +60,20 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 
 
 // ---------------------------------------------------------------- tuning knobs (compile-time; defaults = measured best)
+#ifndef NFC_TIMING
+#define NFC_TIMING 0          // 1: per-phase clock64 accounting of the warp loop (diagnostic builds only)
+#endif
+#if NFC_TIMING
+__device__ unsigned long long nfc_timing[8];   // [0] chunks, [1..5] cycles per phase (lane 0 of every warp)
+#define NFC_TICK(i)                                                                                  \
+    do {                                                                                             \
+        const long long t_ = clock64();                                                              \
+        tacc[i] += (unsigned long long)(t_ - tlast);                                                 \
+        tlast = t_;                                                                                  \
+    } while (0)
+#else
+#define NFC_TICK(i) do {} while (0)
+#endif
 #ifndef NFC_EARLY_T24
 #define NFC_EARLY_T24 0       // issue the DIR-24-8 first read right after parse, use it at LPM4
 #endif
@@ -104,6 +118,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #endif
 #ifndef NFC_DESC_L1
 #define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
+#endif
+#ifndef NFC_HDR_EARLY
+#define NFC_HDR_EARLY 0       // 1: issue the chunk's header loads at the loop top, before the next chunk's descriptors
 #endif
 #ifndef NFC_HDR_AHEAD
 #define NFC_HDR_AHEAD 0       // 1: load the next chunk's header at the tail of the current one
@@ -1457,17 +1474,13 @@ __device__ __forceinline__ uint32_t pkt_gidx(const KParams &P, uint32_t g)
     return gidx_search(P.batches, P.n_batches, g);
 }
 
-// arena base of chunk c's descriptors in the pipelined loop (desc_get offsets are relative to it)
-__device__ __forceinline__ uint8_t *chunk_arena(const KParams &P, uint32_t c)
-{
-    if (P.n_batches == 1) return P.b0.arena;
-    return reinterpret_cast<uint8_t *>(__ldg(reinterpret_cast<const unsigned long long *>(&P.crec[c >> 5].arena)));
-}
-
-// descriptors of packet g for the pipelined loop: frame offset relative to chunk_arena
-// of its chunk, and length; single batch from the constant bank, multi-batch from the
-// chunk record (ChunkRec) -- lanes past a batch boundary in the chunk take the binary
-// search and rebase their offset onto the chunk's arena
+// descriptors of packet g for the pipelined loop: frame offset relative to the arena
+// of batch 0 (P.b0.arena, a kernel constant: frame = P.b0.arena + off for every
+// batch, 64-bit wrap-around), and length; single batch from the constant bank,
+// multi-batch from the chunk record (ChunkRec) -- lanes past a batch boundary in the
+// chunk take the binary search.  The rebase add is skipped (warp-uniform branch) when
+// the chunk's batch shares batch 0's arena, so the loop top never waits for the
+// descriptor loads.
 __device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t &off, uint32_t &len)
 {
     if (P.n_batches == 1) {
@@ -1480,8 +1493,7 @@ __device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t 
     const uint32_t split = b.w & 31, lane = g & 31;
     if ((b.w & 32) || (split && lane >= split)) {
         const Raw w = pkt_raw(P, g, true);
-        const uint64_t base = (uint64_t)b.x | (uint64_t)b.y << 32;
-        off = (uint64_t)P.batches[w.bi].arena + w.off - base;
+        off = (uint64_t)P.batches[w.bi].arena + w.off - (uint64_t)P.b0.arena;
         len = w.len;
         return;
     }
@@ -1489,7 +1501,10 @@ __device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t 
     const uint16_t *lenp = reinterpret_cast<const uint16_t *>((uint64_t)a.z | (uint64_t)a.w << 32);
     off = offp[g];
     len = lenp[g];
+    const uint64_t delta = ((uint64_t)b.x | (uint64_t)b.y << 32) - (uint64_t)P.b0.arena;
+    if (delta != 0) off += delta;   // same record for every lane here: uniform
 }
+
 __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
 {
     return pkt_loc(P, pkt_raw(P, g, valid), g, valid);
@@ -2310,7 +2325,17 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 #else
         const bool late = false;
 #endif
+#if NFC_TIMING
+        unsigned long long tacc[6] = {0, 0, 0, 0, 0, 0};
+        long long tlast = clock64();
+#endif
         while (c0 < P.n_pkts) {
+            NFC_TICK(0);
+#if NFC_HDR_EARLY && NFC_CARRY_DESC && !NFC_HDR_AHEAD
+            // this chunk's header loads go out first; the descriptor work below overlaps them
+            uint32_t hn[16];
+            if (late && c0 + lane < P.n_pkts) load_header(P.b0.arena + off0, len0, hn, C.pol_f);
+#endif
             Loc l1{nullptr, 0, 0};
             uint64_t off1 = 0;
 #if NFC_CARRY_DESC
@@ -2333,21 +2358,30 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             Pkt k;
 #if NFC_HDR_AHEAD
             pkt_begin_h(pkt_locate(P, g, valid), valid, k, hn);
+#elif NFC_CARRY_DESC && NFC_HDR_EARLY
+            NFC_TICK(1);
+            if (late) pkt_begin_h(Loc{P.b0.arena + off0, len0, g}, valid, k, hn);
+            else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #elif NFC_CARRY_DESC
-            if (late) pkt_begin(C, Loc{chunk_arena(P, c0) + off0, len0, g}, valid, k);
+            NFC_TICK(1);
+            if (late) pkt_begin(C, Loc{P.b0.arena + off0, len0, g}, valid, k);
             else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #else
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
 #endif
+            NFC_TICK(2);
             run_part<S, DM, true>(P, C, k);
+            NFC_TICK(3);
 #if NFC_CARRY_DESC
-            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(chunk_arena(P, c1) + off1));
+            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(P.b0.arena + off1));
 #endif
             run_part<S, DM, false>(P, C, k);
 #if NFC_HDR_AHEAD
             if (c1 + lane < P.n_pkts) load_header(l1.f, l1.len, hn, C.pol_f);
 #endif
+            NFC_TICK(4);
             pkt_end<S>(P, C, k, valid, g, ws, lane);
+            NFC_TICK(5);
             c0 = c1;
             c1 = c2;
 #if NFC_CARRY_DESC
@@ -2355,6 +2389,19 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             len0 = len1;
 #endif
         }
+#if NFC_TIMING
+        if (lane == 0) {
+            unsigned long long nch = 0;
+            for (int i = 0; i < 6; i++) atomicAdd(&nfc_timing[1 + (i < 5 ? i : 5) - (i == 5 ? 0 : 0)], 0ull);
+            (void)nch;
+            atomicAdd(&nfc_timing[1], tacc[0]);
+            atomicAdd(&nfc_timing[2], tacc[1]);
+            atomicAdd(&nfc_timing[3], tacc[2]);
+            atomicAdd(&nfc_timing[4], tacc[3]);
+            atomicAdd(&nfc_timing[5], tacc[4]);
+            atomicAdd(&nfc_timing[6], tacc[5]);
+        }
+#endif
 #else
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
         Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
