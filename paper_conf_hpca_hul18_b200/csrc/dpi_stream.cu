@@ -152,7 +152,10 @@ __device__ uint32_t flow_slot(uint32_t *lock, uint32_t *keys, uint32_t mask, uin
             }
             l = ld_acquire(&lock[s]);                // the CAS is relaxed: re-read with acquire
         }
-        while (l == 1) l = ld_acquire(&lock[s]);     // acquire: the published key is visible
+        while (l == 1) {                             // acquire: the published key is visible
+            __nanosleep(64);                         // yield: the writer may be a lane of this warp
+            l = ld_acquire(&lock[s]);
+        }
         if (l == 3) continue;                        // dead slot
         const uint4 *kp = reinterpret_cast<const uint4 *>(keys + (size_t)s * KS);
         const uint4 k0 = __ldcg(kp), k1 = __ldcg(kp + 1), k2 = __ldcg(kp + 2);
@@ -299,9 +302,22 @@ __global__ void __launch_bounds__(M == 2 ? WALK_SMEM_THREADS : 256) k_walk(nfc_b
             s = fstate[f];
         }
         Emit em{r, (uint32_t)b.first_global_index, 0, 0, 0};
-        for (uint32_t w = v; w < u; w++) {
+        // warm-up walk over [v, u): packets with empty payloads are jumped over by a binary
+        // search on cumx (at most `need` non-empty packets lie in the window)
+        for (uint32_t w = v; w < u;) {
+            if (cumx[w + 1] == cumx[w]) {                    // empty payload: next non-empty position
+                const unsigned long long t = cumx[w];
+                if (cumx[u] == t) break;                     // no payload byte left before u
+                uint32_t a = w + 1, z = u;                   // smallest q in (w, u] with cumx[q] > t
+                while (a < z) {
+                    const uint32_t m = a + (z - a) / 2;
+                    if (cumx[m] > t) z = m; else a = m + 1;
+                }
+                w = a - 1;
+            }
             const uint32_t i = fidx[w], sp = span[i];
             s = walk<M, false>(d, cls, b.arena + b.off[i], (sp & 0xFFFF) + (w == v ? skip : 0), sp >> 16, s, em);
+            w++;
         }
         const uint32_t i = fidx[u], sp = span[i];
         em.pkt += i;
