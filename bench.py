@@ -125,10 +125,10 @@ def batch_descs(arena, off, ln, n, first, bp):
 
 
 def alg_bytes_per_step(kinds, lens, fam, rec):
-    """Algorithmic HBM bytes of one pass: per packet
-    off+len (10 B) + header sector(s) min(len,64) [+ the rest of the frame if a payload
-    NF (DPI/IPSEC) is reached in original order] + 16 B record + 32 B header rewrite if a
-    forwarder rewrote it + the ESP output frame if IPsec ran; + 6 B per match pair."""
+    """Algorithmic HBM bytes of one pass: per packet the header bytes
+    min(len, 64) [+ the rest of the frame if a payload NF (DPI/IPSEC) is reached in
+    original order] + 16 B record + 32 B header sector if a forwarder rewrote it + the
+    ESP output frame if IPsec ran (descriptors and match pairs: other_bytes_per_step)."""
     lens = lens.astype(np.int64)
     n = len(lens)
     drop = rec["drop_nf"].astype(np.int64)
@@ -151,14 +151,19 @@ def alg_bytes_per_step(kinds, lens, fam, rec):
             rewritten |= passed(p) & (fam == 6)
         if k == "NAT":      # address/port/checksum sector [32, 64) of IPv4 packets past the NAT
             natw = passed(p) & (fam == 4)
-    rd = 10 * n + int(np.where(payload, lens, np.minimum(lens, 64)).sum())
+    rd = int(np.where(payload, lens, np.minimum(lens, 64)).sum())
     wr = 16 * n + 32 * int(rewritten.sum())
     if "NAT" in kinds:
         wr += 32 * int(natw.sum())
     esp = rec["esp_sa"] != 0xFF
     wr += int(rec["out_len"][esp].astype(np.int64).sum())
-    wr += 6 * int(rec["dpi_nmatch"].astype(np.int64).sum())
     return rd + wr, rd, wr
+
+
+def other_bytes_per_step(n, rec):
+    """Bytes the kernel also moves that SURVEY 8(d)'s per-packet count leaves out: the
+    descriptors (off u64 + len u16 = 10 B per packet) and the match pairs (6 B each)."""
+    return 10 * n + 6 * int(rec["dpi_nmatch"].astype(np.int64).sum())
 
 
 # Algorithmic integer work of IPsec ESP (DESIGN.md "ALU roofline"): a textbook
@@ -678,6 +683,8 @@ def main():
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": traffic,
             "alg_bytes_per_launch": alg, "alg_bytes_per_packet": round(alg / n, 2),
+            "alg_bytes": "SURVEY 8(d): header (+ payload if a payload NF is reached) + 16 B record + 32 B rewrite + ESP output",
+            "other_bytes_per_packet": round(other_bytes_per_step(n, rec_h) / n, 2),
             "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING fallback"}
     ops = esp_alg_ops(rec_h, l4_offsets(b)) if "IPSEC" in w.kinds else 0
     if ops:
@@ -734,6 +741,33 @@ def main():
                "h2d_bytes_per_step": len(b.arena) + n * 10,
                "d2h_bytes_per_step": len(b.arena) + n * 16 + 4 + min(npairs, cap) * 6,
                "steps": len(times), "api": "nfc_process_host (pinned host buffers)"}
+        chain.stats(reset=True)
+
+    # the general multi-batch path: the same batches in shuffled order, so the descriptors
+    # are not one run and the kernel locates packets through per-chunk records
+    general = None
+    if not args.no_unfused and len(descs) > 1 and not restore:
+        perm = np.random.default_rng(11).permutation(len(descs))
+        gdesc = nfc.Chain.batch_array([descs[i] for i in perm])
+
+        def gstep():
+            mc.zero_()
+            chain.process(gdesc, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+        for _ in range(args.warmup):
+            gstep()
+        torch.cuda.synchronize(dev)
+        ge0, ge1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ge0.record(stream)
+        for _ in range(args.steps):
+            gstep()
+        ge1.record(stream)
+        torch.cuda.synchronize(dev)
+        g_t = torch.tensor([ge0.elapsed_time(ge1)], dtype=torch.float64, device=cdev)
+        if world > 1:
+            dist.all_reduce(g_t, op=dist.ReduceOp.MAX)
+        general = {"value": round(n * args.steps * world / (float(g_t.item()) / 1e3) / 1e6, 3), "unit": "Mpps",
+                   "what": "the same batches in shuffled order: not one descriptor run, so packets are located "
+                           "through per-chunk records (k_chunk_recs + the staged record path)"}
         chain.stats(reset=True)
 
     # NEXT-1: the same chain as one kernel per NF with a device-side
@@ -850,6 +884,7 @@ def main():
             "roofline": roof,
             "measured_peaks": {k_: (round(v_, 2) if isinstance(v_, float) else v_) for k_, v_ in mpk.items()},
             "cpu_baseline": cpu,
+            "general_batch_path": general,
             "unfused_baseline": unfused,
             "sfc_parallel": parallel,
             "e2e": e2e,

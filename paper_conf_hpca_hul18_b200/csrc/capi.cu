@@ -349,6 +349,21 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         total += bs[i].n;
     }
     if (total > 0xFFFFFFFFull - 1024) return fail(NFC_EINVAL, "too many packets in one call");
+    // batches that are consecutive slices of one descriptor run (one arena, off/len arrays
+    // and global indices continuing batch to batch -- a NIC RX ring) are one batch to the
+    // kernel: the per-packet results are the same by definition, and the warp loop reads
+    // the descriptors straight from the kernel parameters instead of chunk records
+    if (nb > 1) {
+        bool run = true;
+        for (uint32_t i = 1; i < nb && run; i++)
+            run = hb[i].n == 0 || (hb[i].arena == hb[0].arena && hb[i].off == hb[0].off + hb[i].start &&
+                                   hb[i].len == hb[0].len + hb[i].start && hb[i].first == hb[0].first + hb[i].start);
+        if (run) {
+            hb[0].n = (uint32_t)total;
+            hb.resize(1);
+            nb = 1;
+        }
+    }
     c->last_stream = st;
     if (total == 0) return NFC_OK;
     int rc = set_device(c);
@@ -356,7 +371,9 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     const uint32_t TILE_N = 256;
     uint32_t n_tiles = (uint32_t)((total + TILE_N - 1) / TILE_N);
     CK(c->batches.reserve(hb.size() * sizeof(BatchDev)));
-    CK(cudaMemcpyAsync(c->batches.p, hb.data(), hb.size() * sizeof(BatchDev), cudaMemcpyHostToDevice, st));
+    // one batch travels in the kernel parameters (KParams::b0); only multi-batch calls need
+    // the descriptor array in device memory (a pageable copy: staged by the driver)
+    if (nb > 1) CK(cudaMemcpyAsync(c->batches.p, hb.data(), hb.size() * sizeof(BatchDev), cudaMemcpyHostToDevice, st));
     CK(cudaMemsetAsync(c->counter.p, 0, 4, st));
 
     KParams p{};
@@ -557,37 +574,33 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
     for (int i = 0; i < 2; i++) CK(cudaStreamWaitEvent(c->xs[i], c->xk, 0));
     CK(cudaMemsetAsync(c->h_mc.p, 0, 4, c->xs[0]));
     CK(cudaEventRecord(c->xk, c->xs[0]));          // "previous kernel done" starts as: counter zeroed
-    // chunks: about 16 per call, at least 64 K packets each; their byte ranges must be
-    // disjoint and ascending (frames laid out in index order), else one chunk
-    uint32_t per = std::max<uint32_t>(65536, (n + 15) / 16);
-    std::vector<std::pair<uint64_t, uint64_t>> rg;
-    for (int pass = 0; pass < 2; pass++) {
-        rg.clear();
-        bool ok = true;
-        for (uint32_t a0 = 0; a0 < n; a0 += per) {
-            const uint32_t cnt = std::min(per, n - a0);
-            uint64_t lo = ~0ull, hi = 0;
-            for (uint32_t i = a0; i < a0 + cnt; i++) {
-                lo = std::min(lo, off[i]);
-                hi = std::max(hi, off[i] + len[i]);
-            }
-            lo = lo >= hr ? lo - hr : 0;
-            hi = std::min<uint64_t>(hi + tr, arena_bytes);
-            if (lo > arena_bytes || hi < lo) return fail(NFC_EINVAL, "frame outside the arena");
-            if (!rg.empty() && lo < rg.back().second) ok = false;
-            rg.emplace_back(lo, hi);
-        }
-        if (ok) break;
-        per = n;                                    // overlapping chunk ranges: no pipelining
-    }
+    // chunks: about 16 per call, at least 64 K packets each.  A chunk's byte range is
+    // scanned while the previous chunks' copies and kernels run; a chunk whose range
+    // overlaps an earlier chunk's (frames not laid out in index order) first waits for
+    // everything issued before it, so it reads the rewritten bytes back consistently.
+    const uint32_t per = std::max<uint32_t>(65536, (n + 15) / 16);
     uint8_t *darena = c->h_arena.as<uint8_t>();
     uint64_t *doff = c->h_off.as<uint64_t>();
     uint16_t *dlen = c->h_len.as<uint16_t>();
+    uint64_t max_hi = 0;
     uint32_t k = 0;
     for (uint32_t a0 = 0; a0 < n; a0 += per, k++) {
         const uint32_t cnt = std::min(per, n - a0);
         cudaStream_t st = c->xs[k & 1];
-        const uint64_t lo = rg[k].first, hi = rg[k].second;
+        uint64_t lo = ~0ull, hi = 0;
+        const uint64_t *o = off + a0;
+        const uint16_t *l = len + a0;
+        for (uint32_t i = 0; i < cnt; i++) {
+            const uint64_t x = o[i], e = x + l[i];
+            lo = x < lo ? x : lo;
+            hi = e > hi ? e : hi;
+        }
+        lo = lo >= hr ? lo - hr : 0;
+        hi = std::min<uint64_t>(hi + tr, arena_bytes);
+        if (lo > arena_bytes || hi < lo) return fail(NFC_EINVAL, "frame outside the arena");
+        if (lo < max_hi)
+            for (int i = 0; i < 2; i++) CK(cudaStreamSynchronize(c->xs[i]));
+        max_hi = std::max(max_hi, hi);
         CK(cudaMemcpyAsync(darena + lo, arena + lo, hi - lo, cudaMemcpyHostToDevice, st));
         CK(cudaMemcpyAsync(doff + a0, off + a0, (size_t)cnt * 8, cudaMemcpyHostToDevice, st));
         CK(cudaMemcpyAsync(dlen + a0, len + a0, (size_t)cnt * 2, cudaMemcpyHostToDevice, st));

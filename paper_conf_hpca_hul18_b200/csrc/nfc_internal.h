@@ -179,7 +179,8 @@ struct SmemLayout {
     uint32_t frow0;
     uint32_t nat_nib;             // NAT Toeplitz nibbles
     uint32_t nh4;                 // LPM4 next-hop records (Lpm4Img::nh_smem)
-    uint32_t rk;                  // ESP: AES round keys of every SA, ESP_RK_STRIDE words each               // DM_FULL: row of slot 0 (DpiImg::frows)
+    uint32_t rk;                  // ESP: AES round keys of every SA, ESP_RK_STRIDE words each
+    uint32_t crs;                 // multi-batch: per-warp chunk-record staging (2 x 32 B, cp.async)               // DM_FULL: row of slot 0 (DpiImg::frows)
 };
 
 struct KParams {

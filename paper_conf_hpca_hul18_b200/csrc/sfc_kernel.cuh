@@ -191,6 +191,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     }
     o = (o + 15) & ~15u;
     if ((mask & MASK_LPM4) && p.l4.nh_smem) { L.nh4 = o; o += p.l4.n_nh * 16; }
+    if (p.n_batches > 1 && !(mask & MASK_IPSEC)) { L.crs = o; o += nwarp * 64; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
         L.prefix = o; o += 256 * 4;
@@ -1505,6 +1506,38 @@ __device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t 
     if (delta != 0) off += delta;   // same record for every lane here: uniform
 }
 
+// multi-batch: the chunk record of chunk c copied into this warp's shared-memory slot
+// (cp.async by lanes 0-1: no registers held; consumed a chunk later)
+__device__ __forceinline__ void crec_stage(const KParams &P, uint32_t c, uint32_t slot_addr, uint32_t lane)
+{
+    if (lane < 2 && c < P.n_pkts) {
+        const char *src = reinterpret_cast<const char *>(P.crec + (c >> 5)) + 16 * lane;
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(slot_addr + 16 * lane), "l"(src) : "memory");
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+}
+// desc_get (above) with the chunk record read from its staging slot (after cp.async.wait_all
+// and __syncwarp by the whole warp)
+__device__ __forceinline__ void desc_get_s(const KParams &P, uint32_t g, uint64_t &off, uint32_t &len, uint32_t slot_addr)
+{
+    uint4 a, b;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(a.x), "=r"(a.y), "=r"(a.z), "=r"(a.w) : "r"(slot_addr));
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(b.x), "=r"(b.y), "=r"(b.z), "=r"(b.w) : "r"(slot_addr + 16));
+    const uint32_t split = b.w & 31, lane = g & 31;
+    if ((b.w & 32) || (split && lane >= split)) {
+        const Raw w = pkt_raw(P, g, true);
+        off = (uint64_t)P.batches[w.bi].arena + w.off - (uint64_t)P.b0.arena;
+        len = w.len;
+        return;
+    }
+    const uint64_t *offp = reinterpret_cast<const uint64_t *>((uint64_t)a.x | (uint64_t)a.y << 32);
+    const uint16_t *lenp = reinterpret_cast<const uint16_t *>((uint64_t)a.z | (uint64_t)a.w << 32);
+    off = offp[g];
+    len = lenp[g];
+    const uint64_t delta = ((uint64_t)b.x | (uint64_t)b.y << 32) - (uint64_t)P.b0.arena;
+    if (delta != 0) off += delta;   // same record for every lane here: uniform
+}
+
 __device__ __forceinline__ Loc pkt_locate(const KParams &P, uint32_t g, bool valid)
 {
     return pkt_loc(P, pkt_raw(P, g, valid), g, valid);
@@ -2300,11 +2333,9 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // across a chunk -- and re-loaded (L1 hits) when the frame prefetch and the chunk need them
         auto desc_l1 = [&](uint32_t g) {
             if (g < P.n_pkts) {
-                if (P.n_batches == 1) {
+                if (P.n_batches == 1) {   // (multi-batch: chunk records staged in shared memory)
                     asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.off + g));
                     asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.len + g));
-                } else if (P.crec && lane == 0) {
-                    asm volatile("prefetch.global.L1 [%0];" ::"l"(P.crec + (g >> 5)));
                 }
             }
         };
@@ -2322,6 +2353,11 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         uint32_t len0 = 0;
         const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && (P.n_batches == 1 || P.crec != nullptr);   // warp-uniform
         if (late && c0 + lane < P.n_pkts) desc_get(P, c0 + lane, off0, len0);
+        // multi-batch: chunk records staged two chunks ahead in a per-warp 2-slot ring
+        const bool stg = late && P.n_batches > 1;                                                  // warp-uniform
+        const uint32_t crs = (uint32_t)__cvta_generic_to_shared(smem) + L.crs + warp * 64;
+        uint32_t slot1 = 32;                                                                      // c1's slot
+        if (stg) crec_stage(P, c1, crs + slot1, lane);
 #else
         const bool late = false;
 #endif
@@ -2341,10 +2377,15 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 #if NFC_CARRY_DESC
             uint32_t len1 = 0;
 #endif
+            if (stg) {
+                asm volatile("cp.async.wait_all;" ::: "memory");
+                __syncwarp();
+            }
             if (c1 + lane < P.n_pkts) {
                 if (late) {
 #if NFC_CARRY_DESC
-                    desc_get(P, c1 + lane, off1, len1);   // consumed after the head part (below)
+                    if (stg) desc_get_s(P, c1 + lane, off1, len1, crs + slot1);   // consumed after the head part
+                    else desc_get(P, c1 + lane, off1, len1);
 #endif
                 } else {
                     l1 = pkt_locate(P, c1 + lane, true);
@@ -2353,6 +2394,11 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             }
             const uint32_t c2 = claim();
             desc_l1(c2 + lane);
+            if (stg) {
+                __syncwarp();                              // every lane has read c1's slot
+                slot1 ^= 32;                               // c2 goes to the other slot
+                crec_stage(P, c2, crs + slot1, lane);
+            }
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
             Pkt k;

@@ -5,7 +5,7 @@ TESTS=$1; shift
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
 if [ -n "$TESTS" ]; then
-  timeout 1500 python -m pytest $TESTS -v -x --timeout=300 > gpurun_out/pytest.log 2>&1
+  eval "timeout 1500 python -m pytest $TESTS -v -x --timeout=300" > gpurun_out/pytest.log 2>&1
   echo "pytest rc=$?"; grep -E "PASSED|FAILED|ERROR|Timeout" gpurun_out/pytest.log | tail -3; tail -4 gpurun_out/pytest.log
 fi
 i=0
