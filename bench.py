@@ -44,6 +44,7 @@ def parse_args():
     ap.add_argument("--k", type=int, default=None, help="C5 chain length")
     ap.add_argument("--acl-rules", type=int, default=None, help="N3 (NEXT-3) ACL size: 200 / 1000 / 10000")
     ap.add_argument("--match-ppm", type=int, default=None, help="planted DPI matches per million packets (experiments)")
+    ap.add_argument("--v6-bp", type=int, default=None, help="IPv6 share in basis points (experiments)")
     ap.add_argument("--ring-mb", type=int, default=1024, help="HBM ring size per GPU (>> 126 MB L2)")
     ap.add_argument("--batch-pkts", type=int, default=BATCH,
                     help="packets per nfc_batch descriptor (SURVEY 8(c)(ii)#4: 4,096); 0 = the ring as one batch")
@@ -62,6 +63,8 @@ def make_workload(args):
     w.traffic.ttl = 255  # steps re-process the same ring: keep TTL/hop limit from expiring
     if getattr(args, "match_ppm", None) is not None:
         w.traffic.match_ppm = args.match_ppm
+    if getattr(args, "v6_bp", None) is not None:
+        w.traffic.v6_bp = args.v6_bp
     return w
 
 

@@ -119,6 +119,9 @@ __device__ unsigned long long nfc_timing[8];   // [0] chunks, [1..5] cycles per 
 #ifndef NFC_DESC_L1
 #define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
 #endif
+#ifndef NFC_WALK_AHEAD
+#define NFC_WALK_AHEAD 0      // 1: split-walk payload words loaded one 16-B step ahead
+#endif
 #ifndef NFC_HDR_EARLY
 #define NFC_HDR_EARLY 0       // 1: issue the chunk's header loads at the loop top, before the next chunk's descriptors
 #endif
@@ -264,7 +267,7 @@ __device__ __forceinline__ uint32_t ld_u16_if(bool p, const uint16_t *a, uint32_
 // A DPI walk is a dependent chain of shared-memory lookups, so the bytes ahead of it are
 // prefetched into L2 (NFC_PF_DIST bytes ahead, one 128-B line at a time).
 #ifndef NFC_PF_DIST
-#define NFC_PF_DIST 512
+#define NFC_PF_DIST 512       // split walk: L2 prefetch distance (bytes) ahead of each lane
 #endif
 __device__ __forceinline__ void prefetch_l2(const void *a) { asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a)); }
 
@@ -1717,6 +1720,10 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
         uint32_t x = 0, e0 = 0, v0 = 0, sc = 0, own = 0;
         const uint8_t *f = nullptr;
         Walk pw{0, 0, 0};
+#if NFC_WALK_AHEAD
+        uint4 qn = make_uint4(0, 0, 0, 0);     // the next 16 payload bytes, loaded one step ahead
+        bool have = false;
+#endif
         for (;;) {
             const bool need = x >= e0 && lo < hi;
             if (__any_sync(FULL, need)) {
@@ -1748,6 +1755,9 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
                     }
                     for (uint32_t l = x & ~127u; l < min(e0, x + NFC_PF_DIST); l += 128) prefetch_l2(f + l);
                     lo = ev;
+#if NFC_WALK_AHEAD
+                    have = false;
+#endif
                 }
             }
             const bool run = x < e0;
@@ -1755,7 +1765,15 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
             if (run) {
                 if (x == sc) { pw.cnt = 0; pw.mx = 0; }
                 if ((x & 127) == 0 && x + NFC_PF_DIST < e0) prefetch_l2(f + x + NFC_PF_DIST);
+#if NFC_WALK_AHEAD
+                // software-pipelined payload loads: this step's 16 bytes were loaded during the
+                // previous step; the next 16 go out now, so the walk never waits on the L2
+                const uint4 q = have ? qn : ld_stream16(f + x, C.pol_f);
+                have = x + 16 < e0;
+                if (have) qn = ld_stream16(f + x + 16, C.pol_f);
+#else
                 const uint4 q = ld_stream16(f + x, C.pol_f);
+#endif
                 uint32_t wd[4] = {q.x, q.y, q.z, q.w};
                 if ((DM == DM_FULL || NFC_HOT_FAST) && x >= v0 && x + 16 <= e0) {
 #pragma unroll
