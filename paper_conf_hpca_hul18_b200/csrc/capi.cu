@@ -97,6 +97,13 @@ struct nfc_chain {
     cudaStream_t last_stream = nullptr;
     void *comm = nullptr;                 // attached ncclComm_t (NFC_STATS_ALLREDUCE)
     cudaStream_t xs[2] = {nullptr, nullptr};   // nfc_process_host copy/compute streams
+    // a3 regrouping: mixed IPv4/IPv6 chunks of the last launch, read back asynchronously; the
+    // regrouping kernel variant runs while more than 1/8 of the chunks were mixed
+    DBuf mix_dev;
+    uint32_t *mix_host = nullptr;         // pinned
+    cudaEvent_t mix_ev = nullptr;
+    uint32_t mix_chunks = 0;
+    bool mix_pending = false, rg_on = false;
     cudaEvent_t xe[2] = {nullptr, nullptr}, xk = nullptr;
     DBuf stats_red;                       // all-reduce destination
 };
@@ -179,6 +186,9 @@ void nfc_destroy_chain(nfc_chain *c)
         if (c->xe[i]) cudaEventDestroy(c->xe[i]);
     }
     if (c->xk) cudaEventDestroy(c->xk);
+    if (c->mix_ev) cudaEventDestroy(c->mix_ev);
+    if (c->mix_host) cudaFreeHost(c->mix_host);
+    c->mix_dev.release();
     delete c;
 }
 
@@ -523,12 +533,35 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         p.crec = c->crec.as<ChunkRec>();
         c->launches++;
     }
+    const bool rg_cap = NFC_REGROUP && !par && v.dm == DM_FULL && (c->mask & MASK_ACL) && (c->mask & MASK_DPI) &&
+                        c->kind[0] == NFC_ACL && c->kind[1] == NFC_DPI && !(c->mask & MASK_IPSEC);
+    if (rg_cap) {
+        if (!c->mix_ev) {
+            CK(c->mix_dev.reserve(4));
+            CK(cudaMallocHost(&c->mix_host, 4));
+            CK(cudaEventCreateWithFlags(&c->mix_ev, cudaEventDisableTiming));
+            *c->mix_host = 0;
+        }
+        if (c->mix_pending && cudaEventQuery(c->mix_ev) == cudaSuccess) {   // the last launch's count
+            c->rg_on = (uint64_t)*c->mix_host * 8 > c->mix_chunks;
+            c->mix_pending = false;
+        }
+        v.rg = c->rg_on;
+        p.mix = c->mix_dev.as<uint32_t>();
+        CK(cudaMemsetAsync(p.mix, 0, 4, st));
+    }
     rc = par ? par_launch(p, c->device, st, err, &lc) : sfc_launch(v, p, c->device, st, err, &lc);
+    if (!rc && rg_cap && !c->mix_pending) {
+        CK(cudaMemcpyAsync(c->mix_host, p.mix, 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaEventRecord(c->mix_ev, st));
+        c->mix_chunks = (uint32_t)((total + 31) / 32);
+        c->mix_pending = true;
+    }
     if (rc) return fail(rc, err);
     c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
                               (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states,
                               p.dpi.meta_smem, p.acl.smem_words ? 4 * (p.acl.words4 + p.acl.words6) : 0u};
-    c->launches++;
+    c->launches += lc.launches;
     if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;
     return NFC_OK;
 }

@@ -10,6 +10,11 @@
 
 #include "../../include/nfc.h"
 
+#ifndef NFC_REGROUP
+#define NFC_REGROUP 0         // 1: a3 regrouping -- the IPv6 packets of mixed chunks deferred to a per-warp queue
+                              //    (family-pure chunks); measured slower than the mixed chunks (DESIGN.md a3)
+#endif
+
 namespace nfc {
 
 // ---------------------------------------------------------------- ACL
@@ -169,7 +174,7 @@ enum { MASK_ACL = 1u << NFC_ACL, MASK_DPI = 1u << NFC_DPI, MASK_LPM4 = 1u << NFC
 
 // stats vector layout
 enum { ST_PKTS = 0, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP, ST_DPI_PAIRS,
-       ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS,
+       ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS, ST_MIXED_CHUNKS,
        ST_POS_BASE = 16, ST_VAR_BASE = 64 };
 
 // byte offsets of the kernel's dynamic shared-memory regions (computed on the host per
@@ -180,7 +185,8 @@ struct SmemLayout {
     uint32_t nat_nib;             // NAT Toeplitz nibbles
     uint32_t nh4;                 // LPM4 next-hop records (Lpm4Img::nh_smem)
     uint32_t rk;                  // ESP: AES round keys of every SA, ESP_RK_STRIDE words each
-    uint32_t crs;                 // multi-batch: per-warp chunk-record staging (2 x 32 B, cp.async)               // DM_FULL: row of slot 0 (DpiImg::frows)
+    uint32_t crs;                 // multi-batch: per-warp chunk-record staging (2 x 32 B, cp.async)
+    uint32_t rgq;                 // a3 regrouping: per-warp queue of deferred IPv6 packet indices
 };
 
 struct KParams {
@@ -197,6 +203,7 @@ struct KParams {
     uint32_t n_tiles;
     uint32_t claim;              // 32-packet chunks per work claim (set by the launcher)
     const ChunkRec *crec;        // n_batches > 1: one record per 32-packet chunk (else nullptr)
+    uint32_t *mix;               // a3: mixed IPv4/IPv6 chunks of this launch (device u32, zeroed per launch)
     uint32_t *tile_counter;
     // outputs
     nfc_pkt_result *rec;
@@ -289,11 +296,15 @@ inline uint32_t l6_hash(uint32_t k0, uint32_t k1, uint32_t k2, uint32_t k3)
 
 // kernel launch (sfc_kernel.cu).  The variant is chosen from the chain kinds and
 // the DFA placement (dfa_full: the whole DFA is staged in shared memory).
-struct LaunchCfg { int grid, block; size_t smem; };
+struct LaunchCfg {
+    int grid, block;
+    size_t smem;
+    int launches = 1;            // kernel launches issued
+};
 // DFA placement: DM_HOT = hot rows in shared memory, the rest read through L2;
 // DM_FULL = the whole DFA in shared memory (one CTA per SM).
 enum { DM_HOT = 1, DM_FULL = 2 };
-struct Variant { uint32_t sig; int dm; int threads; bool esp; };
+struct Variant { uint32_t sig; int dm; int threads; bool esp; bool rg = false; };
 Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full);
 // records of every 32-packet chunk of a multi-batch call (ChunkRec), on `stream`
 int chunk_recs_launch(const BatchDev *batches, uint32_t n_batches, uint32_t n_pkts, ChunkRec *out, void *stream,

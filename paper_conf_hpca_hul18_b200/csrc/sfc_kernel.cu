@@ -19,6 +19,14 @@ NFC_DECLARE_LAUNCH(SIG_K5, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_K6, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_N3, DM_HOT)
 NFC_DECLARE_LAUNCH(SIG_ANY, DM_HOT)
+#if NFC_REGROUP
+NFC_DECLARE_LAUNCH_RG(SIG_C1, DM_FULL)
+NFC_DECLARE_LAUNCH_RG(SIG_K2, DM_FULL)
+NFC_DECLARE_LAUNCH_RG(SIG_K4, DM_FULL)
+#define NFC_RG_OR(S) (v.rg ? launch_t<S, DM_FULL, true>(p, dev, stream, err, cfg, q) : launch_t<S, DM_FULL, false>(p, dev, stream, err, cfg, q))
+#else
+#define NFC_RG_OR(S) launch_t<S, DM_FULL, false>(p, dev, stream, err, cfg, q)
+#endif
 
 // chains with a DM_FULL instantiation (no IPsec: the DFA takes the whole CTA's shared memory)
 static bool has_full(uint32_t sig) { return sig == SIG_C1 || sig == SIG_K2 || sig == SIG_K4; }
@@ -61,13 +69,12 @@ static int dispatch(const Variant &v, const KParams &p, int dev, void *stream, s
                     bool q)
 {
 #define NFC_CASE(S)                                                                                        \
-    if (v.sig == S) return v.dm == DM_FULL ? launch_t<S, DM_FULL>(p, dev, stream, err, cfg, q)            \
-                                           : launch_t<S, DM_HOT>(p, dev, stream, err, cfg, q);
+    if (v.sig == S) return v.dm == DM_FULL ? NFC_RG_OR(S) : launch_t<S, DM_HOT, false>(p, dev, stream, err, cfg, q);
     NFC_CASE(SIG_C1)
     NFC_CASE(SIG_K2)
     NFC_CASE(SIG_K4)
 #undef NFC_CASE
-#define NFC_CASE(S) if (v.sig == S) return launch_t<S, DM_HOT>(p, dev, stream, err, cfg, q);
+#define NFC_CASE(S) if (v.sig == S) return launch_t<S, DM_HOT, false>(p, dev, stream, err, cfg, q);
     NFC_CASE(SIG_C2)
     NFC_CASE(SIG_C3)
     NFC_CASE(SIG_K1)
@@ -76,7 +83,7 @@ static int dispatch(const Variant &v, const KParams &p, int dev, void *stream, s
     NFC_CASE(SIG_K6)
     NFC_CASE(SIG_N3)
 #undef NFC_CASE
-    return launch_t<SIG_ANY, DM_HOT>(p, dev, stream, err, cfg, q);
+    return launch_t<SIG_ANY, DM_HOT, false>(p, dev, stream, err, cfg, q);
 }
 
 int sfc_launch(const Variant &v, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out)

@@ -60,20 +60,6 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 
 
 // ---------------------------------------------------------------- tuning knobs (compile-time; defaults = measured best)
-#ifndef NFC_TIMING
-#define NFC_TIMING 0          // 1: per-phase clock64 accounting of the warp loop (diagnostic builds only)
-#endif
-#if NFC_TIMING
-__device__ unsigned long long nfc_timing[8];   // [0] chunks, [1..5] cycles per phase (lane 0 of every warp)
-#define NFC_TICK(i)                                                                                  \
-    do {                                                                                             \
-        const long long t_ = clock64();                                                              \
-        tacc[i] += (unsigned long long)(t_ - tlast);                                                 \
-        tlast = t_;                                                                                  \
-    } while (0)
-#else
-#define NFC_TICK(i) do {} while (0)
-#endif
 #ifndef NFC_EARLY_T24
 #define NFC_EARLY_T24 0       // issue the DIR-24-8 first read right after parse, use it at LPM4
 #endif
@@ -119,11 +105,11 @@ __device__ unsigned long long nfc_timing[8];   // [0] chunks, [1..5] cycles per 
 #ifndef NFC_DESC_L1
 #define NFC_DESC_L1 1         // descriptors prefetched into L1 two chunks ahead instead of held in registers (C1 +11 %)
 #endif
+#ifndef NFC_RGQ
+#define NFC_RGQ 48            // per-warp queue words in shared memory (47 packet indices + the length)
+#endif
 #ifndef NFC_WALK_AHEAD
 #define NFC_WALK_AHEAD 0      // 1: split-walk payload words loaded one 16-B step ahead
-#endif
-#ifndef NFC_HDR_EARLY
-#define NFC_HDR_EARLY 0       // 1: issue the chunk's header loads at the loop top, before the next chunk's descriptors
 #endif
 #ifndef NFC_HDR_AHEAD
 #define NFC_HDR_AHEAD 0       // 1: load the next chunk's header at the tail of the current one
@@ -147,6 +133,12 @@ __host__ __device__ constexpr bool kcfg_big(uint32_t S)
 __host__ __device__ constexpr int kcfg_threads(uint32_t S, int dm) { return kcfg_big(S) ? (dm == DM_FULL ? NFC_FULL_THREADS : NFC_HOTBIG_THREADS) : 256; }
 // per-warp counter slots: the fixed counters + 4 per chain position
 __host__ __device__ constexpr int kcfg_nws(uint32_t S) { return ST_POS_BASE + 4 * (S == SIG_ANY ? NFC_MAX_CHAIN : (int)sig_n(S)); }
+// chains whose warp loop regroups mixed IPv4/IPv6 chunks (NFC_REGROUP): the ones with the
+// IPv4 speculative ACL || DPI block, i.e. ACL -> DPI first with the whole DFA on chip
+__host__ __device__ constexpr bool rg_sig(uint32_t S, int dm)
+{
+    return S != SIG_ANY && dm == DM_FULL && sig_n(S) >= 2 && sig_kind(S, 0) == NFC_ACL && sig_kind(S, 1) == NFC_DPI;
+}
 template <uint32_t S, int DM> struct KCfg {
     static constexpr int nws = kcfg_nws(S);
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
@@ -195,6 +187,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     o = (o + 15) & ~15u;
     if ((mask & MASK_LPM4) && p.l4.nh_smem) { L.nh4 = o; o += p.l4.n_nh * 16; }
     if (p.n_batches > 1 && !(mask & MASK_IPSEC)) { L.crs = o; o += nwarp * 64; }
+    if (dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
         L.prefix = o; o += 256 * 4;
@@ -1509,6 +1502,14 @@ __device__ __forceinline__ void desc_get(const KParams &P, uint32_t g, uint64_t 
     if (delta != 0) off += delta;   // same record for every lane here: uniform
 }
 
+// shared-memory word the warp itself rewrites (volatile: never hoisted or merged)
+__device__ __forceinline__ uint32_t lds_u32_v(uint32_t a)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
+
 // multi-batch: the chunk record of chunk c copied into this warp's shared-memory slot
 // (cp.async by lanes 0-1: no registers held; consumed a chunk later)
 __device__ __forceinline__ void crec_stage(const KParams &P, uint32_t c, uint32_t slot_addr, uint32_t lane)
@@ -2303,7 +2304,7 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
     }
 }
 
-template <uint32_t S, int DM>
+template <uint32_t S, int DM, bool RGV>
 __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_kernel(const KParams P)
 {
     constexpr int NT = KCfg<S, DM>::threads, NW = KCfg<S, DM>::nwarp, WS = KCfg<S, DM>::nws;
@@ -2312,6 +2313,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
     const uint32_t mask = P.present & sig_mask(S);
     const SmemLayout &L = P.lay;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t NP = P.n_pkts;
     unsigned long long *wst = reinterpret_cast<unsigned long long *>(smem + L.wst);
     uint32_t *vst = reinterpret_cast<uint32_t *>(smem + L.vst);
     const uint32_t n_var = P.stats_len - NFIX;
@@ -2350,7 +2352,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         // descriptors (off/len) are prefetched into L1 two chunks ahead -- no registers held
         // across a chunk -- and re-loaded (L1 hits) when the frame prefetch and the chunk need them
         auto desc_l1 = [&](uint32_t g) {
-            if (g < P.n_pkts) {
+            if (g < NP) {
                 if (P.n_batches == 1) {   // (multi-batch: chunk records staged in shared memory)
                     asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.off + g));
                     asm volatile("prefetch.global.L1 [%0];" ::"l"(P.b0.len + g));
@@ -2359,113 +2361,112 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         };
         desc_l1(c0 + lane);
         desc_l1(c1 + lane);
-#if NFC_HDR_AHEAD
-        uint32_t hn[16];
-        if (c0 + lane < P.n_pkts) { const Loc l0 = pkt_locate(P, c0 + lane, true); load_header(l0.f, l0.len, hn, C.pol_f); }
-#endif
-#if NFC_CARRY_DESC
         // the next chunk's descriptors (off/len; multi-batch calls: from its chunk record)
         // are read at the top of the current one and carried into it, so its header loads
         // issue without a descriptor round trip
         uint64_t off0 = 0;
         uint32_t len0 = 0;
-        const bool late = NFC_PF_LATE && !NFC_HDR_AHEAD && (P.n_batches == 1 || P.crec != nullptr);   // warp-uniform
-        if (late && c0 + lane < P.n_pkts) desc_get(P, c0 + lane, off0, len0);
+        const bool late = NFC_PF_LATE && (P.n_batches == 1 || P.crec != nullptr);                 // warp-uniform
+        if (late && c0 + lane < NP) desc_get(P, c0 + lane, off0, len0);
         // multi-batch: chunk records staged two chunks ahead in a per-warp 2-slot ring
         const bool stg = late && P.n_batches > 1;                                                  // warp-uniform
         const uint32_t crs = (uint32_t)__cvta_generic_to_shared(smem) + L.crs + warp * 64;
         uint32_t slot1 = 32;                                                                      // c1's slot
         if (stg) crec_stage(P, c1, crs + slot1, lane);
-#else
-        const bool late = false;
-#endif
-#if NFC_TIMING
-        unsigned long long tacc[6] = {0, 0, 0, 0, 0, 0};
-        long long tlast = clock64();
-#endif
-        while (c0 < P.n_pkts) {
-            NFC_TICK(0);
-#if NFC_HDR_EARLY && NFC_CARRY_DESC && !NFC_HDR_AHEAD
-            // this chunk's header loads go out first; the descriptor work below overlaps them
-            uint32_t hn[16];
-            if (late && c0 + lane < P.n_pkts) load_header(P.b0.arena + off0, len0, hn, C.pol_f);
-#endif
-            Loc l1{nullptr, 0, 0};
+        // a3: family regrouping.  A chunk mixing IPv4 and IPv6 packets runs the
+        // IPv4 speculative block for neither and diverges through every NF.  The RG
+        // instantiation (NFC_REGROUP=1 builds) defers such a chunk's IPv6 packets to a per-warp
+        // queue in shared memory and runs them later as chunks of their own (a "virtual" chunk
+        // once 32 wait, the rest after the last real chunk), so every chunk a warp runs is one
+        // family; the launcher picks it while the chain's previous call saw > 1/8 mixed chunks.
+        // Measured slower on the dual-stack C5 traffic (the deferred chunks lose the descriptor
+        // and header pipelining, and the IPv4 chunks run with their IPv6 lanes idle), so the
+        // default build counts mixed chunks (ST_MIXED_CHUNKS) and runs them as they come.
+        constexpr bool RG = RGV && rg_sig(S, DM);
+        const uint32_t rgq = (uint32_t)__cvta_generic_to_shared(smem) + L.rgq + warp * NFC_RGQ * 4;   // shared address
+        const uint32_t rgn = rgq + 4 * (NFC_RGQ - 1);      // the last word: queue length
+        if (RG && lane == 0) asm volatile("st.shared.u32 [%0], %1;" ::"r"(rgn), "r"(0u) : "memory");
+        __syncwarp();
+        for (;;) {
+            const uint32_t qn = RG ? lds_u32_v(rgn) : 0u;  // deferred packets queued (warp-uniform)
+            const bool virt = RG && (qn >= 32 || (c0 >= NP && qn > 0));          // a deferred chunk
+            if (!virt && c0 >= NP) break;
             uint64_t off1 = 0;
-#if NFC_CARRY_DESC
-            uint32_t len1 = 0;
-#endif
-            if (stg) {
-                asm volatile("cp.async.wait_all;" ::: "memory");
-                __syncwarp();
+            uint32_t len1 = 0, c2 = 0, g;
+            bool valid;
+            Loc loc;
+            if (virt) {
+                valid = lane < qn;
+                g = valid ? lds_u32_v(rgq + 4 * lane) : 0u;
+                loc = pkt_locate(P, g, valid);
+            } else {
+                if (stg) {
+                    asm volatile("cp.async.wait_all;" ::: "memory");
+                    __syncwarp();
+                }
+                if (c1 + lane < NP) {
+                    if (late) {
+                        if (stg) desc_get_s(P, c1 + lane, off1, len1, crs + slot1);   // consumed after the head part
+                        else desc_get(P, c1 + lane, off1, len1);
+                    } else {
+                        asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(pkt_locate(P, c1 + lane, true).f));
+                    }
+                }
+                c2 = claim();
+                desc_l1(c2 + lane);
+                if (stg) {
+                    __syncwarp();                          // every lane has read c1's slot
+                    slot1 ^= 32;                           // c2 goes to the other slot
+                    crec_stage(P, c2, crs + slot1, lane);
+                }
+                g = c0 + lane;
+                valid = g < NP;
+                loc = late ? Loc{P.b0.arena + off0, len0, g} : pkt_locate(P, g, valid);
             }
-            if (c1 + lane < P.n_pkts) {
-                if (late) {
-#if NFC_CARRY_DESC
-                    if (stg) desc_get_s(P, c1 + lane, off1, len1, crs + slot1);   // consumed after the head part
-                    else desc_get(P, c1 + lane, off1, len1);
-#endif
-                } else {
-                    l1 = pkt_locate(P, c1 + lane, true);
-                    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(l1.f));
+            Pkt k;
+            pkt_begin(C, loc, valid, k);
+            if constexpr (rg_sig(S, DM)) {
+                if (!virt) {
+                    const uint32_t FULL = 0xFFFFFFFFu;
+                    const bool v6 = valid && k.alive && k.v.fam != 4;
+                    const uint32_t b6 = __ballot_sync(FULL, v6);
+                    if (b6 && b6 != __ballot_sync(FULL, valid && k.alive)) {     // mixed chunk
+                        if (lane == 0) ws[ST_MIXED_CHUNKS]++;
+                        if constexpr (RG) {                // defer its IPv6 lanes
+                            const uint32_t pos = qn + __popc(b6 & ((1u << lane) - 1));
+                            if (v6 && pos < NFC_RGQ - 1) { // (a full queue: the rest run here)
+                                asm volatile("st.shared.u32 [%0], %1;" ::"r"(rgq + 4 * pos), "r"(g) : "memory");
+                                k.alive = false;           // not processed in this chunk
+                                valid = false;             // no record, no counters here
+                            }
+                            __syncwarp();
+                            if (lane == 0)
+                                asm volatile("st.shared.u32 [%0], %1;" ::"r"(rgn),
+                                             "r"(min(qn + __popc(b6), (uint32_t)NFC_RGQ - 1)) : "memory");
+                            __syncwarp();
+                        }
+                    }
                 }
             }
-            const uint32_t c2 = claim();
-            desc_l1(c2 + lane);
-            if (stg) {
-                __syncwarp();                              // every lane has read c1's slot
-                slot1 ^= 32;                               // c2 goes to the other slot
-                crec_stage(P, c2, crs + slot1, lane);
-            }
-            const uint32_t g = c0 + lane;
-            const bool valid = g < P.n_pkts;
-            Pkt k;
-#if NFC_HDR_AHEAD
-            pkt_begin_h(pkt_locate(P, g, valid), valid, k, hn);
-#elif NFC_CARRY_DESC && NFC_HDR_EARLY
-            NFC_TICK(1);
-            if (late) pkt_begin_h(Loc{P.b0.arena + off0, len0, g}, valid, k, hn);
-            else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
-#elif NFC_CARRY_DESC
-            NFC_TICK(1);
-            if (late) pkt_begin(C, Loc{P.b0.arena + off0, len0, g}, valid, k);
-            else pkt_begin(C, pkt_locate(P, g, valid), valid, k);
-#else
-            pkt_begin(C, pkt_locate(P, g, valid), valid, k);
-#endif
-            NFC_TICK(2);
             run_part<S, DM, true>(P, C, k);
-            NFC_TICK(3);
-#if NFC_CARRY_DESC
-            if (late && c1 + lane < P.n_pkts) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(P.b0.arena + off1));
-#endif
+            if (!virt && late && c1 + lane < NP) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(P.b0.arena + off1));
             run_part<S, DM, false>(P, C, k);
-#if NFC_HDR_AHEAD
-            if (c1 + lane < P.n_pkts) load_header(l1.f, l1.len, hn, C.pol_f);
-#endif
-            NFC_TICK(4);
             pkt_end<S>(P, C, k, valid, g, ws, lane);
-            NFC_TICK(5);
-            c0 = c1;
-            c1 = c2;
-#if NFC_CARRY_DESC
-            off0 = off1;
-            len0 = len1;
-#endif
+            if (virt) {                                     // drop the 32 processed entries
+                const uint32_t rest = qn > 32 ? qn - 32 : 0u;
+                __syncwarp();
+                const uint32_t x = lane < rest ? lds_u32_v(rgq + 4 * (32 + lane)) : 0u;
+                __syncwarp();
+                if (lane < rest) asm volatile("st.shared.u32 [%0], %1;" ::"r"(rgq + 4 * lane), "r"(x) : "memory");
+                if (lane == 0) asm volatile("st.shared.u32 [%0], %1;" ::"r"(rgn), "r"(rest) : "memory");
+                __syncwarp();
+            } else {
+                c0 = c1;
+                c1 = c2;
+                off0 = off1;
+                len0 = len1;
+            }
         }
-#if NFC_TIMING
-        if (lane == 0) {
-            unsigned long long nch = 0;
-            for (int i = 0; i < 6; i++) atomicAdd(&nfc_timing[1 + (i < 5 ? i : 5) - (i == 5 ? 0 : 0)], 0ull);
-            (void)nch;
-            atomicAdd(&nfc_timing[1], tacc[0]);
-            atomicAdd(&nfc_timing[2], tacc[1]);
-            atomicAdd(&nfc_timing[3], tacc[2]);
-            atomicAdd(&nfc_timing[4], tacc[3]);
-            atomicAdd(&nfc_timing[5], tacc[4]);
-            atomicAdd(&nfc_timing[6], tacc[5]);
-        }
-#endif
 #else
         Loc loc = pkt_locate(P, c0 + lane, c0 + lane < P.n_pkts);
         Raw raw1 = pkt_raw(P, c1 + lane, c1 + lane < P.n_pkts);
@@ -2549,6 +2550,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         __syncwarp();
         for (uint32_t idx = lane; idx < WS; idx += 32)
             if (wst[idx]) atomicAdd(&P.stats[idx], wst[idx]);
+        if (lane == 0 && P.mix && wst[ST_MIXED_CHUNKS]) atomicAdd(P.mix, (uint32_t)wst[ST_MIXED_CHUNKS]);
     }
     if (P.smem_stats)
         for (uint32_t i = tid; i < n_var; i += NT)
@@ -2556,7 +2558,7 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
 }
 
 // ---------------------------------------------------------------- host launch
-template <uint32_t S, int DM>
+template <uint32_t S, int DM, bool RGV>
 int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCfg *cfg, bool query_only)
 {
     constexpr int NT = KCfg<S, DM>::threads;
@@ -2566,7 +2568,7 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     static size_t per_sm_smem[64] = {0};
     const int d = dev & 63;
     if ((int)smem > attr_smem[d]) {
-        if (cudaFuncSetAttribute(sfc_kernel<S, DM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+        if (cudaFuncSetAttribute(sfc_kernel<S, DM, RGV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
             err = "cudaFuncSetAttribute failed (shared memory " + std::to_string(smem) + " B)";
             return NFC_ECUDA;
         }
@@ -2574,7 +2576,7 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     }
     int per_sm = per_sm_cache[d];
     if (!per_sm || per_sm_smem[d] != smem) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sfc_kernel<S, DM>, NT, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sfc_kernel<S, DM, RGV>, NT, smem);
         if (per_sm < 1) per_sm = 1;
         per_sm_cache[d] = per_sm;
         per_sm_smem[d] = smem;
@@ -2595,7 +2597,7 @@ int launch_t(const KParams &p, int dev, void *stream, std::string &err, LaunchCf
     KParams q = p;
     q.claim = claim;
     q.lay = smem_layout(p.present & sig_mask(S), KCfg<S, DM>::nwarp, p, KCfg<S, DM>::nws, DM);
-    sfc_kernel<S, DM><<<grid, NT, smem, (cudaStream_t)stream>>>(q);
+    sfc_kernel<S, DM, RGV><<<grid, NT, smem, (cudaStream_t)stream>>>(q);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { err = std::string("sfc_kernel launch: ") + cudaGetErrorString(e); return NFC_ECUDA; }
     return NFC_OK;
@@ -2614,8 +2616,13 @@ static constexpr uint32_t SIG_K6 = make_sig(6, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_L
 static constexpr uint32_t SIG_N3 = make_sig(3, NFC_ACL, NFC_LPM4, NFC_NAT);                       // NEXT-3
 
 #define NFC_DECLARE_LAUNCH(S, DM)                                                                   \
-    extern template int launch_t<S, DM>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+    extern template int launch_t<S, DM, false>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
 #define NFC_INSTANTIATE_LAUNCH(S, DM)                                                               \
-    template int launch_t<S, DM>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+    template int launch_t<S, DM, false>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+// the a3 regrouping instantiation (rg_sig chains only)
+#define NFC_DECLARE_LAUNCH_RG(S, DM)                                                                \
+    extern template int launch_t<S, DM, true>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
+#define NFC_INSTANTIATE_LAUNCH_RG(S, DM)                                                            \
+    template int launch_t<S, DM, true>(const KParams &, int, void *, std::string &, LaunchCfg *, bool);
 
 } // namespace nfc

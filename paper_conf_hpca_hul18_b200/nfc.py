@@ -27,6 +27,7 @@ F_PARALLEL = 2  # nfc_chain_opts.flags: the chain's NFs on different warps + XOR
 # stats vector layout
 ST_PKTS, ST_BYTES_IN, ST_FWD, ST_DROP, ST_BYTES_OUT, ST_PARSE_DROP = 0, 1, 2, 3, 4, 5
 ST_DPI_PAIRS, ST_MATCH_OVF, ST_ESP_PKTS, ST_ESP_BYTES, ST_ESP_BLOCKS, ST_DPI_OVF_PKTS = 6, 7, 8, 9, 10, 11
+ST_MIXED_CHUNKS = 12   # product-only diagnostic: 32-packet chunks mixing IPv4 and IPv6 (a3 regrouping)
 ST_POS_BASE, ST_VAR_BASE = 16, 64
 
 RESULT_DTYPE = np.dtype([("drop_nf", "u1"), ("esp_sa", "u1"), ("port", "<u2"), ("acl_rule", "<u2"),

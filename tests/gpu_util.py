@@ -7,7 +7,7 @@ import numpy as np
 import nfcgen
 import oracle
 
-STATS_SKIP = {11}  # ST_DPI_OVF_PKTS: product-only diagnostic counter
+STATS_SKIP = {11, 12}  # ST_DPI_OVF_PKTS, ST_MIXED_CHUNKS: product-only diagnostic counters
 
 
 def gpu_run(chain, batches, match_cap=1 << 16):
