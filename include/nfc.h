@@ -48,7 +48,7 @@ extern "C" {
 #define NFC_ECUDA (-3)   /* CUDA runtime error (message in nfc_last_error)        */
 #define NFC_ESTATE (-4)  /* tables missing for an NF of the chain, or bad state   */
 #define NFC_ECAP (-5)    /* match pairs overflowed match_cap since last collect  */
-#define NFC_EUNSUP (-6)  /* unsupported chain (length > 6, repeated NF kind)      */
+#define NFC_EUNSUP (-6)  /* unsupported chain (length > 6, repeated IPsec / NAT)  */
 
 /* NF kinds (Table II P:L213-223 rows Firewall, IDS/DPI, LB; P:L128 IPv4/IPv6
  * forwarders; P:L130 IPsec gateway). */
@@ -84,8 +84,10 @@ typedef struct {
     uint32_t max_batch_pkts; /* hint: largest packet count per nfc_process_batch call */
 } nfc_chain_opts;
 
-/* Create a chain. kinds[0..n) = NF kinds in ORIGINAL SFC order; 1 <= n <= 6,
- * each kind at most once (else NFC_EUNSUP).  Allocates device state (stats,
+/* Create a chain. kinds[0..n) = NF kinds in ORIGINAL SFC order; 1 <= n <= 6.
+ * A kind may repeat (the paper's chains of four identical FW or IDS NFs, P:L318
+ * [SV.B.1], Fig. 13): positions of one kind share that kind's tables; NFC_IPSEC
+ * and NFC_NAT at most once (else NFC_EUNSUP).  Allocates device state (stats,
  * ESP sequence counters, scheduling scratch) on opts->device.  *out is owned by
  * the caller and released with nfc_destroy_chain. */
 NFC_API int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opts, nfc_chain **out);
@@ -300,6 +302,14 @@ NFC_API int nfc_rss_shard(int device, const nfc_batch *b, uint32_t n_shards, uin
  * a packet field, per packet family); IPsec always stands alone.  NFC_EINVAL for
  * NULL pointers, n outside 1..6 or an unknown kind. */
 NFC_API int nfc_plan_parallel(const uint32_t *kinds, uint32_t n, uint8_t *group);
+/* The grouping an NFC_F_PARALLEL chain runs (default: nfc_plan_parallel's maximal
+ * groups).  group[p] (n bytes, host) = group of position p: group[0] = 0, each next
+ * position the same group or the next, every group pairwise parallel-legal (R#16);
+ * else NFC_EINVAL.  Groups run one after another, the members of a group at once on
+ * copies of the packet entering it, merged by XOR -- e.g. the paper's
+ * configuration (c) of four identical NFs = groups {0,0,1,1} (Fig. 13). */
+NFC_API int nfc_set_groups(nfc_chain *c, const uint8_t *group);
+NFC_API int nfc_get_groups(const nfc_chain *c, uint8_t *group);
 
 /* ---------------------------------------------------------------- stateful DPI
  * stateful, cross-packet DPI (PAPER.md P:L161 [SIII.B.b]

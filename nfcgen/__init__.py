@@ -555,4 +555,14 @@ def workload(name: str, pkt_len: Optional[int] = None, k: Optional[int] = None,
                            l4csum=1)
         gen_nat(np.random.default_rng(np.random.PCG64(sd + 1000)), tp, t, n_dnat=1000 if not small else 200)
         return Workload(f"N3_{n_acl}", kinds, t, tp, note=f"FW({n_acl})->IPv4 router(1K)->NAT44, SNAT+DNAT")
+    if name in ("NX2", "NX2_FW", "NX2_IDS"):
+        # SURVEY 8(f) NEXT-2 (Figs. 13-14): four identical NFs in sequence,
+        # 64-B TCP traffic, firewall rules that never drop
+        nf = "DPI" if name == "NX2_IDS" else "ACL"
+        kinds = [nf] * 4
+        sd = 7 if seed is None else seed
+        t = make_tables(sd, ["ACL", "DPI"], n_acl=64, n_pat=100, n_r4=1000, acl_deny=0.0)
+        tp = TrafficParams(seed=sd, pkt_len=64 if pkt_len is None else pkt_len, tcp_pct=100)
+        return Workload(f"NX2_{'IDS' if nf == 'DPI' else 'FW'}", kinds, t, tp,
+                        note=f"4 x {'IDS (Aho-Corasick, 100 patterns)' if nf == 'DPI' else 'FW (64 rules, never drop)'}, 64 B TCP")
     raise ValueError(name)

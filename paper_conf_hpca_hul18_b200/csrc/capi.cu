@@ -64,6 +64,7 @@ struct nfc_chain {
     uint32_t mask = 0;
     uint32_t esp_pos = 0xFF;
     uint32_t flags = 0;
+    uint8_t group[NFC_MAX_CHAIN] = {0};   // NFC_F_PARALLEL groups (default: nfc_plan_parallel)
     nfc_launch_info last{};               // shape of the last fused launch
     DBuf uf_list[2], uf_cnt, uf_pass;     // NFC_F_UNFUSED scratch
     bool loaded[8] = {false};
@@ -134,7 +135,11 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
     uint32_t mask = 0;
     for (uint32_t i = 0; i < n; i++) {
         if (kinds[i] < NFC_ACL || kinds[i] > NFC_NAT) return fail(NFC_EINVAL, "unknown NF kind");
-        if (mask & (1u << kinds[i])) return fail(NFC_EUNSUP, "repeated NF kind in chain");
+        // repeated kinds (the paper's four identical FW / IDS NFs, Fig. 13)
+        // share the kind's tables; IPsec and NAT keep per-chain state or decide on metadata
+        // of one position (the ESP sequence look-back, the NAT's egress-port test): once each
+        if ((mask & (1u << kinds[i])) && (kinds[i] == NFC_IPSEC || kinds[i] == NFC_NAT))
+            return fail(NFC_EUNSUP, "IPsec / NAT at most once per chain");
         mask |= 1u << kinds[i];
     }
     const uint32_t flags = opts ? opts->flags : 0;
@@ -153,6 +158,7 @@ int nfc_build_chain(const uint32_t *kinds, uint32_t n, const nfc_chain_opts *opt
         c->kind[i] = kinds[i];
         if (kinds[i] == NFC_IPSEC) c->esp_pos = i;
     }
+    nfc_plan_parallel(kinds, n, c->group);             // NFC_F_PARALLEL grouping (nfc_set_groups)
     int rc = set_device(c);
     if (rc == NFC_OK) {
         cudaError_t e = c->counter.reserve(16);
@@ -389,6 +395,8 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     KParams p{};
     p.n_nf = c->n_nf;
     for (uint32_t i = 0; i < c->n_nf; i++) p.kind[i] = c->kind[i];
+    for (uint32_t i = 0; i < c->n_nf; i++) p.group[i] = c->group[i];
+    p.n_groups = (uint32_t)c->group[c->n_nf - 1] + 1;
     p.esp_pos = c->esp_pos;
     p.present = c->mask;
     p.batches = c->batches.as<BatchDev>();
@@ -694,6 +702,22 @@ int nfc_collect_stats(nfc_chain *c, uint64_t *out, size_t cap, uint32_t flags)
     size_t k = cap < h.size() ? cap : h.size();
     if (k) memcpy(out, h.data(), k * 8);
     if (h[ST_MATCH_OVF]) return fail(NFC_ECAP, "match pairs exceeded match_cap");
+    return NFC_OK;
+}
+
+int nfc_set_groups(nfc_chain *c, const uint8_t *group)
+{
+    if (!c || !group) return fail(NFC_EINVAL, "NULL argument");
+    if (!groups_legal(c->kind, c->n_nf, group))
+        return fail(NFC_EINVAL, "groups must be runs of consecutive, pairwise parallel-legal NFs (nfc_plan_parallel)");
+    for (uint32_t i = 0; i < c->n_nf; i++) c->group[i] = group[i];
+    return NFC_OK;
+}
+
+int nfc_get_groups(const nfc_chain *c, uint8_t *group)
+{
+    if (!c || !group) return fail(NFC_EINVAL, "NULL argument");
+    for (uint32_t i = 0; i < c->n_nf; i++) group[i] = c->group[i];
     return NFC_OK;
 }
 

@@ -204,6 +204,8 @@ struct KParams {
     uint32_t claim;              // 32-packet chunks per work claim (set by the launcher)
     const ChunkRec *crec;        // n_batches > 1: one record per 32-packet chunk (else nullptr)
     uint32_t *mix;               // a3: mixed IPv4/IPv6 chunks of this launch (device u32, zeroed per launch)
+    uint8_t group[NFC_MAX_CHAIN]; // NFC_F_PARALLEL: parallel group of each chain position (runs, in order)
+    uint32_t n_groups;
     uint32_t *tile_counter;
     // outputs
     nfc_pkt_result *rec;
@@ -309,6 +311,9 @@ Variant sfc_variant(const uint32_t *kinds, uint32_t n, bool dfa_full);
 // records of every 32-packet chunk of a multi-batch call (ChunkRec), on `stream`
 int chunk_recs_launch(const BatchDev *batches, uint32_t n_batches, uint32_t n_pkts, ChunkRec *out, void *stream,
                       std::string &err);
+// planner.cpp: true iff every group of `group` is a run of consecutive positions whose
+// members are pairwise parallel-legal (group[0] = 0, steps of 0 or 1)
+bool groups_legal(const uint32_t *kinds, uint32_t n, const uint8_t *group);
 int sfc_launch(const Variant &v, const KParams &p, int device, void *stream, std::string &err, LaunchCfg *cfg_out);
 size_t sfc_smem_bytes(const Variant &v, const KParams &p);
 size_t sfc_smem_limit(int device);      // max dynamic shared memory per CTA (opt-in)

@@ -37,7 +37,7 @@ __host__ __device__ inline uint32_t par_teams(uint32_t n_nf) { return min((uint3
 size_t par_region_bytes(uint32_t n_nf, uint32_t n_fwd)
 {
     const uint32_t teams = par_teams(n_nf);
-    return (size_t)teams * (n_nf * 32 * 16 + n_fwd * 32 * 32 + 16);
+    return (size_t)teams * (n_nf * 32 * 16 + n_fwd * 32 * 32 + 16 + 32 * 4);
 }
 
 __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_t n_fwd)
@@ -58,10 +58,11 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
     __syncthreads();
 
     if (team < teams) {
-        uint8_t *tb = smem + L.par + team * (n * 32 * 16 + n_fwd * 32 * 32 + 16);
+        uint8_t *tb = smem + L.par + team * (n * 32 * 16 + n_fwd * 32 * 32 + 16 + 32 * 4);
         uint4 *eff = reinterpret_cast<uint4 *>(tb);                        // [n][32]
         uint32_t *hcopy = reinterpret_cast<uint32_t *>(tb + n * 32 * 16);  // [n_fwd][8 words][32]
         uint32_t *s_chunk = reinterpret_cast<uint32_t *>(tb + n * 32 * 16 + n_fwd * 32 * 32);
+        uint32_t *s_alive = s_chunk + 4;                                   // [32]: packet alive after a group
         unsigned long long *ws = wst + warp * NWS;
         // slot of this member's header copy (forwarders only)
         uint32_t fslot = 0;
@@ -75,103 +76,125 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
             if (c0 >= P.n_pkts) break;
             const uint32_t g = c0 + lane;
             const bool valid = g < P.n_pkts;
+            const Loc loc = pkt_locate(P, g, valid);
             Pkt k;
-            pkt_begin(C, pkt_locate(P, g, valid), valid, k);             // this member's copy
-            // ---- member j: NF j on its copy, no side effects outside the team
-            uint32_t x = 0, y = 0xFFFFFFFFu, z = 0, w = 0;
-            if (valid && k.alive) {
-                if (kind == NFC_ACL) {
-                    const uint32_t r = nf_acl(C.acl4, C.acl6, P.acl, k.v);
-                    y = (r & 0xFFFF) | 0xFFFF0000u;
-                    x = (r >> 31) << 16;
-                } else if (kind == NFC_DPI) {
-                    const Walk wk = dpi_walk<DM_HOT>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
-                    z = wk.cnt;
-                    w = wk.mx;
-                    bool drop = false;
-                    const uint32_t st = C.dpi.wide ? (wk.mx & 0x7FFFFFFFu) : (wk.mx & 0x7FFFu);
-                    const uint32_t meta = wk.cnt == 1 ? C.meta[st] : 0u;
-                    if (wk.cnt == 1 && meta != DPI_META_NONE) {
-                        drop = (meta >> 31) != 0;
-                    } else if (wk.cnt >= 1) {                             // exact set: DROP flag only
-                        const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt,
-                                        P.match_pat, P.match_cap, P.stats, 0u};
-                        drop = (dpi_slow<DM_HOT>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, pkt_gidx(P, k.g)) >> 31) != 0;
-                    }
-                    x = (uint32_t)drop << 16;
-                } else if (kind == NFC_LPM4 || kind == NFC_LPM6) {
-                    const uint32_t fam = kind == NFC_LPM4 ? 4 : 6;
-                    if (k.v.fam != fam) {
-                        x = 1u << 17;                                      // passes the other family
-                    } else {
-                        uint32_t nh;
-                        if (fam == 4) {
-                            nh = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
-                            if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
-                        } else {
-                            nh = lpm6_lookup(P.l6, k.v.dst);
-                        }
-                        if (nh == 0x7FFF || hbyte(k.h, fam == 4 ? 22 : 21) <= 1) {
-                            x = 1u << 16;
-                        } else {
-                            const uint2 e = __ldg((fam == 4 ? P.l4.nh : P.l6.nh) + nh);
-                            const uint32_t pt = e.y >> 16;
-                            forward_words(k.f, k.h, k.v, e, __ldg((fam == 4 ? P.l4.pmac : P.l6.pmac) + pt));
-                            x = pt | 1u << 18;
-                        }
-                    }
-                } else if (kind == NFC_LB) {
-                    const uint32_t b = (uint32_t)(((uint64_t)toeplitz(C.lb_nib, k.v) * P.lb.n_backends) >> 32);
-                    y = 0xFFFFu | b << 16;
-                    x = __ldg(P.lb.port + b) | 1u << 18;
-                }
-            }
-            eff[j * 32 + lane] = make_uint4(x, y, z, w);
-            if (kind == NFC_LPM4 || kind == NFC_LPM6) {
-#pragma unroll
-                for (int q = 0; q < 8; q++) hcopy[(fslot * 8 + q) * 32 + lane] = k.h[q];
-                if (j == 0 && valid) load_header(k.f, k.flen, k.h, C.pol_f);   // the leader merges against the original
-            }
-            bar_team(bar, bthreads);
-            // ---- leader: merge and commit
-            if (j == 0) {
-                if (valid && k.alive) {
-                    uint32_t acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-                    uint32_t fs = 0;
-                    for (uint32_t p = 0; p < n; p++) {
-                        const uint4 e = eff[p * 32 + lane];
-                        const uint32_t kd = P.kind[p];
-                        if (kd == NFC_LPM4 || kd == NFC_LPM6) {
-#pragma unroll
-                            for (int q = 0; q < 8; q++) acc[q] |= k.h[q] ^ hcopy[(fs * 8 + q) * 32 + lane];
-                            fs++;
-                        }
-                        if (kd == NFC_ACL) {
-                            k.acl_rule = e.y & 0xFFFF;
-                            var_stat(P, C, P.st_acl + (k.acl_rule == 0xFFFF ? P.acl.n_rules : k.acl_rule));
-                        } else if (kd == NFC_DPI && e.z) {
-                            const Walk wk{0, e.z, e.w};
-                            dpi_finish<DM_HOT>(P, C, k, wk);                // emits the pairs, sets nmatch
-                        } else if (kd == NFC_LB) {
-                            k.lb_b = e.y >> 16;
-                            var_stat(P, C, P.st_lb + k.lb_b);
-                        }
-                        if ((e.x >> 18) & 1) k.port = e.x & 0xFFFF;
-                        if ((e.x >> 17) & 1) k.passmask |= 1u << p;
-                        if ((e.x >> 16) & 1) { k.drop = p; k.alive = false; break; }
-                    }
-                    if (k.alive) {                                         // merged header bytes
-                        uint32_t any = 0;
-#pragma unroll
-                        for (int q = 0; q < 8; q++) { k.h[q] ^= acc[q]; any |= acc[q]; }
-                        if (any) {
-                            st_stream16(k.f, make_uint4(k.h[0], k.h[1], k.h[2], k.h[3]), C.pol_f);
-                            st_stream16(k.f + 16, make_uint4(k.h[4], k.h[5], k.h[6], k.h[7]), C.pol_f);
-                        }
+            pkt_begin(C, loc, valid, k);                                  // this member's copy
+            // groups in order (configuration (c) of Fig. 13 has two): the members
+            // of group gi run on copies of the packet that enters gi (the merge of the groups
+            // before it, re-read from memory), the leader merges them, and the next group starts
+            for (uint32_t gi = 0; gi < P.n_groups; gi++) {
+                const bool mem = P.group[j] == gi;
+                if (gi > 0) {
+                    bar_team(bar, bthreads);                               // the leader's merge of gi-1 is out
+                    if (mem) {
+                        pkt_begin(C, loc, valid, k);                       // the packet entering gi
+                        if (!s_alive[lane]) k.alive = false;
                     }
                 }
-                pkt_end<SIG_ANY>(P, C, k, valid, g, ws, lane);
+                // ---- member j of group gi: NF j on its copy, no side effects outside the team
+                if (mem) {
+                    uint32_t x = 0, y = 0xFFFFFFFFu, z = 0, w = 0;
+                    if (valid && k.alive) {
+                        if (kind == NFC_ACL) {
+                            const uint32_t r = nf_acl(C.acl4, C.acl6, P.acl, k.v);
+                            y = (r & 0xFFFF) | 0xFFFF0000u;
+                            x = (r >> 31) << 16;
+                        } else if (kind == NFC_DPI) {
+                            const Walk wk = dpi_walk<DM_HOT>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f);
+                            z = wk.cnt;
+                            w = wk.mx;
+                            bool drop = false;
+                            const uint32_t st = C.dpi.wide ? (wk.mx & 0x7FFFFFFFu) : (wk.mx & 0x7FFFu);
+                            const uint32_t meta = wk.cnt == 1 ? C.meta[st] : 0u;
+                            if (wk.cnt == 1 && meta != DPI_META_NONE) {
+                                drop = (meta >> 31) != 0;
+                            } else if (wk.cnt >= 1) {                     // exact set: DROP flag only
+                                const DpiOvf ov{P.dpi.ovf_bitmap, P.dpi.bitmap_words, P.match_count, P.match_pkt,
+                                                P.match_pat, P.match_cap, P.stats, 0u};
+                                drop = (dpi_slow<DM_HOT>(C.dpi, k.f, k.v.pl_off, k.v.ip_end, C.gtid, ov, pkt_gidx(P, k.g)) >> 31) != 0;
+                            }
+                            x = (uint32_t)drop << 16;
+                        } else if (kind == NFC_LPM4 || kind == NFC_LPM6) {
+                            const uint32_t fam = kind == NFC_LPM4 ? 4 : 6;
+                            if (k.v.fam != fam) {
+                                x = 1u << 17;                              // passes the other family
+                            } else {
+                                uint32_t nh;
+                                if (fam == 4) {
+                                    nh = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
+                                    if (nh & 0x8000) nh = ld_tab16(P.l4.tbllong + ((nh & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
+                                } else {
+                                    nh = lpm6_lookup(P.l6, k.v.dst);
+                                }
+                                if (nh == 0x7FFF || hbyte(k.h, fam == 4 ? 22 : 21) <= 1) {
+                                    x = 1u << 16;
+                                } else {
+                                    const uint2 e = __ldg((fam == 4 ? P.l4.nh : P.l6.nh) + nh);
+                                    const uint32_t pt = e.y >> 16;
+                                    forward_words(k.f, k.h, k.v, e, __ldg((fam == 4 ? P.l4.pmac : P.l6.pmac) + pt));
+                                    x = pt | 1u << 18;
+                                }
+                            }
+                        } else if (kind == NFC_LB) {
+                            const uint32_t b = (uint32_t)(((uint64_t)toeplitz(C.lb_nib, k.v) * P.lb.n_backends) >> 32);
+                            y = 0xFFFFu | b << 16;
+                            x = __ldg(P.lb.port + b) | 1u << 18;
+                        }
+                    }
+                    eff[j * 32 + lane] = make_uint4(x, y, z, w);
+                    if (kind == NFC_LPM4 || kind == NFC_LPM6) {
+#pragma unroll
+                        for (int q = 0; q < 8; q++) hcopy[(fslot * 8 + q) * 32 + lane] = k.h[q];
+                        if (j == 0 && valid) load_header(k.f, k.flen, k.h, C.pol_f);   // the leader merges against the original
+                    }
+                }
+                bar_team(bar, bthreads);
+                // ---- leader: merge group gi and commit
+                if (j == 0) {
+                    if (valid && k.alive) {
+                        uint32_t acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                        uint32_t fs = 0;
+                        for (uint32_t p = 0; p < n; p++) {
+                            const uint32_t kd = P.kind[p];
+                            const bool fwd = kd == NFC_LPM4 || kd == NFC_LPM6;
+                            if (P.group[p] != gi) { fs += fwd; continue; }
+                            const uint4 e = eff[p * 32 + lane];
+                            if (fwd) {
+#pragma unroll
+                                for (int q = 0; q < 8; q++) acc[q] |= k.h[q] ^ hcopy[(fs * 8 + q) * 32 + lane];
+                                fs++;
+                            }
+                            if (kd == NFC_ACL) {
+                                k.acl_rule = e.y & 0xFFFF;
+                                var_stat(P, C, P.st_acl + (k.acl_rule == 0xFFFF ? P.acl.n_rules : k.acl_rule));
+                            } else if (kd == NFC_DPI) {
+                                k.nmatch = 0;
+                                if (e.z) {
+                                    const Walk wk{0, e.z, e.w};
+                                    dpi_finish<DM_HOT>(P, C, k, wk);       // emits the pairs, sets nmatch
+                                }
+                            } else if (kd == NFC_LB) {
+                                k.lb_b = e.y >> 16;
+                                var_stat(P, C, P.st_lb + k.lb_b);
+                            }
+                            if ((e.x >> 18) & 1) k.port = e.x & 0xFFFF;
+                            if ((e.x >> 17) & 1) k.passmask |= 1u << p;
+                            if ((e.x >> 16) & 1) { k.drop = p; k.alive = false; break; }
+                        }
+                        if (k.alive) {                                     // merged header bytes
+                            uint32_t any = 0;
+#pragma unroll
+                            for (int q = 0; q < 8; q++) { k.h[q] ^= acc[q]; any |= acc[q]; }
+                            if (any) {
+                                st_stream16(k.f, make_uint4(k.h[0], k.h[1], k.h[2], k.h[3]), C.pol_f);
+                                st_stream16(k.f + 16, make_uint4(k.h[4], k.h[5], k.h[6], k.h[7]), C.pol_f);
+                            }
+                        }
+                    }
+                    if (gi + 1 < P.n_groups) s_alive[lane] = valid && k.alive;
+                }
             }
+            if (j == 0) pkt_end<SIG_ANY>(P, C, k, valid, g, ws, lane);
         }
     }
     // ---- flush CTA counters (as sfc_kernel)

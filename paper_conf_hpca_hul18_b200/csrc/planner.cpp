@@ -58,6 +58,19 @@ bool legal_pair(uint32_t a, uint32_t b)
 }
 } // namespace
 
+namespace nfc {
+bool groups_legal(const uint32_t *kinds, uint32_t n, const uint8_t *group)
+{
+    if (!kinds || !group || n == 0 || n > NFC_MAX_CHAIN || group[0] != 0) return false;
+    for (uint32_t p = 1; p < n; p++)
+        if (group[p] != group[p - 1] && group[p] != group[p - 1] + 1) return false;
+    for (uint32_t p = 0; p < n; p++)
+        for (uint32_t q = p + 1; q < n && group[q] == group[p]; q++)
+            if (!legal_pair(kinds[p], kinds[q])) return false;
+    return true;
+}
+} // namespace nfc
+
 extern "C" NFC_API int nfc_plan_parallel(const uint32_t *kinds, uint32_t n, uint8_t *group)
 {
     if (!kinds || !group || n == 0 || n > NFC_MAX_CHAIN) return NFC_EINVAL;

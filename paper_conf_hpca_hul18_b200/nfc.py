@@ -94,7 +94,7 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_launch_count", "nfc_last_launch", "nfc_plan_parallel", "nfc_last_error", "nfc_version", "nfc_rss_shard",
            "nfc_dpi_stream_create", "nfc_dpi_stream_create_regex", "nfc_dpi_stream_destroy", "nfc_dpi_stream_reset",
            "nfc_dpi_stream_process", "nfc_dpi_stream_flows", "nfc_comm_unique_id", "nfc_comm_init",
-           "nfc_comm_destroy", "nfc_attach_comm", "nfc_measure_peaks"]
+           "nfc_comm_destroy", "nfc_attach_comm", "nfc_measure_peaks", "nfc_set_groups", "nfc_get_groups"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
                  "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
@@ -131,6 +131,8 @@ def _load_lib():
     L.nfc_comm_destroy.argtypes = [_P]
     L.nfc_attach_comm.argtypes = [_P, _P]
     L.nfc_measure_peaks.argtypes = [ctypes.c_int, _P]
+    L.nfc_set_groups.argtypes = [_P, _P]
+    L.nfc_get_groups.argtypes = [_P, _P]
     L.nfc_last_error.restype = ctypes.c_char_p
     L.nfc_version.restype = ctypes.c_char_p
     P32 = ctypes.POINTER(_u32)
@@ -235,8 +237,9 @@ class Chain:
                                        ext_ports, k.ctypes.data))
 
     def load_tables(self, t):
-        """Load every NF of the chain from an object with the nfcgen.Tables fields."""
-        for k in self.kinds:
+        """Load every NF of the chain from an object with the nfcgen.Tables fields
+        (a repeated kind shares its tables: loaded once)."""
+        for k in dict.fromkeys(self.kinds):
             if k == ACL:
                 self.load_acl(t.acl_rules, t.acl_default)
             elif k == DPI:
@@ -321,6 +324,16 @@ class Chain:
         _check(lib.nfc_collect_stats(self.h, out.ctypes.data, n.value, flags),
                allow=(NFC_ECAP,) if allow_cap else ())
         return out
+
+    def set_groups(self, group):
+        """nfc_set_groups: the parallel grouping of an F_PARALLEL chain (runs of legal NFs)."""
+        g = np.array(list(group) + [0] * (8 - len(group)), dtype=np.uint8)
+        _check(lib.nfc_set_groups(self.h, g.ctypes.data))
+
+    def groups(self) -> list:
+        g = np.zeros(8, dtype=np.uint8)
+        _check(lib.nfc_get_groups(self.h, g.ctypes.data))
+        return [int(x) for x in g[:len(self.kinds)]]
 
     def attach_comm(self, comm: Optional["Comm"]):
         """nfc_attach_comm: the NCCL communicator NFC_STATS_ALLREDUCE sums over (None detaches)."""

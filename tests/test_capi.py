@@ -57,12 +57,14 @@ def test_validation_before_cuda(nfc):
     assert lib.nfc_build_chain(empty, 0, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
     seven = (ctypes.c_uint32 * 7)(1, 2, 3, 4, 5, 6, 1)
     assert lib.nfc_build_chain(seven, 7, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
-    rep = (ctypes.c_uint32 * 2)(1, 1)
+    rep = (ctypes.c_uint32 * 2)(nfc.IPSEC, nfc.IPSEC)   # repeated IPsec / NAT: unsupported (repeated ACL/DPI: NEXT-2)
     assert lib.nfc_build_chain(rep, 2, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
+    rep = (ctypes.c_uint32 * 3)(nfc.ACL, nfc.NAT, nfc.NAT)
+    assert lib.nfc_build_chain(rep, 3, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EUNSUP
     bad = (ctypes.c_uint32 * 1)(9)
     assert lib.nfc_build_chain(bad, 1, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EINVAL
     assert lib.nfc_build_chain(None, 1, ctypes.byref(opts), ctypes.byref(h)) == nfc.NFC_EINVAL
-    assert b"repeated" in lib.nfc_last_error() or len(lib.nfc_last_error()) > 0
+    assert len(lib.nfc_last_error()) > 0
     assert lib.nfc_load_tables(None, 1, None, 0) == nfc.NFC_EINVAL
     assert lib.nfc_collect_stats(None, None, 0, 0) == nfc.NFC_EINVAL
     assert nfc.version().startswith("nfc-b200")

@@ -325,3 +325,56 @@ def test_process_host_pipelined(nfc, cfg, n, shuffle):
     assert np.array_equal(rec.view(np.uint8), want.view(np.uint8))
     compare_bytes(want, arena, b.off, want_arena, b.off, "host")
     assert npairs == wn and np.array_equal(sorted_pairs(mp, mq), sorted_pairs(wp, wq))
+
+
+# ---------------------------------------------------------------- NEXT-2: identical NFs
+REPEATED = [["ACL"] * 4, ["DPI"] * 4, ["ACL", "DPI", "ACL", "LPM4", "LPM4"], ["LB", "ACL", "LB"]]
+
+
+def _rep_workload(kinds):
+    w = nfcgen.workload("NX2_FW")
+    w.tables = nfcgen.make_tables(9, ["ACL", "DPI", "LPM4", "LB"], n_acl=64, n_pat=100, n_r4=1000, acl_deny=0.1)
+    w.kinds = list(kinds)
+    w.traffic.pkt_len, w.traffic.match_ppm, w.traffic.tcp_pct = 1, 200_000, 40
+    w.traffic.edge(50_000)
+    return w
+
+
+@pytest.mark.parametrize("kinds", REPEATED)
+@pytest.mark.parametrize("mode", ["fused", "unfused", "parallel"])
+def test_repeated_kinds_parity(nfc, kinds, mode):
+    """SURVEY 8(f) NEXT-2 (Fig. 13): chains with repeated NF kinds (four identical
+    FW or IDS NFs; a forwarder twice) -- fused (configuration d), one kernel per NF (a),
+    parallel groups (b: nfc_plan_parallel's) -- equal the sequential oracle."""
+    w = _rep_workload(kinds)
+    flags = {"fused": 0, "unfused": nfc.F_UNFUSED, "parallel": nfc.F_PARALLEL}[mode]
+    ch = nfc.Chain(w.kinds, device=0, flags=flags)
+    ch.load_tables(w.tables)
+    check_parity(w, ch, 3001)
+
+
+@pytest.mark.parametrize("kinds,groups", [(["ACL"] * 4, [0, 0, 1, 1]), (["DPI"] * 4, [0, 0, 1, 1]),
+                                          (["DPI"] * 4, [0, 1, 2, 3]), (["ACL", "DPI", "ACL", "LPM4", "LPM4"], [0, 1, 1, 2, 3]),
+                                          (["LB", "ACL", "LB"], [0, 0, 1])])
+def test_parallel_explicit_groups(nfc, kinds, groups):
+    """NFC_F_PARALLEL with a chosen grouping (the paper's configuration (c): two groups of
+    two identical NFs): groups run in order, members on copies of the packet that
+    enters their group, XOR merge -- equal the sequential oracle."""
+    w = _rep_workload(kinds)
+    ch = nfc.Chain(w.kinds, device=0, flags=nfc.F_PARALLEL)
+    ch.load_tables(w.tables)
+    ch.set_groups(groups)
+    assert ch.groups() == groups
+    check_parity(w, ch, 3001)
+
+
+def test_parallel_groups_validated(nfc):
+    ch = nfc.Chain(["ACL", "LPM4", "LPM4"], device=0, flags=nfc.F_PARALLEL)
+    assert ch.groups() == [0, 0, 1]                 # two forwarders write the same fields: apart
+    for bad in ([0, 0, 0], [1, 1, 1], [0, 2, 2], [0, 1, 0]):
+        with pytest.raises(nfc.NfcError) as e:
+            ch.set_groups(bad)
+        assert e.value.code == nfc.NFC_EINVAL
+    with pytest.raises(nfc.NfcError) as e:
+        nfc.Chain(["IPSEC", "ACL", "IPSEC"], device=0)
+    assert e.value.code == nfc.NFC_EUNSUP

@@ -173,3 +173,33 @@ def test_planner_groups(nfc):
         assert g == want, ch
     with pytest.raises(Exception):
         nfc.plan_parallel([])
+    # repeated kinds (NEXT-2's identical NFs): the greedy rule still holds
+    for ch, want in ((["ACL"] * 4, [0, 0, 0, 0]), (["DPI"] * 4, [0, 0, 0, 0]),
+                     (["ACL", "DPI", "ACL", "LPM4", "LPM4"], [0, 0, 0, 0, 1]), (["LB", "ACL", "LB"], [0, 0, 0])):
+        assert nfc.plan_parallel(ch) == want, ch
+
+
+@pytest.mark.parametrize("kinds", [["ACL"] * 4, ["DPI"] * 4, ["ACL", "DPI", "ACL", "LPM4", "LPM4"], ["LB", "ACL", "LB"]])
+def test_repeated_kinds_reorg_equals_sequential(kinds):
+    """NEXT-2's identical NFs (Fig. 13 configurations a-d): a repeated kind shares
+    its tables; every grouping into runs of parallel-legal NFs gives the sequential result
+    (records, bytes, pairs, stats) -- including the paper's (b) one group and (c) two."""
+    w = nfcgen.workload("NX2_FW")
+    t = nfcgen.make_tables(9, ["ACL", "DPI", "LPM4", "LB"], n_acl=64, n_pat=100, n_r4=1000, acl_deny=0.1)
+    w.traffic.pkt_len, w.traffic.match_ppm, w.traffic.tcp_pct = 1, 200_000, 40
+    b = nfcgen.generate(w.traffic, t, 0, 800)
+    seq = oracle.OracleChain(kinds, t)
+    want, wa, (wp, wq), wn = seq.run(b)
+    tried = 0
+    for g in _partitions(len(kinds)):
+        legal = all(_legal(kinds[p], kinds[q]) for p in range(len(kinds)) for q in range(p + 1, len(kinds))
+                    if g[p] == g[q])
+        if not legal:
+            continue
+        tried += 1
+        o = oracle.OracleChain(kinds, t)
+        got, ga, (gp, gq), gn = o.run_reorg(b, g)
+        assert np.array_equal(got.view(np.uint8), want.view(np.uint8)), g
+        assert gn == wn and sorted(zip(gp, gq)) == sorted(zip(wp, wq)), g
+        assert np.array_equal(o.stats, seq.stats), g
+    assert tried >= 2
