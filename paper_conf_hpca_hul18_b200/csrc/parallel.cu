@@ -172,6 +172,7 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
                                 if (e.z) {
                                     const Walk wk{0, e.z, e.w};
                                     dpi_finish<DM_HOT>(P, C, k, wk);       // emits the pairs, sets nmatch
+                                    k.npairs += k.nmatch;
                                 }
                             } else if (kd == NFC_LB) {
                                 k.lb_b = e.y >> 16;

@@ -1388,6 +1388,7 @@ struct Pkt {
     uint32_t h[16];
     PV v;
     uint32_t drop, esp_sa, port, acl_rule, lb_b, nmatch, esp_seq, passmask, esp_bytes, out_len;
+    uint32_t npairs;          // pairs of every DPI applied (a chain may repeat DPI; SIG_ANY)
     uint32_t t24;             // TBL24 entry, loaded right after parse (NFC_EARLY_T24)
     uint32_t mmeta, mslot;    // deferred match-pair emission: closure meta, first pair slot
     uint32_t mbase;           // deferred warp-aggregated claim: base slot (lane 0)
@@ -1551,6 +1552,7 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
+    k.npairs = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
     if (!valid) return;
@@ -1564,6 +1566,7 @@ __device__ __forceinline__ void pkt_begin_h(const Loc &l, bool valid, Pkt &k, co
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
+    k.npairs = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
     if (!valid) return;
@@ -1593,6 +1596,7 @@ template <int DM>
 __device__ __forceinline__ bool dpi_finish(const KParams &P, const Ctx &C, Pkt &k, const Walk w)
 {
     bool dropped = false;
+    k.nmatch = 0;                 // this DPI's count (a chain may repeat DPI: no earlier count carried)
     // DM_FULL: C.meta holds the accepting slots' summaries (index ~slot)
     const uint32_t st = DM == DM_FULL ? ~w.mx : C.dpi.wide ? (w.mx & 0x7FFFFFFFu) : (w.mx & 0x7FFFu);
     const uint32_t meta = w.cnt == 1 ? C.meta[st] : 0u;
@@ -1909,6 +1913,7 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
         dropped = (r >> 31) != 0;
     } else if constexpr (KIND == NFC_DPI) {
         dropped = dpi_finish<DM>(P, C, k, dpi_walk<DM>(P, C.dpi, k.h, k.f, k.v.pl_off, k.v.ip_end, C.pol_f));
+        k.npairs += k.nmatch;
     } else if constexpr (KIND == NFC_LPM4) {
         // DIR-24-8: at most two dependent table reads ("two memory accesses")
         if (k.v.fam != 4) { k.passmask |= 1u << pos; return; }
@@ -2077,7 +2082,7 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
     const uint32_t bin = __reduce_add_sync(FULL, valid ? k.orig_len : 0u);
     const uint32_t bout = __reduce_add_sync(FULL, fwd ? k.out_len : 0u);
     uint32_t pairs = 0, nesp = 0, eb = 0, eblk = 0;
-    if constexpr ((M & MASK_DPI) != 0) pairs = __reduce_add_sync(FULL, k.nmatch);
+    if constexpr ((M & MASK_DPI) != 0) pairs = __reduce_add_sync(FULL, S == SIG_ANY ? k.npairs : k.nmatch);
     if constexpr ((M & MASK_IPSEC) != 0) {
         const bool esp = k.esp_sa != 0xFF;
         nesp = __popc(__ballot_sync(FULL, esp));

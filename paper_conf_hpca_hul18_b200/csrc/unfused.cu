@@ -85,7 +85,12 @@ __global__ void __launch_bounds__(NT, DM == DM_FULL ? 1 : 2)
             k.nmatch = r.z & 0xFFFF;
             k.out_len = r.z >> 16;
         }
-        if (valid && k.alive) nf_apply<KIND, DM>(P, C, k, pos);
+        const bool ran = valid && k.alive;
+        if (ran) nf_apply<KIND, DM>(P, C, k, pos);
+        if constexpr (KIND == NFC_DPI) {                      // pairs of this DPI stage (a chain may repeat DPI)
+            const uint32_t pr = __reduce_add_sync(0xFFFFFFFFu, ran ? k.nmatch : 0u);
+            if (lane == 0 && pr) atomicAdd(&P.stats[ST_DPI_PAIRS], (unsigned long long)pr);
+        }
         if (valid) {
             reinterpret_cast<uint4 *>(P.rec)[g] = uf_pack(k);
             if (k.passmask) passmask[g] |= (uint8_t)k.passmask;
@@ -135,7 +140,6 @@ __global__ void __launch_bounds__(UF_NT) uf_stats_kernel(const KParams P, const 
             atomicAdd(&cnt[ST_PARSE_DROP], (unsigned long long)v[2]);
             atomicAdd(&cnt[ST_BYTES_IN], (unsigned long long)v[3]);
             atomicAdd(&cnt[ST_BYTES_OUT], (unsigned long long)v[4]);
-            atomicAdd(&cnt[ST_DPI_PAIRS], (unsigned long long)v[5]);
             for (int p = 0; p < NFC_MAX_CHAIN; p++) {
                 atomicAdd(&cnt[ST_POS_BASE + 4 * p + 1], (unsigned long long)nd[p]);
                 atomicAdd(&cnt[ST_POS_BASE + 4 * p + 2], (unsigned long long)np[p]);
