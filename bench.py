@@ -561,12 +561,86 @@ def run_stream(args):
         dist.destroy_process_group()
 
 
+def run_next2(args):
+    """--config NX2_FW / NX2_IDS (Figs. 13-14): four identical
+    NFs on 64-B TCP traffic, the paper's configurations on B200 -- (a) sequential: one kernel
+    per NF (NFC_F_UNFUSED), (b) one parallel group of four (NFC_F_PARALLEL), (c) two parallel
+    groups of two, (d) synthesized: the fused kernel -- throughput over the ring and the
+    latency of one 4,096-packet batch (median of 30 launches)."""
+    import torch
+
+    from paper_conf_hpca_hul18_b200 import nfc
+    local_dev = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
+    w = make_workload(args)
+    stream = torch.cuda.current_stream(dev)
+    arena, off, ln, n = prepare_ring(w, args.ring_mb, 0, 1, local_dev, stream)
+    rec = torch.empty((n, 16), dtype=torch.uint8, device=dev)
+    cap = 1 << 22
+    mp = torch.empty(cap, dtype=torch.int32, device=dev)
+    mq = torch.empty(cap, dtype=torch.int16, device=dev)
+    mc = torch.zeros(1, dtype=torch.int32, device=dev)
+    descs = nfc.Chain.batch_array(batch_descs(arena, off, ln, n, 0, args.batch_pkts))
+    one = nfc.Chain.batch_array([(arena.data_ptr(), off.data_ptr(), ln.data_ptr(), min(n, BATCH), 0)])
+    cfgs = {"a_sequential": (nfc.F_UNFUSED, None), "b_parallel_1group": (nfc.F_PARALLEL, [0, 0, 0, 0]),
+            "c_parallel_2groups": (nfc.F_PARALLEL, [0, 0, 1, 1]), "d_synthesized_fused": (0, None)}
+    out, main = {}, None
+    for name, (flags, groups) in cfgs.items():
+        ch = nfc.Chain(w.kinds, device=local_dev, flags=flags)
+        ch.load_tables(w.tables)
+        if groups:
+            ch.set_groups(groups)
+
+        def step(d=descs):
+            mc.zero_()
+            ch.process(d, rec.data_ptr(), mp.data_ptr(), mq.data_ptr(), cap, mc.data_ptr(), stream.cuda_stream)
+        for _ in range(max(3, args.warmup)):
+            step()
+        torch.cuda.synchronize(dev)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(local_dev) as clk:
+            e0.record(stream)
+            for _ in range(args.steps):
+                step()
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+        ms = e0.elapsed_time(e1)
+        lat = []
+        for it in range(40):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            step(one)
+            a1.record(stream)
+            torch.cuda.synchronize(dev)
+            if it >= 10:
+                lat.append(a0.elapsed_time(a1) * 1e3)
+        out[name] = {"mpps": round(n * args.steps / (ms / 1e3) / 1e6, 3), "ms_per_step": round(ms / args.steps, 4),
+                     "batch_latency_us": round(float(np.median(lat)), 2), "groups": ch.groups() if flags == nfc.F_PARALLEL else None}
+        if flags == 0:
+            main = (ms, clk.summary(), ch.launches())
+        ch.close()
+    ms, clocks, _ = main
+    print(json.dumps({
+        "metric": METRIC, "value": out["d_synthesized_fused"]["mpps"], "unit": "Mpps", "n_gpus": 1, "steps": args.steps,
+        "warmup": max(3, args.warmup), "ms_per_step": round(ms / args.steps, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"{w.name}: {w.note} (NEXT-2, configurations a-d of Fig. 13)", "chain": w.kinds,
+                   "packets_per_step_per_gpu": n, "batch_pkts": args.batch_pkts, "latency_batch_pkts": min(n, BATCH)},
+        "next2_configs": out,
+        "paper_context": "P:L330-353: parallelization cuts latency (GPU 24 ms -> 5 ms, a -> b); synthesis (d) "
+                         "raises throughput over (b) by 13-21 % on GPU",
+        "clocks": clocks}))
+
+
 def main():
     args = parse_args()
     if args.impl == "reference":
         return run_reference(args)
     if args.config in ("S1", "S1R"):
         return run_stream(args)
+    if args.config in ("NX2_FW", "NX2_IDS"):
+        return run_next2(args)
     import torch
     import torch.distributed as dist
 
