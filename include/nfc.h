@@ -343,12 +343,16 @@ NFC_API int nfc_dpi_stream_create(int device, const nfc_dpi_spec *spec, uint32_t
 /* Regular-expression variant ("for the regular expression we use a DFA";
  * DESIGN.md R#33): spec->blob[off[j] .. off[j+1]) is expression j (not NUL-
  * terminated) over bytes: literals, \xHH, \<punct>, '.', [..] classes with ranges
- * and '^', (..), '|', '?', {m} and {m,n} with n <= 64.  An occurrence of
- * expression j ends at byte x iff a non-empty substring of the flow stream ending
- * at x is in its language (unanchored search); it is reported like a pattern
- * occurrence.  Every language is finite, so the longest match bounds the re-walk.
- * NFC_EUNSUP for '*' / '+' / {m,}; NFC_EINVAL for a syntax error, an expression
- * that matches the empty string, or a DFA over max_states states (0 = 2^20). */
+ * and '^', (..), '|', '?', '*', '+', {m}, {m,n} with n <= 64 and {m,} with m <= 64.
+ * An occurrence of expression j ends at byte x iff a non-empty substring of the
+ * flow stream ending at x is in its language (unanchored search); it is reported
+ * like a pattern occurrence.  A set whose longest match is at most 1 024 bytes is
+ * walked per packet (a bounded re-walk of the flow's preceding bytes); a longer or
+ * unbounded one is walked flow-serially from the carried state.  NFC_EINVAL for a
+ * syntax error, an expression that matches the empty string, or a DFA over
+ * max_states states (0 = 2^20); NFC_EUNSUP for anchors ('^' / '$' outside a class)
+ * or repeats that expand the NFA beyond 2^16 states; NFC_ENOMEM if the host
+ * compiler runs out of memory. */
 NFC_API int nfc_dpi_stream_create_regex(int device, const nfc_dpi_spec *spec, uint32_t max_flows,
                                         uint32_t max_states, nfc_dpi_stream **out);
 NFC_API int nfc_dpi_stream_destroy(nfc_dpi_stream *s);

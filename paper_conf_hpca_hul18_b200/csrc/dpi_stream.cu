@@ -343,6 +343,32 @@ __global__ void k_plen(uint32_t n, uint32_t none, const uint32_t *fkey, const ui
     plen[u] = l;
 }
 
+// Flow-serial walk (regex sets with unbounded or > 1 024-byte matches: no bounded
+// re-walk reconstructs a packet's start state): one thread per flow segment of the
+// sorted batch walks the flow's packets in stream order from the carried state.
+template <int M>
+__global__ void __launch_bounds__(256) k_walk_serial(nfc_batch b, StreamDfa d, uint32_t none, const uint32_t *fkey,
+                                                     const uint32_t *fidx, const uint32_t *span,
+                                                     const uint32_t *fstate, uint32_t *fin, nfc_stream_result r)
+{
+    __shared__ uint8_t cls[256];
+    for (int k = threadIdx.x; k < 256; k += blockDim.x) cls[k] = d.cls[k];
+    __syncthreads();
+    for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < b.n; u += gridDim.x * blockDim.x) {
+        const uint32_t f = fkey[u];
+        if (f == none || (u > 0 && fkey[u - 1] == f)) continue;   // segment heads only
+        uint32_t s = fstate[f], w = u;
+        for (; w < b.n && fkey[w] == f; w++) {
+            const uint32_t i = fidx[w], sp = span[i];
+            Emit em{r, (uint32_t)b.first_global_index + i, sp & 0xFFFF, 0, 0};
+            s = walk<M, true>(d, cls, b.arena + b.off[i], sp & 0xFFFF, sp >> 16, s, em);
+            r.nocc[i] = em.cnt;
+            r.drop[i] = (uint8_t)em.dr;
+        }
+        fin[w - 1] = s;
+    }
+}
+
 __global__ void k_commit(uint32_t n, uint32_t none, const uint32_t *fkey, const uint32_t *fin, uint32_t *fstate)
 {
     const uint32_t u = blockIdx.x * blockDim.x + threadIdx.x;
@@ -543,7 +569,10 @@ int nfc_dpi_stream_process(nfc_dpi_stream *s, const nfc_batch *b, const nfc_stre
     const uint32_t wb = (b->n + 255) / 256, need = s->maxlen - 1;
     // s->fkey (unsorted keys) is dead after the sort: it holds the flows' final states
     const size_t tbytes = (size_t)s->ncls * s->n_states * 2;
-    if (s->wide) {
+    if (s->maxlen == 0xFFFFFFFFu) {          // unbounded / very long matches: flow-serial
+        if (s->wide) k_walk_serial<1><<<wb, 256, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+        else k_walk_serial<0><<<wb, 256, 0, st>>>(*b, d, none, s->fkey2, s->fidx2, s->span, s->fstate, s->fkey, *r);
+    } else if (s->wide) {
         k_walk<1><<<wb, 256, 0, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span, s->cumx, s->fstate, s->fkey, *r);
     } else if (s->smem_ok && tbytes <= DFA_SMEM_MAX) {
         k_walk<2><<<s->n_sm, WALK_SMEM_THREADS, (tbytes + 15) / 16 * 16, st>>>(*b, d, none, need, s->fkey2, s->fidx2, s->span,

@@ -2,12 +2,13 @@
 // NEXT-4; PAPER.md P:L132 [SIII.A.2] "For the regular expression we use a
 // Deterministic Finite Automata (DFA) implementation"; R#33).
 //
-// Subset (every language finite, so an occurrence has a bounded length and the
-// stream walk's maxlen - 1 warm-up stays exact): literal bytes, escapes \xHH and
-// \<punct>, '.', classes [..] with ranges and '^' negation, groups (..),
-// alternation '|', quantifiers '?' and {m} / {m,n} (n <= 64).  '*' and '+' are
-// rejected (unbounded).  Search is unanchored: an occurrence of regex j ends at
-// byte x iff some substring ending at x is in L(j).
+// Syntax: literal bytes, escapes \xHH and \<punct>, '.', classes [..] with ranges
+// and '^' negation, groups (..), alternation '|', quantifiers '?', '*', '+', {m},
+// {m,n} (n <= 64) and {m,} (m <= 64).  Search is unanchored: an occurrence of regex j
+// ends at byte x iff some non-empty substring ending at x is in L(j).  A set whose
+// longest match is at most 1 024 bytes is walked per packet with a maxlen - 1
+// re-walk of the flow's preceding bytes; a longer or unbounded one (maxlen =
+// 0xFFFFFFFF) flow-serially from the carried state (dpi_stream.cu k_walk_serial).
 //
 // Thompson NFA per regex, one shared start state; subset construction over the
 // 256 byte values with the start state added to every subset (unanchored); the
@@ -27,10 +28,14 @@
 namespace nfc {
 namespace {
 
-// Bounds: the longest word of an expression, and the NFA size while
-// bounded repeats are expanded (nested {m,n} multiply).  Beyond them: NFC_EUNSUP.
-constexpr long long REGEX_MAXLEN = 1024;
-constexpr size_t REGEX_NFA_MAX = 1u << 20;
+// The NFA size while repeats are expanded (nested {m,n} multiply) is bounded (beyond:
+// NFC_EUNSUP).  Longest-match lengths saturate at REGEX_INF ('*', '+', {m,}); a set whose
+// longest match exceeds REGEX_PAR_MAXLEN is walked flow-serially (DpiHost::maxlen =
+// 0xFFFFFFFF), the bounded re-walk of the per-packet walk being too long or unbounded.
+constexpr long long REGEX_INF = 1LL << 40;
+constexpr long long REGEX_PAR_MAXLEN = 1024;
+constexpr size_t REGEX_NFA_MAX = 1u << 16;   // NFA states (subset construction cost grows with it)
+inline long long sat(long long x) { return x > REGEX_INF ? REGEX_INF : x; }
 
 struct Nfa {
     struct St { std::array<uint64_t, 4> set{}; int out = -1; std::vector<int> eps; int accept = -1; };
@@ -78,7 +83,7 @@ struct Parser {
             p++;
             return true;
         }
-        if (c == '*' || c == '+') { err = "regex: unbounded quantifier ('*', '+') not supported"; return false; }
+        if (c == '*' || c == '+') { err = "regex: misplaced quantifier"; return false; }
         if (c == '^' || c == '$') { err = "regex: anchors ('^', '$' outside a class) not supported"; return false; }
         if (c == ')' || c == '?' || c == '{' || c == '|') { err = "regex: misplaced metacharacter"; return false; }
         if (c == '.') { for (int b = 0; b < 256; b++) put(b); }
@@ -129,39 +134,63 @@ struct Parser {
         int lo = (int)n.st.size();
         if (!atom(f, len)) return false;
         int hi = (int)n.st.size();
-        while (p < e && (*p == '?' || *p == '{')) {
+        while (p < e && (*p == '?' || *p == '{' || *p == '*' || *p == '+')) {
             int m = 0, M = 0;
+            bool unb = false;                        // '*', '+', {m,}: no upper bound
             if (*p == '?') { p++; m = 0; M = 1; }
+            else if (*p == '*') { p++; m = 0; unb = true; }
+            else if (*p == '+') { p++; m = 1; unb = true; }
             else {
                 p++;
                 if (!number(m)) { err = "regex: bad {m,n}"; return false; }
                 M = m;
-                if (p < e && *p == ',') { p++; if (!number(M)) { err = "regex: {m,} is unbounded"; return false; } }
-                if (p >= e || *p != '}' || M < m || M > 64 || M == 0) { err = "regex: bad {m,n} (need 0 <= m <= n <= 64, n > 0)"; return false; }
+                if (p < e && *p == ',') {
+                    p++;
+                    if (p < e && *p == '}') unb = true;
+                    else if (!number(M)) { err = "regex: bad {m,n}"; return false; }
+                }
+                if (p >= e || *p != '}' || m > 64 || (!unb && (M < m || M > 64 || M == 0))) {
+                    err = "regex: bad {m,n} (need 0 <= m <= n <= 64, n > 0; {m,} with m <= 64)";
+                    return false;
+                }
                 p++;
             }
-            if (len * M > REGEX_MAXLEN) { err = "regex: longest match above 1024 bytes not supported"; return false; }
-            if (n.st.size() + (size_t)(hi - lo) * (size_t)M + 2 * (size_t)M + 2 > REGEX_NFA_MAX) {
-                err = "regex: NFA above 2^20 states not supported";
+            const int copies = unb ? m + 1 : M;      // unbounded: m mandatory copies + one looped
+            if (n.st.size() + (size_t)(hi - lo) * (size_t)copies + 2 * (size_t)copies + 4 > REGEX_NFA_MAX) {
+                err = "regex: NFA above 2^16 states not supported";
                 return false;
             }
-            // expand: m mandatory copies, M - m optional copies (all copies are
-            // cloned from the untouched fragment before any of them is wired)
+            // expand: every copy is cloned from the untouched fragment before any is wired
             std::vector<Frag> cp{f};
-            for (int k = 1; k < M; k++) cp.push_back(clone(lo, hi, f));
+            for (int k = 1; k < copies; k++) cp.push_back(clone(lo, hi, f));
             const long long olen = len;
             int s0 = n.add(), cur = s0;
-            std::vector<int> skips;
-            for (int k = 0; k < M; k++) {
-                n.st[cur].eps.push_back(cp[k].in);
-                if (k >= m) skips.push_back(cur);
-                int nx = n.add();
-                n.st[cp[k].out].eps.push_back(nx);
-                cur = nx;
+            if (unb) {
+                for (int k = 0; k < m; k++) {            // the mandatory copies
+                    n.st[cur].eps.push_back(cp[k].in);
+                    int nx = n.add();
+                    n.st[cp[k].out].eps.push_back(nx);
+                    cur = nx;
+                }
+                const int ex = n.add();                  // the loop: zero or more further copies
+                n.st[cur].eps.push_back(cp[m].in);
+                n.st[cur].eps.push_back(ex);
+                n.st[cp[m].out].eps.push_back(cur);
+                f = {s0, ex};
+                len = REGEX_INF;
+            } else {
+                std::vector<int> skips;
+                for (int k = 0; k < M; k++) {
+                    n.st[cur].eps.push_back(cp[k].in);
+                    if (k >= m) skips.push_back(cur);
+                    int nx = n.add();
+                    n.st[cp[k].out].eps.push_back(nx);
+                    cur = nx;
+                }
+                for (int x : skips) n.st[x].eps.push_back(cur);
+                f = {s0, cur};
+                len = sat(olen * M);
             }
-            for (int x : skips) n.st[x].eps.push_back(cur);
-            f = {s0, cur};
-            len = olen * M;
             hi = (int)n.st.size();
         }
         return true;
@@ -176,8 +205,7 @@ struct Parser {
             if (!piece(g, l)) return false;
             n.st[f.out].eps.push_back(g.in);
             f.out = g.out;
-            len += l;
-            if (len > REGEX_MAXLEN) { err = "regex: longest match above 1024 bytes not supported"; return false; }
+            len = sat(len + l);
         }
         return true;
     }
@@ -241,7 +269,7 @@ static std::string build_regex_dfa_impl(const nfc_dpi_spec &s, DpiHost &o, uint3
         n.st[acc].accept = (int)j;
         n.st[f.out].eps.push_back(acc);
         n.st[start].eps.push_back(f.in);
-        o.maxlen = std::max(o.maxlen, (uint32_t)len);
+        o.maxlen = len > REGEX_PAR_MAXLEN ? 0xFFFFFFFFu : std::max(o.maxlen, (uint32_t)len);
     }
     const int ns = (int)n.st.size();
     auto closure = [&](std::vector<int> &v) {

@@ -120,18 +120,20 @@ def test_stream_dpi_fails_loudly_without_gpu(nfc):
         nfc.DpiStream(blob, np.array([0, 3], dtype=np.uint32), np.zeros(1, dtype=np.uint8), max_flows=8)
 
 
-@pytest.mark.parametrize("rx,code", [(b"ab*", "NFC_EUNSUP"), (b"a+", "NFC_EUNSUP"), (b"a{2,}", "NFC_EUNSUP"),
+@pytest.mark.parametrize("rx,code", [(b"ab*", "NFC_EOK_CLASS"), (b"a+", "NFC_EOK_CLASS"), (b"a{2,}", "NFC_EOK_CLASS"),
+                                     (b"a*", "NFC_EINVAL"), (b"(ab)*", "NFC_EINVAL"), (b"*a", "NFC_EINVAL"),
                                      (b"a?", "NFC_EINVAL"), (b"(a", "NFC_EINVAL"), (b"[ab", "NFC_EINVAL"),
                                      (b"a)", "NFC_EINVAL"), (b"\\q", "NFC_EINVAL"), (b"a{0}", "NFC_EINVAL"),
                                      # anchors are not silently taken as literal bytes
                                      (b"^GET", "NFC_EUNSUP"), (b"a$", "NFC_EUNSUP"), (b"(x|^y)", "NFC_EUNSUP"),
                                      # longest match above 1024 B / nested repeats: rejected up front, fast
-                                     (b"((a{64}){64}){64}", "NFC_EUNSUP"), (b"(a{64}){17}", "NFC_EUNSUP"),
+                                     (b"((a{64}){64}){64}", "NFC_EUNSUP"), (b"(a{64}){17}", "NFC_EOK_CLASS"),
                                      (b"(((((a{64}){64}){64}){64}){64}){64}", "NFC_EUNSUP"),
                                      (b"[^$]x", "NFC_EOK_CLASS")])
 def test_regex_rejected_before_cuda(nfc, rx, code):
-    """Unbounded quantifiers are NFC_EUNSUP, syntax errors and empty-matching expressions
-    NFC_EINVAL -- decided by the host compiler before any CUDA call (R#33)."""
+    """Syntax errors and empty-matching expressions are NFC_EINVAL, anchors and NFA
+    blow-ups NFC_EUNSUP -- decided by the host compiler before any CUDA call, fast
+    (R#33, R#35)."""
     blob = np.frombuffer(rx, dtype=np.uint8).copy()
     off = np.array([0, len(rx)], dtype=np.uint32)
     act = np.zeros(1, dtype=np.uint8)
@@ -139,7 +141,8 @@ def test_regex_rejected_before_cuda(nfc, rx, code):
     h = ctypes.c_void_p()
     rc = nfc.lib.nfc_dpi_stream_create_regex(0, ctypes.byref(spec), 16, 0, ctypes.byref(h))
     if code == "NFC_EOK_CLASS":
-        # '^' / '$' inside a class are bytes: the compile succeeds and only the CUDA setup can fail
+        # valid: the compile succeeds ('^' / '$' inside a class are bytes; unbounded and long
+        # matches walk flow-serially) and only the CUDA setup can fail
         assert rc in (nfc.NFC_OK, nfc.NFC_ECUDA)
         if rc == nfc.NFC_OK:
             nfc.lib.nfc_dpi_stream_destroy(h)

@@ -274,3 +274,31 @@ def test_stream_rss_sharded_equals_single(nfc):
     assert len(want_all) > 100
     for N in (2, 4):
         assert sorted(got_all[N]) == sorted(want_all), N
+
+
+UNB_REGEXES = [b"ab+c", b"x[0-9]*y", b"(GET|POST) /[a-z]+\\?", b"k{3,}!", b"<[a-z]+>", b"(ab|cd)*ef", b"Q.{2,}Z"]
+UNB_EXAMPLES = [b"abbbbbbc", b"x0123456789y", b"GET /index?", b"kkkkk!", b"<script>", b"abcdabef", b"Qhello worldZ"]
+
+
+@pytest.mark.parametrize("calls", [[250, 1, 250]])
+def test_regex_unbounded_stream_parity(nfc, calls):
+    """NEXT-4: regexes with '*', '+' and {m,} (unbounded matches, walked flow-serially
+    from the carried state: no bounded re-walk reconstructs the start) vs Python re,
+    with occurrences spanning packets and calls."""
+    from oracle.stream_dpi import StreamRegexDPI
+    blob = np.frombuffer(b"".join(UNB_REGEXES), dtype=np.uint8).copy()
+    off = np.cumsum([0] + [len(r) for r in UNB_REGEXES]).astype(np.uint32)
+    act = np.array([0, 1, 0, 0, 1, 0, 0], dtype=np.uint8)
+    ds = nfc.DpiStream(blob, off, act, max_flows=128, regex=True)
+    orc = StreamRegexDPI(UNB_REGEXES, list(act))
+    first, total = 0, 0
+    for c, n in enumerate(calls):
+        sb = stream_batch(300 + c, n, 25, UNB_EXAMPLES, len_choices=[64, 96], plant_frac=0.4,
+                          first_index=first, flow_seed=78)
+        want, wn, wd = orc.process(sb.frames(), first)
+        got, gn, gd, k = _gpu(ds, sb)
+        assert k == len(want) and got == want
+        assert gn == wn and gd == wd
+        first += n
+        total += len(want)
+    assert total > 30
