@@ -97,7 +97,8 @@ struct nfc_chain {
     uint64_t launches = 0;
     cudaStream_t last_stream = nullptr;
     void *comm = nullptr;                 // attached ncclComm_t (NFC_STATS_ALLREDUCE)
-    cudaStream_t xs[2] = {nullptr, nullptr};   // nfc_process_host copy/compute streams
+    static constexpr int NXS = 4;
+    cudaStream_t xs[NXS] = {nullptr, nullptr, nullptr, nullptr};   // nfc_process_host copy/compute streams
     // a3 regrouping: mixed IPv4/IPv6 chunks of the last launch, read back asynchronously; the
     // regrouping kernel variant runs while more than 1/8 of the chunks were mixed
     DBuf mix_dev;
@@ -105,7 +106,7 @@ struct nfc_chain {
     cudaEvent_t mix_ev = nullptr;
     uint32_t mix_chunks = 0;
     bool mix_pending = false, rg_on = false;
-    cudaEvent_t xe[2] = {nullptr, nullptr}, xk = nullptr;
+    cudaEvent_t xk = nullptr;
     DBuf stats_red;                       // all-reduce destination
 };
 
@@ -187,10 +188,8 @@ void nfc_destroy_chain(nfc_chain *c)
                    &c->tile_flag, &c->tile_vec, &c->batches, &c->h_arena, &c->h_off, &c->h_len, &c->h_rec,
                    &c->h_mp, &c->h_mq, &c->h_mc, &c->stats_red, &c->crec};
     for (DBuf *b : all) b->release();
-    for (int i = 0; i < 2; i++) {
+    for (int i = 0; i < nfc_chain::NXS; i++)
         if (c->xs[i]) cudaStreamDestroy(c->xs[i]);
-        if (c->xe[i]) cudaEventDestroy(c->xe[i]);
-    }
     if (c->xk) cudaEventDestroy(c->xk);
     if (c->mix_ev) cudaEventDestroy(c->mix_ev);
     if (c->mix_host) cudaFreeHost(c->mix_host);
@@ -604,22 +603,19 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
     CK(c->h_mq.reserve((size_t)match_cap * 2 + 4));
     CK(c->h_mc.reserve(4));
     if (!c->xs[0]) {
-        for (int i = 0; i < 2; i++) {
-            CK(cudaStreamCreateWithFlags(&c->xs[i], cudaStreamNonBlocking));
-            CK(cudaEventCreateWithFlags(&c->xe[i], cudaEventDisableTiming));
-        }
+        for (int i = 0; i < nfc_chain::NXS; i++) CK(cudaStreamCreateWithFlags(&c->xs[i], cudaStreamNonBlocking));
         CK(cudaEventCreateWithFlags(&c->xk, cudaEventDisableTiming));
     }
     // the copy streams start after the caller's prior work
     CK(cudaEventRecord(c->xk, user));
-    for (int i = 0; i < 2; i++) CK(cudaStreamWaitEvent(c->xs[i], c->xk, 0));
+    for (int i = 0; i < nfc_chain::NXS; i++) CK(cudaStreamWaitEvent(c->xs[i], c->xk, 0));
     CK(cudaMemsetAsync(c->h_mc.p, 0, 4, c->xs[0]));
     CK(cudaEventRecord(c->xk, c->xs[0]));          // "previous kernel done" starts as: counter zeroed
-    // chunks: about 16 per call, at least 64 K packets each.  A chunk's byte range is
+    // chunks: about 32 per call, at least 64 K packets each, round-robin over NXS streams.  A chunk's byte range is
     // scanned while the previous chunks' copies and kernels run; a chunk whose range
     // overlaps an earlier chunk's (frames not laid out in index order) first waits for
     // everything issued before it, so it reads the rewritten bytes back consistently.
-    const uint32_t per = std::max<uint32_t>(65536, (n + 15) / 16);
+    const uint32_t per = std::max<uint32_t>(65536, (n + 31) / 32);
     uint8_t *darena = c->h_arena.as<uint8_t>();
     uint64_t *doff = c->h_off.as<uint64_t>();
     uint16_t *dlen = c->h_len.as<uint16_t>();
@@ -627,7 +623,7 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
     uint32_t k = 0;
     for (uint32_t a0 = 0; a0 < n; a0 += per, k++) {
         const uint32_t cnt = std::min(per, n - a0);
-        cudaStream_t st = c->xs[k & 1];
+        cudaStream_t st = c->xs[k % nfc_chain::NXS];
         uint64_t lo = ~0ull, hi = 0;
         const uint64_t *o = off + a0;
         const uint16_t *l = len + a0;
@@ -640,7 +636,7 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
         hi = std::min<uint64_t>(hi + tr, arena_bytes);
         if (lo > arena_bytes || hi < lo) return fail(NFC_EINVAL, "frame outside the arena");
         if (lo < max_hi)
-            for (int i = 0; i < 2; i++) CK(cudaStreamSynchronize(c->xs[i]));
+            for (int i = 0; i < nfc_chain::NXS; i++) CK(cudaStreamSynchronize(c->xs[i]));
         max_hi = std::max(max_hi, hi);
         CK(cudaMemcpyAsync(darena + lo, arena + lo, hi - lo, cudaMemcpyHostToDevice, st));
         CK(cudaMemcpyAsync(doff + a0, off + a0, (size_t)cnt * 8, cudaMemcpyHostToDevice, st));
@@ -659,7 +655,7 @@ int nfc_process_host(nfc_chain *c, uint8_t *arena, uint64_t arena_bytes, const u
     uint32_t cnt = 0;
     CK(cudaStreamWaitEvent(c->xs[0], c->xk, 0));
     CK(cudaMemcpyAsync(&cnt, c->h_mc.p, 4, cudaMemcpyDeviceToHost, c->xs[0]));
-    for (int i = 0; i < 2; i++) CK(cudaStreamSynchronize(c->xs[i]));
+    for (int i = 0; i < nfc_chain::NXS; i++) CK(cudaStreamSynchronize(c->xs[i]));
     uint32_t m = cnt < match_cap ? cnt : match_cap;
     if (m && match_pkt && match_pat) {
         CK(cudaMemcpyAsync(match_pkt, c->h_mp.p, (size_t)m * 4, cudaMemcpyDeviceToHost, c->xs[0]));
@@ -710,7 +706,7 @@ int nfc_set_groups(nfc_chain *c, const uint8_t *group)
     if (!c || !group) return fail(NFC_EINVAL, "NULL argument");
     if (!groups_legal(c->kind, c->n_nf, group))
         return fail(NFC_EINVAL, "groups must be runs of consecutive, pairwise parallel-legal NFs (nfc_plan_parallel)");
-    for (uint32_t i = 0; i < c->n_nf; i++) c->group[i] = group[i];
+    for (uint32_t i = 0; i < c->n_nf && i < NFC_MAX_CHAIN; i++) c->group[i] = group[i];
     return NFC_OK;
 }
 

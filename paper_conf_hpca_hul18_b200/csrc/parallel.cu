@@ -214,7 +214,6 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
         if (lane + 32 < NWS) wst[lane + 32] = t[1];
         __syncwarp();
         if (lane == 0) {
-            wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
             unsigned long long in = wst[ST_PKTS] - wst[ST_PARSE_DROP];
             for (uint32_t p = 0; p < P.n_nf; p++) {
                 const unsigned long long d = wst[ST_POS_BASE + 4 * p + 1], ps = wst[ST_POS_BASE + 4 * p + 2];
@@ -222,6 +221,8 @@ __global__ void __launch_bounds__(PAR_NT, 1) par_kernel(const KParams P, uint32_
                 wst[ST_POS_BASE + 4 * p + 3] = in - d - ps;
                 in -= d;
             }
+            if (NFC_FWD_DERIVED) wst[ST_FWD] = in;   // survivors of every position
+            wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
         }
         __syncwarp();
         for (uint32_t idx = lane; idx < NWS; idx += 32)

@@ -108,6 +108,12 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_RGQ
 #define NFC_RGQ 48            // per-warp queue words in shared memory (47 packet indices + the length)
 #endif
+#ifndef NFC_T24_L2_EARLY
+#define NFC_T24_L2_EARLY 0    // 1: the DIR-24-8 second-level read issued right after the speculative block
+#endif
+#ifndef NFC_FWD_DERIVED
+#define NFC_FWD_DERIVED 0     // 1: the forwarded count derived at the flush (pkts - parse drops - NF drops)
+#endif
 #ifndef NFC_WALK_AHEAD
 #define NFC_WALK_AHEAD 0      // 1: split-walk payload words loaded one 16-B step ahead
 #endif
@@ -2027,6 +2033,12 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
                 wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
                 if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
             }
+#if NFC_T24_L2_EARLY
+            // the DIR-24-8 second level right after the block (its first level has arrived):
+            // the read overlaps the DPI finish and the match-pair atomic instead of the LPM
+            if constexpr (T24)
+                if (k.t24 & 0x8000) k.t24 = ld_tab16(P.l4.tbllong + ((k.t24 & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
+#endif
             if (NFC_SPEC_V6 && k.alive && k.v.fam != 4) r = nf_acl_fused(P, k.v);   // IPv6 lanes
             if (k.alive) {                     // ACL effects (position 0)
                 const uint32_t rule = r & 0xFFFF;
@@ -2078,7 +2090,7 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
     const bool fwd = valid && k.drop == 0xFF;
     const uint32_t nv = __popc(__ballot_sync(FULL, valid));
     const uint32_t nparse = __popc(__ballot_sync(FULL, valid && k.drop == 0xFE));
-    const uint32_t nfwd = __popc(__ballot_sync(FULL, fwd));
+    const uint32_t nfwd = NFC_FWD_DERIVED ? 0u : __popc(__ballot_sync(FULL, fwd));
     const uint32_t bin = __reduce_add_sync(FULL, valid ? k.orig_len : 0u);
     const uint32_t bout = __reduce_add_sync(FULL, fwd ? k.out_len : 0u);
     uint32_t pairs = 0, nesp = 0, eb = 0, eblk = 0;
@@ -2091,7 +2103,7 @@ __device__ __forceinline__ void pkt_end(const KParams &P, const Ctx &C, Pkt &k, 
     }
     if (lane == 0) {
         ws[ST_PKTS] += nv;
-        ws[ST_FWD] += nfwd;
+        if (!NFC_FWD_DERIVED) ws[ST_FWD] += nfwd;
         ws[ST_PARSE_DROP] += nparse;
         ws[ST_BYTES_IN] += bin;
         ws[ST_BYTES_OUT] += bout;
@@ -2543,7 +2555,6 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
         if (i + 32 < WS) wst[i + 32] = t[1];
         __syncwarp();
         if (lane == 0) {
-            wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
             unsigned long long in = wst[ST_PKTS] - wst[ST_PARSE_DROP];
             for (uint32_t p = 0; p < P.n_nf; p++) {
                 const unsigned long long d = wst[ST_POS_BASE + 4 * p + 1], ps = wst[ST_POS_BASE + 4 * p + 2];
@@ -2551,6 +2562,8 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
                 wst[ST_POS_BASE + 4 * p + 3] = in - d - ps;
                 in -= d;
             }
+            if (NFC_FWD_DERIVED) wst[ST_FWD] = in;   // survivors of every position
+            wst[ST_DROP] = wst[ST_PKTS] - wst[ST_FWD];
         }
         __syncwarp();
         for (uint32_t idx = lane; idx < WS; idx += 32)
