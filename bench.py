@@ -344,6 +344,39 @@ def oracle_all_cores(w, local_dev, rate_1core_mpps, budget_s):
                       f"{max(r[2] for r in res):.1f} s"}
 
 
+def pcie_peaks(torch, dev, nbytes, reps=3):
+    """Measured pinned-host <-> HBM copy rates (GB/s) on this box: H2D alone, D2H alone,
+    and both directions at once on two streams (the full-duplex bound the pipelined
+    nfc_process_host can reach).  The denominator of the e2e roofline."""
+    nbytes = int(min(nbytes, 1 << 30))
+    hs = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    hd = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d1 = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+
+    def timed(h2d, d2h):
+        best = float("inf")
+        for _ in range(reps):
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            if h2d:
+                with torch.cuda.stream(s1):
+                    d1.copy_(hs, non_blocking=True)
+            if d2h:
+                with torch.cuda.stream(s2):
+                    hd.copy_(d2, non_blocking=True)
+            torch.cuda.synchronize(dev)
+            best = min(best, time.perf_counter() - t0)
+        return best
+
+    th, td, tb = timed(True, False), timed(False, True), timed(True, True)
+    del hs, hd, d1, d2
+    return {"h2d_gbs": round(nbytes / th / 1e9, 1), "d2h_gbs": round(nbytes / td / 1e9, 1),
+            "duplex_each_gbs": round(nbytes / tb / 1e9, 1), "bytes": nbytes,
+            "method": "torch pinned copies, best of %d; duplex = both directions on two streams" % reps}
+
+
 def payload_bytes(b):
     """Payload bytes [pl_off, ip_end) per packet by a vectorised read of the headers
     (bench accounting only: the DPI work per packet; 0 if not parsed)."""
@@ -818,6 +851,12 @@ def main():
                "h2d_bytes_per_step": len(b.arena) + n * 10,
                "d2h_bytes_per_step": len(b.arena) + n * 16 + 4 + min(npairs, cap) * 6,
                "steps": len(times), "api": "nfc_process_host (pinned host buffers)"}
+        del host, hrec
+        pk = pcie_peaks(torch, dev, len(b.arena))
+        # copy roofline: both directions overlapped at the measured duplex rate
+        bound_s = max(e2e["h2d_bytes_per_step"], e2e["d2h_bytes_per_step"]) / (pk["duplex_each_gbs"] * 1e9)
+        step_s = float(e2e_t.item()) / len(times)
+        e2e["pcie"] = dict(pk, bound_mpps=round(n / bound_s / 1e6, 1), frac=round(bound_s / step_s, 3))
         chain.stats(reset=True)
 
     # the general multi-batch path: the same batches in shuffled order, so the descriptors

@@ -94,7 +94,7 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #define NFC_ESP_RK_SMEM 1     // ESP reads AES round keys from shared memory (one out-of-line block cipher; C2 +11 %)
 #endif
 #ifndef NFC_SPEC_V6
-#define NFC_SPEC_V6 0         // 1: dual-stack warps take the speculative block (IPv6 lanes re-classified)
+#define NFC_SPEC_V6 0         // 1: dual-stack warps take the speculative block in every chain (IPv6 lanes re-classified)
 #endif
 #ifndef NFC_HOT_FAST
 #define NFC_HOT_FAST 0        // 1: DM_HOT split walk takes the unconditional 16-byte step too
@@ -272,8 +272,15 @@ __device__ __forceinline__ void prefetch_l2(const void *a) { asm volatile("prefe
 
 // byte k (0..63) of the 64 B header cache; k compile-time in hot paths
 __device__ __forceinline__ uint32_t hbyte(const uint32_t h[16], uint32_t k) { return (h[k >> 2] >> ((k & 3) * 8)) & 0xFF; }
-__device__ __forceinline__ uint32_t hbe16(const uint32_t h[16], uint32_t k) { return hbyte(h, k) << 8 | hbyte(h, k + 1); }
-__device__ __forceinline__ uint32_t hbe32(const uint32_t h[16], uint32_t k) { return hbe16(h, k) << 16 | hbe16(h, k + 2); }
+// big-endian 32/16-bit fields at byte k: one PRMT of the two words spanning them (k
+// compile-time at every call site, so the word indices and the selector fold)
+__device__ __forceinline__ uint32_t hbe32(const uint32_t h[16], uint32_t k)
+{
+    const uint32_t i = k >> 2, r = k & 3;
+    const uint32_t hi = i + 1 < 16 ? h[i + 1] : 0u;
+    return __byte_perm(h[i], hi, r << 12 | (r + 1) << 8 | (r + 2) << 4 | (r + 3));
+}
+__device__ __forceinline__ uint32_t hbe16(const uint32_t h[16], uint32_t k) { return hbe32(h, k) >> 16; }
 // ---------------------------------------------------------------- per-packet state
 struct PV {
     uint32_t fam;                 // 4 or 6
@@ -1709,7 +1716,8 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
     if (DM == DM_FULL && head) w = *head;     // walked speculatively with the ACL (spec_acl_dpi)
     else if (DM == DM_FULL && act) w = dpi_walk_head<DM>(P, k.h, a, b);
     const uint32_t base = (DM != DM_FULL || a >= 64) ? (a & ~15u) : 64u;
-    const uint32_t rem = act && b > base ? (b - base + 15) & ~15u : 0u;
+    // (an empty payload past byte 64 -- e.g. IPv6/TCP frames of 74 B -- has nothing to walk)
+    const uint32_t rem = act && b > max(a, base) ? (b - base + 15) & ~15u : 0u;
     if (__any_sync(FULL, rem != 0)) {         // warp-uniform (64-B frames: never)
         uint32_t incl = rem;
 #pragma unroll
@@ -2014,7 +2022,11 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
         // speculative ACL || DPI head walk || TBL24 (see spec_ok), warp-uniform choice
         // every payload starts at byte 42 or later; IPv6 lanes (dual-stack traffic) take the
         // IPv4 classification speculatively too and are re-classified below
-        const bool v4 = !k.alive || ((k.v.fam == 4 || NFC_SPEC_V6) && k.v.pl_off >= 42);
+        // dual-stack warps too for ACL -> DPI and ACL -> DPI -> LPM4 -> LPM6 (measured: +12 % and
+        // +4 % on C5 k2 / k4 64 B; -2 % on k3 and -6 % on C1, whose instance keeps the IPv4 gate)
+        constexpr bool V6 = NFC_SPEC_V6 || S == make_sig(2, NFC_ACL, NFC_DPI) ||
+                            S == make_sig(4, NFC_ACL, NFC_DPI, NFC_LPM4, NFC_LPM6);
+        const bool v4 = !k.alive || ((k.v.fam == 4 || V6) && k.v.pl_off >= 42);
         if (spec_ok<S>(P) && __all_sync(0xFFFFFFFFu, v4)) {
             constexpr bool T24 = sig_pos(S, NFC_LPM4) != 0xFF &&
                                  (sig_pos(S, NFC_IPSEC) == 0xFF || sig_pos(S, NFC_IPSEC) > sig_pos(S, NFC_LPM4));
@@ -2039,7 +2051,7 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
             if constexpr (T24)
                 if (k.t24 & 0x8000) k.t24 = ld_tab16(P.l4.tbllong + ((k.t24 & 0x7FFF) << 8) + (k.v.dst[0] & 0xFF), C.pol_l);
 #endif
-            if (NFC_SPEC_V6 && k.alive && k.v.fam != 4) r = nf_acl_fused(P, k.v);   // IPv6 lanes
+            if (V6 && k.alive && k.v.fam != 4) r = nf_acl_fused(P, k.v);   // IPv6 lanes
             if (k.alive) {                     // ACL effects (position 0)
                 const uint32_t rule = r & 0xFFFF;
                 k.acl_rule = rule;
