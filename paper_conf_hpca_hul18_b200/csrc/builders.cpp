@@ -199,6 +199,44 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
     return "";
 }
 
+// Search image of an IPv4 bit-vector blob (AclImg::f4 layout, nfc_internal.h): the
+// same intervals, bitsets, buckets and rule words, with bucket entries as key addresses
+// and pad entries instead of clamps.  Only for W == 1 (<= 64 rules) and window depth
+// <= 3: the kernel always takes three halvings (8-key window).  key_off / bv_off
+// receive the per-field array offsets.
+void build_acl4_fast(const std::vector<uint32_t> &b, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4])
+{
+    f.clear();
+    if (b.size() < ACLBV_HDR || b[0] == 0 || b[0] > 64 || b[1] != 1 || b[6] != 1 || b[23] > 3) return;
+    const uint32_t m[4] = {b[2], b[3], b[4], b[5]};
+    size_t bytes = ACLF_REC;
+    for (int q = 0; q < 4; q++) {
+        key_off[q] = (uint32_t)bytes;
+        bytes += (4 * (size_t)(m[q] + 8) + 7) & ~(size_t)7;
+        bv_off[q] = (uint32_t)bytes;
+        bytes += 8 * (size_t)(m[q] + 8);
+    }
+    bytes = (bytes + 15) & ~(size_t)15;
+    if (bytes > 65535) return;   // bucket entries are u16 byte offsets
+    f.assign(bytes / 4, 0);
+    uint16_t *bk = reinterpret_cast<uint16_t *>(f.data());
+    for (int q = 0; q < 4; q++) {
+        const uint32_t keys = b[8 + 2 * q], bv = b[9 + 2 * q], bko = b[18 + q];
+        for (uint32_t j = 0; j < m[q] + 8; j++) {
+            const uint32_t jj = std::min(j, m[q] - 1);   // the pad entries repeat the last one
+            f[key_off[q] / 4 + j] = b[keys + jj];
+            f[bv_off[q] / 4 + 2 * j] = b[bv + 2 * jj];
+            f[bv_off[q] / 4 + 2 * j + 1] = b[bv + 2 * jj + 1];
+        }
+        for (uint32_t t = 0; t < 256; t++) {
+            const uint32_t w = b[bko + t / 2], j = (t & 1) ? w >> 16 : w & 0xFFFF;
+            bk[q * 256 + t] = (uint16_t)(key_off[q] + 4 * j);
+        }
+    }
+    for (uint32_t i = 0; i < 512; i++) f[ACLF_PROTO / 4 + i] = b[b[16] + i];
+    for (uint32_t r = 0; r < b[0]; r++) f[ACLF_RULE / 4 + r] = b[b[17] + r];
+}
+
 // ---------------------------------------------------------------- DPI
 // Aho-Corasick (1975) goto/failure construction, converted to a full DFA over
 // byte classes (bytes that occur in no pattern share one class: from every

@@ -69,7 +69,7 @@ struct nfc_chain {
     DBuf uf_list[2], uf_cnt, uf_pass;     // NFC_F_UNFUSED scratch
     bool loaded[8] = {false};
     // tables
-    DBuf acl_r4, acl_r6;
+    DBuf acl_r4, acl_r6, acl_f4;
     AclImg acl{};
     DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta, dpi_sparse, dpi_frows, dpi_accid, dpi_accmeta;
     DpiImg dpi{};
@@ -180,7 +180,7 @@ void nfc_destroy_chain(nfc_chain *c)
     if (!c) return;
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
-    DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
+    DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->acl_f4, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
                    &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->dpi_frows, &c->dpi_accid, &c->dpi_accmeta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->nat_pool, &c->nat_dnat, &c->nat_nib,
@@ -227,6 +227,13 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
                         (uint32_t)b6.size(), s.n_rules, s.default_action, 0, {}, {}};
         std::copy(b4.begin(), b4.begin() + ACLBV_HDR, c->acl.hdr4);
         std::copy(b6.begin(), b6.begin() + ACLBV_HDR, c->acl.hdr6);
+        std::vector<uint32_t> f4;
+        build_acl4_fast(b4, f4, c->acl.f4_key, c->acl.f4_bv);
+        if (!f4.empty()) {
+            CK(c->acl_f4.upload(f4));
+            c->acl.f4 = c->acl_f4.as<uint32_t>();
+            c->acl.words_f4 = (uint32_t)f4.size();
+        }
         c->n_acl_rules = s.n_rules;
         break;
     }
@@ -453,6 +460,9 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     {
         const size_t limit = sfc_smem_limit(c->device);
         p.acl.smem_words = (c->mask & MASK_ACL) ? 1 : 0;
+        // the fused kernel stages the IPv4 record image when there is one (the unfused
+        // and parallel kernels read the bit-vector blob)
+        p.acl.fast = !par && !(c->flags & NFC_F_UNFUSED) && c->acl.f4 != nullptr ? 1u : 0u;
         p.dpi.hot_states = 0;
         p.dpi.sparse_states = 0;
         bool full = false;
@@ -567,7 +577,7 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
     if (rc) return fail(rc, err);
     c->last = nfc_launch_info{(uint32_t)lc.grid, (uint32_t)lc.block, (uint32_t)lc.smem,
                               (c->mask & MASK_DPI) ? (uint32_t)v.dm : 0u, p.dpi.hot_states, p.dpi.sparse_states,
-                              p.dpi.meta_smem, p.acl.smem_words ? 4 * (p.acl.words4 + p.acl.words6) : 0u};
+                              p.dpi.meta_smem, p.acl.smem_words ? 4 * ((p.acl.fast ? p.acl.words_f4 : p.acl.words4) + p.acl.words6) : 0u};
     c->launches += lc.launches;
     if (c->mask & MASK_IPSEC) c->seq_parity ^= 1;
     return NFC_OK;

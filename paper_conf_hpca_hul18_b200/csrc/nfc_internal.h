@@ -34,7 +34,20 @@ struct AclImg {
     uint32_t default_action;
     uint32_t smem_words;              // words staged in shared memory (0 = read from global)
     uint32_t hdr4[ACLBV_HDR], hdr6[ACLBV_HDR];   // image headers, read from the constant bank
+    // Search image of an IPv4 rule set with W == 1 and window depth <= 3 (build_acl4_fast):
+    // what the fused kernel stages in shared memory in place of the IPv4 blob (fast = 1)
+    const uint32_t *f4;               // device copy (nullptr: not representable)
+    uint32_t words_f4;                // its size (u32 words, 16-B multiple)
+    uint32_t fast;                    // per launch: 1 = the fused kernel stages f4 (acl4_fast)
+    uint32_t f4_key[4], f4_bv[4];     // byte offsets of the key and bitset arrays per field
 };
+// Search image layout (byte offsets): four 256-entry u16 bucket tables (src, dst,
+// sport, dport) on the top 8 key bits, each entry the byte offset of the window's
+// first key; the proto bitsets (256 x u64); the rule words (<= 64 x u32); then per
+// field the interval start keys (u32) and, apart, their bitsets (u64), both followed by
+// 8 copies of the last entry, so a 3-halving window search needs no clamp and the
+// bitset of key j sits at a fixed affine image of the key's address (bv + 2 (key - k0)).
+static const uint32_t ACLF_BK = 0, ACLF_PROTO = 2048, ACLF_RULE = 4096, ACLF_REC = 4352;
 
 // ---------------------------------------------------------------- DPI
 // Full Aho-Corasick DFA over byte classes, states numbered in BFS order.
@@ -241,6 +254,8 @@ struct DpiHost;
 std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_states);   // regex.cpp   // capi.cu: nfc_last_error + code
 struct HostImage { std::vector<uint8_t> bytes; };
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
+// the record image (AclImg::f4) of an IPv4 blob; empty if the blob does not qualify
+void build_acl4_fast(const std::vector<uint32_t> &blob4, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4]);
 struct DpiHost {
     std::vector<uint8_t> cls;
     std::vector<uint8_t> trans;   // raw bytes (u16 or u32 entries)

@@ -186,14 +186,15 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     }
     o = (o + 15) & ~15u;
     if (mask & MASK_ACL) {
-        const uint32_t s4 = p.acl.smem_words ? p.acl.words4 : 0, s6 = p.acl.smem_words ? p.acl.words6 : 0;
+        const uint32_t s4 = p.acl.smem_words ? (p.acl.fast ? p.acl.words_f4 : p.acl.words4) : 0,
+                       s6 = p.acl.smem_words ? p.acl.words6 : 0;
         L.acl4 = o; o += s4 * 4;
         L.acl6 = o; o += s6 * 4;
     }
     o = (o + 15) & ~15u;
     if ((mask & MASK_LPM4) && p.l4.nh_smem) { L.nh4 = o; o += p.l4.n_nh * 16; }
     if (p.n_batches > 1 && !(mask & MASK_IPSEC)) { L.crs = o; o += nwarp * 64; }
-    if (dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
+    if (NFC_REGROUP && dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
         L.prefix = o; o += 256 * 4;
@@ -548,6 +549,24 @@ __device__ __forceinline__ uint32_t acl_match_w(const AclMem<SM> &M, const uint3
     }
     return 0xFFFFu | default_action << 31;
 }
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a)
+{
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u16z(uint32_t a)
+{
+    uint32_t v;
+    asm("{\n\t.reg .u16 t;\n\tld.shared.u16 t, [%1];\n\tcvt.u32.u16 %0, t;\n\t}" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds_u64(uint32_t a)
+{
+    uint2 v;
+    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
 // shared-memory window search over absolute 32-bit shared addresses: D halvings
 // (compile-time), each a load at an immediate offset, a compare and a predicated add
 template <uint32_t H4>
@@ -569,12 +588,42 @@ __device__ __forceinline__ void acl_search4_s(uint32_t &as, uint32_t &ad, uint32
         acl_search4_s<D - 1>(as, ad, asp, adp, v);
     }
 }
+// IPv4 ACL from the search image (AclImg::f4) in shared memory at byte offset `img`:
+// per field one bucket read and three window halvings at immediate offsets over the
+// 4-B keys (the pad keys make overshooting the last interval harmless), then the
+// bitset at the key's affine image; returns as acl_core.  Any key stays in bounds
+// (dead lanes included).
+__device__ __forceinline__ uint32_t acl4_fast(uint32_t img, const AclImg &ai, const PV &v)
+{
+    const uint32_t B = (uint32_t)__cvta_generic_to_shared(nfc_smem) + img;
+    const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport & 0xFFFF, kdp = v.dport & 0xFFFF;
+    uint32_t as = B + lds_u16z(B + ACLF_BK + 2 * (ks >> 24));
+    uint32_t ad = B + lds_u16z(B + ACLF_BK + 512 + 2 * (kd >> 24));
+    uint32_t asp = B + lds_u16z(B + ACLF_BK + 1024 + 2 * (ksp >> 8));
+    uint32_t adp = B + lds_u16z(B + ACLF_BK + 1536 + 2 * (kdp >> 8));
+    acl_step_s<16>(as, ks); acl_step_s<16>(ad, kd); acl_step_s<16>(asp, ksp); acl_step_s<16>(adp, kdp);
+    acl_step_s<8>(as, ks); acl_step_s<8>(ad, kd); acl_step_s<8>(asp, ksp); acl_step_s<8>(adp, kdp);
+    acl_step_s<4>(as, ks); acl_step_s<4>(ad, kd); acl_step_s<4>(asp, ksp); acl_step_s<4>(adp, kdp);
+    // bitset address = 2 * key address + (bv - 2 key - B) per field
+    const uint2 a = lds_u64(2 * as + (ai.f4_bv[0] - 2 * ai.f4_key[0] - B));
+    const uint2 b = lds_u64(2 * ad + (ai.f4_bv[1] - 2 * ai.f4_key[1] - B));
+    const uint2 c = lds_u64(2 * asp + (ai.f4_bv[2] - 2 * ai.f4_key[2] - B));
+    const uint2 d = lds_u64(2 * adp + (ai.f4_bv[3] - 2 * ai.f4_key[3] - B));
+    const uint2 e = lds_u64(B + ACLF_PROTO + 8 * (v.proto & 255));
+    const uint32_t lo = a.x & b.x & c.x & d.x & e.x, hi = a.y & b.y & c.y & d.y & e.y;
+    const uint32_t bit = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
+    uint32_t r = 0xFFFFu | ai.default_action << 31;
+    if (lo | hi) r = lds_u32(B + ACLF_RULE + 4 * bit);
+    return r;
+}
 template <bool SM>
 __device__ __forceinline__ uint32_t acl_core(const AclMem<SM> &M4, const AclMem<SM> &M6, const AclImg &ai, const PV &v)
 {
     if (v.fam == 4) {
         const uint32_t *hd = ai.hdr4;
         if (hd[0] == 0) return 0xFFFFu | ai.default_action << 31;
+        if constexpr (SM)
+            if (ai.fast) return acl4_fast(M4.s, ai, v);
         const AclMem<SM> &M = M4;
         const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport, kdp = v.dport;
         // window starts (bucket reads on the top 8 key bits), as byte offsets
@@ -1836,55 +1885,6 @@ __device__ __forceinline__ bool nf_dpi_warp(const KParams &P, const Ctx &C, Pkt 
 // sequential chain (effects in original-order packet state).  Taken when
 // warp-uniformly: IPv4 ACL image with rules, <= 64 rules, depth <= 3, staged in
 // shared memory; otherwise the sequential path runs.
-__device__ __forceinline__ uint32_t lds_u32(uint32_t a)
-{
-    uint32_t v;
-    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint32_t lds_u16z(uint32_t a)
-{
-    uint32_t v;
-    asm("{\n\t.reg .u16 t;\n\tld.shared.u16 t, [%1];\n\tcvt.u32.u16 %0, t;\n\t}" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint2 lds_u64(uint32_t a)
-{
-    uint2 v;
-    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
-    return v;
-}
-// IPv4 ACL, W == 1 image in shared memory, depth <= 3: straight-line (returns as acl_core)
-__device__ __forceinline__ uint32_t acl4_spec(const KParams &P, const PV &v)
-{
-    const uint32_t *hd = P.acl.hdr4;
-    const uint32_t B = (uint32_t)__cvta_generic_to_shared(nfc_smem) + P.lay.acl4;
-    // (lanes whose parse failed carry arbitrary fields: every index below stays in bounds)
-    const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport & 0xFFFF, kdp = v.dport & 0xFFFF;
-    uint32_t as = B + 4 * hd[8] + 4 * lds_u16z(B + 4 * hd[18] + 2 * (ks >> 24));
-    uint32_t ad = B + 4 * hd[10] + 4 * lds_u16z(B + 4 * hd[19] + 2 * (kd >> 24));
-    uint32_t asp = B + 4 * hd[12] + 4 * lds_u16z(B + 4 * hd[20] + 2 * (ksp >> 8));
-    uint32_t adp = B + 4 * hd[14] + 4 * lds_u16z(B + 4 * hd[21] + 2 * (kdp >> 8));
-    const uint32_t D = hd[23];
-#pragma unroll
-    for (int i = 2; i >= 0; i--) {
-        const uint32_t h4 = (uint32_t)i < D ? 4u << i : 0u;    // steps beyond the depth are no-ops
-        as += lds_u32(as + h4) <= ks ? h4 : 0u;
-        ad += lds_u32(ad + h4) <= kd ? h4 : 0u;
-        asp += lds_u32(asp + h4) <= ksp ? h4 : 0u;
-        adp += lds_u32(adp + h4) <= kdp ? h4 : 0u;
-    }
-    const uint32_t js = min((as - B) / 4 - hd[8], hd[2] - 1), jd = min((ad - B) / 4 - hd[10], hd[3] - 1);
-    const uint32_t jsp = min((asp - B) / 4 - hd[12], hd[4] - 1), jdp = min((adp - B) / 4 - hd[14], hd[5] - 1);
-    const uint2 a = lds_u64(B + 4 * hd[9] + 8 * js), b = lds_u64(B + 4 * hd[11] + 8 * jd);
-    const uint2 c = lds_u64(B + 4 * hd[13] + 8 * jsp), d = lds_u64(B + 4 * hd[15] + 8 * jdp);
-    const uint2 e = lds_u64(B + 4 * hd[16] + 8 * (v.proto & 255));   // (dead lanes: any value, in bounds)
-    const uint32_t lo = a.x & b.x & c.x & d.x & e.x, hi = a.y & b.y & c.y & d.y & e.y;
-    const uint32_t bit = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
-    uint32_t r = 0xFFFFu | P.acl.default_action << 31;
-    if (lo | hi) r = lds_u32(B + 4 * (hd[17] + bit));
-    return r;
-}
 // DPI walk of payload bytes [a, min(b, 64)) from the header cache for a >= 42, every
 // step predicated (UDP and TCP payload starts in one code path)
 __device__ __forceinline__ Walk dpi_head_spec(const KParams &P, const uint32_t h[16], uint32_t a, uint32_t b)
@@ -1911,7 +1911,7 @@ template <uint32_t S>
 __device__ __forceinline__ bool spec_ok(const KParams &P)
 {
     return S != SIG_ANY && sig_kind(S, 0) == NFC_ACL && sig_n(S) >= 2 && sig_kind(S, 1) == NFC_DPI &&
-           P.acl.smem_words && P.acl.hdr4[0] != 0 && P.acl.hdr4[1] == 1 && P.acl.hdr4[23] <= 3;
+           P.acl.smem_words && P.acl.fast;
 }
 
 // one NF of kind KIND at chain position pos (KIND compile-time)
@@ -2037,11 +2037,11 @@ __device__ __forceinline__ void run_part(const KParams &P, const Ctx &C, Pkt &k)
             uint32_t r;
             Walk wh;
             if (fastw) {
-                r = acl4_spec(P, k.v);
+                r = acl4_fast(P.lay.acl4, P.acl, k.v);
                 wh = dpi_head_fast(P, k.h, k.v.pl_off == 54);
                 if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
             } else {
-                r = acl4_spec(P, k.v);
+                r = acl4_fast(P.lay.acl4, P.acl, k.v);
                 wh = dpi_head_spec(P, k.h, k.v.pl_off, k.v.ip_end);
                 if constexpr (T24) k.t24 = ld_tab16(P.l4.tbl24 + (k.v.dst[0] >> 8), C.pol_l);
             }
@@ -2255,7 +2255,10 @@ __device__ __forceinline__ void setup_ctx(const KParams &P, uint8_t *smem, const
         if (P.acl.smem_words) {
             uint4 *d4 = reinterpret_cast<uint4 *>(smem + L.acl4);
             uint4 *d6 = reinterpret_cast<uint4 *>(smem + L.acl6);
-            for (uint32_t i = tid; i < P.acl.words4 / 4; i += NT) d4[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv4) + i);
+            if (P.acl.fast)       // the record image (acl4_fast)
+                for (uint32_t i = tid; i < P.acl.words_f4 / 4; i += NT) d4[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.f4) + i);
+            else
+                for (uint32_t i = tid; i < P.acl.words4 / 4; i += NT) d4[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv4) + i);
             for (uint32_t i = tid; i < P.acl.words6 / 4; i += NT) d6[i] = __ldg(reinterpret_cast<const uint4 *>(P.acl.bv6) + i);
             C.acl4 = reinterpret_cast<const uint32_t *>(d4);
             C.acl6 = reinterpret_cast<const uint32_t *>(d6);

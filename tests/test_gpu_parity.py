@@ -378,3 +378,51 @@ def test_parallel_groups_validated(nfc):
     with pytest.raises(nfc.NfcError) as e:
         nfc.Chain(["IPSEC", "ACL", "IPSEC"], device=0)
     assert e.value.code == nfc.NFC_EUNSUP
+
+
+def test_c1_acl_boundary_keys(nfc):
+    """The IPv4 search image (AclImg::f4, three fixed halvings over padded key arrays):
+    5-tuples placed exactly on, just below and just above every rule's interval edges,
+    plus the extreme keys 0 / 2^32-1 and ports 0 / 65535, bit-exact vs the oracle's
+    linear rule scan (DESIGN.md ACL)."""
+    import oracle
+    from tests.gpu_util import compare_bytes, compare_records, gpu_run, sorted_pairs
+    w = nfcgen.workload("C1")
+    n = 4096
+    b = nfcgen.generate(w.traffic, w.tables, 0, n)
+    rules = w.tables.acl_rules
+    rng = np.random.default_rng(77)
+
+    def edges(lo, hi, top):
+        return [lo, hi, (lo - 1) % (top + 1), (hi + 1) % (top + 1), 0, top]
+
+    cand_ip, cand_port = [], []
+    for r in rules:
+        if r["family"] != 4:
+            continue
+        for fld, ln in (("src", "slen"), ("dst", "dlen")):
+            k = int.from_bytes(bytes(r[fld][:4]), "big")
+            m = (0xFFFFFFFF << (32 - int(r[ln]))) & 0xFFFFFFFF if r[ln] else 0
+            cand_ip += edges(k & m, (k & m) | (~m & 0xFFFFFFFF), 0xFFFFFFFF)
+        cand_port += edges(int(r["sp_lo"]), int(r["sp_hi"]), 0xFFFF) + edges(int(r["dp_lo"]), int(r["dp_hi"]), 0xFFFF)
+    ar = b.arena
+    placed = 0
+    for i in range(n):
+        o = int(b.off[i])
+        if int(b.len[i]) < 42 or ar[o + 12] != 0x08 or ar[o + 13] != 0x00 or ar[o + 14] != 0x45:
+            continue
+        ar[o + 26:o + 30] = np.frombuffer(int(rng.choice(cand_ip)).to_bytes(4, "big"), np.uint8)
+        ar[o + 30:o + 34] = np.frombuffer(int(rng.choice(cand_ip)).to_bytes(4, "big"), np.uint8)
+        ar[o + 34:o + 36] = np.frombuffer(int(rng.choice(cand_port)).to_bytes(2, "big"), np.uint8)
+        ar[o + 36:o + 38] = np.frombuffer(int(rng.choice(cand_port)).to_bytes(2, "big"), np.uint8)
+        placed += 1
+    assert placed > 3000
+    orc = oracle.OracleChain(w.kinds, w.tables)
+    want, want_arena, (wp, wq), npairs = orc.run(b, match_cap=1 << 16)
+    ch = _chain(nfc, w)
+    got, arenas, (gp, gq), k = gpu_run(ch, [b])
+    compare_records(got, want, "C1 ACL edges")
+    compare_bytes(want, arenas[0], b.off, want_arena, b.off, "C1 ACL edges")
+    assert k == npairs and np.array_equal(sorted_pairs(gp, gq), sorted_pairs(wp, wq))
+    # the edges exercise many distinct rules (not just the default)
+    assert len(np.unique(got["acl_rule"])) > 10
