@@ -197,7 +197,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     if (NFC_REGROUP && dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
-        L.prefix = o; o += 256 * 4;
+        L.prefix = o; o += (256 + 32) * 4;   // esp_assign prefixes; esp_ctr_tile block prefix + warp totals
     }
     L.total = o;
     return L;
@@ -1307,12 +1307,62 @@ __device__ __forceinline__ void sha1_compress(uint32_t H[5], uint32_t W[16])
 // the L4 bytes are encrypted where they lie, trailer and ICV are appended.
 // Returns the new frame length.  Stream bytes are handled as 32-bit words; memory
 // words are 4-B aligned and related to stream words by a funnel shift of r = A & 3.
+// ESP encapsulation of one packet, everything but the payload cipher and the MAC:
+// the header moves 16 B left (the frame now starts at f - 16), the IP header is
+// fixed up (proto 50, lengths, IPv4 checksum), the ESP header {SPI, seq, IV = 0 || seq}
+// goes to [l4 - 16, l4) of the old frame, and (trailer) the pad bytes 1..p, the pad
+// length and the next header are written as plaintext after the payload
+__device__ __forceinline__ void esp_header(uint8_t *f, const PV &v, uint32_t spi, uint32_t seq, uint32_t p, bool trailer)
+{
+    const uint32_t l4 = v.l4_off;
+    uint32_t *src = reinterpret_cast<uint32_t *>(f);
+    uint32_t *dst = reinterpret_cast<uint32_t *>(f - 16);
+    uint32_t nw = (l4 + 3) >> 2;
+    for (uint32_t i = 0; i < nw; i++) dst[i] = src[i];
+    uint8_t *g = f - 16;
+    if (v.fam == 4) {
+        g[23] = 50;
+        uint32_t tot = ((uint32_t)g[16] << 8 | g[17]) + 30 + p;
+        g[16] = (uint8_t)(tot >> 8); g[17] = (uint8_t)tot;
+        g[24] = 0; g[25] = 0;
+        uint32_t sum = 0;
+        for (uint32_t k = 14; k < l4; k += 2) sum += (uint32_t)g[k] << 8 | g[k + 1];
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        sum = (sum & 0xFFFF) + (sum >> 16);
+        sum = ~sum;
+        g[24] = (uint8_t)(sum >> 8); g[25] = (uint8_t)sum;
+    } else {
+        g[20] = 50;
+        uint32_t pl = ((uint32_t)g[18] << 8 | g[19]) + 30 + p;
+        g[18] = (uint8_t)(pl >> 8); g[19] = (uint8_t)pl;
+    }
+    // the new frame starts at f-16, so its ESP header bytes [l4, l4+16) are f+[l4-16, l4)
+    uint8_t *e = f + l4 - 16;
+    const uint32_t hw[4] = {spi, seq, 0u, seq};
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        e[4 * i] = (uint8_t)(hw[i] >> 24); e[4 * i + 1] = (uint8_t)(hw[i] >> 16);
+        e[4 * i + 2] = (uint8_t)(hw[i] >> 8); e[4 * i + 3] = (uint8_t)hw[i];
+    }
+    if (trailer) {
+        const uint32_t plen = v.ip_end - l4;
+        uint8_t *t = f + l4 + plen;
+        for (uint32_t b = 0; b < p; b++) t[b] = (uint8_t)(b + 1);
+        t[p] = (uint8_t)p;
+        t[p + 1] = (uint8_t)v.proto;
+    }
+}
+// pre: the packet was prepared by esp_prepare (header moved, ESP header and trailer
+// written) and its [A, A + clen) encrypted in place by the tile's balanced AES pass
+// (esp_ctr_tile): only the HMAC is computed here, over the ciphertext in memory
+template <bool pre>
 __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t seq, const uint32_t *te,
                                            const uint32_t *rk_smem)
 {
     const uint32_t l4 = v.l4_off, plen = v.ip_end - l4;
 #if NFC_ESP_PF
-    for (uint32_t o = 128; o < v.ip_end; o += 128) prefetch_l2(f + o);
+    if constexpr (!pre)
+        for (uint32_t o = 128; o < v.ip_end; o += 128) prefetch_l2(f + o);
 #endif
     const uint32_t p = (4 - ((plen + 2) & 3)) & 3;
     const uint32_t clen = plen + p + 2;          // multiple of 4
@@ -1329,43 +1379,17 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
 #endif
     const uint32_t spi = __ldg(&sap->spi), nonce = __ldg(&sap->nonce);
     // 1. move the header 16 B left and fix up the IP header
-    {
-        uint32_t *src = reinterpret_cast<uint32_t *>(f);
-        uint32_t *dst = reinterpret_cast<uint32_t *>(f - 16);
-        uint32_t nw = (l4 + 3) >> 2;
-        for (uint32_t i = 0; i < nw; i++) dst[i] = src[i];
-        uint8_t *g = f - 16;
-        if (v.fam == 4) {
-            g[23] = 50;
-            uint32_t tot = ((uint32_t)g[16] << 8 | g[17]) + 30 + p;
-            g[16] = (uint8_t)(tot >> 8); g[17] = (uint8_t)tot;
-            g[24] = 0; g[25] = 0;
-            uint32_t sum = 0;
-            for (uint32_t k = 14; k < l4; k += 2) sum += (uint32_t)g[k] << 8 | g[k + 1];
-            sum = (sum & 0xFFFF) + (sum >> 16);
-            sum = (sum & 0xFFFF) + (sum >> 16);
-            sum = ~sum;
-            g[24] = (uint8_t)(sum >> 8); g[25] = (uint8_t)sum;
-        } else {
-            g[20] = 50;
-            uint32_t pl = ((uint32_t)g[18] << 8 | g[19]) + 30 + p;
-            g[18] = (uint8_t)(pl >> 8); g[19] = (uint8_t)pl;
-        }
-        // the new frame starts at f-16, so its ESP header bytes [l4, l4+16) are f+[l4-16, l4)
-        uint8_t *e = f + l4 - 16;
-        const uint32_t hw[4] = {spi, seq, 0u, seq};
-#pragma unroll
-        for (int i = 0; i < 4; i++) {
-            e[4 * i] = (uint8_t)(hw[i] >> 24); e[4 * i + 1] = (uint8_t)(hw[i] >> 16);
-            e[4 * i + 2] = (uint8_t)(hw[i] >> 8); e[4 * i + 3] = (uint8_t)hw[i];
-        }
-    }
+    if constexpr (!pre) esp_header(f, v, spi, seq, p, false);
     // 2. encrypt [A, A+clen) in place and MAC [A-16, A+clen), A = f + l4
     uint8_t *A = f + l4;
     const uint32_t r = (uint32_t)(reinterpret_cast<uintptr_t>(A) & 3);
     uint32_t *W0 = reinterpret_cast<uint32_t *>(A - r);   // aligned word 0 (contains stream bytes -r..3-r)
     const uint32_t sh = 32 - 8 * r;                       // funnel amount memory<-stream
-    uint32_t Mcur = W0[0];                                // memory word k (plaintext side)
+    // pre: the ciphertext was XORed in at L2; only the lines holding header bytes can sit
+    // in L1 (esp_header read the header words), so words below `l1` are read L2-only
+    // (ld.cg) and the rest through L1 (one L2 request per line)
+    const uint32_t *l1 = reinterpret_cast<const uint32_t *>((reinterpret_cast<uintptr_t>(f + l4 - 1) | (uintptr_t)127) + 1);
+    uint32_t Mcur = pre ? __ldcg(W0) : W0[0];             // memory word k (plaintext side; ciphertext if pre)
     uint32_t Cprev = r ? (Mcur << (8 * (4 - r))) : 0u;    // carries the IV bytes below A
     uint32_t H[5];
 #pragma unroll
@@ -1385,6 +1409,14 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
                 m = (w == 0) ? spi : (w == 2) ? 0u : seq;
             } else if (i < nmsg) {
                 const uint32_t k = i - 4;                 // stream word
+                if constexpr (pre) {                      // ciphertext already in memory (L2)
+                    const uint32_t Mnext = W0 + k + 1 < l1 ? __ldcg(W0 + k + 1) : W0[k + 1];
+                    const uint32_t C = __funnelshift_rc(Mcur, Mnext, 8 * r);
+                    Cprev = C;
+                    Mcur = Mnext;
+                    W[w] = bswap32(C);
+                    continue;
+                }
                 if ((w & 3) == 0) {                       // new AES counter block every 4 words
 #if NFC_ESP_RK_SMEM
                     const uint4 o = aes128_encrypt_s(te, rks, nonce, 0u, seq, (k >> 2) + 1);
@@ -1454,6 +1486,7 @@ struct Pkt {
     uint32_t t24;             // TBL24 entry, loaded right after parse (NFC_EARLY_T24)
     uint32_t mmeta, mslot;    // deferred match-pair emission: closure meta, first pair slot
     uint32_t mbase;           // deferred warp-aggregated claim: base slot (lane 0)
+    uint32_t esp_pre;         // 1: encapsulated and encrypted by the tile's balanced CTR pass (esp_ctr_tile)
     bool alive;
 };
 
@@ -1614,6 +1647,7 @@ __device__ __forceinline__ void pkt_begin(const Ctx &C, const Loc &l, bool valid
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
+    k.esp_pre = 0;
     k.npairs = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
@@ -1628,6 +1662,7 @@ __device__ __forceinline__ void pkt_begin_h(const Loc &l, bool valid, Pkt &k, co
 {
     k.drop = 0xFF; k.esp_sa = 0xFF; k.port = 0; k.acl_rule = 0xFFFF; k.lb_b = 0xFFFF; k.nmatch = 0;
     k.esp_seq = 0; k.passmask = 0; k.esp_bytes = 0; k.alive = false; k.t24 = 0xFFFFFFFFu; k.mmeta = 0; k.mbase = 0;
+    k.esp_pre = 0;
     k.npairs = 0;
     k.f = l.f; k.flen = k.orig_len = l.len; k.g = l.g;
     k.out_len = k.flen;
@@ -1955,8 +1990,10 @@ __device__ __forceinline__ void nf_apply(const KParams &P, const Ctx &C, Pkt &k,
             k.port = pt;
         }
     } else if constexpr (KIND == NFC_IPSEC) {
-        const uint32_t nl = nf_esp(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te,
-                                   reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.rk) + k.esp_sa * ESP_RK_STRIDE);
+        const uint32_t *rks = reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.rk) + k.esp_sa * ESP_RK_STRIDE;
+        // (two instances: the MAC-only one after the tile's balanced CTR pass, tile-uniform)
+        const uint32_t nl = k.esp_pre ? nf_esp<true>(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te, rks)
+                                      : nf_esp<false>(k.f, k.v, P.esp.sa + k.esp_sa, k.esp_seq, C.te, rks);
         k.esp_bytes = nl - 28 - k.v.l4_off;      // ciphertext bytes |C|
         k.f -= 16;
         k.flen = nl;
@@ -2219,6 +2256,110 @@ __device__ __forceinline__ void esp_assign(const KParams &P, const Ctx &C, uint8
         k.esp_seq = __ldg(P.seq_in + sa) + pref[sa] + wcnt[warp * 256 + sa] + rank + 1;
         var_stat(P, C, P.st_sa + sa);
     }
+}
+
+#ifndef NFC_ESP_BALANCE
+#define NFC_ESP_BALANCE 2     // balanced CTR pass when the tile's largest packet has > this x the mean AES blocks (0: off)
+#endif
+// a3 for the IPsec tiles: the AES-CTR keystream blocks of the tile's
+// SURVIVORS (packets alive at the IPsec position; dropped packets contribute none) are
+// concatenated into one block list and split evenly over the CTA's threads.  With
+// mixed sizes (IMIX) a thread-per-packet cipher runs every warp as long as its longest
+// packet; here each thread encrypts ~total/NT blocks whatever the mix.  Each packet's
+// own thread first writes its ESP header and plaintext trailer (esp_header); after a
+// barrier the block owners XOR the keystream into the frames with fire-and-forget
+// red.global.xor on the aligned words a block touches (a word shared by two blocks gets
+// both halves, in either order); after a second barrier each thread MACs its own packet
+// over the ciphertext (nf_esp, pre).  Tiles whose sizes are balanced (the largest
+// packet within NFC_ESP_BALANCE x the mean) keep the fused per-thread cipher + MAC.
+// AES blocks of this thread's packet (0 unless it reaches IPsec); the warp's inclusive
+// prefix is returned and the warp's total and largest count go to shared memory --
+// before esp_assign, whose barriers publish them (no barrier of its own)
+template <int NW>
+__device__ __forceinline__ uint32_t esp_blocks_scan(uint8_t *smem, const SmemLayout &L, const Pkt &k)
+{
+    constexpr uint32_t NT = NW * 32, FULL = 0xFFFFFFFFu;
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t nb = 0;
+    if (k.alive) {
+        const uint32_t plen = k.v.ip_end - k.v.l4_off;
+        nb = (plen + ((4 - ((plen + 2) & 3)) & 3) + 2 + 15) >> 4;
+    }
+    uint32_t incl = nb;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, d);
+        if (lane >= (uint32_t)d) incl += y;
+    }
+    const uint32_t wmax = __reduce_max_sync(FULL, nb);
+    uint32_t *wtot = reinterpret_cast<uint32_t *>(smem + L.prefix) + NT;
+    if (lane == 31) { wtot[warp] = incl; wtot[NW + warp] = wmax; }
+    return incl;
+}
+template <int NW>
+__device__ __forceinline__ void esp_ctr_tile(const KParams &P, const Ctx &C, uint8_t *smem, const SmemLayout &L, Pkt &k,
+                                             uint32_t incl)
+{
+    constexpr uint32_t NT = NW * 32;
+    const uint32_t tid = threadIdx.x, warp = tid >> 5;
+    const bool e = k.alive;                 // alive at the IPsec position: ESP applies
+    uint32_t *pref = reinterpret_cast<uint32_t *>(smem + L.prefix), *wtot = pref + NT, *wmx = pref + NT + NW;
+    uint32_t off = 0, T = 0, mx = 0;
+#pragma unroll
+    for (int w = 0; w < NW; w++) {
+        const uint32_t t = wtot[w];
+        off += (uint32_t)w < warp ? t : 0u;
+        T += t;
+        mx = max(mx, wmx[w]);
+    }
+    if (NFC_ESP_BALANCE == 0 || T == 0 || (uint64_t)mx * NT <= (uint64_t)NFC_ESP_BALANCE * T) return;   // CTA-uniform
+    incl += off;
+    uint4 *rec = reinterpret_cast<uint4 *>(smem + L.wcnt);   // NT records over esp_assign's scratch
+    __syncthreads();                        // esp_assign's readers of its scratch are done
+    pref[tid] = incl;
+    if (e) {
+        const uint32_t plen = k.v.ip_end - k.v.l4_off, p = (4 - ((plen + 2) & 3)) & 3, clen = plen + p + 2;
+        esp_header(k.f, k.v, __ldg(&P.esp.sa[k.esp_sa].spi), k.esp_seq, p, true);
+        const uint64_t A = reinterpret_cast<uint64_t>(k.f) + k.v.l4_off;
+        rec[tid] = make_uint4((uint32_t)A, (uint32_t)(A >> 32), clen | k.esp_sa << 16, k.esp_seq);
+    }
+    k.esp_pre = 1;
+    __threadfence();                        // the header / trailer bytes are performed at L2 before the XORs
+    __syncthreads();                        // headers, trailers, records and prefixes visible
+    const uint32_t per = (T + NT - 1) / NT;
+    uint32_t q = min(tid * per, T);
+    const uint32_t qe = min(q + per, T);
+    if (q < qe) {
+        uint32_t i = 0;                     // the packet owning block q: first i with pref[i] > q
+#pragma unroll
+        for (uint32_t bit = NT / 2; bit; bit >>= 1)
+            if (pref[i + bit - 1] <= q) i += bit;
+        const uint32_t *rk0 = reinterpret_cast<const uint32_t *>(nfc_smem + P.lay.rk);
+        // one flat loop with one block per iteration: the lanes of a warp stay converged at
+        // the cipher call whatever the packet boundaries inside their ranges
+        for (; q < qe; q++) {
+            while (pref[i] <= q) i++;       // next packet (packets without blocks skipped)
+            const uint32_t j = q - (i ? pref[i - 1] : 0u);
+            const uint4 R = rec[i];
+            const uint32_t cl = R.z & 0xFFFF, sa = R.z >> 16, seq = R.w;
+            const uint64_t A = (uint64_t)R.x | (uint64_t)R.y << 32;
+            const uint32_t r = (uint32_t)(A & 3), sh = 8 * r;
+            uint32_t *Wj = reinterpret_cast<uint32_t *>(A - r) + 4 * j;
+            const uint4 o = aes128_encrypt_s(C.te, rk0 + sa * ESP_RK_STRIDE, __ldg(&P.esp.sa[sa].nonce), 0u, seq, j + 1);
+            const uint32_t ks[4] = {bswap32(o.x), bswap32(o.y), bswap32(o.z), bswap32(o.w)};
+            const uint32_t nw = min(4u, (cl - 16 * j) >> 2);          // clen is a multiple of 4
+            uint32_t carry = 0;
+#pragma unroll
+            for (int w = 0; w < 4; w++)
+                if ((uint32_t)w < nw) {
+                    atomicXor(Wj + w, (ks[w] << sh) | carry);
+                    carry = r ? ks[w] >> (32 - sh) : 0u;
+                }
+            if (r) atomicXor(Wj + nw, carry);
+        }
+    }
+    __threadfence();                        // every XOR performed at L2 ...
+    __syncthreads();                        // ... before the MACs read the ciphertext (ld.cg)
 }
 
 // Per-CTA context: pointers into the tables, staged into shared memory for the NFs of
@@ -2549,7 +2690,14 @@ __global__ void __launch_bounds__(KCfg<S, DM>::threads, KCfg<S, DM>::minb) sfc_k
             Pkt k;
             pkt_begin(C, pkt_locate(P, g, valid), valid, k);
             run_part<S, DM, true>(P, C, k);
+#if NFC_ESP_RK_SMEM
+            uint32_t bincl = 0;
+            if constexpr (S != SIG_ANY) bincl = esp_blocks_scan<NW>(smem, L, k);
+#endif
             esp_assign<NW>(P, C, smem, L, tile, k);
+#if NFC_ESP_RK_SMEM
+            if constexpr (S != SIG_ANY) esp_ctr_tile<NW>(P, C, smem, L, k, bincl);   // (the generic kernel: fused cipher)
+#endif
             run_part<S, DM, false>(P, C, k);
             pkt_end<S>(P, C, k, valid, g, ws, lane);
         }

@@ -426,3 +426,19 @@ def test_c1_acl_boundary_keys(nfc):
     assert k == npairs and np.array_equal(sorted_pairs(gp, gq), sorted_pairs(wp, wq))
     # the edges exercise many distinct rules (not just the default)
     assert len(np.unique(got["acl_rule"])) > 10
+
+
+@pytest.mark.parametrize("cfg,k", [("C2", None), ("C4", None), ("C5", 5), ("C5", 6)])
+def test_esp_balanced_ctr_imix(nfc, cfg, k):
+    """a3 for the IPsec tiles (esp_ctr_tile): IMIX tiles take the balanced CTR pass (the
+    survivors' AES blocks split evenly over the CTA, XORed in with red.xor, then MAC-only
+    nf_esp).  Edge frames (IPv4 options, IPv6, fragments, malformed) and drops before IPsec
+    mixed in; per-SA sequence numbers carried across two calls; bit-exact vs the oracle."""
+    w = nfcgen.workload(cfg, k=k, pkt_len=0, small=(cfg != "C2"))
+    w.traffic.tcp_pct = 30
+    w.traffic.edge(80_000)
+    w.traffic.malformed_ppm = 10_000
+    ch = _chain(nfc, w)
+    got, _ = check_parity(w, ch, 5000, split=[1700])
+    assert (got["esp_sa"] != 0xFF).sum() > 2000
+    check_parity(w, ch, 3000, first=5000)
