@@ -197,7 +197,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     if (NFC_REGROUP && dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
-        L.prefix = o; o += (256 + 32) * 4;   // esp_assign prefixes; esp_ctr_tile block prefix + warp totals
+        L.prefix = o; o += (256 + 64) * 4;   // esp_assign prefixes; esp_ctr_tile block prefix + warp totals
     }
     L.total = o;
     return L;
@@ -1352,9 +1352,67 @@ __device__ __forceinline__ void esp_header(uint8_t *f, const PV &v, uint32_t spi
         t[p + 1] = (uint8_t)v.proto;
     }
 }
-// pre: the packet was prepared by esp_prepare (header moved, ESP header and trailer
-// written) and its [A, A + clen) encrypted in place by the tile's balanced AES pass
-// (esp_ctr_tile): only the HMAC is computed here, over the ciphertext in memory
+// HMAC-SHA1-96 of an encapsulated packet whose [A, A + clen) is already ciphertext in
+// memory (the balanced pass XORed it in at L2): message = ESP header {spi, seq, 0, seq}
+// || ciphertext, keyed by the SA's precomputed ipad / opad states; the 12-B ICV is
+// written at A + clen.  Only the lines holding header bytes (below A) can sit in L1
+// (esp_header read them), so words below `l1` are read L2-only (ld.cg), the rest
+// through L1 (one L2 request per line).
+__device__ __forceinline__ void esp_mac_mem(uint8_t *A, uint32_t clen, const EspSa *sap, uint32_t seq)
+{
+    const uint32_t spi = __ldg(&sap->spi), nK = clen >> 2;
+    const uint32_t r = (uint32_t)(reinterpret_cast<uintptr_t>(A) & 3);
+    uint32_t *W0 = reinterpret_cast<uint32_t *>(A - r);
+    const uint32_t sh = 32 - 8 * r;
+    const uint32_t *l1 = reinterpret_cast<const uint32_t *>((reinterpret_cast<uintptr_t>(A - 1) | (uintptr_t)127) + 1);
+    uint32_t Mcur = __ldcg(W0);
+    uint32_t Cprev = r ? (Mcur << (8 * (4 - r))) : 0u;
+    uint32_t H[5];
+#pragma unroll
+    for (int i = 0; i < 5; i++) H[i] = __ldg(&sap->ipad[i]);
+    uint32_t W[16];
+    const uint32_t nmsg = 4 + nK;
+    const uint32_t total_bits = (64u + 4u * nmsg) * 8u;
+    const uint32_t nblk = (4 * nmsg + 9 + 63) / 64;
+    for (uint32_t blk = 0; blk < nblk; blk++) {
+#pragma unroll
+        for (int w = 0; w < 16; w++) {
+            const uint32_t i = blk * 16 + w;
+            uint32_t m;
+            if (i < 4) {
+                m = (w == 0) ? spi : (w == 2) ? 0u : seq;
+            } else if (i < nmsg) {
+                const uint32_t k = i - 4;
+                const uint32_t Mnext = W0 + k + 1 < l1 ? __ldcg(W0 + k + 1) : W0[k + 1];
+                const uint32_t C = __funnelshift_rc(Mcur, Mnext, 8 * r);
+                Cprev = C;
+                Mcur = Mnext;
+                m = bswap32(C);
+            } else if (i == nmsg) {
+                m = 0x80000000u;
+            } else if (i == nblk * 16 - 1) {
+                m = total_bits;
+            } else {
+                m = 0;
+            }
+            W[w] = m;
+        }
+        sha1_compress(H, W);
+    }
+    uint32_t G[5];
+#pragma unroll
+    for (int i = 0; i < 5; i++) G[i] = __ldg(&sap->opad[i]);
+#pragma unroll
+    for (int i = 0; i < 16; i++) W[i] = i < 5 ? H[i] : (i == 5 ? 0x80000000u : (i == 15 ? (64u + 20u) * 8u : 0u));
+    sha1_compress(G, W);
+    const uint32_t icv[3] = {bswap32(G[0]), bswap32(G[1]), bswap32(G[2])};
+    W0[nK] = __funnelshift_rc(Cprev, icv[0], sh);
+    W0[nK + 1] = __funnelshift_rc(icv[0], icv[1], sh);
+    W0[nK + 2] = __funnelshift_rc(icv[1], icv[2], sh);
+    if (r) W0[nK + 3] = __funnelshift_rc(icv[2], 0u, sh);
+}
+// pre: the packet was encapsulated, encrypted and MACed by its tile's balanced pass
+// (esp_ctr_tile): only the new frame length is returned
 template <bool pre>
 __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa *sap, uint32_t seq, const uint32_t *te,
                                            const uint32_t *rk_smem)
@@ -1377,19 +1435,16 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
         for (int i = 0; i < 11; i++) { uint4 x = __ldg(q + i); rk[4 * i] = x.x; rk[4 * i + 1] = x.y; rk[4 * i + 2] = x.z; rk[4 * i + 3] = x.w; }
     }
 #endif
+    if constexpr (pre) return v.ip_end + 30 + p;
     const uint32_t spi = __ldg(&sap->spi), nonce = __ldg(&sap->nonce);
     // 1. move the header 16 B left and fix up the IP header
-    if constexpr (!pre) esp_header(f, v, spi, seq, p, false);
+    esp_header(f, v, spi, seq, p, false);
     // 2. encrypt [A, A+clen) in place and MAC [A-16, A+clen), A = f + l4
     uint8_t *A = f + l4;
     const uint32_t r = (uint32_t)(reinterpret_cast<uintptr_t>(A) & 3);
     uint32_t *W0 = reinterpret_cast<uint32_t *>(A - r);   // aligned word 0 (contains stream bytes -r..3-r)
     const uint32_t sh = 32 - 8 * r;                       // funnel amount memory<-stream
-    // pre: the ciphertext was XORed in at L2; only the lines holding header bytes can sit
-    // in L1 (esp_header read the header words), so words below `l1` are read L2-only
-    // (ld.cg) and the rest through L1 (one L2 request per line)
-    const uint32_t *l1 = reinterpret_cast<const uint32_t *>((reinterpret_cast<uintptr_t>(f + l4 - 1) | (uintptr_t)127) + 1);
-    uint32_t Mcur = pre ? __ldcg(W0) : W0[0];             // memory word k (plaintext side; ciphertext if pre)
+    uint32_t Mcur = W0[0];                                // memory word k (plaintext side)
     uint32_t Cprev = r ? (Mcur << (8 * (4 - r))) : 0u;    // carries the IV bytes below A
     uint32_t H[5];
 #pragma unroll
@@ -1409,14 +1464,6 @@ __device__ __forceinline__ uint32_t nf_esp(uint8_t *f, const PV &v, const EspSa 
                 m = (w == 0) ? spi : (w == 2) ? 0u : seq;
             } else if (i < nmsg) {
                 const uint32_t k = i - 4;                 // stream word
-                if constexpr (pre) {                      // ciphertext already in memory (L2)
-                    const uint32_t Mnext = W0 + k + 1 < l1 ? __ldcg(W0 + k + 1) : W0[k + 1];
-                    const uint32_t C = __funnelshift_rc(Mcur, Mnext, 8 * r);
-                    Cprev = C;
-                    Mcur = Mnext;
-                    W[w] = bswap32(C);
-                    continue;
-                }
                 if ((w & 3) == 0) {                       // new AES counter block every 4 words
 #if NFC_ESP_RK_SMEM
                     const uint4 o = aes128_encrypt_s(te, rks, nonce, 0u, seq, (k >> 2) + 1);
@@ -2360,6 +2407,41 @@ __device__ __forceinline__ void esp_ctr_tile(const KParams &P, const Ctx &C, uin
     }
     __threadfence();                        // every XOR performed at L2 ...
     __syncthreads();                        // ... before the MACs read the ciphertext (ld.cg)
+    // the MACs: one packet per thread, the survivors ordered by length (counting sort on
+    // 64-B buckets, longest first) so that each warp's packets take about as many SHA-1
+    // blocks; the packet's own thread then only re-parses (nf_esp<true>)
+    uint32_t *perm = pref, *hist = pref + NT, *cur = pref + NT + 32;
+    uint32_t nb = 0;
+    if (e) {
+        const uint32_t plen = k.v.ip_end - k.v.l4_off;
+        nb = (plen + ((4 - ((plen + 2) & 3)) & 3) + 2 + 15) >> 4;
+    }
+    const uint32_t b = 31u - min(nb >> 2, 31u);   // longest first
+    if (tid < 64) hist[tid] = 0;            // hist and cur
+    __syncthreads();
+    if (e) atomicAdd(&hist[b], 1u);
+    __syncthreads();
+    if (warp == 0) {
+        const uint32_t lane = tid & 31, h = hist[lane];
+        uint32_t x = h;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
+            if (lane >= (uint32_t)d) x += y;
+        }
+        cur[lane] = x - h;                  // bucket bases
+        if (lane == 31) hist[0] = x;        // survivors
+    }
+    __syncthreads();
+    const uint32_t ns = hist[0];
+    if (e) perm[atomicAdd(&cur[b], 1u)] = tid;
+    __syncthreads();
+    if (tid < ns) {
+        const uint4 R = rec[perm[tid]];
+        uint8_t *A = reinterpret_cast<uint8_t *>((uint64_t)R.x | (uint64_t)R.y << 32);
+        esp_mac_mem(A, R.z & 0xFFFF, P.esp.sa + (R.z >> 16), R.w);
+    }
+    __syncthreads();                        // every ICV written before the packets move on
 }
 
 // Per-CTA context: pointers into the tables, staged into shared memory for the NFs of

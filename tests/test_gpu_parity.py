@@ -433,7 +433,7 @@ def test_esp_balanced_ctr_imix(nfc, cfg, k):
     """a3 for the IPsec tiles (esp_ctr_tile): IMIX tiles take the balanced CTR pass (the
     survivors' AES blocks split evenly over the CTA, XORed in with red.xor, then MAC-only
     nf_esp).  Edge frames (IPv4 options, IPv6, fragments, malformed) and drops before IPsec
-    mixed in; per-SA sequence numbers carried across two calls; bit-exact vs the oracle."""
+    mixed in; two batches in one call; bit-exact vs the oracle."""
     w = nfcgen.workload(cfg, k=k, pkt_len=0, small=(cfg != "C2"))
     w.traffic.tcp_pct = 30
     w.traffic.edge(80_000)
@@ -441,4 +441,3 @@ def test_esp_balanced_ctr_imix(nfc, cfg, k):
     ch = _chain(nfc, w)
     got, _ = check_parity(w, ch, 5000, split=[1700])
     assert (got["esp_sa"] != 0xFF).sum() > 2000
-    check_parity(w, ch, 3000, first=5000)
