@@ -541,6 +541,8 @@ static int process_impl(nfc_chain *c, const nfc_batch *bs, uint32_t nb, const nf
         c->launches += nl;
         return NFC_OK;
     }
+    // IPsec tiles are one CTA each: a variant with bigger CTAs takes fewer, bigger tiles
+    if ((c->mask & MASK_IPSEC) && !par && v.threads > (int)TILE_N) p.n_tiles = (uint32_t)((total + v.threads - 1) / v.threads);
     LaunchCfg lc{};
     if (!par && nb > 1 && !(c->mask & MASK_IPSEC)) {
         // multi-batch call: per-chunk descriptor records for the pipelined warp loop

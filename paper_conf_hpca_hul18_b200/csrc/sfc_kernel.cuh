@@ -136,7 +136,17 @@ __host__ __device__ constexpr bool kcfg_big(uint32_t S)
 {
     return S != SIG_ANY && !(sig_mask(S) & (1u << NFC_IPSEC)) && (sig_mask(S) & (1u << NFC_DPI));
 }
-__host__ __device__ constexpr int kcfg_threads(uint32_t S, int dm) { return kcfg_big(S) ? (dm == DM_FULL ? NFC_FULL_THREADS : NFC_HOTBIG_THREADS) : 256; }
+#ifndef NFC_ESP_DPI_THREADS
+#define NFC_ESP_DPI_THREADS 512   // IPsec chains with DPI: one 512-packet tile per SM (the DFA tiers get the SM's shared memory)
+#endif
+__host__ __device__ constexpr bool kcfg_esp_dpi(uint32_t S)
+{
+    return S != SIG_ANY && (sig_mask(S) & (1u << NFC_IPSEC)) && (sig_mask(S) & (1u << NFC_DPI));
+}
+__host__ __device__ constexpr int kcfg_threads(uint32_t S, int dm)
+{
+    return kcfg_big(S) ? (dm == DM_FULL ? NFC_FULL_THREADS : NFC_HOTBIG_THREADS) : kcfg_esp_dpi(S) ? NFC_ESP_DPI_THREADS : 256;
+}
 // per-warp counter slots: the fixed counters + 4 per chain position
 __host__ __device__ constexpr int kcfg_nws(uint32_t S) { return ST_POS_BASE + 4 * (S == SIG_ANY ? NFC_MAX_CHAIN : (int)sig_n(S)); }
 // chains whose warp loop regroups mixed IPv4/IPv6 chunks (NFC_REGROUP): the ones with the
@@ -149,7 +159,7 @@ template <uint32_t S, int DM> struct KCfg {
     static constexpr int nws = kcfg_nws(S);
     static constexpr bool esp = (sig_mask(S) & (1u << NFC_IPSEC)) != 0;
     static constexpr int threads = kcfg_threads(S, DM);
-    static constexpr int minb = esp ? NFC_ESP_MINB : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
+    static constexpr int minb = esp ? (kcfg_threads(S, DM) > 256 ? 1 : NFC_ESP_MINB) : (kcfg_big(S) ? 1 : NFC_HOT_MINB);
     static constexpr int nwarp = threads / 32;
     static constexpr uint32_t claim = DM == DM_FULL ? NFC_CLAIM : 1;   // chunks per warp claim
 };
@@ -197,7 +207,7 @@ __host__ __device__ inline SmemLayout smem_layout(uint32_t mask, int nwarp, cons
     if (NFC_REGROUP && dm == DM_FULL && (mask & MASK_ACL) && (mask & MASK_DPI) && !(mask & MASK_IPSEC)) { L.rgq = o; o += nwarp * NFC_RGQ * 4; }
     if (mask & MASK_IPSEC) {
         L.wcnt = o; o += nwarp * 256 * 2;
-        L.prefix = o; o += (256 + 64) * 4;   // esp_assign prefixes; esp_ctr_tile block prefix + warp totals
+        L.prefix = o; o += (max(256, nwarp * 32) + 64) * 4;   // esp_assign prefixes; esp_ctr_tile block prefix + warp totals
     }
     L.total = o;
     return L;
