@@ -114,6 +114,9 @@ __host__ __device__ constexpr uint32_t make_sig(uint32_t n, uint32_t k0, uint32_
 #ifndef NFC_FWD_DERIVED
 #define NFC_FWD_DERIVED 0     // 1: the forwarded count derived at the flush (pkts - parse drops - NF drops)
 #endif
+#ifndef NFC_LD256
+#define NFC_LD256 1           // 256-bit header loads / rewrite stores for 32-B aligned frames
+#endif
 #ifndef NFC_WALK_AHEAD
 #define NFC_WALK_AHEAD 0      // 1: split-walk payload words loaded one 16-B step ahead
 #endif
@@ -248,6 +251,22 @@ __device__ __forceinline__ uint4 ld_stream16(const void *a, uint64_t pol)
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a), "l"(pol));
     return v;
 }
+// 32-B (256-bit) versions: one L1TEX data-pipe wavefront per 128-B line for twice the
+// bytes of a 16-B access -- the fused kernel's header loads and rewrite stores touch
+// 16 lines per warp instruction (32 frames), so they cost half the wavefronts (needs a
+// 32-B aligned address)
+__device__ __forceinline__ void ld_stream32(const void *a, uint64_t pol, uint32_t *v)
+{
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                 : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+                 : "l"(a), "l"(pol));
+}
+__device__ __forceinline__ void st_stream32(void *a, const uint32_t *v, uint64_t pol)
+{
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;"
+                 ::"l"(a), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "l"(pol)
+                 : "memory");
+}
 __device__ __forceinline__ void st_stream16(void *a, uint4 v, uint64_t pol)
 {
     asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;"
@@ -303,6 +322,14 @@ struct PV {
 __device__ __forceinline__ void load_header(const uint8_t *f, uint32_t flen, uint32_t h[16], uint64_t pol)
 {
     const uint32_t nch = min(4u, (flen + 15) >> 4);
+#if NFC_LD256
+    // frames of >= 64 B at 32-B aligned offsets (every 64-B-multiple ring): two 256-bit loads
+    if (nch == 4 && (reinterpret_cast<uintptr_t>(f) & 31) == 0) {
+        ld_stream32(f, pol, h);
+        ld_stream32(f + 32, pol, h + 8);
+        return;
+    }
+#endif
 #pragma unroll
     for (int c = 0; c < 4; c++) {
         uint4 v = c < (int)nch ? ld_stream16(f + 16 * c, pol) : make_uint4(0, 0, 0, 0);
@@ -1109,6 +1136,12 @@ __device__ __forceinline__ void forward_words(uint8_t *f, uint32_t h[16], const 
 __device__ __forceinline__ void forward_rewrite(uint8_t *f, uint32_t h[16], const PV &v, uint2 nh, uint2 pm, uint64_t pol)
 {
     forward_words(f, h, v, nh, pm);
+#if NFC_LD256
+    if ((reinterpret_cast<uintptr_t>(f) & 31) == 0) {
+        st_stream32(f, h, pol);
+        return;
+    }
+#endif
     st_stream16(f, make_uint4(h[0], h[1], h[2], h[3]), pol);
     st_stream16(f + 16, make_uint4(h[4], h[5], h[6], h[7]), pol);
 }
