@@ -199,6 +199,41 @@ std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::
     return "";
 }
 
+// 16-bit first level of an IPv4 bit-vector blob with W > 32 (> 2K rules; AclImg::x4): per field the
+// interval containing each 16-bit key prefix (addresses: then a window search whose
+// depth is the widest 16-bit bucket, usually 0-2 halvings instead of 5-7 after the 8-bit
+// buckets) or each port (exact: no search).  Empty if the blob does not qualify.
+void build_acl4_index(const std::vector<uint32_t> &b, std::vector<uint16_t> &x, uint32_t &d16)
+{
+    x.clear();
+    d16 = 0;
+    // (measured: +15 % at 10K rules, -1.5 % at 1K and -13 % at 200 rules, whose images mostly hit in L1)
+    if (b.size() < ACLBV_HDR || b[0] == 0 || b[1] <= 32 || b[6] != 1) return;
+    x.assign(4 * 65536, 0);
+    for (int q = 0; q < 4; q++) {
+        const uint32_t m = b[2 + q], *keys = &b[b[8 + 2 * q]];
+        if (m > 65535) { x.clear(); d16 = 0; return; }
+        uint32_t j = 0, widest = 1;
+        for (uint32_t t = 0; t < 65536; t++) {
+            const uint32_t first = q < 2 ? t << 16 : t;        // first key of the bucket / the port
+            while (j + 1 < m && keys[j + 1] <= first) j++;
+            x[q * 65536 + t] = (uint16_t)j;
+            if (q < 2) {                                         // the bucket's window [j, j_last]
+                const uint32_t last = first | 0xFFFFu;
+                uint32_t e = j;
+                while (e + 1 < m && keys[e + 1] <= last) e++;
+                widest = std::max(widest, e - j + 1);
+            }
+        }
+        if (q < 2) {
+            uint32_t st = 0;
+            while ((1u << st) < widest) st++;
+            if (st > b[23]) st = b[23];   // never wider than the 8-bit buckets' (the key pad covers those)
+            d16 |= st << (8 * q);
+        }
+    }
+}
+
 // Search image of an IPv4 bit-vector blob (AclImg::f4 layout, nfc_internal.h): the
 // same intervals, bitsets, buckets and rule words, with bucket entries as key addresses
 // and pad entries instead of clamps.  Only for W == 1 (<= 64 rules) and window depth

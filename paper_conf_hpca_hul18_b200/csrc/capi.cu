@@ -69,7 +69,7 @@ struct nfc_chain {
     DBuf uf_list[2], uf_cnt, uf_pass;     // NFC_F_UNFUSED scratch
     bool loaded[8] = {false};
     // tables
-    DBuf acl_r4, acl_r6, acl_f4;
+    DBuf acl_r4, acl_r6, acl_f4, acl_x4;
     AclImg acl{};
     DBuf dpi_cls, dpi_trans, dpi_off, dpi_ids, dpi_act, dpi_bitmap, dpi_meta, dpi_sparse, dpi_frows, dpi_accid, dpi_accmeta;
     DpiImg dpi{};
@@ -180,7 +180,7 @@ void nfc_destroy_chain(nfc_chain *c)
     if (!c) return;
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
-    DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->acl_f4, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
+    DBuf *all[] = {&c->acl_r4, &c->acl_r6, &c->acl_f4, &c->acl_x4, &c->dpi_cls, &c->dpi_trans, &c->dpi_off, &c->dpi_ids, &c->dpi_act,
                    &c->dpi_bitmap, &c->dpi_meta, &c->dpi_sparse, &c->dpi_frows, &c->dpi_accid, &c->dpi_accmeta, &c->uf_list[0], &c->uf_list[1], &c->uf_cnt, &c->uf_pass, &c->l4_tbl24, &c->l4_long, &c->l4_nh, &c->l4_pmac, &c->l6_lens, &c->l6_base,
                    &c->l6_mask, &c->l6_ent, &c->l6_nh, &c->l6_pmac, &c->esp_sa, &c->esp_te, &c->esp_nib,
                    &c->esp_seq[0], &c->esp_seq[1], &c->lb_port, &c->lb_nib, &c->nat_pool, &c->nat_dnat, &c->nat_nib,
@@ -227,6 +227,12 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
                         (uint32_t)b6.size(), s.n_rules, s.default_action, 0, {}, {}};
         std::copy(b4.begin(), b4.begin() + ACLBV_HDR, c->acl.hdr4);
         std::copy(b6.begin(), b6.begin() + ACLBV_HDR, c->acl.hdr6);
+        std::vector<uint16_t> x4;
+        build_acl4_index(b4, x4, c->acl.d16);
+        if (!x4.empty()) {
+            CK(c->acl_x4.upload(x4));
+            c->acl.x4 = c->acl_x4.as<uint16_t>();
+        }
         std::vector<uint32_t> f4;
         build_acl4_fast(b4, f4, c->acl.f4_key, c->acl.f4_bv);
         if (!f4.empty()) {

@@ -40,6 +40,12 @@ struct AclImg {
     uint32_t words_f4;                // its size (u32 words, 16-B multiple)
     uint32_t fast;                    // per launch: 1 = the fused kernel stages f4 (acl4_fast)
     uint32_t f4_key[4], f4_bv[4];     // byte offsets of the key and bitset arrays per field
+    // 16-bit first level of an IPv4 rule set read from global memory (W > 32: the 10K
+    // rule set), build_acl4_index: 4 x 65536 u16 -- the interval of (src >> 16) << 16 and
+    // of (dst >> 16) << 16 (window searches of d16 & 255 / d16 >> 8 halvings follow),
+    // and the interval of every source / destination port (no search)
+    const uint16_t *x4;
+    uint32_t d16;
 };
 // Search image layout (byte offsets): four 256-entry u16 bucket tables (src, dst,
 // sport, dport) on the top 8 key bits, each entry the byte offset of the window's
@@ -255,6 +261,7 @@ std::string build_regex_dfa(const nfc_dpi_spec &s, DpiHost &o, uint32_t max_stat
 struct HostImage { std::vector<uint8_t> bytes; };
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
 // the record image (AclImg::f4) of an IPv4 blob; empty if the blob does not qualify
+void build_acl4_index(const std::vector<uint32_t> &blob4, std::vector<uint16_t> &x, uint32_t &d16);
 void build_acl4_fast(const std::vector<uint32_t> &blob4, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4]);
 struct DpiHost {
     std::vector<uint8_t> cls;

@@ -662,6 +662,21 @@ __device__ __forceinline__ uint32_t acl_core(const AclMem<SM> &M4, const AclMem<
         if constexpr (SM)
             if (ai.fast) return acl4_fast(M4.s, ai, v);
         const AclMem<SM> &M = M4;
+        if constexpr (!SM)
+            if (ai.x4 != nullptr) {          // 16-bit first level (large rule sets, global image)
+                const uint32_t ks = v.src[0], kd = v.dst[0];
+                uint32_t js = __ldg(ai.x4 + (ks >> 16)), jd = __ldg(ai.x4 + 65536 + (kd >> 16));
+                const uint32_t jsp = __ldg(ai.x4 + 131072 + (v.sport & 0xFFFF)), jdp = __ldg(ai.x4 + 196608 + (v.dport & 0xFFFF));
+                for (int i = (int)(ai.d16 & 255) - 1; i >= 0; i--) {
+                    const uint32_t h = 1u << i;
+                    js += M.template at<uint32_t>(4 * (hd[8] + js + h)) <= ks ? h : 0u;
+                }
+                for (int i = (int)(ai.d16 >> 8) - 1; i >= 0; i--) {
+                    const uint32_t h = 1u << i;
+                    jd += M.template at<uint32_t>(4 * (hd[10] + jd + h)) <= kd ? h : 0u;
+                }
+                return acl_match_w<SM>(M, hd, ai.default_action, js, jd, jsp, jdp, v.proto);
+            }
         const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport, kdp = v.dport;
         // window starts (bucket reads on the top 8 key bits), as byte offsets
         uint32_t os = 4 * hd[8] + 4 * M.template at<uint16_t>(4 * hd[18] + 2 * (ks >> 24));
