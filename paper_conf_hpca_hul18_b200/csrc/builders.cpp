@@ -239,11 +239,32 @@ void build_acl4_index(const std::vector<uint32_t> &b, std::vector<uint16_t> &x, 
 // and pad entries instead of clamps.  Only for W == 1 (<= 64 rules) and window depth
 // <= 3: the kernel always takes three halvings (8-key window).  key_off / bv_off
 // receive the per-field array offsets.
-void build_acl4_fast(const std::vector<uint32_t> &b, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4])
+void build_acl4_fast(const std::vector<uint32_t> &b, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4],
+                     uint32_t &d3)
 {
     f.clear();
-    if (b.size() < ACLBV_HDR || b[0] == 0 || b[0] > 64 || b[1] != 1 || b[6] != 1 || b[23] > 3) return;
+    d3 = 0;
+    if (b.size() < ACLBV_HDR || b[0] == 0 || b[0] > 64 || b[1] != 1 || b[6] != 1) return;
     const uint32_t m[4] = {b[2], b[3], b[4], b[5]};
+    // bucket t of a field: the interval of its first key; the window [bk(t), bk(t+1)]
+    // (the interval of the bucket's last key) must fit the kernel's 2 or 3 halvings
+    std::vector<uint32_t> bk[4];
+    uint32_t widest = 1;
+    for (int q = 0; q < 4; q++) {
+        const uint32_t *keys = &b[b[8 + 2 * q]], kb = q < 2 ? 32 : 16;
+        bk[q].resize(ACLF_NB);
+        uint32_t j = 0;
+        for (uint32_t t = 0; t < ACLF_NB; t++) {
+            const uint32_t first = t << (kb - NFC_ACLF_BITS), last = first | ((1u << (kb - NFC_ACLF_BITS)) - 1);
+            while (j + 1 < m[q] && keys[j + 1] <= first) j++;
+            uint32_t e = j;
+            while (e + 1 < m[q] && keys[e + 1] <= last) e++;
+            bk[q][t] = j;
+            widest = std::max(widest, e - j + 1);
+        }
+    }
+    if (widest > 8) return;           // more than three halvings: the bit-vector blob path
+    d3 = widest > 4 ? 1 : 0;
     size_t bytes = ACLF_REC;
     for (int q = 0; q < 4; q++) {
         key_off[q] = (uint32_t)bytes;
@@ -254,19 +275,16 @@ void build_acl4_fast(const std::vector<uint32_t> &b, std::vector<uint32_t> &f, u
     bytes = (bytes + 15) & ~(size_t)15;
     if (bytes > 65535) return;   // bucket entries are u16 byte offsets
     f.assign(bytes / 4, 0);
-    uint16_t *bk = reinterpret_cast<uint16_t *>(f.data());
+    uint16_t *bkt = reinterpret_cast<uint16_t *>(f.data());
     for (int q = 0; q < 4; q++) {
-        const uint32_t keys = b[8 + 2 * q], bv = b[9 + 2 * q], bko = b[18 + q];
+        const uint32_t keys = b[8 + 2 * q], bv = b[9 + 2 * q];
         for (uint32_t j = 0; j < m[q] + 8; j++) {
             const uint32_t jj = std::min(j, m[q] - 1);   // the pad entries repeat the last one
             f[key_off[q] / 4 + j] = b[keys + jj];
             f[bv_off[q] / 4 + 2 * j] = b[bv + 2 * jj];
             f[bv_off[q] / 4 + 2 * j + 1] = b[bv + 2 * jj + 1];
         }
-        for (uint32_t t = 0; t < 256; t++) {
-            const uint32_t w = b[bko + t / 2], j = (t & 1) ? w >> 16 : w & 0xFFFF;
-            bk[q * 256 + t] = (uint16_t)(key_off[q] + 4 * j);
-        }
+        for (uint32_t t = 0; t < ACLF_NB; t++) bkt[q * ACLF_NB + t] = (uint16_t)(key_off[q] + 4 * bk[q][t]);
     }
     for (uint32_t i = 0; i < 512; i++) f[ACLF_PROTO / 4 + i] = b[b[16] + i];
     for (uint32_t r = 0; r < b[0]; r++) f[ACLF_RULE / 4 + r] = b[b[17] + r];

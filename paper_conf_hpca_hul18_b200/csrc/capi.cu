@@ -234,7 +234,7 @@ int nfc_load_tables(nfc_chain *c, uint32_t kind, const void *spec, size_t spec_b
             c->acl.x4 = c->acl_x4.as<uint16_t>();
         }
         std::vector<uint32_t> f4;
-        build_acl4_fast(b4, f4, c->acl.f4_key, c->acl.f4_bv);
+        build_acl4_fast(b4, f4, c->acl.f4_key, c->acl.f4_bv, c->acl.f4_d3);
         if (!f4.empty()) {
             CK(c->acl_f4.upload(f4));
             c->acl.f4 = c->acl_f4.as<uint32_t>();

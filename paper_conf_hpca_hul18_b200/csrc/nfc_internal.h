@@ -40,6 +40,7 @@ struct AclImg {
     uint32_t words_f4;                // its size (u32 words, 16-B multiple)
     uint32_t fast;                    // per launch: 1 = the fused kernel stages f4 (acl4_fast)
     uint32_t f4_key[4], f4_bv[4];     // byte offsets of the key and bitset arrays per field
+    uint32_t f4_d3;                   // 1: some bucket window needs a third halving (else two)
     // 16-bit first level of an IPv4 rule set read from global memory (W > 32: the 10K
     // rule set), build_acl4_index: 4 x 65536 u16 -- the interval of (src >> 16) << 16 and
     // of (dst >> 16) << 16 (window searches of d16 & 255 / d16 >> 8 halvings follow),
@@ -53,7 +54,11 @@ struct AclImg {
 // field the interval start keys (u32) and, apart, their bitsets (u64), both followed by
 // 8 copies of the last entry, so a 3-halving window search needs no clamp and the
 // bitset of key j sits at a fixed affine image of the key's address (bv + 2 (key - k0)).
-static const uint32_t ACLF_BK = 0, ACLF_PROTO = 2048, ACLF_RULE = 4096, ACLF_REC = 4352;
+#ifndef NFC_ACLF_BITS
+#define NFC_ACLF_BITS 10      // search image buckets: the top NFC_ACLF_BITS bits of each key
+#endif
+static const uint32_t ACLF_NB = 1u << NFC_ACLF_BITS;                 // buckets per field
+static const uint32_t ACLF_BK = 0, ACLF_PROTO = 8 * ACLF_NB, ACLF_RULE = ACLF_PROTO + 2048, ACLF_REC = ACLF_RULE + 256;
 
 // ---------------------------------------------------------------- DPI
 // Full Aho-Corasick DFA over byte classes, states numbered in BFS order.
@@ -262,7 +267,8 @@ struct HostImage { std::vector<uint8_t> bytes; };
 std::string build_acl(const nfc_acl_spec &s, std::vector<uint32_t> &blob4, std::vector<uint32_t> &blob6);
 // the record image (AclImg::f4) of an IPv4 blob; empty if the blob does not qualify
 void build_acl4_index(const std::vector<uint32_t> &blob4, std::vector<uint16_t> &x, uint32_t &d16);
-void build_acl4_fast(const std::vector<uint32_t> &blob4, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4]);
+void build_acl4_fast(const std::vector<uint32_t> &blob4, std::vector<uint32_t> &f, uint32_t key_off[4], uint32_t bv_off[4],
+                     uint32_t &d3);
 struct DpiHost {
     std::vector<uint8_t> cls;
     std::vector<uint8_t> trans;   // raw bytes (u16 or u32 entries)

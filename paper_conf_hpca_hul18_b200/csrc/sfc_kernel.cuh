@@ -626,7 +626,7 @@ __device__ __forceinline__ void acl_search4_s(uint32_t &as, uint32_t &ad, uint32
     }
 }
 // IPv4 ACL from the search image (AclImg::f4) in shared memory at byte offset `img`:
-// per field one bucket read and three window halvings at immediate offsets over the
+// per field one bucket read and two or three window halvings at immediate offsets over the
 // 4-B keys (the pad keys make overshooting the last interval harmless), then the
 // bitset at the key's affine image; returns as acl_core.  Any key stays in bounds
 // (dead lanes included).
@@ -634,11 +634,12 @@ __device__ __forceinline__ uint32_t acl4_fast(uint32_t img, const AclImg &ai, co
 {
     const uint32_t B = (uint32_t)__cvta_generic_to_shared(nfc_smem) + img;
     const uint32_t ks = v.src[0], kd = v.dst[0], ksp = v.sport & 0xFFFF, kdp = v.dport & 0xFFFF;
-    uint32_t as = B + lds_u16z(B + ACLF_BK + 2 * (ks >> 24));
-    uint32_t ad = B + lds_u16z(B + ACLF_BK + 512 + 2 * (kd >> 24));
-    uint32_t asp = B + lds_u16z(B + ACLF_BK + 1024 + 2 * (ksp >> 8));
-    uint32_t adp = B + lds_u16z(B + ACLF_BK + 1536 + 2 * (kdp >> 8));
-    acl_step_s<16>(as, ks); acl_step_s<16>(ad, kd); acl_step_s<16>(asp, ksp); acl_step_s<16>(adp, kdp);
+    constexpr uint32_t NB2 = 2 * ACLF_NB;
+    uint32_t as = B + lds_u16z(B + ACLF_BK + 2 * (ks >> (32 - NFC_ACLF_BITS)));
+    uint32_t ad = B + lds_u16z(B + ACLF_BK + NB2 + 2 * (kd >> (32 - NFC_ACLF_BITS)));
+    uint32_t asp = B + lds_u16z(B + ACLF_BK + 2 * NB2 + 2 * (ksp >> (16 - NFC_ACLF_BITS)));
+    uint32_t adp = B + lds_u16z(B + ACLF_BK + 3 * NB2 + 2 * (kdp >> (16 - NFC_ACLF_BITS)));
+    if (ai.f4_d3) { acl_step_s<16>(as, ks); acl_step_s<16>(ad, kd); acl_step_s<16>(asp, ksp); acl_step_s<16>(adp, kdp); }
     acl_step_s<8>(as, ks); acl_step_s<8>(ad, kd); acl_step_s<8>(asp, ksp); acl_step_s<8>(adp, kdp);
     acl_step_s<4>(as, ks); acl_step_s<4>(ad, kd); acl_step_s<4>(asp, ksp); acl_step_s<4>(adp, kdp);
     // bitset address = 2 * key address + (bv - 2 key - B) per field
