@@ -380,14 +380,16 @@ def test_parallel_groups_validated(nfc):
     assert e.value.code == nfc.NFC_EUNSUP
 
 
-def test_c1_acl_boundary_keys(nfc):
-    """The IPv4 search image (AclImg::f4, three fixed halvings over padded key arrays):
-    5-tuples placed exactly on, just below and just above every rule's interval edges,
-    plus the extreme keys 0 / 2^32-1 and ports 0 / 65535, bit-exact vs the oracle's
-    linear rule scan (DESIGN.md ACL)."""
+@pytest.mark.parametrize("cfg,n_acl", [("C1", None), ("N3", 10000)])
+def test_c1_acl_boundary_keys(nfc, cfg, n_acl):
+    """The IPv4 search image (AclImg::f4: 10-bit buckets, two or three halvings over
+    padded key arrays; C1) and the 16-bit first level of large rule sets (AclImg::x4; the
+    10K-rule FW of NEXT-3): 5-tuples placed exactly on, just below and just above every
+    rule's interval edges, plus the extreme keys 0 / 2^32-1 and ports 0 / 65535,
+    bit-exact vs the oracle's linear rule scan (DESIGN.md ACL)."""
     import oracle
     from tests.gpu_util import compare_bytes, compare_records, gpu_run, sorted_pairs
-    w = nfcgen.workload("C1")
+    w = nfcgen.workload(cfg, acl_rules=n_acl, pkt_len=64 if cfg == "N3" else None)
     n = 4096
     b = nfcgen.generate(w.traffic, w.tables, 0, n)
     rules = w.tables.acl_rules
@@ -421,8 +423,8 @@ def test_c1_acl_boundary_keys(nfc):
     want, want_arena, (wp, wq), npairs = orc.run(b, match_cap=1 << 16)
     ch = _chain(nfc, w)
     got, arenas, (gp, gq), k = gpu_run(ch, [b])
-    compare_records(got, want, "C1 ACL edges")
-    compare_bytes(want, arenas[0], b.off, want_arena, b.off, "C1 ACL edges")
+    compare_records(got, want, f"{cfg} ACL edges")
+    compare_bytes(want, arenas[0], b.off, want_arena, b.off, f"{cfg} ACL edges")
     assert k == npairs and np.array_equal(sorted_pairs(gp, gq), sorted_pairs(wp, wq))
     # the edges exercise many distinct rules (not just the default)
     assert len(np.unique(got["acl_rule"])) > 10
