@@ -54,6 +54,11 @@ NFC_API int nfc_dbg_lpm6_levels(nfc_dbg *d, uint32_t *n_levels);
 /* ACL: first matching rule (0xFFFF none) and the resulting action (0 permit / 1 deny). */
 NFC_API int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *dst, uint16_t sport,
                         uint16_t dport, uint8_t proto, uint32_t *rule, uint32_t *action);
+/* ACL, IPv4, through the fused kernel's other images: which = 0 the search image of <= 64-rule
+ * sets (AclImg::f4), 1 the 16-bit first level of > 2K-rule sets (AclImg::x4); addresses as
+ * host-order u32.  NFC_EUNSUP if the rule set has no such image. */
+NFC_API int nfc_dbg_acl4_image(nfc_dbg *d, uint32_t which, uint32_t src, uint32_t dst, uint16_t sport, uint16_t dport,
+                               uint8_t proto, uint32_t *rule, uint32_t *action);
 /* Crypto / hash primitives as the kernel computes them (T-tables, nibble tables, ipad/opad states). */
 NFC_API int nfc_dbg_aes128_block(const uint8_t key[16], const uint8_t in[16], uint8_t out[16]);
 NFC_API int nfc_dbg_toeplitz(const uint8_t key[40], const uint8_t *in, size_t n, uint32_t *h);

@@ -21,6 +21,11 @@ struct nfc_dbg {
     std::vector<uint2> nh, pmac;
     Lpm6Host l6;
     NatHost nat;
+    // the fused kernel's IPv4 search image (AclImg::f4) and 16-bit first level (AclImg::x4)
+    std::vector<uint32_t> f4;
+    uint32_t f4_key[4] = {0}, f4_bv[4] = {0}, f4_d3 = 0;
+    std::vector<uint16_t> x4;
+    uint32_t d16 = 0;
 };
 
 static inline uint32_t be32(const uint8_t *p) { return (uint32_t)p[0] << 24 | (uint32_t)p[1] << 16 | (uint32_t)p[2] << 8 | p[3]; }
@@ -41,6 +46,10 @@ int nfc_dbg_build(uint32_t kind, const void *spec, size_t spec_bytes, nfc_dbg **
         err = build_acl(*static_cast<const nfc_acl_spec *>(spec), d->r4, d->r6);
         d->n_rules = static_cast<const nfc_acl_spec *>(spec)->n_rules;
         d->default_action = static_cast<const nfc_acl_spec *>(spec)->default_action;
+        if (err.empty()) {
+            build_acl4_fast(d->r4, d->f4, d->f4_key, d->f4_bv, d->f4_d3);
+            build_acl4_index(d->r4, d->x4, d->d16);
+        }
         break;
     case NFC_DPI:
         if (spec_bytes != sizeof(nfc_dpi_spec)) break;
@@ -302,6 +311,74 @@ int nfc_dbg_acl(nfc_dbg *d, uint32_t family, const uint8_t *src, const uint8_t *
             uint64_t x = bv(A[9], js, w) & bv(A[11], jd, w) & bv(A[13], jsp, w) & bv(A[15], jdp, w) & bv(A[16], proto, w);
             if (x) {
                 uint32_t e = A[A[17] + 64 * w + __builtin_ctzll(x)];
+                *rule = e & 0xFFFF;
+                *action = e >> 31;
+                return NFC_OK;
+            }
+            cand &= cand - 1;
+        }
+    }
+    return NFC_OK;
+}
+
+// IPv4 lookups through the fused kernel's other ACL images, as the kernel does them:
+// which = 0: the search image (acl4_fast: bucket on the top NFC_ACLF_BITS bits, two or
+// three halvings over the padded keys, bitsets at the affine image of the key address);
+// which = 1: the 16-bit first level (acl_core's x4 path: per-prefix / per-port interval,
+// d16 halvings for the addresses), then the bit-vector match.  NFC_EUNSUP if the rule
+// set has no such image.
+int nfc_dbg_acl4_image(nfc_dbg *d, uint32_t which, uint32_t src, uint32_t dst, uint16_t sport, uint16_t dport,
+                       uint8_t proto, uint32_t *rule, uint32_t *action)
+{
+    if (!d || d->kind != NFC_ACL || !rule || !action) return NFC_EINVAL;
+    const uint32_t *A = d->r4.data();
+    if (which == 0) {
+        if (d->f4.empty()) return NFC_EUNSUP;
+        const uint8_t *F = reinterpret_cast<const uint8_t *>(d->f4.data());
+        auto u16 = [&](uint32_t o) { uint16_t v; memcpy(&v, F + o, 2); return (uint32_t)v; };
+        auto u32 = [&](uint32_t o) { uint32_t v; memcpy(&v, F + o, 4); return v; };
+        const uint32_t key[4] = {src, dst, sport, dport};
+        uint64_t x = 0;
+        memcpy(&x, F + ACLF_PROTO + 8 * proto, 8);
+        for (int q = 0; q < 4; q++) {
+            const uint32_t kb = q < 2 ? 32 : 16;
+            uint32_t a = u16(ACLF_BK + 2 * ACLF_NB * q + 2 * (key[q] >> (kb - NFC_ACLF_BITS)));   // key byte offset
+            if (d->f4_d3) a += u32(a + 16) <= key[q] ? 16 : 0;
+            a += u32(a + 8) <= key[q] ? 8 : 0;
+            a += u32(a + 4) <= key[q] ? 4 : 0;
+            uint64_t bv;
+            memcpy(&bv, F + d->f4_bv[q] + 2 * (a - d->f4_key[q]), 8);
+            x &= bv;
+        }
+        *rule = 0xFFFF;
+        *action = d->default_action;
+        if (x) {
+            const uint32_t e = u32(ACLF_RULE + 4 * (uint32_t)__builtin_ctzll(x));
+            *rule = e & 0xFFFF;
+            *action = e >> 31;
+        }
+        return NFC_OK;
+    }
+    if (d->x4.empty()) return NFC_EUNSUP;
+    uint32_t js = d->x4[src >> 16], jd = d->x4[65536 + (dst >> 16)];
+    const uint32_t jsp = d->x4[131072 + sport], jdp = d->x4[196608 + dport];
+    for (int i = (int)(d->d16 & 255) - 1; i >= 0; i--) js += A[A[8] + js + (1u << i)] <= src ? 1u << i : 0u;
+    for (int i = (int)(d->d16 >> 8) - 1; i >= 0; i--) jd += A[A[10] + jd + (1u << i)] <= dst ? 1u << i : 0u;
+    js = std::min(js, A[2] - 1);
+    jd = std::min(jd, A[3] - 1);
+    const uint32_t W = A[1], WA = A[29];
+    auto row = [&](uint32_t off, uint32_t j, uint32_t w, uint32_t stride) { uint64_t v; memcpy(&v, A + off + 2 * ((size_t)j * stride + w), 8); return v; };
+    *rule = 0xFFFF;
+    *action = d->default_action;
+    for (uint32_t a = 0; a < WA; a++) {
+        uint64_t cand = row(A[24], js, a, WA) & row(A[25], jd, a, WA) & row(A[26], jsp, a, WA) & row(A[27], jdp, a, WA) &
+                        row(A[28], proto, a, WA);
+        while (cand) {
+            const uint32_t w = 64 * a + (uint32_t)__builtin_ctzll(cand);
+            const uint64_t x = row(A[9], js, w, W) & row(A[11], jd, w, W) & row(A[13], jsp, w, W) & row(A[15], jdp, w, W) &
+                               row(A[16], proto, w, W);
+            if (x) {
+                const uint32_t e = A[A[17] + 64 * w + (uint32_t)__builtin_ctzll(x)];
                 *rule = e & 0xFFFF;
                 *action = e >> 31;
                 return NFC_OK;

@@ -97,7 +97,7 @@ EXPORTS = ["nfc_build_chain", "nfc_destroy_chain", "nfc_chain_room", "nfc_load_t
            "nfc_comm_destroy", "nfc_attach_comm", "nfc_measure_peaks", "nfc_set_groups", "nfc_get_groups"]
 DEBUG_EXPORTS = ["nfc_dbg_build", "nfc_dbg_destroy", "nfc_dbg_dpi", "nfc_dbg_dpi_shape", "nfc_dbg_dpi_tier",
                  "nfc_dbg_dpi_tier_shape", "nfc_dbg_dpi_slot", "nfc_dbg_nat", "nfc_dbg_lpm4",
-                 "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_aes128_block",
+                 "nfc_dbg_lpm6", "nfc_dbg_lpm6_levels", "nfc_dbg_acl", "nfc_dbg_acl4_image", "nfc_dbg_aes128_block",
                  "nfc_dbg_toeplitz", "nfc_dbg_hmac_sha1"]
 
 
@@ -150,6 +150,7 @@ def _load_lib():
     L.nfc_dbg_lpm6.argtypes = [_P, _P, P32, P32, P32]
     L.nfc_dbg_lpm6_levels.argtypes = [_P, P32]
     L.nfc_dbg_acl.argtypes = [_P, _u32, _P, _P, ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint8, P32, P32]
+    L.nfc_dbg_acl4_image.argtypes = [_P, _u32, _u32, _u32, ctypes.c_uint16, ctypes.c_uint16, ctypes.c_uint8, P32, P32]
     L.nfc_dbg_aes128_block.argtypes = [_P, _P, _P]
     L.nfc_dbg_toeplitz.argtypes = [_P, _P, ctypes.c_size_t, P32]
     L.nfc_dbg_hmac_sha1.argtypes = [_P, _P, ctypes.c_size_t, _P]
@@ -560,6 +561,16 @@ class HostImage:
         r, a = _u32(), _u32()
         _check(lib.nfc_dbg_acl(self.h, family, _cbuf(src), _cbuf(dst), sport, dport, proto,
                                ctypes.byref(r), ctypes.byref(a)))
+        return r.value, a.value
+
+    def acl4_image(self, which, src: int, dst: int, sport, dport, proto):
+        """IPv4 lookup through the search image (which=0) or the 16-bit first level (1);
+        None if the rule set has no such image."""
+        r, a = _u32(), _u32()
+        rc = lib.nfc_dbg_acl4_image(self.h, which, src, dst, sport, dport, proto, ctypes.byref(r), ctypes.byref(a))
+        if rc == NFC_EUNSUP:
+            return None
+        _check(rc)
         return r.value, a.value
 
 

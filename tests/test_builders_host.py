@@ -320,3 +320,50 @@ def test_nat_image_vs_oracle(nfc):
     with pytest.raises(Exception):
         nfc.HostImage("NAT", inside=t.nat_inside, pool=t.nat_pool, port_lo=9, port_hi=2, dnat=t.nat_dnat,
                       key=t.nat_key)
+
+
+@pytest.mark.parametrize("n,which", [(64, 0), (40, 0), (3000, 1), (10000, 1)])
+def test_acl4_fused_images_vs_oracle(nfc, n, which):
+    """The fused kernel's other IPv4 ACL images, looked up as the kernel does: the search
+    image of <= 64-rule sets (10-bit buckets, two or three halvings over padded keys,
+    bitsets at an affine image of the key address) and the 16-bit first level of > 2K-rule
+    sets (per-prefix / per-port intervals) == the oracle's linear first-match scan, on
+    random 5-tuples, tuples inside rules, and tuples on every rule's interval edges
+    (including 0 / 2^32-1 and ports 0 / 65535)."""
+    rng = np.random.default_rng(900 + n)
+    rules = nfcgen.gen_acl(rng, n, 4)
+    t = nfcgen.Tables(acl_rules=rules, acl_default=1)
+    img = nfc.HostImage("ACL", rules=rules, default_action=1)
+    orc = oracle.OracleChain(["ACL"], t)
+    assert img.acl4_image(which, 0, 0, 0, 0, 6) is not None, "the rule set should have this image"
+    edges_ip, edges_port = [0, 0xFFFFFFFF], [0, 65535]
+    for ru in rules:
+        for fld, ln in (("src", "slen"), ("dst", "dlen")):
+            k = int.from_bytes(bytes(ru[fld][:4]), "big")
+            L = int(ru[ln])
+            m = (0xFFFFFFFF << (32 - L)) & 0xFFFFFFFF if L else 0
+            lo, hi = k & m, (k & m) | (~m & 0xFFFFFFFF)
+            edges_ip += [lo, hi, (lo - 1) & 0xFFFFFFFF, (hi + 1) & 0xFFFFFFFF]
+        for a, b in ((int(ru["sp_lo"]), int(ru["sp_hi"])), (int(ru["dp_lo"]), int(ru["dp_hi"]))):
+            edges_port += [a, b, (a - 1) & 0xFFFF, (b + 1) & 0xFFFF]
+    r = random.Random(n)
+    for it in range(4000):
+        mode = it % 3
+        if mode == 0:
+            src, dst, sp, dp = r.getrandbits(32), r.getrandbits(32), r.getrandbits(16), r.getrandbits(16)
+        elif mode == 1:
+            src, dst = r.choice(edges_ip), r.choice(edges_ip)
+            sp, dp = r.choice(edges_port), r.choice(edges_port)
+        else:
+            ru = rules[r.randrange(len(rules))]
+            def inside(p, L):
+                k = int.from_bytes(bytes(p[:4]), "big")
+                m = (0xFFFFFFFF << (32 - L)) & 0xFFFFFFFF if L else 0
+                return (k & m) | (r.getrandbits(32) & ~m & 0xFFFFFFFF)
+            src, dst = inside(ru["src"], int(ru["slen"])), inside(ru["dst"], int(ru["dlen"]))
+            sp, dp = r.randint(int(ru["sp_lo"]), int(ru["sp_hi"])), r.randint(int(ru["dp_lo"]), int(ru["dp_hi"]))
+        proto = r.choice([1, 6, 17])
+        got = img.acl4_image(which, src, dst, sp, dp, proto)
+        want = orc.acl(4, src.to_bytes(4, "big"), dst.to_bytes(4, "big"), sp, dp, proto)
+        assert got[0] == (0xFFFF if want < 0 else want), (it, mode, hex(src), hex(dst), sp, dp, proto, got, want)
+        assert got[1] == (1 if want < 0 else int(rules[want]["action"]))
